@@ -1,0 +1,148 @@
+"""Script generation (TEST INFRASTRUCTURE ONLY — see oracle/__init__.py).
+
+Written from SPEC_SCRIPT.md §S and §E in the paper's order (§III-B1):
+super-graph with summed loss (L205) -> level sort by maximum depth from the sources (L139) ->
+forward traversal emitting one CISC instruction per node (L141, L159) -> signal/wait between
+consecutive levels (L165) -> reverse traversal for back-propagation (L167) with min-load
+assignment (L167) -> per-VPP scripts concatenated behind the prefix sum of their lengths (L169).
+"""
+from __future__ import annotations
+
+NONE = 0xFFFFFFFF
+OP = dict(S=0x01, W=0x02, LSTM_F=0x10, LSTM_B=0x11, LEAF_F=0x20, LEAF_B=0x21, INT_F=0x22, INT_B=0x23,
+          CS_F=0x30, CS_B=0x31, HEAD_F=0x40, HEAD_B=0x41)
+
+
+def _a32(x: int) -> int:
+    return (x + 31) // 32 * 32
+
+
+def pre(op: str, length: int) -> int:
+    """4-byte preamble: operation type and input tensor length (L159; reading R-16)."""
+    assert 0 <= length < (1 << 24)
+    return OP[op] | (length << 8)
+
+
+def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 148):
+    """Returns dict(words, pool_words, zero_words, loss_word, n_bar, levels, nodes)."""
+    # S1/S2: super-graph node list
+    nodes = []          # dict(kind, graph, cell(local), children(global ids), token, label, cellnode)
+    for b, g in enumerate(graphs):
+        base = len(nodes)
+        for v, (ch, tok, lab) in enumerate(g):
+            if cell == "binary":
+                kind = "LEAF" if len(ch) == 0 else "INT"
+            elif cell == "childsum":
+                kind = "CS"
+            else:
+                kind = "LSTM"
+            nodes.append(dict(kind=kind, children=[base + k for k in ch], token=tok, label=lab))
+        for v, (ch, tok, lab) in enumerate(g):
+            if lab >= 0:
+                nodes.append(dict(kind="HEAD", children=[base + v], token=-1, label=lab))
+    # S3: levels
+    level = []
+    for n in nodes:
+        level.append(0 if not n["children"] else 1 + max(level[k] for k in n["children"]))
+    L = max(level)
+    # S7: pool plan
+    n_bar = 2 * L + 1
+    z_loss = _a32(n_bar + 1)
+    off = _a32(z_loss + 1)
+    adj = [NONE] * len(nodes)
+    for i, n in enumerate(nodes):
+        if n["kind"] != "HEAD":
+            adj[i] = off
+            off = _a32(off + 2 * H)
+    zero_words = off
+    rec = [0] * len(nodes)
+    for i, n in enumerate(nodes):
+        rec[i] = off
+        size = {"LSTM": 6 * H, "LEAF": 5 * H, "INT": 7 * H, "CS": (5 + len(n["children"])) * H,
+                "HEAD": C + 1}[n["kind"]]
+        off = _a32(off + size)
+    pool_words = off
+
+    def cost(n):
+        k = n["kind"]
+        if k == "LEAF":
+            return 3 * H * E
+        if k == "INT":
+            return 6 * H * H + 2 * H * H
+        if k == "CS":
+            return (4 * H * E if n["token"] >= 0 else 0) + (3 * H * H + len(n["children"]) * H * H
+                                                            if n["children"] else 0)
+        if k == "LSTM":
+            return 4 * H * E + (4 * H * H if n["children"] else 0)
+        return C * H
+
+    def tok(t):
+        return NONE if t < 0 else t
+
+    def instr(i, fwd):
+        n = nodes[i]
+        k = n["kind"]
+        ch = n["children"]
+        if k == "LEAF":
+            return [pre("LEAF_F", E), rec[i], n["token"]] if fwd else [pre("LEAF_B", E), rec[i], adj[i], n["token"]]
+        if k == "INT":
+            l, r = ch
+            return ([pre("INT_F", 2 * H), rec[i], rec[l], rec[r]] if fwd else
+                    [pre("INT_B", 2 * H), rec[i], adj[i], rec[l], adj[l], rec[r], adj[r]])
+        if k == "LSTM":
+            p = ch[0] if ch else None
+            if fwd:
+                return [pre("LSTM_F", E + H), rec[i], n["token"], rec[p] if p is not None else NONE]
+            return [pre("LSTM_B", E + H), rec[i], adj[i], n["token"], rec[p] if p is not None else NONE,
+                    adj[p] if p is not None else NONE]
+        if k == "CS":
+            if fwd:
+                return [pre("CS_F", len(ch)), rec[i], tok(n["token"])] + [rec[c] for c in ch]
+            w = [pre("CS_B", len(ch)), rec[i], adj[i], tok(n["token"])]
+            for c in ch:
+                w += [rec[c], adj[c]]
+            return w
+        c = ch[0]
+        return ([pre("HEAD_F", H), rec[i], rec[c], n["label"]] if fwd else
+                [pre("HEAD_B", H), rec[i], rec[c], adj[c], n["label"]])
+
+    # S4/S5: phases and min-load group assignment
+    P = 2 * L + 2
+    by_level = [[] for _ in range(L + 1)]
+    for i in range(len(nodes)):
+        by_level[level[i]].append(i)
+    phase_instrs = []            # per phase: per group list of words
+    part = []
+    for p in range(P):
+        fwd = p <= L
+        lv = p if fwd else 2 * L + 1 - p
+        load = [0] * G
+        per_g = [[] for _ in range(G)]
+        for i in by_level[lv]:
+            g = min(range(G), key=lambda x: (load[x], x))
+            load[g] += cost(nodes[i])
+            per_g[g].extend(instr(i, fwd))
+        phase_instrs.append(per_g)
+        part.append([g for g in range(G) if per_g[g]])
+    # S6: signal / wait
+    streams = [[] for _ in range(G)]
+    for p in range(P):
+        for g in range(G):
+            if g not in part[p]:
+                continue
+            if p >= 1:
+                streams[g].append(pre("W", p))
+            streams[g].extend(phase_instrs[p][g])
+            if p < P - 1:
+                streams[g].append(pre("S", p + 1))
+    targets = [0] + [n_act * len(part[p - 1]) for p in range(1, n_bar + 1)]
+    # §E: header (prefix sums, L169), streams, barrier targets
+    prefix = [0]
+    for s in streams:
+        prefix.append(prefix[-1] + len(s))
+    words = [G, n_bar] + prefix
+    for s in streams:
+        words += s
+    words += targets
+    return dict(words=[w & 0xFFFFFFFF for w in words], pool_words=pool_words, zero_words=zero_words,
+                loss_word=z_loss, n_bar=n_bar, levels=level, nodes=nodes, rec=rec, adj=adj)

@@ -1,0 +1,369 @@
+// C ABI of libvpps (include/vpps.h): argument checking, object lifetime, the one H2D script copy,
+// the cooperative launch of the persistent kernel and loss bookkeeping.  No torch types here.
+#include <cuda_runtime.h>
+#include <climits>
+#include <cstring>
+#include <memory>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/vpps.h"
+#include "host/host.h"
+#include "kernels/vpps_kernel.cuh"
+
+using namespace vpps;
+
+namespace {
+thread_local std::string g_err;
+
+vpps_status fail(vpps_status st, const std::string& msg) {
+    g_err = msg;
+    return st;
+}
+vpps_status cuda_fail(cudaError_t e, const char* what) {
+    g_err = std::string(what) + ": " + cudaGetErrorString(e);
+    return VPPS_E_CUDA;
+}
+#define CK(call)                                               \
+    do {                                                       \
+        cudaError_t _e = (call);                               \
+        if (_e != cudaSuccess) return cuda_fail(_e, #call);    \
+    } while (0)
+
+std::vector<Shape> expected_shapes(int32_t cell, int32_t H, int32_t E, int32_t C) {
+    switch (cell) {
+        case CELL_LSTM: return {{4 * H, E}, {4 * H, H}, {C, H}, {4 * H, 1}, {C, 1}};
+        case CELL_BINARY: return {{3 * H, E}, {3 * H, 2 * H}, {H, H}, {H, H}, {C, H}, {3 * H, 1}, {H, 1}, {C, 1}};
+        case CELL_CHILDSUM: return {{3 * H, E}, {H, E}, {3 * H, H}, {H, H}, {C, H}, {3 * H, 1}, {H, 1}, {C, 1}};
+    }
+    return {};
+}
+}  // namespace
+
+struct vpps_model_s {
+    Plan plan;
+    std::vector<Shape> shapes;
+    std::vector<int64_t> offsets;
+    int64_t n_floats = 0;
+    bool plan_only = true;
+    int device = 0;
+    const Variant* var = nullptr;
+    size_t smem = 0;
+    float* params = nullptr;
+    float* grads = nullptr;
+    float* pool = nullptr;
+    int64_t pool_cap = 0, last_pool_words = 0;
+    float* h_loss = nullptr;            // pinned [2]
+    cudaEvent_t ev[2] = {nullptr, nullptr};
+    int64_t passes = 0;
+};
+
+struct vpps_script_s {
+    vpps_model model = nullptr;
+    Script s;
+    uint32_t* d_words = nullptr;
+    uint32_t* h_pinned = nullptr;
+    bool uploaded = false;
+};
+
+extern "C" {
+
+const char* vpps_last_error(void) { return g_err.c_str(); }
+
+int32_t vpps_variants(int32_t* out4, int32_t cap) {
+    int32_t n = 0;
+    const Variant* v = variants(&n);
+    for (int32_t i = 0; i < n && i < cap && out4; ++i) {
+        out4[4 * i] = v[i].cell; out4[4 * i + 1] = v[i].H; out4[4 * i + 2] = v[i].E; out4[4 * i + 3] = v[i].umax;
+    }
+    return n;
+}
+
+vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const vpps_opset* ops,
+                              const vpps_options* opt, vpps_model* out) {
+    if (!params || !ops || !out) return fail(VPPS_E_INVALID, "null argument");
+    *out = nullptr;
+    vpps_options o{};
+    if (opt) o = *opt;
+    const int32_t cell = ops->cell, H = ops->H, E = ops->E, C = ops->C;
+    if (cell < 0 || cell > 2 || H <= 0 || E <= 0 || C <= 0) return fail(VPPS_E_INVALID, "bad op set");
+    std::vector<Shape> want = expected_shapes(cell, H, E, C);
+    if ((int32_t)want.size() != n_params) return fail(VPPS_E_INVALID, "wrong number of parameters for the op set");
+    for (int32_t i = 0; i < n_params; ++i)
+        if (params[i].rows != want[i].rows || params[i].cols != want[i].cols)
+            return fail(VPPS_E_INVALID, "parameter " + std::to_string(i) + " has the wrong shape for the op set");
+    if (o.groups == 0) o.groups = 1;
+    if (o.ctas_per_sm == 0) o.ctas_per_sm = 1;
+    if (o.ctas_per_sm != 1) return fail(VPPS_E_INVALID, "ctas_per_sm must be 1 in v1");
+
+    std::unique_ptr<vpps_model_s> m(new (std::nothrow) vpps_model_s);
+    if (!m) return fail(VPPS_E_NOMEM, "out of host memory");
+    m->plan_only = o.plan_only != 0;
+    m->shapes = want;
+    int64_t cur = 0;
+    for (const Shape& s : want) {
+        m->offsets.push_back(cur);
+        cur += ((int64_t)s.rows * s.cols + 3) / 4 * 4;
+    }
+    m->n_floats = cur;
+    int32_t n_sm = o.n_sm;
+    if (!m->plan_only) {
+        m->device = o.device;
+        CK(cudaSetDevice(o.device));
+        cudaDeviceProp prop;
+        CK(cudaGetDeviceProperties(&prop, o.device));
+        if (prop.major != 10) return fail(VPPS_E_INVALID, "libvpps is built for sm_100a (B200) only");
+        if (n_sm == 0) n_sm = prop.multiProcessorCount;
+        if (n_sm > prop.multiProcessorCount) return fail(VPPS_E_INVALID, "n_sm exceeds the device's SM count");
+        if (o.groups != 1) return fail(VPPS_E_INVALID, "replica groups > 1 are plan-only in v1");
+    } else if (n_sm == 0) {
+        n_sm = 148;
+    }
+    std::string err;
+    if (!unit_plan(cell, H, E, C, n_sm, o.ctas_per_sm, o.groups, &m->plan, &err))
+        return fail(err.rfind("NOFIT", 0) == 0 ? VPPS_E_NOFIT : VPPS_E_INVALID, err);
+    if (!m->plan_only) {
+        if (H % 4 || E % 4) return fail(VPPS_E_INVALID, "H and E must be multiples of 4");
+        int32_t nv = 0;
+        const Variant* v = variants(&nv);
+        for (int32_t i = 0; i < nv; ++i)
+            if (v[i].cell == cell && v[i].H == H && v[i].E == E && v[i].umax == m->plan.umax) m->var = &v[i];
+        if (!m->var)
+            return fail(VPPS_E_NOFIT, "no kernel specialisation for cell " + std::to_string(cell) + " H=" +
+                                          std::to_string(H) + " E=" + std::to_string(E) +
+                                          " units/CTA=" + std::to_string(m->plan.umax));
+        m->smem = m->var->smem_bytes(C);
+        if (m->smem > 227 * 1024) return fail(VPPS_E_NOFIT, "head does not fit in shared memory");
+        CK(cudaFuncSetAttribute(m->var->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)m->smem));
+        int blocks = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, m->var->fn, 256, m->smem));
+        if (blocks < 1) return fail(VPPS_E_NOFIT, "kernel cannot be resident (registers/shared memory)");
+        CK(cudaMallocHost(&m->h_loss, 2 * sizeof(float)));
+        m->h_loss[0] = m->h_loss[1] = 0.f;
+        CK(cudaEventCreateWithFlags(&m->ev[0], cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&m->ev[1], cudaEventDisableTiming));
+    }
+    *out = m.release();
+    return VPPS_OK;
+}
+
+vpps_status vpps_layout(vpps_model m, int64_t* n_floats, int64_t* offsets) {
+    if (!m) return fail(VPPS_E_INVALID, "null model");
+    if (n_floats) *n_floats = m->n_floats;
+    if (offsets) std::memcpy(offsets, m->offsets.data(), m->offsets.size() * sizeof(int64_t));
+    return VPPS_OK;
+}
+
+vpps_status vpps_bind_buffers(vpps_model m, float* params_flat, float* grads_flat) {
+    if (!m || !params_flat || !grads_flat) return fail(VPPS_E_INVALID, "null argument");
+    if (m->plan_only) return fail(VPPS_E_STATE, "plan-only model");
+    if (((uintptr_t)params_flat | (uintptr_t)grads_flat) & 15) return fail(VPPS_E_INVALID, "buffers must be 16-byte aligned");
+    m->params = params_flat;
+    m->grads = grads_flat;
+    return VPPS_OK;
+}
+
+vpps_status vpps_partition_table(vpps_model m, const int32_t** rows8, int64_t* n_rows) {
+    if (!m || !rows8 || !n_rows) return fail(VPPS_E_INVALID, "null argument");
+    *rows8 = m->plan.table.data();
+    *n_rows = (int64_t)m->plan.table.size() / 8;
+    return VPPS_OK;
+}
+
+vpps_status vpps_plan_info(vpps_model m, int32_t* n_cta, int32_t* n_g, int32_t* n_act, int32_t* umax) {
+    if (!m) return fail(VPPS_E_INVALID, "null model");
+    if (n_cta) *n_cta = m->plan.n_cta;
+    if (n_g) *n_g = m->plan.n_g;
+    if (n_act) *n_act = m->plan.n_act;
+    if (umax) *umax = m->plan.umax;
+    return VPPS_OK;
+}
+
+vpps_status vpps_paper_deal(const vpps_shape* mats, int32_t n_mats, int32_t n_cta, int32_t tb, int32_t rpw,
+                            int32_t pack_rows, int32_t grads, int32_t* out6, int64_t* n_rows, int64_t* n_slots) {
+    if (!mats || n_mats <= 0 || n_cta <= 0 || tb <= 0 || tb % 32 || rpw <= 0 || !n_rows || !n_slots)
+        return fail(VPPS_E_INVALID, "bad argument");
+    std::vector<Shape> v(n_mats);
+    for (int32_t i = 0; i < n_mats; ++i) v[i] = {mats[i].rows, mats[i].cols};
+    std::vector<DealRow> rows;
+    paper_deal(v, n_cta, tb, rpw, pack_rows != 0, grads != 0, &rows, n_slots);
+    *n_rows = (int64_t)rows.size();
+    if (out6)
+        for (size_t i = 0; i < rows.size(); ++i) {
+            const DealRow& r = rows[i];
+            const int32_t x[6] = {r.matrix, r.row, r.cta, r.partition, r.warp, r.is_grad};
+            std::memcpy(out6 + 6 * i, x, sizeof(x));
+        }
+    return VPPS_OK;
+}
+
+int32_t vpps_paper_choose_cps(const vpps_shape* mats, int32_t n_mats, int32_t n_sm, int32_t tb, int32_t rpw,
+                              int32_t pack_rows) {
+    std::vector<Shape> v(n_mats);
+    for (int32_t i = 0; i < n_mats; ++i) v[i] = {mats[i].rows, mats[i].cols};
+    return paper_choose_cps(v, n_sm, tb, rpw, pack_rows != 0);
+}
+
+vpps_status vpps_build_script(vpps_model m, const vpps_batch* batch, vpps_script* out) {
+    if (!m || !batch || !out) return fail(VPPS_E_INVALID, "null argument");
+    *out = nullptr;
+    std::unique_ptr<vpps_script_s> s(new (std::nothrow) vpps_script_s);
+    if (!s) return fail(VPPS_E_NOMEM, "out of host memory");
+    s->model = m;
+    BatchIn b{batch->n_graphs, batch->graph_ptr, batch->child_ptr, batch->children, batch->token, batch->label};
+    std::string err;
+    // the input table's row count is not known here; token range is re-checked against it at run time
+    const int rc = build_script(m->plan, b, INT64_MAX, &s->s, &err);
+    if (rc != 0) return fail(rc == -4 ? VPPS_E_GRAPH : VPPS_E_INVALID, err);
+    if (!m->plan_only) {
+        const size_t bytes = s->s.words.size() * sizeof(uint32_t);
+        CK(cudaMallocHost(&s->h_pinned, bytes));                 // pinned staging (L169)
+        std::memcpy(s->h_pinned, s->s.words.data(), bytes);
+        CK(cudaMalloc(&s->d_words, bytes));
+    }
+    *out = s.release();
+    return VPPS_OK;
+}
+
+vpps_status vpps_script_words(vpps_script s, const uint32_t** words, int64_t* n) {
+    if (!s || !words || !n) return fail(VPPS_E_INVALID, "null argument");
+    *words = s->s.words.data();
+    *n = (int64_t)s->s.words.size();
+    return VPPS_OK;
+}
+
+vpps_status vpps_script_info_get(vpps_script s, vpps_script_info* info) {
+    if (!s || !info) return fail(VPPS_E_INVALID, "null argument");
+    info->n_words = (int64_t)s->s.words.size();
+    info->pool_words = s->s.pool_words;
+    info->zero_words = s->s.zero_words;
+    info->loss_word = s->s.loss_word;
+    info->n_barriers = s->s.n_bar;
+    info->n_levels = s->s.n_levels;
+    info->n_nodes = s->s.n_nodes;
+    info->n_heads = s->s.n_heads;
+    info->flops = s->s.flops;
+    info->act_bytes = s->s.act_bytes;
+    return VPPS_OK;
+}
+
+vpps_status vpps_upload_script(vpps_script s, void* stream) {
+    if (!s) return fail(VPPS_E_INVALID, "null script");
+    if (s->model->plan_only) return fail(VPPS_E_STATE, "plan-only model");
+    CK(cudaMemcpyAsync(s->d_words, s->h_pinned, s->s.words.size() * sizeof(uint32_t), cudaMemcpyHostToDevice,
+                       (cudaStream_t)stream));
+    s->uploaded = true;
+    return VPPS_OK;
+}
+
+static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t n_rows, float* d_inputs,
+                       int mode, float lr, float wd, void* stream_) {
+    if (!m || !s) return fail(VPPS_E_INVALID, "null argument");
+    if (m->plan_only) return fail(VPPS_E_STATE, "plan-only model");
+    if (s->model != m) return fail(VPPS_E_STATE, "script was built for another model");
+    if (!m->params || !m->grads) return fail(VPPS_E_STATE, "buffers not bound (vpps_bind_buffers)");
+    if (!inputs || n_rows <= 0) return fail(VPPS_E_INVALID, "null input table");
+    if (s->s.max_token >= n_rows) return fail(VPPS_E_GRAPH, "token out of range of the input table");
+    if (((uintptr_t)inputs | (uintptr_t)d_inputs) & 15) return fail(VPPS_E_INVALID, "input tables must be 16-byte aligned");
+    cudaStream_t st = (cudaStream_t)stream_;
+    CK(cudaSetDevice(m->device));
+    if (s->s.pool_words > m->pool_cap) {
+        if (m->pool) { CK(cudaStreamSynchronize(st)); CK(cudaFree(m->pool)); m->pool = nullptr; }
+        const int64_t cap = s->s.pool_words + s->s.pool_words / 4 + 1024;
+        CK(cudaMalloc(&m->pool, cap * sizeof(float)));
+        m->pool_cap = cap;
+    }
+    m->last_pool_words = s->s.pool_words;
+    if (!s->uploaded) {
+        vpps_status r = vpps_upload_script(s, stream_);
+        if (r != VPPS_OK) return r;
+    }
+    CK(cudaMemsetAsync(m->pool, 0, s->s.zero_words * sizeof(float), st));
+    if (d_inputs) CK(cudaMemsetAsync(d_inputs, 0, (size_t)n_rows * m->plan.E * sizeof(float), st));
+    KParams kp{};
+    kp.params = m->params;
+    kp.grads = m->grads;
+    kp.inputs = inputs;
+    kp.d_inputs = d_inputs;
+    kp.pool = m->pool;
+    kp.script = s->d_words;
+    for (size_t i = 0; i < m->offsets.size() && i < 8; ++i) kp.off[i] = m->offsets[i];
+    kp.n_g = m->plan.n_g;
+    kp.n_act = m->plan.n_act;
+    kp.C = m->plan.C;
+    kp.mode = mode;
+    kp.loss_word = s->s.loss_word;
+    kp.lr = lr;
+    kp.wd = wd;
+    void* args[] = {&kp};
+    CK(cudaLaunchCooperativeKernel(m->var->fn, dim3(m->plan.n_cta), dim3(256), args, m->smem, st));
+    const int slot = (int)(m->passes & 1);
+    CK(cudaMemcpyAsync(m->h_loss + slot, m->pool + s->s.loss_word, sizeof(float), cudaMemcpyDeviceToHost, st));
+    CK(cudaEventRecord(m->ev[slot], st));
+    ++m->passes;
+    return VPPS_OK;
+}
+
+vpps_status vpps_fwd_bwd(vpps_model m, vpps_script s, const float* inputs, int64_t n_input_rows, float* d_inputs,
+                         void* stream) {
+    return run(m, s, inputs, n_input_rows, d_inputs, 0, 0.f, 0.f, stream);
+}
+
+vpps_status vpps_fwd_bwd_sgd(vpps_model m, vpps_script s, const float* inputs, int64_t n_input_rows,
+                             float* d_inputs, float lr, float weight_decay, void* stream) {
+    return run(m, s, inputs, n_input_rows, d_inputs, 1, lr, weight_decay, stream);
+}
+
+vpps_status vpps_sgd_step(vpps_model m, float lr, float weight_decay, void* stream) {
+    if (!m) return fail(VPPS_E_INVALID, "null model");
+    if (m->plan_only || !m->params) return fail(VPPS_E_STATE, "buffers not bound");
+    launch_sgd(m->params, m->grads, m->n_floats, lr, weight_decay, (cudaStream_t)stream);
+    CK(cudaGetLastError());
+    return VPPS_OK;
+}
+
+vpps_status vpps_get_stale_loss(vpps_model m, float* loss) {
+    if (!m || !loss) return fail(VPPS_E_INVALID, "null argument");
+    if (m->plan_only) return fail(VPPS_E_STATE, "plan-only model");
+    if (m->passes < 2) { *loss = 0.f; return VPPS_OK; }
+    const int slot = (int)((m->passes - 2) & 1);
+    CK(cudaEventSynchronize(m->ev[slot]));
+    *loss = m->h_loss[slot];
+    return VPPS_OK;
+}
+
+vpps_status vpps_sync_get_latest_loss(vpps_model m, float* loss) {
+    if (!m || !loss) return fail(VPPS_E_INVALID, "null argument");
+    if (m->plan_only) return fail(VPPS_E_STATE, "plan-only model");
+    if (m->passes < 1) { *loss = 0.f; return VPPS_OK; }
+    const int slot = (int)((m->passes - 1) & 1);
+    CK(cudaEventSynchronize(m->ev[slot]));
+    *loss = m->h_loss[slot];
+    return VPPS_OK;
+}
+
+vpps_status vpps_pool_ptr(vpps_model m, float** pool, int64_t* pool_words) {
+    if (!m || !pool) return fail(VPPS_E_INVALID, "null argument");
+    *pool = m->pool;
+    if (pool_words) *pool_words = m->last_pool_words;
+    return VPPS_OK;
+}
+
+void vpps_destroy_script(vpps_script s) {
+    if (!s) return;
+    if (s->d_words) cudaFree(s->d_words);
+    if (s->h_pinned) cudaFreeHost(s->h_pinned);
+    delete s;
+}
+
+void vpps_destroy_model(vpps_model m) {
+    if (!m) return;
+    if (m->pool) cudaFree(m->pool);
+    if (m->h_loss) cudaFreeHost(m->h_loss);
+    for (cudaEvent_t e : m->ev)
+        if (e) cudaEventDestroy(e);
+    delete m;
+}
+
+}  // extern "C"

@@ -1,0 +1,62 @@
+// Host-side data structures of libvpps (partition plan, super-graph, script).
+// Written from SPEC_SCRIPT.md; PAPER.md line citations at each function.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+namespace vpps {
+
+constexpr uint32_t NONE = 0xFFFFFFFFu;
+
+enum Cell : int32_t { CELL_LSTM = 0, CELL_BINARY = 1, CELL_CHILDSUM = 2 };
+
+enum Op : uint32_t {
+    OP_S = 0x01, OP_W = 0x02,
+    OP_LSTM_F = 0x10, OP_LSTM_B = 0x11,
+    OP_LEAF_F = 0x20, OP_LEAF_B = 0x21, OP_INT_F = 0x22, OP_INT_B = 0x23,
+    OP_CS_F = 0x30, OP_CS_B = 0x31,
+    OP_HEAD_F = 0x40, OP_HEAD_B = 0x41,
+};
+
+struct Shape { int32_t rows, cols; };
+
+// ---- SPEC P0: paper-literal dealer --------------------------------------------------------
+struct DealRow { int32_t matrix, row, cta, partition, warp, is_grad; };
+int32_t regs_per_row(int32_t row_max);
+int32_t reg_budget(int32_t tb, int32_t cps);
+void paper_deal(const std::vector<Shape>& mats, int32_t n_cta, int32_t tb, int32_t rpw, bool pack_rows,
+                bool grads, std::vector<DealRow>* rows, int64_t* n_slots);
+int32_t paper_choose_cps(const std::vector<Shape>& mats, int32_t n_sm, int32_t tb, int32_t rpw, bool pack_rows);
+
+// ---- SPEC P1: unit-bundle plan --------------------------------------------------------------
+struct Plan {
+    int32_t cell, H, E, C;
+    int32_t n_cta, n_g, n_act, umax, G;
+    std::vector<int32_t> table;   // rows of 8 int32
+};
+bool unit_plan(int32_t cell, int32_t H, int32_t E, int32_t C, int32_t n_sm, int32_t cps, int32_t G,
+               Plan* out, std::string* err);
+
+// ---- SPEC §S/§E: script ----------------------------------------------------------------------
+struct BatchIn {
+    int32_t n_graphs;
+    const int32_t* graph_ptr;
+    const int32_t* child_ptr;
+    const int32_t* children;
+    const int32_t* token;
+    const int32_t* label;
+};
+
+struct Script {
+    std::vector<uint32_t> words;
+    int64_t pool_words = 0, zero_words = 0, loss_word = 0;
+    int32_t n_bar = 0, n_levels = 0;
+    int64_t n_nodes = 0, n_heads = 0, max_token = -1;
+    double flops = 0.0, act_bytes = 0.0;
+};
+
+// Returns 0 on success, -4 (graph error) or -1 (invalid) with a message.
+int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Script* out, std::string* err);
+
+}  // namespace vpps

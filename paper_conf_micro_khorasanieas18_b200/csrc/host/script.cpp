@@ -1,0 +1,246 @@
+// Per-batch script generation (SPEC_SCRIPT.md §S, §E).
+//
+// PAPER.md §III-B1: super-graph with aggregated loss (L205); nodes sorted by maximum depth from the
+// sources (L139); forward traversal level by level emitting one CISC instruction per node (L141,
+// L159: 4-byte preamble with op type and input tensor length, then 4-byte pool offsets); signal and
+// wait between consecutive levels among the participating virtual processors (L165); reverse
+// traversal for back-propagation with min-load assignment (L167); scripts concatenated behind the
+// prefix sum of their lengths for one host-to-device copy (L169).
+#include <algorithm>
+#include <cstring>
+#include "host.h"
+
+namespace vpps {
+namespace {
+
+inline int64_t align32(int64_t x) { return (x + 31) / 32 * 32; }
+inline uint32_t preamble(uint32_t op, int64_t len) { return op | (uint32_t)(len << 8); }
+
+enum Kind : int8_t { K_LEAF, K_INT, K_CS, K_LSTM, K_HEAD };
+
+struct Node {
+    Kind kind;
+    int32_t token, label;
+    int32_t ch_begin, ch_count;   // into Graph::kids (global ids)
+};
+
+}  // namespace
+
+int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Script* out, std::string* err) {
+    const int64_t H = plan.H, E = plan.E, C = plan.C;
+    if (b.n_graphs < 0 || (b.n_graphs > 0 && (!b.graph_ptr || !b.child_ptr || !b.token || !b.label))) {
+        *err = "null batch array";
+        return -1;
+    }
+    // ---- S1/S2: super-graph (cells in given order, then heads of labelled cells) -----------------
+    std::vector<Node> nodes;
+    std::vector<int32_t> kids;
+    std::vector<int32_t> parents_seen;
+    for (int32_t g = 0; g < b.n_graphs; ++g) {
+        const int32_t first = b.graph_ptr[g], last = b.graph_ptr[g + 1];
+        if (last < first) { *err = "graph_ptr not monotone"; return -4; }
+        const int32_t base = (int32_t)nodes.size();
+        parents_seen.assign(last - first, 0);
+        for (int32_t v = first; v < last; ++v) {
+            const int32_t local = v - first;
+            const int32_t c0 = b.child_ptr[v], c1 = b.child_ptr[v + 1];
+            const int32_t nch = c1 - c0, tok = b.token[v], lab = b.label[v];
+            if (nch < 0) { *err = "child_ptr not monotone"; return -4; }
+            if (tok < -1 || tok >= n_input_rows) { *err = "token out of range"; return -4; }
+            if (lab < -1 || lab >= C) { *err = "label out of range"; return -4; }
+            Node nd{K_CS, tok, lab, (int32_t)kids.size(), nch};
+            for (int32_t k = c0; k < c1; ++k) {
+                const int32_t ch = b.children[k];
+                if (ch < 0 || ch >= local) { *err = "children must precede their parent"; return -4; }
+                if (++parents_seen[ch] > 1) { *err = "a node may have at most one parent"; return -4; }
+                kids.push_back(base + ch);
+            }
+            switch (plan.cell) {
+                case CELL_BINARY:
+                    if (nch == 0 && tok >= 0) nd.kind = K_LEAF;
+                    else if (nch == 2 && tok < 0) nd.kind = K_INT;
+                    else { *err = "binary Tree-LSTM: leaves carry a token, internal nodes have 2 children"; return -4; }
+                    break;
+                case CELL_LSTM:
+                    if (nch > 1 || tok < 0 || (nch == 1 && b.children[c0] != local - 1)) {
+                        *err = "LSTM chain: node t has child t-1 and a token";
+                        return -4;
+                    }
+                    nd.kind = K_LSTM;
+                    break;
+                default:
+                    if (nch > 8) { *err = "child-sum node with more than 8 children"; return -4; }
+                    nd.kind = K_CS;
+            }
+            nodes.push_back(nd);
+        }
+        for (int32_t v = first; v < last; ++v)
+            if (b.label[v] >= 0) {
+                nodes.push_back(Node{K_HEAD, -1, b.label[v], (int32_t)kids.size(), 1});
+                kids.push_back(base + (v - first));
+            }
+    }
+    const int64_t N = (int64_t)nodes.size();
+    if (N == 0) { *err = "empty batch"; return -4; }
+
+    // ---- S3: level = maximum depth from the sources (L139) --------------------------------------
+    std::vector<int32_t> level(N, 0);
+    int32_t L = 0;
+    for (int64_t i = 0; i < N; ++i) {
+        int32_t lv = 0;
+        for (int32_t k = 0; k < nodes[i].ch_count; ++k)
+            lv = std::max(lv, level[kids[nodes[i].ch_begin + k]] + 1);
+        level[i] = lv;
+        L = std::max(L, lv);
+    }
+
+    // ---- S7: pool plan ------------------------------------------------------------------------
+    const int32_t n_bar = 2 * L + 1;
+    const int64_t loss_word = align32(n_bar + 1);
+    int64_t cursor = align32(loss_word + 1);
+    std::vector<uint32_t> adj(N, NONE), rec(N, 0);
+    for (int64_t i = 0; i < N; ++i)
+        if (nodes[i].kind != K_HEAD) { adj[i] = (uint32_t)cursor; cursor = align32(cursor + 2 * H); }
+    const int64_t zero_words = cursor;
+    for (int64_t i = 0; i < N; ++i) {
+        int64_t sz = 0;
+        switch (nodes[i].kind) {
+            case K_LSTM: sz = 6 * H; break;
+            case K_LEAF: sz = 5 * H; break;
+            case K_INT: sz = 7 * H; break;
+            case K_CS: sz = (5 + nodes[i].ch_count) * H; break;
+            case K_HEAD: sz = C + 1; break;
+        }
+        rec[i] = (uint32_t)cursor;
+        cursor = align32(cursor + sz);
+    }
+    if (cursor >= (int64_t)NONE) { *err = "pool exceeds 2^32 words (16 GiB, L159)"; return -1; }
+
+    // ---- per-node cost (MACs; L167 "relatively higher load" for cached-matrix ops) and FLOPs -----
+    auto macs = [&](int64_t i) -> int64_t {
+        const Node& n = nodes[i];
+        switch (n.kind) {
+            case K_LEAF: return 3 * H * E;
+            case K_INT: return 8 * H * H;
+            case K_CS: return (n.token >= 0 ? 4 * H * E : 0) + (n.ch_count ? (3 + n.ch_count) * H * H : 0);
+            case K_LSTM: return 4 * H * E + (n.ch_count ? 4 * H * H : 0);
+            case K_HEAD: return C * H;
+        }
+        return 0;
+    };
+    double flops = 0.0, abytes = 0.0;
+    for (int64_t i = 0; i < N; ++i) {
+        flops += 6.0 * (double)macs(i);   // forward, weight gradient, input/hidden gradient (2 FLOP/MAC)
+        const Node& n = nodes[i];
+        const double nc = n.ch_count;
+        double kin = 0, recsz = 0;
+        switch (n.kind) {
+            case K_LEAF: kin = E; recsz = 5 * H; break;
+            case K_INT: kin = 2 * H; recsz = 7 * H; break;
+            case K_CS: kin = E + H * (1 + nc); recsz = (5 + nc) * H; break;
+            case K_LSTM: kin = E + H; recsz = 6 * H; break;
+            case K_HEAD: kin = H; recsz = C + 1; break;
+        }
+        if (n.kind == K_HEAD) abytes += 4.0 * (H + (C + 1) + (C + 1) + 2 * H);
+        else abytes += 4.0 * ((kin + nc * H + recsz) + (recsz + 2 * H + kin + nc * H + nc * 2 * H));
+    }
+
+    // ---- instruction encoding (§E) -------------------------------------------------------------
+    auto emit = [&](std::vector<uint32_t>& w, int64_t i, bool fwd) {
+        const Node& n = nodes[i];
+        const int32_t* ch = kids.data() + n.ch_begin;
+        const uint32_t tok = n.token < 0 ? NONE : (uint32_t)n.token;
+        switch (n.kind) {
+            case K_LEAF:
+                if (fwd) w.insert(w.end(), {preamble(OP_LEAF_F, E), rec[i], tok});
+                else w.insert(w.end(), {preamble(OP_LEAF_B, E), rec[i], adj[i], tok});
+                break;
+            case K_INT:
+                if (fwd) w.insert(w.end(), {preamble(OP_INT_F, 2 * H), rec[i], rec[ch[0]], rec[ch[1]]});
+                else w.insert(w.end(), {preamble(OP_INT_B, 2 * H), rec[i], adj[i], rec[ch[0]], adj[ch[0]],
+                                        rec[ch[1]], adj[ch[1]]});
+                break;
+            case K_LSTM: {
+                const uint32_t pr = n.ch_count ? rec[ch[0]] : NONE, pa = n.ch_count ? adj[ch[0]] : NONE;
+                if (fwd) w.insert(w.end(), {preamble(OP_LSTM_F, E + H), rec[i], tok, pr});
+                else w.insert(w.end(), {preamble(OP_LSTM_B, E + H), rec[i], adj[i], tok, pr, pa});
+                break;
+            }
+            case K_CS:
+                if (fwd) {
+                    w.insert(w.end(), {preamble(OP_CS_F, n.ch_count), rec[i], tok});
+                    for (int32_t k = 0; k < n.ch_count; ++k) w.push_back(rec[ch[k]]);
+                } else {
+                    w.insert(w.end(), {preamble(OP_CS_B, n.ch_count), rec[i], adj[i], tok});
+                    for (int32_t k = 0; k < n.ch_count; ++k) { w.push_back(rec[ch[k]]); w.push_back(adj[ch[k]]); }
+                }
+                break;
+            case K_HEAD:
+                if (fwd) w.insert(w.end(), {preamble(OP_HEAD_F, H), rec[i], rec[ch[0]], (uint32_t)n.label});
+                else w.insert(w.end(), {preamble(OP_HEAD_B, H), rec[i], rec[ch[0]], adj[ch[0]], (uint32_t)n.label});
+                break;
+        }
+    };
+
+    // ---- S4-S6: phases, min-load groups, signal/wait ------------------------------------------
+    const int32_t G = plan.G, P = 2 * L + 2;
+    std::vector<std::vector<int64_t>> at_level(L + 1);
+    for (int64_t i = 0; i < N; ++i) at_level[level[i]].push_back(i);   // ascending global id
+    std::vector<std::vector<uint32_t>> streams(G);
+    std::vector<uint32_t> targets(n_bar + 1, 0);
+    std::vector<std::vector<uint32_t>> body(G);
+    std::vector<int64_t> load(G);
+    std::vector<char> was_active(G, 0);
+    for (int32_t p = 0; p < P; ++p) {
+        const bool fwd = p <= L;
+        const int32_t lv = fwd ? p : 2 * L + 1 - p;
+        for (int32_t g = 0; g < G; ++g) { body[g].clear(); load[g] = 0; }
+        for (int64_t i : at_level[lv]) {
+            int32_t best = 0;
+            for (int32_t g = 1; g < G; ++g)
+                if (load[g] < load[best]) best = g;
+            load[best] += macs(i);
+            emit(body[best], i, fwd);
+        }
+        int32_t active_prev = 0;
+        for (int32_t g = 0; g < G; ++g) active_prev += was_active[g];
+        if (p >= 1) targets[p] = (uint32_t)(plan.n_act * active_prev);
+        for (int32_t g = 0; g < G; ++g) {
+            const bool active = !body[g].empty();
+            if (active) {
+                if (p >= 1) streams[g].push_back(preamble(OP_W, p));
+                streams[g].insert(streams[g].end(), body[g].begin(), body[g].end());
+                if (p < P - 1) streams[g].push_back(preamble(OP_S, p + 1));
+            }
+            was_active[g] = active;
+        }
+    }
+
+    // ---- header: [G, n_bar, prefix sums], streams, barrier targets (L169) ---------------------
+    Script& s = *out;
+    s.words.clear();
+    s.words.push_back((uint32_t)G);
+    s.words.push_back((uint32_t)n_bar);
+    uint32_t run = 0;
+    s.words.push_back(0);
+    for (int32_t g = 0; g < G; ++g) { run += (uint32_t)streams[g].size(); s.words.push_back(run); }
+    for (int32_t g = 0; g < G; ++g) s.words.insert(s.words.end(), streams[g].begin(), streams[g].end());
+    s.words.insert(s.words.end(), targets.begin(), targets.end());
+    s.pool_words = cursor;
+    s.zero_words = zero_words;
+    s.loss_word = loss_word;
+    s.n_bar = n_bar;
+    s.n_levels = L + 1;
+    s.n_nodes = N;
+    s.n_heads = 0;
+    s.max_token = -1;
+    for (const Node& n : nodes) {
+        s.n_heads += n.kind == K_HEAD;
+        s.max_token = std::max<int64_t>(s.max_token, n.token);
+    }
+    s.flops = flops;
+    s.act_bytes = abytes;
+    return 0;
+}
+
+}  // namespace vpps

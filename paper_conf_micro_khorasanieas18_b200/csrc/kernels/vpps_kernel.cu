@@ -1,0 +1,797 @@
+// The VPPS persistent forward-backward kernel for sm_100a (B200).
+//
+// PAPER.md §III: one kernel per training step does forward, backward and the parameter update
+// (L25, L84) with the model's weight matrices held in registers for the whole pass (L23, L92).
+// Each CTA is a virtual CISC-like vector processor (L25, L137) that fetches its script into shared
+// memory and loops decode->execute (L171-177, Fig.7), synchronising with the other processors through
+// signal/wait counters in global memory (L165).  Prologue: load cached weights from the DRAM master
+// copy and zero the gradient registers (L123, L129).  Epilogue: apply the gradients (L129, L197).
+//
+// B200 design: 148 persistent CTAs x 256 threads (L102, L106), gate-colocated unit
+// bundles (SPEC P1): the CTA that owns hidden unit j holds every gate row of j, so a cell update is
+// CTA-local and needs no barrier between matvec and cell; thread tau of a unit's thread group holds
+// columns CG*(tau + TU*t) + q of every gate row (coalesced, 16-B vectorised staging/reads), partial dot
+// products are reduced by warp shuffles then across the group's warps in shared memory; the transposed
+// product of the backward pass is issued as vector red.global.add.v4.f32 (L94, fn4 L100).
+#include <cstdio>
+#include "vpps_kernel.cuh"
+
+namespace vpps {
+namespace dev {
+
+constexpr int NTH = 256;       // CTA width (L102)
+constexpr int NBMAX = 16;      // instructions executed as one batch
+constexpr int CHUNK = 4096;    // script words staged in shared memory (L171)
+constexpr int CHMAX = 8;       // child-sum children per node
+constexpr int CHSLOT = 32;     // child vectors staged per child-sum batch
+constexpr uint32_t NONE = 0xFFFFFFFFu;
+constexpr int CELL_LSTM = 0, CELL_BINARY = 1, CELL_CHILDSUM = 2;
+enum : uint32_t {
+    OP_S = 0x01, OP_W = 0x02, OP_LSTM_F = 0x10, OP_LSTM_B = 0x11, OP_LEAF_F = 0x20, OP_LEAF_B = 0x21,
+    OP_INT_F = 0x22, OP_INT_B = 0x23, OP_CS_F = 0x30, OP_CS_B = 0x31, OP_HEAD_F = 0x40, OP_HEAD_B = 0x41
+};
+
+__device__ __forceinline__ int instr_words(uint32_t w) {
+    const uint32_t len = w >> 8;
+    switch (w & 0xFF) {
+        case OP_LSTM_F: return 4;
+        case OP_LSTM_B: return 6;
+        case OP_LEAF_F: return 3;
+        case OP_LEAF_B: return 4;
+        case OP_INT_F: return 4;
+        case OP_INT_B: return 7;
+        case OP_CS_F: return 3 + (int)len;
+        case OP_CS_B: return 4 + 2 * (int)len;
+        case OP_HEAD_F: return 4;
+        case OP_HEAD_B: return 5;
+        default: return 1;
+    }
+}
+
+// Column layout of a K-long bundle row over TU threads: granules of CG consecutive floats.
+template <int K, int TU>
+struct Lay {
+    static constexpr int CG = (K >= 4 * TU) ? 4 : ((K >= 2 * TU) ? 2 : 1);
+    static constexpr int NT = (K + CG * TU - 1) / (CG * TU);
+    static constexpr int NREG = NT * CG;
+    static constexpr int KP = NT * CG * TU;   // padded row length of the staged input
+};
+
+constexpr int cmax(int a, int b) { return a > b ? a : b; }
+constexpr int a4(int x) { return (x + 3) / 4 * 4; }
+
+template <int CELL, int H, int E, int UMAX>
+struct Cfg {
+    static constexpr int TU = NTH / UMAX;
+    static constexpr int WPU = TU / 32;
+    static constexpr bool BIN = CELL == CELL_BINARY, CS = CELL == CELL_CHILDSUM, LS = CELL == CELL_LSTM;
+    static constexpr int KA = BIN ? E : E + H;
+    static constexpr int RA = BIN ? 3 : 4;
+    static constexpr int KB = BIN ? 2 * H : 4;
+    static constexpr int RB = BIN ? 4 : 1;
+    using LA = Lay<KA, TU>;
+    using LB = Lay<KB, TU>;
+    static constexpr int KPMAX = BIN ? cmax(LA::KP, LB::KP) : LA::KP;
+    static constexpr int RO = BIN ? 5 : (LS ? 4 : 4 + CHMAX);
+    static constexpr int GO = BIN ? 5 : (LS ? 4 : 4 + CHMAX);
+    static constexpr int O_X = CHUNK;
+    static constexpr int O_CH = O_X + NBMAX * KPMAX;
+    static constexpr int O_RED = O_CH + (CS ? CHSLOT * KPMAX : 0);
+    static constexpr int O_GB = O_RED + 8 * NBMAX * RO;
+    static constexpr int O_BIAS = O_GB + UMAX * NBMAX * GO;
+    static constexpr int O_DBIAS = O_BIAS + UMAX * 4;
+    static constexpr int O_IPOS = O_DBIAS + UMAX * 4;
+    static constexpr int O_CSLOT = O_IPOS + NBMAX;
+    static constexpr int O_HEAD = a4(O_CSLOT + NBMAX);
+    static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 3 * C + H + 8); }
+};
+
+__device__ __forceinline__ float sigm(float x) { return 1.0f / (1.0f + expf(-x)); }
+
+__device__ __forceinline__ float4 ld4cg(const float* p) { return __ldcg(reinterpret_cast<const float4*>(p)); }
+__device__ __forceinline__ float4 ld4g(const float* p) { return __ldg(reinterpret_cast<const float4*>(p)); }
+
+// Vectorised no-return float add in L2 (REDG.E.ADD.F32x4 on sm_90+): remote accumulation of the
+// transposed matrix-vector product (fn4 L100).
+template <int CG>
+__device__ __forceinline__ void red_add(float* p, const float* v) {
+    if constexpr (CG == 4) {
+        asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(v[0]), "f"(v[1]), "f"(v[2]),
+                     "f"(v[3])
+                     : "memory");
+    } else if constexpr (CG == 2) {
+        asm volatile("red.global.add.v2.f32 [%0], {%1, %2};" ::"l"(p), "f"(v[0]), "f"(v[1]) : "memory");
+    } else {
+        atomicAdd(p, v[0]);
+    }
+}
+
+template <int CG>
+__device__ __forceinline__ void lds(const float* p, float* v) {
+    if constexpr (CG == 4) {
+        const float4 t = *reinterpret_cast<const float4*>(p);
+        v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
+    } else if constexpr (CG == 2) {
+        const float2 t = *reinterpret_cast<const float2*>(p);
+        v[0] = t.x; v[1] = t.y;
+    } else {
+        v[0] = *p;
+    }
+}
+
+template <int N>
+__device__ __forceinline__ void warp_allreduce(float (&a)[N], int n_used) {
+#pragma unroll
+    for (int o = 0; o < N; ++o) {
+        if (o < n_used) {
+#pragma unroll
+            for (int s = 16; s >= 1; s >>= 1) a[o] += __shfl_xor_sync(0xffffffffu, a[o], s);
+        }
+    }
+}
+
+// Signal/wait barriers (L165): release-add on a global counter; acquire-spin until the target count.
+__device__ __forceinline__ void bar_signal(unsigned* ctr) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(ctr) : "memory");
+    }
+}
+__device__ __forceinline__ void bar_wait(const unsigned* ctr, unsigned target) {
+    if (threadIdx.x == 0) {
+        unsigned v;
+        while (true) {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+            if (v >= target) break;
+            __nanosleep(32);
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+template <int CELL, int H, int E, int UMAX>
+__global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
+    using T = Cfg<CELL, H, E, UMAX>;
+    using LA = typename T::LA;
+    using LB = typename T::LB;
+    constexpr int TU = T::TU, WPU = T::WPU;
+    constexpr bool BIN = T::BIN, CS = T::CS, LS = T::LS;
+    constexpr int KA = T::KA, KB = T::KB, RA = T::RA, RB = T::RB, RO = T::RO, GO = T::GO;
+
+    extern __shared__ __align__(16) uint32_t smw[];
+    float* sm = reinterpret_cast<float*>(smw);
+    uint32_t* chunk = smw;
+    float* xs = sm + T::O_X;
+    float* chs = sm + T::O_CH;
+    float* red = sm + T::O_RED;
+    float* gb = sm + T::O_GB;
+    float* bias = sm + T::O_BIAS;
+    float* dbias = sm + T::O_DBIAS;
+    int* ipos = reinterpret_cast<int*>(smw + T::O_IPOS);
+    int* cslot = reinterpret_cast<int*>(smw + T::O_CSLOT);
+    const int C = P.C;
+    float* Wo = sm + T::O_HEAD;
+    float* dWo = Wo + C * H;
+    float* bo = dWo + C * H;
+    float* dbo = bo + C;
+    float* zs = dbo + C;
+    float* hbuf = zs + C;
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int lc = blockIdx.x % P.n_g, grp = blockIdx.x / P.n_g;
+    if (lc >= P.n_act) return;                       // holds no atom: not a participant
+    const uint32_t* S = P.script;
+    const uint32_t G = S[0];
+    const uint32_t hdr = 2 + G + 1;
+    const uint32_t s0 = hdr + S[2 + grp], s1 = hdr + S[3 + grp];
+    const uint32_t* target = S + hdr + S[2 + G];
+    unsigned* bar = reinterpret_cast<unsigned*>(P.pool);
+    float* pool = P.pool;
+    const float* __restrict__ inputs = P.inputs;
+
+    const int u = tid / TU, tu = tid % TU;
+    const int j = lc + u * P.n_g;                    // hidden unit owned by this thread's slot
+    const bool unit_ok = j < H;
+    const bool holds_head = (lc == H % P.n_g);
+    const int64_t* off = P.off;
+
+    // ---------------- prologue: weights DRAM -> registers, zero gradient registers (L123, L129) ----
+    auto idxA = [&](int r, int col) -> int64_t {
+        if constexpr (BIN) return off[0] + (int64_t)(r * H + j) * E + col;
+        else if constexpr (LS)
+            return col < E ? off[0] + (int64_t)(r * H + j) * E + col : off[1] + (int64_t)(r * H + j) * H + (col - E);
+        else {
+            if (r < 3) return col < E ? off[0] + (int64_t)(r * H + j) * E + col : off[2] + (int64_t)(r * H + j) * H + (col - E);
+            return col < E ? off[1] + (int64_t)j * E + col : off[3] + (int64_t)j * H + (col - E);
+        }
+    };
+    auto idxB = [&](int r, int col) -> int64_t {
+        if (r < 3) return off[1] + (int64_t)(r * H + j) * (2 * H) + col;
+        return col < H ? off[2] + (int64_t)j * H + col : off[3] + (int64_t)j * H + (col - H);
+    };
+    float wa[RA][LA::NREG], dwa[RA][LA::NREG];
+    float wb[RB][LB::NREG], dwb[RB][LB::NREG];
+#pragma unroll
+    for (int r = 0; r < RA; ++r)
+#pragma unroll
+        for (int t = 0; t < LA::NT; ++t)
+#pragma unroll
+            for (int q = 0; q < LA::CG; ++q) {
+                const int col = LA::CG * (tu + TU * t) + q;
+                wa[r][t * LA::CG + q] = (unit_ok && col < KA) ? __ldg(P.params + idxA(r, col)) : 0.f;
+                dwa[r][t * LA::CG + q] = 0.f;
+            }
+    if constexpr (BIN) {
+#pragma unroll
+        for (int r = 0; r < RB; ++r)
+#pragma unroll
+            for (int t = 0; t < LB::NT; ++t)
+#pragma unroll
+                for (int q = 0; q < LB::CG; ++q) {
+                    const int col = LB::CG * (tu + TU * t) + q;
+                    wb[r][t * LB::CG + q] = (unit_ok && col < KB) ? __ldg(P.params + idxB(r, col)) : 0.f;
+                    dwb[r][t * LB::CG + q] = 0.f;
+                }
+    }
+    const int bias_m0 = LS ? 3 : 5;                  // first bias parameter
+    if (tid < UMAX * 4) {
+        const int uu = tid / 4, k = tid % 4, jj = lc + uu * P.n_g;
+        float v = 0.f;
+        if (jj < H) v = (LS || k < 3) ? __ldg(P.params + off[bias_m0] + k * H + jj) : __ldg(P.params + off[6] + jj);
+        bias[tid] = v;
+        dbias[tid] = 0.f;
+    }
+    const int wout_m = LS ? 2 : 4, bout_m = LS ? 4 : 7;
+    if (holds_head) {
+        for (int i = tid; i < C * H; i += NTH) { Wo[i] = __ldg(P.params + off[wout_m] + i); dWo[i] = 0.f; }
+        for (int i = tid; i < C; i += NTH) { bo[i] = __ldg(P.params + off[bout_m] + i); dbo[i] = 0.f; }
+    }
+
+    // ---------------- script interpretation (L171-177) ---------------------------------------------
+    uint32_t cbase = s0;
+    auto refill = [&](uint32_t from) {
+        __syncthreads();
+        for (uint32_t i = tid; i < (uint32_t)CHUNK && from + i < s1; i += NTH) chunk[i] = S[from + i];
+        __syncthreads();
+        cbase = from;
+    };
+    refill(s0);
+    uint32_t pos = s0;
+    while (pos < s1) {
+        if (pos + 640 > cbase + CHUNK && cbase + CHUNK < s1) refill(pos);
+        const uint32_t pre = chunk[pos - cbase];
+        const uint32_t op = pre & 0xFF;
+        if (op == OP_S) { bar_signal(bar + (pre >> 8)); ++pos; continue; }
+        if (op == OP_W) { bar_wait(bar + (pre >> 8), target[pre >> 8]); ++pos; continue; }
+        // gather a batch of consecutive instructions with the same opcode
+        __syncthreads();
+        int nb = 0, used = 0;
+        uint32_t p = pos;
+        while (p < s1 && nb < NBMAX) {
+            const uint32_t w = chunk[p - cbase];
+            if ((w & 0xFF) != op) break;
+            const int sz = instr_words(w);
+            if (p + sz > cbase + CHUNK) break;
+            const bool cs_op = CS && (op == OP_CS_F || op == OP_CS_B);
+            if (cs_op && used + (int)(w >> 8) > CHSLOT) break;
+            if (tid == 0) { ipos[nb] = (int)(p - cbase); cslot[nb] = used; }
+            if (cs_op) used += (int)(w >> 8);
+            ++nb;
+            p += sz;
+        }
+        __syncthreads();
+        const bool is_head = (op == OP_HEAD_F || op == OP_HEAD_B);
+        if (is_head) {
+            if (holds_head) {
+                for (int n = 0; n < nb; ++n) {
+                    const uint32_t* I = chunk + ipos[n];
+                    const uint32_t rec = I[1], crec = I[2];
+                    const int y = (int)(op == OP_HEAD_F ? I[3] : I[4]);
+                    for (int k = tid; k < H; k += NTH) hbuf[k] = __ldcg(pool + crec + k);
+                    if (op == OP_HEAD_B)
+                        for (int c = tid; c < C; c += NTH) zs[c] = __ldcg(pool + rec + c) - (c == y ? 1.f : 0.f);
+                    __syncthreads();
+                    if (op == OP_HEAD_F) {
+                        for (int c = warp; c < C; c += NTH / 32) {
+                            float s = 0.f;
+                            for (int k = lane; k < H; k += 32) s += Wo[c * H + k] * hbuf[k];
+#pragma unroll
+                            for (int sh = 16; sh >= 1; sh >>= 1) s += __shfl_xor_sync(0xffffffffu, s, sh);
+                            if (lane == 0) zs[c] = s + bo[c];
+                        }
+                        __syncthreads();
+                        if (warp == 0) {
+                            float m = -INFINITY;
+                            for (int c = lane; c < C; c += 32) m = fmaxf(m, zs[c]);
+#pragma unroll
+                            for (int sh = 16; sh >= 1; sh >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, sh));
+                            float se = 0.f;
+                            for (int c = lane; c < C; c += 32) se += expf(zs[c] - m);
+#pragma unroll
+                            for (int sh = 16; sh >= 1; sh >>= 1) se += __shfl_xor_sync(0xffffffffu, se, sh);
+                            const float lse = m + logf(se);
+                            for (int c = lane; c < C; c += 32) pool[rec + c] = expf(zs[c] - lse);
+                            if (lane == 0) {
+                                const float loss = lse - zs[y];
+                                pool[rec + C] = loss;
+                                atomicAdd(pool + P.loss_word, loss);   // aggregated loss node (L205)
+                            }
+                        }
+                    } else {
+                        const uint32_t cadj = I[3];
+                        for (int c = tid; c < C; c += NTH) dbo[c] += zs[c];
+                        for (int i = tid; i < C * H; i += NTH) dWo[i] += zs[i / H] * hbuf[i % H];
+                        for (int k = tid; k < H; k += NTH) {
+                            float s = 0.f;
+                            for (int c = 0; c < C; ++c) s += Wo[c * H + k] * zs[c];
+                            atomicAdd(pool + cadj + k, s);
+                        }
+                    }
+                    __syncthreads();
+                }
+            }
+            pos = p;
+            continue;
+        }
+
+        const bool fwd = (op & 1) == 0;
+        const bool kindB = BIN && (op == OP_INT_F || op == OP_INT_B);
+        // ---- stage the node inputs (coalesced 16-B loads) into shared memory ----
+        {
+            const int KP = kindB ? LB::KP : LA::KP;
+            const int q4 = KP / 4;
+            for (int i = tid; i < nb * q4; i += NTH) {
+                const int n = i / q4, c = (i - n * q4) * 4;
+                const uint32_t* I = chunk + ipos[n];
+                float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+                if constexpr (BIN) {
+                    if (!kindB) {
+                        const uint32_t tok = fwd ? I[2] : I[3];
+                        if (c < E) v = ld4g(inputs + (int64_t)tok * E + c);
+                    } else {
+                        const uint32_t rl = fwd ? I[2] : I[3], rr = fwd ? I[3] : I[5];
+                        if (c < H) v = ld4cg(pool + rl + c);
+                        else if (c < 2 * H) v = ld4cg(pool + rr + (c - H));
+                    }
+                } else if constexpr (LS) {
+                    const uint32_t tok = fwd ? I[2] : I[3], prv = fwd ? I[3] : I[4];
+                    if (c < E) v = ld4g(inputs + (int64_t)tok * E + c);
+                    else if (c < E + H && prv != NONE) v = ld4cg(pool + prv + (c - E));
+                } else {
+                    const uint32_t tok = fwd ? I[2] : I[3];
+                    const int nch = (int)(I[0] >> 8);
+                    if (c < E) {
+                        if (tok != NONE) v = ld4g(inputs + (int64_t)tok * E + c);
+                    } else if (c < E + H) {
+                        for (int k = 0; k < nch; ++k) {
+                            const uint32_t ck = fwd ? I[3 + k] : I[4 + 2 * k];
+                            const float4 hv = ld4cg(pool + ck + (c - E));
+                            v.x += hv.x; v.y += hv.y; v.z += hv.z; v.w += hv.w;
+                            *reinterpret_cast<float4*>(chs + (cslot[n] + k) * KP + c) = hv;
+                        }
+                    }
+                    if (!(c >= E && c < E + H))
+                        for (int k = 0; k < nch; ++k)
+                            *reinterpret_cast<float4*>(chs + (cslot[n] + k) * KP + c) = make_float4(0.f, 0.f, 0.f, 0.f);
+                }
+                *reinterpret_cast<float4*>(xs + n * KP + c) = v;
+            }
+        }
+
+        if (fwd) {
+            __syncthreads();
+            // ---- matrix-vector products from registers (L123): partial sums per warp ----
+            for (int n = 0; n < nb; ++n) {
+                float acc[RO];
+#pragma unroll
+                for (int o = 0; o < RO; ++o) acc[o] = 0.f;
+                int n_used = RO;
+                if (kindB) {
+                    if constexpr (BIN) {
+                        const float* x = xs + n * LB::KP;
+#pragma unroll
+                        for (int t = 0; t < LB::NT; ++t) {
+                            const int col0 = LB::CG * (tu + TU * t);
+                            float xv[LB::CG];
+                            lds<LB::CG>(x + col0, xv);
+                            const bool lo = col0 < H;
+#pragma unroll
+                            for (int q = 0; q < LB::CG; ++q) {
+                                const int k = t * LB::CG + q;
+#pragma unroll
+                                for (int r = 0; r < 3; ++r) acc[r] = fmaf(wb[r][k], xv[q], acc[r]);
+                                const float pf = wb[3][k] * xv[q];
+                                acc[3] += lo ? pf : 0.f;
+                                acc[4] += lo ? 0.f : pf;
+                            }
+                        }
+                    }
+                } else {
+                    const float* x = xs + n * LA::KP;
+#pragma unroll
+                    for (int t = 0; t < LA::NT; ++t) {
+                        const int col0 = LA::CG * (tu + TU * t);
+                        float xv[LA::CG];
+                        lds<LA::CG>(x + col0, xv);
+#pragma unroll
+                        for (int q = 0; q < LA::CG; ++q) {
+                            const int k = t * LA::CG + q;
+                            if constexpr (BIN) {
+#pragma unroll
+                                for (int r = 0; r < 3; ++r) acc[r] = fmaf(wa[r][k], xv[q], acc[r]);
+                            } else if constexpr (LS) {
+#pragma unroll
+                                for (int r = 0; r < 4; ++r) acc[r] = fmaf(wa[r][k], xv[q], acc[r]);
+                            } else {
+#pragma unroll
+                                for (int r = 0; r < 3; ++r) acc[r] = fmaf(wa[r][k], xv[q], acc[r]);
+                                if (col0 < E) acc[3] = fmaf(wa[3][k], xv[q], acc[3]);
+                            }
+                        }
+                    }
+                    if constexpr (CS) {
+                        const uint32_t* I = chunk + ipos[n];
+                        const int nch = (int)(I[0] >> 8);
+                        n_used = 4 + nch;
+#pragma unroll
+                        for (int kc = 0; kc < CHMAX; ++kc) {
+                            if (kc < nch) {
+                                const float* y = chs + (cslot[n] + kc) * LA::KP;
+#pragma unroll
+                                for (int t = 0; t < LA::NT; ++t) {
+                                    const int col0 = LA::CG * (tu + TU * t);
+                                    float yv[LA::CG];
+                                    lds<LA::CG>(y + col0, yv);
+#pragma unroll
+                                    for (int q = 0; q < LA::CG; ++q)
+                                        acc[4 + kc] = fmaf(wa[3][t * LA::CG + q], yv[q], acc[4 + kc]);
+                                }
+                            }
+                        }
+                    } else if constexpr (BIN) {
+                        n_used = 3;
+                    }
+                }
+                warp_allreduce<RO>(acc, n_used);
+                if (lane == 0) {
+#pragma unroll
+                    for (int o = 0; o < RO; ++o)
+                        if (o < n_used) red[(warp * NBMAX + n) * RO + o] = acc[o];
+                }
+            }
+            __syncthreads();
+            // ---- cell update, one thread per (unit slot, node): CTA-local thanks to gate colocation ----
+            if (tid < UMAX * NBMAX) {
+                const int uu = tid / NBMAX, n = tid % NBMAX, jj = lc + uu * P.n_g;
+                if (n < nb && jj < H) {
+                    const uint32_t* I = chunk + ipos[n];
+                    const uint32_t rec = I[1];
+                    float a[RO];
+#pragma unroll
+                    for (int o = 0; o < RO; ++o) {
+                        float s = 0.f;
+#pragma unroll
+                        for (int w = 0; w < WPU; ++w) s += red[((uu * WPU + w) * NBMAX + n) * RO + o];
+                        a[o] = s;
+                    }
+                    const float* b = bias + uu * 4;
+                    if constexpr (BIN) {
+                        const float i = sigm(a[0] + b[0]), o = sigm(a[1] + b[1]), uv = tanhf(a[2] + b[2]);
+                        float c = i * uv;
+                        if (kindB) {
+                            const float fl = sigm(a[3] + b[3]), fr = sigm(a[4] + b[3]);
+                            c += fl * __ldcg(pool + I[2] + H + jj) + fr * __ldcg(pool + I[3] + H + jj);
+                            pool[rec + 5 * H + jj] = fl;
+                            pool[rec + 6 * H + jj] = fr;
+                        }
+                        pool[rec + jj] = o * tanhf(c);
+                        pool[rec + H + jj] = c;
+                        pool[rec + 2 * H + jj] = i;
+                        pool[rec + 3 * H + jj] = o;
+                        pool[rec + 4 * H + jj] = uv;
+                    } else if constexpr (LS) {
+                        const float i = sigm(a[0] + b[0]), f = sigm(a[1] + b[1]), o = sigm(a[2] + b[2]),
+                                    g = tanhf(a[3] + b[3]);
+                        const float cp = I[3] != NONE ? __ldcg(pool + I[3] + H + jj) : 0.f;
+                        const float c = f * cp + i * g;
+                        pool[rec + jj] = o * tanhf(c);
+                        pool[rec + H + jj] = c;
+                        pool[rec + 2 * H + jj] = i;
+                        pool[rec + 3 * H + jj] = f;
+                        pool[rec + 4 * H + jj] = o;
+                        pool[rec + 5 * H + jj] = g;
+                    } else {
+                        const int nch = (int)(I[0] >> 8);
+                        const float i = sigm(a[0] + b[0]), o = sigm(a[1] + b[1]), uv = tanhf(a[2] + b[2]);
+                        const float fx = a[3] + b[3];
+                        float c = i * uv;
+#pragma unroll
+                        for (int kc = 0; kc < CHMAX; ++kc) {
+                            if (kc < nch) {
+                                const float f = sigm(fx + a[4 + kc]);
+                                c += f * __ldcg(pool + I[3 + kc] + H + jj);
+                                pool[rec + (5 + kc) * H + jj] = f;
+                            }
+                        }
+                        pool[rec + jj] = o * tanhf(c);
+                        pool[rec + H + jj] = c;
+                        pool[rec + 2 * H + jj] = i;
+                        pool[rec + 3 * H + jj] = o;
+                        pool[rec + 4 * H + jj] = uv;
+                    }
+                }
+            }
+        } else {
+            // ---- backward: cell backward per (unit slot, node) -> gate gradients in smem ----
+            if (tid < UMAX * NBMAX) {
+                const int uu = tid / NBMAX, n = tid % NBMAX, jj = lc + uu * P.n_g;
+                if (n < nb && jj < H) {
+                    const uint32_t* I = chunk + ipos[n];
+                    const uint32_t rec = I[1], adj = I[2];
+                    const float dh = __ldcg(pool + adj + jj), dc = __ldcg(pool + adj + H + jj);
+                    const float c = __ldcg(pool + rec + H + jj);
+                    const float th = tanhf(c);
+                    float* g = gb + (uu * NBMAX + n) * GO;
+                    float* db = dbias + uu * 4;
+                    if constexpr (BIN || CS) {
+                        const float i = __ldcg(pool + rec + 2 * H + jj), o = __ldcg(pool + rec + 3 * H + jj),
+                                    uv = __ldcg(pool + rec + 4 * H + jj);
+                        const float dov = dh * th;
+                        const float chat = dc + dh * o * (1.f - th * th);
+                        const float gi = chat * uv * i * (1.f - i), go = dov * o * (1.f - o),
+                                    gu = chat * i * (1.f - uv * uv);
+                        g[0] = gi; g[1] = go; g[2] = gu;
+                        atomicAdd(db + 0, gi); atomicAdd(db + 1, go); atomicAdd(db + 2, gu);
+                        if constexpr (BIN) {
+                            if (kindB) {
+                                const float fl = __ldcg(pool + rec + 5 * H + jj), fr = __ldcg(pool + rec + 6 * H + jj);
+                                const float cl = __ldcg(pool + I[3] + H + jj), cr = __ldcg(pool + I[5] + H + jj);
+                                const float gfl = chat * cl * fl * (1.f - fl), gfr = chat * cr * fr * (1.f - fr);
+                                pool[I[4] + H + jj] = chat * fl;     // dc of the left child (unique parent)
+                                pool[I[6] + H + jj] = chat * fr;
+                                g[3] = gfl; g[4] = gfr;
+                                atomicAdd(db + 3, gfl + gfr);
+                            }
+                        } else {
+                            const int nch = (int)(I[0] >> 8);
+                            float gfs = 0.f;
+#pragma unroll
+                            for (int kc = 0; kc < CHMAX; ++kc) {
+                                float gf = 0.f;
+                                if (kc < nch) {
+                                    const float f = __ldcg(pool + rec + (5 + kc) * H + jj);
+                                    const float ck = __ldcg(pool + I[4 + 2 * kc] + H + jj);
+                                    gf = chat * ck * f * (1.f - f);
+                                    pool[I[5 + 2 * kc] + H + jj] = chat * f;
+                                }
+                                g[4 + kc] = gf;
+                                gfs += gf;
+                            }
+                            g[3] = gfs;
+                            atomicAdd(db + 3, gfs);
+                        }
+                    } else {
+                        const float i = __ldcg(pool + rec + 2 * H + jj), f = __ldcg(pool + rec + 3 * H + jj),
+                                    o = __ldcg(pool + rec + 4 * H + jj), gg = __ldcg(pool + rec + 5 * H + jj);
+                        const uint32_t prv = I[4], padj = I[5];
+                        const float cp = prv != NONE ? __ldcg(pool + prv + H + jj) : 0.f;
+                        const float dov = dh * th;
+                        const float chat = dc + dh * o * (1.f - th * th);
+                        g[0] = chat * gg * i * (1.f - i);
+                        g[1] = chat * cp * f * (1.f - f);
+                        g[2] = dov * o * (1.f - o);
+                        g[3] = chat * i * (1.f - gg * gg);
+                        if (prv != NONE) pool[padj + H + jj] = chat * f;
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) atomicAdd(db + k, g[k]);
+                    }
+                }
+            }
+            __syncthreads();
+            // ---- in-register outer products (dW, L104) and transposed products (L94, fn4) ----
+            if (unit_ok) {
+                for (int n = 0; n < nb; ++n) {
+                    const uint32_t* I = chunk + ipos[n];
+                    const float* g = gb + (u * NBMAX + n) * GO;
+                    if (kindB) {
+                        if constexpr (BIN) {
+                            const float* x = xs + n * LB::KP;
+                            const float g0 = g[0], g1 = g[1], g2 = g[2], g3 = g[3], g4 = g[4];
+#pragma unroll
+                            for (int t = 0; t < LB::NT; ++t) {
+                                const int col0 = LB::CG * (tu + TU * t);
+                                float xv[LB::CG], dx[LB::CG];
+                                lds<LB::CG>(x + col0, xv);
+                                const float gf = col0 < H ? g3 : g4;
+#pragma unroll
+                                for (int q = 0; q < LB::CG; ++q) {
+                                    const int k = t * LB::CG + q;
+                                    dwb[0][k] = fmaf(g0, xv[q], dwb[0][k]);
+                                    dwb[1][k] = fmaf(g1, xv[q], dwb[1][k]);
+                                    dwb[2][k] = fmaf(g2, xv[q], dwb[2][k]);
+                                    dwb[3][k] = fmaf(gf, xv[q], dwb[3][k]);
+                                    dx[q] = wb[0][k] * g0 + wb[1][k] * g1 + wb[2][k] * g2 + wb[3][k] * gf;
+                                }
+                                if (col0 < 2 * H) {
+                                    float* dst = col0 < H ? pool + I[4] + col0 : pool + I[6] + (col0 - H);
+                                    red_add<LB::CG>(dst, dx);
+                                }
+                            }
+                        }
+                    } else {
+                        const float* x = xs + n * LA::KP;
+                        if constexpr (BIN) {
+                            const float g0 = g[0], g1 = g[1], g2 = g[2];
+                            const uint32_t tok = I[3];
+#pragma unroll
+                            for (int t = 0; t < LA::NT; ++t) {
+                                const int col0 = LA::CG * (tu + TU * t);
+                                float xv[LA::CG], dx[LA::CG];
+                                lds<LA::CG>(x + col0, xv);
+#pragma unroll
+                                for (int q = 0; q < LA::CG; ++q) {
+                                    const int k = t * LA::CG + q;
+                                    dwa[0][k] = fmaf(g0, xv[q], dwa[0][k]);
+                                    dwa[1][k] = fmaf(g1, xv[q], dwa[1][k]);
+                                    dwa[2][k] = fmaf(g2, xv[q], dwa[2][k]);
+                                    dx[q] = wa[0][k] * g0 + wa[1][k] * g1 + wa[2][k] * g2;
+                                }
+                                if (P.d_inputs && col0 < E) red_add<LA::CG>(P.d_inputs + (int64_t)tok * E + col0, dx);
+                            }
+                        } else if constexpr (LS) {
+                            const float g0 = g[0], g1 = g[1], g2 = g[2], g3 = g[3];
+                            const uint32_t tok = I[3], padj = I[5];
+#pragma unroll
+                            for (int t = 0; t < LA::NT; ++t) {
+                                const int col0 = LA::CG * (tu + TU * t);
+                                float xv[LA::CG], dx[LA::CG];
+                                lds<LA::CG>(x + col0, xv);
+#pragma unroll
+                                for (int q = 0; q < LA::CG; ++q) {
+                                    const int k = t * LA::CG + q;
+                                    dwa[0][k] = fmaf(g0, xv[q], dwa[0][k]);
+                                    dwa[1][k] = fmaf(g1, xv[q], dwa[1][k]);
+                                    dwa[2][k] = fmaf(g2, xv[q], dwa[2][k]);
+                                    dwa[3][k] = fmaf(g3, xv[q], dwa[3][k]);
+                                    dx[q] = wa[0][k] * g0 + wa[1][k] * g1 + wa[2][k] * g2 + wa[3][k] * g3;
+                                }
+                                if (col0 < E) {
+                                    if (P.d_inputs) red_add<LA::CG>(P.d_inputs + (int64_t)tok * E + col0, dx);
+                                } else if (col0 < E + H && padj != NONE) {
+                                    red_add<LA::CG>(pool + padj + (col0 - E), dx);
+                                }
+                            }
+                        } else {
+                            const float g0 = g[0], g1 = g[1], g2 = g[2], gfs = g[3];
+                            const uint32_t tok = I[3];
+                            const int nch = (int)(I[0] >> 8);
+#pragma unroll
+                            for (int t = 0; t < LA::NT; ++t) {
+                                const int col0 = LA::CG * (tu + TU * t);
+                                float xv[LA::CG], dio[LA::CG];
+                                lds<LA::CG>(x + col0, xv);
+#pragma unroll
+                                for (int q = 0; q < LA::CG; ++q) {
+                                    const int k = t * LA::CG + q;
+                                    dwa[0][k] = fmaf(g0, xv[q], dwa[0][k]);
+                                    dwa[1][k] = fmaf(g1, xv[q], dwa[1][k]);
+                                    dwa[2][k] = fmaf(g2, xv[q], dwa[2][k]);
+                                    dio[q] = wa[0][k] * g0 + wa[1][k] * g1 + wa[2][k] * g2;
+                                }
+                                if (col0 < E) {
+                                    float dx[LA::CG];
+#pragma unroll
+                                    for (int q = 0; q < LA::CG; ++q) {
+                                        const int k = t * LA::CG + q;
+                                        dwa[3][k] = fmaf(gfs, xv[q], dwa[3][k]);
+                                        dx[q] = dio[q] + wa[3][k] * gfs;
+                                    }
+                                    if (P.d_inputs && tok != NONE) red_add<LA::CG>(P.d_inputs + (int64_t)tok * E + col0, dx);
+                                } else if (col0 < E + H) {
+#pragma unroll
+                                    for (int kc = 0; kc < CHMAX; ++kc) {
+                                        if (kc < nch) {
+                                            const float gf = g[4 + kc];
+                                            float yv[LA::CG], dh[LA::CG];
+                                            lds<LA::CG>(chs + (cslot[n] + kc) * LA::KP + col0, yv);
+#pragma unroll
+                                            for (int q = 0; q < LA::CG; ++q) {
+                                                const int k = t * LA::CG + q;
+                                                dwa[3][k] = fmaf(gf, yv[q], dwa[3][k]);
+                                                dh[q] = dio[q] + wa[3][k] * gf;
+                                            }
+                                            red_add<LA::CG>(pool + I[5 + 2 * kc] + (col0 - E), dh);
+                                        }
+                                    }
+                                }
+                            }
+                        }
+                    }
+                }
+            }
+        }
+        pos = p;
+    }
+
+    // ---------------- epilogue: apply gradients to the master copy, or write them (L129, L197) -----
+    __syncthreads();
+    const bool sgd = P.mode == 1;
+    float* gout = P.grads;
+    auto put = [&](int64_t idx, float w, float dw) {
+        if (sgd) P.params[idx] = w - P.lr * (dw + P.wd * w);
+        else gout[idx] = dw;
+    };
+    if (unit_ok) {
+#pragma unroll
+        for (int r = 0; r < RA; ++r)
+#pragma unroll
+            for (int t = 0; t < LA::NT; ++t)
+#pragma unroll
+                for (int q = 0; q < LA::CG; ++q) {
+                    const int col = LA::CG * (tu + TU * t) + q;
+                    if (col < KA) put(idxA(r, col), wa[r][t * LA::CG + q], dwa[r][t * LA::CG + q]);
+                }
+        if constexpr (BIN) {
+#pragma unroll
+            for (int r = 0; r < RB; ++r)
+#pragma unroll
+                for (int t = 0; t < LB::NT; ++t)
+#pragma unroll
+                    for (int q = 0; q < LB::CG; ++q) {
+                        const int col = LB::CG * (tu + TU * t) + q;
+                        if (col < KB) put(idxB(r, col), wb[r][t * LB::CG + q], dwb[r][t * LB::CG + q]);
+                    }
+        }
+    }
+    if (tid < UMAX * 4) {
+        const int uu = tid / 4, k = tid % 4, jj = lc + uu * P.n_g;
+        if (jj < H) put((LS || k < 3) ? off[bias_m0] + k * H + jj : off[6] + jj, bias[tid], dbias[tid]);
+    }
+    if (holds_head) {
+        for (int i = tid; i < C * H; i += NTH) put(off[wout_m] + i, Wo[i], dWo[i]);
+        for (int i = tid; i < C; i += NTH) put(off[bout_m] + i, bo[i], dbo[i]);
+    }
+}
+
+__global__ void sgd_kernel(float* __restrict__ p, const float* __restrict__ g, int64_t n, float lr, float wd) {
+    const int64_t n4 = n / 4;
+    float4* p4 = reinterpret_cast<float4*>(p);
+    const float4* g4 = reinterpret_cast<const float4*>(g);
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x) {
+        float4 a = p4[i];
+        const float4 b = g4[i];
+        a.x -= lr * (b.x + wd * a.x); a.y -= lr * (b.y + wd * a.y);
+        a.z -= lr * (b.z + wd * a.z); a.w -= lr * (b.w + wd * a.w);
+        p4[i] = a;
+    }
+    for (int64_t i = n4 * 4 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        p[i] -= lr * (g[i] + wd * p[i]);
+}
+
+}  // namespace dev
+
+#define VPPS_VARIANT(CELL, H, E, U) \
+    {CELL, H, E, U, (const void*)&dev::vpps_fb<CELL, H, E, U>, &dev::Cfg<CELL, H, E, U>::smem_bytes}
+
+static const Variant kVariants[] = {
+    VPPS_VARIANT(dev::CELL_BINARY, 256, 256, 2),    // target: binary Tree-LSTM H = E = 256 on 148 SMs
+    VPPS_VARIANT(dev::CELL_BINARY, 128, 128, 1),
+    VPPS_VARIANT(dev::CELL_BINARY, 32, 32, 1),
+    VPPS_VARIANT(dev::CELL_CHILDSUM, 128, 128, 1),  // config 2
+    VPPS_VARIANT(dev::CELL_CHILDSUM, 32, 32, 1),
+    VPPS_VARIANT(dev::CELL_LSTM, 32, 32, 1),        // config 1
+    VPPS_VARIANT(dev::CELL_LSTM, 256, 256, 2),
+};
+
+const Variant* variants(int32_t* n) {
+    *n = (int32_t)(sizeof(kVariants) / sizeof(kVariants[0]));
+    return kVariants;
+}
+
+void launch_sgd(float* p, const float* g, int64_t n, float lr, float wd, cudaStream_t s) {
+    dev::sgd_kernel<<<148 * 4, 256, 0, s>>>(p, g, n, lr, wd);
+}
+
+}  // namespace vpps

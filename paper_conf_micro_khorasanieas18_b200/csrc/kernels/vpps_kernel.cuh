@@ -1,0 +1,32 @@
+// Kernel-side declarations shared by the launcher (api.cu) and the kernel translation unit.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace vpps {
+
+struct KParams {
+    float* params;          // DRAM master copy (flat, vpps_layout offsets)
+    float* grads;           // gradient output (mode 0)
+    const float* inputs;    // caller's input table [rows x E]
+    float* d_inputs;        // gradient of the input table, or nullptr
+    float* pool;            // activation pool (SPEC §S7)
+    const uint32_t* script; // encoded script (SPEC §E)
+    int64_t off[8];         // parameter offsets in floats
+    int32_t n_g, n_act, C, mode;   // mode 0: write grads; 1: fused SGD update
+    int64_t loss_word;
+    float lr, wd;
+};
+
+struct Variant {
+    int32_t cell, H, E, umax;
+    const void* fn;
+    size_t (*smem_bytes)(int32_t C);
+};
+
+// Table of compiled specialisations (vpps_kernel.cu).
+const Variant* variants(int32_t* n);
+// Elementwise SGD on the flat buffer (K3): p -= lr * (g + wd * p).
+void launch_sgd(float* p, const float* g, int64_t n, float lr, float wd, cudaStream_t s);
+
+}  // namespace vpps

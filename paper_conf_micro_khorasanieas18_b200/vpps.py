@@ -1,0 +1,274 @@
+"""Thin ctypes binding of libvpps.so (include/vpps.h) — argument marshalling only.
+
+Every step of the hot path runs in the CUDA library; this module converts Python graphs to the
+CSR `vpps_batch`, passes torch device pointers and the current CUDA stream, and turns status codes
+into exceptions.  There is no CPU fallback: if libvpps.so is missing, importing raises.
+"""
+from __future__ import annotations
+
+import ctypes as ct
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libvpps.so")
+
+CELLS = {"lstm": 0, "binary": 1, "childsum": 2}
+STATUS = {0: "OK", -1: "INVALID", -2: "NOFIT", -3: "CUDA", -4: "GRAPH", -5: "STATE", -6: "NOMEM"}
+
+
+class VppsError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"VPPS_E_{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class _Shape(ct.Structure):
+    _fields_ = [("rows", ct.c_int32), ("cols", ct.c_int32)]
+
+
+class _Opset(ct.Structure):
+    _fields_ = [("cell", ct.c_int32), ("E", ct.c_int32), ("H", ct.c_int32), ("C", ct.c_int32)]
+
+
+class _Options(ct.Structure):
+    _fields_ = [("n_sm", ct.c_int32), ("ctas_per_sm", ct.c_int32), ("groups", ct.c_int32),
+                ("device", ct.c_int32), ("plan_only", ct.c_int32)]
+
+
+class _Batch(ct.Structure):
+    _fields_ = [("n_graphs", ct.c_int32), ("graph_ptr", ct.c_void_p), ("child_ptr", ct.c_void_p),
+                ("children", ct.c_void_p), ("token", ct.c_void_p), ("label", ct.c_void_p)]
+
+
+class _Info(ct.Structure):
+    _fields_ = [("n_words", ct.c_int64), ("pool_words", ct.c_int64), ("zero_words", ct.c_int64),
+                ("loss_word", ct.c_int64), ("n_barriers", ct.c_int32), ("n_levels", ct.c_int32),
+                ("n_nodes", ct.c_int64), ("n_heads", ct.c_int64), ("flops", ct.c_double),
+                ("act_bytes", ct.c_double)]
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: run `python -c 'import __graft_entry__ as g; g.build()'` "
+                          "(the VPPS path has no CPU fallback)")
+    lib = ct.CDLL(LIB_PATH)
+    P, I32, I64, F, VP = ct.POINTER, ct.c_int32, ct.c_int64, ct.c_float, ct.c_void_p
+    sig = {
+        "vpps_define_model": [P(_Shape), I32, P(_Opset), P(_Options), P(VP)],
+        "vpps_layout": [VP, P(I64), P(I64)],
+        "vpps_bind_buffers": [VP, VP, VP],
+        "vpps_partition_table": [VP, P(P(I32)), P(I64)],
+        "vpps_plan_info": [VP, P(I32), P(I32), P(I32), P(I32)],
+        "vpps_paper_deal": [P(_Shape), I32, I32, I32, I32, I32, I32, VP, P(I64), P(I64)],
+        "vpps_paper_choose_cps": [P(_Shape), I32, I32, I32, I32, I32],
+        "vpps_build_script": [VP, P(_Batch), P(VP)],
+        "vpps_script_words": [VP, P(P(ct.c_uint32)), P(I64)],
+        "vpps_script_info_get": [VP, P(_Info)],
+        "vpps_upload_script": [VP, VP],
+        "vpps_fwd_bwd": [VP, VP, VP, I64, VP, VP],
+        "vpps_fwd_bwd_sgd": [VP, VP, VP, I64, VP, F, F, VP],
+        "vpps_sgd_step": [VP, F, F, VP],
+        "vpps_get_stale_loss": [VP, P(F)],
+        "vpps_sync_get_latest_loss": [VP, P(F)],
+        "vpps_pool_ptr": [VP, P(VP), P(I64)],
+        "vpps_destroy_script": [VP],
+        "vpps_destroy_model": [VP],
+        "vpps_last_error": [],
+        "vpps_variants": [VP, I32],
+    }
+    for name, args in sig.items():
+        fn = getattr(lib, name)
+        fn.argtypes = args
+        fn.restype = ct.c_int32
+    lib.vpps_last_error.restype = ct.c_char_p
+    lib.vpps_destroy_script.restype = None
+    lib.vpps_destroy_model.restype = None
+    return lib
+
+
+_lib = _load()
+
+
+def _check(st: int):
+    if st != 0:
+        raise VppsError(st, _lib.vpps_last_error().decode())
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        import torch
+        return ct.c_void_p(torch.cuda.current_stream().cuda_stream)
+    if isinstance(stream, int):
+        return ct.c_void_p(stream)
+    return ct.c_void_p(stream.cuda_stream)
+
+
+def param_shapes(cell: str, H: int, E: int, C: int):
+    """Parameter order of vpps_define_model (include/vpps.h); bias shapes are (n,)."""
+    if cell == "lstm":
+        return [("W", (4 * H, E)), ("U", (4 * H, H)), ("W_out", (C, H)), ("b", (4 * H,)), ("b_out", (C,))]
+    if cell == "binary":
+        return [("W_iou", (3 * H, E)), ("U_iou", (3 * H, 2 * H)), ("U_fl", (H, H)), ("U_fr", (H, H)),
+                ("W_out", (C, H)), ("b_iou", (3 * H,)), ("b_f", (H,)), ("b_out", (C,))]
+    if cell == "childsum":
+        return [("W_iou", (3 * H, E)), ("W_f", (H, E)), ("U_iou", (3 * H, H)), ("U_f", (H, H)),
+                ("W_out", (C, H)), ("b_iou", (3 * H,)), ("b_f", (H,)), ("b_out", (C,))]
+    raise ValueError(cell)
+
+
+def variants():
+    buf = (ct.c_int32 * 256)()
+    n = _lib.vpps_variants(ct.cast(buf, ct.c_void_p), 64)
+    inv = {v: k for k, v in CELLS.items()}
+    return [(inv[buf[4 * i]], buf[4 * i + 1], buf[4 * i + 2], buf[4 * i + 3]) for i in range(n)]
+
+
+def paper_deal(mats, n_cta, tb, rpw, pack_rows=True, grads=False):
+    """SPEC P0 dealer -> (rows int32 [n, 6] = matrix,row,cta,partition,warp,is_grad ; n_slots)."""
+    sh = (_Shape * len(mats))(*[_Shape(r, c) for r, c in mats])
+    n, slots = ct.c_int64(), ct.c_int64()
+    _check(_lib.vpps_paper_deal(sh, len(mats), n_cta, tb, rpw, int(pack_rows), int(grads), None,
+                                ct.byref(n), ct.byref(slots)))
+    out = np.zeros((n.value, 6), dtype=np.int32)
+    _check(_lib.vpps_paper_deal(sh, len(mats), n_cta, tb, rpw, int(pack_rows), int(grads),
+                                out.ctypes.data_as(ct.c_void_p), ct.byref(n), ct.byref(slots)))
+    return out, slots.value
+
+
+def paper_choose_cps(mats, n_sm, tb=256, rpw=1, pack_rows=True):
+    sh = (_Shape * len(mats))(*[_Shape(r, c) for r, c in mats])
+    return int(_lib.vpps_paper_choose_cps(sh, len(mats), n_sm, tb, rpw, int(pack_rows)))
+
+
+def to_csr(graphs):
+    """Graphs as lists of (children, token, label) -> CSR int32 arrays of vpps_batch."""
+    gp, cp, ch, tok, lab = [0], [0], [], [], []
+    for g in graphs:
+        for (c, t, l) in g:
+            ch.extend(c)
+            cp.append(len(ch))
+            tok.append(t)
+            lab.append(l)
+        gp.append(len(tok))
+    as32 = lambda a: np.ascontiguousarray(np.asarray(a, dtype=np.int32))
+    return as32(gp), as32(cp), as32(ch if ch else [0]), as32(tok), as32(lab)
+
+
+class Script:
+    def __init__(self, model: "Model", handle: ct.c_void_p):
+        self._model = model
+        self._h = handle
+
+    @property
+    def handle(self):
+        return self._h
+
+    def words(self) -> np.ndarray:
+        p = ct.POINTER(ct.c_uint32)()
+        n = ct.c_int64()
+        _check(_lib.vpps_script_words(self._h, ct.byref(p), ct.byref(n)))
+        return np.ctypeslib.as_array(p, shape=(n.value,)).copy() if n.value else np.zeros(0, np.uint32)
+
+    def info(self) -> dict:
+        i = _Info()
+        _check(_lib.vpps_script_info_get(self._h, ct.byref(i)))
+        return {f: getattr(i, f) for f, _ in _Info._fields_}
+
+    def upload(self, stream=None):
+        _check(_lib.vpps_upload_script(self._h, _stream_ptr(stream)))
+
+    def __del__(self):
+        if getattr(self, "_h", None):
+            _lib.vpps_destroy_script(self._h)
+            self._h = None
+
+
+class Model:
+    """vpps_define_model + vpps_bind_buffers (`vpps::handle hndl(model)`)."""
+
+    def __init__(self, cell: str, H: int, E: int, C: int, device: int = 0, n_sm: int = 0, groups: int = 1,
+                 plan_only: bool = False):
+        self.cell, self.H, self.E, self.C = cell, H, E, C
+        self.shapes = param_shapes(cell, H, E, C)
+        sh = (_Shape * len(self.shapes))(*[_Shape(s[0], s[1] if len(s) == 2 else 1) for _, s in self.shapes])
+        ops = _Opset(CELLS[cell], E, H, C)
+        opt = _Options(n_sm, 1, groups, device, int(plan_only))
+        h = ct.c_void_p()
+        _check(_lib.vpps_define_model(sh, len(self.shapes), ct.byref(ops), ct.byref(opt), ct.byref(h)))
+        self._h = h
+        n = ct.c_int64()
+        offs = (ct.c_int64 * len(self.shapes))()
+        _check(_lib.vpps_layout(self._h, ct.byref(n), offs))
+        self.n_floats = n.value
+        self.offsets = list(offs)
+        self._bound = None
+
+    # ---- layout helpers (views into a flat buffer) ----
+    def views(self, flat):
+        out = {}
+        for (name, shape), o in zip(self.shapes, self.offsets):
+            size = int(np.prod(shape))
+            out[name] = flat[o:o + size].view(*shape) if hasattr(flat, "view") and not isinstance(flat, np.ndarray) \
+                else flat[o:o + size].reshape(shape)
+        return out
+
+    def bind(self, params, grads):
+        """params/grads: contiguous float32 CUDA tensors of n_floats (caller-owned)."""
+        assert params.is_cuda and grads.is_cuda and params.dtype == grads.dtype
+        assert params.numel() == self.n_floats and grads.numel() == self.n_floats
+        _check(_lib.vpps_bind_buffers(self._h, ct.c_void_p(params.data_ptr()), ct.c_void_p(grads.data_ptr())))
+        self._bound = (params, grads)
+
+    def partition_table(self) -> np.ndarray:
+        p = ct.POINTER(ct.c_int32)()
+        n = ct.c_int64()
+        _check(_lib.vpps_partition_table(self._h, ct.byref(p), ct.byref(n)))
+        return np.ctypeslib.as_array(p, shape=(n.value * 8,)).reshape(n.value, 8).copy()
+
+    def plan_info(self) -> dict:
+        a, b, c, d = ct.c_int32(), ct.c_int32(), ct.c_int32(), ct.c_int32()
+        _check(_lib.vpps_plan_info(self._h, ct.byref(a), ct.byref(b), ct.byref(c), ct.byref(d)))
+        return dict(n_cta=a.value, n_g=b.value, n_act=c.value, umax=d.value)
+
+    def build_script(self, graphs) -> Script:
+        gp, cp, ch, tok, lab = to_csr(graphs)
+        b = _Batch(len(graphs), gp.ctypes.data, cp.ctypes.data, ch.ctypes.data, tok.ctypes.data, lab.ctypes.data)
+        h = ct.c_void_p()
+        _check(_lib.vpps_build_script(self._h, ct.byref(b), ct.byref(h)))
+        return Script(self, h)
+
+    def fwd_bwd(self, script: Script, inputs, d_inputs=None, stream=None):
+        _check(_lib.vpps_fwd_bwd(self._h, script.handle, ct.c_void_p(inputs.data_ptr()), inputs.shape[0],
+                                 ct.c_void_p(d_inputs.data_ptr()) if d_inputs is not None else None,
+                                 _stream_ptr(stream)))
+
+    def fwd_bwd_sgd(self, script: Script, inputs, d_inputs=None, lr=0.0, weight_decay=0.0, stream=None):
+        _check(_lib.vpps_fwd_bwd_sgd(self._h, script.handle, ct.c_void_p(inputs.data_ptr()), inputs.shape[0],
+                                     ct.c_void_p(d_inputs.data_ptr()) if d_inputs is not None else None,
+                                     lr, weight_decay, _stream_ptr(stream)))
+
+    def sgd_step(self, lr: float, weight_decay: float = 0.0, stream=None):
+        _check(_lib.vpps_sgd_step(self._h, lr, weight_decay, _stream_ptr(stream)))
+
+    def stale_loss(self) -> float:
+        v = ct.c_float()
+        _check(_lib.vpps_get_stale_loss(self._h, ct.byref(v)))
+        return v.value
+
+    def latest_loss(self) -> float:
+        v = ct.c_float()
+        _check(_lib.vpps_sync_get_latest_loss(self._h, ct.byref(v)))
+        return v.value
+
+    def pool(self):
+        """(device pointer, words) of the activation pool of the last pass."""
+        p, n = ct.c_void_p(), ct.c_int64()
+        _check(_lib.vpps_pool_ptr(self._h, ct.byref(p), ct.byref(n)))
+        return p.value, n.value
+
+    def __del__(self):
+        if getattr(self, "_h", None):
+            _lib.vpps_destroy_model(self._h)
+            self._h = None

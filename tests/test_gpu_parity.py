@@ -1,0 +1,170 @@
+"""GPU parity: the CUDA path (through the C ABI) against the FP64 oracle on the same seeded inputs.
+
+Tolerance (BASELINE.json north_star; reading R-22): per tensor ‖g − o‖∞ / ‖o‖∞ ≤ 1e-4,
+loss |L − L_o| / |L_o| ≤ 1e-4.  FP32 accumulation order differs (atomics), so bitwise equality is
+not expected for floats; the integer artefacts are checked bit-exactly in test_host_parity.py.
+"""
+import numpy as np
+import pytest
+
+import synth
+from oracle import models as M
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+TOL = 1e-4
+
+
+def _vpps():
+    from paper_conf_micro_khorasanieas18_b200 import vpps
+    return vpps
+
+
+def run_case(cell, H, E, C, graphs, V, seed=0, want_dx=True, sgd=None):
+    vpps = _vpps()
+    rng = np.random.default_rng(seed)
+    shapes = vpps.param_shapes(cell, H, E, C)
+    P = synth.init_params(shapes, rng)
+    X = synth.input_table(rng, V, E)
+    m = vpps.Model(cell, H, E, C, device=0)
+    dev = torch.device("cuda:0")
+    params = torch.zeros(m.n_floats, dtype=torch.float32, device=dev)
+    grads = torch.full_like(params, float("nan"))
+    views = m.views(params)
+    for name, _ in shapes:
+        views[name].copy_(torch.from_numpy(P[name]).float())
+    m.bind(params, grads)
+    inputs = torch.from_numpy(X).float().to(dev)
+    dX = torch.full_like(inputs, float("nan")) if want_dx else None
+    s = m.build_script(graphs)
+    if sgd is None:
+        m.fwd_bwd(s, inputs, dX)
+    else:
+        m.fwd_bwd_sgd(s, inputs, dX, lr=sgd[0], weight_decay=sgd[1])
+    loss = m.latest_loss()
+    torch.cuda.synchronize()
+    return m, P, X, loss, params, grads, dX
+
+
+def rel(a, b):
+    return float(np.abs(np.asarray(a, np.float64) - b).max() / max(np.abs(b).max(), 1e-30))
+
+
+def check(cell, H, E, C, graphs, V, seed=0, want_dx=True):
+    m, P, X, loss, params, grads, dX = run_case(cell, H, E, C, graphs, V, seed, want_dx)
+    lo, Go, dXo = M.forward_backward(cell, P, X, graphs, H)
+    assert abs(loss - lo) <= TOL * abs(lo), (loss, lo)
+    gv = m.views(grads.cpu())
+    for name, _ in m.shapes:
+        assert rel(gv[name].numpy(), Go[name]) <= TOL, name
+    if want_dx:
+        assert rel(dX.cpu().numpy(), dXo) <= TOL, "dX"
+    return loss, lo
+
+
+def _trees(seed, batch, leaves, V, C):
+    return synth.tree_batch(np.random.default_rng(seed), batch, leaves, V, C)
+
+
+@pytest.mark.parametrize("H", [32, 128])
+def test_binary_small(H):
+    check("binary", H, H, 5, _trees(1, 5, (1, 12), 40, 5), 40)
+
+
+def test_binary_target_config():
+    """TGT: binary Tree-LSTM H = E = 256, batch 16 SST-shaped trees (5-50 leaves), 148 SMs."""
+    graphs = synth.config_batch("tgt", 0)
+    check("binary", 256, 256, 5, graphs, 4096, seed=3)
+
+
+def test_binary_target_other_batches():
+    for b in (1, 7):
+        check("binary", 256, 256, 5, synth.config_batch("tgt", b), 4096, seed=b)
+
+
+def test_binary_degenerate_single_leaf_and_no_dx():
+    graphs = [[((), 3, 2)], [((), 1, 0)]]               # lone labelled leaves: one cell level + heads
+    check("binary", 32, 32, 5, graphs, 8)
+    check("binary", 32, 32, 5, _trees(4, 3, (2, 6), 8, 5), 8, want_dx=False)
+
+
+def test_binary_labels_on_inner_nodes():
+    t = [((), 0, 1), ((), 1, -1), ((0, 1), -1, 3), ((), 2, -1), ((2, 3), -1, 0)]
+    check("binary", 32, 32, 5, [t, t], 4)
+
+
+def test_childsum_config2():
+    graphs = synth.config_batch("c2", 0)
+    check("childsum", 128, 128, 5, graphs, 4096, seed=2)
+
+
+def test_childsum_arity_and_missing_tokens():
+    g = [((), -1, -1), ((0,), 3, 2), ((), 4, -1), ((), 5, -1), ((1, 2, 3), -1, 1), ((), 1, -1),
+         ((4, 5), 2, 4)]
+    check("childsum", 32, 32, 5, [g] + _trees(5, 2, (1, 7), 8, 5), 8)
+
+
+def test_lstm_config1():
+    graphs = synth.config_batch("c1", 0)
+    check("lstm", 32, 32, 16, graphs, 16, seed=1)
+
+
+def test_lstm_h256_small_vocab():
+    rng = np.random.default_rng(9)
+    graphs = [synth.chain(rng, int(rng.integers(5, 30)), 16) for _ in range(4)]
+    check("lstm", 256, 256, 16, graphs, 16, seed=9)
+
+
+def test_fused_sgd_update():
+    graphs = _trees(6, 4, (1, 9), 20, 5)
+    lr, wd = 0.05, 1e-3
+    m, P, X, loss, params, grads, dX = run_case("binary", 32, 32, 5, graphs, 20, seed=6, sgd=(lr, wd))
+    lo, Go, _ = M.forward_backward("binary", P, X, graphs, 32)
+    Pn = M.sgd(P, Go, lr, wd)
+    pv = m.views(params.cpu())
+    for name, _ in m.shapes:
+        # compare the update itself: (new - old) vs the oracle's step
+        assert rel(pv[name].numpy() - P[name], Pn[name] - P[name]) <= 1e-3, name
+
+
+def test_dp_split_equals_union():
+    """Data parallelism invariant on one GPU: Σ gradients of the shards == gradient of the union."""
+    graphs = synth.config_batch("tgt", 2)
+    g_all = run_case("binary", 256, 256, 5, graphs, 4096, seed=4)[5].cpu().numpy()
+    g_a = run_case("binary", 256, 256, 5, graphs[:7], 4096, seed=4)[5].cpu().numpy()
+    g_b = run_case("binary", 256, 256, 5, graphs[7:], 4096, seed=4)[5].cpu().numpy()
+    assert rel(g_a + g_b, g_all) <= TOL
+
+
+def test_stale_and_latest_loss():
+    vpps = _vpps()
+    rng = np.random.default_rng(7)
+    H, C, V = 32, 5, 16
+    shapes = vpps.param_shapes("binary", H, H, C)
+    P = synth.init_params(shapes, rng)
+    m = vpps.Model("binary", H, H, C)
+    params = torch.zeros(m.n_floats, device="cuda")
+    grads = torch.zeros_like(params)
+    for name, _ in shapes:
+        m.views(params)[name].copy_(torch.from_numpy(P[name]).float())
+    m.bind(params, grads)
+    X = torch.from_numpy(synth.input_table(rng, V, H)).float().cuda()
+    batches = [_trees(10 + i, 3, (1, 6), V, C) for i in range(3)]
+    losses = []
+    for b in batches:
+        m.fwd_bwd(m.build_script(b), X)
+        losses.append(M.forward_backward("binary", P, X.cpu().double().numpy(), b, H)[0])
+    stale = m.stale_loss()          # loss of batch 1 (the pass before the most recent)
+    latest = m.latest_loss()        # loss of batch 2
+    assert abs(stale - losses[1]) <= TOL * abs(losses[1])
+    assert abs(latest - losses[2]) <= TOL * abs(losses[2])
+
+
+def test_errors_are_loud():
+    vpps = _vpps()
+    with pytest.raises(vpps.VppsError):
+        vpps.Model("binary", 4096, 4096, 5)               # NOFIT
+    m = vpps.Model("binary", 32, 32, 5)
+    s = m.build_script(_trees(1, 2, (1, 5), 8, 5))
+    with pytest.raises(vpps.VppsError):                   # buffers not bound
+        m.fwd_bwd(s, torch.zeros(8, 32, device="cuda"))

@@ -1,0 +1,138 @@
+"""Bit-exact parity of the C++ host library (libvpps.so, plan-only mode: no GPU needed) with the
+independent Python implementation in oracle/ of SPEC_SCRIPT.md (partition table, script words,
+pool plan), plus the C-ABI export check against include/vpps.h."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import models as M
+from oracle import plan as oplan
+from oracle import script as oscript
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def vpps():
+    from paper_conf_micro_khorasanieas18_b200 import vpps as v
+    return v
+
+
+def test_abi_exports_every_declared_symbol():
+    hdr = open(os.path.join(ROOT, "include", "vpps.h")).read()
+    names = set(re.findall(r"\b(vpps_[a-z_]+)\s*\(", hdr))
+    assert len(names) >= 20
+    lib = ctypes.CDLL(os.path.join(ROOT, "paper_conf_micro_khorasanieas18_b200", "libvpps.so"))
+    for n in sorted(names):
+        assert hasattr(lib, n), n
+
+
+def test_param_shapes_agree_with_oracle(vpps):
+    for cell in ("lstm", "binary", "childsum"):
+        a = [(n, tuple(s)) for n, s in vpps.param_shapes(cell, 8, 4, 3)]
+        b = [(n, tuple(s)) for n, s in M.param_shapes(cell, 8, 4, 3)]
+        assert a == b
+
+
+@pytest.mark.parametrize("rows_a", [9, 16, 40])
+@pytest.mark.parametrize("pack", [0, 1])
+def test_paper_deal_bit_exact(vpps, rows_a, pack):
+    mats = [(rows_a, 128), (24, 96), (5, 256)]
+    for grads in (0, 1):
+        c_rows, c_slots = vpps.paper_deal(mats, 4, 128, 2, pack, grads)
+        o_rows, o_slots = oplan.paper_deal(mats, 4, 128, 2, bool(pack), bool(grads))
+        assert c_slots == o_slots
+        assert np.array_equal(c_rows, np.array(o_rows, dtype=np.int32))
+
+
+def test_paper_choose_cps_bit_exact(vpps):
+    for H in (128, 256, 384, 512):
+        mats = [s for (_, s) in M.param_shapes("binary", H, 128, 5) if len(s) == 2]
+        for n_sm in (80, 148):
+            assert vpps.paper_choose_cps(mats, n_sm) == oplan.choose_cps(mats, n_sm)
+    mats = [s for (_, s) in M.param_shapes("binary", 256, 128, 5) if len(s) == 2]
+    assert vpps.paper_choose_cps(mats, 80) == 2      # L241 via the C++ path too
+
+
+@pytest.mark.parametrize("cell,H,E,C", [("binary", 256, 256, 5), ("binary", 1024, 1024, 5),
+                                        ("lstm", 32, 32, 16), ("childsum", 128, 128, 5), ("lstm", 256, 256, 1000)])
+@pytest.mark.parametrize("G", [1, 2, 4])
+def test_partition_table_bit_exact(vpps, cell, H, E, C, G):
+    try:
+        ref = oplan.unit_plan(cell, H, E, C, n_sm=148, G=G)
+    except ValueError:
+        with pytest.raises(vpps.VppsError) as e:
+            vpps.Model(cell, H, E, C, n_sm=148, groups=G, plan_only=True)
+        assert e.value.status == -2
+        return
+    m = vpps.Model(cell, H, E, C, n_sm=148, groups=G, plan_only=True)
+    info = m.plan_info()
+    assert (info["n_g"], info["n_act"], info["umax"]) == (ref["n_g"], ref["n_act"], ref["umax"])
+    assert np.array_equal(m.partition_table(), np.array(ref["table"], dtype=np.int32))
+
+
+def _batches(cell, rng, n):
+    out = []
+    for _ in range(n):
+        b = int(rng.integers(1, 9))
+        if cell == "lstm":
+            out.append([synth.chain(rng, int(rng.integers(1, 12)), 7) for _ in range(b)])
+        elif cell == "binary":
+            out.append(synth.tree_batch(rng, b, (1, 20), 50, 5))
+        else:
+            gs = synth.tree_batch(rng, b, (1, 15), 50, 5)
+            # child-sum: vary arity and token presence
+            gs.append([((), -1, -1), ((0,), 3, 2), ((), 4, -1), ((), 5, -1), ((1, 2, 3), -1, 1)])
+            out.append(gs)
+    return out
+
+
+@pytest.mark.parametrize("cell", ["binary", "lstm", "childsum"])
+@pytest.mark.parametrize("G", [1, 2, 4])
+def test_script_words_bit_exact(vpps, cell, G):
+    H, E, C = 8, 8, 7
+    m = vpps.Model(cell, H, E, C, n_sm=16, groups=G, plan_only=True)
+    rng = np.random.default_rng(100 + G)
+    n_act = m.plan_info()["n_act"]
+    for graphs in _batches(cell, rng, 12):
+        s = m.build_script(graphs)
+        ref = oscript.build(cell, graphs, H, E, C, G=G, n_act=n_act)
+        w = s.words()
+        assert np.array_equal(w, np.array(ref["words"], dtype=np.uint32))
+        info = s.info()
+        assert (info["pool_words"], info["zero_words"], info["loss_word"], info["n_barriers"]) == \
+            (ref["pool_words"], ref["zero_words"], ref["loss_word"], ref["n_bar"])
+        assert info["flops"] == M.flop_count(cell, graphs, H, E, C)
+
+
+def test_script_words_target_config(vpps):
+    """TGT shapes (binary H = E = 256, batch 16 SST-shaped trees) on 148 SMs."""
+    m = vpps.Model("binary", 256, 256, 5, n_sm=148, plan_only=True)
+    for b in range(3):
+        graphs = synth.config_batch("tgt", b)
+        s = m.build_script(graphs)
+        ref = oscript.build("binary", graphs, 256, 256, 5, G=1, n_act=148)
+        assert np.array_equal(s.words(), np.array(ref["words"], dtype=np.uint32))
+
+
+def test_graph_errors(vpps):
+    m = vpps.Model("binary", 8, 8, 3, n_sm=16, plan_only=True)
+    with pytest.raises(vpps.VppsError) as e:
+        m.build_script([[((), 0, -1), ((0,), -1, 1)]])          # unary internal node (R-26)
+    assert e.value.status == -4
+    with pytest.raises(vpps.VppsError):
+        m.build_script([[((), 0, -1), ((), 1, -1), ((0, 0), -1, 1)]])   # two parents edges to one child
+    with pytest.raises(vpps.VppsError):
+        m.build_script([[((), 0, 5)]])                            # label out of range
+    with pytest.raises(vpps.VppsError):
+        vpps.Model("binary", 8, 8, 3, n_sm=16, plan_only=True).build_script([[((1,), 0, -1), ((), 0, -1)]])
+
+
+def test_nofit_and_bad_shapes(vpps):
+    with pytest.raises(vpps.VppsError) as e:
+        vpps.Model("binary", 4096, 4096, 5, n_sm=148, plan_only=True)
+    assert e.value.status == -2
