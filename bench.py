@@ -1,0 +1,319 @@
+#!/usr/bin/env python
+"""VPPS benchmark: binary Tree-LSTM (H = E = 256) training samples/s on N B200s (BASELINE.json).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl vpps|reference] [--batch B]
+
+One step = one pass of the whole hot path on one batch of B synthetic SST-shaped trees per GPU:
+  N = 1: vpps_fwd_bwd_sgd — forward, backward and SGD update in one persistent kernel
+  N > 1: vpps_fwd_bwd -> NCCL all-reduce of the flat gradient -> vpps_sgd_step (weak scaling)
+64 distinct pre-built batches per rank are cycled (every step sees a new graph shape, L44); the L2 is
+flushed (256 MiB write) before every timed step, outside the timed region.  Rank 0 prints one JSON line.
+`--impl reference` times the FP64 CPU oracle (oracle/) on the same workload (bounded sample per step).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+METRIC = "Tree-LSTM training samples/sec at 1/2/4/8 B200; DRAM bytes/pass vs weights-once"
+H = E = 256
+C = 5
+V = 4096
+N_BATCHES = 64
+WORKLOAD = ("tgt: binary Tree-LSTM (M4) H=E=256, C=5, SST-shaped synthetic trees with 5-50 leaves, "
+            "input table 4096x256, fwd+bwd+dX+SGD")
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+def fp32_peak_tflops(mhz: float) -> float:
+    """FP32 FFMA peak: 148 SMs x 128 FP32 lanes x 2 FLOP x SM clock."""
+    return 148 * 128 * 2 * mhz * 1e6 / 1e12
+
+
+class ClockSampler:
+    """nvidia-smi clocks and throttle reasons sampled during the timed region (B200_PROFILING.md)."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) >= 9:
+                self.rows.append(parts)
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in self.rows for k in range(4) if r[5 + k].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": float(self.rows[0][2]) if self.rows[0][2].replace(".", "").isdigit() else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def make_batches(rank: int, batch: int):
+    # rank r's batches are config 'tgt' batches r*N_BATCHES .. r*N_BATCHES+63 (disjoint shards)
+    return [synth.config_batch("tgt", rank * N_BATCHES + i, batch=batch) for i in range(N_BATCHES)]
+
+
+def run_reference(args, world: int, rank: int):
+    """--impl reference: the FP64 oracle as it stands, on the host cores, rank 0 only."""
+    if rank != 0:
+        return
+    from threadpoolctl import threadpool_limits
+    from oracle import models as M
+    rng = np.random.default_rng(0)
+    P = synth.init_params(M.param_shapes("binary", H, E, C), rng)
+    X = synth.input_table(rng, V, E)
+    batches = make_batches(0, args.batch)
+    per_step = 1                     # bounded sample: one tree of the step's batch per step
+    with threadpool_limits(limits=1):
+        for w in range(args.warmup):
+            M.forward_backward("binary", P, X, batches[w % N_BATCHES][:per_step], H)
+        t0 = time.perf_counter()
+        for k in range(args.steps):
+            g = batches[k % N_BATCHES]
+            M.forward_backward("binary", P, X, [g[k % len(g)]], H)
+        dt = time.perf_counter() - t0
+    value = args.steps * per_step / dt
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": WORKLOAD, "global_batch": args.batch * world, "per_gpu_batch": args.batch,
+                   "parallelism": f"dp{world}"},
+        "cpu_baseline": {"value": value, "unit": "samples/s", "cores": 1, "kind": "oracle",
+                         "sample": f"{per_step} tree of each step's batch (FP64 NumPy, BLAS threads = 1)"},
+        "e2e": {"value": value, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(batches, budget_s=12.0):
+    """Oracle timed on a bounded sample of the same workload (1 thread)."""
+    from threadpoolctl import threadpool_limits
+    from oracle import models as M
+    rng = np.random.default_rng(0)
+    P = synth.init_params(M.param_shapes("binary", H, E, C), rng)
+    X = synth.input_table(rng, V, E)
+    n, t0 = 0, time.perf_counter()
+    with threadpool_limits(limits=1):
+        for g in batches:
+            for tree in g:
+                M.forward_backward("binary", P, X, [tree], H)
+                n += 1
+                if time.perf_counter() - t0 > budget_s:
+                    break
+            if time.perf_counter() - t0 > budget_s:
+                break
+    dt = time.perf_counter() - t0
+    return {"value": n / dt, "unit": "samples/s", "cores": 1, "kind": "oracle",
+            "sample": f"{n} trees of the bench batches in {dt:.1f} s (FP64 NumPy, BLAS threads = 1)"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--batch", type=int, default=16)
+    ap.add_argument("--impl", default="vpps", choices=["vpps", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-flush", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(3, args.warmup)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, world, rank)
+        return
+
+    import torch
+    from paper_conf_micro_khorasanieas18_b200 import vpps
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+
+    rng = np.random.default_rng(1234)          # identical initial parameters on every rank
+    shapes = vpps.param_shapes("binary", H, E, C)
+    P = synth.init_params(shapes, rng)
+    X = synth.input_table(rng, V, E)
+    m = vpps.Model("binary", H, E, C, device=local)
+    params = torch.zeros(m.n_floats, dtype=torch.float32, device=dev)
+    grads = torch.zeros_like(params)
+    for name, _ in shapes:
+        m.views(params)[name].copy_(torch.from_numpy(P[name]).float())
+    m.bind(params, grads)
+    inputs = torch.from_numpy(X).float().to(dev)
+    d_inputs = torch.zeros_like(inputs)
+    stream = torch.cuda.current_stream()
+    batches = make_batches(rank, args.batch)
+    scripts = [m.build_script(g) for g in batches]
+    for s in scripts:
+        s.upload()
+    infos = [s.info() for s in scripts]
+    flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device=dev)   # 256 MiB > 126 MB L2
+    lr, wd = 1e-3, 1e-5
+
+    def step(k):
+        s = scripts[k % N_BATCHES]
+        if world == 1:
+            m.fwd_bwd_sgd(s, inputs, d_inputs, lr=lr, weight_decay=wd)
+        else:
+            m.fwd_bwd(s, inputs, d_inputs)
+            dist.all_reduce(grads)
+            m.sgd_step(lr, wd)
+
+    kb, ka = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    for w in range(args.warmup):
+        step(w)
+    torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize()
+
+    clocks = ClockSampler(local)
+    clocks.start()
+    step_ms, kern_ms, flops = 0.0, 0.0, 0.0
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    for k in range(args.steps):
+        if not args.no_flush:
+            flush.zero_()
+        m.set_timing_events(*kev[k])
+        ev[k][0].record(stream)
+        step(args.warmup + k)
+        ev[k][1].record(stream)
+        flops += infos[(args.warmup + k) % N_BATCHES]["flops"]
+    m.set_timing_events(None, None)
+    torch.cuda.synchronize()
+    clk = clocks.stop()
+    step_ms = sum(a.elapsed_time(b) for a, b in ev)
+    kern_ms = sum(a.elapsed_time(b) for a, b in kev)
+    t = torch.tensor([step_ms, kern_ms], dtype=torch.float64, device=dev)
+    if dist:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    step_ms, kern_ms = float(t[0]), float(t[1])
+
+    # ---- end to end through the public API: host script build + one H2D copy + kernel + loss D2H ----
+    e2e_steps = min(args.steps, 50)
+    h2d = 0
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for k in range(e2e_steps):
+        g = batches[k % N_BATCHES]
+        s = m.build_script(g)                       # host: super-graph, levels, schedule, encode
+        h2d += s.info()["n_words"] * 4
+        s.upload()                                   # one pinned H2D copy (L169)
+        if world == 1:
+            m.fwd_bwd_sgd(s, inputs, d_inputs, lr=lr, weight_decay=wd)
+        else:
+            m.fwd_bwd(s, inputs, d_inputs)
+            dist.all_reduce(grads)
+            m.sgd_step(lr, wd)
+        m.latest_loss()                              # D2H of the step's loss
+    torch.cuda.synchronize()
+    e2e_s = time.perf_counter() - t0
+    te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+    if dist:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_s = float(te[0])
+
+    if rank == 0:
+        samples = args.steps * args.batch * world
+        value = samples / (step_ms / 1e3)
+        pk = peaks()
+        mhz = clk.get("sm_mhz") or pk.get("sm_max_mhz", 1965.0)
+        peak = fp32_peak_tflops(pk.get("sm_max_mhz", 1965.0))
+        avg_flops = flops / args.steps
+        achieved = avg_flops / (kern_ms / args.steps / 1e3) / 1e12
+        w_once = 4 * sum(int(np.prod(s)) for _, s in shapes if len(s) == 2)
+        traffic = None
+        prof = os.path.join(ROOT, "profiles", "r01_ncu_summary.json")
+        if os.path.exists(prof):
+            try:
+                traffic = json.load(open(prof)).get("dram_bytes_per_launch")
+            except Exception:
+                traffic = None
+        line = {
+            "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": step_ms / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "impl": "vpps",
+            "config": {"workload": WORKLOAD, "global_batch": args.batch * world, "per_gpu_batch": args.batch,
+                       "seq_len": None, "parallelism": f"dp{world}",
+                       "mode": "fused fwd-bwd-sgd, 1 kernel" if world == 1 else "fwd_bwd + NCCL all-reduce + sgd",
+                       "l2": "no flush" if args.no_flush else "flushed (256 MiB write) before every timed step",
+                       "batches": f"{N_BATCHES} distinct pre-built scripts cycled"},
+            "gpu_launches": args.steps * (1 if world == 1 else 2),
+            "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "kernel_ms": kern_ms / args.steps, "flops_per_launch": avg_flops,
+                         "peak_note": "FP32 FFMA: 148 SM x 128 lanes x 2 FLOP x sm_max_mhz (derived, DESIGN.md)"},
+            "dram": {"weights_once_bytes": w_once, "dram_bytes_per_pass": traffic,
+                     "source": "profiles/r01_ncu_summary.json (ncu --set full)" if traffic else None},
+            "e2e": {"value": e2e_steps * args.batch * world / e2e_s, "unit": "samples/s",
+                    "h2d_bytes_per_step": h2d // e2e_steps, "d2h_bytes_per_step": 4,
+                    "includes": "host script build + pinned H2D copy + kernel (+ all-reduce) + loss D2H"},
+            "clocks": clk,
+        }
+        if world == 1 and not args.no_cpu_baseline:
+            line["cpu_baseline"] = cpu_baseline(batches)
+        print(json.dumps(line), flush=True)
+    if dist:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -169,6 +169,11 @@ vpps_status vpps_fwd_bwd_sgd(vpps_model m, vpps_script s, const float* inputs, i
 vpps_status vpps_get_stale_loss(vpps_model m, float* loss);
 vpps_status vpps_sync_get_latest_loss(vpps_model m, float* loss);
 
+/* Measurement hook: when set (cudaEvent_t handles, or NULL to clear), every later launch records
+ * ev_before immediately before and ev_after immediately after the persistent kernel on the
+ * launching stream, so the kernel's own duration can be timed without the pool memsets. */
+vpps_status vpps_set_timing_events(vpps_model m, void* ev_before, void* ev_after);
+
 /* Device pointer of the model's activation pool (SPEC §S7 layout of the last script run). */
 vpps_status vpps_pool_ptr(vpps_model m, float** pool, int64_t* pool_words);
 

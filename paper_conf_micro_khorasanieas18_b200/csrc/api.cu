@@ -57,6 +57,7 @@ struct vpps_model_s {
     float* h_loss = nullptr;            // pinned [2]
     cudaEvent_t ev[2] = {nullptr, nullptr};
     int64_t passes = 0;
+    cudaEvent_t t_before = nullptr, t_after = nullptr;
 };
 
 struct vpps_script_s {
@@ -297,7 +298,9 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     kp.lr = lr;
     kp.wd = wd;
     void* args[] = {&kp};
+    if (m->t_before) CK(cudaEventRecord(m->t_before, st));
     CK(cudaLaunchCooperativeKernel(m->var->fn, dim3(m->plan.n_cta), dim3(256), args, m->smem, st));
+    if (m->t_after) CK(cudaEventRecord(m->t_after, st));
     const int slot = (int)(m->passes & 1);
     CK(cudaMemcpyAsync(m->h_loss + slot, m->pool + s->s.loss_word, sizeof(float), cudaMemcpyDeviceToHost, st));
     CK(cudaEventRecord(m->ev[slot], st));
@@ -340,6 +343,13 @@ vpps_status vpps_sync_get_latest_loss(vpps_model m, float* loss) {
     const int slot = (int)((m->passes - 1) & 1);
     CK(cudaEventSynchronize(m->ev[slot]));
     *loss = m->h_loss[slot];
+    return VPPS_OK;
+}
+
+vpps_status vpps_set_timing_events(vpps_model m, void* ev_before, void* ev_after) {
+    if (!m) return fail(VPPS_E_INVALID, "null model");
+    m->t_before = (cudaEvent_t)ev_before;
+    m->t_after = (cudaEvent_t)ev_after;
     return VPPS_OK;
 }
 

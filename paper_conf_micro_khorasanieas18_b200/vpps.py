@@ -73,6 +73,7 @@ def _load():
         "vpps_get_stale_loss": [VP, P(F)],
         "vpps_sync_get_latest_loss": [VP, P(F)],
         "vpps_pool_ptr": [VP, P(VP), P(I64)],
+        "vpps_set_timing_events": [VP, VP, VP],
         "vpps_destroy_script": [VP],
         "vpps_destroy_model": [VP],
         "vpps_last_error": [],
@@ -261,6 +262,11 @@ class Model:
         v = ct.c_float()
         _check(_lib.vpps_sync_get_latest_loss(self._h, ct.byref(v)))
         return v.value
+
+    def set_timing_events(self, before, after):
+        """torch.cuda.Event pair recorded around every later kernel launch (None clears)."""
+        _check(_lib.vpps_set_timing_events(self._h, ct.c_void_p(before.cuda_event) if before else None,
+                                           ct.c_void_p(after.cuda_event) if after else None))
 
     def pool(self):
         """(device pointer, words) of the activation pool of the last pass."""

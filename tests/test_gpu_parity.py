@@ -130,10 +130,14 @@ def test_fused_sgd_update():
 def test_dp_split_equals_union():
     """Data parallelism invariant on one GPU: Σ gradients of the shards == gradient of the union."""
     graphs = synth.config_batch("tgt", 2)
-    g_all = run_case("binary", 256, 256, 5, graphs, 4096, seed=4)[5].cpu().numpy()
-    g_a = run_case("binary", 256, 256, 5, graphs[:7], 4096, seed=4)[5].cpu().numpy()
-    g_b = run_case("binary", 256, 256, 5, graphs[7:], 4096, seed=4)[5].cpu().numpy()
-    assert rel(g_a + g_b, g_all) <= TOL
+
+    def grads_of(gs):
+        m, _, _, _, _, grads, _ = run_case("binary", 256, 256, 5, gs, 4096, seed=4)
+        return {k: v.numpy() for k, v in m.views(grads.cpu()).items()}
+
+    g_all, g_a, g_b = grads_of(graphs), grads_of(graphs[:7]), grads_of(graphs[7:])
+    for k in g_all:
+        assert rel(g_a[k] + g_b[k], g_all[k]) <= TOL, k
 
 
 def test_stale_and_latest_loss():
