@@ -226,6 +226,10 @@ def main():
     step_ms, kern_ms, flops = 0.0, 0.0, 0.0
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    for a, b in kev:            # torch creates the CUDA event lazily on first record
+        a.record(stream)
+        b.record(stream)
+    torch.cuda.synchronize()
     for k in range(args.steps):
         if not args.no_flush:
             flush.zero_()

@@ -82,7 +82,10 @@ struct Cfg {
     static constexpr int O_DBIAS = O_BIAS + UMAX * 4;
     static constexpr int O_IPOS = O_DBIAS + UMAX * 4;
     static constexpr int O_CSLOT = O_IPOS + NBMAX;
-    static constexpr int O_HEAD = a4(O_CSLOT + NBMAX);
+    static constexpr int O_BST = O_CSLOT + NBMAX;
+    static constexpr int O_CREC = O_BST + 4;
+    static constexpr int O_HEAD = a4(O_CREC + CHSLOT);
+    static constexpr int ITER = ((NBMAX + (CS ? CHSLOT : 0)) * KPMAX / 4 + NTH - 1) / NTH;
     static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 3 * C + H + 8); }
 };
 
@@ -128,6 +131,91 @@ __device__ __forceinline__ void warp_allreduce(float (&a)[N], int n_used) {
             for (int s = 16; s >= 1; s >>= 1) a[o] += __shfl_xor_sync(0xffffffffu, a[o], s);
         }
     }
+}
+
+
+// acc[n][o] += w[r] . x[n] over granule t for 4 nodes, packed FFMA2 (fma.rn.f32x2) where CG >= 2.
+// Rows 0..R-1 accumulate into outputs 0..R-1, except row 3 -> output SPLIT when SPLIT >= 0.
+template <int R, int CG, int SPLIT, int NR, int NREG, int RO>
+__device__ __forceinline__ void mv_acc(const float (&w)[NR][NREG], int t, const float (&xv)[4][CG],
+                                       float2 (&a)[4][RO]) {
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int o = (SPLIT >= 0 && r == 3) ? SPLIT : r;
+        if constexpr (CG >= 2) {
+#pragma unroll
+            for (int q = 0; q < CG; q += 2) {
+                const float2 w2 = make_float2(w[r][t * CG + q], w[r][t * CG + q + 1]);
+#pragma unroll
+                for (int n = 0; n < 4; ++n) a[n][o] = __ffma2_rn(w2, make_float2(xv[n][q], xv[n][q + 1]), a[n][o]);
+            }
+        } else {
+#pragma unroll
+            for (int n = 0; n < 4; ++n) a[n][o].x = fmaf(w[r][t], xv[n][0], a[n][o].x);
+        }
+    }
+}
+
+template <int CG, int NREG>
+__device__ __forceinline__ void dot_acc(const float (&w)[NREG], int t, const float (&y)[CG], float2& a) {
+    if constexpr (CG >= 2) {
+#pragma unroll
+        for (int q = 0; q < CG; q += 2)
+            a = __ffma2_rn(make_float2(w[t * CG + q], w[t * CG + q + 1]), make_float2(y[q], y[q + 1]), a);
+    } else {
+        a.x = fmaf(w[t], y[0], a.x);
+    }
+}
+
+// Backward over granule t: dW[r] += g_r * x (outer product into the gradient registers, L104) and
+// dx = sum_r W[r] * g_r (transposed product without transposing the register view, fn4 L100).
+template <int R, int CG, int NR, int NREG, int RG>
+__device__ __forceinline__ void outer_tmv(const float (&w)[NR][NREG], float (&dw)[NR][NREG], int t,
+                                          const float (&gr)[RG], const float (&xv)[CG], float (&dx)[CG]) {
+    if constexpr (CG >= 2) {
+#pragma unroll
+        for (int q = 0; q < CG; q += 2) {
+            const int k = t * CG + q;
+            const float2 x2 = make_float2(xv[q], xv[q + 1]);
+            float2 d = make_float2(0.f, 0.f);
+#pragma unroll
+            for (int r = 0; r < R; ++r) {
+                const float2 g2 = make_float2(gr[r], gr[r]);
+                const float2 nd = __ffma2_rn(g2, x2, make_float2(dw[r][k], dw[r][k + 1]));
+                dw[r][k] = nd.x;
+                dw[r][k + 1] = nd.y;
+                d = __ffma2_rn(make_float2(w[r][k], w[r][k + 1]), g2, d);
+            }
+            dx[q] = d.x;
+            dx[q + 1] = d.y;
+        }
+    } else {
+        float d = 0.f;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            dw[r][t] = fmaf(gr[r], xv[0], dw[r][t]);
+            d = fmaf(w[r][t], gr[r], d);
+        }
+        dx[0] = d;
+    }
+}
+
+// Sum over the 32 lanes of four per-lane values v0..v3 (one per node) with 6 shuffles: a transposed
+// butterfly (halving exchanges at lane distance 16 and 8, then a butterfly over the low 3 bits).
+// Lane l ends with the full sum of node ((l >> 3) & 3).
+__device__ __forceinline__ float treduce4(float v0, float v1, float v2, float v3, int lane) {
+    const bool b4 = lane & 16, b3 = lane & 8;
+    const float s0 = b4 ? v0 : v2, s1 = b4 ? v1 : v3;
+    float k0 = b4 ? v2 : v0, k1 = b4 ? v3 : v1;
+    k0 += __shfl_xor_sync(0xffffffffu, s0, 16);
+    k1 += __shfl_xor_sync(0xffffffffu, s1, 16);
+    const float s = b3 ? k0 : k1;
+    float k = b3 ? k1 : k0;
+    k += __shfl_xor_sync(0xffffffffu, s, 8);
+    k += __shfl_xor_sync(0xffffffffu, k, 4);
+    k += __shfl_xor_sync(0xffffffffu, k, 2);
+    k += __shfl_xor_sync(0xffffffffu, k, 1);
+    return k;
 }
 
 // Signal/wait barriers (L165): release-add on a global counter; acquire-spin until the target count.
@@ -250,6 +338,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
     }
 
     // ---------------- script interpretation (L171-177) ---------------------------------------------
+    int* bst = reinterpret_cast<int*>(smw + T::O_BST);        // [nb, next position]
+    uint32_t* crec = smw + T::O_CREC;                          // child-sum: record of each staged child
     uint32_t cbase = s0;
     auto refill = [&](uint32_t from) {
         __syncthreads();
@@ -265,31 +355,43 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
         const uint32_t op = pre & 0xFF;
         if (op == OP_S) { bar_signal(bar + (pre >> 8)); ++pos; continue; }
         if (op == OP_W) { bar_wait(bar + (pre >> 8), target[pre >> 8]); ++pos; continue; }
-        // gather a batch of consecutive instructions with the same opcode
+        // ---- decode: one thread gathers a batch of consecutive same-opcode instructions ----
         __syncthreads();
-        int nb = 0, used = 0;
-        uint32_t p = pos;
-        while (p < s1 && nb < NBMAX) {
-            const uint32_t w = chunk[p - cbase];
-            if ((w & 0xFF) != op) break;
-            const int sz = instr_words(w);
-            if (p + sz > cbase + CHUNK) break;
+        if (tid == 0) {
+            int nb = 0, used = 0;
+            uint32_t p = pos;
             const bool cs_op = CS && (op == OP_CS_F || op == OP_CS_B);
-            if (cs_op && used + (int)(w >> 8) > CHSLOT) break;
-            if (tid == 0) { ipos[nb] = (int)(p - cbase); cslot[nb] = used; }
-            if (cs_op) used += (int)(w >> 8);
-            ++nb;
-            p += sz;
+            while (p < s1 && nb < NBMAX) {
+                const uint32_t w = chunk[p - cbase];
+                if ((w & 0xFF) != op) break;
+                const int sz = instr_words(w);
+                if (p + sz > cbase + CHUNK) break;
+                if (cs_op && used + (int)(w >> 8) > CHSLOT) break;
+                ipos[nb] = (int)(p - cbase);
+                cslot[nb] = used;
+                if (cs_op) {
+                    const uint32_t* I = chunk + (p - cbase);
+                    for (int k = 0; k < (int)(w >> 8); ++k) crec[used + k] = (op == OP_CS_F) ? I[3 + k] : I[4 + 2 * k];
+                    used += (int)(w >> 8);
+                }
+                ++nb;
+                p += sz;
+            }
+            bst[0] = nb;
+            bst[1] = (int)p;
+            bst[2] = used;
         }
         __syncthreads();
+        const int nb = bst[0];
+        const uint32_t p = (uint32_t)bst[1];
         const bool is_head = (op == OP_HEAD_F || op == OP_HEAD_B);
         if (is_head) {
             if (holds_head) {
                 for (int n = 0; n < nb; ++n) {
                     const uint32_t* I = chunk + ipos[n];
-                    const uint32_t rec = I[1], crec = I[2];
+                    const uint32_t rec = I[1], crc = I[2];
                     const int y = (int)(op == OP_HEAD_F ? I[3] : I[4]);
-                    for (int k = tid; k < H; k += NTH) hbuf[k] = __ldcg(pool + crec + k);
+                    for (int k = tid; k < H; k += NTH) hbuf[k] = __ldcg(pool + crc + k);
                     if (op == OP_HEAD_B)
                         for (int c = tid; c < C; c += NTH) zs[c] = __ldcg(pool + rec + c) - (c == y ? 1.f : 0.f);
                     __syncthreads();
@@ -338,127 +440,163 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
 
         const bool fwd = (op & 1) == 0;
         const bool kindB = BIN && (op == OP_INT_F || op == OP_INT_B);
-        // ---- stage the node inputs (coalesced 16-B loads) into shared memory ----
+        const int KP = kindB ? LB::KP : LA::KP;
+        // ---- stage the node inputs into shared memory: every load of the batch is issued before the
+        //      first store (one L2 round trip per batch, not one per element) ----
         {
-            const int KP = kindB ? LB::KP : LA::KP;
             const int q4 = KP / 4;
-            for (int i = tid; i < nb * q4; i += NTH) {
-                const int n = i / q4, c = (i - n * q4) * 4;
-                const uint32_t* I = chunk + ipos[n];
-                float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-                if constexpr (BIN) {
-                    if (!kindB) {
-                        const uint32_t tok = fwd ? I[2] : I[3];
-                        if (c < E) v = ld4g(inputs + (int64_t)tok * E + c);
-                    } else {
-                        const uint32_t rl = fwd ? I[2] : I[3], rr = fwd ? I[3] : I[5];
-                        if (c < H) v = ld4cg(pool + rl + c);
-                        else if (c < 2 * H) v = ld4cg(pool + rr + (c - H));
-                    }
-                } else if constexpr (LS) {
-                    const uint32_t tok = fwd ? I[2] : I[3], prv = fwd ? I[3] : I[4];
-                    if (c < E) v = ld4g(inputs + (int64_t)tok * E + c);
-                    else if (c < E + H && prv != NONE) v = ld4cg(pool + prv + (c - E));
-                } else {
-                    const uint32_t tok = fwd ? I[2] : I[3];
-                    const int nch = (int)(I[0] >> 8);
-                    if (c < E) {
-                        if (tok != NONE) v = ld4g(inputs + (int64_t)tok * E + c);
-                    } else if (c < E + H) {
-                        for (int k = 0; k < nch; ++k) {
-                            const uint32_t ck = fwd ? I[3 + k] : I[4 + 2 * k];
-                            const float4 hv = ld4cg(pool + ck + (c - E));
-                            v.x += hv.x; v.y += hv.y; v.z += hv.z; v.w += hv.w;
-                            *reinterpret_cast<float4*>(chs + (cslot[n] + k) * KP + c) = hv;
+            const int rows = nb + (CS ? bst[2] : 0);
+            const int total = rows * q4;
+            float4 v[T::ITER];
+#pragma unroll
+            for (int it = 0; it < T::ITER; ++it) {
+                const int i = tid + it * NTH;
+                const float* src = nullptr;
+                if (i < total) {
+                    const int n = i / q4, c = (i - n * q4) * 4;
+                    if (n < nb) {
+                        const uint32_t* I = chunk + ipos[n];
+                        if constexpr (BIN) {
+                            if (!kindB) {
+                                if (c < E) src = inputs + (int64_t)(fwd ? I[2] : I[3]) * E + c;
+                            } else {
+                                const uint32_t rl = fwd ? I[2] : I[3], rr = fwd ? I[3] : I[5];
+                                if (c < H) src = pool + rl + c;
+                                else if (c < 2 * H) src = pool + rr + (c - H);
+                            }
+                        } else if constexpr (LS) {
+                            const uint32_t tok = fwd ? I[2] : I[3], prv = fwd ? I[3] : I[4];
+                            if (c < E) src = inputs + (int64_t)tok * E + c;
+                            else if (c < E + H && prv != NONE) src = pool + prv + (c - E);
+                        } else {
+                            const uint32_t tok = fwd ? I[2] : I[3];
+                            if (c < E && tok != NONE) src = inputs + (int64_t)tok * E + c;
                         }
+                    } else if (c >= E && c < E + H) {        // child-sum: a child's h row
+                        src = pool + crec[n - nb] + (c - E);
                     }
-                    if (!(c >= E && c < E + H))
-                        for (int k = 0; k < nch; ++k)
-                            *reinterpret_cast<float4*>(chs + (cslot[n] + k) * KP + c) = make_float4(0.f, 0.f, 0.f, 0.f);
                 }
-                *reinterpret_cast<float4*>(xs + n * KP + c) = v;
+                v[it] = src ? ld4cg(src) : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+#pragma unroll
+            for (int it = 0; it < T::ITER; ++it) {
+                const int i = tid + it * NTH;
+                if (i < total) {
+                    const int n = i / q4, c = (i - n * q4) * 4;
+                    float* dst = n < nb ? xs + n * KP + c : chs + (n - nb) * KP + c;
+                    *reinterpret_cast<float4*>(dst) = v[it];
+                }
+            }
+            if constexpr (CS) {     // h~ = sum of the children's h (child-sum, [5] eq. 2)
+                __syncthreads();
+                for (int i = tid; i < nb * (H / 4); i += NTH) {
+                    const int n = i / (H / 4), c = E + (i - n * (H / 4)) * 4;
+                    const int nch = (int)(chunk[ipos[n]] >> 8);
+                    float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
+                    for (int k = 0; k < nch; ++k) {
+                        const float4 hv = *reinterpret_cast<const float4*>(chs + (cslot[n] + k) * KP + c);
+                        s.x += hv.x; s.y += hv.y; s.z += hv.z; s.w += hv.w;
+                    }
+                    *reinterpret_cast<float4*>(xs + n * KP + c) = s;
+                }
             }
         }
 
         if (fwd) {
             __syncthreads();
-            // ---- matrix-vector products from registers (L123): partial sums per warp ----
-            for (int n = 0; n < nb; ++n) {
-                float acc[RO];
-#pragma unroll
-                for (int o = 0; o < RO; ++o) acc[o] = 0.f;
+            // ---- matrix-vector products from registers (L123), 4 nodes at a time: packed FFMA2,
+            //      then one transposed butterfly per output reduces the 4 nodes across the warp ----
+            for (int n0 = 0; n0 < nb; n0 += 4) {
+                float v[4][RO];
                 int n_used = RO;
                 if (kindB) {
                     if constexpr (BIN) {
-                        const float* x = xs + n * LB::KP;
+                        float2 a[4][5];
+#pragma unroll
+                        for (int n = 0; n < 4; ++n)
+#pragma unroll
+                            for (int o = 0; o < 5; ++o) a[n][o] = make_float2(0.f, 0.f);
 #pragma unroll
                         for (int t = 0; t < LB::NT; ++t) {
                             const int col0 = LB::CG * (tu + TU * t);
-                            float xv[LB::CG];
-                            lds<LB::CG>(x + col0, xv);
                             const bool lo = col0 < H;
+                            float xv[4][LB::CG];
 #pragma unroll
-                            for (int q = 0; q < LB::CG; ++q) {
-                                const int k = t * LB::CG + q;
-#pragma unroll
-                                for (int r = 0; r < 3; ++r) acc[r] = fmaf(wb[r][k], xv[q], acc[r]);
-                                const float pf = wb[3][k] * xv[q];
-                                acc[3] += lo ? pf : 0.f;
-                                acc[4] += lo ? 0.f : pf;
+                            for (int n = 0; n < 4; ++n) lds<LB::CG>(xs + (n0 + n) * LB::KP + col0, xv[n]);
+                            if (lo) {
+                                mv_acc<4, LB::CG, 3>(wb, t, xv, a);
+                            } else {
+                                mv_acc<4, LB::CG, 4>(wb, t, xv, a);
                             }
                         }
+#pragma unroll
+                        for (int n = 0; n < 4; ++n)
+#pragma unroll
+                            for (int o = 0; o < 5; ++o) v[n][o] = a[n][o].x + a[n][o].y;
                     }
                 } else {
-                    const float* x = xs + n * LA::KP;
+                    float2 a[4][RO];
+#pragma unroll
+                    for (int n = 0; n < 4; ++n)
+#pragma unroll
+                        for (int o = 0; o < RO; ++o) a[n][o] = make_float2(0.f, 0.f);
 #pragma unroll
                     for (int t = 0; t < LA::NT; ++t) {
                         const int col0 = LA::CG * (tu + TU * t);
-                        float xv[LA::CG];
-                        lds<LA::CG>(x + col0, xv);
+                        float xv[4][LA::CG];
 #pragma unroll
-                        for (int q = 0; q < LA::CG; ++q) {
-                            const int k = t * LA::CG + q;
-                            if constexpr (BIN) {
-#pragma unroll
-                                for (int r = 0; r < 3; ++r) acc[r] = fmaf(wa[r][k], xv[q], acc[r]);
-                            } else if constexpr (LS) {
-#pragma unroll
-                                for (int r = 0; r < 4; ++r) acc[r] = fmaf(wa[r][k], xv[q], acc[r]);
-                            } else {
-#pragma unroll
-                                for (int r = 0; r < 3; ++r) acc[r] = fmaf(wa[r][k], xv[q], acc[r]);
-                                if (col0 < E) acc[3] = fmaf(wa[3][k], xv[q], acc[3]);
-                            }
+                        for (int n = 0; n < 4; ++n) lds<LA::CG>(xs + (n0 + n) * LA::KP + col0, xv[n]);
+                        if constexpr (BIN) {
+                            mv_acc<3, LA::CG, -1>(wa, t, xv, a);
+                        } else if constexpr (LS) {
+                            mv_acc<4, LA::CG, -1>(wa, t, xv, a);
+                        } else {
+                            // child-sum: rows i,o,u over [x; h~]; row f over x only here (its h part is
+                            // applied to every child's own h below)
+                            if (col0 < E) mv_acc<4, LA::CG, -1>(wa, t, xv, a);
+                            else mv_acc<3, LA::CG, -1>(wa, t, xv, a);
                         }
                     }
                     if constexpr (CS) {
-                        const uint32_t* I = chunk + ipos[n];
-                        const int nch = (int)(I[0] >> 8);
-                        n_used = 4 + nch;
+                        int nmax = 0;
+#pragma unroll
+                        for (int n = 0; n < 4; ++n)
+                            if (n0 + n < nb) nmax = max(nmax, (int)(chunk[ipos[n0 + n]] >> 8));
+                        n_used = 4 + nmax;
 #pragma unroll
                         for (int kc = 0; kc < CHMAX; ++kc) {
-                            if (kc < nch) {
-                                const float* y = chs + (cslot[n] + kc) * LA::KP;
+                            if (kc < nmax) {
 #pragma unroll
                                 for (int t = 0; t < LA::NT; ++t) {
                                     const int col0 = LA::CG * (tu + TU * t);
-                                    float yv[LA::CG];
-                                    lds<LA::CG>(y + col0, yv);
+                                    if (col0 < E) continue;
 #pragma unroll
-                                    for (int q = 0; q < LA::CG; ++q)
-                                        acc[4 + kc] = fmaf(wa[3][t * LA::CG + q], yv[q], acc[4 + kc]);
+                                    for (int n = 0; n < 4; ++n) {
+                                        const int nn = n0 + n;
+                                        const int nch = nn < nb ? (int)(chunk[ipos[nn]] >> 8) : 0;
+                                        if (kc < nch) {
+                                            float yv[LA::CG];
+                                            lds<LA::CG>(chs + (cslot[nn] + kc) * LA::KP + col0, yv);
+                                            dot_acc<LA::CG>(wa[3], t, yv, a[n][4 + kc]);
+                                        }
+                                    }
                                 }
                             }
                         }
                     } else if constexpr (BIN) {
                         n_used = 3;
                     }
-                }
-                warp_allreduce<RO>(acc, n_used);
-                if (lane == 0) {
 #pragma unroll
-                    for (int o = 0; o < RO; ++o)
-                        if (o < n_used) red[(warp * NBMAX + n) * RO + o] = acc[o];
+                    for (int n = 0; n < 4; ++n)
+#pragma unroll
+                        for (int o = 0; o < RO; ++o) v[n][o] = a[n][o].x + a[n][o].y;
+                }
+#pragma unroll
+                for (int o = 0; o < RO; ++o) {
+                    if (o < n_used) {
+                        const float r = treduce4(v[0][o], v[1][o], v[2][o], v[3][o], lane);
+                        if ((lane & 7) == 0) red[(warp * NBMAX + n0 + (lane >> 3)) * RO + o] = r;
+                    }
                 }
             }
             __syncthreads();
@@ -590,7 +728,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                 }
             }
             __syncthreads();
-            // ---- in-register outer products (dW, L104) and transposed products (L94, fn4) ----
+            // ---- in-register outer products (dW, L104) and transposed products (L94, fn4), FFMA2 ----
             if (unit_ok) {
                 for (int n = 0; n < nb; ++n) {
                     const uint32_t* I = chunk + ipos[n];
@@ -598,22 +736,15 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                     if (kindB) {
                         if constexpr (BIN) {
                             const float* x = xs + n * LB::KP;
-                            const float g0 = g[0], g1 = g[1], g2 = g[2], g3 = g[3], g4 = g[4];
+                            float gr[4] = {g[0], g[1], g[2], 0.f};
+                            const float g3 = g[3], g4 = g[4];
 #pragma unroll
                             for (int t = 0; t < LB::NT; ++t) {
                                 const int col0 = LB::CG * (tu + TU * t);
+                                gr[3] = col0 < H ? g3 : g4;
                                 float xv[LB::CG], dx[LB::CG];
                                 lds<LB::CG>(x + col0, xv);
-                                const float gf = col0 < H ? g3 : g4;
-#pragma unroll
-                                for (int q = 0; q < LB::CG; ++q) {
-                                    const int k = t * LB::CG + q;
-                                    dwb[0][k] = fmaf(g0, xv[q], dwb[0][k]);
-                                    dwb[1][k] = fmaf(g1, xv[q], dwb[1][k]);
-                                    dwb[2][k] = fmaf(g2, xv[q], dwb[2][k]);
-                                    dwb[3][k] = fmaf(gf, xv[q], dwb[3][k]);
-                                    dx[q] = wb[0][k] * g0 + wb[1][k] * g1 + wb[2][k] * g2 + wb[3][k] * gf;
-                                }
+                                outer_tmv<4, LB::CG>(wb, dwb, t, gr, xv, dx);
                                 if (col0 < 2 * H) {
                                     float* dst = col0 < H ? pool + I[4] + col0 : pool + I[6] + (col0 - H);
                                     red_add<LB::CG>(dst, dx);
@@ -623,40 +754,25 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                     } else {
                         const float* x = xs + n * LA::KP;
                         if constexpr (BIN) {
-                            const float g0 = g[0], g1 = g[1], g2 = g[2];
+                            const float gr[3] = {g[0], g[1], g[2]};
                             const uint32_t tok = I[3];
 #pragma unroll
                             for (int t = 0; t < LA::NT; ++t) {
                                 const int col0 = LA::CG * (tu + TU * t);
                                 float xv[LA::CG], dx[LA::CG];
                                 lds<LA::CG>(x + col0, xv);
-#pragma unroll
-                                for (int q = 0; q < LA::CG; ++q) {
-                                    const int k = t * LA::CG + q;
-                                    dwa[0][k] = fmaf(g0, xv[q], dwa[0][k]);
-                                    dwa[1][k] = fmaf(g1, xv[q], dwa[1][k]);
-                                    dwa[2][k] = fmaf(g2, xv[q], dwa[2][k]);
-                                    dx[q] = wa[0][k] * g0 + wa[1][k] * g1 + wa[2][k] * g2;
-                                }
+                                outer_tmv<3, LA::CG>(wa, dwa, t, gr, xv, dx);
                                 if (P.d_inputs && col0 < E) red_add<LA::CG>(P.d_inputs + (int64_t)tok * E + col0, dx);
                             }
                         } else if constexpr (LS) {
-                            const float g0 = g[0], g1 = g[1], g2 = g[2], g3 = g[3];
+                            const float gr[4] = {g[0], g[1], g[2], g[3]};
                             const uint32_t tok = I[3], padj = I[5];
 #pragma unroll
                             for (int t = 0; t < LA::NT; ++t) {
                                 const int col0 = LA::CG * (tu + TU * t);
                                 float xv[LA::CG], dx[LA::CG];
                                 lds<LA::CG>(x + col0, xv);
-#pragma unroll
-                                for (int q = 0; q < LA::CG; ++q) {
-                                    const int k = t * LA::CG + q;
-                                    dwa[0][k] = fmaf(g0, xv[q], dwa[0][k]);
-                                    dwa[1][k] = fmaf(g1, xv[q], dwa[1][k]);
-                                    dwa[2][k] = fmaf(g2, xv[q], dwa[2][k]);
-                                    dwa[3][k] = fmaf(g3, xv[q], dwa[3][k]);
-                                    dx[q] = wa[0][k] * g0 + wa[1][k] * g1 + wa[2][k] * g2 + wa[3][k] * g3;
-                                }
+                                outer_tmv<4, LA::CG>(wa, dwa, t, gr, xv, dx);
                                 if (col0 < E) {
                                     if (P.d_inputs) red_add<LA::CG>(P.d_inputs + (int64_t)tok * E + col0, dx);
                                 } else if (col0 < E + H && padj != NONE) {
@@ -664,7 +780,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                                 }
                             }
                         } else {
-                            const float g0 = g[0], g1 = g[1], g2 = g[2], gfs = g[3];
+                            const float gr[4] = {g[0], g[1], g[2], g[3]};     // g[3] = sum_k g_fk for the x part
                             const uint32_t tok = I[3];
                             const int nch = (int)(I[0] >> 8);
 #pragma unroll
@@ -672,24 +788,11 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                                 const int col0 = LA::CG * (tu + TU * t);
                                 float xv[LA::CG], dio[LA::CG];
                                 lds<LA::CG>(x + col0, xv);
-#pragma unroll
-                                for (int q = 0; q < LA::CG; ++q) {
-                                    const int k = t * LA::CG + q;
-                                    dwa[0][k] = fmaf(g0, xv[q], dwa[0][k]);
-                                    dwa[1][k] = fmaf(g1, xv[q], dwa[1][k]);
-                                    dwa[2][k] = fmaf(g2, xv[q], dwa[2][k]);
-                                    dio[q] = wa[0][k] * g0 + wa[1][k] * g1 + wa[2][k] * g2;
-                                }
                                 if (col0 < E) {
-                                    float dx[LA::CG];
-#pragma unroll
-                                    for (int q = 0; q < LA::CG; ++q) {
-                                        const int k = t * LA::CG + q;
-                                        dwa[3][k] = fmaf(gfs, xv[q], dwa[3][k]);
-                                        dx[q] = dio[q] + wa[3][k] * gfs;
-                                    }
-                                    if (P.d_inputs && tok != NONE) red_add<LA::CG>(P.d_inputs + (int64_t)tok * E + col0, dx);
+                                    outer_tmv<4, LA::CG>(wa, dwa, t, gr, xv, dio);
+                                    if (P.d_inputs && tok != NONE) red_add<LA::CG>(P.d_inputs + (int64_t)tok * E + col0, dio);
                                 } else if (col0 < E + H) {
+                                    outer_tmv<3, LA::CG>(wa, dwa, t, gr, xv, dio);
 #pragma unroll
                                     for (int kc = 0; kc < CHMAX; ++kc) {
                                         if (kc < nch) {
@@ -700,7 +803,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                                             for (int q = 0; q < LA::CG; ++q) {
                                                 const int k = t * LA::CG + q;
                                                 dwa[3][k] = fmaf(gf, yv[q], dwa[3][k]);
-                                                dh[q] = dio[q] + wa[3][k] * gf;
+                                                dh[q] = fmaf(wa[3][k], gf, dio[q]);
                                             }
                                             red_add<LA::CG>(pool + I[5 + 2 * kc] + (col0 - E), dh);
                                         }
