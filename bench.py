@@ -204,14 +204,14 @@ def main():
     flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device=dev)   # 256 MiB > 126 MB L2
     lr, wd = 1e-3, 1e-5
 
+    from paper_conf_micro_khorasanieas18_b200 import dp
+
     def step(k):
         s = scripts[k % N_BATCHES]
         if world == 1:
             m.fwd_bwd_sgd(s, inputs, d_inputs, lr=lr, weight_decay=wd)
         else:
-            m.fwd_bwd(s, inputs, d_inputs)
-            dist.all_reduce(grads)
-            m.sgd_step(lr, wd)
+            dp.dp_step(m, s, inputs, d_inputs, grads, lr, wd)
 
     kb, ka = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     for w in range(args.warmup):
@@ -263,9 +263,7 @@ def main():
         if world == 1:
             m.fwd_bwd_sgd(s, inputs, d_inputs, lr=lr, weight_decay=wd)
         else:
-            m.fwd_bwd(s, inputs, d_inputs)
-            dist.all_reduce(grads)
-            m.sgd_step(lr, wd)
+            dp.dp_step(m, s, inputs, d_inputs, grads, lr, wd)
         m.latest_loss()                              # D2H of the step's loss
     torch.cuda.synchronize()
     e2e_s = time.perf_counter() - t0

@@ -174,6 +174,11 @@ vpps_status vpps_sync_get_latest_loss(vpps_model m, float* loss);
  * launching stream, so the kernel's own duration can be timed without the pool memsets. */
 vpps_status vpps_set_timing_events(vpps_model m, void* ev_before, void* ev_after);
 
+/* In-kernel phase trace (measurement only): when buf != NULL (dev, >= n_cta*stride uint64), every
+ * later launch writes per CTA, from %globaltimer (ns): [0] start of interpretation, [1] end, and for
+ * barrier b: [2+3b] signal, [3+3b] wait begin, [4+3b] wait end.  stride >= 2 + 3*(n_barriers+1). */
+vpps_status vpps_set_profile_buffer(vpps_model m, uint64_t* buf, int64_t stride);
+
 /* Device pointer of the model's activation pool (SPEC §S7 layout of the last script run). */
 vpps_status vpps_pool_ptr(vpps_model m, float** pool, int64_t* pool_words);
 

@@ -58,6 +58,8 @@ struct vpps_model_s {
     cudaEvent_t ev[2] = {nullptr, nullptr};
     int64_t passes = 0;
     cudaEvent_t t_before = nullptr, t_after = nullptr;
+    uint64_t* prof = nullptr;
+    int64_t prof_stride = 0;
 };
 
 struct vpps_script_s {
@@ -297,6 +299,10 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     kp.loss_word = s->s.loss_word;
     kp.lr = lr;
     kp.wd = wd;
+    if (m->prof && m->prof_stride < 2 + 3 * (int64_t)(s->s.n_bar + 1))
+        return fail(VPPS_E_INVALID, "profile buffer stride too small for this script");
+    kp.prof = m->prof;
+    kp.prof_stride = m->prof_stride;
     void* args[] = {&kp};
     if (m->t_before) CK(cudaEventRecord(m->t_before, st));
     CK(cudaLaunchCooperativeKernel(m->var->fn, dim3(m->plan.n_cta), dim3(256), args, m->smem, st));
@@ -350,6 +356,13 @@ vpps_status vpps_set_timing_events(vpps_model m, void* ev_before, void* ev_after
     if (!m) return fail(VPPS_E_INVALID, "null model");
     m->t_before = (cudaEvent_t)ev_before;
     m->t_after = (cudaEvent_t)ev_after;
+    return VPPS_OK;
+}
+
+vpps_status vpps_set_profile_buffer(vpps_model m, uint64_t* buf, int64_t stride) {
+    if (!m) return fail(VPPS_E_INVALID, "null model");
+    m->prof = buf;
+    m->prof_stride = stride;
     return VPPS_OK;
 }
 

@@ -219,15 +219,24 @@ __device__ __forceinline__ float treduce4(float v0, float v1, float v2, float v3
 }
 
 // Signal/wait barriers (L165): release-add on a global counter; acquire-spin until the target count.
-__device__ __forceinline__ void bar_signal(unsigned* ctr) {
+__device__ __forceinline__ uint64_t gtimer() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+// prof (optional, VPPS profiling): per CTA [start, end, then per barrier b: signal, wait-begin, wait-end]
+__device__ __forceinline__ void bar_signal(unsigned* ctr, uint64_t* prof) {
     __syncthreads();
     if (threadIdx.x == 0) {
+        if (prof) prof[0] = gtimer();
         __threadfence();
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(ctr) : "memory");
     }
 }
-__device__ __forceinline__ void bar_wait(const unsigned* ctr, unsigned target) {
+__device__ __forceinline__ void bar_wait(const unsigned* ctr, unsigned target, uint64_t* prof) {
     if (threadIdx.x == 0) {
+        if (prof) prof[1] = gtimer();
         unsigned v;
         while (true) {
             asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
@@ -235,6 +244,7 @@ __device__ __forceinline__ void bar_wait(const unsigned* ctr, unsigned target) {
             __nanosleep(32);
         }
         __threadfence();
+        if (prof) prof[2] = gtimer();
     }
     __syncthreads();
 }
@@ -337,6 +347,9 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
         for (int i = tid; i < C; i += NTH) { bo[i] = __ldg(P.params + off[bout_m] + i); dbo[i] = 0.f; }
     }
 
+    uint64_t* prof = P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
+    __syncthreads();
+    if (prof && tid == 0) prof[0] = gtimer();
     // ---------------- script interpretation (L171-177) ---------------------------------------------
     int* bst = reinterpret_cast<int*>(smw + T::O_BST);        // [nb, next position]
     uint32_t* crec = smw + T::O_CREC;                          // child-sum: record of each staged child
@@ -353,8 +366,12 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
         if (pos + 640 > cbase + CHUNK && cbase + CHUNK < s1) refill(pos);
         const uint32_t pre = chunk[pos - cbase];
         const uint32_t op = pre & 0xFF;
-        if (op == OP_S) { bar_signal(bar + (pre >> 8)); ++pos; continue; }
-        if (op == OP_W) { bar_wait(bar + (pre >> 8), target[pre >> 8]); ++pos; continue; }
+        if (op == OP_S) { bar_signal(bar + (pre >> 8), prof ? prof + 2 + 3 * (pre >> 8) : nullptr); ++pos; continue; }
+        if (op == OP_W) {
+            bar_wait(bar + (pre >> 8), target[pre >> 8], prof ? prof + 2 + 3 * (pre >> 8) : nullptr);
+            ++pos;
+            continue;
+        }
         // ---- decode: one thread gathers a batch of consecutive same-opcode instructions ----
         __syncthreads();
         if (tid == 0) {
@@ -820,6 +837,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
 
     // ---------------- epilogue: apply gradients to the master copy, or write them (L129, L197) -----
     __syncthreads();
+    if (prof && tid == 0) prof[1] = gtimer();
     const bool sgd = P.mode == 1;
     float* gout = P.grads;
     auto put = [&](int64_t idx, float w, float dw) {

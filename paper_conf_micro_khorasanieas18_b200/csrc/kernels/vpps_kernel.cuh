@@ -16,6 +16,8 @@ struct KParams {
     int32_t n_g, n_act, C, mode;   // mode 0: write grads; 1: fused SGD update
     int64_t loss_word;
     float lr, wd;
+    uint64_t* prof;         // optional globaltimer trace (vpps_set_profile_buffer), or nullptr
+    int64_t prof_stride;
 };
 
 struct Variant {

@@ -74,6 +74,7 @@ def _load():
         "vpps_sync_get_latest_loss": [VP, P(F)],
         "vpps_pool_ptr": [VP, P(VP), P(I64)],
         "vpps_set_timing_events": [VP, VP, VP],
+        "vpps_set_profile_buffer": [VP, VP, I64],
         "vpps_destroy_script": [VP],
         "vpps_destroy_model": [VP],
         "vpps_last_error": [],
@@ -267,6 +268,11 @@ class Model:
         """torch.cuda.Event pair recorded around every later kernel launch (None clears)."""
         _check(_lib.vpps_set_timing_events(self._h, ct.c_void_p(before.cuda_event) if before else None,
                                            ct.c_void_p(after.cuda_event) if after else None))
+
+    def set_profile_buffer(self, buf=None, stride=0):
+        """int64 CUDA tensor [n_cta, stride] receiving the in-kernel globaltimer trace (None clears)."""
+        _check(_lib.vpps_set_profile_buffer(self._h, ct.c_void_p(buf.data_ptr()) if buf is not None else None,
+                                            stride))
 
     def pool(self):
         """(device pointer, words) of the activation pool of the last pass."""
