@@ -136,6 +136,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
             return fail(VPPS_E_NOFIT, "no kernel specialisation for cell " + std::to_string(cell) + " H=" +
                                           std::to_string(H) + " E=" + std::to_string(E) +
                                           " units/CTA=" + std::to_string(m->plan.umax));
+        if (C > 32) return fail(VPPS_E_NOFIT, "single-CTA loss head supports C <= 32 classes in v1");
         m->smem = m->var->smem_bytes(C);
         if (m->smem > 227 * 1024) return fail(VPPS_E_NOFIT, "head does not fit in shared memory");
         CK(cudaFuncSetAttribute(m->var->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)m->smem));

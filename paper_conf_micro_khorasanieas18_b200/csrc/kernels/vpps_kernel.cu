@@ -9,10 +9,12 @@
 //
 // B200 design: 148 persistent CTAs x 256 threads (L102, L106), gate-colocated unit
 // bundles (SPEC P1): the CTA that owns hidden unit j holds every gate row of j, so a cell update is
-// CTA-local and needs no barrier between matvec and cell; thread tau of a unit's thread group holds
-// columns CG*(tau + TU*t) + q of every gate row (coalesced, 16-B vectorised staging/reads), partial dot
-// products are reduced by warp shuffles then across the group's warps in shared memory; the transposed
-// product of the backward pass is issued as vector red.global.add.v4.f32 (L94, fn4 L100).
+// CTA-local and needs no barrier between matvec and cell.  Thread tau of a unit's thread group holds
+// columns CG*(tau + TU*t) + q of every gate row.  Consecutive same-opcode instructions run as one batch:
+// one warp decodes them in parallel, every global load the batch needs (input vectors and the
+// per-unit cell operands) is issued in one round trip, the matvecs use packed FFMA2, partial dot
+// products are reduced with a transposed butterfly over 4 nodes, and the transposed products of the
+// backward pass are vector red.global.add.v4.f32 (L94, fn4 L100).
 #include <cstdio>
 #include "vpps_kernel.cuh"
 
@@ -20,11 +22,11 @@ namespace vpps {
 namespace dev {
 
 constexpr int NTH = 256;       // CTA width (L102)
-constexpr int NBMAX = 16;      // instructions executed as one batch
 constexpr int CHUNK = 4096;    // script words staged in shared memory (L171)
 constexpr int CHMAX = 8;       // child-sum children per node
-constexpr int CHSLOT = 32;     // child vectors staged per child-sum batch
+constexpr int ZC = 32;         // classes per head handled by one warp (C <= 32)
 constexpr uint32_t NONE = 0xFFFFFFFFu;
+constexpr uint32_t FULL = 0xFFFFFFFFu;
 constexpr int CELL_LSTM = 0, CELL_BINARY = 1, CELL_CHILDSUM = 2;
 enum : uint32_t {
     OP_S = 0x01, OP_W = 0x02, OP_LSTM_F = 0x10, OP_LSTM_B = 0x11, OP_LEAF_F = 0x20, OP_LEAF_B = 0x21,
@@ -48,6 +50,20 @@ __device__ __forceinline__ int instr_words(uint32_t w) {
     }
 }
 
+// Per-(node, unit) cell operands fetched with the batch's input vectors (see cin_src).
+__device__ __forceinline__ int n_cin(uint32_t op) {
+    switch (op) {
+        case OP_INT_F: return 2;
+        case OP_INT_B: return 10;
+        case OP_LEAF_B: return 6;
+        case OP_LSTM_F: return 1;
+        case OP_LSTM_B: return 8;
+        case OP_CS_F: return CHMAX;
+        case OP_CS_B: return 6 + 2 * CHMAX;
+        default: return 0;
+    }
+}
+
 // Column layout of a K-long bundle row over TU threads: granules of CG consecutive floats.
 template <int K, int TU>
 struct Lay {
@@ -58,6 +74,7 @@ struct Lay {
 };
 
 constexpr int cmax(int a, int b) { return a > b ? a : b; }
+constexpr int cmin(int a, int b) { return a < b ? a : b; }
 constexpr int a4(int x) { return (x + 3) / 4 * 4; }
 
 template <int CELL, int H, int E, int UMAX>
@@ -72,38 +89,42 @@ struct Cfg {
     using LA = Lay<KA, TU>;
     using LB = Lay<KB, TU>;
     static constexpr int KPMAX = BIN ? cmax(LA::KP, LB::KP) : LA::KP;
-    static constexpr int RO = BIN ? 5 : (LS ? 4 : 4 + CHMAX);
-    static constexpr int GO = BIN ? 5 : (LS ? 4 : 4 + CHMAX);
+    static constexpr int NB = cmin(CS ? 16 : 32, (16384 / KPMAX) / 4 * 4);   // nodes per batch (<= 64 KB staged)
+    static constexpr int CHSLOT = CS ? 2 * NB : 0;                  // child rows staged per batch
+    static constexpr int RO = BIN ? 5 : (LS ? 4 : 4 + CHMAX);        // matvec outputs per node
+    static constexpr int GO = BIN ? 5 : (LS ? 4 : 4 + CHMAX);        // gate gradients per node
+    static constexpr int CINMAX = BIN ? 10 : (LS ? 8 : 6 + 2 * CHMAX);
     static constexpr int O_X = CHUNK;
-    static constexpr int O_CH = O_X + NBMAX * KPMAX;
-    static constexpr int O_RED = O_CH + (CS ? CHSLOT * KPMAX : 0);
-    static constexpr int O_GB = O_RED + 8 * NBMAX * RO;
-    static constexpr int O_BIAS = O_GB + UMAX * NBMAX * GO;
+    static constexpr int O_CH = O_X + NB * KPMAX;
+    static constexpr int O_RED = O_CH + CHSLOT * KPMAX;
+    static constexpr int O_GB = O_RED + 8 * NB * RO;
+    static constexpr int O_CIN = O_GB + UMAX * NB * GO;
+    static constexpr int O_BIAS = O_CIN + NB * UMAX * CINMAX;
     static constexpr int O_DBIAS = O_BIAS + UMAX * 4;
     static constexpr int O_IPOS = O_DBIAS + UMAX * 4;
-    static constexpr int O_CSLOT = O_IPOS + NBMAX;
-    static constexpr int O_BST = O_CSLOT + NBMAX;
+    static constexpr int O_CSLOT = O_IPOS + NB;
+    static constexpr int O_BST = O_CSLOT + NB;
     static constexpr int O_CREC = O_BST + 4;
-    static constexpr int O_HEAD = a4(O_CREC + CHSLOT);
-    static constexpr int ITER = ((NBMAX + (CS ? CHSLOT : 0)) * KPMAX / 4 + NTH - 1) / NTH;
-    static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 3 * C + H + 8); }
+    static constexpr int O_ZS = a4(O_CREC + cmax(CHSLOT, 1));
+    static constexpr int O_HEAD = O_ZS + 8 * ZC;
+    static constexpr int ITER = ((NB + CHSLOT) * KPMAX / 4 + NTH - 1) / NTH;
+    static constexpr int ITER2 = (NB * UMAX * CINMAX + NTH - 1) / NTH;
+    static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 2 * C + 8); }
 };
 
 __device__ __forceinline__ float sigm(float x) { return 1.0f / (1.0f + expf(-x)); }
-
 __device__ __forceinline__ float4 ld4cg(const float* p) { return __ldcg(reinterpret_cast<const float4*>(p)); }
-__device__ __forceinline__ float4 ld4g(const float* p) { return __ldg(reinterpret_cast<const float4*>(p)); }
+__device__ __forceinline__ float4 f4zero() { return make_float4(0.f, 0.f, 0.f, 0.f); }
 
 // Vectorised no-return float add in L2 (REDG.E.ADD.F32x4 on sm_90+): remote accumulation of the
-// transposed matrix-vector product (fn4 L100).
+// transposed matrix-vector product (fn4 L100).  The data is only read after a barrier.
 template <int CG>
 __device__ __forceinline__ void red_add(float* p, const float* v) {
     if constexpr (CG == 4) {
         asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(v[0]), "f"(v[1]), "f"(v[2]),
-                     "f"(v[3])
-                     : "memory");
+                     "f"(v[3]));
     } else if constexpr (CG == 2) {
-        asm volatile("red.global.add.v2.f32 [%0], {%1, %2};" ::"l"(p), "f"(v[0]), "f"(v[1]) : "memory");
+        asm volatile("red.global.add.v2.f32 [%0], {%1, %2};" ::"l"(p), "f"(v[0]), "f"(v[1]));
     } else {
         atomicAdd(p, v[0]);
     }
@@ -121,18 +142,6 @@ __device__ __forceinline__ void lds(const float* p, float* v) {
         v[0] = *p;
     }
 }
-
-template <int N>
-__device__ __forceinline__ void warp_allreduce(float (&a)[N], int n_used) {
-#pragma unroll
-    for (int o = 0; o < N; ++o) {
-        if (o < n_used) {
-#pragma unroll
-            for (int s = 16; s >= 1; s >>= 1) a[o] += __shfl_xor_sync(0xffffffffu, a[o], s);
-        }
-    }
-}
-
 
 // acc[n][o] += w[r] . x[n] over granule t for 4 nodes, packed FFMA2 (fma.rn.f32x2) where CG >= 2.
 // Rows 0..R-1 accumulate into outputs 0..R-1, except row 3 -> output SPLIT when SPLIT >= 0.
@@ -207,30 +216,42 @@ __device__ __forceinline__ float treduce4(float v0, float v1, float v2, float v3
     const bool b4 = lane & 16, b3 = lane & 8;
     const float s0 = b4 ? v0 : v2, s1 = b4 ? v1 : v3;
     float k0 = b4 ? v2 : v0, k1 = b4 ? v3 : v1;
-    k0 += __shfl_xor_sync(0xffffffffu, s0, 16);
-    k1 += __shfl_xor_sync(0xffffffffu, s1, 16);
+    k0 += __shfl_xor_sync(FULL, s0, 16);
+    k1 += __shfl_xor_sync(FULL, s1, 16);
     const float s = b3 ? k0 : k1;
     float k = b3 ? k1 : k0;
-    k += __shfl_xor_sync(0xffffffffu, s, 8);
-    k += __shfl_xor_sync(0xffffffffu, k, 4);
-    k += __shfl_xor_sync(0xffffffffu, k, 2);
-    k += __shfl_xor_sync(0xffffffffu, k, 1);
+    k += __shfl_xor_sync(FULL, s, 8);
+    k += __shfl_xor_sync(FULL, k, 4);
+    k += __shfl_xor_sync(FULL, k, 2);
+    k += __shfl_xor_sync(FULL, k, 1);
     return k;
 }
 
-// Signal/wait barriers (L165): release-add on a global counter; acquire-spin until the target count.
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+    for (int s = 16; s >= 1; s >>= 1) v += __shfl_xor_sync(FULL, v, s);
+    return v;
+}
+__device__ __forceinline__ float warp_max(float v) {
+#pragma unroll
+    for (int s = 16; s >= 1; s >>= 1) v = fmaxf(v, __shfl_xor_sync(FULL, v, s));
+    return v;
+}
+
 __device__ __forceinline__ uint64_t gtimer() {
     uint64_t t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
 
-// prof (optional, VPPS profiling): per CTA [start, end, then per barrier b: signal, wait-begin, wait-end]
+// Signal/wait barriers (L165).  Producer: CTA barrier, then one release-add on the global counter;
+// consumer: one thread acquire-spins until the target count, then a CTA barrier.  The release/acquire
+// pair at gpu scope plus bar.sync order every thread's writes before every other CTA's later reads.
+// prof (optional trace): [signal, wait-begin, wait-end] globaltimer stamps of this barrier.
 __device__ __forceinline__ void bar_signal(unsigned* ctr, uint64_t* prof) {
     __syncthreads();
     if (threadIdx.x == 0) {
         if (prof) prof[0] = gtimer();
-        __threadfence();
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(ctr) : "memory");
     }
 }
@@ -238,15 +259,54 @@ __device__ __forceinline__ void bar_wait(const unsigned* ctr, unsigned target, u
     if (threadIdx.x == 0) {
         if (prof) prof[1] = gtimer();
         unsigned v;
-        while (true) {
+        do {
             asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
-            if (v >= target) break;
-            __nanosleep(32);
-        }
-        __threadfence();
+        } while (v < target);
         if (prof) prof[2] = gtimer();
     }
     __syncthreads();
+}
+
+// Address of cell operand k of (instruction I, unit jj); nullptr -> 0.  Record layouts: SPEC §S7.
+template <int H>
+__device__ __forceinline__ const float* cin_src(uint32_t op, const uint32_t* I, int k, int jj, const float* pool) {
+    switch (op) {
+        case OP_INT_F:
+            return pool + (k == 0 ? I[2] : I[3]) + H + jj;                       // c_l, c_r
+        case OP_INT_B: {
+            const uint32_t rec = I[1], adj = I[2];
+            if (k < 2) return pool + adj + k * H + jj;                           // dh, dc
+            if (k < 8) return pool + rec + (k - 1) * H + jj;                     // c i o u fl fr
+            return pool + (k == 8 ? I[3] : I[5]) + H + jj;                       // c_l, c_r
+        }
+        case OP_LEAF_B: {
+            const uint32_t rec = I[1], adj = I[2];
+            if (k < 2) return pool + adj + k * H + jj;
+            return pool + rec + (k - 1) * H + jj;                                // c i o u
+        }
+        case OP_LSTM_F:
+            return I[3] != NONE ? pool + I[3] + H + jj : nullptr;               // c_prev
+        case OP_LSTM_B: {
+            const uint32_t rec = I[1], adj = I[2];
+            if (k < 2) return pool + adj + k * H + jj;
+            if (k < 7) return pool + rec + (k - 1) * H + jj;                     // c i f o g
+            return I[4] != NONE ? pool + I[4] + H + jj : nullptr;               // c_prev
+        }
+        case OP_CS_F: {
+            const int nch = (int)(I[0] >> 8);
+            return k < nch ? pool + I[3 + k] + H + jj : nullptr;                 // c_k
+        }
+        case OP_CS_B: {
+            const uint32_t rec = I[1], adj = I[2];
+            const int nch = (int)(I[0] >> 8);
+            if (k < 2) return pool + adj + k * H + jj;
+            if (k < 6) return pool + rec + (k - 1) * H + jj;                     // c i o u
+            if (k < 6 + CHMAX) return (k - 6) < nch ? pool + rec + (5 + k - 6) * H + jj : nullptr;   // f_k
+            return (k - 6 - CHMAX) < nch ? pool + I[4 + 2 * (k - 6 - CHMAX)] + H + jj : nullptr;   // c_k
+        }
+        default:
+            return nullptr;
+    }
 }
 
 template <int CELL, int H, int E, int UMAX>
@@ -254,9 +314,10 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
     using T = Cfg<CELL, H, E, UMAX>;
     using LA = typename T::LA;
     using LB = typename T::LB;
-    constexpr int TU = T::TU, WPU = T::WPU;
+    constexpr int TU = T::TU, WPU = T::WPU, NB = T::NB;
     constexpr bool BIN = T::BIN, CS = T::CS, LS = T::LS;
-    constexpr int KA = T::KA, KB = T::KB, RA = T::RA, RB = T::RB, RO = T::RO, GO = T::GO;
+    constexpr int KA = T::KA, KB = T::KB, RA = T::RA, RB = T::RB, RO = T::RO, GO = T::GO, CINMAX = T::CINMAX;
+    constexpr int HT = (H + 127) / 128;             // float4 granules of a hidden vector per lane
 
     extern __shared__ __align__(16) uint32_t smw[];
     float* sm = reinterpret_cast<float*>(smw);
@@ -265,17 +326,19 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
     float* chs = sm + T::O_CH;
     float* red = sm + T::O_RED;
     float* gb = sm + T::O_GB;
+    float* cin = sm + T::O_CIN;
     float* bias = sm + T::O_BIAS;
     float* dbias = sm + T::O_DBIAS;
     int* ipos = reinterpret_cast<int*>(smw + T::O_IPOS);
     int* cslot = reinterpret_cast<int*>(smw + T::O_CSLOT);
+    int* bst = reinterpret_cast<int*>(smw + T::O_BST);
+    uint32_t* crec = smw + T::O_CREC;
+    float* zs = sm + T::O_ZS;
     const int C = P.C;
     float* Wo = sm + T::O_HEAD;
     float* dWo = Wo + C * H;
     float* bo = dWo + C * H;
     float* dbo = bo + C;
-    float* zs = dbo + C;
-    float* hbuf = zs + C;
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int lc = blockIdx.x % P.n_g, grp = blockIdx.x / P.n_g;
@@ -350,13 +413,20 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
     uint64_t* prof = P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
     __syncthreads();
     if (prof && tid == 0) prof[0] = gtimer();
+
     // ---------------- script interpretation (L171-177) ---------------------------------------------
-    int* bst = reinterpret_cast<int*>(smw + T::O_BST);        // [nb, next position]
-    uint32_t* crec = smw + T::O_CREC;                          // child-sum: record of each staged child
     uint32_t cbase = s0;
-    auto refill = [&](uint32_t from) {
+    auto refill = [&](uint32_t from) {          // all loads of the chunk in flight before any store
         __syncthreads();
-        for (uint32_t i = tid; i < (uint32_t)CHUNK && from + i < s1; i += NTH) chunk[i] = S[from + i];
+        constexpr int PER = CHUNK / NTH;
+        uint32_t w[PER];
+#pragma unroll
+        for (int i = 0; i < PER; ++i) {
+            const uint32_t k = tid + i * NTH;
+            w[i] = from + k < s1 ? __ldg(S + from + k) : 0u;
+        }
+#pragma unroll
+        for (int i = 0; i < PER; ++i) chunk[tid + i * NTH] = w[i];
         __syncthreads();
         cbase = from;
     };
@@ -372,83 +442,116 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
             ++pos;
             continue;
         }
-        // ---- decode: one thread gathers a batch of consecutive same-opcode instructions ----
+        // ---- decode (warp 0): a batch of up to NB consecutive instructions with this opcode ----
         __syncthreads();
-        if (tid == 0) {
-            int nb = 0, used = 0;
-            uint32_t p = pos;
-            const bool cs_op = CS && (op == OP_CS_F || op == OP_CS_B);
-            while (p < s1 && nb < NBMAX) {
-                const uint32_t w = chunk[p - cbase];
-                if ((w & 0xFF) != op) break;
-                const int sz = instr_words(w);
-                if (p + sz > cbase + CHUNK) break;
-                if (cs_op && used + (int)(w >> 8) > CHSLOT) break;
-                ipos[nb] = (int)(p - cbase);
-                cslot[nb] = used;
-                if (cs_op) {
+        if (warp == 0) {
+            const uint32_t lim = min(s1, cbase + (uint32_t)CHUNK);
+            if (!(op == OP_CS_F || op == OP_CS_B)) {
+                const uint32_t sz = (uint32_t)instr_words(pre);
+                int nb = 0;
+                for (int base = 0; base < NB; base += 32) {
+                    const int n = base + lane;
+                    const uint32_t q = pos + (uint32_t)n * sz;
+                    const bool ok = n < NB && q + sz <= lim && (chunk[q - cbase] & 0xFF) == op;
+                    const unsigned m = __ballot_sync(FULL, ok);
+                    const int cnt = (m == FULL) ? 32 : (__ffs(~m) - 1);
+                    if (lane < cnt) ipos[n] = (int)(q - cbase);
+                    nb += cnt;
+                    if (cnt < 32) break;
+                }
+                if (lane == 0) { bst[0] = nb; bst[1] = (int)(pos + nb * sz); bst[2] = 0; }
+            } else if (lane == 0) {
+                int nb = 0, used = 0;
+                uint32_t p = pos;
+                while (p < lim && nb < NB) {
+                    const uint32_t w = chunk[p - cbase];
+                    if ((w & 0xFF) != op) break;
+                    const int sz = instr_words(w);
+                    if (p + sz > lim || used + (int)(w >> 8) > T::CHSLOT) break;
+                    ipos[nb] = (int)(p - cbase);
+                    cslot[nb] = used;
                     const uint32_t* I = chunk + (p - cbase);
                     for (int k = 0; k < (int)(w >> 8); ++k) crec[used + k] = (op == OP_CS_F) ? I[3 + k] : I[4 + 2 * k];
                     used += (int)(w >> 8);
+                    ++nb;
+                    p += sz;
                 }
-                ++nb;
-                p += sz;
+                bst[0] = nb; bst[1] = (int)p; bst[2] = used;
             }
-            bst[0] = nb;
-            bst[1] = (int)p;
-            bst[2] = used;
         }
         __syncthreads();
         const int nb = bst[0];
         const uint32_t p = (uint32_t)bst[1];
-        const bool is_head = (op == OP_HEAD_F || op == OP_HEAD_B);
-        if (is_head) {
+
+        // ---- loss heads (L42), one warp per head, on the CTA that holds W_out ----
+        if (op == OP_HEAD_F || op == OP_HEAD_B) {
             if (holds_head) {
-                for (int n = 0; n < nb; ++n) {
+                for (int n = warp; n < nb; n += NTH / 32) {
                     const uint32_t* I = chunk + ipos[n];
                     const uint32_t rec = I[1], crc = I[2];
-                    const int y = (int)(op == OP_HEAD_F ? I[3] : I[4]);
-                    for (int k = tid; k < H; k += NTH) hbuf[k] = __ldcg(pool + crc + k);
-                    if (op == OP_HEAD_B)
-                        for (int c = tid; c < C; c += NTH) zs[c] = __ldcg(pool + rec + c) - (c == y ? 1.f : 0.f);
-                    __syncthreads();
+                    float4 hv[HT];
+#pragma unroll
+                    for (int t = 0; t < HT; ++t) {
+                        const int k = 4 * (lane + 32 * t);
+                        hv[t] = k < H ? ld4cg(pool + crc + k) : f4zero();
+                    }
+                    float* z = zs + warp * ZC;
                     if (op == OP_HEAD_F) {
-                        for (int c = warp; c < C; c += NTH / 32) {
+                        const int y = (int)I[3];
+                        for (int c = 0; c < C; ++c) {
                             float s = 0.f;
-                            for (int k = lane; k < H; k += 32) s += Wo[c * H + k] * hbuf[k];
 #pragma unroll
-                            for (int sh = 16; sh >= 1; sh >>= 1) s += __shfl_xor_sync(0xffffffffu, s, sh);
-                            if (lane == 0) zs[c] = s + bo[c];
-                        }
-                        __syncthreads();
-                        if (warp == 0) {
-                            float m = -INFINITY;
-                            for (int c = lane; c < C; c += 32) m = fmaxf(m, zs[c]);
-#pragma unroll
-                            for (int sh = 16; sh >= 1; sh >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, sh));
-                            float se = 0.f;
-                            for (int c = lane; c < C; c += 32) se += expf(zs[c] - m);
-#pragma unroll
-                            for (int sh = 16; sh >= 1; sh >>= 1) se += __shfl_xor_sync(0xffffffffu, se, sh);
-                            const float lse = m + logf(se);
-                            for (int c = lane; c < C; c += 32) pool[rec + c] = expf(zs[c] - lse);
-                            if (lane == 0) {
-                                const float loss = lse - zs[y];
-                                pool[rec + C] = loss;
-                                atomicAdd(pool + P.loss_word, loss);   // aggregated loss node (L205)
+                            for (int t = 0; t < HT; ++t) {
+                                const int k = 4 * (lane + 32 * t);
+                                if (k < H) {
+                                    const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                                    s += w4.x * hv[t].x + w4.y * hv[t].y + w4.z * hv[t].z + w4.w * hv[t].w;
+                                }
                             }
+                            s = warp_sum(s);
+                            if (lane == 0) z[c] = s + bo[c];
+                        }
+                        __syncwarp();
+                        const float zl = lane < C ? z[lane] : -INFINITY;
+                        const float m = warp_max(zl);
+                        const float se = warp_sum(lane < C ? expf(zl - m) : 0.f);
+                        const float lse = m + logf(se);
+                        if (lane < C) pool[rec + lane] = expf(zl - lse);
+                        const float zy = __shfl_sync(FULL, zl, y);
+                        if (lane == 0) {
+                            pool[rec + C] = lse - zy;
+                            atomicAdd(pool + P.loss_word, lse - zy);   // aggregated loss node (L205)
                         }
                     } else {
                         const uint32_t cadj = I[3];
-                        for (int c = tid; c < C; c += NTH) dbo[c] += zs[c];
-                        for (int i = tid; i < C * H; i += NTH) dWo[i] += zs[i / H] * hbuf[i % H];
-                        for (int k = tid; k < H; k += NTH) {
-                            float s = 0.f;
-                            for (int c = 0; c < C; ++c) s += Wo[c * H + k] * zs[c];
-                            atomicAdd(pool + cadj + k, s);
+                        const int y = (int)I[4];
+                        const float dz = lane < C ? __ldcg(pool + rec + lane) - (lane == y ? 1.f : 0.f) : 0.f;
+                        if (lane < C) atomicAdd(dbo + lane, dz);
+                        float4 dh[HT];
+#pragma unroll
+                        for (int t = 0; t < HT; ++t) dh[t] = f4zero();
+                        for (int c = 0; c < C; ++c) {
+                            const float dzc = __shfl_sync(FULL, dz, c);
+#pragma unroll
+                            for (int t = 0; t < HT; ++t) {
+                                const int k = 4 * (lane + 32 * t);
+                                if (k < H) {
+                                    float* dw = dWo + c * H + k;
+                                    atomicAdd(dw + 0, dzc * hv[t].x); atomicAdd(dw + 1, dzc * hv[t].y);
+                                    atomicAdd(dw + 2, dzc * hv[t].z); atomicAdd(dw + 3, dzc * hv[t].w);
+                                    const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                                    dh[t].x += w4.x * dzc; dh[t].y += w4.y * dzc;
+                                    dh[t].z += w4.z * dzc; dh[t].w += w4.w * dzc;
+                                }
+                            }
+                        }
+#pragma unroll
+                        for (int t = 0; t < HT; ++t) {
+                            const int k = 4 * (lane + 32 * t);
+                            const float v4[4] = {dh[t].x, dh[t].y, dh[t].z, dh[t].w};
+                            if (k < H) red_add<4>(pool + cadj + k, v4);
                         }
                     }
-                    __syncthreads();
                 }
             }
             pos = p;
@@ -458,13 +561,16 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
         const bool fwd = (op & 1) == 0;
         const bool kindB = BIN && (op == OP_INT_F || op == OP_INT_B);
         const int KP = kindB ? LB::KP : LA::KP;
-        // ---- stage the node inputs into shared memory: every load of the batch is issued before the
-        //      first store (one L2 round trip per batch, not one per element) ----
+        // ---- one round trip: every input row and cell operand of the batch is loaded before the
+        //      first shared-memory store ----
         {
             const int q4 = KP / 4;
             const int rows = nb + (CS ? bst[2] : 0);
             const int total = rows * q4;
+            const int ncin = n_cin(op);
+            const int total2 = nb * UMAX * ncin;
             float4 v[T::ITER];
+            float s2[T::ITER2];
 #pragma unroll
             for (int it = 0; it < T::ITER; ++it) {
                 const int i = tid + it * NTH;
@@ -493,7 +599,18 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                         src = pool + crec[n - nb] + (c - E);
                     }
                 }
-                v[it] = src ? ld4cg(src) : make_float4(0.f, 0.f, 0.f, 0.f);
+                v[it] = src ? ld4cg(src) : f4zero();
+            }
+#pragma unroll
+            for (int it = 0; it < T::ITER2; ++it) {
+                const int i = tid + it * NTH;
+                const float* src = nullptr;
+                if (i < total2) {
+                    const int n = i / (UMAX * ncin), rem = i - n * (UMAX * ncin);
+                    const int uu = rem / ncin, k = rem - uu * ncin, jj = lc + uu * P.n_g;
+                    if (jj < H) src = cin_src<H>(op, chunk + ipos[n], k, jj, pool);
+                }
+                s2[it] = src ? __ldcg(src) : 0.f;
             }
 #pragma unroll
             for (int it = 0; it < T::ITER; ++it) {
@@ -504,12 +621,21 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                     *reinterpret_cast<float4*>(dst) = v[it];
                 }
             }
+#pragma unroll
+            for (int it = 0; it < T::ITER2; ++it) {
+                const int i = tid + it * NTH;
+                if (i < total2) {
+                    const int n = i / (UMAX * ncin), rem = i - n * (UMAX * ncin);
+                    const int uu = rem / ncin, k = rem - uu * ncin;
+                    cin[(n * UMAX + uu) * CINMAX + k] = s2[it];
+                }
+            }
             if constexpr (CS) {     // h~ = sum of the children's h (child-sum, [5] eq. 2)
                 __syncthreads();
                 for (int i = tid; i < nb * (H / 4); i += NTH) {
                     const int n = i / (H / 4), c = E + (i - n * (H / 4)) * 4;
                     const int nch = (int)(chunk[ipos[n]] >> 8);
-                    float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
+                    float4 s = f4zero();
                     for (int k = 0; k < nch; ++k) {
                         const float4 hv = *reinterpret_cast<const float4*>(chs + (cslot[n] + k) * KP + c);
                         s.x += hv.x; s.y += hv.y; s.z += hv.z; s.w += hv.w;
@@ -518,9 +644,9 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                 }
             }
         }
+        __syncthreads();
 
         if (fwd) {
-            __syncthreads();
             // ---- matrix-vector products from registers (L123), 4 nodes at a time: packed FFMA2,
             //      then one transposed butterfly per output reduces the 4 nodes across the warp ----
             for (int n0 = 0; n0 < nb; n0 += 4) {
@@ -536,15 +662,11 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
 #pragma unroll
                         for (int t = 0; t < LB::NT; ++t) {
                             const int col0 = LB::CG * (tu + TU * t);
-                            const bool lo = col0 < H;
                             float xv[4][LB::CG];
 #pragma unroll
                             for (int n = 0; n < 4; ++n) lds<LB::CG>(xs + (n0 + n) * LB::KP + col0, xv[n]);
-                            if (lo) {
-                                mv_acc<4, LB::CG, 3>(wb, t, xv, a);
-                            } else {
-                                mv_acc<4, LB::CG, 4>(wb, t, xv, a);
-                            }
+                            if (col0 < H) mv_acc<4, LB::CG, 3>(wb, t, xv, a);
+                            else mv_acc<4, LB::CG, 4>(wb, t, xv, a);
                         }
 #pragma unroll
                         for (int n = 0; n < 4; ++n)
@@ -568,8 +690,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                         } else if constexpr (LS) {
                             mv_acc<4, LA::CG, -1>(wa, t, xv, a);
                         } else {
-                            // child-sum: rows i,o,u over [x; h~]; row f over x only here (its h part is
-                            // applied to every child's own h below)
+                            // child-sum: rows i,o,u over [x; h~]; row f over x here (its h part meets
+                            // every child's own h below)
                             if (col0 < E) mv_acc<4, LA::CG, -1>(wa, t, xv, a);
                             else mv_acc<3, LA::CG, -1>(wa, t, xv, a);
                         }
@@ -612,144 +734,136 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                 for (int o = 0; o < RO; ++o) {
                     if (o < n_used) {
                         const float r = treduce4(v[0][o], v[1][o], v[2][o], v[3][o], lane);
-                        if ((lane & 7) == 0) red[(warp * NBMAX + n0 + (lane >> 3)) * RO + o] = r;
+                        if ((lane & 7) == 0) red[(warp * NB + n0 + (lane >> 3)) * RO + o] = r;
                     }
                 }
             }
             __syncthreads();
             // ---- cell update, one thread per (unit slot, node): CTA-local thanks to gate colocation ----
-            if (tid < UMAX * NBMAX) {
-                const int uu = tid / NBMAX, n = tid % NBMAX, jj = lc + uu * P.n_g;
-                if (n < nb && jj < H) {
-                    const uint32_t* I = chunk + ipos[n];
-                    const uint32_t rec = I[1];
-                    float a[RO];
+            for (int ci = tid; ci < UMAX * NB; ci += NTH) {
+                const int uu = ci / NB, n = ci % NB, jj = lc + uu * P.n_g;
+                if (n >= nb || jj >= H) continue;
+                const uint32_t* I = chunk + ipos[n];
+                const uint32_t rec = I[1];
+                const float* cv = cin + (n * UMAX + uu) * CINMAX;
+                float a[RO];
 #pragma unroll
-                    for (int o = 0; o < RO; ++o) {
-                        float s = 0.f;
+                for (int o = 0; o < RO; ++o) {
+                    float s = 0.f;
 #pragma unroll
-                        for (int w = 0; w < WPU; ++w) s += red[((uu * WPU + w) * NBMAX + n) * RO + o];
-                        a[o] = s;
+                    for (int w = 0; w < WPU; ++w) s += red[((uu * WPU + w) * NB + n) * RO + o];
+                    a[o] = s;
+                }
+                const float* b = bias + uu * 4;
+                if constexpr (BIN) {
+                    const float i = sigm(a[0] + b[0]), o = sigm(a[1] + b[1]), uv = tanhf(a[2] + b[2]);
+                    float c = i * uv;
+                    if (kindB) {
+                        const float fl = sigm(a[3] + b[3]), fr = sigm(a[4] + b[3]);
+                        c += fl * cv[0] + fr * cv[1];
+                        pool[rec + 5 * H + jj] = fl;
+                        pool[rec + 6 * H + jj] = fr;
                     }
-                    const float* b = bias + uu * 4;
-                    if constexpr (BIN) {
-                        const float i = sigm(a[0] + b[0]), o = sigm(a[1] + b[1]), uv = tanhf(a[2] + b[2]);
-                        float c = i * uv;
-                        if (kindB) {
-                            const float fl = sigm(a[3] + b[3]), fr = sigm(a[4] + b[3]);
-                            c += fl * __ldcg(pool + I[2] + H + jj) + fr * __ldcg(pool + I[3] + H + jj);
-                            pool[rec + 5 * H + jj] = fl;
-                            pool[rec + 6 * H + jj] = fr;
-                        }
-                        pool[rec + jj] = o * tanhf(c);
-                        pool[rec + H + jj] = c;
-                        pool[rec + 2 * H + jj] = i;
-                        pool[rec + 3 * H + jj] = o;
-                        pool[rec + 4 * H + jj] = uv;
-                    } else if constexpr (LS) {
-                        const float i = sigm(a[0] + b[0]), f = sigm(a[1] + b[1]), o = sigm(a[2] + b[2]),
-                                    g = tanhf(a[3] + b[3]);
-                        const float cp = I[3] != NONE ? __ldcg(pool + I[3] + H + jj) : 0.f;
-                        const float c = f * cp + i * g;
-                        pool[rec + jj] = o * tanhf(c);
-                        pool[rec + H + jj] = c;
-                        pool[rec + 2 * H + jj] = i;
-                        pool[rec + 3 * H + jj] = f;
-                        pool[rec + 4 * H + jj] = o;
-                        pool[rec + 5 * H + jj] = g;
-                    } else {
-                        const int nch = (int)(I[0] >> 8);
-                        const float i = sigm(a[0] + b[0]), o = sigm(a[1] + b[1]), uv = tanhf(a[2] + b[2]);
-                        const float fx = a[3] + b[3];
-                        float c = i * uv;
+                    pool[rec + jj] = o * tanhf(c);
+                    pool[rec + H + jj] = c;
+                    pool[rec + 2 * H + jj] = i;
+                    pool[rec + 3 * H + jj] = o;
+                    pool[rec + 4 * H + jj] = uv;
+                } else if constexpr (LS) {
+                    const float i = sigm(a[0] + b[0]), f = sigm(a[1] + b[1]), o = sigm(a[2] + b[2]),
+                                g = tanhf(a[3] + b[3]);
+                    const float c = f * cv[0] + i * g;
+                    pool[rec + jj] = o * tanhf(c);
+                    pool[rec + H + jj] = c;
+                    pool[rec + 2 * H + jj] = i;
+                    pool[rec + 3 * H + jj] = f;
+                    pool[rec + 4 * H + jj] = o;
+                    pool[rec + 5 * H + jj] = g;
+                } else {
+                    const int nch = (int)(I[0] >> 8);
+                    const float i = sigm(a[0] + b[0]), o = sigm(a[1] + b[1]), uv = tanhf(a[2] + b[2]);
+                    const float fx = a[3] + b[3];
+                    float c = i * uv;
 #pragma unroll
-                        for (int kc = 0; kc < CHMAX; ++kc) {
-                            if (kc < nch) {
-                                const float f = sigm(fx + a[4 + kc]);
-                                c += f * __ldcg(pool + I[3 + kc] + H + jj);
-                                pool[rec + (5 + kc) * H + jj] = f;
-                            }
+                    for (int kc = 0; kc < CHMAX; ++kc) {
+                        if (kc < nch) {
+                            const float f = sigm(fx + a[4 + kc]);
+                            c += f * cv[kc];
+                            pool[rec + (5 + kc) * H + jj] = f;
                         }
-                        pool[rec + jj] = o * tanhf(c);
-                        pool[rec + H + jj] = c;
-                        pool[rec + 2 * H + jj] = i;
-                        pool[rec + 3 * H + jj] = o;
-                        pool[rec + 4 * H + jj] = uv;
                     }
+                    pool[rec + jj] = o * tanhf(c);
+                    pool[rec + H + jj] = c;
+                    pool[rec + 2 * H + jj] = i;
+                    pool[rec + 3 * H + jj] = o;
+                    pool[rec + 4 * H + jj] = uv;
                 }
             }
         } else {
             // ---- backward: cell backward per (unit slot, node) -> gate gradients in smem ----
-            if (tid < UMAX * NBMAX) {
-                const int uu = tid / NBMAX, n = tid % NBMAX, jj = lc + uu * P.n_g;
-                if (n < nb && jj < H) {
-                    const uint32_t* I = chunk + ipos[n];
-                    const uint32_t rec = I[1], adj = I[2];
-                    const float dh = __ldcg(pool + adj + jj), dc = __ldcg(pool + adj + H + jj);
-                    const float c = __ldcg(pool + rec + H + jj);
-                    const float th = tanhf(c);
-                    float* g = gb + (uu * NBMAX + n) * GO;
-                    float* db = dbias + uu * 4;
-                    if constexpr (BIN || CS) {
-                        const float i = __ldcg(pool + rec + 2 * H + jj), o = __ldcg(pool + rec + 3 * H + jj),
-                                    uv = __ldcg(pool + rec + 4 * H + jj);
-                        const float dov = dh * th;
-                        const float chat = dc + dh * o * (1.f - th * th);
-                        const float gi = chat * uv * i * (1.f - i), go = dov * o * (1.f - o),
-                                    gu = chat * i * (1.f - uv * uv);
-                        g[0] = gi; g[1] = go; g[2] = gu;
-                        atomicAdd(db + 0, gi); atomicAdd(db + 1, go); atomicAdd(db + 2, gu);
-                        if constexpr (BIN) {
-                            if (kindB) {
-                                const float fl = __ldcg(pool + rec + 5 * H + jj), fr = __ldcg(pool + rec + 6 * H + jj);
-                                const float cl = __ldcg(pool + I[3] + H + jj), cr = __ldcg(pool + I[5] + H + jj);
-                                const float gfl = chat * cl * fl * (1.f - fl), gfr = chat * cr * fr * (1.f - fr);
-                                pool[I[4] + H + jj] = chat * fl;     // dc of the left child (unique parent)
-                                pool[I[6] + H + jj] = chat * fr;
-                                g[3] = gfl; g[4] = gfr;
-                                atomicAdd(db + 3, gfl + gfr);
-                            }
-                        } else {
-                            const int nch = (int)(I[0] >> 8);
-                            float gfs = 0.f;
-#pragma unroll
-                            for (int kc = 0; kc < CHMAX; ++kc) {
-                                float gf = 0.f;
-                                if (kc < nch) {
-                                    const float f = __ldcg(pool + rec + (5 + kc) * H + jj);
-                                    const float ck = __ldcg(pool + I[4 + 2 * kc] + H + jj);
-                                    gf = chat * ck * f * (1.f - f);
-                                    pool[I[5 + 2 * kc] + H + jj] = chat * f;
-                                }
-                                g[4 + kc] = gf;
-                                gfs += gf;
-                            }
-                            g[3] = gfs;
-                            atomicAdd(db + 3, gfs);
+            for (int ci = tid; ci < UMAX * NB; ci += NTH) {
+                const int uu = ci / NB, n = ci % NB, jj = lc + uu * P.n_g;
+                if (n >= nb || jj >= H) continue;
+                const uint32_t* I = chunk + ipos[n];
+                const float* cv = cin + (n * UMAX + uu) * CINMAX;
+                const float dh = cv[0], dc = cv[1], c = cv[2];
+                const float th = tanhf(c);
+                float* g = gb + (uu * NB + n) * GO;
+                float* db = dbias + uu * 4;
+                if constexpr (BIN || CS) {
+                    const float i = cv[3], o = cv[4], uv = cv[5];
+                    const float dov = dh * th;
+                    const float chat = dc + dh * o * (1.f - th * th);
+                    const float gi = chat * uv * i * (1.f - i), go = dov * o * (1.f - o), gu = chat * i * (1.f - uv * uv);
+                    g[0] = gi; g[1] = go; g[2] = gu;
+                    atomicAdd(db + 0, gi); atomicAdd(db + 1, go); atomicAdd(db + 2, gu);
+                    if constexpr (BIN) {
+                        if (kindB) {
+                            const float fl = cv[6], fr = cv[7], cl = cv[8], cr = cv[9];
+                            const float gfl = chat * cl * fl * (1.f - fl), gfr = chat * cr * fr * (1.f - fr);
+                            pool[I[4] + H + jj] = chat * fl;     // dc of the left child (unique parent)
+                            pool[I[6] + H + jj] = chat * fr;
+                            g[3] = gfl; g[4] = gfr;
+                            atomicAdd(db + 3, gfl + gfr);
                         }
                     } else {
-                        const float i = __ldcg(pool + rec + 2 * H + jj), f = __ldcg(pool + rec + 3 * H + jj),
-                                    o = __ldcg(pool + rec + 4 * H + jj), gg = __ldcg(pool + rec + 5 * H + jj);
-                        const uint32_t prv = I[4], padj = I[5];
-                        const float cp = prv != NONE ? __ldcg(pool + prv + H + jj) : 0.f;
-                        const float dov = dh * th;
-                        const float chat = dc + dh * o * (1.f - th * th);
-                        g[0] = chat * gg * i * (1.f - i);
-                        g[1] = chat * cp * f * (1.f - f);
-                        g[2] = dov * o * (1.f - o);
-                        g[3] = chat * i * (1.f - gg * gg);
-                        if (prv != NONE) pool[padj + H + jj] = chat * f;
+                        const int nch = (int)(I[0] >> 8);
+                        float gfs = 0.f;
 #pragma unroll
-                        for (int k = 0; k < 4; ++k) atomicAdd(db + k, g[k]);
+                        for (int kc = 0; kc < CHMAX; ++kc) {
+                            float gf = 0.f;
+                            if (kc < nch) {
+                                const float f = cv[6 + kc], ck = cv[6 + CHMAX + kc];
+                                gf = chat * ck * f * (1.f - f);
+                                pool[I[5 + 2 * kc] + H + jj] = chat * f;
+                            }
+                            g[4 + kc] = gf;
+                            gfs += gf;
+                        }
+                        g[3] = gfs;
+                        atomicAdd(db + 3, gfs);
                     }
+                } else {
+                    const float i = cv[3], f = cv[4], o = cv[5], gg = cv[6], cp = cv[7];
+                    const uint32_t prv = I[4], padj = I[5];
+                    const float dov = dh * th;
+                    const float chat = dc + dh * o * (1.f - th * th);
+                    g[0] = chat * gg * i * (1.f - i);
+                    g[1] = chat * cp * f * (1.f - f);
+                    g[2] = dov * o * (1.f - o);
+                    g[3] = chat * i * (1.f - gg * gg);
+                    if (prv != NONE) pool[padj + H + jj] = chat * f;
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) atomicAdd(db + k, g[k]);
                 }
             }
             __syncthreads();
             // ---- in-register outer products (dW, L104) and transposed products (L94, fn4), FFMA2 ----
             if (unit_ok) {
+#pragma unroll 2
                 for (int n = 0; n < nb; ++n) {
                     const uint32_t* I = chunk + ipos[n];
-                    const float* g = gb + (u * NBMAX + n) * GO;
+                    const float* g = gb + (u * NB + n) * GO;
                     if (kindB) {
                         if constexpr (BIN) {
                             const float* x = xs + n * LB::KP;
