@@ -258,8 +258,7 @@ def main():
     for k in range(e2e_steps):
         g = batches[k % N_BATCHES]
         s = m.build_script(g)                       # host: super-graph, levels, schedule, encode
-        h2d += s.info()["n_words"] * 4
-        s.upload()                                   # one pinned H2D copy (L169)
+        h2d += s.info()["n_words"] * 4               # staged by the call below: one pinned H2D copy (L169)
         if world == 1:
             m.fwd_bwd_sgd(s, inputs, d_inputs, lr=lr, weight_decay=wd)
         else:

@@ -60,13 +60,24 @@ struct vpps_model_s {
     cudaEvent_t t_before = nullptr, t_after = nullptr;
     uint64_t* prof = nullptr;
     int64_t prof_stride = 0;
+    // Pre-allocated staging ring for per-batch scripts: a pinned host buffer and a
+    // device buffer per slot; a slot is reused once the kernel that last read it has finished.
+    struct Slot {
+        uint32_t* h = nullptr;
+        uint32_t* d = nullptr;
+        size_t cap = 0;
+        cudaEvent_t done = nullptr;
+        bool used = false;
+    };
+    static constexpr int kSlots = 3;
+    Slot ring[kSlots];
+    int next_slot = 0;
 };
 
 struct vpps_script_s {
     vpps_model model = nullptr;
     Script s;
-    uint32_t* d_words = nullptr;
-    uint32_t* h_pinned = nullptr;
+    uint32_t* d_words = nullptr;   // dedicated device copy after vpps_upload_script (resident script)
     bool uploaded = false;
 };
 
@@ -119,7 +130,6 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
         if (prop.major != 10) return fail(VPPS_E_INVALID, "libvpps is built for sm_100a (B200) only");
         if (n_sm == 0) n_sm = prop.multiProcessorCount;
         if (n_sm > prop.multiProcessorCount) return fail(VPPS_E_INVALID, "n_sm exceeds the device's SM count");
-        if (o.groups != 1) return fail(VPPS_E_INVALID, "replica groups > 1 are plan-only in v1");
     } else if (n_sm == 0) {
         n_sm = 148;
     }
@@ -220,12 +230,6 @@ vpps_status vpps_build_script(vpps_model m, const vpps_batch* batch, vpps_script
     // the input table's row count is not known here; token range is re-checked against it at run time
     const int rc = build_script(m->plan, b, INT64_MAX, &s->s, &err);
     if (rc != 0) return fail(rc == -4 ? VPPS_E_GRAPH : VPPS_E_INVALID, err);
-    if (!m->plan_only) {
-        const size_t bytes = s->s.words.size() * sizeof(uint32_t);
-        CK(cudaMallocHost(&s->h_pinned, bytes));                 // pinned staging (L169)
-        std::memcpy(s->h_pinned, s->s.words.data(), bytes);
-        CK(cudaMalloc(&s->d_words, bytes));
-    }
     *out = s.release();
     return VPPS_OK;
 }
@@ -255,9 +259,36 @@ vpps_status vpps_script_info_get(vpps_script s, vpps_script_info* info) {
 vpps_status vpps_upload_script(vpps_script s, void* stream) {
     if (!s) return fail(VPPS_E_INVALID, "null script");
     if (s->model->plan_only) return fail(VPPS_E_STATE, "plan-only model");
-    CK(cudaMemcpyAsync(s->d_words, s->h_pinned, s->s.words.size() * sizeof(uint32_t), cudaMemcpyHostToDevice,
-                       (cudaStream_t)stream));
+    if (s->uploaded) return VPPS_OK;
+    const size_t bytes = s->s.words.size() * sizeof(uint32_t);
+    CK(cudaMalloc(&s->d_words, bytes));
+    CK(cudaMemcpyAsync(s->d_words, s->s.words.data(), bytes, cudaMemcpyHostToDevice, (cudaStream_t)stream));
+    CK(cudaStreamSynchronize((cudaStream_t)stream));     // pageable source: complete before returning
     s->uploaded = true;
+    return VPPS_OK;
+}
+
+// Stage a non-resident script through the next ring slot: wait until the kernel that last read the
+// slot is done, copy the words into the slot's pinned buffer, one H2D copy (L169).
+static vpps_status stage_script(vpps_model m, vpps_script s, cudaStream_t st, int* slot_out,
+                                const uint32_t** dwords) {
+    const int k = m->next_slot;
+    m->next_slot = (k + 1) % vpps_model_s::kSlots;
+    vpps_model_s::Slot& sl = m->ring[k];
+    const size_t n = s->s.words.size();
+    if (!sl.done) CK(cudaEventCreateWithFlags(&sl.done, cudaEventDisableTiming));
+    if (sl.used) CK(cudaEventSynchronize(sl.done));
+    if (n > sl.cap) {
+        if (sl.h) CK(cudaFreeHost(sl.h));
+        if (sl.d) CK(cudaFree(sl.d));
+        sl.cap = n + n / 2 + 1024;
+        CK(cudaMallocHost(&sl.h, sl.cap * sizeof(uint32_t)));
+        CK(cudaMalloc(&sl.d, sl.cap * sizeof(uint32_t)));
+    }
+    std::memcpy(sl.h, s->s.words.data(), n * sizeof(uint32_t));
+    CK(cudaMemcpyAsync(sl.d, sl.h, n * sizeof(uint32_t), cudaMemcpyHostToDevice, st));
+    *slot_out = k;
+    *dwords = sl.d;
     return VPPS_OK;
 }
 
@@ -279,11 +310,14 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         m->pool_cap = cap;
     }
     m->last_pool_words = s->s.pool_words;
+    int ring_slot = -1;
+    const uint32_t* dwords = s->d_words;
     if (!s->uploaded) {
-        vpps_status r = vpps_upload_script(s, stream_);
+        vpps_status r = stage_script(m, s, st, &ring_slot, &dwords);
         if (r != VPPS_OK) return r;
     }
     CK(cudaMemsetAsync(m->pool, 0, s->s.zero_words * sizeof(float), st));
+    if (m->plan.G > 1) CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));
     if (d_inputs) CK(cudaMemsetAsync(d_inputs, 0, (size_t)n_rows * m->plan.E * sizeof(float), st));
     KParams kp{};
     kp.params = m->params;
@@ -291,10 +325,11 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     kp.inputs = inputs;
     kp.d_inputs = d_inputs;
     kp.pool = m->pool;
-    kp.script = s->d_words;
+    kp.script = dwords;
     for (size_t i = 0; i < m->offsets.size() && i < 8; ++i) kp.off[i] = m->offsets[i];
     kp.n_g = m->plan.n_g;
     kp.n_act = m->plan.n_act;
+    kp.G = m->plan.G;
     kp.C = m->plan.C;
     kp.mode = mode;
     kp.loss_word = s->s.loss_word;
@@ -308,6 +343,10 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     if (m->t_before) CK(cudaEventRecord(m->t_before, st));
     CK(cudaLaunchCooperativeKernel(m->var->fn, dim3(m->plan.n_cta), dim3(256), args, m->smem, st));
     if (m->t_after) CK(cudaEventRecord(m->t_after, st));
+    if (ring_slot >= 0) {
+        CK(cudaEventRecord(m->ring[ring_slot].done, st));
+        m->ring[ring_slot].used = true;
+    }
     const int slot = (int)(m->passes & 1);
     CK(cudaMemcpyAsync(m->h_loss + slot, m->pool + s->s.loss_word, sizeof(float), cudaMemcpyDeviceToHost, st));
     CK(cudaEventRecord(m->ev[slot], st));
@@ -377,7 +416,6 @@ vpps_status vpps_pool_ptr(vpps_model m, float** pool, int64_t* pool_words) {
 void vpps_destroy_script(vpps_script s) {
     if (!s) return;
     if (s->d_words) cudaFree(s->d_words);
-    if (s->h_pinned) cudaFreeHost(s->h_pinned);
     delete s;
 }
 
@@ -387,6 +425,11 @@ void vpps_destroy_model(vpps_model m) {
     if (m->h_loss) cudaFreeHost(m->h_loss);
     for (cudaEvent_t e : m->ev)
         if (e) cudaEventDestroy(e);
+    for (auto& sl : m->ring) {
+        if (sl.done) cudaEventSynchronize(sl.done), cudaEventDestroy(sl.done);
+        if (sl.h) cudaFreeHost(sl.h);
+        if (sl.d) cudaFree(sl.d);
+    }
     delete m;
 }
 

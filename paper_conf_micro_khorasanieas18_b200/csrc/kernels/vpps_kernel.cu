@@ -954,39 +954,55 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
     if (prof && tid == 0) prof[1] = gtimer();
     const bool sgd = P.mode == 1;
     float* gout = P.grads;
-    auto put = [&](int64_t idx, float w, float dw) {
-        if (sgd) P.params[idx] = w - P.lr * (dw + P.wd * w);
-        else gout[idx] = dw;
-    };
-    if (unit_ok) {
+    // every parameter element this CTA owns: f(flat index, cached weight, accumulated gradient)
+    auto visit = [&](auto&& f) {
+        if (unit_ok) {
 #pragma unroll
-        for (int r = 0; r < RA; ++r)
+            for (int r = 0; r < RA; ++r)
 #pragma unroll
-            for (int t = 0; t < LA::NT; ++t)
+                for (int t = 0; t < LA::NT; ++t)
 #pragma unroll
-                for (int q = 0; q < LA::CG; ++q) {
-                    const int col = LA::CG * (tu + TU * t) + q;
-                    if (col < KA) put(idxA(r, col), wa[r][t * LA::CG + q], dwa[r][t * LA::CG + q]);
-                }
-        if constexpr (BIN) {
-#pragma unroll
-            for (int r = 0; r < RB; ++r)
-#pragma unroll
-                for (int t = 0; t < LB::NT; ++t)
-#pragma unroll
-                    for (int q = 0; q < LB::CG; ++q) {
-                        const int col = LB::CG * (tu + TU * t) + q;
-                        if (col < KB) put(idxB(r, col), wb[r][t * LB::CG + q], dwb[r][t * LB::CG + q]);
+                    for (int q = 0; q < LA::CG; ++q) {
+                        const int col = LA::CG * (tu + TU * t) + q;
+                        if (col < KA) f(idxA(r, col), wa[r][t * LA::CG + q], dwa[r][t * LA::CG + q]);
                     }
+            if constexpr (BIN) {
+#pragma unroll
+                for (int r = 0; r < RB; ++r)
+#pragma unroll
+                    for (int t = 0; t < LB::NT; ++t)
+#pragma unroll
+                        for (int q = 0; q < LB::CG; ++q) {
+                            const int col = LB::CG * (tu + TU * t) + q;
+                            if (col < KB) f(idxB(r, col), wb[r][t * LB::CG + q], dwb[r][t * LB::CG + q]);
+                        }
+            }
         }
-    }
-    if (tid < UMAX * 4) {
-        const int uu = tid / 4, k = tid % 4, jj = lc + uu * P.n_g;
-        if (jj < H) put((LS || k < 3) ? off[bias_m0] + k * H + jj : off[6] + jj, bias[tid], dbias[tid]);
-    }
-    if (holds_head) {
-        for (int i = tid; i < C * H; i += NTH) put(off[wout_m] + i, Wo[i], dWo[i]);
-        for (int i = tid; i < C; i += NTH) put(off[bout_m] + i, bo[i], dbo[i]);
+        if (tid < UMAX * 4) {
+            const int uu = tid / 4, k = tid % 4, jj = lc + uu * P.n_g;
+            if (jj < H) f((LS || k < 3) ? off[bias_m0] + k * H + jj : off[6] + jj, bias[tid], dbias[tid]);
+        }
+        if (holds_head) {
+            for (int i = tid; i < C * H; i += NTH) f(off[wout_m] + i, Wo[i], dWo[i]);
+            for (int i = tid; i < C; i += NTH) f(off[bout_m] + i, bo[i], dbo[i]);
+        }
+    };
+    if (P.G == 1) {
+        // one replica: each element has exactly one owner -> plain stores
+        visit([&](int64_t idx, float w, float dw) {
+            if (sgd) P.params[idx] = w - P.lr * (dw + P.wd * w);
+            else gout[idx] = dw;
+        });
+    } else {
+        // G replicas: sum the partial gradients of all groups in L2 (grads zeroed by the host)...
+        visit([&](int64_t idx, float, float dw) { atomicAdd(gout + idx, dw); });
+        if (sgd) {
+            // ...then, after a barrier over every CTA, group 0's owner applies the update
+            bar_signal(bar, nullptr);
+            bar_wait(bar, (unsigned)(P.G * P.n_act), nullptr);
+            if (grp == 0)
+                visit([&](int64_t idx, float w, float) { P.params[idx] = w - P.lr * (__ldcg(gout + idx) + P.wd * w); });
+        }
     }
 }
 
@@ -1011,7 +1027,9 @@ __global__ void sgd_kernel(float* __restrict__ p, const float* __restrict__ g, i
     {CELL, H, E, U, (const void*)&dev::vpps_fb<CELL, H, E, U>, &dev::Cfg<CELL, H, E, U>::smem_bytes}
 
 static const Variant kVariants[] = {
-    VPPS_VARIANT(dev::CELL_BINARY, 256, 256, 2),    // target: binary Tree-LSTM H = E = 256 on 148 SMs
+    VPPS_VARIANT(dev::CELL_BINARY, 256, 256, 2),    // target: binary Tree-LSTM H = E = 256 on 148 SMs, G = 1
+    VPPS_VARIANT(dev::CELL_BINARY, 256, 256, 4),    // ... G = 2 replica groups of 74 CTAs
+    VPPS_VARIANT(dev::CELL_BINARY, 256, 256, 8),    // ... G = 4 replica groups of 37 CTAs
     VPPS_VARIANT(dev::CELL_BINARY, 128, 128, 1),
     VPPS_VARIANT(dev::CELL_BINARY, 32, 32, 1),
     VPPS_VARIANT(dev::CELL_CHILDSUM, 128, 128, 1),  // config 2

@@ -14,6 +14,7 @@ struct KParams {
     const uint32_t* script; // encoded script (SPEC §E)
     int64_t off[8];         // parameter offsets in floats
     int32_t n_g, n_act, C, mode;   // mode 0: write grads; 1: fused SGD update
+    int32_t G;                     // replica groups (SPEC P1); G > 1 sums gradients across groups
     int64_t loss_word;
     float lr, wd;
     uint64_t* prof;         // optional globaltimer trace (vpps_set_profile_buffer), or nullptr

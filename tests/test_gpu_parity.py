@@ -20,13 +20,13 @@ def _vpps():
     return vpps
 
 
-def run_case(cell, H, E, C, graphs, V, seed=0, want_dx=True, sgd=None):
+def run_case(cell, H, E, C, graphs, V, seed=0, want_dx=True, sgd=None, groups=1):
     vpps = _vpps()
     rng = np.random.default_rng(seed)
     shapes = vpps.param_shapes(cell, H, E, C)
     P = synth.init_params(shapes, rng)
     X = synth.input_table(rng, V, E)
-    m = vpps.Model(cell, H, E, C, device=0)
+    m = vpps.Model(cell, H, E, C, device=0, groups=groups)
     dev = torch.device("cuda:0")
     params = torch.zeros(m.n_floats, dtype=torch.float32, device=dev)
     grads = torch.full_like(params, float("nan"))
@@ -50,8 +50,8 @@ def rel(a, b):
     return float(np.abs(np.asarray(a, np.float64) - b).max() / max(np.abs(b).max(), 1e-30))
 
 
-def check(cell, H, E, C, graphs, V, seed=0, want_dx=True):
-    m, P, X, loss, params, grads, dX = run_case(cell, H, E, C, graphs, V, seed, want_dx)
+def check(cell, H, E, C, graphs, V, seed=0, want_dx=True, groups=1):
+    m, P, X, loss, params, grads, dX = run_case(cell, H, E, C, graphs, V, seed, want_dx, groups=groups)
     lo, Go, dXo = M.forward_backward(cell, P, X, graphs, H)
     assert abs(loss - lo) <= TOL * abs(lo), (loss, lo)
     gv = m.views(grads.cpu())
@@ -75,6 +75,25 @@ def test_binary_target_config():
     """TGT: binary Tree-LSTM H = E = 256, batch 16 SST-shaped trees (5-50 leaves), 148 SMs."""
     graphs = synth.config_batch("tgt", 0)
     check("binary", 256, 256, 5, graphs, 4096, seed=3)
+
+
+@pytest.mark.parametrize("groups", [2, 4])
+def test_binary_target_replica_groups(groups):
+    """SPEC P1 replica groups: nodes spread over G groups, gradients summed across groups in-kernel."""
+    check("binary", 256, 256, 5, synth.config_batch("tgt", 3), 4096, seed=5, groups=groups)
+
+
+@pytest.mark.parametrize("groups", [1, 2, 4])
+def test_fused_sgd_target_groups(groups):
+    graphs = synth.config_batch("tgt", 4)
+    lr, wd = 0.05, 1e-3
+    m, P, X, loss, params, grads, dX = run_case("binary", 256, 256, 5, graphs, 4096, seed=6, sgd=(lr, wd),
+                                                groups=groups)
+    lo, Go, _ = M.forward_backward("binary", P, X, graphs, 256)
+    Pn = M.sgd(P, Go, lr, wd)
+    pv = m.views(params.cpu())
+    for name, _ in m.shapes:
+        assert rel(pv[name].numpy() - P[name], Pn[name] - P[name]) <= 1e-3, name
 
 
 def test_binary_target_other_batches():

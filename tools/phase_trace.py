@@ -21,6 +21,8 @@ def main():
     ap.add_argument("--batch-idx", type=int, default=0)
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--config", default="tgt")
+    ap.add_argument("--groups", type=int, default=1)
+    ap.add_argument("--quiet", action="store_true")
     args = ap.parse_args()
     import torch
     import synth
@@ -30,7 +32,7 @@ def main():
     rng = np.random.default_rng(0)
     shapes = vpps.param_shapes(cell, H, E, C)
     P = synth.init_params(shapes, rng)
-    m = vpps.Model(cell, H, E, C)
+    m = vpps.Model(cell, H, E, C, groups=args.groups)
     params = torch.zeros(m.n_floats, device="cuda")
     grads = torch.zeros_like(params)
     for n, _ in shapes:
@@ -54,8 +56,12 @@ def main():
         ev[1].record()
     torch.cuda.synchronize()
     kernel_us = ev[0].elapsed_time(ev[1]) * 1e3
-    t = buf.cpu().numpy()[:n_act].astype(np.float64)
-    t0 = t[:, 0].min()
+    n_g = m.plan_info()["n_g"]
+    raw = buf.cpu().numpy().astype(np.float64)
+    rows = [c for c in range(n_cta) if c % n_g < n_act]
+    t = raw[rows]
+    t[t == 0] = np.nan                       # stamps of phases a group did not take part in
+    t0 = np.nanmin(t[:, 0])
     t = t - t0
     L = (nbar - 1) // 2
     # node counts per phase from the script words (cell/head instructions of stream 0)
@@ -64,19 +70,23 @@ def main():
     lv = ref["levels"]
     counts = [sum(1 for x in lv if x == (p if p <= L else 2 * L + 1 - p)) for p in range(nbar + 1)]
     print(f"{args.config}: {len(graphs)} graphs, {info['n_nodes']} nodes, {nbar} barriers, kernel "
-          f"{kernel_us:.1f} us (event, incl. memsets), trace span {(t[:, 1].max()):.0f} ns")
+          f"{kernel_us:.1f} us (event, incl. memsets), trace span {np.nanmax(t[:, 1]):.0f} ns, groups {args.groups}")
     work_tot = bar_tot = 0.0
-    print(" phase  nodes   work_max   work_mean   barrier(last sig->last release)")
+    if not args.quiet:
+        print(" phase  nodes   work_max   work_mean   barrier(last sig->last release)")
     for p in range(nbar + 1):
         start = t[:, 0] if p == 0 else t[:, 4 + 3 * p]
         end = t[:, 1] if p == nbar else t[:, 2 + 3 * (p + 1)]
         w = end - start
         bl = 0.0
         if p >= 1:
-            bl = t[:, 2 + 3 * p + 2].max() - t[:, 2 + 3 * p].max()
-        work_tot += w.max()
+            bl = np.nanmax(t[:, 2 + 3 * p + 2]) - np.nanmax(t[:, 2 + 3 * p])
+        wmax = np.nanmax(w) if np.any(~np.isnan(w)) else 0.0
+        wmean = np.nanmean(w) if np.any(~np.isnan(w)) else 0.0
+        work_tot += wmax
         bar_tot += bl
-        print(f" {p:5d} {counts[p]:6d} {w.max()/1e3:9.2f}us {w.mean()/1e3:9.2f}us {bl/1e3:9.2f}us")
+        if not args.quiet:
+            print(f" {p:5d} {counts[p]:6d} {wmax/1e3:9.2f}us {wmean/1e3:9.2f}us {bl/1e3:9.2f}us")
     print(f"sum work_max {work_tot/1e3:.1f} us, sum barrier {bar_tot/1e3:.1f} us")
 
 
