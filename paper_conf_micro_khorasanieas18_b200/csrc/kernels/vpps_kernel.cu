@@ -105,10 +105,12 @@ struct Cfg {
     static constexpr int O_CSLOT = O_IPOS + NB;
     static constexpr int O_BST = O_CSLOT + NB;
     static constexpr int O_CREC = O_BST + 4;
-    static constexpr int O_ZS = a4(O_CREC + cmax(CHSLOT, 1));
-    static constexpr int O_HEAD = O_ZS + 8 * ZC;
-    static constexpr int ITER = ((NB + CHSLOT) * KPMAX / 4 + NTH - 1) / NTH;
+    static constexpr int O_MBAR = a4(O_CREC + cmax(CHSLOT, 1));     // one mbarrier (8-byte aligned)
+    static constexpr int O_ZS = O_MBAR + 4;
+    static constexpr int O_HEAD = O_ZS + NB * ZC;
     static constexpr int ITER2 = (NB * UMAX * CINMAX + NTH - 1) / NTH;
+    static_assert(UMAX * NB <= NTH && NB <= 32 && 32 % NB == 0, "one (unit, node) pair per thread");
+    static_assert(KPMAX >= H, "head rows are staged in the input rows");
     static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 2 * C + 8); }
 };
 
@@ -238,6 +240,33 @@ __device__ __forceinline__ float warp_max(float v) {
     return v;
 }
 
+// ---- TMA bulk copies global -> shared with an mbarrier transaction count (sm_90+) ----
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect(uint64_t* b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+    asm volatile(
+        "{\n .reg .pred p;\n"
+        "VPPS_WAIT_%=:\n"
+        " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        " @!p bra VPPS_WAIT_%=;\n}" ::"r"(smem_u32(b)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* b) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(b))
+                 : "memory");
+}
+__device__ __forceinline__ void fence_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
+__device__ __forceinline__ void fence_async_shared() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
 __device__ __forceinline__ uint64_t gtimer() {
     uint64_t t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -334,6 +363,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
     int* bst = reinterpret_cast<int*>(smw + T::O_BST);
     uint32_t* crec = smw + T::O_CREC;
     float* zs = sm + T::O_ZS;
+    uint64_t* mbar = reinterpret_cast<uint64_t*>(smw + T::O_MBAR);
+    uint32_t mphase = 0;
     const int C = P.C;
     float* Wo = sm + T::O_HEAD;
     float* dWo = Wo + C * H;
@@ -411,8 +442,34 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
     }
 
     uint64_t* prof = P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
+    // section clocks (thread 0, trace only): 0 decode, 1 staging, 2 matvec, 3 cell, 4 cell-bwd,
+    // 5 outer/transposed, 6 heads, 7 signal, 8 wait, 9 other
+    uint64_t sec[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
+    uint64_t sec_last = 0;
+    int sec_cur = 9;
+    auto mark = [&](int k) {
+        if (prof && tid == 0) {
+            const uint64_t now = clock64();
+            const uint64_t d = now - sec_last;
+            switch (sec_cur) {
+                case 0: sec[0] += d; break;
+                case 1: sec[1] += d; break;
+                case 2: sec[2] += d; break;
+                case 3: sec[3] += d; break;
+                case 4: sec[4] += d; break;
+                case 5: sec[5] += d; break;
+                case 6: sec[6] += d; break;
+                case 7: sec[7] += d; break;
+                case 8: sec[8] += d; break;
+                default: sec[9] += d; break;
+            }
+            sec_cur = k;
+            sec_last = now;
+        }
+    };
+    if (tid == 0) mbar_init(mbar, 1);
     __syncthreads();
-    if (prof && tid == 0) prof[0] = gtimer();
+    if (prof && tid == 0) { prof[0] = gtimer(); sec_last = clock64(); }
 
     // ---------------- script interpretation (L171-177) ---------------------------------------------
     uint32_t cbase = s0;
@@ -436,171 +493,131 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
         if (pos + 640 > cbase + CHUNK && cbase + CHUNK < s1) refill(pos);
         const uint32_t pre = chunk[pos - cbase];
         const uint32_t op = pre & 0xFF;
-        if (op == OP_S) { bar_signal(bar + (pre >> 8), prof ? prof + 2 + 3 * (pre >> 8) : nullptr); ++pos; continue; }
+        if (op == OP_S) {
+            mark(7);
+            bar_signal(bar + (pre >> 8), prof ? prof + 2 + 3 * (pre >> 8) : nullptr);
+            ++pos;
+            continue;
+        }
         if (op == OP_W) {
+            mark(8);
             bar_wait(bar + (pre >> 8), target[pre >> 8], prof ? prof + 2 + 3 * (pre >> 8) : nullptr);
             ++pos;
             continue;
         }
-        // ---- decode (warp 0): a batch of up to NB consecutive instructions with this opcode ----
+        // ---- decode (warp 0): a batch of up to NB consecutive instructions with this opcode, then the
+        //      batch's input rows are fetched by TMA bulk copies (cp.async.bulk) into shared memory ----
+        const bool is_head = (op == OP_HEAD_F || op == OP_HEAD_B);
+        const bool fwd = (op & 1) == 0;
+        const bool kindB = BIN && (op == OP_INT_F || op == OP_INT_B);
+        const int KP = is_head ? LA::KP : (kindB ? LB::KP : LA::KP);
+        fence_async_shared();            // our generic reads of the staging buffers precede the next async writes
         __syncthreads();
+        mark(0);
         if (warp == 0) {
             const uint32_t lim = min(s1, cbase + (uint32_t)CHUNK);
+            int nbw = 0, usedw = 0;
             if (!(op == OP_CS_F || op == OP_CS_B)) {
                 const uint32_t sz = (uint32_t)instr_words(pre);
-                int nb = 0;
-                for (int base = 0; base < NB; base += 32) {
-                    const int n = base + lane;
-                    const uint32_t q = pos + (uint32_t)n * sz;
-                    const bool ok = n < NB && q + sz <= lim && (chunk[q - cbase] & 0xFF) == op;
-                    const unsigned m = __ballot_sync(FULL, ok);
-                    const int cnt = (m == FULL) ? 32 : (__ffs(~m) - 1);
-                    if (lane < cnt) ipos[n] = (int)(q - cbase);
-                    nb += cnt;
-                    if (cnt < 32) break;
+                const uint32_t q = pos + (uint32_t)lane * sz;
+                const bool ok = lane < NB && q + sz <= lim && (chunk[q - cbase] & 0xFF) == op;
+                const unsigned msk = __ballot_sync(FULL, ok);
+                nbw = (msk == FULL) ? 32 : (__ffs(~msk) - 1);
+                if (lane < nbw) ipos[lane] = (int)(q - cbase);
+                if (lane == 0) { bst[0] = nbw; bst[1] = (int)(pos + nbw * sz); bst[2] = 0; }
+            } else {
+                if (lane == 0) {
+                    uint32_t p = pos;
+                    while (p < lim && nbw < NB) {
+                        const uint32_t w = chunk[p - cbase];
+                        if ((w & 0xFF) != op) break;
+                        const int sz = instr_words(w);
+                        if (p + sz > lim || usedw + (int)(w >> 8) > T::CHSLOT) break;
+                        ipos[nbw] = (int)(p - cbase);
+                        cslot[nbw] = usedw;
+                        const uint32_t* I = chunk + (p - cbase);
+                        for (int k = 0; k < (int)(w >> 8); ++k)
+                            crec[usedw + k] = (op == OP_CS_F) ? I[3 + k] : I[4 + 2 * k];
+                        usedw += (int)(w >> 8);
+                        ++nbw;
+                        p += sz;
+                    }
+                    bst[0] = nbw; bst[1] = (int)p; bst[2] = usedw;
                 }
-                if (lane == 0) { bst[0] = nb; bst[1] = (int)(pos + nb * sz); bst[2] = 0; }
-            } else if (lane == 0) {
-                int nb = 0, used = 0;
-                uint32_t p = pos;
-                while (p < lim && nb < NB) {
-                    const uint32_t w = chunk[p - cbase];
-                    if ((w & 0xFF) != op) break;
-                    const int sz = instr_words(w);
-                    if (p + sz > lim || used + (int)(w >> 8) > T::CHSLOT) break;
-                    ipos[nb] = (int)(p - cbase);
-                    cslot[nb] = used;
-                    const uint32_t* I = chunk + (p - cbase);
-                    for (int k = 0; k < (int)(w >> 8); ++k) crec[used + k] = (op == OP_CS_F) ? I[3 + k] : I[4 + 2 * k];
-                    used += (int)(w >> 8);
-                    ++nb;
-                    p += sz;
-                }
-                bst[0] = nb; bst[1] = (int)p; bst[2] = used;
+                nbw = __shfl_sync(FULL, nbw, 0);
+                usedw = __shfl_sync(FULL, usedw, 0);
             }
+            __syncwarp();
+            // segments of node n = lane: (source, destination offset in its row, bytes)
+            const bool issue = !is_head || holds_head;
+            const float* src0 = nullptr; const float* src1 = nullptr;
+            int off0 = 0, off1 = 0;
+            uint32_t b0 = 0, b1 = 0;
+            if (issue && lane < nbw) {
+                const uint32_t* I = chunk + ipos[lane];
+                if (is_head) {
+                    src0 = pool + I[2]; b0 = H * 4;                                       // h of the cell
+                } else if constexpr (BIN) {
+                    if (!kindB) {
+                        src0 = inputs + (int64_t)(fwd ? I[2] : I[3]) * E; b0 = E * 4;
+                    } else {
+                        src0 = pool + (fwd ? I[2] : I[3]); b0 = H * 4;                    // [h_l; h_r]
+                        src1 = pool + (fwd ? I[3] : I[5]); b1 = H * 4; off1 = H;
+                    }
+                } else if constexpr (LS) {
+                    const uint32_t tok = fwd ? I[2] : I[3], prv = fwd ? I[3] : I[4];
+                    src0 = inputs + (int64_t)tok * E; b0 = E * 4;
+                    if (prv != NONE) { src1 = pool + prv; b1 = H * 4; off1 = E; }
+                } else {
+                    const uint32_t tok = fwd ? I[2] : I[3];
+                    if (tok != NONE) { src0 = inputs + (int64_t)tok * E; b0 = E * 4; }
+                }
+            }
+            uint32_t bytes = b0 + b1;
+            if (CS && issue && !is_head)
+                for (int k = lane; k < usedw; k += 32) bytes += H * 4;
+#pragma unroll
+            for (int s = 16; s >= 1; s >>= 1) bytes += __shfl_xor_sync(FULL, bytes, s);
+            fence_async_global();        // rows written by other CTAs (acquired at the last wait) -> async proxy
+            if (lane == 0) mbar_arrive_expect(mbar, bytes);
+            __syncwarp();
+            if (b0) bulk_g2s(xs + lane * KP + off0, src0, b0, mbar);
+            if (b1) bulk_g2s(xs + lane * KP + off1, src1, b1, mbar);
+            if (CS && issue && !is_head)
+                for (int k = lane; k < usedw; k += 32) bulk_g2s(chs + k * KP + E, pool + crec[k], H * 4, mbar);
         }
         __syncthreads();
         const int nb = bst[0];
         const uint32_t p = (uint32_t)bst[1];
 
-        // ---- loss heads (L42), one warp per head, on the CTA that holds W_out ----
-        if (op == OP_HEAD_F || op == OP_HEAD_B) {
-            if (holds_head) {
-                for (int n = warp; n < nb; n += NTH / 32) {
+        mark(1);
+        // ---- while the bulk copies fly: zero the parts of the rows no copy writes and load every
+        //      per-(unit, node) cell operand (one round trip) ----
+        if (!is_head) {
+            const int Kk = kindB ? KB : KA;
+            if (KP > Kk || LS || CS) {           // padding beyond K, absent h_prev (t = 0), absent word
+                const int q4 = KP / 4;
+                for (int i = tid; i < nb * q4; i += NTH) {
+                    const int n = i / q4, c = (i - n * q4) * 4;
                     const uint32_t* I = chunk + ipos[n];
-                    const uint32_t rec = I[1], crc = I[2];
-                    float4 hv[HT];
-#pragma unroll
-                    for (int t = 0; t < HT; ++t) {
-                        const int k = 4 * (lane + 32 * t);
-                        hv[t] = k < H ? ld4cg(pool + crc + k) : f4zero();
-                    }
-                    float* z = zs + warp * ZC;
-                    if (op == OP_HEAD_F) {
-                        const int y = (int)I[3];
-                        for (int c = 0; c < C; ++c) {
-                            float s = 0.f;
-#pragma unroll
-                            for (int t = 0; t < HT; ++t) {
-                                const int k = 4 * (lane + 32 * t);
-                                if (k < H) {
-                                    const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
-                                    s += w4.x * hv[t].x + w4.y * hv[t].y + w4.z * hv[t].z + w4.w * hv[t].w;
-                                }
-                            }
-                            s = warp_sum(s);
-                            if (lane == 0) z[c] = s + bo[c];
-                        }
-                        __syncwarp();
-                        const float zl = lane < C ? z[lane] : -INFINITY;
-                        const float m = warp_max(zl);
-                        const float se = warp_sum(lane < C ? expf(zl - m) : 0.f);
-                        const float lse = m + logf(se);
-                        if (lane < C) pool[rec + lane] = expf(zl - lse);
-                        const float zy = __shfl_sync(FULL, zl, y);
-                        if (lane == 0) {
-                            pool[rec + C] = lse - zy;
-                            atomicAdd(pool + P.loss_word, lse - zy);   // aggregated loss node (L205)
-                        }
-                    } else {
-                        const uint32_t cadj = I[3];
-                        const int y = (int)I[4];
-                        const float dz = lane < C ? __ldcg(pool + rec + lane) - (lane == y ? 1.f : 0.f) : 0.f;
-                        if (lane < C) atomicAdd(dbo + lane, dz);
-                        float4 dh[HT];
-#pragma unroll
-                        for (int t = 0; t < HT; ++t) dh[t] = f4zero();
-                        for (int c = 0; c < C; ++c) {
-                            const float dzc = __shfl_sync(FULL, dz, c);
-#pragma unroll
-                            for (int t = 0; t < HT; ++t) {
-                                const int k = 4 * (lane + 32 * t);
-                                if (k < H) {
-                                    float* dw = dWo + c * H + k;
-                                    atomicAdd(dw + 0, dzc * hv[t].x); atomicAdd(dw + 1, dzc * hv[t].y);
-                                    atomicAdd(dw + 2, dzc * hv[t].z); atomicAdd(dw + 3, dzc * hv[t].w);
-                                    const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
-                                    dh[t].x += w4.x * dzc; dh[t].y += w4.y * dzc;
-                                    dh[t].z += w4.z * dzc; dh[t].w += w4.w * dzc;
-                                }
-                            }
-                        }
-#pragma unroll
-                        for (int t = 0; t < HT; ++t) {
-                            const int k = 4 * (lane + 32 * t);
-                            const float v4[4] = {dh[t].x, dh[t].y, dh[t].z, dh[t].w};
-                            if (k < H) red_add<4>(pool + cadj + k, v4);
+                    bool z = c >= Kk;
+                    if constexpr (LS) z = z || (c >= E && c < E + H && (fwd ? I[3] : I[4]) == NONE);
+                    if constexpr (CS) z = z || (c < E && (fwd ? I[2] : I[3]) == NONE);
+                    if (z) *reinterpret_cast<float4*>(xs + n * KP + c) = f4zero();
+                }
+                if constexpr (CS) {
+                    if (KP > E + H) {
+                        const int qp = (KP - E - H) / 4;
+                        for (int i = tid; i < bst[2] * qp; i += NTH) {
+                            const int r = i / qp, c = E + H + (i - r * qp) * 4;
+                            *reinterpret_cast<float4*>(chs + r * KP + c) = f4zero();
                         }
                     }
                 }
             }
-            pos = p;
-            continue;
-        }
-
-        const bool fwd = (op & 1) == 0;
-        const bool kindB = BIN && (op == OP_INT_F || op == OP_INT_B);
-        const int KP = kindB ? LB::KP : LA::KP;
-        // ---- one round trip: every input row and cell operand of the batch is loaded before the
-        //      first shared-memory store ----
-        {
-            const int q4 = KP / 4;
-            const int rows = nb + (CS ? bst[2] : 0);
-            const int total = rows * q4;
             const int ncin = n_cin(op);
             const int total2 = nb * UMAX * ncin;
-            float4 v[T::ITER];
             float s2[T::ITER2];
-#pragma unroll
-            for (int it = 0; it < T::ITER; ++it) {
-                const int i = tid + it * NTH;
-                const float* src = nullptr;
-                if (i < total) {
-                    const int n = i / q4, c = (i - n * q4) * 4;
-                    if (n < nb) {
-                        const uint32_t* I = chunk + ipos[n];
-                        if constexpr (BIN) {
-                            if (!kindB) {
-                                if (c < E) src = inputs + (int64_t)(fwd ? I[2] : I[3]) * E + c;
-                            } else {
-                                const uint32_t rl = fwd ? I[2] : I[3], rr = fwd ? I[3] : I[5];
-                                if (c < H) src = pool + rl + c;
-                                else if (c < 2 * H) src = pool + rr + (c - H);
-                            }
-                        } else if constexpr (LS) {
-                            const uint32_t tok = fwd ? I[2] : I[3], prv = fwd ? I[3] : I[4];
-                            if (c < E) src = inputs + (int64_t)tok * E + c;
-                            else if (c < E + H && prv != NONE) src = pool + prv + (c - E);
-                        } else {
-                            const uint32_t tok = fwd ? I[2] : I[3];
-                            if (c < E && tok != NONE) src = inputs + (int64_t)tok * E + c;
-                        }
-                    } else if (c >= E && c < E + H) {        // child-sum: a child's h row
-                        src = pool + crec[n - nb] + (c - E);
-                    }
-                }
-                v[it] = src ? ld4cg(src) : f4zero();
-            }
 #pragma unroll
             for (int it = 0; it < T::ITER2; ++it) {
                 const int i = tid + it * NTH;
@@ -613,15 +630,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                 s2[it] = src ? __ldcg(src) : 0.f;
             }
 #pragma unroll
-            for (int it = 0; it < T::ITER; ++it) {
-                const int i = tid + it * NTH;
-                if (i < total) {
-                    const int n = i / q4, c = (i - n * q4) * 4;
-                    float* dst = n < nb ? xs + n * KP + c : chs + (n - nb) * KP + c;
-                    *reinterpret_cast<float4*>(dst) = v[it];
-                }
-            }
-#pragma unroll
             for (int it = 0; it < T::ITER2; ++it) {
                 const int i = tid + it * NTH;
                 if (i < total2) {
@@ -630,8 +638,11 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                     cin[(n * UMAX + uu) * CINMAX + k] = s2[it];
                 }
             }
-            if constexpr (CS) {     // h~ = sum of the children's h (child-sum, [5] eq. 2)
-                __syncthreads();
+        }
+        mbar_wait(mbar, mphase);                // the batch's bulk copies have landed
+        mphase ^= 1;
+        if constexpr (CS) {                     // h~ = sum of the children's h (child-sum, [5] eq. 2)
+            if (!is_head) {
                 for (int i = tid; i < nb * (H / 4); i += NTH) {
                     const int n = i / (H / 4), c = E + (i - n * (H / 4)) * 4;
                     const int nch = (int)(chunk[ipos[n]] >> 8);
@@ -645,6 +656,74 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
             }
         }
         __syncthreads();
+
+        // ---- loss heads (L42) on the CTA that holds W_out; no two threads write the same element ----
+        if (is_head) {
+            mark(6);
+            if (holds_head) {
+                if (op == OP_HEAD_F) {
+                    for (int pi = warp; pi < nb * C; pi += NTH / 32) {      // z[n][c], one warp per pair
+                        const int n = pi / C, c = pi - n * C;
+                        float s = 0.f;
+                        for (int k = 4 * lane; k < H; k += 128) {
+                            const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                            const float4 h4 = *reinterpret_cast<const float4*>(xs + n * KP + k);
+                            s += w4.x * h4.x + w4.y * h4.y + w4.z * h4.z + w4.w * h4.w;
+                        }
+                        s = warp_sum(s);
+                        if (lane == 0) zs[n * ZC + c] = s + bo[c];
+                    }
+                    __syncthreads();
+                    for (int n = warp; n < nb; n += NTH / 32) {             // softmax-NLL, one warp per head
+                        const uint32_t* I = chunk + ipos[n];
+                        const uint32_t rec = I[1];
+                        const int y = (int)I[3];
+                        const float zl = lane < C ? zs[n * ZC + lane] : -INFINITY;
+                        const float m = warp_max(zl);
+                        const float se = warp_sum(lane < C ? expf(zl - m) : 0.f);
+                        const float lse = m + logf(se);
+                        if (lane < C) pool[rec + lane] = expf(zl - lse);
+                        const float zy = __shfl_sync(FULL, zl, y);
+                        if (lane == 0) {
+                            pool[rec + C] = lse - zy;
+                            atomicAdd(pool + P.loss_word, lse - zy);   // aggregated loss node (L205)
+                        }
+                    }
+                } else {
+                    for (int i = tid; i < nb * C; i += NTH) {              // dz = softmax - onehot(y)
+                        const int n = i / C, c = i - n * C;
+                        const uint32_t* I = chunk + ipos[n];
+                        zs[n * ZC + c] = __ldcg(pool + I[1] + c) - (c == (int)I[4] ? 1.f : 0.f);
+                    }
+                    __syncthreads();
+                    for (int c = tid; c < C; c += NTH) {
+                        float s = 0.f;
+                        for (int n = 0; n < nb; ++n) s += zs[n * ZC + c];
+                        dbo[c] += s;
+                    }
+                    for (int i = tid; i < C * H; i += NTH) {              // dW_out += dz h^T
+                        const int c = i / H, k = i - c * H;
+                        float s = 0.f;
+                        for (int n = 0; n < nb; ++n) s = fmaf(zs[n * ZC + c], xs[n * KP + k], s);
+                        dWo[i] += s;
+                    }
+                    for (int i = tid; i < nb * (H / 4); i += NTH) {       // dh = W_out^T dz -> the cell's dh
+                        const int n = i / (H / 4), k = (i - n * (H / 4)) * 4;
+                        float v4[4] = {0.f, 0.f, 0.f, 0.f};
+                        for (int c = 0; c < C; ++c) {
+                            const float dzc = zs[n * ZC + c];
+                            const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                            v4[0] = fmaf(w4.x, dzc, v4[0]); v4[1] = fmaf(w4.y, dzc, v4[1]);
+                            v4[2] = fmaf(w4.z, dzc, v4[2]); v4[3] = fmaf(w4.w, dzc, v4[3]);
+                        }
+                        red_add<4>(pool + chunk[ipos[n] + 3] + k, v4);
+                    }
+                }
+            }
+            pos = p;
+            continue;
+        }
+        mark(fwd ? 2 : 4);
 
         if (fwd) {
             // ---- matrix-vector products from registers (L123), 4 nodes at a time: packed FFMA2,
@@ -739,6 +818,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                 }
             }
             __syncthreads();
+            mark(3);
             // ---- cell update, one thread per (unit slot, node): CTA-local thanks to gate colocation ----
             for (int ci = tid; ci < UMAX * NB; ci += NTH) {
                 const int uu = ci / NB, n = ci % NB, jj = lc + uu * P.n_g;
@@ -800,64 +880,76 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                 }
             }
         } else {
-            // ---- backward: cell backward per (unit slot, node) -> gate gradients in smem ----
-            for (int ci = tid; ci < UMAX * NB; ci += NTH) {
-                const int uu = ci / NB, n = ci % NB, jj = lc + uu * P.n_g;
-                if (n >= nb || jj >= H) continue;
-                const uint32_t* I = chunk + ipos[n];
-                const float* cv = cin + (n * UMAX + uu) * CINMAX;
-                const float dh = cv[0], dc = cv[1], c = cv[2];
-                const float th = tanhf(c);
-                float* g = gb + (uu * NB + n) * GO;
-                float* db = dbias + uu * 4;
-                if constexpr (BIN || CS) {
-                    const float i = cv[3], o = cv[4], uv = cv[5];
-                    const float dov = dh * th;
-                    const float chat = dc + dh * o * (1.f - th * th);
-                    const float gi = chat * uv * i * (1.f - i), go = dov * o * (1.f - o), gu = chat * i * (1.f - uv * uv);
-                    g[0] = gi; g[1] = go; g[2] = gu;
-                    atomicAdd(db + 0, gi); atomicAdd(db + 1, go); atomicAdd(db + 2, gu);
-                    if constexpr (BIN) {
-                        if (kindB) {
-                            const float fl = cv[6], fr = cv[7], cl = cv[8], cr = cv[9];
-                            const float gfl = chat * cl * fl * (1.f - fl), gfr = chat * cr * fr * (1.f - fr);
-                            pool[I[4] + H + jj] = chat * fl;     // dc of the left child (unique parent)
-                            pool[I[6] + H + jj] = chat * fr;
-                            g[3] = gfl; g[4] = gfr;
-                            atomicAdd(db + 3, gfl + gfr);
+            // ---- backward: cell backward per (unit slot, node) -> gate gradients in smem; the bias
+            //      gradients are summed over the batch's nodes with a segmented warp reduction ----
+            {
+                const int uu = tid / NB, n = tid % NB, jj = lc + uu * P.n_g;
+                const bool act = uu < UMAX && n < nb && jj < H;
+                float db4[4] = {0.f, 0.f, 0.f, 0.f};
+                if (act) {
+                    const uint32_t* I = chunk + ipos[n];
+                    const float* cv = cin + (n * UMAX + uu) * CINMAX;
+                    const float dh = cv[0], dc = cv[1], c = cv[2];
+                    const float th = tanhf(c);
+                    float* g = gb + (uu * NB + n) * GO;
+                    if constexpr (BIN || CS) {
+                        const float i = cv[3], o = cv[4], uv = cv[5];
+                        const float dov = dh * th;
+                        const float chat = dc + dh * o * (1.f - th * th);
+                        const float gi = chat * uv * i * (1.f - i), go = dov * o * (1.f - o), gu = chat * i * (1.f - uv * uv);
+                        g[0] = gi; g[1] = go; g[2] = gu;
+                        db4[0] = gi; db4[1] = go; db4[2] = gu;
+                        if constexpr (BIN) {
+                            if (kindB) {
+                                const float fl = cv[6], fr = cv[7], cl = cv[8], cr = cv[9];
+                                const float gfl = chat * cl * fl * (1.f - fl), gfr = chat * cr * fr * (1.f - fr);
+                                pool[I[4] + H + jj] = chat * fl;     // dc of the left child (unique parent)
+                                pool[I[6] + H + jj] = chat * fr;
+                                g[3] = gfl; g[4] = gfr;
+                                db4[3] = gfl + gfr;
+                            }
+                        } else {
+                            const int nch = (int)(I[0] >> 8);
+                            float gfs = 0.f;
+#pragma unroll
+                            for (int kc = 0; kc < CHMAX; ++kc) {
+                                float gf = 0.f;
+                                if (kc < nch) {
+                                    const float f = cv[6 + kc], ck = cv[6 + CHMAX + kc];
+                                    gf = chat * ck * f * (1.f - f);
+                                    pool[I[5 + 2 * kc] + H + jj] = chat * f;
+                                }
+                                g[4 + kc] = gf;
+                                gfs += gf;
+                            }
+                            g[3] = gfs;
+                            db4[3] = gfs;
                         }
                     } else {
-                        const int nch = (int)(I[0] >> 8);
-                        float gfs = 0.f;
+                        const float i = cv[3], f = cv[4], o = cv[5], gg = cv[6], cp = cv[7];
+                        const uint32_t prv = I[4], padj = I[5];
+                        const float dov = dh * th;
+                        const float chat = dc + dh * o * (1.f - th * th);
+                        g[0] = chat * gg * i * (1.f - i);
+                        g[1] = chat * cp * f * (1.f - f);
+                        g[2] = dov * o * (1.f - o);
+                        g[3] = chat * i * (1.f - gg * gg);
+                        if (prv != NONE) pool[padj + H + jj] = chat * f;
 #pragma unroll
-                        for (int kc = 0; kc < CHMAX; ++kc) {
-                            float gf = 0.f;
-                            if (kc < nch) {
-                                const float f = cv[6 + kc], ck = cv[6 + CHMAX + kc];
-                                gf = chat * ck * f * (1.f - f);
-                                pool[I[5 + 2 * kc] + H + jj] = chat * f;
-                            }
-                            g[4 + kc] = gf;
-                            gfs += gf;
-                        }
-                        g[3] = gfs;
-                        atomicAdd(db + 3, gfs);
+                        for (int k = 0; k < 4; ++k) db4[k] = g[k];
                     }
-                } else {
-                    const float i = cv[3], f = cv[4], o = cv[5], gg = cv[6], cp = cv[7];
-                    const uint32_t prv = I[4], padj = I[5];
-                    const float dov = dh * th;
-                    const float chat = dc + dh * o * (1.f - th * th);
-                    g[0] = chat * gg * i * (1.f - i);
-                    g[1] = chat * cp * f * (1.f - f);
-                    g[2] = dov * o * (1.f - o);
-                    g[3] = chat * i * (1.f - gg * gg);
-                    if (prv != NONE) pool[padj + H + jj] = chat * f;
+                }
 #pragma unroll
-                    for (int k = 0; k < 4; ++k) atomicAdd(db + k, g[k]);
+                for (int k = 0; k < 4; ++k)
+#pragma unroll
+                    for (int s = NB / 2; s >= 1; s >>= 1) db4[k] += __shfl_xor_sync(FULL, db4[k], s);
+                if (n == 0 && uu < UMAX) {
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) dbias[uu * 4 + k] += db4[k];
                 }
             }
             __syncthreads();
+            mark(5);
             // ---- in-register outer products (dW, L104) and transposed products (L94, fn4), FFMA2 ----
             if (unit_ok) {
 #pragma unroll 2
@@ -951,7 +1043,13 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
 
     // ---------------- epilogue: apply gradients to the master copy, or write them (L129, L197) -----
     __syncthreads();
-    if (prof && tid == 0) prof[1] = gtimer();
+    mark(9);
+    if (prof && tid == 0) {
+        prof[1] = gtimer();
+        uint64_t* o = prof + 2 + 3 * (S[1] + 1);
+#pragma unroll
+        for (int k = 0; k < 10; ++k) o[k] = sec[k];
+    }
     const bool sgd = P.mode == 1;
     float* gout = P.grads;
     // every parameter element this CTA owns: f(flat index, cached weight, accumulated gradient)

@@ -19,7 +19,7 @@ sys.path.insert(0, ROOT)
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--batch-idx", type=int, default=0)
-    ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--reps", type=int, default=1)
     ap.add_argument("--config", default="tgt")
     ap.add_argument("--groups", type=int, default=1)
     ap.add_argument("--quiet", action="store_true")
@@ -46,7 +46,7 @@ def main():
     nbar = info["n_barriers"]
     n_cta = m.plan_info()["n_cta"]
     n_act = m.plan_info()["n_act"]
-    stride = 2 + 3 * (nbar + 1)
+    stride = 2 + 3 * (nbar + 1) + 10
     buf = torch.zeros((n_cta, stride), dtype=torch.int64, device="cuda")
     m.set_profile_buffer(buf, stride)
     ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
@@ -88,6 +88,13 @@ def main():
         if not args.quiet:
             print(f" {p:5d} {counts[p]:6d} {wmax/1e3:9.2f}us {wmean/1e3:9.2f}us {bl/1e3:9.2f}us")
     print(f"sum work_max {work_tot/1e3:.1f} us, sum barrier {bar_tot/1e3:.1f} us")
+    secs = raw[rows][:, 2 + 3 * (nbar + 1): 2 + 3 * (nbar + 1) + 10]
+    names = ["decode", "staging", "matvec", "cell", "cell-bwd", "outer/tmv", "heads", "signal", "wait", "other"]
+    mean = secs.mean(0)
+    mx = secs[secs.sum(1).argmax()]
+    tot = mean.sum()
+    print("section cycles (mean over CTAs | slowest CTA):")
+    print("  " + ", ".join(f"{n} {m/1e3:.0f}k ({m/tot*100:.0f}%) | {x/1e3:.0f}k" for n, m, x in zip(names, mean, mx)))
 
 
 if __name__ == "__main__":
