@@ -107,7 +107,9 @@ struct Cfg {
     static constexpr int O_CREC = O_BST + 4;
     static constexpr int O_MBAR = a4(O_CREC + cmax(CHSLOT, 1));     // one mbarrier (8-byte aligned)
     static constexpr int O_ZS = O_MBAR + 4;
-    static constexpr int O_HEAD = O_ZS + NB * ZC;
+    static constexpr int NC = 4;                                       // nodes per transposed-product chunk
+    static constexpr int O_DXB = O_ZS + NB * ZC;
+    static constexpr int O_HEAD = O_DXB + (CS ? 0 : UMAX * NC * KPMAX);
     static constexpr int ITER2 = (NB * UMAX * CINMAX + NTH - 1) / NTH;
     static_assert(UMAX * NB <= NTH && NB <= 32 && 32 % NB == 0, "one (unit, node) pair per thread");
     static_assert(KPMAX >= H, "head rows are staged in the input rows");
@@ -364,6 +366,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
     uint32_t* crec = smw + T::O_CREC;
     float* zs = sm + T::O_ZS;
     uint64_t* mbar = reinterpret_cast<uint64_t*>(smw + T::O_MBAR);
+    float* dxb = sm + T::O_DXB;
     uint32_t mphase = 0;
     const int C = P.C;
     float* Wo = sm + T::O_HEAD;
@@ -502,6 +505,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
         if (op == OP_W) {
             mark(8);
             bar_wait(bar + (pre >> 8), target[pre >> 8], prof ? prof + 2 + 3 * (pre >> 8) : nullptr);
+            // rows written by other CTAs before this barrier are read by the async proxy (TMA) below
+            if (warp == 0) fence_async_global();
             ++pos;
             continue;
         }
@@ -578,7 +583,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                 for (int k = lane; k < usedw; k += 32) bytes += H * 4;
 #pragma unroll
             for (int s = 16; s >= 1; s >>= 1) bytes += __shfl_xor_sync(FULL, bytes, s);
-            fence_async_global();        // rows written by other CTAs (acquired at the last wait) -> async proxy
             if (lane == 0) mbar_arrive_expect(mbar, bytes);
             __syncwarp();
             if (b0) bulk_g2s(xs + lane * KP + off0, src0, b0, mbar);
@@ -950,87 +954,121 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
             }
             __syncthreads();
             mark(5);
-            // ---- in-register outer products (dW, L104) and transposed products (L94, fn4), FFMA2 ----
-            if (unit_ok) {
-#pragma unroll 2
-                for (int n = 0; n < nb; ++n) {
-                    const uint32_t* I = chunk + ipos[n];
-                    const float* g = gb + (u * NB + n) * GO;
-                    if (kindB) {
-                        if constexpr (BIN) {
-                            const float* x = xs + n * LB::KP;
-                            float gr[4] = {g[0], g[1], g[2], 0.f};
-                            const float g3 = g[3], g4 = g[4];
+            // ---- in-register outer products (dW, L104) and transposed products (L94, fn4), FFMA2.
+            //      The UMAX units' partial transposed products are summed in shared memory, NC nodes at a
+            //      time, before one vector red.global.add per 4 columns goes to the destination ----
+            if constexpr (!CS) {
+                constexpr int NC = T::NC;
+                for (int n0 = 0; n0 < nb; n0 += NC) {
 #pragma unroll
-                            for (int t = 0; t < LB::NT; ++t) {
-                                const int col0 = LB::CG * (tu + TU * t);
-                                gr[3] = col0 < H ? g3 : g4;
-                                float xv[LB::CG], dx[LB::CG];
-                                lds<LB::CG>(x + col0, xv);
-                                outer_tmv<4, LB::CG>(wb, dwb, t, gr, xv, dx);
-                                if (col0 < 2 * H) {
-                                    float* dst = col0 < H ? pool + I[4] + col0 : pool + I[6] + (col0 - H);
-                                    red_add<LB::CG>(dst, dx);
+                    for (int dn = 0; dn < NC; ++dn) {
+                        const int n = n0 + dn;
+                        if (n < nb) {
+                            const float* g = gb + (u * NB + n) * GO;
+                            float* drow = dxb + (u * NC + dn) * KP;
+                            if (kindB) {
+                                if constexpr (BIN) {
+                                    const float* x = xs + n * LB::KP;
+                                    float gr[4] = {g[0], g[1], g[2], 0.f};
+                                    const float g3 = g[3], g4 = g[4];
+#pragma unroll
+                                    for (int t = 0; t < LB::NT; ++t) {
+                                        const int col0 = LB::CG * (tu + TU * t);
+                                        gr[3] = col0 < H ? g3 : g4;
+                                        float xv[LB::CG], dx[LB::CG];
+                                        lds<LB::CG>(x + col0, xv);
+                                        outer_tmv<4, LB::CG>(wb, dwb, t, gr, xv, dx);
+#pragma unroll
+                                        for (int q = 0; q < LB::CG; ++q) drow[col0 + q] = unit_ok ? dx[q] : 0.f;
+                                    }
+                                }
+                            } else {
+                                const float* x = xs + n * LA::KP;
+                                if constexpr (BIN) {
+                                    const float gr[3] = {g[0], g[1], g[2]};
+#pragma unroll
+                                    for (int t = 0; t < LA::NT; ++t) {
+                                        const int col0 = LA::CG * (tu + TU * t);
+                                        float xv[LA::CG], dx[LA::CG];
+                                        lds<LA::CG>(x + col0, xv);
+                                        outer_tmv<3, LA::CG>(wa, dwa, t, gr, xv, dx);
+#pragma unroll
+                                        for (int q = 0; q < LA::CG; ++q) drow[col0 + q] = unit_ok ? dx[q] : 0.f;
+                                    }
+                                } else {
+                                    const float gr[4] = {g[0], g[1], g[2], g[3]};
+#pragma unroll
+                                    for (int t = 0; t < LA::NT; ++t) {
+                                        const int col0 = LA::CG * (tu + TU * t);
+                                        float xv[LA::CG], dx[LA::CG];
+                                        lds<LA::CG>(x + col0, xv);
+                                        outer_tmv<4, LA::CG>(wa, dwa, t, gr, xv, dx);
+#pragma unroll
+                                        for (int q = 0; q < LA::CG; ++q) drow[col0 + q] = unit_ok ? dx[q] : 0.f;
+                                    }
                                 }
                             }
                         }
-                    } else {
-                        const float* x = xs + n * LA::KP;
-                        if constexpr (BIN) {
-                            const float gr[3] = {g[0], g[1], g[2]};
-                            const uint32_t tok = I[3];
-#pragma unroll
-                            for (int t = 0; t < LA::NT; ++t) {
-                                const int col0 = LA::CG * (tu + TU * t);
-                                float xv[LA::CG], dx[LA::CG];
-                                lds<LA::CG>(x + col0, xv);
-                                outer_tmv<3, LA::CG>(wa, dwa, t, gr, xv, dx);
-                                if (P.d_inputs && col0 < E) red_add<LA::CG>(P.d_inputs + (int64_t)tok * E + col0, dx);
-                            }
-                        } else if constexpr (LS) {
-                            const float gr[4] = {g[0], g[1], g[2], g[3]};
-                            const uint32_t tok = I[3], padj = I[5];
-#pragma unroll
-                            for (int t = 0; t < LA::NT; ++t) {
-                                const int col0 = LA::CG * (tu + TU * t);
-                                float xv[LA::CG], dx[LA::CG];
-                                lds<LA::CG>(x + col0, xv);
-                                outer_tmv<4, LA::CG>(wa, dwa, t, gr, xv, dx);
-                                if (col0 < E) {
-                                    if (P.d_inputs) red_add<LA::CG>(P.d_inputs + (int64_t)tok * E + col0, dx);
-                                } else if (col0 < E + H && padj != NONE) {
-                                    red_add<LA::CG>(pool + padj + (col0 - E), dx);
-                                }
-                            }
+                    }
+                    __syncthreads();
+                    const int q4 = KP / 4;
+                    for (int i = tid; i < NC * q4; i += NTH) {
+                        const int dn = i / q4, c = (i - dn * q4) * 4, n = n0 + dn;
+                        if (n >= nb) continue;
+                        const uint32_t* I = chunk + ipos[n];
+                        float* dst = nullptr;
+                        if (kindB) {
+                            if (c < H) dst = pool + I[4] + c;
+                            else if (c < 2 * H) dst = pool + I[6] + (c - H);
+                        } else if constexpr (BIN) {
+                            if (P.d_inputs && c < E) dst = P.d_inputs + (int64_t)I[3] * E + c;
                         } else {
-                            const float gr[4] = {g[0], g[1], g[2], g[3]};     // g[3] = sum_k g_fk for the x part
-                            const uint32_t tok = I[3];
-                            const int nch = (int)(I[0] >> 8);
+                            if (c < E) { if (P.d_inputs) dst = P.d_inputs + (int64_t)I[3] * E + c; }
+                            else if (c < E + H && I[5] != NONE) dst = pool + I[5] + (c - E);
+                        }
+                        if (dst) {
+                            float s[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
-                            for (int t = 0; t < LA::NT; ++t) {
-                                const int col0 = LA::CG * (tu + TU * t);
-                                float xv[LA::CG], dio[LA::CG];
-                                lds<LA::CG>(x + col0, xv);
-                                if (col0 < E) {
-                                    outer_tmv<4, LA::CG>(wa, dwa, t, gr, xv, dio);
-                                    if (P.d_inputs && tok != NONE) red_add<LA::CG>(P.d_inputs + (int64_t)tok * E + col0, dio);
-                                } else if (col0 < E + H) {
-                                    outer_tmv<3, LA::CG>(wa, dwa, t, gr, xv, dio);
+                            for (int uu = 0; uu < UMAX; ++uu) {
+                                const float4 v = *reinterpret_cast<const float4*>(dxb + (uu * NC + dn) * KP + c);
+                                s[0] += v.x; s[1] += v.y; s[2] += v.z; s[3] += v.w;
+                            }
+                            red_add<4>(dst, s);
+                        }
+                    }
+                    __syncthreads();
+                }
+            } else if (unit_ok) {
+                for (int n = 0; n < nb; ++n) {
+                    const uint32_t* I = chunk + ipos[n];
+                    const float* g = gb + (u * NB + n) * GO;
+                    const float* x = xs + n * LA::KP;
+                    const float gr[4] = {g[0], g[1], g[2], g[3]};     // g[3] = sum_k g_fk for the x part
+                    const uint32_t tok = I[3];
+                    const int nch = (int)(I[0] >> 8);
 #pragma unroll
-                                    for (int kc = 0; kc < CHMAX; ++kc) {
-                                        if (kc < nch) {
-                                            const float gf = g[4 + kc];
-                                            float yv[LA::CG], dh[LA::CG];
-                                            lds<LA::CG>(chs + (cslot[n] + kc) * LA::KP + col0, yv);
+                    for (int t = 0; t < LA::NT; ++t) {
+                        const int col0 = LA::CG * (tu + TU * t);
+                        float xv[LA::CG], dio[LA::CG];
+                        lds<LA::CG>(x + col0, xv);
+                        if (col0 < E) {
+                            outer_tmv<4, LA::CG>(wa, dwa, t, gr, xv, dio);
+                            if (P.d_inputs && tok != NONE) red_add<LA::CG>(P.d_inputs + (int64_t)tok * E + col0, dio);
+                        } else if (col0 < E + H) {
+                            outer_tmv<3, LA::CG>(wa, dwa, t, gr, xv, dio);
 #pragma unroll
-                                            for (int q = 0; q < LA::CG; ++q) {
-                                                const int k = t * LA::CG + q;
-                                                dwa[3][k] = fmaf(gf, yv[q], dwa[3][k]);
-                                                dh[q] = fmaf(wa[3][k], gf, dio[q]);
-                                            }
-                                            red_add<LA::CG>(pool + I[5 + 2 * kc] + (col0 - E), dh);
-                                        }
+                            for (int kc = 0; kc < CHMAX; ++kc) {
+                                if (kc < nch) {
+                                    const float gf = g[4 + kc];
+                                    float yv[LA::CG], dh[LA::CG];
+                                    lds<LA::CG>(chs + (cslot[n] + kc) * LA::KP + col0, yv);
+#pragma unroll
+                                    for (int q = 0; q < LA::CG; ++q) {
+                                        const int k = t * LA::CG + q;
+                                        dwa[3][k] = fmaf(gf, yv[q], dwa[3][k]);
+                                        dh[q] = fmaf(wa[3][k], gf, dio[q]);
                                     }
+                                    red_add<LA::CG>(pool + I[5 + 2 * kc] + (col0 - E), dh);
                                 }
                             }
                         }
