@@ -335,7 +335,7 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     kp.loss_word = s->s.loss_word;
     kp.lr = lr;
     kp.wd = wd;
-    if (m->prof && m->prof_stride < 2 + 3 * (int64_t)(s->s.n_bar + 1) + 10)
+    if (m->prof && m->prof_stride < 2 + 3 * (int64_t)(s->s.n_bar + 1) + 10 * (int64_t)(s->s.n_bar + 2))
         return fail(VPPS_E_INVALID, "profile buffer stride too small for this script");
     kp.prof = m->prof;
     kp.prof_stride = m->prof_stride;

@@ -105,8 +105,8 @@ struct Cfg {
     static constexpr int O_CSLOT = O_IPOS + NB;
     static constexpr int O_BST = O_CSLOT + NB;
     static constexpr int O_CREC = O_BST + 4;
-    static constexpr int O_MBAR = a4(O_CREC + cmax(CHSLOT, 1));     // one mbarrier (8-byte aligned)
-    static constexpr int O_ZS = O_MBAR + 4;
+    static constexpr int O_SEGP = a4(O_CREC + cmax(CHSLOT, 1));     // NB x 2 source pointers (8-byte aligned)
+    static constexpr int O_ZS = O_SEGP + 4 * NB;
     static constexpr int NC = 4;                                       // nodes per transposed-product chunk
     static constexpr int O_DXB = O_ZS + NB * ZC;
     static constexpr int O_HEAD = O_DXB + (CS ? 0 : UMAX * NC * KPMAX);
@@ -242,32 +242,18 @@ __device__ __forceinline__ float warp_max(float v) {
     return v;
 }
 
-// ---- TMA bulk copies global -> shared with an mbarrier transaction count (sm_90+) ----
+// ---- asynchronous global -> shared copies (cp.async / LDGSTS): no registers, zero fill when
+//      src_bytes < size ----
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-__device__ __forceinline__ void mbar_arrive_expect(uint64_t* b, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
-    asm volatile(
-        "{\n .reg .pred p;\n"
-        "VPPS_WAIT_%=:\n"
-        " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-        " @!p bra VPPS_WAIT_%=;\n}" ::"r"(smem_u32(b)),
-        "r"(parity)
-        : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* b) {
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                     smem_u32(dst)),
-                 "l"(src), "r"(bytes), "r"(smem_u32(b))
+__device__ __forceinline__ void cp_async16(void* dst, const void* src, uint32_t src_bytes) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src), "r"(src_bytes)
                  : "memory");
 }
-__device__ __forceinline__ void fence_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
-__device__ __forceinline__ void fence_async_shared() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void cp_async4(void* dst, const void* src, uint32_t src_bytes) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(smem_u32(dst)), "l"(src), "r"(src_bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
 __device__ __forceinline__ uint64_t gtimer() {
     uint64_t t;
@@ -365,9 +351,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
     int* bst = reinterpret_cast<int*>(smw + T::O_BST);
     uint32_t* crec = smw + T::O_CREC;
     float* zs = sm + T::O_ZS;
-    uint64_t* mbar = reinterpret_cast<uint64_t*>(smw + T::O_MBAR);
+    const float** segp = reinterpret_cast<const float**>(smw + T::O_SEGP);
     float* dxb = sm + T::O_DXB;
-    uint32_t mphase = 0;
     const int C = P.C;
     float* Wo = sm + T::O_HEAD;
     float* dWo = Wo + C * H;
@@ -470,7 +455,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
             sec_last = now;
         }
     };
-    if (tid == 0) mbar_init(mbar, 1);
     __syncthreads();
     if (prof && tid == 0) { prof[0] = gtimer(); sec_last = clock64(); }
 
@@ -498,6 +482,11 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
         const uint32_t op = pre & 0xFF;
         if (op == OP_S) {
             mark(7);
+            if (prof && tid == 0) {         // cumulative section clocks at the end of phase (pre >> 8) - 1
+                uint64_t* o = prof + 2 + 3 * (S[1] + 1) + 10 + 10 * (pre >> 8);
+#pragma unroll
+                for (int k = 0; k < 10; ++k) o[k] = sec[k];
+            }
             bar_signal(bar + (pre >> 8), prof ? prof + 2 + 3 * (pre >> 8) : nullptr);
             ++pos;
             continue;
@@ -505,23 +494,20 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
         if (op == OP_W) {
             mark(8);
             bar_wait(bar + (pre >> 8), target[pre >> 8], prof ? prof + 2 + 3 * (pre >> 8) : nullptr);
-            // rows written by other CTAs before this barrier are read by the async proxy (TMA) below
-            if (warp == 0) fence_async_global();
             ++pos;
             continue;
         }
-        // ---- decode (warp 0): a batch of up to NB consecutive instructions with this opcode, then the
-        //      batch's input rows are fetched by TMA bulk copies (cp.async.bulk) into shared memory ----
+        // ---- decode (warp 0): a batch of up to NB consecutive instructions with this opcode, and the
+        //      global source of every input-row segment of the batch ----
         const bool is_head = (op == OP_HEAD_F || op == OP_HEAD_B);
         const bool fwd = (op & 1) == 0;
         const bool kindB = BIN && (op == OP_INT_F || op == OP_INT_B);
         const int KP = is_head ? LA::KP : (kindB ? LB::KP : LA::KP);
-        fence_async_shared();            // our generic reads of the staging buffers precede the next async writes
         __syncthreads();
         mark(0);
         if (warp == 0) {
             const uint32_t lim = min(s1, cbase + (uint32_t)CHUNK);
-            int nbw = 0, usedw = 0;
+            int nbw = 0;
             if (!(op == OP_CS_F || op == OP_CS_B)) {
                 const uint32_t sz = (uint32_t)instr_words(pre);
                 const uint32_t q = pos + (uint32_t)lane * sz;
@@ -532,6 +518,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                 if (lane == 0) { bst[0] = nbw; bst[1] = (int)(pos + nbw * sz); bst[2] = 0; }
             } else {
                 if (lane == 0) {
+                    int usedw = 0;
                     uint32_t p = pos;
                     while (p < lim && nbw < NB) {
                         const uint32_t w = chunk[p - cbase];
@@ -550,103 +537,75 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                     bst[0] = nbw; bst[1] = (int)p; bst[2] = usedw;
                 }
                 nbw = __shfl_sync(FULL, nbw, 0);
-                usedw = __shfl_sync(FULL, usedw, 0);
             }
             __syncwarp();
-            // segments of node n = lane: (source, destination offset in its row, bytes)
-            const bool issue = !is_head || holds_head;
-            const float* src0 = nullptr; const float* src1 = nullptr;
-            int off0 = 0, off1 = 0;
-            uint32_t b0 = 0, b1 = 0;
-            if (issue && lane < nbw) {
+            // node n = lane: row segment 0 and segment 1 sources (nullptr = absent -> zeros)
+            const float* s0p = nullptr;
+            const float* s1p = nullptr;
+            if (lane < nbw && (!is_head || holds_head)) {
                 const uint32_t* I = chunk + ipos[lane];
                 if (is_head) {
-                    src0 = pool + I[2]; b0 = H * 4;                                       // h of the cell
+                    s0p = pool + I[2];                                        // h of the cell
                 } else if constexpr (BIN) {
                     if (!kindB) {
-                        src0 = inputs + (int64_t)(fwd ? I[2] : I[3]) * E; b0 = E * 4;
+                        s0p = inputs + (int64_t)(fwd ? I[2] : I[3]) * E;          // x
                     } else {
-                        src0 = pool + (fwd ? I[2] : I[3]); b0 = H * 4;                    // [h_l; h_r]
-                        src1 = pool + (fwd ? I[3] : I[5]); b1 = H * 4; off1 = H;
+                        s0p = pool + (fwd ? I[2] : I[3]);                         // [h_l; h_r]
+                        s1p = pool + (fwd ? I[3] : I[5]);
                     }
                 } else if constexpr (LS) {
-                    const uint32_t tok = fwd ? I[2] : I[3], prv = fwd ? I[3] : I[4];
-                    src0 = inputs + (int64_t)tok * E; b0 = E * 4;
-                    if (prv != NONE) { src1 = pool + prv; b1 = H * 4; off1 = E; }
+                    const uint32_t prv = fwd ? I[3] : I[4];
+                    s0p = inputs + (int64_t)(fwd ? I[2] : I[3]) * E;              // [x; h_prev]
+                    if (prv != NONE) s1p = pool + prv;
                 } else {
                     const uint32_t tok = fwd ? I[2] : I[3];
-                    if (tok != NONE) { src0 = inputs + (int64_t)tok * E; b0 = E * 4; }
+                    if (tok != NONE) s0p = inputs + (int64_t)tok * E;             // [x; h~]
                 }
             }
-            uint32_t bytes = b0 + b1;
-            if (CS && issue && !is_head)
-                for (int k = lane; k < usedw; k += 32) bytes += H * 4;
-#pragma unroll
-            for (int s = 16; s >= 1; s >>= 1) bytes += __shfl_xor_sync(FULL, bytes, s);
-            if (lane == 0) mbar_arrive_expect(mbar, bytes);
-            __syncwarp();
-            if (b0) bulk_g2s(xs + lane * KP + off0, src0, b0, mbar);
-            if (b1) bulk_g2s(xs + lane * KP + off1, src1, b1, mbar);
-            if (CS && issue && !is_head)
-                for (int k = lane; k < usedw; k += 32) bulk_g2s(chs + k * KP + E, pool + crec[k], H * 4, mbar);
+            if (lane < NB) { segp[2 * lane] = s0p; segp[2 * lane + 1] = s1p; }
         }
         __syncthreads();
         const int nb = bst[0];
         const uint32_t p = (uint32_t)bst[1];
-
         mark(1);
-        // ---- while the bulk copies fly: zero the parts of the rows no copy writes and load every
-        //      per-(unit, node) cell operand (one round trip) ----
-        if (!is_head) {
-            const int Kk = kindB ? KB : KA;
-            if (KP > Kk || LS || CS) {           // padding beyond K, absent h_prev (t = 0), absent word
-                const int q4 = KP / 4;
-                for (int i = tid; i < nb * q4; i += NTH) {
-                    const int n = i / q4, c = (i - n * q4) * 4;
-                    const uint32_t* I = chunk + ipos[n];
-                    bool z = c >= Kk;
-                    if constexpr (LS) z = z || (c >= E && c < E + H && (fwd ? I[3] : I[4]) == NONE);
-                    if constexpr (CS) z = z || (c < E && (fwd ? I[2] : I[3]) == NONE);
-                    if (z) *reinterpret_cast<float4*>(xs + n * KP + c) = f4zero();
-                }
-                if constexpr (CS) {
-                    if (KP > E + H) {
-                        const int qp = (KP - E - H) / 4;
-                        for (int i = tid; i < bst[2] * qp; i += NTH) {
-                            const int r = i / qp, c = E + H + (i - r * qp) * 4;
-                            *reinterpret_cast<float4*>(chs + r * KP + c) = f4zero();
-                        }
+        // ---- staging: asynchronous 16-byte copies global -> shared (cp.async; zero fill for absent
+        //      segments and padding) of every input row and every per-(unit, node) cell operand, all in
+        //      flight together: one round trip per batch ----
+        {
+            const int q4 = KP / 4;
+            int A = E, B = 0;                         // row = [seg0 (A floats) | seg1 (B floats) | zeros]
+            if (is_head) { A = H; B = 0; }
+            else if (kindB) { A = H; B = H; }
+            else if (LS) { A = E; B = H; }
+            const int rows = (is_head && !holds_head) ? 0 : nb;
+            for (int i = tid; i < rows * q4; i += NTH) {
+                const int n = i / q4, c = (i - n * q4) * 4;
+                const float* src = nullptr;
+                if (c < A) { const float* b = segp[2 * n]; if (b) src = b + c; }
+                else if (c < A + B) { const float* b = segp[2 * n + 1]; if (b) src = b + (c - A); }
+                cp_async16(xs + n * KP + c, src ? src : pool, src ? 16u : 0u);
+            }
+            if constexpr (CS) {
+                if (!is_head) {
+                    for (int i = tid; i < bst[2] * q4; i += NTH) {     // child rows: h at [E, E + H)
+                        const int r = i / q4, c = (i - r * q4) * 4;
+                        const bool in = c >= E && c < E + H;
+                        cp_async16(chs + r * KP + c, in ? pool + crec[r] + (c - E) : pool, in ? 16u : 0u);
                     }
                 }
             }
-            const int ncin = n_cin(op);
-            const int total2 = nb * UMAX * ncin;
-            float s2[T::ITER2];
-#pragma unroll
-            for (int it = 0; it < T::ITER2; ++it) {
-                const int i = tid + it * NTH;
-                const float* src = nullptr;
-                if (i < total2) {
-                    const int n = i / (UMAX * ncin), rem = i - n * (UMAX * ncin);
-                    const int uu = rem / ncin, k = rem - uu * ncin, jj = lc + uu * P.n_g;
-                    if (jj < H) src = cin_src<H>(op, chunk + ipos[n], k, jj, pool);
-                }
-                s2[it] = src ? __ldcg(src) : 0.f;
+            const int ncin = is_head ? 0 : n_cin(op);
+            for (int i = tid; i < nb * UMAX * ncin; i += NTH) {
+                const int n = i / (UMAX * ncin), rem = i - n * (UMAX * ncin);
+                const int uu = rem / ncin, k = rem - uu * ncin, jj = lc + uu * P.n_g;
+                const float* src = jj < H ? cin_src<H>(op, chunk + ipos[n], k, jj, pool) : nullptr;
+                cp_async4(cin + (n * UMAX + uu) * CINMAX + k, src ? src : pool, src ? 4u : 0u);
             }
-#pragma unroll
-            for (int it = 0; it < T::ITER2; ++it) {
-                const int i = tid + it * NTH;
-                if (i < total2) {
-                    const int n = i / (UMAX * ncin), rem = i - n * (UMAX * ncin);
-                    const int uu = rem / ncin, k = rem - uu * ncin;
-                    cin[(n * UMAX + uu) * CINMAX + k] = s2[it];
-                }
-            }
+            cp_async_wait_all();
         }
-        mbar_wait(mbar, mphase);                // the batch's bulk copies have landed
-        mphase ^= 1;
         if constexpr (CS) {                     // h~ = sum of the children's h (child-sum, [5] eq. 2)
             if (!is_head) {
+                __syncthreads();
                 for (int i = tid; i < nb * (H / 4); i += NTH) {
                     const int n = i / (H / 4), c = E + (i - n * (H / 4)) * 4;
                     const int nch = (int)(chunk[ipos[n]] >> 8);

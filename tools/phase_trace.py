@@ -23,6 +23,7 @@ def main():
     ap.add_argument("--config", default="tgt")
     ap.add_argument("--groups", type=int, default=1)
     ap.add_argument("--quiet", action="store_true")
+    ap.add_argument("--sections", action="store_true")
     args = ap.parse_args()
     import torch
     import synth
@@ -46,7 +47,7 @@ def main():
     nbar = info["n_barriers"]
     n_cta = m.plan_info()["n_cta"]
     n_act = m.plan_info()["n_act"]
-    stride = 2 + 3 * (nbar + 1) + 10
+    stride = 2 + 3 * (nbar + 1) + 10 * (nbar + 2)
     buf = torch.zeros((n_cta, stride), dtype=torch.int64, device="cuda")
     m.set_profile_buffer(buf, stride)
     ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
@@ -95,6 +96,18 @@ def main():
     tot = mean.sum()
     print("section cycles (mean over CTAs | slowest CTA):")
     print("  " + ", ".join(f"{n} {m/1e3:.0f}k ({m/tot*100:.0f}%) | {x/1e3:.0f}k" for n, m, x in zip(names, mean, mx)))
+    if args.sections:
+        # per-phase section clocks of CTA 0 (cumulative snapshots at each signal)
+        base = 2 + 3 * (nbar + 1) + 10
+        cum = raw[0, base: base + 10 * (nbar + 1)].reshape(nbar + 1, 10)
+        final = raw[0, 2 + 3 * (nbar + 1): 2 + 3 * (nbar + 1) + 10]
+        cum = np.vstack([cum[1:], final])            # snapshot b = end of phase b-1
+        prev = np.zeros(10)
+        print(" phase " + " ".join(f"{n[:8]:>8s}" for n in names) + "   (kcycles, CTA 0)")
+        for p in range(nbar + 1):
+            d = cum[p] - prev
+            prev = cum[p]
+            print(f" {p:5d} " + " ".join(f"{v/1e3:8.1f}" for v in d))
 
 
 if __name__ == "__main__":
