@@ -163,6 +163,7 @@ def main():
     ap.add_argument("--impl", default="vpps", choices=["vpps", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--groups", type=int, default=4, help="replica groups G (SPEC P1); 148 = 4 x 37")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
 
@@ -187,7 +188,7 @@ def main():
     shapes = vpps.param_shapes("binary", H, E, C)
     P = synth.init_params(shapes, rng)
     X = synth.input_table(rng, V, E)
-    m = vpps.Model("binary", H, E, C, device=local)
+    m = vpps.Model("binary", H, E, C, device=local, groups=args.groups)
     params = torch.zeros(m.n_floats, dtype=torch.float32, device=dev)
     grads = torch.zeros_like(params)
     for name, _ in shapes:
@@ -293,7 +294,7 @@ def main():
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "impl": "vpps",
             "config": {"workload": WORKLOAD, "global_batch": args.batch * world, "per_gpu_batch": args.batch,
-                       "seq_len": None, "parallelism": f"dp{world}",
+                       "seq_len": None, "parallelism": f"dp{world}", "replica_groups": args.groups,
                        "mode": "fused fwd-bwd-sgd, 1 kernel" if world == 1 else "fwd_bwd + NCCL all-reduce + sgd",
                        "l2": "no flush" if args.no_flush else "flushed (256 MiB write) before every timed step",
                        "batches": f"{N_BATCHES} distinct pre-built scripts cycled"},

@@ -147,6 +147,17 @@ __device__ __forceinline__ void lds(const float* p, float* v) {
     }
 }
 
+template <int CG>
+__device__ __forceinline__ void sts_granule(float* p, const float (&v)[CG], bool keep) {
+    if constexpr (CG == 4) {
+        *reinterpret_cast<float4*>(p) = keep ? make_float4(v[0], v[1], v[2], v[3]) : f4zero();
+    } else if constexpr (CG == 2) {
+        *reinterpret_cast<float2*>(p) = keep ? make_float2(v[0], v[1]) : make_float2(0.f, 0.f);
+    } else {
+        *p = keep ? v[0] : 0.f;
+    }
+}
+
 // acc[n][o] += w[r] . x[n] over granule t for 4 nodes, packed FFMA2 (fma.rn.f32x2) where CG >= 2.
 // Rows 0..R-1 accumulate into outputs 0..R-1, except row 3 -> output SPLIT when SPLIT >= 0.
 template <int R, int CG, int SPLIT, int NR, int NREG, int RO>
@@ -937,8 +948,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                                         float xv[LB::CG], dx[LB::CG];
                                         lds<LB::CG>(x + col0, xv);
                                         outer_tmv<4, LB::CG>(wb, dwb, t, gr, xv, dx);
-#pragma unroll
-                                        for (int q = 0; q < LB::CG; ++q) drow[col0 + q] = unit_ok ? dx[q] : 0.f;
+                                        sts_granule<LB::CG>(drow + col0, dx, unit_ok);
                                     }
                                 }
                             } else {
@@ -951,8 +961,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                                         float xv[LA::CG], dx[LA::CG];
                                         lds<LA::CG>(x + col0, xv);
                                         outer_tmv<3, LA::CG>(wa, dwa, t, gr, xv, dx);
-#pragma unroll
-                                        for (int q = 0; q < LA::CG; ++q) drow[col0 + q] = unit_ok ? dx[q] : 0.f;
+                                        sts_granule<LA::CG>(drow + col0, dx, unit_ok);
                                     }
                                 } else {
                                     const float gr[4] = {g[0], g[1], g[2], g[3]};
@@ -962,8 +971,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                                         float xv[LA::CG], dx[LA::CG];
                                         lds<LA::CG>(x + col0, xv);
                                         outer_tmv<4, LA::CG>(wa, dwa, t, gr, xv, dx);
-#pragma unroll
-                                        for (int q = 0; q < LA::CG; ++q) drow[col0 + q] = unit_ok ? dx[q] : 0.f;
+                                        sts_granule<LA::CG>(drow + col0, dx, unit_ok);
                                     }
                                 }
                             }
@@ -971,7 +979,11 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                     }
                     __syncthreads();
                     const int q4 = KP / 4;
-                    for (int i = tid; i < NC * q4; i += NTH) {
+                    // every CTA of the group pushes to the same rows: start each CTA at a different
+                    // column so the L2 atomics of different CTAs hit different addresses at a time
+                    const int tot = NC * q4, rot = (lc * 37) % tot;
+                    for (int i0 = tid; i0 < tot; i0 += NTH) {
+                        const int i = i0 + rot < tot ? i0 + rot : i0 + rot - tot;
                         const int dn = i / q4, c = (i - dn * q4) * 4, n = n0 + dn;
                         if (n >= nb) continue;
                         const uint32_t* I = chunk + ipos[n];

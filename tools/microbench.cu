@@ -85,7 +85,53 @@ __global__ void __launch_bounds__(256, 1) mb(const float* __restrict__ src, floa
     }
 }
 
+// FP32 FMA throughput: 8 independent accumulators per thread, plain FFMA vs packed FFMA2.
+template <bool PACKED>
+__global__ void __launch_bounds__(256, 1) fma_tp(float* out, long long* cyc, int iters) {
+    float a[16];
+    for (int i = 0; i < 16; ++i) a[i] = threadIdx.x * 1e-3f + i;
+    const float b = 0.999f, c = 1e-4f;
+    __syncthreads();
+    const long long t0 = clock64();
+    for (int it = 0; it < iters; ++it) {
+        if constexpr (PACKED) {
+#pragma unroll
+            for (int i = 0; i < 16; i += 2) {
+                float2 r = __ffma2_rn(make_float2(a[i], a[i + 1]), make_float2(b, b), make_float2(c, c));
+                a[i] = r.x; a[i + 1] = r.y;
+            }
+        } else {
+#pragma unroll
+            for (int i = 0; i < 16; ++i) a[i] = fmaf(a[i], b, c);
+        }
+    }
+    __syncthreads();
+    const long long t1 = clock64();
+    float s = 0.f;
+    for (int i = 0; i < 16; ++i) s += a[i];
+    out[blockIdx.x * 256 + threadIdx.x] = s;
+    if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
+}
+
 int main() {
+    {
+        float* o;
+        long long* cy;
+        cudaMalloc(&o, 148 * 256 * 4);
+        cudaMalloc(&cy, 148 * 8);
+        const int iters = 4096;
+        for (int packed = 0; packed < 2; ++packed) {
+            if (packed) fma_tp<true><<<148, 256>>>(o, cy, iters);
+            else fma_tp<false><<<148, 256>>>(o, cy, iters);
+            cudaDeviceSynchronize();
+            long long h[148];
+            cudaMemcpy(h, cy, sizeof(h), cudaMemcpyDeviceToHost);
+            double mean = 0;
+            for (int i = 0; i < 148; ++i) mean += h[i] / 148.0;
+            printf("%s: %.1f FMA/clk/SM (256 threads, 16 independent accumulators)\n", packed ? "FFMA2" : "FFMA ",
+                   256.0 * 16 * iters / mean);
+        }
+    }
     const int nseg = 64, segf = 256;
     float *src, *sink;
     unsigned* ctr;
