@@ -76,6 +76,10 @@ typedef struct {
     int32_t groups;      /* replica groups G (SPEC P1); 0 = 1.  G > 1 is plan-only in v1       */
     int32_t device;      /* CUDA device ordinal; ignored when plan_only                         */
     int32_t plan_only;   /* 1: no CUDA calls (partition + script generation only, CPU tests)   */
+    int32_t cluster;     /* > 1: each replica group is one thread-block cluster of this many CTAs
+                            that owns whole graphs (SPEC S5g), synchronised by the hardware
+                            cluster barrier; groups = the number of co-resident clusters (or the
+                            given `groups` when plan_only).  0 = grid-wide groups (SPEC S5). */
 } vpps_options;
 
 /* A batch of graphs in CSR form (the super-graph of L205 is built from it).

@@ -103,8 +103,8 @@ def unit_plan(cell: str, H: int, E: int, C: int, n_sm: int, cps: int = 1, G: int
     umax = 1
     while umax < umax_needed:
         umax *= 2
-    if umax > 8:
-        raise ValueError("NOFIT: more than 8 units per CTA")
+    if umax > 16:
+        raise ValueError("NOFIT: more than 16 units per CTA")
     cols = {
         "lstm": [E, H, H], "binary": [E, 2 * H, H, H, H], "childsum": [E, E, H, H, H],
     }[cell]

@@ -23,8 +23,11 @@ def pre(op: str, length: int) -> int:
     return OP[op] | (length << 8)
 
 
-def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 148):
-    """Returns dict(words, pool_words, zero_words, loss_word, n_bar, levels, nodes)."""
+def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 148, by_graph: bool = False):
+    """Returns dict(words, pool_words, zero_words, loss_word, n_bar, levels, nodes).
+
+    by_graph: SPEC S5g — whole graphs are assigned to groups (min-load over graph MACs, batch order)
+    instead of single nodes per level."""
     # S1/S2: super-graph node list
     nodes = []          # dict(kind, graph, cell(local), children(global ids), token, label, cellnode)
     for b, g in enumerate(graphs):
@@ -36,10 +39,10 @@ def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 14
                 kind = "CS"
             else:
                 kind = "LSTM"
-            nodes.append(dict(kind=kind, children=[base + k for k in ch], token=tok, label=lab))
+            nodes.append(dict(kind=kind, children=[base + k for k in ch], token=tok, label=lab, graph=b))
         for v, (ch, tok, lab) in enumerate(g):
             if lab >= 0:
-                nodes.append(dict(kind="HEAD", children=[base + v], token=-1, label=lab))
+                nodes.append(dict(kind="HEAD", children=[base + v], token=-1, label=lab, graph=b))
     # S3: levels
     level = []
     for n in nodes:
@@ -58,7 +61,9 @@ def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 14
     rec = [0] * len(nodes)
     for i, n in enumerate(nodes):
         rec[i] = off
-        size = {"LSTM": 6 * H, "LEAF": 5 * H, "INT": 7 * H, "CS": (5 + len(n["children"])) * H,
+        nch = len(n["children"])
+        # forward fields, then the gate gradients written by the backward pass (SPEC §S7)
+        size = {"LSTM": (6 + 4) * H, "LEAF": (5 + 3) * H, "INT": (7 + 5) * H, "CS": (5 + nch + 3 + nch) * H,
                 "HEAD": C + 1}[n["kind"]]
         off = _a32(off + size)
     pool_words = off
@@ -111,6 +116,15 @@ def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 14
     by_level = [[] for _ in range(L + 1)]
     for i in range(len(nodes)):
         by_level[level[i]].append(i)
+    graph_group = None
+    if by_graph:
+        # S5g: whole graphs to the least-loaded group (graph cost = Σ node costs), batch order, ties lowest
+        gload = [0] * G
+        graph_group = []
+        for b in range(len(graphs)):
+            g = min(range(G), key=lambda x: (gload[x], x))
+            gload[g] += sum(cost(n) for n in nodes if n["graph"] == b)
+            graph_group.append(g)
     phase_instrs = []            # per phase: per group list of words
     part = []
     for p in range(P):
@@ -119,8 +133,11 @@ def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 14
         load = [0] * G
         per_g = [[] for _ in range(G)]
         for i in by_level[lv]:
-            g = min(range(G), key=lambda x: (load[x], x))
-            load[g] += cost(nodes[i])
+            if by_graph:
+                g = graph_group[nodes[i]["graph"]]
+            else:
+                g = min(range(G), key=lambda x: (load[x], x))
+                load[g] += cost(nodes[i])
             per_g[g].extend(instr(i, fwd))
         phase_instrs.append(per_g)
         part.append([g for g in range(G) if per_g[g]])

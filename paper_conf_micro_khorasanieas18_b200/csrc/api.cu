@@ -1,6 +1,7 @@
 // C ABI of libvpps (include/vpps.h): argument checking, object lifetime, the one H2D script copy,
 // the cooperative launch of the persistent kernel and loss bookkeeping.  No torch types here.
 #include <cuda_runtime.h>
+#include <algorithm>
 #include <climits>
 #include <cstring>
 #include <memory>
@@ -60,6 +61,7 @@ struct vpps_model_s {
     cudaEvent_t t_before = nullptr, t_after = nullptr;
     uint64_t* prof = nullptr;
     int64_t prof_stride = 0;
+    int32_t cluster = 0;                // > 1: cluster-replica path (vpps_cluster.cu)
     // Pre-allocated staging ring for per-batch scripts: a pinned host buffer and a
     // device buffer per slot; a slot is reused once the kernel that last read it has finished.
     struct Slot {
@@ -122,6 +124,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     }
     m->n_floats = cur;
     int32_t n_sm = o.n_sm;
+    m->cluster = o.cluster > 1 ? o.cluster : 0;
     if (!m->plan_only) {
         m->device = o.device;
         CK(cudaSetDevice(o.device));
@@ -131,12 +134,48 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
         if (n_sm == 0) n_sm = prop.multiProcessorCount;
         if (n_sm > prop.multiProcessorCount) return fail(VPPS_E_INVALID, "n_sm exceeds the device's SM count");
     } else if (n_sm == 0) {
-        n_sm = 148;
+        n_sm = m->cluster ? m->cluster * o.groups : 148;
+    }
+    if (m->cluster && !m->plan_only) {
+        // cluster replicas (SPEC S5g): one group per co-resident cluster of `cluster` CTAs
+        int32_t nv = 0;
+        const Variant* v = cluster_variants(&nv);
+        for (int32_t i = 0; i < nv; ++i)
+            if (v[i].cell == cell && v[i].H == H && v[i].E == E && v[i].umax == m->cluster) m->var = &v[i];
+        if (!m->var) return fail(VPPS_E_NOFIT, "no cluster specialisation for this op set and cluster size");
+        if (C > 32) return fail(VPPS_E_NOFIT, "single-CTA loss head supports C <= 32 classes in v1");
+        m->smem = m->var->smem_bytes(C);
+        CK(cudaFuncSetAttribute(m->var->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)m->smem));
+        CK(cudaFuncSetAttribute(m->var->fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+        cudaLaunchConfig_t cfg = {};
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = m->cluster;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
+        cfg.gridDim = dim3(m->cluster);
+        cfg.blockDim = dim3(256);
+        cfg.dynamicSmemBytes = m->smem;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        int ncl = 0;
+        CK(cudaOccupancyMaxActiveClusters(&ncl, m->var->fn, &cfg));
+        ncl = std::min(ncl, n_sm / m->cluster);
+        if (ncl < 1) return fail(VPPS_E_NOFIT, "no cluster of this size can be resident");
+        o.groups = ncl;
+        n_sm = ncl * m->cluster;
     }
     std::string err;
     if (!unit_plan(cell, H, E, C, n_sm, o.ctas_per_sm, o.groups, &m->plan, &err))
         return fail(err.rfind("NOFIT", 0) == 0 ? VPPS_E_NOFIT : VPPS_E_INVALID, err);
-    if (!m->plan_only) {
+    m->plan.by_graph = m->cluster != 0;
+    if (m->cluster && m->plan.n_g != m->cluster) return fail(VPPS_E_INVALID, "groups x cluster must equal n_sm");
+    if (m->cluster && !m->plan_only) {
+        CK(cudaMallocHost(&m->h_loss, 2 * sizeof(float)));
+        m->h_loss[0] = m->h_loss[1] = 0.f;
+        CK(cudaEventCreateWithFlags(&m->ev[0], cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&m->ev[1], cudaEventDisableTiming));
+    } else if (!m->plan_only) {
         if (H % 4 || E % 4) return fail(VPPS_E_INVALID, "H and E must be multiples of 4");
         int32_t nv = 0;
         const Variant* v = variants(&nv);
@@ -260,9 +299,9 @@ vpps_status vpps_upload_script(vpps_script s, void* stream) {
     if (!s) return fail(VPPS_E_INVALID, "null script");
     if (s->model->plan_only) return fail(VPPS_E_STATE, "plan-only model");
     if (s->uploaded) return VPPS_OK;
-    const size_t bytes = s->s.words.size() * sizeof(uint32_t);
+    const size_t bytes = s->s.blob.size() * sizeof(uint32_t);
     CK(cudaMalloc(&s->d_words, bytes));
-    CK(cudaMemcpyAsync(s->d_words, s->s.words.data(), bytes, cudaMemcpyHostToDevice, (cudaStream_t)stream));
+    CK(cudaMemcpyAsync(s->d_words, s->s.blob.data(), bytes, cudaMemcpyHostToDevice, (cudaStream_t)stream));
     CK(cudaStreamSynchronize((cudaStream_t)stream));     // pageable source: complete before returning
     s->uploaded = true;
     return VPPS_OK;
@@ -275,7 +314,7 @@ static vpps_status stage_script(vpps_model m, vpps_script s, cudaStream_t st, in
     const int k = m->next_slot;
     m->next_slot = (k + 1) % vpps_model_s::kSlots;
     vpps_model_s::Slot& sl = m->ring[k];
-    const size_t n = s->s.words.size();
+    const size_t n = s->s.blob.size();
     if (!sl.done) CK(cudaEventCreateWithFlags(&sl.done, cudaEventDisableTiming));
     if (sl.used) CK(cudaEventSynchronize(sl.done));
     if (n > sl.cap) {
@@ -285,7 +324,7 @@ static vpps_status stage_script(vpps_model m, vpps_script s, cudaStream_t st, in
         CK(cudaMallocHost(&sl.h, sl.cap * sizeof(uint32_t)));
         CK(cudaMalloc(&sl.d, sl.cap * sizeof(uint32_t)));
     }
-    std::memcpy(sl.h, s->s.words.data(), n * sizeof(uint32_t));
+    std::memcpy(sl.h, s->s.blob.data(), n * sizeof(uint32_t));
     CK(cudaMemcpyAsync(sl.d, sl.h, n * sizeof(uint32_t), cudaMemcpyHostToDevice, st));
     *slot_out = k;
     *dwords = sl.d;
@@ -317,7 +356,7 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         if (r != VPPS_OK) return r;
     }
     CK(cudaMemsetAsync(m->pool, 0, s->s.zero_words * sizeof(float), st));
-    if (m->plan.G > 1) CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));
+    if (m->plan.G > 1 || m->cluster) CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));
     if (d_inputs) CK(cudaMemsetAsync(d_inputs, 0, (size_t)n_rows * m->plan.E * sizeof(float), st));
     KParams kp{};
     kp.params = m->params;
@@ -341,7 +380,29 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     kp.prof_stride = m->prof_stride;
     void* args[] = {&kp};
     if (m->t_before) CK(cudaEventRecord(m->t_before, st));
-    CK(cudaLaunchCooperativeKernel(m->var->fn, dim3(m->plan.n_cta), dim3(256), args, m->smem, st));
+    if (m->cluster) {
+        // one cluster per replica group; clusters never wait on each other (graphs are whole per group)
+        cudaLaunchConfig_t cfg = {};
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = m->cluster;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
+        cfg.gridDim = dim3(m->plan.n_cta);
+        cfg.blockDim = dim3(256);
+        cfg.dynamicSmemBytes = m->smem;
+        cfg.stream = st;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        CK(cudaLaunchKernelExC(&cfg, m->var->fn, args));
+        // dW of the weight matrices from the recorded operands, fused SGD in mode 1
+        const uint32_t* lists = dwords + s->s.words.size();
+        launch_dw_gemm(m->pool, inputs, m->params, m->grads, lists, (int32_t)s->s.n_int, lists + 3 * s->s.n_int,
+                       (int32_t)s->s.n_leaf, m->plan.H, m->plan.E, m->offsets.data(), m->n_floats, mode, lr, wd, st);
+        CK(cudaGetLastError());
+    } else {
+        CK(cudaLaunchCooperativeKernel(m->var->fn, dim3(m->plan.n_cta), dim3(256), args, m->smem, st));
+    }
     if (m->t_after) CK(cudaEventRecord(m->t_after, st));
     if (ring_slot >= 0) {
         CK(cudaEventRecord(m->ring[ring_slot].done, st));

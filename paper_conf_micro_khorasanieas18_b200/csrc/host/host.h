@@ -33,6 +33,7 @@ int32_t paper_choose_cps(const std::vector<Shape>& mats, int32_t n_sm, int32_t t
 struct Plan {
     int32_t cell, H, E, C;
     int32_t n_cta, n_g, n_act, umax, G;
+    bool by_graph = false;   // SPEC S5g: whole graphs assigned to groups (cluster replicas)
     std::vector<int32_t> table;   // rows of 8 int32
 };
 bool unit_plan(int32_t cell, int32_t H, int32_t E, int32_t C, int32_t n_sm, int32_t cps, int32_t G,
@@ -53,6 +54,10 @@ struct Script {
     int64_t pool_words = 0, zero_words = 0, loss_word = 0;
     int32_t n_bar = 0, n_levels = 0;
     int64_t n_nodes = 0, n_heads = 0, max_token = -1;
+    // device upload blob = words ‖ (rec, rec_l, rec_r) per internal node ‖ (rec, token) per leaf; the node
+    // lists drive the gradient GEMM of the cluster path.  Not part of the SPEC words.
+    std::vector<uint32_t> blob;
+    int64_t n_int = 0, n_leaf = 0;
     double flops = 0.0, act_bytes = 0.0;
 };
 

@@ -68,7 +68,7 @@ bool unit_plan(int32_t cell, int32_t H, int32_t E, int32_t C, int32_t n_sm, int3
     const int32_t need = (H + p.n_g - 1) / p.n_g;
     p.umax = 1;
     while (p.umax < need) p.umax *= 2;
-    if (p.umax > 8) { *err = "NOFIT: more than 8 hidden units per CTA"; return false; }
+    if (p.umax > 16) { *err = "NOFIT: more than 16 hidden units per CTA"; return false; }
 
     // (matrix, gate rows of unit j) for each cell family, matrices in parameter order
     struct Block { int32_t matrix, gates, cols; };

@@ -22,6 +22,7 @@ struct Node {
     Kind kind;
     int32_t token, label;
     int32_t ch_begin, ch_count;   // into Graph::kids (global ids)
+    int32_t graph;
 };
 
 }  // namespace
@@ -48,7 +49,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
             if (nch < 0) { *err = "child_ptr not monotone"; return -4; }
             if (tok < -1 || tok >= n_input_rows) { *err = "token out of range"; return -4; }
             if (lab < -1 || lab >= C) { *err = "label out of range"; return -4; }
-            Node nd{K_CS, tok, lab, (int32_t)kids.size(), nch};
+            Node nd{K_CS, tok, lab, (int32_t)kids.size(), nch, g};
             for (int32_t k = c0; k < c1; ++k) {
                 const int32_t ch = b.children[k];
                 if (ch < 0 || ch >= local) { *err = "children must precede their parent"; return -4; }
@@ -76,7 +77,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
         }
         for (int32_t v = first; v < last; ++v)
             if (b.label[v] >= 0) {
-                nodes.push_back(Node{K_HEAD, -1, b.label[v], (int32_t)kids.size(), 1});
+                nodes.push_back(Node{K_HEAD, -1, b.label[v], (int32_t)kids.size(), 1, g});
                 kids.push_back(base + (v - first));
             }
     }
@@ -105,10 +106,10 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     for (int64_t i = 0; i < N; ++i) {
         int64_t sz = 0;
         switch (nodes[i].kind) {
-            case K_LSTM: sz = 6 * H; break;
-            case K_LEAF: sz = 5 * H; break;
-            case K_INT: sz = 7 * H; break;
-            case K_CS: sz = (5 + nodes[i].ch_count) * H; break;
+            case K_LSTM: sz = (6 + 4) * H; break;          // forward fields + gate gradients (§S7)
+            case K_LEAF: sz = (5 + 3) * H; break;
+            case K_INT: sz = (7 + 5) * H; break;
+            case K_CS: sz = (8 + 2 * nodes[i].ch_count) * H; break;
             case K_HEAD: sz = C + 1; break;
         }
         rec[i] = (uint32_t)cursor;
@@ -191,15 +192,34 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     std::vector<std::vector<uint32_t>> body(G);
     std::vector<int64_t> load(G);
     std::vector<char> was_active(G, 0);
+    // S5g (cluster replicas): every graph goes whole to the least-loaded group, in batch order
+    std::vector<int32_t> graph_group;
+    if (plan.by_graph) {
+        std::vector<int64_t> gcost(b.n_graphs, 0);
+        for (int64_t i = 0; i < N; ++i) gcost[nodes[i].graph] += macs(i);
+        std::vector<int64_t> gload(G, 0);
+        graph_group.resize(b.n_graphs);
+        for (int32_t gi = 0; gi < b.n_graphs; ++gi) {
+            int32_t best = 0;
+            for (int32_t g = 1; g < G; ++g)
+                if (gload[g] < gload[best]) best = g;
+            gload[best] += gcost[gi];
+            graph_group[gi] = best;
+        }
+    }
     for (int32_t p = 0; p < P; ++p) {
         const bool fwd = p <= L;
         const int32_t lv = fwd ? p : 2 * L + 1 - p;
         for (int32_t g = 0; g < G; ++g) { body[g].clear(); load[g] = 0; }
         for (int64_t i : at_level[lv]) {
             int32_t best = 0;
-            for (int32_t g = 1; g < G; ++g)
-                if (load[g] < load[best]) best = g;
-            load[best] += macs(i);
+            if (plan.by_graph) {
+                best = graph_group[nodes[i].graph];
+            } else {
+                for (int32_t g = 1; g < G; ++g)
+                    if (load[g] < load[best]) best = g;
+                load[best] += macs(i);
+            }
             emit(body[best], i, fwd);
         }
         int32_t active_prev = 0;
@@ -240,6 +260,20 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     }
     s.flops = flops;
     s.act_bytes = abytes;
+    // device blob: the words, then the operand lists of the per-matrix gradient GEMM (binary cells)
+    s.blob = s.words;
+    s.n_int = s.n_leaf = 0;
+    for (int64_t i = 0; i < N; ++i)
+        if (nodes[i].kind == K_INT) {
+            const int32_t* ch = kids.data() + nodes[i].ch_begin;
+            s.blob.insert(s.blob.end(), {rec[i], rec[ch[0]], rec[ch[1]]});
+            ++s.n_int;
+        }
+    for (int64_t i = 0; i < N; ++i)
+        if (nodes[i].kind == K_LEAF) {
+            s.blob.insert(s.blob.end(), {rec[i], (uint32_t)nodes[i].token});
+            ++s.n_leaf;
+        }
     return 0;
 }
 

@@ -1,0 +1,694 @@
+// VPPS on thread-block clusters (sm_100a) — binary Tree-LSTM.
+//
+// A replica group of the partition plan (SPEC P1) is one cluster of 16 CTAs on 16 SMs: together their
+// register files hold every weight matrix of the model once (weights cached in registers
+// for the whole pass).  Whole graphs are assigned to clusters (SPEC S5g), so no node depends on another
+// cluster and the signal/wait instructions of the script (L165) become the hardware cluster barrier
+// (barrier.cluster.arrive.release / wait.acquire, ~400 cycles) instead of a grid-wide counter barrier.
+// Registers cannot hold the weights and their gradients at 16 CTAs per replica, so the kernel applies
+// the paper's gradient-accumulation strategy (L185, §III-C2): it records the outer-product operands
+// (the gate gradients, next to the activations already in the pool) and one GEMM per weight matrix
+// (vpps_dw_gemm below) forms dW = Σ g xᵀ afterwards, fused with the SGD update (L129, L197).
+#include "vpps_kernel.cuh"
+#include "dev_common.cuh"
+
+namespace vpps {
+namespace dev {
+namespace cl {
+
+constexpr int NTH = 256;
+constexpr int CHUNK = 4096;    // script words staged in shared memory (L171)
+constexpr int NB = 16;         // nodes per batch: one node per lane of a unit's 16-lane group
+constexpr int NC = 4;          // nodes per transposed-product chunk
+constexpr int ZC = 32;         // classes per head (C <= 32)
+constexpr int CINMAX = 10;
+constexpr uint32_t NONE = 0xFFFFFFFFu;
+enum : uint32_t { S = 0x01, W = 0x02, LEAF_F = 0x20, LEAF_B = 0x21, INT_F = 0x22, INT_B = 0x23, HEAD_F = 0x40, HEAD_B = 0x41 };
+
+__device__ __forceinline__ int words(uint32_t w) {
+    switch (w & 0xFF) {
+        case LEAF_F: return 3;
+        case LEAF_B: return 4;
+        case INT_F: return 4;
+        case INT_B: return 7;
+        case HEAD_F: return 4;
+        case HEAD_B: return 5;
+        default: return 1;
+    }
+}
+__device__ __forceinline__ int n_cin(uint32_t op) {
+    return op == INT_F ? 2 : op == INT_B ? 10 : op == LEAF_B ? 6 : 0;
+}
+// Address of cell operand k of (instruction I, unit jj); records [h c i o u (fl fr) | g...] (SPEC §S7).
+template <int H>
+__device__ __forceinline__ const float* cin_src(uint32_t op, const uint32_t* I, int k, int jj, const float* pool) {
+    if (op == INT_F) return pool + (k == 0 ? I[2] : I[3]) + H + jj;                // c_l, c_r
+    const uint32_t rec = I[1], adj = I[2];
+    if (k < 2) return pool + adj + k * H + jj;                                     // dh, dc
+    if (k < 8) return pool + rec + (k - 1) * H + jj;                               // c i o u (fl fr)
+    return pool + (k == 8 ? I[3] : I[5]) + H + jj;                                 // c_l, c_r
+}
+
+__device__ __forceinline__ void cluster_arrive() { asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory"); }
+__device__ __forceinline__ void cluster_wait() { asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory"); }
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ uint32_t cluster_index() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%clusterid.x;" : "=r"(r));
+    return r;
+}
+
+template <int K, int TU>
+struct Lay {
+    static constexpr int CG = (K >= 4 * TU) ? 4 : ((K >= 2 * TU) ? 2 : 1);
+    static constexpr int NT = (K + CG * TU - 1) / (CG * TU);
+    static constexpr int NREG = NT * CG;
+    static constexpr int KP = NT * CG * TU;
+};
+
+// Sum over a 16-lane group of four per-lane values (one per node): transposed halving at distances 8
+// and 4, then a butterfly over the low two bits.  Lane l ends with node 2*bit3(l) + bit2(l).
+__device__ __forceinline__ float treduce4_16(float v0, float v1, float v2, float v3, int lane) {
+    const bool b3 = lane & 8, b2 = lane & 4;
+    const float s0 = b3 ? v0 : v2, s1 = b3 ? v1 : v3;
+    float k0 = b3 ? v2 : v0, k1 = b3 ? v3 : v1;
+    k0 += __shfl_xor_sync(FULLMASK, s0, 8);
+    k1 += __shfl_xor_sync(FULLMASK, s1, 8);
+    const float s = b2 ? k0 : k1;
+    float k = b2 ? k1 : k0;
+    k += __shfl_xor_sync(FULLMASK, s, 4);
+    k += __shfl_xor_sync(FULLMASK, k, 2);
+    k += __shfl_xor_sync(FULLMASK, k, 1);
+    return k;
+}
+
+template <int H, int E>
+struct CCfg {
+    static constexpr int NCL = 16;                 // CTAs per cluster (= per replica)
+    static constexpr int UM = H / NCL;             // hidden units per CTA
+    static constexpr int TU = NTH / UM;            // threads per unit
+    static_assert(H % NCL == 0 && TU == 16, "cluster kernel: 16 units per CTA, 16 threads per unit");
+    using LA = Lay<E, TU>;                         // leaf bundle rows (i, o, u of W_iou) over x
+    using LB = Lay<2 * H, TU>;                     // internal bundle rows (i, o, u of U_iou; f) over [h_l; h_r]
+    static constexpr int KPMAX = LA::KP > LB::KP ? LA::KP : LB::KP;
+    static constexpr int O_X = CHUNK;
+    static constexpr int O_DXB = O_X + NB * KPMAX;
+    static constexpr int O_CIN = O_DXB + 8 * NC * KPMAX;
+    static constexpr int O_BIAS = O_CIN + NB * UM * CINMAX;
+    static constexpr int O_IPOS = O_BIAS + UM * 4;
+    static constexpr int O_BST = O_IPOS + NB;
+    static constexpr int O_SEGP = O_BST + 4;                 // NB x 2 pointers (8-byte aligned)
+    static constexpr int O_ZS = O_SEGP + 4 * NB;
+    static constexpr int O_HEAD = O_ZS + NB * ZC;
+    static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 2 * C + 8); }
+};
+
+template <int H, int E>
+__global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
+    using T = CCfg<H, E>;
+    using LA = typename T::LA;
+    using LB = typename T::LB;
+    constexpr int TU = T::TU, UM = T::UM, NCL = T::NCL;
+    extern __shared__ __align__(16) uint32_t smw[];
+    float* sm = reinterpret_cast<float*>(smw);
+    uint32_t* chunk = smw;
+    float* xs = sm + T::O_X;
+    float* dxb = sm + T::O_DXB;
+    float* cin = sm + T::O_CIN;
+    float* bias = sm + T::O_BIAS;
+    int* ipos = reinterpret_cast<int*>(smw + T::O_IPOS);
+    int* bst = reinterpret_cast<int*>(smw + T::O_BST);
+    const float** segp = reinterpret_cast<const float**>(smw + T::O_SEGP);
+    float* zs = sm + T::O_ZS;
+    const int C = P.C;
+    float* Wo = sm + T::O_HEAD;
+    float* dWo = Wo + C * H;
+    float* bo = dWo + C * H;
+    float* dbo = bo + C;
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int lc = (int)cluster_rank(), grp = (int)cluster_index();
+    const uint32_t* S_ = P.script;
+    const uint32_t G = S_[0];
+    const uint32_t hdr = 2 + G + 1;
+    const uint32_t s0 = hdr + S_[2 + grp], s1 = hdr + S_[3 + grp];
+    float* pool = P.pool;
+    const float* __restrict__ inputs = P.inputs;
+    const int64_t* off = P.off;
+    const int u = tid / TU, tu = tid % TU, gl = lane & 15;      // unit slot, thread in unit, lane in group
+    const int j = lc + u * NCL;                                 // hidden unit of this thread
+    const bool holds_head = (lc == H % NCL);
+
+    // ---- prologue: this CTA's slice of every weight matrix DRAM -> registers (L123, L129) ----
+    float wa[3][LA::NREG], wb[4][LB::NREG];
+#pragma unroll
+    for (int r = 0; r < 3; ++r)
+#pragma unroll
+        for (int t = 0; t < LA::NT; ++t)
+#pragma unroll
+            for (int q = 0; q < LA::CG; ++q) {
+                const int col = LA::CG * (tu + TU * t) + q;
+                wa[r][t * LA::CG + q] = col < E ? __ldg(P.params + off[0] + (int64_t)(r * H + j) * E + col) : 0.f;
+            }
+#pragma unroll
+    for (int r = 0; r < 4; ++r)
+#pragma unroll
+        for (int t = 0; t < LB::NT; ++t)
+#pragma unroll
+            for (int q = 0; q < LB::CG; ++q) {
+                const int col = LB::CG * (tu + TU * t) + q;
+                float v = 0.f;
+                if (col < 2 * H) {
+                    if (r < 3) v = __ldg(P.params + off[1] + (int64_t)(r * H + j) * (2 * H) + col);
+                    else v = __ldg(P.params + (col < H ? off[2] + (int64_t)j * H + col : off[3] + (int64_t)j * H + col - H));
+                }
+                wb[r][t * LB::CG + q] = v;
+            }
+    if (tid < UM * 4) {
+        const int uu = tid / 4, k = tid % 4, jj = lc + uu * NCL;
+        bias[tid] = k < 3 ? __ldg(P.params + off[5] + k * H + jj) : __ldg(P.params + off[6] + jj);
+    }
+    if (holds_head) {
+        for (int i = tid; i < C * H; i += NTH) { Wo[i] = __ldg(P.params + off[4] + i); dWo[i] = 0.f; }
+        for (int i = tid; i < C; i += NTH) { bo[i] = __ldg(P.params + off[7] + i); dbo[i] = 0.f; }
+    }
+    float dbacc[4] = {0.f, 0.f, 0.f, 0.f};       // bias gradients of (unit u) over the nodes of slot gl
+    uint64_t* prof = P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
+    __syncthreads();
+    if (prof && tid == 0) prof[0] = gtimer();
+
+    // ---- script interpretation (L171-177) ----
+    uint32_t cbase = s0;
+    auto refill = [&](uint32_t from) {
+        __syncthreads();
+        constexpr int PER = CHUNK / NTH;
+        uint32_t w[PER];
+#pragma unroll
+        for (int i = 0; i < PER; ++i) {
+            const uint32_t k = tid + i * NTH;
+            w[i] = from + k < s1 ? __ldg(S_ + from + k) : 0u;
+        }
+#pragma unroll
+        for (int i = 0; i < PER; ++i) chunk[tid + i * NTH] = w[i];
+        __syncthreads();
+        cbase = from;
+    };
+    if (s0 < s1) refill(s0);
+    bool pending = false;
+    uint32_t pos = s0;
+    while (pos < s1) {
+        if (pos + 640 > cbase + CHUNK && cbase + CHUNK < s1) refill(pos);
+        const uint32_t pre = chunk[pos - cbase];
+        const uint32_t op = pre & 0xFF;
+        if (op == S) {            // signal (L165): arrive on the cluster barrier, release our writes
+            if (prof && tid == 0) prof[2 + 3 * (pre >> 8)] = gtimer();
+            cluster_arrive();
+            pending = true;
+            ++pos;
+            continue;
+        }
+        if (op == W) {            // wait (L165): all 16 CTAs of the replica have signalled
+            if (prof && tid == 0) prof[3 + 3 * (pre >> 8)] = gtimer();
+            cluster_wait();
+            pending = false;
+            if (prof && tid == 0) prof[4 + 3 * (pre >> 8)] = gtimer();
+            ++pos;
+            continue;
+        }
+        const bool is_head = (op == HEAD_F || op == HEAD_B);
+        const bool fwd = (op & 1) == 0;
+        const bool kindB = (op == INT_F || op == INT_B);
+        const int KP = kindB ? LB::KP : LA::KP;
+        // ---- decode (warp 0): up to NB consecutive instructions with this opcode + row sources ----
+        __syncthreads();
+        if (warp == 0) {
+            const uint32_t lim = min(s1, cbase + (uint32_t)CHUNK);
+            const uint32_t sz = (uint32_t)words(pre);
+            const uint32_t q = pos + (uint32_t)lane * sz;
+            const bool ok = lane < NB && q + sz <= lim && (chunk[q - cbase] & 0xFF) == op;
+            const unsigned msk = __ballot_sync(FULLMASK, ok);
+            const int nbw = (msk == FULLMASK) ? 32 : (__ffs(~msk) - 1);
+            if (lane < nbw) ipos[lane] = (int)(q - cbase);
+            if (lane == 0) { bst[0] = nbw; bst[1] = (int)(pos + nbw * sz); }
+            __syncwarp();
+            const float* sp0 = nullptr;
+            const float* sp1 = nullptr;
+            if (lane < nbw && (!is_head || holds_head)) {
+                const uint32_t* I = chunk + ipos[lane];
+                if (is_head) sp0 = pool + I[2];
+                else if (!kindB) sp0 = inputs + (int64_t)(fwd ? I[2] : I[3]) * E;
+                else { sp0 = pool + (fwd ? I[2] : I[3]); sp1 = pool + (fwd ? I[3] : I[5]); }
+            }
+            if (lane < NB) { segp[2 * lane] = sp0; segp[2 * lane + 1] = sp1; }
+        }
+        __syncthreads();
+        const int nb = bst[0];
+        const uint32_t p = (uint32_t)bst[1];
+        // ---- staging: cp.async of every input row and cell operand of the batch (one round trip) ----
+        {
+            const int q4 = KP / 4;
+            const int A = is_head ? H : (kindB ? H : E), B = kindB ? H : 0;
+            const int rows = (is_head && !holds_head) ? 0 : nb;
+            for (int i = tid; i < rows * q4; i += NTH) {
+                const int n = i / q4, c = (i - n * q4) * 4;
+                const float* src = nullptr;
+                if (c < A) { const float* b = segp[2 * n]; if (b) src = b + c; }
+                else if (c < A + B) { const float* b = segp[2 * n + 1]; if (b) src = b + (c - A); }
+                cp_async16(xs + n * KP + c, src ? src : pool, src ? 16u : 0u);
+            }
+            const int ncin = is_head ? 0 : n_cin(op);
+            for (int i = tid; i < nb * UM * ncin; i += NTH) {
+                const int n = i / (UM * ncin), rem = i - n * (UM * ncin);
+                const int uu = rem / ncin, k = rem - uu * ncin;
+                cp_async4(cin + (n * UM + uu) * CINMAX + k, cin_src<H>(op, chunk + ipos[n], k, lc + uu * NCL, pool), 4u);
+            }
+            cp_async_wait_all();
+        }
+        __syncthreads();
+
+        if (is_head) {            // loss heads (L42) on the CTA holding W_out
+            if (holds_head) {
+                if (op == HEAD_F) {
+                    for (int pi = warp; pi < nb * C; pi += NTH / 32) {
+                        const int n = pi / C, c = pi - n * C;
+                        float s = 0.f;
+                        for (int k = 4 * lane; k < H; k += 128) {
+                            const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                            const float4 h4 = *reinterpret_cast<const float4*>(xs + n * KP + k);
+                            s += w4.x * h4.x + w4.y * h4.y + w4.z * h4.z + w4.w * h4.w;
+                        }
+                        s = warp_sum(s);
+                        if (lane == 0) zs[n * ZC + c] = s + bo[c];
+                    }
+                    __syncthreads();
+                    for (int n = warp; n < nb; n += NTH / 32) {
+                        const uint32_t* I = chunk + ipos[n];
+                        const float zl = lane < C ? zs[n * ZC + lane] : -INFINITY;
+                        const float m = warp_max(zl);
+                        const float lse = m + logf(warp_sum(lane < C ? expf(zl - m) : 0.f));
+                        if (lane < C) pool[I[1] + lane] = expf(zl - lse);
+                        const float zy = __shfl_sync(FULLMASK, zl, (int)I[3]);
+                        if (lane == 0) {
+                            pool[I[1] + C] = lse - zy;
+                            atomicAdd(pool + P.loss_word, lse - zy);   // aggregated loss node (L205)
+                        }
+                    }
+                } else {
+                    for (int i = tid; i < nb * C; i += NTH) {
+                        const int n = i / C, c = i - n * C;
+                        const uint32_t* I = chunk + ipos[n];
+                        zs[n * ZC + c] = __ldcg(pool + I[1] + c) - (c == (int)I[4] ? 1.f : 0.f);
+                    }
+                    __syncthreads();
+                    for (int c = tid; c < C; c += NTH) {
+                        float s = 0.f;
+                        for (int n = 0; n < nb; ++n) s += zs[n * ZC + c];
+                        dbo[c] += s;
+                    }
+                    for (int i = tid; i < C * H; i += NTH) {
+                        const int c = i / H, k = i - c * H;
+                        float s = 0.f;
+                        for (int n = 0; n < nb; ++n) s = fmaf(zs[n * ZC + c], xs[n * KP + k], s);
+                        dWo[i] += s;
+                    }
+                    for (int i = tid; i < nb * (H / 4); i += NTH) {
+                        const int n = i / (H / 4), k = (i - n * (H / 4)) * 4;
+                        float v4[4] = {0.f, 0.f, 0.f, 0.f};
+                        for (int c = 0; c < C; ++c) {
+                            const float dzc = zs[n * ZC + c];
+                            const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                            v4[0] = fmaf(w4.x, dzc, v4[0]); v4[1] = fmaf(w4.y, dzc, v4[1]);
+                            v4[2] = fmaf(w4.z, dzc, v4[2]); v4[3] = fmaf(w4.w, dzc, v4[3]);
+                        }
+                        red_add<4>(pool + chunk[ipos[n] + 3] + k, v4);
+                    }
+                }
+            }
+            pos = p;
+            continue;
+        }
+
+        if (fwd) {
+            // ---- forward: matvec from registers (L123), 4 nodes at a time; the unit's 16 lanes reduce
+            //      with a transposed butterfly and the lane holding node n's gates does its cell update ----
+            for (int n0 = 0; n0 < nb; n0 += 4) {
+                float v[4][5];
+                if (kindB) {
+                    float2 a[4][5];
+#pragma unroll
+                    for (int n = 0; n < 4; ++n)
+#pragma unroll
+                        for (int o = 0; o < 5; ++o) a[n][o] = make_float2(0.f, 0.f);
+#pragma unroll
+                    for (int t = 0; t < LB::NT; ++t) {
+                        const int col0 = LB::CG * (tu + TU * t);
+                        const int of = col0 < H ? 3 : 4;
+#pragma unroll
+                        for (int n = 0; n < 4; ++n) {
+                            float xv[LB::CG];
+                            lds<LB::CG>(xs + (n0 + n) * LB::KP + col0, xv);
+#pragma unroll
+                            for (int q = 0; q < LB::CG; q += 2) {
+                                const float2 x2 = make_float2(xv[q], xv[q + 1]);
+                                const int k = t * LB::CG + q;
+#pragma unroll
+                                for (int r = 0; r < 3; ++r)
+                                    a[n][r] = __ffma2_rn(make_float2(wb[r][k], wb[r][k + 1]), x2, a[n][r]);
+                                const float2 f2 = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), x2, make_float2(0.f, 0.f));
+                                if (of == 3) { a[n][3].x += f2.x; a[n][3].y += f2.y; }
+                                else { a[n][4].x += f2.x; a[n][4].y += f2.y; }
+                            }
+                        }
+                    }
+#pragma unroll
+                    for (int n = 0; n < 4; ++n)
+#pragma unroll
+                        for (int o = 0; o < 5; ++o) v[n][o] = a[n][o].x + a[n][o].y;
+                } else {
+                    float2 a[4][3];
+#pragma unroll
+                    for (int n = 0; n < 4; ++n)
+#pragma unroll
+                        for (int o = 0; o < 3; ++o) a[n][o] = make_float2(0.f, 0.f);
+#pragma unroll
+                    for (int t = 0; t < LA::NT; ++t) {
+                        const int col0 = LA::CG * (tu + TU * t);
+#pragma unroll
+                        for (int n = 0; n < 4; ++n) {
+                            float xv[LA::CG];
+                            lds<LA::CG>(xs + (n0 + n) * LA::KP + col0, xv);
+#pragma unroll
+                            for (int q = 0; q < LA::CG; q += 2) {
+                                const float2 x2 = make_float2(xv[q], xv[q + 1]);
+                                const int k = t * LA::CG + q;
+#pragma unroll
+                                for (int r = 0; r < 3; ++r)
+                                    a[n][r] = __ffma2_rn(make_float2(wa[r][k], wa[r][k + 1]), x2, a[n][r]);
+                            }
+                        }
+                    }
+#pragma unroll
+                    for (int n = 0; n < 4; ++n) {
+#pragma unroll
+                        for (int o = 0; o < 3; ++o) v[n][o] = a[n][o].x + a[n][o].y;
+                        v[n][3] = v[n][4] = 0.f;
+                    }
+                }
+                float g5[5];
+#pragma unroll
+                for (int o = 0; o < 5; ++o) g5[o] = treduce4_16(v[0][o], v[1][o], v[2][o], v[3][o], gl);
+                const int n = n0 + (gl >> 2);
+                if ((gl & 3) == 0 && n < nb) {
+                    const uint32_t* I = chunk + ipos[n];
+                    const uint32_t rec = I[1];
+                    const float* b = bias + u * 4;
+                    const float i = sigm(g5[0] + b[0]), o = sigm(g5[1] + b[1]), uv = tanhf(g5[2] + b[2]);
+                    float c = i * uv;
+                    if (kindB) {
+                        const float* cv = cin + (n * UM + u) * CINMAX;
+                        const float fl = sigm(g5[3] + b[3]), fr = sigm(g5[4] + b[3]);
+                        c += fl * cv[0] + fr * cv[1];
+                        pool[rec + 5 * H + j] = fl;
+                        pool[rec + 6 * H + j] = fr;
+                    }
+                    pool[rec + j] = o * tanhf(c);
+                    pool[rec + H + j] = c;
+                    pool[rec + 2 * H + j] = i;
+                    pool[rec + 3 * H + j] = o;
+                    pool[rec + 4 * H + j] = uv;
+                }
+            }
+        } else {
+            // ---- backward: cell backward by thread (unit u, node gl); its gate gradients are recorded
+            //      in the node's record for the dW GEMM (L185) and broadcast to the unit's lanes ----
+            float g[5] = {0.f, 0.f, 0.f, 0.f, 0.f};
+            if (gl < nb) {
+                const uint32_t* I = chunk + ipos[gl];
+                const uint32_t rec = I[1];
+                const float* cv = cin + (gl * UM + u) * CINMAX;
+                const float dh = cv[0], dc = cv[1], c = cv[2], i = cv[3], o = cv[4], uv = cv[5];
+                const float th = tanhf(c);
+                const float chat = dc + dh * o * (1.f - th * th);
+                g[0] = chat * uv * i * (1.f - i);
+                g[1] = dh * th * o * (1.f - o);
+                g[2] = chat * i * (1.f - uv * uv);
+                if (kindB) {
+                    const float fl = cv[6], fr = cv[7], cl = cv[8], cr = cv[9];
+                    g[3] = chat * cl * fl * (1.f - fl);
+                    g[4] = chat * cr * fr * (1.f - fr);
+                    pool[I[4] + H + j] = chat * fl;          // dc of the children (unique parent)
+                    pool[I[6] + H + j] = chat * fr;
+                    pool[rec + 10 * H + j] = g[3];
+                    pool[rec + 11 * H + j] = g[4];
+                    pool[rec + 7 * H + j] = g[0];
+                    pool[rec + 8 * H + j] = g[1];
+                    pool[rec + 9 * H + j] = g[2];
+                } else {
+                    pool[rec + 5 * H + j] = g[0];
+                    pool[rec + 6 * H + j] = g[1];
+                    pool[rec + 7 * H + j] = g[2];
+                }
+                dbacc[0] += g[0]; dbacc[1] += g[1]; dbacc[2] += g[2]; dbacc[3] += g[3] + g[4];
+            }
+            // transposed products (L94, fn4): per node, dx = Σ_r W[r] g_r over this thread's columns,
+            // the warp's two units summed by a shuffle, the 8 warps summed in shared memory, then one
+            // vector red.global.add per 4 columns into the children's dh (or dX for leaves)
+            const int src = lane & 16;
+            for (int n0 = 0; n0 < nb; n0 += NC) {
+#pragma unroll
+                for (int dn = 0; dn < NC; ++dn) {
+                    const int n = n0 + dn;
+                    float gr[5];
+#pragma unroll
+                    for (int r = 0; r < 5; ++r) gr[r] = __shfl_sync(FULLMASK, g[r], src | (n & 15));
+                    float* drow = dxb + (warp * NC + dn) * KP;
+                    if (kindB) {
+#pragma unroll
+                        for (int t = 0; t < LB::NT; ++t) {
+                            const int col0 = LB::CG * (tu + TU * t);
+                            const float gf = col0 < H ? gr[3] : gr[4];
+                            float dx[LB::CG];
+#pragma unroll
+                            for (int q = 0; q < LB::CG; q += 2) {
+                                const int k = t * LB::CG + q;
+                                float2 d = make_float2(0.f, 0.f);
+#pragma unroll
+                                for (int r = 0; r < 3; ++r)
+                                    d = __ffma2_rn(make_float2(wb[r][k], wb[r][k + 1]), make_float2(gr[r], gr[r]), d);
+                                d = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), make_float2(gf, gf), d);
+                                dx[q] = d.x + __shfl_xor_sync(FULLMASK, d.x, 16);
+                                dx[q + 1] = d.y + __shfl_xor_sync(FULLMASK, d.y, 16);
+                            }
+                            if (lane < 16) sts_granule<LB::CG>(drow + col0, dx, n < nb);
+                        }
+                    } else {
+#pragma unroll
+                        for (int t = 0; t < LA::NT; ++t) {
+                            const int col0 = LA::CG * (tu + TU * t);
+                            float dx[LA::CG];
+#pragma unroll
+                            for (int q = 0; q < LA::CG; q += 2) {
+                                const int k = t * LA::CG + q;
+                                float2 d = make_float2(0.f, 0.f);
+#pragma unroll
+                                for (int r = 0; r < 3; ++r)
+                                    d = __ffma2_rn(make_float2(wa[r][k], wa[r][k + 1]), make_float2(gr[r], gr[r]), d);
+                                dx[q] = d.x + __shfl_xor_sync(FULLMASK, d.x, 16);
+                                dx[q + 1] = d.y + __shfl_xor_sync(FULLMASK, d.y, 16);
+                            }
+                            if (lane < 16) sts_granule<LA::CG>(drow + col0, dx, n < nb);
+                        }
+                    }
+                }
+                __syncthreads();
+                const int q4 = KP / 4, tot = NC * q4;
+                for (int i = tid; i < tot; i += NTH) {
+                    const int dn = i / q4, c = (i - dn * q4) * 4, n = n0 + dn;
+                    if (n >= nb) continue;
+                    const uint32_t* I = chunk + ipos[n];
+                    float* dst = nullptr;
+                    if (kindB) dst = c < H ? pool + I[4] + c : pool + I[6] + (c - H);
+                    else if (P.d_inputs && c < E) dst = P.d_inputs + (int64_t)I[3] * E + c;
+                    if (dst) {
+                        float s[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+                        for (int w = 0; w < 8; ++w) {
+                            const float4 x = *reinterpret_cast<const float4*>(dxb + (w * NC + dn) * KP + c);
+                            s[0] += x.x; s[1] += x.y; s[2] += x.z; s[3] += x.w;
+                        }
+                        red_add<4>(dst, s);
+                    }
+                }
+                __syncthreads();
+            }
+        }
+        pos = p;
+    }
+    if (pending) cluster_wait();
+    if (prof && tid == 0) prof[1] = gtimer();
+
+    // ---- epilogue: bias and head gradients of this replica summed into grads (zeroed by the host);
+    //      the weight-matrix gradients come from vpps_dw_gemm (L185) ----
+#pragma unroll
+    for (int k = 0; k < 4; ++k)
+#pragma unroll
+        for (int s = 8; s >= 1; s >>= 1) dbacc[k] += __shfl_xor_sync(FULLMASK, dbacc[k], s);
+    if (gl == 0) {
+#pragma unroll
+        for (int k = 0; k < 3; ++k) atomicAdd(P.grads + off[5] + k * H + j, dbacc[k]);
+        atomicAdd(P.grads + off[6] + j, dbacc[3]);
+    }
+    if (holds_head) {
+        __syncthreads();
+        for (int i = tid; i < C * H; i += NTH) atomicAdd(P.grads + off[4] + i, dWo[i]);
+        for (int i = tid; i < C; i += NTH) atomicAdd(P.grads + off[7] + i, dbo[i]);
+    }
+}
+
+// ---- dW = Σ_nodes g xᵀ per weight matrix ("concatenate all the left hand side and all the
+//      right hand side tensors that participate in the outer-product for each weight matrix, and use
+//      dense matrix-matrix multiplication"), fused with SGD (L129, L197) or written to grads ----
+struct GemmParams {
+    const float* pool;
+    const float* inputs;
+    float* params;
+    float* grads;
+    const uint32_t* int_nodes;   // n_int x (rec, rec_l, rec_r)
+    const uint32_t* leaf_nodes;  // n_leaf x (rec, token)
+    int32_t n_int, n_leaf, H, E, mode;
+    int64_t off[8];
+    int64_t n_floats;
+    float lr, wd;
+    int32_t tiles[4];            // tiles per matrix (U_iou, U_fl, U_fr, W_iou)
+};
+
+constexpr int GT = 64;           // tile rows / cols
+constexpr int GK = 16;           // nodes per K step
+
+__global__ void __launch_bounds__(256) vpps_dw_gemm(const GemmParams P) {
+    __shared__ __align__(16) float Gs[2][GK][GT];
+    __shared__ __align__(16) float Xs[2][GK][GT];
+    const int tid = threadIdx.x, H = P.H, E = P.E;
+    int b = blockIdx.x, m = 0;
+    while (m < 4 && b >= P.tiles[m]) { b -= P.tiles[m]; ++m; }
+    if (m == 4) {
+        // elementwise SGD of the parameters the GEMM tiles do not cover (W_out and the biases)
+        if (P.mode == 1) {
+            const int64_t lo = P.off[4], hi = P.n_floats;
+            for (int64_t i = (int64_t)b * 256 + tid; i < hi - lo; i += (int64_t)256 * (gridDim.x - (P.tiles[0] + P.tiles[1] + P.tiles[2] + P.tiles[3]))) {
+                const float w = P.params[lo + i];
+                P.params[lo + i] = w - P.lr * (P.grads[lo + i] + P.wd * w);
+            }
+        }
+        return;
+    }
+    const int rows = (m == 0 || m == 3) ? 3 * H : H;
+    const int cols = m == 0 ? 2 * H : (m == 3 ? E : H);
+    const int tiles_c = cols / GT;
+    const int r0 = (b / tiles_c) * GT, c0 = (b % tiles_c) * GT;
+    const int K = m == 3 ? P.n_leaf : P.n_int;
+    const int goff = m == 0 ? 7 * H : (m == 1 ? 10 * H : (m == 2 ? 11 * H : 5 * H));
+    const int ty = tid / 16, tx = tid % 16;
+    float acc[4][4];
+#pragma unroll
+    for (int a = 0; a < 4; ++a)
+#pragma unroll
+        for (int c = 0; c < 4; ++c) acc[a][c] = 0.f;
+    // stage K-step s into buffer buf: 16 nodes x 64 rows of g and 16 nodes x 64 cols of x (cp.async)
+    auto stage = [&](int s, int buf) {
+        const int k = tid / 16, piece = (tid % 16) * 4;
+        const int node = s * GK + k;
+        const float* gsrc = nullptr;
+        const float* xsrc = nullptr;
+        if (node < K) {
+            if (m == 3) {
+                const uint32_t rec = P.leaf_nodes[2 * node], tok = P.leaf_nodes[2 * node + 1];
+                gsrc = P.pool + rec + goff + r0 + piece;
+                xsrc = P.inputs + (int64_t)tok * E + c0 + piece;
+            } else {
+                const uint32_t rec = P.int_nodes[3 * node];
+                const uint32_t xl = P.int_nodes[3 * node + 1], xr = P.int_nodes[3 * node + 2];
+                gsrc = P.pool + rec + goff + r0 + piece;
+                const int c = c0 + piece;
+                if (m == 0) xsrc = c < H ? P.pool + xl + c : P.pool + xr + (c - H);
+                else xsrc = P.pool + (m == 1 ? xl : xr) + c;
+            }
+        }
+        cp_async16(&Gs[buf][k][piece], gsrc ? gsrc : P.pool, gsrc ? 16u : 0u);
+        cp_async16(&Xs[buf][k][piece], xsrc ? xsrc : P.pool, xsrc ? 16u : 0u);
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    const int steps = (K + GK - 1) / GK;
+    if (steps > 0) stage(0, 0);
+    for (int s = 0; s < steps; ++s) {
+        if (s + 1 < steps) {
+            stage(s + 1, (s + 1) & 1);
+            asm volatile("cp.async.wait_group 1;" ::: "memory");
+        } else {
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
+        }
+        __syncthreads();
+        const int buf = s & 1;
+#pragma unroll
+        for (int k = 0; k < GK; ++k) {
+            const float4 gv = *reinterpret_cast<const float4*>(&Gs[buf][k][ty * 4]);
+            const float4 xv = *reinterpret_cast<const float4*>(&Xs[buf][k][tx * 4]);
+            const float ga[4] = {gv.x, gv.y, gv.z, gv.w}, xa[4] = {xv.x, xv.y, xv.z, xv.w};
+#pragma unroll
+            for (int a = 0; a < 4; ++a)
+#pragma unroll
+                for (int c = 0; c < 4; ++c) acc[a][c] = fmaf(ga[a], xa[c], acc[a][c]);
+        }
+        __syncthreads();
+    }
+    const int64_t base = P.off[m == 3 ? 0 : m + 1];
+#pragma unroll
+    for (int a = 0; a < 4; ++a)
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+            const int64_t idx = base + (int64_t)(r0 + ty * 4 + a) * cols + c0 + tx * 4 + c;
+            if (P.mode == 1) {
+                const float w = P.params[idx];
+                P.params[idx] = w - P.lr * (acc[a][c] + P.wd * w);
+            } else {
+                P.grads[idx] = acc[a][c];
+            }
+        }
+}
+
+}  // namespace cl
+}  // namespace dev
+
+#define VPPS_CLUSTER_VARIANT(H, E) \
+    {1, H, E, 16, (const void*)&dev::cl::vpps_cl<H, E>, &dev::cl::CCfg<H, E>::smem_bytes}
+
+static const Variant kClusterVariants[] = {
+    VPPS_CLUSTER_VARIANT(256, 256),    // target: binary Tree-LSTM H = E = 256, 16-CTA clusters
+};
+
+const Variant* cluster_variants(int32_t* n) {
+    *n = (int32_t)(sizeof(kClusterVariants) / sizeof(kClusterVariants[0]));
+    return kClusterVariants;
+}
+
+void launch_dw_gemm(const float* pool, const float* inputs, float* params, float* grads, const uint32_t* int_nodes,
+                    int32_t n_int, const uint32_t* leaf_nodes, int32_t n_leaf, int32_t H, int32_t E,
+                    const int64_t* off, int64_t n_floats, int32_t mode, float lr, float wd, cudaStream_t s) {
+    dev::cl::GemmParams g{};
+    g.pool = pool; g.inputs = inputs; g.params = params; g.grads = grads;
+    g.int_nodes = int_nodes; g.leaf_nodes = leaf_nodes; g.n_int = n_int; g.n_leaf = n_leaf;
+    g.H = H; g.E = E; g.mode = mode; g.n_floats = n_floats; g.lr = lr; g.wd = wd;
+    for (int i = 0; i < 8; ++i) g.off[i] = off[i];
+    g.tiles[0] = (3 * H / dev::cl::GT) * (2 * H / dev::cl::GT);
+    g.tiles[1] = (H / dev::cl::GT) * (H / dev::cl::GT);
+    g.tiles[2] = g.tiles[1];
+    g.tiles[3] = (3 * H / dev::cl::GT) * (E / dev::cl::GT);
+    const int tiles = g.tiles[0] + g.tiles[1] + g.tiles[2] + g.tiles[3];
+    dev::cl::vpps_dw_gemm<<<tiles + 16, 256, 0, s>>>(g);
+}
+
+}  // namespace vpps

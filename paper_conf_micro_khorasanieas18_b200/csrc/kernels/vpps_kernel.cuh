@@ -29,6 +29,12 @@ struct Variant {
 
 // Table of compiled specialisations (vpps_kernel.cu).
 const Variant* variants(int32_t* n);
+// Cluster-replica specialisations (vpps_cluster.cu); Variant.umax holds the cluster size.
+const Variant* cluster_variants(int32_t* n);
+// dW = Σ g xᵀ per weight matrix from the recorded operands, fused SGD when mode == 1.
+void launch_dw_gemm(const float* pool, const float* inputs, float* params, float* grads, const uint32_t* int_nodes,
+                    int32_t n_int, const uint32_t* leaf_nodes, int32_t n_leaf, int32_t H, int32_t E,
+                    const int64_t* off, int64_t n_floats, int32_t mode, float lr, float wd, cudaStream_t s);
 // Elementwise SGD on the flat buffer (K3): p -= lr * (g + wd * p).
 void launch_sgd(float* p, const float* g, int64_t n, float lr, float wd, cudaStream_t s);
 

@@ -20,13 +20,13 @@ def _vpps():
     return vpps
 
 
-def run_case(cell, H, E, C, graphs, V, seed=0, want_dx=True, sgd=None, groups=1):
+def run_case(cell, H, E, C, graphs, V, seed=0, want_dx=True, sgd=None, groups=1, cluster=0):
     vpps = _vpps()
     rng = np.random.default_rng(seed)
     shapes = vpps.param_shapes(cell, H, E, C)
     P = synth.init_params(shapes, rng)
     X = synth.input_table(rng, V, E)
-    m = vpps.Model(cell, H, E, C, device=0, groups=groups)
+    m = vpps.Model(cell, H, E, C, device=0, groups=groups, cluster=cluster)
     dev = torch.device("cuda:0")
     params = torch.zeros(m.n_floats, dtype=torch.float32, device=dev)
     grads = torch.full_like(params, float("nan"))
@@ -50,8 +50,9 @@ def rel(a, b):
     return float(np.abs(np.asarray(a, np.float64) - b).max() / max(np.abs(b).max(), 1e-30))
 
 
-def check(cell, H, E, C, graphs, V, seed=0, want_dx=True, groups=1):
-    m, P, X, loss, params, grads, dX = run_case(cell, H, E, C, graphs, V, seed, want_dx, groups=groups)
+def check(cell, H, E, C, graphs, V, seed=0, want_dx=True, groups=1, cluster=0):
+    m, P, X, loss, params, grads, dX = run_case(cell, H, E, C, graphs, V, seed, want_dx, groups=groups,
+                                                cluster=cluster)
     lo, Go, dXo = M.forward_backward(cell, P, X, graphs, H)
     assert abs(loss - lo) <= TOL * abs(lo), (loss, lo)
     gv = m.views(grads.cpu())
@@ -83,12 +84,23 @@ def test_binary_target_replica_groups(groups):
     check("binary", 256, 256, 5, synth.config_batch("tgt", 3), 4096, seed=5, groups=groups)
 
 
-@pytest.mark.parametrize("groups", [1, 2, 4])
-def test_fused_sgd_target_groups(groups):
+@pytest.mark.parametrize("b", [0, 5])
+def test_binary_target_cluster_replicas(b):
+    """Cluster path: 16-CTA cluster replicas, whole trees per cluster, dW by the gradient GEMM (L185)."""
+    check("binary", 256, 256, 5, synth.config_batch("tgt", b), 4096, seed=11 + b, cluster=16)
+
+
+def test_cluster_degenerate_batches():
+    check("binary", 256, 256, 5, [[((), 3, 2)]], 8, cluster=16)              # one leaf: most clusters idle
+    check("binary", 256, 256, 5, _trees(12, 3, (1, 9), 30, 5), 30, cluster=16, want_dx=False)
+
+
+@pytest.mark.parametrize("groups,cluster", [(1, 0), (2, 0), (4, 0), (1, 16)])
+def test_fused_sgd_target_groups(groups, cluster):
     graphs = synth.config_batch("tgt", 4)
     lr, wd = 0.05, 1e-3
     m, P, X, loss, params, grads, dX = run_case("binary", 256, 256, 5, graphs, 4096, seed=6, sgd=(lr, wd),
-                                                groups=groups)
+                                                groups=groups, cluster=cluster)
     lo, Go, _ = M.forward_backward("binary", P, X, graphs, 256)
     Pn = M.sgd(P, Go, lr, wd)
     pv = m.views(params.cpu())

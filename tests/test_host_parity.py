@@ -109,6 +109,36 @@ def test_script_words_bit_exact(vpps, cell, G):
         assert info["flops"] == M.flop_count(cell, graphs, H, E, C)
 
 
+@pytest.mark.parametrize("cell", ["binary", "lstm", "childsum"])
+def test_script_words_bit_exact_graph_groups(vpps, cell):
+    """SPEC S5g (cluster replicas): whole graphs per group, min-load over graph MACs."""
+    H, E, C = 16, 16, 7
+    m = vpps.Model(cell, H, E, C, n_sm=7 * 16, groups=7, cluster=16, plan_only=True)
+    assert m.plan_info()["n_g"] == 16
+    rng = np.random.default_rng(77)
+    for graphs in _batches(cell, rng, 10):
+        s = m.build_script(graphs)
+        ref = oscript.build(cell, graphs, H, E, C, G=7, n_act=m.plan_info()["n_act"], by_graph=True)
+        assert np.array_equal(s.words(), np.array(ref["words"], dtype=np.uint32))
+
+
+def test_graph_groups_keep_graphs_whole():
+    graphs = synth.tree_batch(np.random.default_rng(5), 9, (2, 12), 50, 5)
+    ref = oscript.build("binary", graphs, 8, 8, 5, G=4, n_act=9, by_graph=True)
+    w = ref["words"]
+    G = w[0]
+    pre = w[2:2 + G + 1]
+    base = 2 + G + 1
+    owner = {}
+    for g in range(G):
+        st = w[base + pre[g]: base + pre[g + 1]]
+        # every record operand in group g's stream belongs to a graph owned by g
+        for x in st:
+            if x in ref["rec"]:
+                gid = ref["nodes"][ref["rec"].index(x)]["graph"]
+                assert owner.setdefault(gid, g) == g
+
+
 def test_script_words_target_config(vpps):
     """TGT shapes (binary H = E = 256, batch 16 SST-shaped trees) on 148 SMs."""
     m = vpps.Model("binary", 256, 256, 5, n_sm=148, plan_only=True)
