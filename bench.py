@@ -164,6 +164,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--groups", type=int, default=4, help="replica groups G (SPEC P1); 148 = 4 x 37")
+    ap.add_argument("--cluster", type=int, default=16,
+                    help="> 1: cluster-replica path (one 16-CTA cluster per replica, SPEC S5g)")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
 
@@ -188,7 +190,7 @@ def main():
     shapes = vpps.param_shapes("binary", H, E, C)
     P = synth.init_params(shapes, rng)
     X = synth.input_table(rng, V, E)
-    m = vpps.Model("binary", H, E, C, device=local, groups=args.groups)
+    m = vpps.Model("binary", H, E, C, device=local, groups=args.groups, cluster=args.cluster)
     params = torch.zeros(m.n_floats, dtype=torch.float32, device=dev)
     grads = torch.zeros_like(params)
     for name, _ in shapes:
@@ -294,11 +296,13 @@ def main():
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "impl": "vpps",
             "config": {"workload": WORKLOAD, "global_batch": args.batch * world, "per_gpu_batch": args.batch,
-                       "seq_len": None, "parallelism": f"dp{world}", "replica_groups": args.groups,
+                       "seq_len": None, "parallelism": f"dp{world}",
+                       "replica_groups": m.plan_info()["n_cta"] // m.plan_info()["n_g"],
+                       "cluster": args.cluster or None, "ctas": m.plan_info()["n_cta"],
                        "mode": "fused fwd-bwd-sgd, 1 kernel" if world == 1 else "fwd_bwd + NCCL all-reduce + sgd",
                        "l2": "no flush" if args.no_flush else "flushed (256 MiB write) before every timed step",
                        "batches": f"{N_BATCHES} distinct pre-built scripts cycled"},
-            "gpu_launches": args.steps * (1 if world == 1 else 2),
+            "gpu_launches": args.steps * ((2 if args.cluster else 1) + (0 if world == 1 else 1)),
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "kernel_ms": kern_ms / args.steps, "flops_per_launch": avg_flops,

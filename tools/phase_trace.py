@@ -24,6 +24,7 @@ def main():
     ap.add_argument("--groups", type=int, default=1)
     ap.add_argument("--quiet", action="store_true")
     ap.add_argument("--sections", action="store_true")
+    ap.add_argument("--cluster", type=int, default=0)
     args = ap.parse_args()
     import torch
     import synth
@@ -33,7 +34,7 @@ def main():
     rng = np.random.default_rng(0)
     shapes = vpps.param_shapes(cell, H, E, C)
     P = synth.init_params(shapes, rng)
-    m = vpps.Model(cell, H, E, C, groups=args.groups)
+    m = vpps.Model(cell, H, E, C, groups=args.groups, cluster=args.cluster)
     params = torch.zeros(m.n_floats, device="cuda")
     grads = torch.zeros_like(params)
     for n, _ in shapes:
