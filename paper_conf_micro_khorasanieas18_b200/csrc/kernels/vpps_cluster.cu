@@ -551,78 +551,78 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
 
 // ---- dW = Σ_nodes g xᵀ per weight matrix ("concatenate all the left hand side and all the
 //      right hand side tensors that participate in the outer-product for each weight matrix, and use
-//      dense matrix-matrix multiplication"), fused with SGD (L129, L197) or written to grads ----
+//      dense matrix-matrix multiplication").  Split-K: one CTA per (128 x 64 tile, chunk of KCH nodes);
+//      partial tiles are summed into grads (zeroed by the host) with vector L2 reductions; the SGD update
+//      (L129, L197) follows as one elementwise pass over the flat parameters ----
 struct GemmParams {
     const float* pool;
     const float* inputs;
-    float* params;
     float* grads;
     const uint32_t* int_nodes;   // n_int x (rec, rec_l, rec_r)
     const uint32_t* leaf_nodes;  // n_leaf x (rec, token)
-    int32_t n_int, n_leaf, H, E, mode;
+    int32_t n_int, n_leaf, H, E;
     int64_t off[8];
-    int64_t n_floats;
-    float lr, wd;
-    int32_t tiles[4];            // tiles per matrix (U_iou, U_fl, U_fr, W_iou)
+    int32_t items[4];            // work items per matrix (U_iou, U_fl, U_fr, W_iou)
 };
 
-constexpr int GT = 64;           // tile rows / cols
-constexpr int GK = 16;           // nodes per K step
+constexpr int TM = 128;          // tile rows (gate-gradient rows)
+constexpr int TN = 64;           // tile cols (input columns)
+constexpr int KS = 16;           // nodes per pipeline stage
+constexpr int KCH = 96;          // nodes per work item (split-K)
 
 __global__ void __launch_bounds__(256) vpps_dw_gemm(const GemmParams P) {
-    __shared__ __align__(16) float Gs[2][GK][GT];
-    __shared__ __align__(16) float Xs[2][GK][GT];
+    __shared__ __align__(16) float Gs[2][KS][TM];
+    __shared__ __align__(16) float Xs[2][KS][TN];
     const int tid = threadIdx.x, H = P.H, E = P.E;
     int b = blockIdx.x, m = 0;
-    while (m < 4 && b >= P.tiles[m]) { b -= P.tiles[m]; ++m; }
-    if (m == 4) {
-        // elementwise SGD of the parameters the GEMM tiles do not cover (W_out and the biases)
-        if (P.mode == 1) {
-            const int64_t lo = P.off[4], hi = P.n_floats;
-            for (int64_t i = (int64_t)b * 256 + tid; i < hi - lo; i += (int64_t)256 * (gridDim.x - (P.tiles[0] + P.tiles[1] + P.tiles[2] + P.tiles[3]))) {
-                const float w = P.params[lo + i];
-                P.params[lo + i] = w - P.lr * (P.grads[lo + i] + P.wd * w);
-            }
-        }
-        return;
-    }
+    while (m < 4 && b >= P.items[m]) { b -= P.items[m]; ++m; }
+    if (m == 4) return;
     const int rows = (m == 0 || m == 3) ? 3 * H : H;
     const int cols = m == 0 ? 2 * H : (m == 3 ? E : H);
-    const int tiles_c = cols / GT;
-    const int r0 = (b / tiles_c) * GT, c0 = (b % tiles_c) * GT;
     const int K = m == 3 ? P.n_leaf : P.n_int;
+    const int tiles_r = rows / TM, tiles_c = cols / TN;
+    const int kc = b / (tiles_r * tiles_c), t = b - kc * (tiles_r * tiles_c);
+    const int r0 = (t / tiles_c) * TM, c0 = (t % tiles_c) * TN;
+    const int k0 = kc * KCH, k1 = min(K, k0 + KCH);
     const int goff = m == 0 ? 7 * H : (m == 1 ? 10 * H : (m == 2 ? 11 * H : 5 * H));
-    const int ty = tid / 16, tx = tid % 16;
-    float acc[4][4];
+    const int ty = tid / 16, tx = tid % 16;        // rows ty*8 .. +7, cols tx*4 .. +3
+    float acc[8][4];
 #pragma unroll
-    for (int a = 0; a < 4; ++a)
+    for (int a = 0; a < 8; ++a)
 #pragma unroll
         for (int c = 0; c < 4; ++c) acc[a][c] = 0.f;
-    // stage K-step s into buffer buf: 16 nodes x 64 rows of g and 16 nodes x 64 cols of x (cp.async)
+    // stage: KS nodes x 128 rows of g (2 x 16 B per thread) and KS nodes x 64 cols of x (16 B per thread)
     auto stage = [&](int s, int buf) {
-        const int k = tid / 16, piece = (tid % 16) * 4;
-        const int node = s * GK + k;
-        const float* gsrc = nullptr;
-        const float* xsrc = nullptr;
-        if (node < K) {
-            if (m == 3) {
-                const uint32_t rec = P.leaf_nodes[2 * node], tok = P.leaf_nodes[2 * node + 1];
-                gsrc = P.pool + rec + goff + r0 + piece;
-                xsrc = P.inputs + (int64_t)tok * E + c0 + piece;
-            } else {
-                const uint32_t rec = P.int_nodes[3 * node];
-                const uint32_t xl = P.int_nodes[3 * node + 1], xr = P.int_nodes[3 * node + 2];
-                gsrc = P.pool + rec + goff + r0 + piece;
-                const int c = c0 + piece;
-                if (m == 0) xsrc = c < H ? P.pool + xl + c : P.pool + xr + (c - H);
-                else xsrc = P.pool + (m == 1 ? xl : xr) + c;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int e = tid + h * 256, k = e / 32, piece = (e % 32) * 4;
+            const int node = k0 + s * KS + k;
+            const float* src = nullptr;
+            if (node < k1) {
+                const uint32_t rec = m == 3 ? P.leaf_nodes[2 * node] : P.int_nodes[3 * node];
+                src = P.pool + rec + goff + r0 + piece;
             }
+            cp_async16(&Gs[buf][k][piece], src ? src : P.pool, src ? 16u : 0u);
         }
-        cp_async16(&Gs[buf][k][piece], gsrc ? gsrc : P.pool, gsrc ? 16u : 0u);
-        cp_async16(&Xs[buf][k][piece], xsrc ? xsrc : P.pool, xsrc ? 16u : 0u);
+        {
+            const int k = tid / 16, piece = (tid % 16) * 4;
+            const int node = k0 + s * KS + k;
+            const float* src = nullptr;
+            if (node < k1) {
+                const int c = c0 + piece;
+                if (m == 3) {
+                    src = P.inputs + (int64_t)P.leaf_nodes[2 * node + 1] * E + c;
+                } else {
+                    const uint32_t xl = P.int_nodes[3 * node + 1], xr = P.int_nodes[3 * node + 2];
+                    if (m == 0) src = c < H ? P.pool + xl + c : P.pool + xr + (c - H);
+                    else src = P.pool + (m == 1 ? xl : xr) + c;
+                }
+            }
+            cp_async16(&Xs[buf][k][piece], src ? src : P.pool, src ? 16u : 0u);
+        }
         asm volatile("cp.async.commit_group;" ::: "memory");
     };
-    const int steps = (K + GK - 1) / GK;
+    const int steps = (k1 - k0 + KS - 1) / KS;
     if (steps > 0) stage(0, 0);
     for (int s = 0; s < steps; ++s) {
         if (s + 1 < steps) {
@@ -634,30 +634,23 @@ __global__ void __launch_bounds__(256) vpps_dw_gemm(const GemmParams P) {
         __syncthreads();
         const int buf = s & 1;
 #pragma unroll
-        for (int k = 0; k < GK; ++k) {
-            const float4 gv = *reinterpret_cast<const float4*>(&Gs[buf][k][ty * 4]);
+        for (int k = 0; k < KS; ++k) {
+            const float4 g0 = *reinterpret_cast<const float4*>(&Gs[buf][k][ty * 8]);
+            const float4 g1 = *reinterpret_cast<const float4*>(&Gs[buf][k][ty * 8 + 4]);
             const float4 xv = *reinterpret_cast<const float4*>(&Xs[buf][k][tx * 4]);
-            const float ga[4] = {gv.x, gv.y, gv.z, gv.w}, xa[4] = {xv.x, xv.y, xv.z, xv.w};
+            const float ga[8] = {g0.x, g0.y, g0.z, g0.w, g1.x, g1.y, g1.z, g1.w};
+            const float xa[4] = {xv.x, xv.y, xv.z, xv.w};
 #pragma unroll
-            for (int a = 0; a < 4; ++a)
+            for (int a = 0; a < 8; ++a)
 #pragma unroll
                 for (int c = 0; c < 4; ++c) acc[a][c] = fmaf(ga[a], xa[c], acc[a][c]);
         }
         __syncthreads();
     }
-    const int64_t base = P.off[m == 3 ? 0 : m + 1];
+    if (steps == 0) return;
+    float* base = P.grads + P.off[m == 3 ? 0 : m + 1];
 #pragma unroll
-    for (int a = 0; a < 4; ++a)
-#pragma unroll
-        for (int c = 0; c < 4; ++c) {
-            const int64_t idx = base + (int64_t)(r0 + ty * 4 + a) * cols + c0 + tx * 4 + c;
-            if (P.mode == 1) {
-                const float w = P.params[idx];
-                P.params[idx] = w - P.lr * (acc[a][c] + P.wd * w);
-            } else {
-                P.grads[idx] = acc[a][c];
-            }
-        }
+    for (int a = 0; a < 8; ++a) red_add<4>(base + (int64_t)(r0 + ty * 8 + a) * cols + c0 + tx * 4, acc[a]);
 }
 
 }  // namespace cl
@@ -678,17 +671,20 @@ const Variant* cluster_variants(int32_t* n) {
 void launch_dw_gemm(const float* pool, const float* inputs, float* params, float* grads, const uint32_t* int_nodes,
                     int32_t n_int, const uint32_t* leaf_nodes, int32_t n_leaf, int32_t H, int32_t E,
                     const int64_t* off, int64_t n_floats, int32_t mode, float lr, float wd, cudaStream_t s) {
-    dev::cl::GemmParams g{};
-    g.pool = pool; g.inputs = inputs; g.params = params; g.grads = grads;
+    using namespace dev::cl;
+    GemmParams g{};
+    g.pool = pool; g.inputs = inputs; g.grads = grads;
     g.int_nodes = int_nodes; g.leaf_nodes = leaf_nodes; g.n_int = n_int; g.n_leaf = n_leaf;
-    g.H = H; g.E = E; g.mode = mode; g.n_floats = n_floats; g.lr = lr; g.wd = wd;
+    g.H = H; g.E = E;
     for (int i = 0; i < 8; ++i) g.off[i] = off[i];
-    g.tiles[0] = (3 * H / dev::cl::GT) * (2 * H / dev::cl::GT);
-    g.tiles[1] = (H / dev::cl::GT) * (H / dev::cl::GT);
-    g.tiles[2] = g.tiles[1];
-    g.tiles[3] = (3 * H / dev::cl::GT) * (E / dev::cl::GT);
-    const int tiles = g.tiles[0] + g.tiles[1] + g.tiles[2] + g.tiles[3];
-    dev::cl::vpps_dw_gemm<<<tiles + 16, 256, 0, s>>>(g);
+    const int ki = (n_int + KCH - 1) / KCH, kl = (n_leaf + KCH - 1) / KCH;
+    g.items[0] = (3 * H / TM) * (2 * H / TN) * ki;
+    g.items[1] = (H / TM) * (H / TN) * ki;
+    g.items[2] = g.items[1];
+    g.items[3] = (3 * H / TM) * (E / TN) * kl;
+    const int items = g.items[0] + g.items[1] + g.items[2] + g.items[3];
+    if (items > 0) vpps_dw_gemm<<<items, 256, 0, s>>>(g);
+    if (mode == 1) launch_sgd(params, grads, n_floats, lr, wd, s);   // W -= lr (dW + wd W), every parameter
 }
 
 }  // namespace vpps
