@@ -394,9 +394,16 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         cfg.stream = st;
         cfg.attrs = attr;
         cfg.numAttrs = 1;
-        CK(cudaLaunchKernelExC(&cfg, m->var->fn, args));
-        // dW of the weight matrices from the recorded operands, fused SGD in mode 1
         const uint32_t* lists = dwords + s->s.words.size();
+        const uint32_t* leaf_list = lists + 3 * s->s.n_int;
+        const float* W_iou = m->params + m->offsets[0];
+        // level 0 (all leaves share W_iou on their word vectors) as one dense GEMM + cell pass
+        launch_leaf_fwd(W_iou, m->params + m->offsets[5], inputs, m->pool, leaf_list, (int32_t)s->s.n_leaf,
+                        m->plan.H, m->plan.E, st);
+        CK(cudaLaunchKernelExC(&cfg, m->var->fn, args));
+        // dX of the leaves = W_iouᵀ g_leaf (words are inputs), then dW of the weight matrices
+        // from the recorded operands, fused SGD in mode 1
+        launch_leaf_dx(W_iou, m->pool, d_inputs, leaf_list, (int32_t)s->s.n_leaf, m->plan.H, m->plan.E, st);
         launch_dw_gemm(m->pool, inputs, m->params, m->grads, lists, (int32_t)s->s.n_int, lists + 3 * s->s.n_int,
                        (int32_t)s->s.n_leaf, m->plan.H, m->plan.E, m->offsets.data(), m->n_floats, mode, lr, wd, st);
         CK(cudaGetLastError());

@@ -19,7 +19,7 @@ namespace cl {
 constexpr int NTH = 256;
 constexpr int CHUNK = 4096;    // script words staged in shared memory (L171)
 constexpr int NB = 16;         // nodes per batch: one node per lane of a unit's 16-lane group
-constexpr int NC = 4;          // nodes per transposed-product chunk
+constexpr int NC = 2;          // nodes per transposed-product chunk
 constexpr int ZC = 32;         // classes per head (C <= 32)
 constexpr int CINMAX = 10;
 constexpr uint32_t NONE = 0xFFFFFFFFu;
@@ -97,7 +97,7 @@ struct CCfg {
     static constexpr int KPMAX = LA::KP > LB::KP ? LA::KP : LB::KP;
     static constexpr int O_X = CHUNK;
     static constexpr int O_DXB = O_X + NB * KPMAX;
-    static constexpr int O_CIN = O_DXB + 8 * NC * KPMAX;
+    static constexpr int O_CIN = O_DXB + UM * NC * KPMAX;
     static constexpr int O_BIAS = O_CIN + NB * UM * CINMAX;
     static constexpr int O_IPOS = O_BIAS + UM * 4;
     static constexpr int O_BST = O_IPOS + NB;
@@ -144,16 +144,9 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
     const bool holds_head = (lc == H % NCL);
 
     // ---- prologue: this CTA's slice of every weight matrix DRAM -> registers (L123, L129) ----
-    float wa[3][LA::NREG], wb[4][LB::NREG];
-#pragma unroll
-    for (int r = 0; r < 3; ++r)
-#pragma unroll
-        for (int t = 0; t < LA::NT; ++t)
-#pragma unroll
-            for (int q = 0; q < LA::CG; ++q) {
-                const int col = LA::CG * (tu + TU * t) + q;
-                wa[r][t * LA::CG + q] = col < E ? __ldg(P.params + off[0] + (int64_t)(r * H + j) * E + col) : 0.f;
-            }
+    // Only the recurrent matrices (U_iou, U_fl, U_fr) live in registers: the leaf level is one dense
+    // GEMM over all leaves (same W_iou), done by vpps_leaf_fwd / vpps_leaf_dx around this kernel.
+    float wb[4][LB::NREG];
 #pragma unroll
     for (int r = 0; r < 4; ++r)
 #pragma unroll
@@ -178,8 +171,32 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
     }
     float dbacc[4] = {0.f, 0.f, 0.f, 0.f};       // bias gradients of (unit u) over the nodes of slot gl
     uint64_t* prof = P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
+    // section clocks (trace only): 0 decode, 1 staging, 2 forward, 3 cell-bwd, 4 transposed, 5 heads,
+    // 6 signal, 7 wait, 8/9 other
+    uint64_t sec[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
+    uint64_t sec_last = 0;
+    int sec_cur = 9;
+    auto mark = [&](int k) {
+        if (prof && tid == 0) {
+            const uint64_t now = clock64(), d = now - sec_last;
+            switch (sec_cur) {
+                case 0: sec[0] += d; break;
+                case 1: sec[1] += d; break;
+                case 2: sec[2] += d; break;
+                case 3: sec[3] += d; break;
+                case 4: sec[4] += d; break;
+                case 5: sec[5] += d; break;
+                case 6: sec[6] += d; break;
+                case 7: sec[7] += d; break;
+                case 8: sec[8] += d; break;
+                default: sec[9] += d; break;
+            }
+            sec_cur = k;
+            sec_last = now;
+        }
+    };
     __syncthreads();
-    if (prof && tid == 0) prof[0] = gtimer();
+    if (prof && tid == 0) { prof[0] = gtimer(); sec_last = clock64(); }
 
     // ---- script interpretation (L171-177) ----
     uint32_t cbase = s0;
@@ -205,18 +222,29 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
         const uint32_t pre = chunk[pos - cbase];
         const uint32_t op = pre & 0xFF;
         if (op == S) {            // signal (L165): arrive on the cluster barrier, release our writes
-            if (prof && tid == 0) prof[2 + 3 * (pre >> 8)] = gtimer();
+            mark(6);
+            if (prof && tid == 0) {
+                prof[2 + 3 * (pre >> 8)] = gtimer();
+                uint64_t* o = prof + 2 + 3 * (S_[1] + 1) + 10 + 10 * (pre >> 8);
+#pragma unroll
+                for (int k = 0; k < 10; ++k) o[k] = sec[k];
+            }
             cluster_arrive();
             pending = true;
             ++pos;
             continue;
         }
         if (op == W) {            // wait (L165): all 16 CTAs of the replica have signalled
+            mark(7);
             if (prof && tid == 0) prof[3 + 3 * (pre >> 8)] = gtimer();
             cluster_wait();
             pending = false;
             if (prof && tid == 0) prof[4 + 3 * (pre >> 8)] = gtimer();
             ++pos;
+            continue;
+        }
+        if (op == LEAF_F) {       // leaf cells were computed by vpps_leaf_fwd (one GEMM over all leaves)
+            pos += 3;
             continue;
         }
         const bool is_head = (op == HEAD_F || op == HEAD_B);
@@ -225,6 +253,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
         const int KP = kindB ? LB::KP : LA::KP;
         // ---- decode (warp 0): up to NB consecutive instructions with this opcode + row sources ----
         __syncthreads();
+        mark(0);
         if (warp == 0) {
             const uint32_t lim = min(s1, cbase + (uint32_t)CHUNK);
             const uint32_t sz = (uint32_t)words(pre);
@@ -248,6 +277,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
         __syncthreads();
         const int nb = bst[0];
         const uint32_t p = (uint32_t)bst[1];
+        mark(1);
         // ---- staging: cp.async of every input row and cell operand of the batch (one round trip) ----
         {
             const int q4 = KP / 4;
@@ -270,6 +300,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
         }
         __syncthreads();
 
+        mark(is_head ? 5 : (fwd ? 2 : 3));
         if (is_head) {            // loss heads (L42) on the CTA holding W_out
             if (holds_head) {
                 if (op == HEAD_F) {
@@ -333,93 +364,56 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
         }
 
         if (fwd) {
-            // ---- forward: matvec from registers (L123), 4 nodes at a time; the unit's 16 lanes reduce
-            //      with a transposed butterfly and the lane holding node n's gates does its cell update ----
+            // ---- forward of internal cells: matvec from registers (L123), 4 nodes at a time; the unit's
+            //      16 lanes reduce with a transposed butterfly and the lane holding node n's gates does its
+            //      cell update ----
             for (int n0 = 0; n0 < nb; n0 += 4) {
-                float v[4][5];
-                if (kindB) {
-                    float2 a[4][5];
+                float2 a[4][5];
 #pragma unroll
-                    for (int n = 0; n < 4; ++n)
+                for (int n = 0; n < 4; ++n)
 #pragma unroll
-                        for (int o = 0; o < 5; ++o) a[n][o] = make_float2(0.f, 0.f);
+                    for (int o = 0; o < 5; ++o) a[n][o] = make_float2(0.f, 0.f);
 #pragma unroll
-                    for (int t = 0; t < LB::NT; ++t) {
-                        const int col0 = LB::CG * (tu + TU * t);
-                        const int of = col0 < H ? 3 : 4;
-#pragma unroll
-                        for (int n = 0; n < 4; ++n) {
-                            float xv[LB::CG];
-                            lds<LB::CG>(xs + (n0 + n) * LB::KP + col0, xv);
-#pragma unroll
-                            for (int q = 0; q < LB::CG; q += 2) {
-                                const float2 x2 = make_float2(xv[q], xv[q + 1]);
-                                const int k = t * LB::CG + q;
-#pragma unroll
-                                for (int r = 0; r < 3; ++r)
-                                    a[n][r] = __ffma2_rn(make_float2(wb[r][k], wb[r][k + 1]), x2, a[n][r]);
-                                const float2 f2 = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), x2, make_float2(0.f, 0.f));
-                                if (of == 3) { a[n][3].x += f2.x; a[n][3].y += f2.y; }
-                                else { a[n][4].x += f2.x; a[n][4].y += f2.y; }
-                            }
-                        }
-                    }
-#pragma unroll
-                    for (int n = 0; n < 4; ++n)
-#pragma unroll
-                        for (int o = 0; o < 5; ++o) v[n][o] = a[n][o].x + a[n][o].y;
-                } else {
-                    float2 a[4][3];
-#pragma unroll
-                    for (int n = 0; n < 4; ++n)
-#pragma unroll
-                        for (int o = 0; o < 3; ++o) a[n][o] = make_float2(0.f, 0.f);
-#pragma unroll
-                    for (int t = 0; t < LA::NT; ++t) {
-                        const int col0 = LA::CG * (tu + TU * t);
-#pragma unroll
-                        for (int n = 0; n < 4; ++n) {
-                            float xv[LA::CG];
-                            lds<LA::CG>(xs + (n0 + n) * LA::KP + col0, xv);
-#pragma unroll
-                            for (int q = 0; q < LA::CG; q += 2) {
-                                const float2 x2 = make_float2(xv[q], xv[q + 1]);
-                                const int k = t * LA::CG + q;
-#pragma unroll
-                                for (int r = 0; r < 3; ++r)
-                                    a[n][r] = __ffma2_rn(make_float2(wa[r][k], wa[r][k + 1]), x2, a[n][r]);
-                            }
-                        }
-                    }
+                for (int t = 0; t < LB::NT; ++t) {
+                    const int col0 = LB::CG * (tu + TU * t);
+                    const int of = col0 < H ? 3 : 4;
 #pragma unroll
                     for (int n = 0; n < 4; ++n) {
+                        float xv[LB::CG];
+                        lds<LB::CG>(xs + (n0 + n) * LB::KP + col0, xv);
 #pragma unroll
-                        for (int o = 0; o < 3; ++o) v[n][o] = a[n][o].x + a[n][o].y;
-                        v[n][3] = v[n][4] = 0.f;
+                        for (int q = 0; q < LB::CG; q += 2) {
+                            const float2 x2 = make_float2(xv[q], xv[q + 1]);
+                            const int k = t * LB::CG + q;
+#pragma unroll
+                            for (int r = 0; r < 3; ++r)
+                                a[n][r] = __ffma2_rn(make_float2(wb[r][k], wb[r][k + 1]), x2, a[n][r]);
+                            const float2 f2 = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), x2, make_float2(0.f, 0.f));
+                            if (of == 3) { a[n][3].x += f2.x; a[n][3].y += f2.y; }
+                            else { a[n][4].x += f2.x; a[n][4].y += f2.y; }
+                        }
                     }
                 }
                 float g5[5];
 #pragma unroll
-                for (int o = 0; o < 5; ++o) g5[o] = treduce4_16(v[0][o], v[1][o], v[2][o], v[3][o], gl);
+                for (int o = 0; o < 5; ++o)
+                    g5[o] = treduce4_16(a[0][o].x + a[0][o].y, a[1][o].x + a[1][o].y, a[2][o].x + a[2][o].y,
+                                        a[3][o].x + a[3][o].y, gl);
                 const int n = n0 + (gl >> 2);
                 if ((gl & 3) == 0 && n < nb) {
-                    const uint32_t* I = chunk + ipos[n];
-                    const uint32_t rec = I[1];
+                    const uint32_t rec = chunk[ipos[n] + 1];
                     const float* b = bias + u * 4;
+                    const float* cv = cin + (n * UM + u) * CINMAX;
                     const float i = sigm(g5[0] + b[0]), o = sigm(g5[1] + b[1]), uv = tanhf(g5[2] + b[2]);
-                    float c = i * uv;
-                    if (kindB) {
-                        const float* cv = cin + (n * UM + u) * CINMAX;
-                        const float fl = sigm(g5[3] + b[3]), fr = sigm(g5[4] + b[3]);
-                        c += fl * cv[0] + fr * cv[1];
-                        pool[rec + 5 * H + j] = fl;
-                        pool[rec + 6 * H + j] = fr;
-                    }
+                    const float fl = sigm(g5[3] + b[3]), fr = sigm(g5[4] + b[3]);
+                    const float c = i * uv + fl * cv[0] + fr * cv[1];
                     pool[rec + j] = o * tanhf(c);
                     pool[rec + H + j] = c;
                     pool[rec + 2 * H + j] = i;
                     pool[rec + 3 * H + j] = o;
                     pool[rec + 4 * H + j] = uv;
+                    pool[rec + 5 * H + j] = fl;
+                    pool[rec + 6 * H + j] = fr;
                 }
             }
         } else {
@@ -454,19 +448,21 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
                 }
                 dbacc[0] += g[0]; dbacc[1] += g[1]; dbacc[2] += g[2]; dbacc[3] += g[3] + g[4];
             }
-            // transposed products (L94, fn4): per node, dx = Σ_r W[r] g_r over this thread's columns,
-            // the warp's two units summed by a shuffle, the 8 warps summed in shared memory, then one
-            // vector red.global.add per 4 columns into the children's dh (or dX for leaves)
-            const int src = lane & 16;
-            for (int n0 = 0; n0 < nb; n0 += NC) {
+            mark(4);
+            // transposed products of internal nodes (L94, fn4): per node, dx = Σ_r W[r] g_r over this
+            // thread's columns for its unit; the 16 units' slices are summed in shared memory and one
+            // vector red.global.add per 4 columns goes into the children's dh.  (Leaves: dX is formed by
+            // vpps_leaf_dx after the kernel.)
+            if (kindB) {
+                const int src = lane & 16;
+                for (int n0 = 0; n0 < nb; n0 += NC) {
 #pragma unroll
-                for (int dn = 0; dn < NC; ++dn) {
-                    const int n = n0 + dn;
-                    float gr[5];
+                    for (int dn = 0; dn < NC; ++dn) {
+                        const int n = n0 + dn;
+                        float gr[5];
 #pragma unroll
-                    for (int r = 0; r < 5; ++r) gr[r] = __shfl_sync(FULLMASK, g[r], src | (n & 15));
-                    float* drow = dxb + (warp * NC + dn) * KP;
-                    if (kindB) {
+                        for (int r = 0; r < 5; ++r) gr[r] = __shfl_sync(FULLMASK, g[r], src | (n & 15));
+                        float* drow = dxb + (u * NC + dn) * LB::KP;
 #pragma unroll
                         for (int t = 0; t < LB::NT; ++t) {
                             const int col0 = LB::CG * (tu + TU * t);
@@ -475,61 +471,45 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
 #pragma unroll
                             for (int q = 0; q < LB::CG; q += 2) {
                                 const int k = t * LB::CG + q;
-                                float2 d = make_float2(0.f, 0.f);
-#pragma unroll
-                                for (int r = 0; r < 3; ++r)
-                                    d = __ffma2_rn(make_float2(wb[r][k], wb[r][k + 1]), make_float2(gr[r], gr[r]), d);
+                                float2 d = __ffma2_rn(make_float2(wb[0][k], wb[0][k + 1]), make_float2(gr[0], gr[0]),
+                                                      make_float2(0.f, 0.f));
+                                d = __ffma2_rn(make_float2(wb[1][k], wb[1][k + 1]), make_float2(gr[1], gr[1]), d);
+                                d = __ffma2_rn(make_float2(wb[2][k], wb[2][k + 1]), make_float2(gr[2], gr[2]), d);
                                 d = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), make_float2(gf, gf), d);
-                                dx[q] = d.x + __shfl_xor_sync(FULLMASK, d.x, 16);
-                                dx[q + 1] = d.y + __shfl_xor_sync(FULLMASK, d.y, 16);
+                                dx[q] = d.x;
+                                dx[q + 1] = d.y;
                             }
-                            if (lane < 16) sts_granule<LB::CG>(drow + col0, dx, n < nb);
-                        }
-                    } else {
-#pragma unroll
-                        for (int t = 0; t < LA::NT; ++t) {
-                            const int col0 = LA::CG * (tu + TU * t);
-                            float dx[LA::CG];
-#pragma unroll
-                            for (int q = 0; q < LA::CG; q += 2) {
-                                const int k = t * LA::CG + q;
-                                float2 d = make_float2(0.f, 0.f);
-#pragma unroll
-                                for (int r = 0; r < 3; ++r)
-                                    d = __ffma2_rn(make_float2(wa[r][k], wa[r][k + 1]), make_float2(gr[r], gr[r]), d);
-                                dx[q] = d.x + __shfl_xor_sync(FULLMASK, d.x, 16);
-                                dx[q + 1] = d.y + __shfl_xor_sync(FULLMASK, d.y, 16);
-                            }
-                            if (lane < 16) sts_granule<LA::CG>(drow + col0, dx, n < nb);
+                            sts_granule<LB::CG>(drow + col0, dx, n < nb);
                         }
                     }
-                }
-                __syncthreads();
-                const int q4 = KP / 4, tot = NC * q4;
-                for (int i = tid; i < tot; i += NTH) {
-                    const int dn = i / q4, c = (i - dn * q4) * 4, n = n0 + dn;
-                    if (n >= nb) continue;
-                    const uint32_t* I = chunk + ipos[n];
-                    float* dst = nullptr;
-                    if (kindB) dst = c < H ? pool + I[4] + c : pool + I[6] + (c - H);
-                    else if (P.d_inputs && c < E) dst = P.d_inputs + (int64_t)I[3] * E + c;
-                    if (dst) {
+                    __syncthreads();
+                    constexpr int q4 = LB::KP / 4;
+                    for (int i = tid; i < NC * q4; i += NTH) {
+                        const int dn = i / q4, c = (i - dn * q4) * 4, n = n0 + dn;
+                        if (n >= nb || c >= 2 * H) continue;
+                        const uint32_t* I = chunk + ipos[n];
                         float s[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
-                        for (int w = 0; w < 8; ++w) {
-                            const float4 x = *reinterpret_cast<const float4*>(dxb + (w * NC + dn) * KP + c);
+                        for (int uu = 0; uu < UM; ++uu) {
+                            const float4 x = *reinterpret_cast<const float4*>(dxb + (uu * NC + dn) * LB::KP + c);
                             s[0] += x.x; s[1] += x.y; s[2] += x.z; s[3] += x.w;
                         }
-                        red_add<4>(dst, s);
+                        red_add<4>(c < H ? pool + I[4] + c : pool + I[6] + (c - H), s);
                     }
+                    __syncthreads();
                 }
-                __syncthreads();
             }
         }
         pos = p;
     }
     if (pending) cluster_wait();
-    if (prof && tid == 0) prof[1] = gtimer();
+    mark(8);
+    if (prof && tid == 0) {
+        prof[1] = gtimer();
+        uint64_t* o = prof + 2 + 3 * (S_[1] + 1);
+#pragma unroll
+        for (int k = 0; k < 10; ++k) o[k] = sec[k];
+    }
 
     // ---- epilogue: bias and head gradients of this replica summed into grads (zeroed by the host);
     //      the weight-matrix gradients come from vpps_dw_gemm (L185) ----
