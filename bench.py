@@ -299,10 +299,11 @@ def main():
                        "seq_len": None, "parallelism": f"dp{world}",
                        "replica_groups": m.plan_info()["n_cta"] // m.plan_info()["n_g"],
                        "cluster": args.cluster or None, "ctas": m.plan_info()["n_cta"],
-                       "mode": "fused fwd-bwd-sgd, 1 kernel" if world == 1 else "fwd_bwd + NCCL all-reduce + sgd",
+                       "mode": ("leaf GEMM + leaf cell + cluster fwd/bwd + leaf dX GEMM + dW GEMM + SGD" if args.cluster
+                                else "fused fwd-bwd-sgd, 1 kernel") + ("" if world == 1 else ", NCCL all-reduce before SGD"),
                        "l2": "no flush" if args.no_flush else "flushed (256 MiB write) before every timed step",
                        "batches": f"{N_BATCHES} distinct pre-built scripts cycled"},
-            "gpu_launches": args.steps * ((2 if args.cluster else 1) + (0 if world == 1 else 1)),
+            "gpu_launches": args.steps * (6 if args.cluster else (1 if world == 1 else 2)),
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "kernel_ms": kern_ms / args.steps, "flops_per_launch": avg_flops,

@@ -401,10 +401,9 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         launch_leaf_fwd(W_iou, m->params + m->offsets[5], inputs, m->pool, leaf_list, (int32_t)s->s.n_leaf,
                         m->plan.H, m->plan.E, st);
         CK(cudaLaunchKernelExC(&cfg, m->var->fn, args));
-        // dX of the leaves = W_iouᵀ g_leaf (words are inputs), then dW of the weight matrices
-        // from the recorded operands, fused SGD in mode 1
-        launch_leaf_dx(W_iou, m->pool, d_inputs, leaf_list, (int32_t)s->s.n_leaf, m->plan.H, m->plan.E, st);
-        launch_dw_gemm(m->pool, inputs, m->params, m->grads, lists, (int32_t)s->s.n_int, lists + 3 * s->s.n_int,
+        // dW of the weight matrices from the recorded operands and dX of the leaves
+        // = W_iouᵀ g_leaf (words are inputs) in one launch; SGD in mode 1
+        launch_dw_gemm(m->pool, inputs, d_inputs, m->params, m->grads, lists, (int32_t)s->s.n_int, leaf_list,
                        (int32_t)s->s.n_leaf, m->plan.H, m->plan.E, m->offsets.data(), m->n_floats, mode, lr, wd, st);
         CK(cudaGetLastError());
     } else {

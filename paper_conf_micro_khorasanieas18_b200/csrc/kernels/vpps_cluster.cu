@@ -22,7 +22,7 @@ constexpr int NB = 16;         // nodes per batch: one node per lane of a unit's
 constexpr int NC = 2;          // nodes per transposed-product chunk
 constexpr int ZC = 32;         // classes per head (C <= 32)
 constexpr int CINMAX = 10;
-constexpr uint32_t NONE = 0xFFFFFFFFu;
+constexpr int DFW = 10;        // deferred-store entry: 3 addresses + up to 7 values
 enum : uint32_t { S = 0x01, W = 0x02, LEAF_F = 0x20, LEAF_B = 0x21, INT_F = 0x22, INT_B = 0x23, HEAD_F = 0x40, HEAD_B = 0x41 };
 
 __device__ __forceinline__ int words(uint32_t w) {
@@ -103,7 +103,8 @@ struct CCfg {
     static constexpr int O_BST = O_IPOS + NB;
     static constexpr int O_SEGP = O_BST + 4;                 // NB x 2 pointers (8-byte aligned)
     static constexpr int O_ZS = O_SEGP + 4 * NB;
-    static constexpr int O_HEAD = O_ZS + NB * ZC;
+    static constexpr int O_DFW = O_ZS + NB * ZC;             // deferred stores: NB x UM entries of DFW words
+    static constexpr int O_HEAD = O_DFW + NB * UM * DFW;
     static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 2 * C + 8); }
 };
 
@@ -124,6 +125,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
     int* bst = reinterpret_cast<int*>(smw + T::O_BST);
     const float** segp = reinterpret_cast<const float**>(smw + T::O_SEGP);
     float* zs = sm + T::O_ZS;
+    uint32_t* dfw = smw + T::O_DFW;
     const int C = P.C;
     float* Wo = sm + T::O_HEAD;
     float* dWo = Wo + C * H;
@@ -137,7 +139,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
     const uint32_t hdr = 2 + G + 1;
     const uint32_t s0 = hdr + S_[2 + grp], s1 = hdr + S_[3 + grp];
     float* pool = P.pool;
-    const float* __restrict__ inputs = P.inputs;
     const int64_t* off = P.off;
     const int u = tid / TU, tu = tid % TU, gl = lane & 15;      // unit slot, thread in unit, lane in group
     const int j = lc + u * NCL;                                 // hidden unit of this thread
@@ -216,7 +217,96 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
     };
     if (s0 < s1) refill(s0);
     bool pending = false;
+    bool predecoded = false;
+    int n_dfr = 0;                 // deferred record stores of the last batch (entries n * UM + u)
+    uint32_t dfr_op = 0;
     uint32_t pos = s0;
+    // Deferred stores: the record fields no other CTA reads during the pass (c, gates, gate gradients,
+    // dc of the children) are parked in shared memory and written after the next barrier arrive, so the
+    // arrive's release only waits for the cross-CTA data (h, dh) and the writes drain during the wait.
+    auto flush = [&]() {
+        if (n_dfr == 0) return;
+        __syncthreads();
+        if (tid < n_dfr) {
+            const uint32_t* e = dfw + tid * DFW;
+            const float* v = reinterpret_cast<const float*>(e + 3);
+            const int jj = lc + (tid % UM) * NCL;
+            if (dfr_op == INT_F) {
+#pragma unroll
+                for (int k = 0; k < 6; ++k) pool[e[0] + (k + 1) * H + jj] = v[k];          // c i o u fl fr
+            } else if (dfr_op == INT_B) {
+#pragma unroll
+                for (int k = 0; k < 5; ++k) pool[e[0] + (7 + k) * H + jj] = v[k];          // g_i g_o g_u g_fl g_fr
+                pool[e[1] + H + jj] = v[5];                                                // dc of the children
+                pool[e[2] + H + jj] = v[6];
+            } else {
+#pragma unroll
+                for (int k = 0; k < 3; ++k) pool[e[0] + (5 + k) * H + jj] = v[k];          // leaf g_i g_o g_u
+            }
+        }
+        n_dfr = 0;
+    };
+    // decode (warp 0): up to NB consecutive instructions with the opcode at `at` + their row sources
+    auto decode = [&](uint32_t at) {
+        flush();
+        __syncthreads();
+        if (warp == 0) {
+            const uint32_t pre_ = chunk[at - cbase], op_ = pre_ & 0xFF;
+            const bool head_ = (op_ == HEAD_F || op_ == HEAD_B);
+            const uint32_t lim = min(s1, cbase + (uint32_t)CHUNK);
+            const uint32_t sz = (uint32_t)words(pre_);
+            const uint32_t q = at + (uint32_t)lane * sz;
+            const bool ok = lane < NB && q + sz <= lim && (chunk[q - cbase] & 0xFF) == op_;
+            const unsigned msk = __ballot_sync(FULLMASK, ok);
+            const int nbw = (msk == FULLMASK) ? 32 : (__ffs(~msk) - 1);
+            if (lane < nbw) ipos[lane] = (int)(q - cbase);
+            if (lane == 0) { bst[0] = nbw; bst[1] = (int)(at + nbw * sz); bst[2] = (int)op_; }
+            __syncwarp();
+            const float* sp0 = nullptr;
+            const float* sp1 = nullptr;
+            if (lane < nbw) {           // rows: [h_l; h_r] for internal forward, h for the heads
+                const uint32_t* I = chunk + ipos[lane];
+                if (op_ == INT_F) { sp0 = pool + I[2]; sp1 = pool + I[3]; }
+                else if (head_ && holds_head) sp0 = pool + I[2];
+            }
+            if (lane < NB) { segp[2 * lane] = sp0; segp[2 * lane + 1] = sp1; }
+        }
+        __syncthreads();
+    };
+    // cell operands k0 <= k < k1 of every (node, unit) of the decoded batch -> cin (cp.async, 4 B)
+    auto stage_cin = [&](uint32_t op_, int nb_, int k0, int k1) {
+        const int kk = k1 - k0;
+        for (int i = tid; i < nb_ * UM * kk; i += NTH) {
+            const int n = i / (UM * kk), rem = i - n * (UM * kk);
+            const int uu = rem / kk, k = k0 + rem - uu * kk;
+            cp_async4(cin + (n * UM + uu) * CINMAX + k, cin_src<H>(op_, chunk + ipos[n], k, lc + uu * NCL, pool), 4u);
+        }
+    };
+    // before the barrier wait: operands this CTA wrote itself (children's c; c, gates and dc of a node)
+    auto stage_pre = [&]() {
+        const uint32_t op_ = (uint32_t)bst[2];
+        const int nb_ = bst[0];
+        if (op_ == INT_F) stage_cin(op_, nb_, 0, 2);
+        else if (op_ == INT_B || op_ == LEAF_B) stage_cin(op_, nb_, 1, n_cin(op_));
+    };
+    // after it: data written by the other CTAs of the cluster (h rows, dh)
+    auto stage_post = [&]() {
+        const uint32_t op_ = (uint32_t)bst[2];
+        const int nb_ = bst[0];
+        if (op_ == INT_B || op_ == LEAF_B) { stage_cin(op_, nb_, 0, 1); return; }
+        const bool head_ = (op_ == HEAD_F || op_ == HEAD_B);
+        if (head_ && !holds_head) return;
+        const int KPr = op_ == INT_F ? LB::KP : LA::KP;
+        const int q4 = KPr / 4;
+        const int A = H, B = op_ == INT_F ? H : 0;
+        for (int i = tid; i < nb_ * q4; i += NTH) {
+            const int n = i / q4, c = (i - n * q4) * 4;
+            const float* src = nullptr;
+            if (c < A) { const float* b = segp[2 * n]; if (b) src = b + c; }
+            else if (c < A + B) { const float* b = segp[2 * n + 1]; if (b) src = b + (c - A); }
+            cp_async16(xs + n * KPr + c, src ? src : pool, src ? 16u : 0u);
+        }
+    };
     while (pos < s1) {
         if (pos + 640 > cbase + CHUNK && cbase + CHUNK < s1) refill(pos);
         const uint32_t pre = chunk[pos - cbase];
@@ -232,6 +322,25 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
             cluster_arrive();
             pending = true;
             ++pos;
+            mark(8);
+            flush();
+            // between arrive and wait (L165: independent work may sit between a signal and its wait):
+            // decode the next batch and stage the operands this CTA produced itself
+            if (pos < s1 && (chunk[pos - cbase] & 0xFF) == W) {
+                const uint32_t wpre = chunk[pos - cbase];
+                uint32_t nx = pos + 1;
+                if (nx < s1 && nx + 640 > cbase + CHUNK && cbase + CHUNK < s1) refill(nx);
+                bool ahead = false;
+                if (nx < s1) { const uint32_t nop = chunk[nx - cbase] & 0xFF; ahead = nop != S && nop != W && nop != LEAF_F; }
+                if (ahead) { mark(0); decode(nx); mark(1); stage_pre(); }
+                mark(7);
+                if (prof && tid == 0) prof[3 + 3 * (wpre >> 8)] = gtimer();
+                cluster_wait();
+                pending = false;
+                if (prof && tid == 0) prof[4 + 3 * (wpre >> 8)] = gtimer();
+                pos = nx;
+                predecoded = ahead;
+            }
             continue;
         }
         if (op == W) {            // wait (L165): all 16 CTAs of the replica have signalled
@@ -251,53 +360,13 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
         const bool fwd = (op & 1) == 0;
         const bool kindB = (op == INT_F || op == INT_B);
         const int KP = kindB ? LB::KP : LA::KP;
-        // ---- decode (warp 0): up to NB consecutive instructions with this opcode + row sources ----
-        __syncthreads();
-        mark(0);
-        if (warp == 0) {
-            const uint32_t lim = min(s1, cbase + (uint32_t)CHUNK);
-            const uint32_t sz = (uint32_t)words(pre);
-            const uint32_t q = pos + (uint32_t)lane * sz;
-            const bool ok = lane < NB && q + sz <= lim && (chunk[q - cbase] & 0xFF) == op;
-            const unsigned msk = __ballot_sync(FULLMASK, ok);
-            const int nbw = (msk == FULLMASK) ? 32 : (__ffs(~msk) - 1);
-            if (lane < nbw) ipos[lane] = (int)(q - cbase);
-            if (lane == 0) { bst[0] = nbw; bst[1] = (int)(pos + nbw * sz); }
-            __syncwarp();
-            const float* sp0 = nullptr;
-            const float* sp1 = nullptr;
-            if (lane < nbw && (!is_head || holds_head)) {
-                const uint32_t* I = chunk + ipos[lane];
-                if (is_head) sp0 = pool + I[2];
-                else if (!kindB) sp0 = inputs + (int64_t)(fwd ? I[2] : I[3]) * E;
-                else { sp0 = pool + (fwd ? I[2] : I[3]); sp1 = pool + (fwd ? I[3] : I[5]); }
-            }
-            if (lane < NB) { segp[2 * lane] = sp0; segp[2 * lane + 1] = sp1; }
-        }
-        __syncthreads();
+        if (!predecoded) { mark(0); decode(pos); mark(1); stage_pre(); }
+        predecoded = false;
         const int nb = bst[0];
         const uint32_t p = (uint32_t)bst[1];
         mark(1);
-        // ---- staging: cp.async of every input row and cell operand of the batch (one round trip) ----
-        {
-            const int q4 = KP / 4;
-            const int A = is_head ? H : (kindB ? H : E), B = kindB ? H : 0;
-            const int rows = (is_head && !holds_head) ? 0 : nb;
-            for (int i = tid; i < rows * q4; i += NTH) {
-                const int n = i / q4, c = (i - n * q4) * 4;
-                const float* src = nullptr;
-                if (c < A) { const float* b = segp[2 * n]; if (b) src = b + c; }
-                else if (c < A + B) { const float* b = segp[2 * n + 1]; if (b) src = b + (c - A); }
-                cp_async16(xs + n * KP + c, src ? src : pool, src ? 16u : 0u);
-            }
-            const int ncin = is_head ? 0 : n_cin(op);
-            for (int i = tid; i < nb * UM * ncin; i += NTH) {
-                const int n = i / (UM * ncin), rem = i - n * (UM * ncin);
-                const int uu = rem / ncin, k = rem - uu * ncin;
-                cp_async4(cin + (n * UM + uu) * CINMAX + k, cin_src<H>(op, chunk + ipos[n], k, lc + uu * NCL, pool), 4u);
-            }
-            cp_async_wait_all();
-        }
+        stage_post();
+        cp_async_wait_all();
         __syncthreads();
 
         mark(is_head ? 5 : (fwd ? 2 : 3));
@@ -407,15 +476,15 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
                     const float i = sigm(g5[0] + b[0]), o = sigm(g5[1] + b[1]), uv = tanhf(g5[2] + b[2]);
                     const float fl = sigm(g5[3] + b[3]), fr = sigm(g5[4] + b[3]);
                     const float c = i * uv + fl * cv[0] + fr * cv[1];
-                    pool[rec + j] = o * tanhf(c);
-                    pool[rec + H + j] = c;
-                    pool[rec + 2 * H + j] = i;
-                    pool[rec + 3 * H + j] = o;
-                    pool[rec + 4 * H + j] = uv;
-                    pool[rec + 5 * H + j] = fl;
-                    pool[rec + 6 * H + j] = fr;
+                    pool[rec + j] = o * tanhf(c);                  // h: read by every CTA of the cluster
+                    uint32_t* e = dfw + (n * UM + u) * DFW;        // the rest only by this CTA / the GEMMs
+                    float* v = reinterpret_cast<float*>(e + 3);
+                    e[0] = rec;
+                    v[0] = c; v[1] = i; v[2] = o; v[3] = uv; v[4] = fl; v[5] = fr;
                 }
             }
+            n_dfr = nb * UM;
+            dfr_op = op;
         } else {
             // ---- backward: cell backward by thread (unit u, node gl); its gate gradients are recorded
             //      in the node's record for the dW GEMM (L185) and broadcast to the unit's lanes ----
@@ -430,24 +499,21 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
                 g[0] = chat * uv * i * (1.f - i);
                 g[1] = dh * th * o * (1.f - o);
                 g[2] = chat * i * (1.f - uv * uv);
+                uint32_t* e = dfw + (gl * UM + u) * DFW;      // deferred: only this CTA / the GEMMs read these
+                float* v = reinterpret_cast<float*>(e + 3);
+                e[0] = rec;
+                v[0] = g[0]; v[1] = g[1]; v[2] = g[2];
                 if (kindB) {
                     const float fl = cv[6], fr = cv[7], cl = cv[8], cr = cv[9];
                     g[3] = chat * cl * fl * (1.f - fl);
                     g[4] = chat * cr * fr * (1.f - fr);
-                    pool[I[4] + H + j] = chat * fl;          // dc of the children (unique parent)
-                    pool[I[6] + H + j] = chat * fr;
-                    pool[rec + 10 * H + j] = g[3];
-                    pool[rec + 11 * H + j] = g[4];
-                    pool[rec + 7 * H + j] = g[0];
-                    pool[rec + 8 * H + j] = g[1];
-                    pool[rec + 9 * H + j] = g[2];
-                } else {
-                    pool[rec + 5 * H + j] = g[0];
-                    pool[rec + 6 * H + j] = g[1];
-                    pool[rec + 7 * H + j] = g[2];
+                    e[1] = I[4]; e[2] = I[6];                   // dc of the children (unique parent)
+                    v[3] = g[3]; v[4] = g[4]; v[5] = chat * fl; v[6] = chat * fr;
                 }
                 dbacc[0] += g[0]; dbacc[1] += g[1]; dbacc[2] += g[2]; dbacc[3] += g[3] + g[4];
             }
+            n_dfr = nb * UM;
+            dfr_op = op;
             mark(4);
             // transposed products of internal nodes (L94, fn4): per node, dx = Σ_r W[r] g_r over this
             // thread's columns for its unit; the 16 units' slices are summed in shared memory and one
@@ -502,6 +568,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
         }
         pos = p;
     }
+    flush();
     if (pending) cluster_wait();
     mark(8);
     if (prof && tid == 0) {
@@ -542,21 +609,88 @@ struct GemmParams {
     const uint32_t* leaf_nodes;  // n_leaf x (rec, token)
     int32_t n_int, n_leaf, H, E;
     int64_t off[8];
-    int32_t items[4];            // work items per matrix (U_iou, U_fl, U_fr, W_iou)
+    const float* w_iou;          // W_iou (params), for the leaf input gradient
+    float* d_inputs;             // dX, or nullptr
+    int32_t items[5];            // work items per job (dU_iou, dU_fl, dU_fr, dW_iou, leaf dX)
 };
 
 constexpr int TM = 128;          // tile rows (gate-gradient rows)
 constexpr int TN = 64;           // tile cols (input columns)
 constexpr int KS = 16;           // nodes per pipeline stage
 constexpr int KCH = 96;          // nodes per work item (split-K)
+constexpr int NST = 3;           // cp.async pipeline stages
+
+// leaf input gradient dX[tok_l] += Σ_r g_l[r] W_iou[r][:] (word vectors are inputs of the
+// leaves).  Tile 64 leaves x 64 columns, split-K over the 3H gate rows in chunks of DXK, 4 x 4 per thread;
+// the leaf gate gradients are staged row-major ([leaf][k], stride 20: conflict-free column reads).
+constexpr int DXM = 64, DXN = 64, DXK = 128, DXS = 20;
+__device__ __forceinline__ void leaf_dx_tile(const GemmParams& P, int b, float* As, float* Bs) {
+    const int tid = threadIdx.x, H = P.H, E = P.E;
+    const int tiles_c = E / DXN, tiles_r = (P.n_leaf + DXM - 1) / DXM;
+    const int kc = b / (tiles_r * tiles_c), t = b - kc * (tiles_r * tiles_c);
+    const int r0 = (t / tiles_c) * DXM, c0 = (t % tiles_c) * DXN;
+    const int k0 = kc * DXK, k1 = min(3 * H, k0 + DXK);
+    const int ty = tid / 16, tx = tid % 16;          // leaves r0 + ty + 16a, columns c0 + 4tx .. +3
+    float2 acc2[4][2];
+#pragma unroll
+    for (int a = 0; a < 4; ++a) acc2[a][0] = acc2[a][1] = make_float2(0.f, 0.f);
+    auto stage = [&](int s, int buf) {
+        {
+            const int l = tid / 4, piece = (tid % 4) * 4, row = r0 + l;
+            const float* src = row < P.n_leaf ? P.pool + P.leaf_nodes[2 * row] + 5 * H + k0 + s * KS + piece : nullptr;
+            cp_async16(As + buf * DXM * DXS + l * DXS + piece, src ? src : P.pool, src ? 16u : 0u);
+        }
+        {
+            const int k = tid / 16, piece = (tid % 16) * 4;
+            cp_async16(Bs + buf * KS * TN + k * TN + piece, P.w_iou + (int64_t)(k0 + s * KS + k) * E + c0 + piece, 16u);
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    const int steps = (k1 - k0) / KS;
+    stage(0, 0);
+    if (steps > 1) stage(1, 1);
+    for (int s = 0; s < steps; ++s) {
+        if (s + 2 < steps) {
+            stage(s + 2, (s + 2) % NST);
+            asm volatile("cp.async.wait_group 2;" ::: "memory");
+        } else if (s + 1 < steps) {
+            asm volatile("cp.async.wait_group 1;" ::: "memory");
+        } else {
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
+        }
+        __syncthreads();
+        const float* A = As + (s % NST) * DXM * DXS;
+        const float* B = Bs + (s % NST) * KS * TN;
+#pragma unroll
+        for (int k = 0; k < KS; ++k) {
+            const float4 bv = *reinterpret_cast<const float4*>(B + k * TN + tx * 4);
+            const float2 b01 = make_float2(bv.x, bv.y), b23 = make_float2(bv.z, bv.w);
+#pragma unroll
+            for (int a = 0; a < 4; ++a) {
+                const float av = A[(ty + 16 * a) * DXS + k];
+                const float2 aa = make_float2(av, av);
+                acc2[a][0] = __ffma2_rn(aa, b01, acc2[a][0]);
+                acc2[a][1] = __ffma2_rn(aa, b23, acc2[a][1]);
+            }
+        }
+        __syncthreads();
+    }
+#pragma unroll
+    for (int a = 0; a < 4; ++a) {
+        const int row = r0 + ty + 16 * a;
+        const float v[4] = {acc2[a][0].x, acc2[a][0].y, acc2[a][1].x, acc2[a][1].y};
+        if (row < P.n_leaf) red_add<4>(P.d_inputs + (int64_t)P.leaf_nodes[2 * row + 1] * E + c0 + tx * 4, v);
+    }
+}
 
 __global__ void __launch_bounds__(256) vpps_dw_gemm(const GemmParams P) {
-    __shared__ __align__(16) float Gs[2][KS][TM];
-    __shared__ __align__(16) float Xs[2][KS][TN];
+    __shared__ __align__(16) float Gs[NST][KS][TM];
+    __shared__ __align__(16) float Xs[NST][KS][TN];
     const int tid = threadIdx.x, H = P.H, E = P.E;
     int b = blockIdx.x, m = 0;
-    while (m < 4 && b >= P.items[m]) { b -= P.items[m]; ++m; }
-    if (m == 4) return;
+    while (m < 5 && b >= P.items[m]) { b -= P.items[m]; ++m; }
+    if (m == 5) return;
+    if (m == 4) { leaf_dx_tile(P, b, &Gs[0][0][0], &Xs[0][0][0]); return; }
     const int rows = (m == 0 || m == 3) ? 3 * H : H;
     const int cols = m == 0 ? 2 * H : (m == 3 ? E : H);
     const int K = m == 3 ? P.n_leaf : P.n_int;
@@ -566,11 +700,9 @@ __global__ void __launch_bounds__(256) vpps_dw_gemm(const GemmParams P) {
     const int k0 = kc * KCH, k1 = min(K, k0 + KCH);
     const int goff = m == 0 ? 7 * H : (m == 1 ? 10 * H : (m == 2 ? 11 * H : 5 * H));
     const int ty = tid / 16, tx = tid % 16;        // rows ty*8 .. +7, cols tx*4 .. +3
-    float acc[8][4];
+    float2 acc[8][2];
 #pragma unroll
-    for (int a = 0; a < 8; ++a)
-#pragma unroll
-        for (int c = 0; c < 4; ++c) acc[a][c] = 0.f;
+    for (int a = 0; a < 8; ++a) acc[a][0] = acc[a][1] = make_float2(0.f, 0.f);
     // stage: KS nodes x 128 rows of g (2 x 16 B per thread) and KS nodes x 64 cols of x (16 B per thread)
     auto stage = [&](int s, int buf) {
 #pragma unroll
@@ -603,34 +735,42 @@ __global__ void __launch_bounds__(256) vpps_dw_gemm(const GemmParams P) {
         asm volatile("cp.async.commit_group;" ::: "memory");
     };
     const int steps = (k1 - k0 + KS - 1) / KS;
-    if (steps > 0) stage(0, 0);
+    if (steps <= 0) return;
+    stage(0, 0);
+    if (steps > 1) stage(1, 1);
     for (int s = 0; s < steps; ++s) {
-        if (s + 1 < steps) {
-            stage(s + 1, (s + 1) & 1);
+        if (s + 2 < steps) {
+            stage(s + 2, (s + 2) % NST);
+            asm volatile("cp.async.wait_group 2;" ::: "memory");
+        } else if (s + 1 < steps) {
             asm volatile("cp.async.wait_group 1;" ::: "memory");
         } else {
             asm volatile("cp.async.wait_group 0;" ::: "memory");
         }
         __syncthreads();
-        const int buf = s & 1;
+        const int buf = s % NST;
 #pragma unroll
         for (int k = 0; k < KS; ++k) {
             const float4 g0 = *reinterpret_cast<const float4*>(&Gs[buf][k][ty * 8]);
             const float4 g1 = *reinterpret_cast<const float4*>(&Gs[buf][k][ty * 8 + 4]);
             const float4 xv = *reinterpret_cast<const float4*>(&Xs[buf][k][tx * 4]);
             const float ga[8] = {g0.x, g0.y, g0.z, g0.w, g1.x, g1.y, g1.z, g1.w};
-            const float xa[4] = {xv.x, xv.y, xv.z, xv.w};
+            const float2 x01 = make_float2(xv.x, xv.y), x23 = make_float2(xv.z, xv.w);
 #pragma unroll
-            for (int a = 0; a < 8; ++a)
-#pragma unroll
-                for (int c = 0; c < 4; ++c) acc[a][c] = fmaf(ga[a], xa[c], acc[a][c]);
+            for (int a = 0; a < 8; ++a) {
+                const float2 gg = make_float2(ga[a], ga[a]);
+                acc[a][0] = __ffma2_rn(gg, x01, acc[a][0]);
+                acc[a][1] = __ffma2_rn(gg, x23, acc[a][1]);
+            }
         }
         __syncthreads();
     }
-    if (steps == 0) return;
     float* base = P.grads + P.off[m == 3 ? 0 : m + 1];
 #pragma unroll
-    for (int a = 0; a < 8; ++a) red_add<4>(base + (int64_t)(r0 + ty * 8 + a) * cols + c0 + tx * 4, acc[a]);
+    for (int a = 0; a < 8; ++a) {
+        const float v[4] = {acc[a][0].x, acc[a][0].y, acc[a][1].x, acc[a][1].y};
+        red_add<4>(base + (int64_t)(r0 + ty * 8 + a) * cols + c0 + tx * 4, v);
+    }
 }
 
 }  // namespace cl
@@ -648,9 +788,9 @@ const Variant* cluster_variants(int32_t* n) {
     return kClusterVariants;
 }
 
-void launch_dw_gemm(const float* pool, const float* inputs, float* params, float* grads, const uint32_t* int_nodes,
-                    int32_t n_int, const uint32_t* leaf_nodes, int32_t n_leaf, int32_t H, int32_t E,
-                    const int64_t* off, int64_t n_floats, int32_t mode, float lr, float wd, cudaStream_t s) {
+void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, float* params, float* grads,
+                    const uint32_t* int_nodes, int32_t n_int, const uint32_t* leaf_nodes, int32_t n_leaf, int32_t H,
+                    int32_t E, const int64_t* off, int64_t n_floats, int32_t mode, float lr, float wd, cudaStream_t s) {
     using namespace dev::cl;
     GemmParams g{};
     g.pool = pool; g.inputs = inputs; g.grads = grads;
@@ -662,7 +802,11 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* params, float
     g.items[1] = (H / TM) * (H / TN) * ki;
     g.items[2] = g.items[1];
     g.items[3] = (3 * H / TM) * (E / TN) * kl;
-    const int items = g.items[0] + g.items[1] + g.items[2] + g.items[3];
+    g.w_iou = params + off[0];
+    g.d_inputs = d_inputs;
+    g.items[4] = d_inputs ? ((n_leaf + DXM - 1) / DXM) * (E / DXN) * ((3 * H + DXK - 1) / DXK) : 0;
+    if (n_leaf == 0) g.items[4] = 0;
+    const int items = g.items[0] + g.items[1] + g.items[2] + g.items[3] + g.items[4];
     if (items > 0) vpps_dw_gemm<<<items, 256, 0, s>>>(g);
     if (mode == 1) launch_sgd(params, grads, n_floats, lr, wd, s);   // W -= lr (dW + wd W), every parameter
 }

@@ -32,15 +32,14 @@ const Variant* variants(int32_t* n);
 // Cluster-replica specialisations (vpps_cluster.cu); Variant.umax holds the cluster size.
 const Variant* cluster_variants(int32_t* n);
 // dW = Σ g xᵀ per weight matrix from the recorded operands, fused SGD when mode == 1.
-void launch_dw_gemm(const float* pool, const float* inputs, float* params, float* grads, const uint32_t* int_nodes,
-                    int32_t n_int, const uint32_t* leaf_nodes, int32_t n_leaf, int32_t H, int32_t E,
-                    const int64_t* off, int64_t n_floats, int32_t mode, float lr, float wd, cudaStream_t s);
-// Leaf level of the binary cell as GEMMs (vpps_leaf.cu): records h, c, i, o, u of every leaf before the
-// cluster kernel; dX[tok] += W_iouᵀ g_leaf after it (no-op when d_inputs is null).
+// Also forms the leaf input gradient dX[tok] += W_iouᵀ g_leaf when d_inputs is not null.
+void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, float* params, float* grads,
+                    const uint32_t* int_nodes, int32_t n_int, const uint32_t* leaf_nodes, int32_t n_leaf, int32_t H,
+                    int32_t E, const int64_t* off, int64_t n_floats, int32_t mode, float lr, float wd, cudaStream_t s);
+// Leaf level of the binary cell as one GEMM + fused cell (vpps_leaf.cu): records h, c, i, o, u of every
+// leaf before the cluster kernel.
 void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float* pool, const uint32_t* leaves,
                      int32_t n_leaf, int32_t H, int32_t E, cudaStream_t s);
-void launch_leaf_dx(const float* W, const float* pool, float* d_inputs, const uint32_t* leaves, int32_t n_leaf,
-                    int32_t H, int32_t E, cudaStream_t s);
 // Elementwise SGD on the flat buffer (K3): p -= lr * (g + wd * p).
 void launch_sgd(float* p, const float* g, int64_t n, float lr, float wd, cudaStream_t s);
 

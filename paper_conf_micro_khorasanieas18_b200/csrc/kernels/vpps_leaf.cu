@@ -1,13 +1,19 @@
-// The leaf level of the binary Tree-LSTM as dense GEMMs (cluster path).
+// The leaf level of the binary Tree-LSTM as a dense GEMM with the leaf cell fused into its epilogue
+// (cluster path).
 //
 // Every leaf of a batch uses the same matrix W_iou on its word vector (words enter the
-// Tree-LSTM at the leaves), so level 0 is one real dense GEMM — the case where north_star allows a
-// GEMM instead of per-node matrix-vector products.  The recurrent matrices (U_iou, U_fl, U_fr) stay
-// register-resident in vpps_cl.  Three kernels:
-//   vpps_leaf_gemm<FWD>  pre-activations  A[l][r] = W_iou[r] · x_l        -> leaf record gate slots
-//   vpps_leaf_cell       leaf cell        i,o = σ, u = tanh, c = i u, h = o tanh c  (in place)
-//   vpps_leaf_gemm<DX>   input gradient   dX[tok_l] += W_iouᵀ g_l          (split-K, L2 reductions)
-// FP32 SIMT: 64 x 64 output tiles, 16-deep K stages in shared memory (cp.async), 4 x 4 per thread.
+// Tree-LSTM at the leaves), so level 0 is one dense GEMM — the case where north_star allows a GEMM
+// instead of per-node matrix-vector products.  The recurrent matrices (U_iou, U_fl, U_fr) stay
+// register-resident in vpps_cl.
+//
+//   vpps_leaf_fwd: a = W_iou x_l + b_iou; i, o = σ, u = tanh; c = i u; h = o tanh c  -> leaf record [h c i o u]
+//
+// Tile: 32 leaves x 32 hidden units x 3 gates (i, o, u of the same units, so the cell runs in the
+// epilogue).  The whole K range of the tile's 128 rows is staged with one batch of cp.async (the GEMM is
+// small and DRAM-latency bound after the L2 flush, so one round trip beats a K pipeline); 512 threads =
+// four K quarters of 128; each thread owns 4 leaves x 2 units x 3 gates and reads 16-byte K slices.
+// The input-table gradient dX = W_iouᵀ g_leaf is a job of the gradient GEMM (vpps_dw_gemm, vpps_cluster.cu).
+// Requires E <= KMAX and H % 32 == 0 (the cluster variants are H = E = 256).
 #include "vpps_kernel.cuh"
 #include "dev_common.cuh"
 
@@ -15,115 +21,105 @@ namespace vpps {
 namespace dev {
 namespace leaf {
 
-struct Params {
-    const float* W;           // W_iou [3H x E] row-major
-    const float* b;           // b_iou [3H]
-    const float* inputs;      // [rows x E]
-    float* pool;
-    float* d_inputs;          // DX only
-    const uint32_t* leaves;   // n_leaf x (rec, token)
-    int32_t n_leaf, H, E, kchunk;
-};
+constexpr int LM = 32;          // leaves per tile
+constexpr int LU = 32;          // hidden units per tile (x 3 gates)
+constexpr int NT = 512;
+constexpr int KMAX = 256;       // E <= KMAX: the whole K range is staged at once (one DRAM round trip)
+constexpr int KS = KMAX + 4;    // row stride in floats (≡ 4 mod 32: conflict-free 16-byte column reads)
+constexpr size_t SMEM = (size_t)(LM + 3 * LU) * KS * sizeof(float);
 
-constexpr int BM = 64, BN = 64, BK = 16;
-
-// FWD: C[l][n] = Σ_k x_l[k] W[n][k], K = E, N = 3H, written to pool[rec_l + 2H + n] (i, o, u slots)
-// DX : C[l][n] = Σ_k g_l[k] W[k][n], K = 3H (this CTA's k chunk), N = E, added to d_inputs[tok_l][n]
-template <bool FWD>
-__global__ void __launch_bounds__(256) vpps_leaf_gemm(const Params P) {
-    __shared__ __align__(16) float As[2][BM][BK];          // [m][k]
-    __shared__ __align__(16) float Bs[2][BK][BN + 4];      // [k][n]
-    const int tid = threadIdx.x, H = P.H, E = P.E;
-    const int N = FWD ? 3 * H : E;
-    const int tiles_n = N / BN, tiles_m = (P.n_leaf + BM - 1) / BM;
-    int b = blockIdx.x;
-    const int kc = b / (tiles_m * tiles_n);
-    b -= kc * tiles_m * tiles_n;
-    const int m0 = (b / tiles_n) * BM, n0 = (b % tiles_n) * BN;
-    const int K = FWD ? E : 3 * H;
-    const int k0 = FWD ? 0 : kc * P.kchunk, k1 = FWD ? K : min(K, k0 + P.kchunk);
-    const int ty = tid / 16, tx = tid % 16;
-    float acc[4][4];
+__global__ void __launch_bounds__(NT, 1) vpps_leaf_fwd(const float* __restrict__ W, const float* __restrict__ b,
+                                                    const float* __restrict__ inputs, float* pool,
+                                                    const uint32_t* __restrict__ leaves, int n_leaf, int H, int E) {
+    extern __shared__ __align__(16) float lsm[];
+    float* As = lsm;                 // [32 leaves][KS]: x rows
+    float* Bs = lsm + LM * KS;       // [96 rows][KS]: W_iou rows g*H + j0 + uu, row index g*32 + uu
+    const int tid = threadIdx.x;
+    const int tiles_u = H / LU;
+    const int l0 = (blockIdx.x / tiles_u) * LM, j0 = (blockIdx.x % tiles_u) * LU;
+    // stage everything: 128 rows x E floats, 16-byte cp.async pieces, zero-filled past the last leaf
+    const int q = E / 4;
+    for (int i = tid; i < (LM + 3 * LU) * q; i += NT) {
+        const int row = i / q, c = (i - row * q) * 4;
+        const float* src = nullptr;
+        if (row < LM) {
+            const int l = l0 + row;
+            if (l < n_leaf) src = inputs + (int64_t)leaves[2 * l + 1] * E + c;
+        } else {
+            const int r = row - LM, g = r / LU, uu = r % LU;
+            src = W + (int64_t)(g * H + j0 + uu) * E + c;
+        }
+        cp_async16(lsm + row * KS + c, src ? src : W, src ? 16u : 0u);
+    }
+    cp_async_wait_all();
+    __syncthreads();
+    // 4 K quarters x 128 threads; a thread owns 4 leaves x 2 units x 3 gates (24 accumulators): per 4-wide K
+    // step 4 + 6 LDS.128 feed 96 FMA, so the FMA pipe, not shared memory, is the limit
+    const int part = tid >> 7, tt = tid & 127, lq = tt >> 4, up = tt & 15;
+    float acc[4][3][2];
 #pragma unroll
     for (int a = 0; a < 4; ++a)
 #pragma unroll
-        for (int c = 0; c < 4; ++c) acc[a][c] = 0.f;
-    auto stage = [&](int kk, int buf) {
-        {   // A: 64 rows x 16 k, one 16-byte piece per thread
-            const int m = tid / 4, piece = (tid % 4) * 4, row = m0 + m;
-            const float* src = nullptr;
-            if (row < P.n_leaf) {
-                const uint32_t rec = P.leaves[2 * row], tok = P.leaves[2 * row + 1];
-                src = FWD ? P.inputs + (int64_t)tok * E + kk + piece : P.pool + rec + 5 * H + kk + piece;
+        for (int g = 0; g < 3; ++g) acc[a][g][0] = acc[a][g][1] = 0.f;
+    const int kq = E / 4, kb = part * kq;
+    const float* ap = As + (4 * lq) * KS + kb;
+    const float* bw = Bs + up * KS + kb;
+#pragma unroll 2
+    for (int k = 0; k < kq; k += 4) {
+        float4 x[4];
+#pragma unroll
+        for (int a = 0; a < 4; ++a) x[a] = *reinterpret_cast<const float4*>(ap + a * KS + k);
+#pragma unroll
+        for (int g = 0; g < 3; ++g)
+#pragma unroll
+            for (int c = 0; c < 2; ++c) {
+                const float4 w = *reinterpret_cast<const float4*>(bw + (g * LU + 16 * c) * KS + k);
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+                    acc[a][g][c] = fmaf(x[a].x, w.x, fmaf(x[a].y, w.y, fmaf(x[a].z, w.z, fmaf(x[a].w, w.w, acc[a][g][c]))));
             }
-            cp_async16(&As[buf][m][piece], src ? src : P.pool, src ? 16u : 0u);
-        }
-        if (FWD) {   // B[k][n] = W[n0 + n][kk + k]: 64 rows of W x 16 k, stored transposed (scalar STS)
-            const int n = tid / 4, piece = (tid % 4) * 4;
-            const float4 w = __ldg(reinterpret_cast<const float4*>(P.W + (int64_t)(n0 + n) * E + kk + piece));
-            Bs[buf][piece + 0][n] = w.x; Bs[buf][piece + 1][n] = w.y;
-            Bs[buf][piece + 2][n] = w.z; Bs[buf][piece + 3][n] = w.w;
-        } else {     // B[k][n] = W[kk + k][n0 + n]: 16 rows x 64 cols
-            const int k = tid / 16, piece = (tid % 16) * 4;
-            cp_async16(&Bs[buf][k][piece], P.W + (int64_t)(kk + k) * E + n0 + piece, 16u);
-        }
-        asm volatile("cp.async.commit_group;" ::: "memory");
-    };
-    const int steps = (k1 - k0) / BK;
-    if (steps > 0) stage(k0, 0);
-    for (int s = 0; s < steps; ++s) {
-        if (s + 1 < steps) {
-            stage(k0 + (s + 1) * BK, (s + 1) & 1);
-            asm volatile("cp.async.wait_group 1;" ::: "memory");
-        } else {
-            asm volatile("cp.async.wait_group 0;" ::: "memory");
-        }
-        __syncthreads();
-        const int buf = s & 1;
-#pragma unroll
-        for (int k = 0; k < BK; ++k) {
-            float av[4];
-#pragma unroll
-            for (int a = 0; a < 4; ++a) av[a] = As[buf][ty * 4 + a][k];
-            const float4 bv = *reinterpret_cast<const float4*>(&Bs[buf][k][tx * 4]);
-            const float bb[4] = {bv.x, bv.y, bv.z, bv.w};
-#pragma unroll
-            for (int a = 0; a < 4; ++a)
-#pragma unroll
-                for (int c = 0; c < 4; ++c) acc[a][c] = fmaf(av[a], bb[c], acc[a][c]);
-        }
-        __syncthreads();
     }
+    __syncthreads();
+    float* red = lsm;                // [3 parts][128][25]: partial sums of K quarters 1..3 (aliases the staging)
+    if (part > 0) {
+        float* o = red + ((part - 1) * 128 + tt) * 25;
+#pragma unroll
+        for (int a = 0; a < 4; ++a)
+#pragma unroll
+            for (int g = 0; g < 3; ++g) { o[a * 6 + g * 2] = acc[a][g][0]; o[a * 6 + g * 2 + 1] = acc[a][g][1]; }
+    }
+    __syncthreads();
+    if (part > 0) return;
+#pragma unroll
+    for (int p = 0; p < 3; ++p) {
+        const float* o = red + (p * 128 + tt) * 25;
+#pragma unroll
+        for (int a = 0; a < 4; ++a)
+#pragma unroll
+            for (int g = 0; g < 3; ++g) { acc[a][g][0] += o[a * 6 + g * 2]; acc[a][g][1] += o[a * 6 + g * 2 + 1]; }
+    }
+    float bb[3][2];
+#pragma unroll
+    for (int g = 0; g < 3; ++g)
+#pragma unroll
+        for (int c = 0; c < 2; ++c) bb[g][c] = __ldg(b + g * H + j0 + up + 16 * c);
 #pragma unroll
     for (int a = 0; a < 4; ++a) {
-        const int row = m0 + ty * 4 + a;
-        if (row >= P.n_leaf) continue;
-        const uint32_t rec = P.leaves[2 * row], tok = P.leaves[2 * row + 1];
-        const int n = n0 + tx * 4;
-        if (FWD) {
-            *reinterpret_cast<float4*>(P.pool + rec + 2 * H + n) = make_float4(acc[a][0], acc[a][1], acc[a][2], acc[a][3]);
-        } else if (P.d_inputs) {
-            red_add<4>(P.d_inputs + (int64_t)tok * E + n, acc[a]);
+        const int l = l0 + 4 * lq + a;
+        if (l >= n_leaf) continue;
+        float* r = pool + leaves[2 * l];
+#pragma unroll
+        for (int c = 0; c < 2; ++c) {
+            const int j = j0 + up + 16 * c;
+            const float ig = sigm(acc[a][0][c] + bb[0][c]), og = sigm(acc[a][1][c] + bb[1][c]);
+            const float ug = tanhf(acc[a][2][c] + bb[2][c]);
+            const float cc = ig * ug;
+            r[j] = og * tanhf(cc);
+            r[H + j] = cc;
+            r[2 * H + j] = ig;
+            r[3 * H + j] = og;
+            r[4 * H + j] = ug;
         }
-    }
-}
-
-// leaf cell (Tai et al. [5] N-ary leaf): a = pre-activation + b_iou; c = σ(a_i) tanh(a_u); h = σ(a_o) tanh(c)
-__global__ void vpps_leaf_cell(const Params P) {
-    const int H = P.H;
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < (int64_t)P.n_leaf * H;
-         i += (int64_t)gridDim.x * blockDim.x) {
-        const int l = (int)(i / H), j = (int)(i - (int64_t)l * H);
-        float* r = P.pool + P.leaves[2 * l];
-        const float ig = sigm(r[2 * H + j] + __ldg(P.b + j));
-        const float og = sigm(r[3 * H + j] + __ldg(P.b + H + j));
-        const float ug = tanhf(r[4 * H + j] + __ldg(P.b + 2 * H + j));
-        const float c = ig * ug;
-        r[j] = og * tanhf(c);
-        r[H + j] = c;
-        r[2 * H + j] = ig;
-        r[3 * H + j] = og;
-        r[4 * H + j] = ug;
     }
 }
 
@@ -134,20 +130,13 @@ void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float*
                      int32_t n_leaf, int32_t H, int32_t E, cudaStream_t s) {
     using namespace dev::leaf;
     if (n_leaf <= 0) return;
-    Params p{W, b, inputs, pool, nullptr, leaves, n_leaf, H, E, 0};
-    const int tiles = ((n_leaf + BM - 1) / BM) * (3 * H / BN);
-    vpps_leaf_gemm<true><<<tiles, 256, 0, s>>>(p);
-    vpps_leaf_cell<<<(int)std::min<int64_t>(1184, ((int64_t)n_leaf * H + 255) / 256), 256, 0, s>>>(p);
-}
-
-void launch_leaf_dx(const float* W, const float* pool, float* d_inputs, const uint32_t* leaves, int32_t n_leaf,
-                    int32_t H, int32_t E, cudaStream_t s) {
-    using namespace dev::leaf;
-    if (n_leaf <= 0 || !d_inputs) return;
-    const int kchunk = 128;
-    Params p{W, nullptr, nullptr, const_cast<float*>(pool), d_inputs, leaves, n_leaf, H, E, kchunk};
-    const int tiles = ((n_leaf + BM - 1) / BM) * (E / BN) * ((3 * H + kchunk - 1) / kchunk);
-    vpps_leaf_gemm<false><<<tiles, 256, 0, s>>>(p);
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(vpps_leaf_fwd, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+        attr = true;
+    }
+    const int tiles = ((n_leaf + LM - 1) / LM) * (H / LU);
+    vpps_leaf_fwd<<<tiles, NT, SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H, E);
 }
 
 }  // namespace vpps

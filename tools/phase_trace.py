@@ -92,6 +92,8 @@ def main():
     print(f"sum work_max {work_tot/1e3:.1f} us, sum barrier {bar_tot/1e3:.1f} us")
     secs = raw[rows][:, 2 + 3 * (nbar + 1): 2 + 3 * (nbar + 1) + 10]
     names = ["decode", "staging", "matvec", "cell", "cell-bwd", "outer/tmv", "heads", "signal", "wait", "other"]
+    if args.cluster:
+        names = ["decode", "staging", "forward", "cell-bwd", "transp", "heads", "arrive", "wait", "tail", "other"]
     mean = secs.mean(0)
     mx = secs[secs.sum(1).argmax()]
     tot = mean.sum()
