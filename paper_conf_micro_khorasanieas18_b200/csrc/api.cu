@@ -62,6 +62,8 @@ struct vpps_model_s {
     uint64_t* prof = nullptr;
     int64_t prof_stride = 0;
     int32_t cluster = 0;                // > 1: cluster-replica path (vpps_cluster.cu)
+    int32_t* done = nullptr;            // cluster path: per-group completion counters [kMaxGroups]
+    static constexpr int kMaxGroups = 16;
     // Pre-allocated staging ring for per-batch scripts: a pinned host buffer and a
     // device buffer per slot; a slot is reused once the kernel that last read it has finished.
     struct Slot {
@@ -171,6 +173,8 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     m->plan.by_graph = m->cluster != 0;
     if (m->cluster && m->plan.n_g != m->cluster) return fail(VPPS_E_INVALID, "groups x cluster must equal n_sm");
     if (m->cluster && !m->plan_only) {
+        if (m->plan.G > vpps_model_s::kMaxGroups) return fail(VPPS_E_NOFIT, "more than 16 cluster replicas");
+        CK(cudaMalloc(&m->done, vpps_model_s::kMaxGroups * sizeof(int32_t)));
         CK(cudaMallocHost(&m->h_loss, 2 * sizeof(float)));
         m->h_loss[0] = m->h_loss[1] = 0.f;
         CK(cudaEventCreateWithFlags(&m->ev[0], cudaEventDisableTiming));
@@ -357,6 +361,7 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     }
     CK(cudaMemsetAsync(m->pool, 0, s->s.zero_words * sizeof(float), st));
     if (m->plan.G > 1 || m->cluster) CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));
+    if (m->cluster) CK(cudaMemsetAsync(m->done, 0, vpps_model_s::kMaxGroups * sizeof(int32_t), st));
     if (d_inputs) CK(cudaMemsetAsync(d_inputs, 0, (size_t)n_rows * m->plan.E * sizeof(float), st));
     KParams kp{};
     kp.params = m->params;
@@ -381,19 +386,25 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     void* args[] = {&kp};
     if (m->t_before) CK(cudaEventRecord(m->t_before, st));
     if (m->cluster) {
-        // one cluster per replica group; clusters never wait on each other (graphs are whole per group)
+        // one cluster per replica group; clusters never wait on each other (graphs are whole per group).
+        // Launch order: leaf GEMM -> vpps_cl (programmatic dependent: weight prologue overlaps the leaf
+        // tail, griddepcontrol.wait before level 1) -> gradient GEMM (programmatic dependent: a group's
+        // tiles start when its cluster's 16 CTAs have counted themselves done) -> SGD.
+        kp.done = m->done;
         cudaLaunchConfig_t cfg = {};
-        cudaLaunchAttribute attr[1];
+        cudaLaunchAttribute attr[2];
         attr[0].id = cudaLaunchAttributeClusterDimension;
         attr[0].val.clusterDim.x = m->cluster;
         attr[0].val.clusterDim.y = 1;
         attr[0].val.clusterDim.z = 1;
+        attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        attr[1].val.programmaticStreamSerializationAllowed = 1;
         cfg.gridDim = dim3(m->plan.n_cta);
         cfg.blockDim = dim3(256);
         cfg.dynamicSmemBytes = m->smem;
         cfg.stream = st;
         cfg.attrs = attr;
-        cfg.numAttrs = 1;
+        cfg.numAttrs = 2;
         const uint32_t* lists = dwords + s->s.words.size();
         const uint32_t* leaf_list = lists + 3 * s->s.n_int;
         const float* W_iou = m->params + m->offsets[0];
@@ -402,9 +413,18 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
                         m->plan.H, m->plan.E, st);
         CK(cudaLaunchKernelExC(&cfg, m->var->fn, args));
         // dW of the weight matrices from the recorded operands and dX of the leaves
-        // = W_iouᵀ g_leaf (words are inputs) in one launch; SGD in mode 1
-        launch_dw_gemm(m->pool, inputs, d_inputs, m->params, m->grads, lists, (int32_t)s->s.n_int, leaf_list,
-                       (int32_t)s->s.n_leaf, m->plan.H, m->plan.E, m->offsets.data(), m->n_floats, mode, lr, wd, st);
+        // = W_iouᵀ g_leaf (words are inputs) in one launch; SGD in mode 1.  Groups whose
+        // cluster should finish first (fewest levels, then fewest nodes) get the lowest tile indices.
+        const int32_t n_grp = (int32_t)s->s.int_off.size() - 1;
+        std::vector<int32_t> order(n_grp);
+        for (int32_t g = 0; g < n_grp; ++g) order[g] = g;
+        std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
+            if (s->s.grp_levels[a] != s->s.grp_levels[b]) return s->s.grp_levels[a] < s->s.grp_levels[b];
+            return s->s.grp_nodes[a] < s->s.grp_nodes[b];
+        });
+        launch_dw_gemm(m->pool, inputs, d_inputs, m->params, m->grads, lists, leaf_list, n_grp, s->s.int_off.data(),
+                       s->s.leaf_off.data(), order.data(), m->done, m->cluster, true, m->plan.H, m->plan.E,
+                       m->offsets.data(), m->n_floats, mode, lr, wd, st);
         CK(cudaGetLastError());
     } else {
         CK(cudaLaunchCooperativeKernel(m->var->fn, dim3(m->plan.n_cta), dim3(256), args, m->smem, st));
@@ -489,6 +509,7 @@ void vpps_destroy_script(vpps_script s) {
 void vpps_destroy_model(vpps_model m) {
     if (!m) return;
     if (m->pool) cudaFree(m->pool);
+    if (m->done) cudaFree(m->done);
     if (m->h_loss) cudaFreeHost(m->h_loss);
     for (cudaEvent_t e : m->ev)
         if (e) cudaEventDestroy(e);

@@ -58,6 +58,9 @@ struct Script {
     // lists drive the gradient GEMM of the cluster path.  Not part of the SPEC words.
     std::vector<uint32_t> blob;
     int64_t n_int = 0, n_leaf = 0;
+    // per replica group g (S5g plans; one group otherwise): its internal / leaf nodes are list entries
+    // [int_off[g], int_off[g+1]) / [leaf_off[g], leaf_off[g+1]); node count and deepest level
+    std::vector<int32_t> int_off, leaf_off, grp_nodes, grp_levels;
     double flops = 0.0, act_bytes = 0.0;
 };
 

@@ -261,19 +261,41 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     s.flops = flops;
     s.act_bytes = abytes;
     // device blob: the words, then the operand lists of the per-matrix gradient GEMM (binary cells)
+    // (grouped by replica group when graphs are assigned whole, S5g: the GEMM tiles of a group can then
+    // start as soon as that group's cluster has finished)
     s.blob = s.words;
     s.n_int = s.n_leaf = 0;
-    for (int64_t i = 0; i < N; ++i)
-        if (nodes[i].kind == K_INT) {
-            const int32_t* ch = kids.data() + nodes[i].ch_begin;
-            s.blob.insert(s.blob.end(), {rec[i], rec[ch[0]], rec[ch[1]]});
-            ++s.n_int;
-        }
-    for (int64_t i = 0; i < N; ++i)
-        if (nodes[i].kind == K_LEAF) {
-            s.blob.insert(s.blob.end(), {rec[i], (uint32_t)nodes[i].token});
-            ++s.n_leaf;
-        }
+    const int32_t n_grp = plan.by_graph ? G : 1;
+    auto group_of = [&](int64_t i) { return plan.by_graph ? graph_group[nodes[i].graph] : 0; };
+    s.int_off.assign(n_grp + 1, 0);
+    s.leaf_off.assign(n_grp + 1, 0);
+    s.grp_nodes.assign(n_grp, 0);
+    s.grp_levels.assign(n_grp, 0);
+    for (int64_t i = 0; i < N; ++i) {
+        if (nodes[i].kind == K_HEAD) continue;
+        const int32_t g = group_of(i);
+        ++s.grp_nodes[g];
+        s.grp_levels[g] = std::max(s.grp_levels[g], level[i]);
+    }
+    for (int32_t g = 0; g < n_grp; ++g) {
+        s.int_off[g] = (int32_t)s.n_int;
+        for (int64_t i = 0; i < N; ++i)
+            if (nodes[i].kind == K_INT && group_of(i) == g) {
+                const int32_t* ch = kids.data() + nodes[i].ch_begin;
+                s.blob.insert(s.blob.end(), {rec[i], rec[ch[0]], rec[ch[1]]});
+                ++s.n_int;
+            }
+    }
+    s.int_off[n_grp] = (int32_t)s.n_int;
+    for (int32_t g = 0; g < n_grp; ++g) {
+        s.leaf_off[g] = (int32_t)s.n_leaf;
+        for (int64_t i = 0; i < N; ++i)
+            if (nodes[i].kind == K_LEAF && group_of(i) == g) {
+                s.blob.insert(s.blob.end(), {rec[i], (uint32_t)nodes[i].token});
+                ++s.n_leaf;
+            }
+    }
+    s.leaf_off[n_grp] = (int32_t)s.n_leaf;
     return 0;
 }
 

@@ -144,6 +144,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
     const int j = lc + u * NCL;                                 // hidden unit of this thread
     const bool holds_head = (lc == H % NCL);
 
+    // the gradient GEMM may launch now (programmatic dependent launch): its tiles wait on P.done per group
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     // ---- prologue: this CTA's slice of every weight matrix DRAM -> registers (L123, L129) ----
     // Only the recurrent matrices (U_iou, U_fl, U_fr) live in registers: the leaf level is one dense
     // GEMM over all leaves (same W_iou), done by vpps_leaf_fwd / vpps_leaf_dx around this kernel.
@@ -196,6 +198,9 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
             sec_last = now;
         }
     };
+    // the leaf level (vpps_leaf_fwd, the preceding grid) must be complete and visible from here on; the
+    // weight loads above overlapped its tail
+    asm volatile("griddepcontrol.wait;" ::: "memory");
     __syncthreads();
     if (prof && tid == 0) { prof[0] = gtimer(); sec_last = clock64(); }
 
@@ -594,6 +599,13 @@ __global__ void __launch_bounds__(NTH, 1) vpps_cl(const KParams P) {
         for (int i = tid; i < C * H; i += NTH) atomicAdd(P.grads + off[4] + i, dWo[i]);
         for (int i = tid; i < C; i += NTH) atomicAdd(P.grads + off[7] + i, dbo[i]);
     }
+    // this CTA's records and gradient contributions are complete: count it for the gradient GEMM tiles
+    // of its group (release: every thread fences its own writes, then one increment per CTA)
+    if (P.done) {
+        __threadfence();
+        __syncthreads();
+        if (tid == 0) atomicAdd(P.done + grp, 1);
+    }
 }
 
 // ---- dW = Σ_nodes g xᵀ per weight matrix ("concatenate all the left hand side and all the
@@ -605,13 +617,18 @@ struct GemmParams {
     const float* pool;
     const float* inputs;
     float* grads;
-    const uint32_t* int_nodes;   // n_int x (rec, rec_l, rec_r)
-    const uint32_t* leaf_nodes;  // n_leaf x (rec, token)
-    int32_t n_int, n_leaf, H, E;
+    const uint32_t* int_nodes;   // n_int x (rec, rec_l, rec_r), grouped by replica group
+    const uint32_t* leaf_nodes;  // n_leaf x (rec, token), grouped by replica group
+    int32_t H, E;
     int64_t off[8];
     const float* w_iou;          // W_iou (params), for the leaf input gradient
     float* d_inputs;             // dX, or nullptr
-    int32_t items[5];            // work items per job (dU_iou, dU_fl, dU_fr, dW_iou, leaf dX)
+    const int32_t* done;         // per-group completion counters written by vpps_cl (nullptr: no wait)
+    int32_t done_target;         // CTAs per cluster
+    int32_t n_grp;
+    int32_t grp[16];             // groups in processing order (clusters expected to finish first go first)
+    int32_t int_off[17], leaf_off[17];
+    int32_t items[16];           // work items of grp[q]
 };
 
 constexpr int TM = 128;          // tile rows (gate-gradient rows)
@@ -620,13 +637,18 @@ constexpr int KS = 16;           // nodes per pipeline stage
 constexpr int KCH = 96;          // nodes per work item (split-K)
 constexpr int NST = 3;           // cp.async pipeline stages
 
+// work items of one group: job m = 0 dU_iou, 1 dU_fl, 2 dU_fr, 3 dW_iou (split-K over the group's nodes),
+// 4 leaf dX (split-K over the 3H gate rows)
+__host__ __device__ inline int job_items(int m, int n_int, int n_leaf, int H, int E, bool dx);
+
 // leaf input gradient dX[tok_l] += Σ_r g_l[r] W_iou[r][:] (word vectors are inputs of the
 // leaves).  Tile 64 leaves x 64 columns, split-K over the 3H gate rows in chunks of DXK, 4 x 4 per thread;
 // the leaf gate gradients are staged row-major ([leaf][k], stride 20: conflict-free column reads).
 constexpr int DXM = 64, DXN = 64, DXK = 128, DXS = 20;
-__device__ __forceinline__ void leaf_dx_tile(const GemmParams& P, int b, float* As, float* Bs) {
+__device__ __forceinline__ void leaf_dx_tile(const GemmParams& P, const uint32_t* leaf_nodes, int n_leaf, int b,
+                                             float* As, float* Bs) {
     const int tid = threadIdx.x, H = P.H, E = P.E;
-    const int tiles_c = E / DXN, tiles_r = (P.n_leaf + DXM - 1) / DXM;
+    const int tiles_c = E / DXN, tiles_r = (n_leaf + DXM - 1) / DXM;
     const int kc = b / (tiles_r * tiles_c), t = b - kc * (tiles_r * tiles_c);
     const int r0 = (t / tiles_c) * DXM, c0 = (t % tiles_c) * DXN;
     const int k0 = kc * DXK, k1 = min(3 * H, k0 + DXK);
@@ -637,7 +659,7 @@ __device__ __forceinline__ void leaf_dx_tile(const GemmParams& P, int b, float* 
     auto stage = [&](int s, int buf) {
         {
             const int l = tid / 4, piece = (tid % 4) * 4, row = r0 + l;
-            const float* src = row < P.n_leaf ? P.pool + P.leaf_nodes[2 * row] + 5 * H + k0 + s * KS + piece : nullptr;
+            const float* src = row < n_leaf ? P.pool + leaf_nodes[2 * row] + 5 * H + k0 + s * KS + piece : nullptr;
             cp_async16(As + buf * DXM * DXS + l * DXS + piece, src ? src : P.pool, src ? 16u : 0u);
         }
         {
@@ -679,21 +701,57 @@ __device__ __forceinline__ void leaf_dx_tile(const GemmParams& P, int b, float* 
     for (int a = 0; a < 4; ++a) {
         const int row = r0 + ty + 16 * a;
         const float v[4] = {acc2[a][0].x, acc2[a][0].y, acc2[a][1].x, acc2[a][1].y};
-        if (row < P.n_leaf) red_add<4>(P.d_inputs + (int64_t)P.leaf_nodes[2 * row + 1] * E + c0 + tx * 4, v);
+        if (row < n_leaf) red_add<4>(P.d_inputs + (int64_t)leaf_nodes[2 * row + 1] * E + c0 + tx * 4, v);
     }
 }
 
-__global__ void __launch_bounds__(256) vpps_dw_gemm(const GemmParams P) {
+__host__ __device__ inline int job_items(int m, int n_int, int n_leaf, int H, int E, bool dx) {
+    const int ki = (n_int + KCH - 1) / KCH, kl = (n_leaf + KCH - 1) / KCH;
+    switch (m) {
+        case 0: return (3 * H / TM) * (2 * H / TN) * ki;
+        case 1:
+        case 2: return (H / TM) * (H / TN) * ki;
+        case 3: return (3 * H / TM) * (E / TN) * kl;
+        default: return (dx && n_leaf > 0) ? ((n_leaf + DXM - 1) / DXM) * (E / DXN) * ((3 * H + DXK - 1) / DXK) : 0;
+    }
+}
+
+__global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
     __shared__ __align__(16) float Gs[NST][KS][TM];
     __shared__ __align__(16) float Xs[NST][KS][TN];
     const int tid = threadIdx.x, H = P.H, E = P.E;
-    int b = blockIdx.x, m = 0;
-    while (m < 5 && b >= P.items[m]) { b -= P.items[m]; ++m; }
+    // item -> (group g, job m, local index b)
+    int b = blockIdx.x, q = 0;
+    while (q < P.n_grp && b >= P.items[q]) { b -= P.items[q]; ++q; }
+    if (q == P.n_grp) return;
+    const int g = P.grp[q];
+    const int n_int = P.int_off[g + 1] - P.int_off[g], n_leaf = P.leaf_off[g + 1] - P.leaf_off[g];
+    const uint32_t* int_nodes = P.int_nodes + 3 * P.int_off[g];
+    const uint32_t* leaf_nodes = P.leaf_nodes + 2 * P.leaf_off[g];
+    int m = 0;
+    while (m < 5) {
+        const int n = job_items(m, n_int, n_leaf, H, E, P.d_inputs != nullptr);
+        if (b < n) break;
+        b -= n;
+        ++m;
+    }
     if (m == 5) return;
-    if (m == 4) { leaf_dx_tile(P, b, &Gs[0][0][0], &Xs[0][0][0]); return; }
+    // launched early (programmatic dependent launch): wait until every CTA of this group's cluster is done
+    if (P.done) {
+        if (tid == 0) {
+            uint32_t v;
+            while (true) {
+                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(P.done + g) : "memory");
+                if ((int)v >= P.done_target) break;
+                __nanosleep(200);
+            }
+        }
+        __syncthreads();
+    }
+    if (m == 4) { leaf_dx_tile(P, leaf_nodes, n_leaf, b, &Gs[0][0][0], &Xs[0][0][0]); return; }
     const int rows = (m == 0 || m == 3) ? 3 * H : H;
     const int cols = m == 0 ? 2 * H : (m == 3 ? E : H);
-    const int K = m == 3 ? P.n_leaf : P.n_int;
+    const int K = m == 3 ? n_leaf : n_int;
     const int tiles_r = rows / TM, tiles_c = cols / TN;
     const int kc = b / (tiles_r * tiles_c), t = b - kc * (tiles_r * tiles_c);
     const int r0 = (t / tiles_c) * TM, c0 = (t % tiles_c) * TN;
@@ -711,7 +769,7 @@ __global__ void __launch_bounds__(256) vpps_dw_gemm(const GemmParams P) {
             const int node = k0 + s * KS + k;
             const float* src = nullptr;
             if (node < k1) {
-                const uint32_t rec = m == 3 ? P.leaf_nodes[2 * node] : P.int_nodes[3 * node];
+                const uint32_t rec = m == 3 ? leaf_nodes[2 * node] : int_nodes[3 * node];
                 src = P.pool + rec + goff + r0 + piece;
             }
             cp_async16(&Gs[buf][k][piece], src ? src : P.pool, src ? 16u : 0u);
@@ -723,9 +781,9 @@ __global__ void __launch_bounds__(256) vpps_dw_gemm(const GemmParams P) {
             if (node < k1) {
                 const int c = c0 + piece;
                 if (m == 3) {
-                    src = P.inputs + (int64_t)P.leaf_nodes[2 * node + 1] * E + c;
+                    src = P.inputs + (int64_t)leaf_nodes[2 * node + 1] * E + c;
                 } else {
-                    const uint32_t xl = P.int_nodes[3 * node + 1], xr = P.int_nodes[3 * node + 2];
+                    const uint32_t xl = int_nodes[3 * node + 1], xr = int_nodes[3 * node + 2];
                     if (m == 0) src = c < H ? P.pool + xl + c : P.pool + xr + (c - H);
                     else src = P.pool + (m == 1 ? xl : xr) + c;
                 }
@@ -789,25 +847,44 @@ const Variant* cluster_variants(int32_t* n) {
 }
 
 void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, float* params, float* grads,
-                    const uint32_t* int_nodes, int32_t n_int, const uint32_t* leaf_nodes, int32_t n_leaf, int32_t H,
-                    int32_t E, const int64_t* off, int64_t n_floats, int32_t mode, float lr, float wd, cudaStream_t s) {
+                    const uint32_t* int_nodes, const uint32_t* leaf_nodes, int32_t n_grp, const int32_t* int_off,
+                    const int32_t* leaf_off, const int32_t* order, const int32_t* done, int32_t done_target,
+                    bool early, int32_t H, int32_t E, const int64_t* off, int64_t n_floats, int32_t mode, float lr,
+                    float wd, cudaStream_t s) {
     using namespace dev::cl;
     GemmParams g{};
     g.pool = pool; g.inputs = inputs; g.grads = grads;
-    g.int_nodes = int_nodes; g.leaf_nodes = leaf_nodes; g.n_int = n_int; g.n_leaf = n_leaf;
+    g.int_nodes = int_nodes; g.leaf_nodes = leaf_nodes;
     g.H = H; g.E = E;
     for (int i = 0; i < 8; ++i) g.off[i] = off[i];
-    const int ki = (n_int + KCH - 1) / KCH, kl = (n_leaf + KCH - 1) / KCH;
-    g.items[0] = (3 * H / TM) * (2 * H / TN) * ki;
-    g.items[1] = (H / TM) * (H / TN) * ki;
-    g.items[2] = g.items[1];
-    g.items[3] = (3 * H / TM) * (E / TN) * kl;
     g.w_iou = params + off[0];
     g.d_inputs = d_inputs;
-    g.items[4] = d_inputs ? ((n_leaf + DXM - 1) / DXM) * (E / DXN) * ((3 * H + DXK - 1) / DXK) : 0;
-    if (n_leaf == 0) g.items[4] = 0;
-    const int items = g.items[0] + g.items[1] + g.items[2] + g.items[3] + g.items[4];
-    if (items > 0) vpps_dw_gemm<<<items, 256, 0, s>>>(g);
+    g.done = done;
+    g.done_target = done_target;
+    g.n_grp = n_grp;
+    int items = 0;
+    for (int q = 0; q < n_grp; ++q) {
+        const int gi = order ? order[q] : q;
+        g.grp[q] = gi;
+        const int ni = int_off[gi + 1] - int_off[gi], nl = leaf_off[gi + 1] - leaf_off[gi];
+        int n = 0;
+        for (int m = 0; m < 5; ++m) n += job_items(m, ni, nl, H, E, d_inputs != nullptr);
+        g.items[q] = n;
+        items += n;
+    }
+    for (int i = 0; i <= n_grp; ++i) { g.int_off[i] = int_off[i]; g.leaf_off[i] = leaf_off[i]; }
+    if (items > 0) {
+        cudaLaunchConfig_t cfg = {};
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        attr[0].val.programmaticStreamSerializationAllowed = 1;
+        cfg.gridDim = dim3(items);
+        cfg.blockDim = dim3(256);
+        cfg.stream = s;
+        cfg.attrs = attr;
+        cfg.numAttrs = early ? 1 : 0;
+        cudaLaunchKernelEx(&cfg, vpps_dw_gemm, g);
+    }
     if (mode == 1) launch_sgd(params, grads, n_floats, lr, wd, s);   // W -= lr (dW + wd W), every parameter
 }
 

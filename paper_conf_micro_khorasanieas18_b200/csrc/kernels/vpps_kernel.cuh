@@ -19,6 +19,7 @@ struct KParams {
     float lr, wd;
     uint64_t* prof;         // optional globaltimer trace (vpps_set_profile_buffer), or nullptr
     int64_t prof_stride;
+    int32_t* done;          // cluster path: per-group completion counters (one increment per CTA), or nullptr
 };
 
 struct Variant {
@@ -32,10 +33,14 @@ const Variant* variants(int32_t* n);
 // Cluster-replica specialisations (vpps_cluster.cu); Variant.umax holds the cluster size.
 const Variant* cluster_variants(int32_t* n);
 // dW = Σ g xᵀ per weight matrix from the recorded operands, fused SGD when mode == 1.
-// Also forms the leaf input gradient dX[tok] += W_iouᵀ g_leaf when d_inputs is not null.
+// Also forms the leaf input gradient dX[tok] += W_iouᵀ g_leaf when d_inputs is not null.  Node lists are
+// grouped by replica group (offsets int_off / leaf_off, n_grp + 1 entries); with `early` the kernel is a
+// programmatic dependent launch of vpps_cl and each group's tiles wait for done[group] >= done_target.
 void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, float* params, float* grads,
-                    const uint32_t* int_nodes, int32_t n_int, const uint32_t* leaf_nodes, int32_t n_leaf, int32_t H,
-                    int32_t E, const int64_t* off, int64_t n_floats, int32_t mode, float lr, float wd, cudaStream_t s);
+                    const uint32_t* int_nodes, const uint32_t* leaf_nodes, int32_t n_grp, const int32_t* int_off,
+                    const int32_t* leaf_off, const int32_t* order, const int32_t* done, int32_t done_target,
+                    bool early, int32_t H, int32_t E, const int64_t* off, int64_t n_floats, int32_t mode, float lr,
+                    float wd, cudaStream_t s);
 // Leaf level of the binary cell as one GEMM + fused cell (vpps_leaf.cu): records h, c, i, o, u of every
 // leaf before the cluster kernel.
 void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float* pool, const uint32_t* leaves,
