@@ -165,7 +165,10 @@ def main():
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--groups", type=int, default=4, help="replica groups G (SPEC P1); 148 = 4 x 37")
     ap.add_argument("--cluster", type=int, default=16,
-                    help="> 1: cluster-replica path (one 16-CTA cluster per replica, SPEC S5g)")
+                    help="> 1: whole-graph replica groups of this many CTAs (SPEC S5g)")
+    ap.add_argument("--sync", choices=["dataflow", "cluster"], default="dataflow",
+                    help="dataflow: epoch-tagged slots, cooperative groups (vpps_df); cluster: hardware "
+                         "cluster barrier (vpps_cl)")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
 
@@ -190,7 +193,8 @@ def main():
     shapes = vpps.param_shapes("binary", H, E, C)
     P = synth.init_params(shapes, rng)
     X = synth.input_table(rng, V, E)
-    m = vpps.Model("binary", H, E, C, device=local, groups=args.groups, cluster=args.cluster)
+    m = vpps.Model("binary", H, E, C, device=local, groups=args.groups, cluster=args.cluster,
+                   dataflow=bool(args.cluster) and args.sync == "dataflow")
     params = torch.zeros(m.n_floats, dtype=torch.float32, device=dev)
     grads = torch.zeros_like(params)
     for name, _ in shapes:
@@ -299,11 +303,12 @@ def main():
                        "seq_len": None, "parallelism": f"dp{world}",
                        "replica_groups": m.plan_info()["n_cta"] // m.plan_info()["n_g"],
                        "cluster": args.cluster or None, "ctas": m.plan_info()["n_cta"],
-                       "mode": ("leaf GEMM + leaf cell + cluster fwd/bwd + leaf dX GEMM + dW GEMM + SGD" if args.cluster
+                       "sync": (args.sync if args.cluster else "grid barrier"),
+                       "mode": ("leaf GEMM + replica-group fwd/bwd + dW/dX GEMM + SGD" if args.cluster
                                 else "fused fwd-bwd-sgd, 1 kernel") + ("" if world == 1 else ", NCCL all-reduce before SGD"),
                        "l2": "no flush" if args.no_flush else "flushed (256 MiB write) before every timed step",
                        "batches": f"{N_BATCHES} distinct pre-built scripts cycled"},
-            "gpu_launches": args.steps * (6 if args.cluster else (1 if world == 1 else 2)),
+            "gpu_launches": args.steps * (4 if args.cluster else (1 if world == 1 else 2)),
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "kernel_ms": kern_ms / args.steps, "flops_per_launch": avg_flops,

@@ -80,6 +80,10 @@ typedef struct {
                             that owns whole graphs (SPEC S5g), synchronised by the hardware
                             cluster barrier; groups = the number of co-resident clusters (or the
                             given `groups` when plan_only).  0 = grid-wide groups (SPEC S5). */
+    int32_t dataflow;    /* 1 (with cluster = 16): the groups are ordinary co-resident CTAs of a
+                            cooperative launch (floor(n_sm / 16) groups) and the signal/wait of L165
+                            is replaced by epoch-tagged 64-bit slots that consumers poll (vpps_df);
+                            0 = barrier synchronisation. */
 } vpps_options;
 
 /* A batch of graphs in CSR form (the super-graph of L205 is built from it).

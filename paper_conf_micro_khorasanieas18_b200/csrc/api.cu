@@ -63,6 +63,8 @@ struct vpps_model_s {
     int64_t prof_stride = 0;
     int32_t cluster = 0;                // > 1: cluster-replica path (vpps_cluster.cu)
     int32_t* done = nullptr;            // cluster path: per-group completion counters [kMaxGroups]
+    bool dataflow = false;              // groups of co-resident CTAs synchronised by tagged slots (vpps_df)
+    uint32_t epoch = 0;                 // dataflow pass counter (slot tags)
     static constexpr int kMaxGroups = 16;
     // Pre-allocated staging ring for per-batch scripts: a pinned host buffer and a
     // device buffer per slot; a slot is reused once the kernel that last read it has finished.
@@ -127,6 +129,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     m->n_floats = cur;
     int32_t n_sm = o.n_sm;
     m->cluster = o.cluster > 1 ? o.cluster : 0;
+    m->dataflow = m->cluster && o.dataflow;
     if (!m->plan_only) {
         m->device = o.device;
         CK(cudaSetDevice(o.device));
@@ -138,7 +141,23 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     } else if (n_sm == 0) {
         n_sm = m->cluster ? m->cluster * o.groups : 148;
     }
-    if (m->cluster && !m->plan_only) {
+    if (m->dataflow && !m->plan_only) {
+        // dataflow groups (SPEC S5g): floor(n_sm / cluster) groups of co-resident CTAs (cooperative launch)
+        int32_t nv = 0;
+        const Variant* v = df_variants(&nv);
+        for (int32_t i = 0; i < nv; ++i)
+            if (v[i].cell == cell && v[i].H == H && v[i].E == E && v[i].umax == m->cluster) m->var = &v[i];
+        if (!m->var) return fail(VPPS_E_NOFIT, "no dataflow specialisation for this op set and group size");
+        if (C > 32) return fail(VPPS_E_NOFIT, "single-CTA loss head supports C <= 32 classes in v1");
+        m->smem = m->var->smem_bytes(C);
+        CK(cudaFuncSetAttribute(m->var->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)m->smem));
+        int per_sm = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, m->var->fn, 256, m->smem));
+        if (per_sm < 1) return fail(VPPS_E_NOFIT, "dataflow kernel does not fit on an SM");
+        o.groups = std::min(n_sm / m->cluster, vpps_model_s::kMaxGroups);
+        if (o.groups < 1) return fail(VPPS_E_NOFIT, "fewer SMs than one group");
+        n_sm = o.groups * m->cluster;
+    } else if (m->cluster && !m->plan_only) {
         // cluster replicas (SPEC S5g): one group per co-resident cluster of `cluster` CTAs
         int32_t nv = 0;
         const Variant* v = cluster_variants(&nv);
@@ -346,12 +365,16 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     if (((uintptr_t)inputs | (uintptr_t)d_inputs) & 15) return fail(VPPS_E_INVALID, "input tables must be 16-byte aligned");
     cudaStream_t st = (cudaStream_t)stream_;
     CK(cudaSetDevice(m->device));
-    if (s->s.pool_words > m->pool_cap) {
+    const int64_t need = s->s.pool_words + (m->dataflow ? s->s.df_words : 0);
+    if (need > m->pool_cap) {
         if (m->pool) { CK(cudaStreamSynchronize(st)); CK(cudaFree(m->pool)); m->pool = nullptr; }
-        const int64_t cap = s->s.pool_words + s->s.pool_words / 4 + 1024;
+        const int64_t cap = need + need / 4 + 1024;
         CK(cudaMalloc(&m->pool, cap * sizeof(float)));
+        // tagged slots (dataflow) must never carry a live epoch before they are written: zero once
+        CK(cudaMemsetAsync(m->pool, 0, cap * sizeof(float), st));
         m->pool_cap = cap;
     }
+    if (m->dataflow && s->s.df_off < 0) return fail(VPPS_E_INVALID, "script has no dataflow program (binary cell only)");
     m->last_pool_words = s->s.pool_words;
     int ring_slot = -1;
     const uint32_t* dwords = s->d_words;
@@ -379,13 +402,65 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     kp.loss_word = s->s.loss_word;
     kp.lr = lr;
     kp.wd = wd;
-    if (m->prof && m->prof_stride < 2 + 3 * (int64_t)(s->s.n_bar + 1) + 10 * (int64_t)(s->s.n_bar + 2))
+    if (m->prof && !m->dataflow && m->prof_stride < 2 + 3 * (int64_t)(s->s.n_bar + 1) + 10 * (int64_t)(s->s.n_bar + 2))
         return fail(VPPS_E_INVALID, "profile buffer stride too small for this script");
+    if (m->prof && m->dataflow && m->prof_stride < 11) return fail(VPPS_E_INVALID, "profile buffer stride < 11");
     kp.prof = m->prof;
     kp.prof_stride = m->prof_stride;
     void* args[] = {&kp};
     if (m->t_before) CK(cudaEventRecord(m->t_before, st));
-    if (m->cluster) {
+    if (m->dataflow) {
+        // leaf GEMM -> vpps_df (cooperative: the groups' CTAs must be co-resident because consumers
+        // spin on producers; programmatic dependent: weight prologue overlaps the leaf tail) -> gradient
+        // GEMM (programmatic dependent, per-group completion counters) -> SGD
+        DfParams dp{};
+        dp.params = m->params;
+        dp.grads = m->grads;
+        dp.pool = m->pool;
+        dp.script = dwords;
+        dp.df_off = s->s.df_off;
+        for (size_t i = 0; i < m->offsets.size() && i < 8; ++i) dp.off[i] = m->offsets[i];
+        dp.C = m->plan.C;
+        dp.epoch = ++m->epoch;
+        if (dp.epoch == 0) dp.epoch = ++m->epoch;      // 0 is the value of never-written slots
+        dp.loss_word = s->s.loss_word;
+        dp.df_hx = s->s.df_hx;
+        dp.df_part = s->s.df_part;
+        dp.df_hd = s->s.df_hd;
+        dp.prof = m->prof;
+        dp.prof_stride = m->prof_stride;
+        dp.done = m->done;
+        void* dargs[] = {&dp};
+        cudaLaunchConfig_t cfg = {};
+        cudaLaunchAttribute attr[2];
+        attr[0].id = cudaLaunchAttributeCooperative;
+        attr[0].val.cooperative = 1;
+        attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        attr[1].val.programmaticStreamSerializationAllowed = 1;
+        cfg.gridDim = dim3(m->plan.n_cta);
+        cfg.blockDim = dim3(256);
+        cfg.dynamicSmemBytes = m->smem;
+        cfg.stream = st;
+        cfg.attrs = attr;
+        cfg.numAttrs = 2;
+        const uint32_t* lists = dwords + s->s.words.size();
+        const uint32_t* leaf_list = lists + 3 * s->s.n_int;
+        const float* W_iou = m->params + m->offsets[0];
+        launch_leaf_fwd(W_iou, m->params + m->offsets[5], inputs, m->pool, leaf_list, (int32_t)s->s.n_leaf,
+                        m->plan.H, m->plan.E, st);
+        CK(cudaLaunchKernelExC(&cfg, m->var->fn, dargs));
+        const int32_t n_grp = (int32_t)s->s.int_off.size() - 1;
+        std::vector<int32_t> order(n_grp);
+        for (int32_t g = 0; g < n_grp; ++g) order[g] = g;
+        std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
+            if (s->s.grp_levels[a] != s->s.grp_levels[b]) return s->s.grp_levels[a] < s->s.grp_levels[b];
+            return s->s.grp_nodes[a] < s->s.grp_nodes[b];
+        });
+        launch_dw_gemm(m->pool, inputs, d_inputs, m->params, m->grads, lists, leaf_list, n_grp, s->s.int_off.data(),
+                       s->s.leaf_off.data(), order.data(), m->done, m->cluster, true, m->plan.H, m->plan.E,
+                       m->offsets.data(), m->n_floats, mode, lr, wd, st);
+        CK(cudaGetLastError());
+    } else if (m->cluster) {
         // one cluster per replica group; clusters never wait on each other (graphs are whole per group).
         // Launch order: leaf GEMM -> vpps_cl (programmatic dependent: weight prologue overlaps the leaf
         // tail, griddepcontrol.wait before level 1) -> gradient GEMM (programmatic dependent: a group's

@@ -61,6 +61,10 @@ struct Script {
     // per replica group g (S5g plans; one group otherwise): its internal / leaf nodes are list entries
     // [int_off[g], int_off[g+1]) / [leaf_off[g], leaf_off[g+1]); node count and deepest level
     std::vector<int32_t> int_off, leaf_off, grp_nodes, grp_levels;
+    // dataflow program of the binary cell for whole-graph groups (vpps_df): blob word offset (-1: none),
+    // tagged-slot counts and their pool word offsets (regions behind pool_words, df_words long)
+    int64_t df_off = -1, n_hx = 0, n_part = 0, n_hd = 0;
+    int64_t df_hx = 0, df_part = 0, df_hd = 0, df_words = 0;
     double flops = 0.0, act_bytes = 0.0;
 };
 

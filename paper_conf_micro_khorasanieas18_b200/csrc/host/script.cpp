@@ -296,6 +296,105 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
             }
     }
     s.leaf_off[n_grp] = (int32_t)s.n_leaf;
+
+    // ---- dataflow lowering of the binary cell for whole-graph groups (vpps_df) ------------------
+    // Per group: batches of <= 16 nodes of one opcode, forward levels 1..L then backward levels L..0
+    // (level 0 leaves run as a GEMM before the kernel).  Cross-CTA values live in epoch-tagged 64-bit
+    // slots so consumers wait on the data itself: HX (h of an internal node with a consumer, 256
+    // slots), PART (transposed-product partials of an internal node, [consumer CTA][producer CTA][32]:
+    // 16 units of dh_l then 16 of dh_r), HD (head contribution to a labelled node's dh, 256 slots).
+    s.df_off = -1;
+    s.n_hx = s.n_part = s.n_hd = 0;
+    s.df_words = 0;
+    if (plan.by_graph && plan.cell == CELL_BINARY) {
+        std::vector<int64_t> parent(N, -1), head_of(N, -1);
+        std::vector<int32_t> side(N, 0);
+        for (int64_t i = 0; i < N; ++i) {
+            const int32_t* ch = kids.data() + nodes[i].ch_begin;
+            if (nodes[i].kind == K_INT) {
+                parent[ch[0]] = i; side[ch[0]] = 0;
+                parent[ch[1]] = i; side[ch[1]] = 1;
+            } else if (nodes[i].kind == K_HEAD) {
+                head_of[ch[0]] = i;
+            }
+        }
+        std::vector<uint32_t> hx(N, NONE), pp(N, NONE), hd(N, NONE);
+        for (int64_t i = 0; i < N; ++i) {
+            if (nodes[i].kind == K_INT && (parent[i] >= 0 || head_of[i] >= 0)) hx[i] = (uint32_t)s.n_hx++;
+            if (nodes[i].kind == K_INT) pp[i] = (uint32_t)s.n_part++;
+            if (head_of[i] >= 0) hd[i] = (uint32_t)s.n_hd++;
+        }
+        auto dsrc = [&](int64_t i) -> uint32_t {
+            return parent[i] >= 0 ? (pp[parent[i]] << 1) | (uint32_t)side[i] : NONE;
+        };
+        std::vector<std::vector<uint32_t>> prog(G);
+        auto emit_batches = [&](int32_t g, uint32_t op, const std::vector<int64_t>& list) {
+            for (size_t b0 = 0; b0 < list.size(); b0 += 16) {
+                const size_t nb = std::min<size_t>(16, list.size() - b0);
+                std::vector<uint32_t>& w = prog[g];
+                w.push_back(op | (uint32_t)(nb << 8));
+                for (size_t k = b0; k < b0 + nb; ++k) {
+                    const int64_t i = list[k];
+                    const int32_t* ch = kids.data() + nodes[i].ch_begin;
+                    switch (op) {
+                        case OP_INT_F:
+                            w.insert(w.end(), {rec[i], hx[i], rec[ch[0]], hx[ch[0]], rec[ch[1]], hx[ch[1]]});
+                            break;
+                        case OP_HEAD_F:
+                            w.insert(w.end(), {rec[i], rec[ch[0]], (uint32_t)nodes[i].label, hx[ch[0]]});
+                            break;
+                        case OP_HEAD_B:
+                            w.insert(w.end(), {rec[i], rec[ch[0]], (uint32_t)nodes[i].label, hd[ch[0]], hx[ch[0]]});
+                            break;
+                        case OP_INT_B:
+                            w.insert(w.end(), {rec[i], adj[i], dsrc(i), hd[i], pp[i], rec[ch[0]], adj[ch[0]],
+                                               rec[ch[1]], adj[ch[1]]});
+                            break;
+                        default:   // OP_LEAF_B
+                            w.insert(w.end(), {rec[i], adj[i], dsrc(i), hd[i]});
+                    }
+                }
+            }
+        };
+        std::vector<std::vector<int64_t>> lists(5);
+        for (int32_t g = 0; g < G; ++g) {
+            for (int32_t lv = 1; lv <= L; ++lv) {
+                for (auto& l : lists) l.clear();
+                for (int64_t i : at_level[lv]) {
+                    if (graph_group[nodes[i].graph] != g) continue;
+                    if (nodes[i].kind == K_INT) lists[0].push_back(i);
+                    else if (nodes[i].kind == K_HEAD) lists[1].push_back(i);
+                }
+                emit_batches(g, OP_INT_F, lists[0]);
+                emit_batches(g, OP_HEAD_F, lists[1]);
+            }
+            for (int32_t lv = L; lv >= 0; --lv) {
+                for (auto& l : lists) l.clear();
+                for (int64_t i : at_level[lv]) {
+                    if (graph_group[nodes[i].graph] != g) continue;
+                    if (nodes[i].kind == K_HEAD) lists[2].push_back(i);
+                    else if (nodes[i].kind == K_INT) lists[3].push_back(i);
+                    else if (nodes[i].kind == K_LEAF) lists[4].push_back(i);
+                }
+                emit_batches(g, OP_HEAD_B, lists[2]);
+                emit_batches(g, OP_INT_B, lists[3]);
+                emit_batches(g, OP_LEAF_B, lists[4]);
+            }
+        }
+        s.df_off = (int64_t)s.blob.size();
+        s.blob.push_back((uint32_t)G);
+        uint32_t run2 = 0;
+        s.blob.push_back(0);
+        for (int32_t g = 0; g < G; ++g) { run2 += (uint32_t)prog[g].size(); s.blob.push_back(run2); }
+        for (int32_t g = 0; g < G; ++g) s.blob.insert(s.blob.end(), prog[g].begin(), prog[g].end());
+        // tagged regions behind the SPEC pool (64-bit slots = 2 words each)
+        int64_t cur = align32(s.pool_words);
+        // HX: H slots per node; PART: 16 consumer x 16 producer CTAs x 2 (H / 16) slots per parent; HD: H
+        s.df_hx = cur;   cur = align32(cur + 2 * H * s.n_hx);
+        s.df_part = cur; cur = align32(cur + 2 * 32 * H * s.n_part);
+        s.df_hd = cur;   cur = align32(cur + 2 * H * s.n_hd);
+        s.df_words = cur - s.pool_words;
+    }
     return 0;
 }
 

@@ -62,30 +62,6 @@ __device__ __forceinline__ uint32_t cluster_index() {
     return r;
 }
 
-template <int K, int TU>
-struct Lay {
-    static constexpr int CG = (K >= 4 * TU) ? 4 : ((K >= 2 * TU) ? 2 : 1);
-    static constexpr int NT = (K + CG * TU - 1) / (CG * TU);
-    static constexpr int NREG = NT * CG;
-    static constexpr int KP = NT * CG * TU;
-};
-
-// Sum over a 16-lane group of four per-lane values (one per node): transposed halving at distances 8
-// and 4, then a butterfly over the low two bits.  Lane l ends with node 2*bit3(l) + bit2(l).
-__device__ __forceinline__ float treduce4_16(float v0, float v1, float v2, float v3, int lane) {
-    const bool b3 = lane & 8, b2 = lane & 4;
-    const float s0 = b3 ? v0 : v2, s1 = b3 ? v1 : v3;
-    float k0 = b3 ? v2 : v0, k1 = b3 ? v3 : v1;
-    k0 += __shfl_xor_sync(FULLMASK, s0, 8);
-    k1 += __shfl_xor_sync(FULLMASK, s1, 8);
-    const float s = b2 ? k0 : k1;
-    float k = b2 ? k1 : k0;
-    k += __shfl_xor_sync(FULLMASK, s, 4);
-    k += __shfl_xor_sync(FULLMASK, k, 2);
-    k += __shfl_xor_sync(FULLMASK, k, 1);
-    return k;
-}
-
 template <int H, int E>
 struct CCfg {
     static constexpr int NCL = 16;                 // CTAs per cluster (= per replica)

@@ -1,0 +1,541 @@
+// VPPS with dataflow synchronisation (sm_100a) — binary Tree-LSTM.
+//
+// Same work split as the cluster kernel (vpps_cluster.cu): a replica group of 16 CTAs holds every
+// recurrent weight matrix once in registers, each CTA owns 16 consecutive hidden
+// units, whole graphs are assigned to groups (SPEC S5g) and the leaf level runs as a GEMM before the
+// kernel.  What changes is the signal/wait of L165: instead of a barrier per level (whose release has to
+// wait for the CTA's outstanding stores, ~1.8K cycles, before the consumer can even start its L2 round
+// trip), every value another CTA reads is stored as a single-copy-atomic 64-bit slot {value, epoch} and
+// the consumer polls the data itself:
+//   HX[node][H]          h of an internal node that has a consumer (parent or loss head)
+//   PART[node][m][k][2U] partial transposed products of a parent: CTA k's contribution to the dh of both
+//                        children over the U units CTA m owns (m reads its 16 x 2U slots and sums them
+//                        in a fixed order — deterministic, no atomics)
+//   HD[node][H]          the loss head's contribution to a labelled node's dh
+// The epoch is the pass counter, so slots never need clearing.  Without hardware clusters the groups
+// are ordinary co-resident CTAs of a cooperative launch: 9 groups on 144 SMs instead of 7 clusters.
+#include "vpps_kernel.cuh"
+#include "dev_common.cuh"
+
+namespace vpps {
+namespace dev {
+namespace df {
+
+constexpr int NTH = 256;
+constexpr int NCL = 16;        // CTAs per group
+constexpr int CHUNK = 4096;    // program words staged in shared memory
+constexpr int NB = 16;         // nodes per batch
+constexpr int NC = 2;          // nodes per transposed-product chunk
+constexpr int ZC = 32;         // classes per head (C <= 32)
+constexpr int CINMAX = 10;
+constexpr uint32_t NONE = 0xFFFFFFFFu;
+enum : uint32_t { LEAF_B = 0x21, INT_F = 0x22, INT_B = 0x23, HEAD_F = 0x40, HEAD_B = 0x41 };
+
+__device__ __forceinline__ int entry_words(uint32_t op) {
+    switch (op) {
+        case INT_F: return 6;    // rec, hx, rec_l, hx_l, rec_r, hx_r
+        case INT_B: return 9;    // rec, adj, dsrc, hd, pp, rec_l, adj_l, rec_r, adj_r
+        case HEAD_B: return 5;   // rec, rec_c, label, hd_c, hx_c
+        default: return 4;       // HEAD_F: rec, rec_c, label, hx_c | LEAF_B: rec, adj, dsrc, hd
+    }
+}
+
+typedef unsigned long long u64;
+__device__ __forceinline__ u64 tagv(float v, uint32_t e) { return ((u64)e << 32) | __float_as_uint(v); }
+__device__ __forceinline__ void st_tag(u64* p, float v, uint32_t e) {
+    asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(tagv(v, e)) : "memory");
+}
+__device__ __forceinline__ void st_tag4(u64* p, const float* v, uint32_t e) {
+    asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(tagv(v[0], e)), "l"(tagv(v[1], e)) : "memory");
+    asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p + 2), "l"(tagv(v[2], e)), "l"(tagv(v[3], e)) : "memory");
+}
+// value of a slot once it carries epoch e (spins; the producer is a co-resident CTA of the group)
+__device__ __forceinline__ float wait_tag(const u64* p, u64 seen, uint32_t e) {
+    while ((uint32_t)(seen >> 32) != e) {
+        __nanosleep(32);
+        asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(seen) : "l"(p) : "memory");
+    }
+    return __uint_as_float((uint32_t)seen);
+}
+__device__ __forceinline__ void cp_async8(void* dst, const void* src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+
+template <int H, int E>
+struct DCfg {
+    static constexpr int UM = H / NCL;             // hidden units per CTA
+    static constexpr int TU = NTH / UM;            // threads per unit
+    static_assert(H % NCL == 0 && TU == 16, "dataflow kernel: 16 units per CTA, 16 threads per unit");
+    using LB = Lay<2 * H, TU>;                     // internal bundle rows (i, o, u of U_iou; f) over [h_l; h_r]
+    static constexpr int KP = LB::KP;              // 2H
+    static constexpr int O_X = CHUNK;                               // xs [NB][KP] floats
+    static constexpr int O_DXB = O_X + NB * KP;                     // dxb [UM][NC][KP] floats / u64 scratch
+    static constexpr int O_CIN = O_DXB + UM * NC * KP;
+    static constexpr int O_BIAS = O_CIN + NB * UM * CINMAX;
+    static constexpr int O_ZS = O_BIAS + UM * 4;
+    static constexpr int O_HEAD = O_ZS + NB * ZC;
+    static_assert(UM * NC * KP >= 2 * NB * KP && UM * NC * KP >= 2 * NB * NCL * 2 * UM, "u64 staging fits in dxb");
+    static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 2 * C + 8); }
+};
+
+template <int H, int E>
+__global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
+    using T = DCfg<H, E>;
+    using LB = typename T::LB;
+    constexpr int TU = T::TU, UM = T::UM, KP = T::KP;
+    extern __shared__ __align__(16) uint32_t smw[];
+    float* sm = reinterpret_cast<float*>(smw);
+    uint32_t* chunk = smw;
+    float* xs = sm + T::O_X;
+    float* dxb = sm + T::O_DXB;
+    u64* tbuf = reinterpret_cast<u64*>(sm + T::O_DXB);     // tagged staging (aliases dxb)
+    float* cin = sm + T::O_CIN;
+    float* bias = sm + T::O_BIAS;
+    float* zs = sm + T::O_ZS;
+    const int C = P.C;
+    float* Wo = sm + T::O_HEAD;
+    float* dWo = Wo + C * H;
+    float* bo = dWo + C * H;
+    float* dbo = bo + C;
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int grp = blockIdx.x / NCL, lc = blockIdx.x % NCL;
+    float* pool = P.pool;
+    const int64_t* off = P.off;
+    const uint32_t ep = P.epoch;
+    u64* HX = reinterpret_cast<u64*>(pool + P.df_hx);
+    u64* PART = reinterpret_cast<u64*>(pool + P.df_part);
+    u64* HD = reinterpret_cast<u64*>(pool + P.df_hd);
+    const int u = tid / TU, tu = tid % TU, gl = lane & 15;      // unit slot, thread in unit, lane in group
+    const int j = lc * UM + u;                                  // hidden unit of this thread (blocked)
+    const bool holds_head = (lc == 0);
+
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    // ---- prologue: this CTA's rows of U_iou, U_fl, U_fr -> registers (L123, L129) ----
+    float wb[4][LB::NREG];
+#pragma unroll
+    for (int r = 0; r < 4; ++r)
+#pragma unroll
+        for (int t = 0; t < LB::NT; ++t) {
+            const int col = LB::CG * (tu + TU * t);
+            const float* src = r < 3 ? P.params + off[1] + (int64_t)(r * H + j) * (2 * H) + col
+                                     : (col < H ? P.params + off[2] + (int64_t)j * H + col
+                                                : P.params + off[3] + (int64_t)j * H + col - H);
+            if constexpr (LB::CG == 4) {
+                const float4 v = __ldg(reinterpret_cast<const float4*>(src));
+                wb[r][t * 4] = v.x; wb[r][t * 4 + 1] = v.y; wb[r][t * 4 + 2] = v.z; wb[r][t * 4 + 3] = v.w;
+            } else {
+#pragma unroll
+                for (int q = 0; q < LB::CG; ++q) wb[r][t * LB::CG + q] = __ldg(src + q);
+            }
+        }
+    if (tid < UM * 4) {
+        const int uu = tid / 4, k = tid % 4, jj = lc * UM + uu;
+        bias[tid] = k < 3 ? __ldg(P.params + off[5] + k * H + jj) : __ldg(P.params + off[6] + jj);
+    }
+    if (holds_head) {
+        for (int i = tid; i < C * H; i += NTH) { Wo[i] = __ldg(P.params + off[4] + i); dWo[i] = 0.f; }
+        for (int i = tid; i < C; i += NTH) { bo[i] = __ldg(P.params + off[7] + i); dbo[i] = 0.f; }
+    }
+    float dbacc[4] = {0.f, 0.f, 0.f, 0.f};
+    uint64_t* prof = P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
+    // section clocks (trace only): 0 program, 1 staging, 2 tag wait, 3 forward, 4 cell-bwd, 5 transposed,
+    // 6 heads, 7 other
+    uint64_t sec[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    uint64_t sec_last = 0;
+    int sec_cur = 7;
+    auto mark = [&](int k) {
+        if (prof && tid == 0) {
+            const uint64_t now = clock64(), d = now - sec_last;
+            switch (sec_cur) {
+                case 0: sec[0] += d; break;
+                case 1: sec[1] += d; break;
+                case 2: sec[2] += d; break;
+                case 3: sec[3] += d; break;
+                case 4: sec[4] += d; break;
+                case 5: sec[5] += d; break;
+                case 6: sec[6] += d; break;
+                default: sec[7] += d; break;
+            }
+            sec_cur = k;
+            sec_last = now;
+        }
+    };
+    // the leaf records (vpps_leaf_fwd, the preceding grid) are complete and visible from here on
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    __syncthreads();
+    if (prof && tid == 0) { prof[0] = gtimer(); sec_last = clock64(); }
+
+    // ---- program of this group: batches [op | nb << 8, nb entries] ----
+    const uint32_t* S_ = P.script + P.df_off;
+    const uint32_t G = S_[0];
+    const uint32_t s0 = 2 + G + S_[1 + grp], s1 = 2 + G + S_[2 + grp];
+    uint32_t cbase = s0;
+    auto refill = [&](uint32_t from) {
+        __syncthreads();
+        for (int i = tid; i < CHUNK; i += NTH) chunk[i] = from + i < s1 ? __ldg(S_ + from + i) : 0u;
+        __syncthreads();
+        cbase = from;
+    };
+    if (s0 < s1) refill(s0);
+    uint32_t pos = s0;
+    int nbatch = 0;
+    while (pos < s1) {
+        if (pos + 1 + NB * 9 > cbase + CHUNK && cbase + CHUNK < s1) refill(pos);
+        mark(0);
+        const uint32_t hdr = chunk[pos - cbase];
+        const uint32_t op = hdr & 0xFF;
+        const int nb = (int)(hdr >> 8);
+        const int sz = entry_words(op);
+        const uint32_t* ent = chunk + (pos - cbase) + 1;
+        const uint32_t next = pos + 1 + nb * sz;
+        const bool is_head = (op == HEAD_F || op == HEAD_B);
+        if (is_head && !holds_head) { pos = next; continue; }
+        ++nbatch;
+        mark(1);
+        if (op == INT_F || is_head) {
+            // rows: [h_l; h_r] (INT_F) or h of the labelled node (heads): tagged HX slots of internal
+            // children -> u64 scratch, leaf records (written by the leaf GEMM) -> xs directly
+            const int A = op == INT_F ? 2 : 1;
+            const int q16 = H / 4;                          // 16-byte pieces per half row of floats
+            for (int i = tid; i < nb * A * q16; i += NTH) {
+                const int n = i / (A * q16), rem = i - n * (A * q16), half = rem / q16, c = (rem - half * q16) * 4;
+                const uint32_t* e = ent + n * sz;
+                const uint32_t rec = op == INT_F ? e[2 + 2 * half] : e[1];
+                const uint32_t hx = op == INT_F ? e[3 + 2 * half] : (op == HEAD_F ? e[3] : e[4]);
+                if (hx == NONE) {
+                    cp_async16(xs + n * KP + half * H + c, pool + rec + c, 16u);
+                } else {
+                    const u64* src = HX + (int64_t)hx * H + c;
+                    u64* dst = tbuf + n * KP + half * H + c;
+                    cp_async16(dst, src, 16u);
+                    cp_async16(dst + 2, src + 2, 16u);
+                }
+            }
+            if (op == INT_F) {                              // c_l, c_r of this CTA's units (own records)
+                for (int i = tid; i < nb * UM * 2; i += NTH) {
+                    const int n = i / (UM * 2), rem = i - n * (UM * 2), uu = rem >> 1, k = rem & 1;
+                    const uint32_t* e = ent + n * sz;
+                    cp_async4(cin + (n * UM + uu) * CINMAX + k, pool + e[2 + 2 * k] + H + lc * UM + uu, 4u);
+                }
+            }
+            cp_async_wait_all();
+            __syncthreads();
+            mark(2);
+            // tagged columns: check the epoch, wait for late producers, convert to floats
+            for (int i = tid; i < nb * A * (H / 2); i += NTH) {
+                const int n = i / (A * (H / 2)), rem = i - n * (A * (H / 2)), half = rem / (H / 2);
+                const int c = (rem - half * (H / 2)) * 2;
+                const uint32_t* e = ent + n * sz;
+                const uint32_t hx = op == INT_F ? e[3 + 2 * half] : (op == HEAD_F ? e[3] : e[4]);
+                if (hx == NONE) continue;
+                const u64* t = tbuf + n * KP + half * H + c;
+                const u64* g = HX + (int64_t)hx * H + c;
+                xs[n * KP + half * H + c] = wait_tag(g, t[0], ep);
+                xs[n * KP + half * H + c + 1] = wait_tag(g + 1, t[1], ep);
+            }
+            __syncthreads();
+        } else {
+            // backward: dh = Σ_k PART[parent][lc][k][side*U + u] (+ HD) -> u64 scratch [n][k][U], [n][16][U]
+            for (int i = tid; i < nb * (NCL + 1) * (UM / 2); i += NTH) {
+                const int n = i / ((NCL + 1) * (UM / 2)), rem = i - n * ((NCL + 1) * (UM / 2));
+                const int k = rem / (UM / 2), c = (rem - k * (UM / 2)) * 2;
+                const uint32_t* e = ent + n * sz;
+                const uint32_t dsrc = e[2], hd = e[3];
+                const u64* src = nullptr;
+                if (k < NCL) {
+                    if (dsrc != NONE)
+                        src = PART + ((((int64_t)(dsrc >> 1) * NCL + lc) * NCL + k) * 2 + (dsrc & 1)) * UM + c;
+                } else if (hd != NONE) {
+                    src = HD + (int64_t)hd * H + lc * UM + c;
+                }
+                if (src) cp_async16(tbuf + (n * (NCL + 1) + k) * UM + c, src, 16u);
+            }
+            // own operands: dc (adj + H), c i o u (fl fr) (rec + H..), c_l c_r (children's records)
+            const int ncin = op == INT_B ? 10 : 6;
+            for (int i = tid; i < nb * UM * (ncin - 1); i += NTH) {
+                const int n = i / (UM * (ncin - 1)), rem = i - n * (UM * (ncin - 1));
+                const int uu = rem / (ncin - 1), k = 1 + rem - uu * (ncin - 1);
+                const uint32_t* e = ent + n * sz;
+                const int jj = lc * UM + uu;
+                const float* src;
+                if (k == 1) src = pool + e[1] + H + jj;
+                else if (k < 8) src = pool + e[0] + (k - 1) * H + jj;
+                else src = pool + (k == 8 ? e[5] : e[7]) + H + jj;
+                cp_async4(cin + (n * UM + uu) * CINMAX + k, src, 4u);
+            }
+            cp_async_wait_all();
+            __syncthreads();
+            mark(2);
+            {   // thread (n = tid / U, u = tid % U): the 16 partials (+ head) in fixed order
+                const int n = tid / UM, uu = tid % UM;
+                if (n < nb) {
+                    const uint32_t* e = ent + n * sz;
+                    const uint32_t dsrc = e[2], hd = e[3];
+                    float dh = 0.f;
+                    if (dsrc != NONE) {
+                        const u64* g = PART + (((int64_t)(dsrc >> 1) * NCL + lc) * NCL * 2 + (dsrc & 1)) * UM + uu;
+#pragma unroll 4
+                        for (int k = 0; k < NCL; ++k)
+                            dh += wait_tag(g + (int64_t)k * 2 * UM, tbuf[(n * (NCL + 1) + k) * UM + uu], ep);
+                    }
+                    if (hd != NONE) {
+                        const u64* g = HD + (int64_t)hd * H + lc * UM + uu;
+                        dh += wait_tag(g, tbuf[(n * (NCL + 1) + NCL) * UM + uu], ep);
+                    }
+                    cin[(n * UM + uu) * CINMAX] = dh;
+                }
+            }
+            __syncthreads();
+        }
+
+        mark(is_head ? 6 : (op == INT_F ? 3 : 4));
+        if (is_head) {            // loss heads (L42) on the CTA holding W_out
+            constexpr int KPH = KP;
+            if (op == HEAD_F) {
+                for (int pi = warp; pi < nb * C; pi += NTH / 32) {
+                    const int n = pi / C, c = pi - n * C;
+                    float s = 0.f;
+                    for (int k = 4 * lane; k < H; k += 128) {
+                        const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                        const float4 h4 = *reinterpret_cast<const float4*>(xs + n * KPH + k);
+                        s += w4.x * h4.x + w4.y * h4.y + w4.z * h4.z + w4.w * h4.w;
+                    }
+                    s = warp_sum(s);
+                    if (lane == 0) zs[n * ZC + c] = s + bo[c];
+                }
+                __syncthreads();
+                for (int n = warp; n < nb; n += NTH / 32) {
+                    const uint32_t* e = ent + n * sz;
+                    const float zl = lane < C ? zs[n * ZC + lane] : -INFINITY;
+                    const float m = warp_max(zl);
+                    const float lse = m + logf(warp_sum(lane < C ? expf(zl - m) : 0.f));
+                    if (lane < C) pool[e[0] + lane] = expf(zl - lse);
+                    const float zy = __shfl_sync(FULLMASK, zl, (int)e[2]);
+                    if (lane == 0) {
+                        pool[e[0] + C] = lse - zy;
+                        atomicAdd(pool + P.loss_word, lse - zy);   // aggregated loss node (L205)
+                    }
+                }
+            } else {
+                for (int i = tid; i < nb * C; i += NTH) {
+                    const int n = i / C, c = i - n * C;
+                    const uint32_t* e = ent + n * sz;
+                    zs[n * ZC + c] = pool[e[0] + c] - (c == (int)e[2] ? 1.f : 0.f);
+                }
+                __syncthreads();
+                for (int c = tid; c < C; c += NTH) {
+                    float s = 0.f;
+                    for (int n = 0; n < nb; ++n) s += zs[n * ZC + c];
+                    dbo[c] += s;
+                }
+                for (int i = tid; i < C * H; i += NTH) {
+                    const int c = i / H, k = i - c * H;
+                    float s = 0.f;
+                    for (int n = 0; n < nb; ++n) s = fmaf(zs[n * ZC + c], xs[n * KPH + k], s);
+                    dWo[i] += s;
+                }
+                for (int i = tid; i < nb * (H / 4); i += NTH) {   // dh of the labelled node -> HD slots
+                    const int n = i / (H / 4), k = (i - n * (H / 4)) * 4;
+                    float v4[4] = {0.f, 0.f, 0.f, 0.f};
+                    for (int c = 0; c < C; ++c) {
+                        const float dzc = zs[n * ZC + c];
+                        const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                        v4[0] = fmaf(w4.x, dzc, v4[0]); v4[1] = fmaf(w4.y, dzc, v4[1]);
+                        v4[2] = fmaf(w4.z, dzc, v4[2]); v4[3] = fmaf(w4.w, dzc, v4[3]);
+                    }
+                    const uint32_t hd = ent[n * sz + 3];
+                    if (hd != NONE) st_tag4(HD + (int64_t)hd * H + k, v4, ep);
+                }
+            }
+        } else if (op == INT_F) {
+            // ---- forward of internal cells: matvec from registers (L123), 4 nodes at a time; the unit's
+            //      16 lanes reduce with a transposed butterfly; the lane holding node n's gates updates it ----
+            for (int n0 = 0; n0 < nb; n0 += 4) {
+                float2 a[4][5];
+#pragma unroll
+                for (int n = 0; n < 4; ++n)
+#pragma unroll
+                    for (int o = 0; o < 5; ++o) a[n][o] = make_float2(0.f, 0.f);
+#pragma unroll
+                for (int t = 0; t < LB::NT; ++t) {
+                    const int col0 = LB::CG * (tu + TU * t);
+                    const int of = col0 < H ? 3 : 4;
+#pragma unroll
+                    for (int n = 0; n < 4; ++n) {
+                        float xv[LB::CG];
+                        lds<LB::CG>(xs + (n0 + n) * KP + col0, xv);
+#pragma unroll
+                        for (int q = 0; q < LB::CG; q += 2) {
+                            const float2 x2 = make_float2(xv[q], xv[q + 1]);
+                            const int k = t * LB::CG + q;
+#pragma unroll
+                            for (int r = 0; r < 3; ++r)
+                                a[n][r] = __ffma2_rn(make_float2(wb[r][k], wb[r][k + 1]), x2, a[n][r]);
+                            const float2 f2 = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), x2, make_float2(0.f, 0.f));
+                            if (of == 3) { a[n][3].x += f2.x; a[n][3].y += f2.y; }
+                            else { a[n][4].x += f2.x; a[n][4].y += f2.y; }
+                        }
+                    }
+                }
+                float g5[5];
+#pragma unroll
+                for (int o = 0; o < 5; ++o)
+                    g5[o] = treduce4_16(a[0][o].x + a[0][o].y, a[1][o].x + a[1][o].y, a[2][o].x + a[2][o].y,
+                                        a[3][o].x + a[3][o].y, gl);
+                const int n = n0 + (gl >> 2);
+                if ((gl & 3) == 0 && n < nb) {
+                    const uint32_t* e = ent + n * sz;
+                    const uint32_t rec = e[0];
+                    const float* b = bias + u * 4;
+                    const float* cv = cin + (n * UM + u) * CINMAX;
+                    const float i = sigm(g5[0] + b[0]), o = sigm(g5[1] + b[1]), uv = tanhf(g5[2] + b[2]);
+                    const float fl = sigm(g5[3] + b[3]), fr = sigm(g5[4] + b[3]);
+                    const float c = i * uv + fl * cv[0] + fr * cv[1];
+                    const float h = o * tanhf(c);
+                    if (e[1] != NONE) st_tag(HX + (int64_t)e[1] * H + j, h, ep);   // read by the whole group
+                    pool[rec + j] = h;                                              // the rest: this CTA, GEMMs
+                    pool[rec + H + j] = c;
+                    pool[rec + 2 * H + j] = i;
+                    pool[rec + 3 * H + j] = o;
+                    pool[rec + 4 * H + j] = uv;
+                    pool[rec + 5 * H + j] = fl;
+                    pool[rec + 6 * H + j] = fr;
+                }
+            }
+        } else {
+            // ---- backward: cell backward by thread (unit u, node gl); gate gradients recorded for the dW
+            //      GEMM (L185) and broadcast to the unit's lanes ----
+            const bool kindB = op == INT_B;
+            float g[5] = {0.f, 0.f, 0.f, 0.f, 0.f};
+            if (gl < nb) {
+                const uint32_t* e = ent + gl * sz;
+                const uint32_t rec = e[0];
+                const float* cv = cin + (gl * UM + u) * CINMAX;
+                const float dh = cv[0], dc = cv[1], c = cv[2], i = cv[3], o = cv[4], uv = cv[5];
+                const float th = tanhf(c);
+                const float chat = dc + dh * o * (1.f - th * th);
+                g[0] = chat * uv * i * (1.f - i);
+                g[1] = dh * th * o * (1.f - o);
+                g[2] = chat * i * (1.f - uv * uv);
+                if (kindB) {
+                    const float fl = cv[6], fr = cv[7], cl = cv[8], cr = cv[9];
+                    g[3] = chat * cl * fl * (1.f - fl);
+                    g[4] = chat * cr * fr * (1.f - fr);
+                    pool[e[6] + H + j] = chat * fl;          // dc of the children (unique parent; own units)
+                    pool[e[8] + H + j] = chat * fr;
+                    pool[rec + 7 * H + j] = g[0];
+                    pool[rec + 8 * H + j] = g[1];
+                    pool[rec + 9 * H + j] = g[2];
+                    pool[rec + 10 * H + j] = g[3];
+                    pool[rec + 11 * H + j] = g[4];
+                } else {
+                    pool[rec + 5 * H + j] = g[0];
+                    pool[rec + 6 * H + j] = g[1];
+                    pool[rec + 7 * H + j] = g[2];
+                }
+                dbacc[0] += g[0]; dbacc[1] += g[1]; dbacc[2] += g[2]; dbacc[3] += g[3] + g[4];
+            }
+            mark(5);
+            // transposed products (L94, fn4): per node, this CTA's partial dx = Σ_r W[r] g_r over all 2H
+            // columns; the 16 unit slices are summed in shared memory and published as tagged PART slots
+            if (kindB) {
+                const int src = lane & 16;
+                for (int n0 = 0; n0 < nb; n0 += NC) {
+#pragma unroll
+                    for (int dn = 0; dn < NC; ++dn) {
+                        const int n = n0 + dn;
+                        float gr[5];
+#pragma unroll
+                        for (int r = 0; r < 5; ++r) gr[r] = __shfl_sync(FULLMASK, g[r], src | (n & 15));
+                        float* drow = dxb + (u * NC + dn) * KP;
+#pragma unroll
+                        for (int t = 0; t < LB::NT; ++t) {
+                            const int col0 = LB::CG * (tu + TU * t);
+                            const float gf = col0 < H ? gr[3] : gr[4];
+                            float dx[LB::CG];
+#pragma unroll
+                            for (int q = 0; q < LB::CG; q += 2) {
+                                const int k = t * LB::CG + q;
+                                float2 d = __ffma2_rn(make_float2(wb[0][k], wb[0][k + 1]), make_float2(gr[0], gr[0]),
+                                                      make_float2(0.f, 0.f));
+                                d = __ffma2_rn(make_float2(wb[1][k], wb[1][k + 1]), make_float2(gr[1], gr[1]), d);
+                                d = __ffma2_rn(make_float2(wb[2][k], wb[2][k + 1]), make_float2(gr[2], gr[2]), d);
+                                d = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), make_float2(gf, gf), d);
+                                dx[q] = d.x;
+                                dx[q + 1] = d.y;
+                            }
+                            sts_granule<LB::CG>(drow + col0, dx, n < nb);
+                        }
+                    }
+                    __syncthreads();
+                    constexpr int q4 = KP / 4;
+                    for (int i = tid; i < NC * q4; i += NTH) {
+                        const int dn = i / q4, c = (i - dn * q4) * 4, n = n0 + dn;
+                        if (n >= nb) continue;
+                        float s[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+                        for (int uu = 0; uu < UM; ++uu) {
+                            const float4 x = *reinterpret_cast<const float4*>(dxb + (uu * NC + dn) * KP + c);
+                            s[0] += x.x; s[1] += x.y; s[2] += x.z; s[3] += x.w;
+                        }
+                        // column c: child side = c / H, unit jj = c % H, owner CTA m = jj / U, slot jj % U
+                        const int side = c >= H, jj = c - side * H, m = jj / UM;
+                        const uint32_t pp = ent[n * sz + 4];
+                        st_tag4(PART + ((((int64_t)pp * NCL + m) * NCL + lc) * 2 + side) * UM + (jj - m * UM), s, ep);
+                    }
+                    __syncthreads();
+                }
+            }
+        }
+        __syncthreads();
+        pos = next;
+    }
+    mark(7);
+    if (prof && tid == 0) {
+        prof[1] = gtimer();
+        prof[2] = (uint64_t)nbatch;
+#pragma unroll
+        for (int k = 0; k < 8; ++k) prof[3 + k] = sec[k];
+    }
+
+    // ---- epilogue: bias and head gradients of this group summed into grads (zeroed by the host); the
+    //      weight-matrix gradients come from vpps_dw_gemm (L185) ----
+#pragma unroll
+    for (int k = 0; k < 4; ++k)
+#pragma unroll
+        for (int s = 8; s >= 1; s >>= 1) dbacc[k] += __shfl_xor_sync(FULLMASK, dbacc[k], s);
+    if (gl == 0) {
+#pragma unroll
+        for (int k = 0; k < 3; ++k) atomicAdd(P.grads + off[5] + k * H + j, dbacc[k]);
+        atomicAdd(P.grads + off[6] + j, dbacc[3]);
+    }
+    if (holds_head) {
+        __syncthreads();
+        for (int i = tid; i < C * H; i += NTH) atomicAdd(P.grads + off[4] + i, dWo[i]);
+        for (int i = tid; i < C; i += NTH) atomicAdd(P.grads + off[7] + i, dbo[i]);
+    }
+    // this CTA's records and gradient contributions are complete: count it for the GEMM tiles of its group
+    if (P.done) {
+        __threadfence();
+        __syncthreads();
+        if (tid == 0) atomicAdd(P.done + grp, 1);
+    }
+}
+
+}  // namespace df
+}  // namespace dev
+
+#define VPPS_DF_VARIANT(H, E) \
+    {1, H, E, 16, (const void*)&dev::df::vpps_df<H, E>, &dev::df::DCfg<H, E>::smem_bytes}
+
+static const Variant kDfVariants[] = {
+    VPPS_DF_VARIANT(256, 256),    // target: binary Tree-LSTM H = E = 256, groups of 16 CTAs
+};
+
+const Variant* df_variants(int32_t* n) {
+    *n = (int32_t)(sizeof(kDfVariants) / sizeof(kDfVariants[0]));
+    return kDfVariants;
+}
+
+}  // namespace vpps

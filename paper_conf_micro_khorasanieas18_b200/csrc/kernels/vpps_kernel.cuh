@@ -22,6 +22,23 @@ struct KParams {
     int32_t* done;          // cluster path: per-group completion counters (one increment per CTA), or nullptr
 };
 
+// Dataflow kernel (vpps_dataflow.cu): groups of 16 co-resident CTAs, epoch-tagged cross-CTA slots.
+struct DfParams {
+    float* params;
+    float* grads;
+    float* pool;
+    const uint32_t* script;     // device blob; the group programs start at df_off
+    int64_t df_off;
+    int64_t off[8];
+    int32_t C;
+    uint32_t epoch;             // pass counter (>= 1): tag of every slot written by this pass
+    int64_t loss_word;
+    int64_t df_hx, df_part, df_hd;   // word offsets of the tagged regions in the pool
+    uint64_t* prof;
+    int64_t prof_stride;
+    int32_t* done;              // per-group completion counters, or nullptr
+};
+
 struct Variant {
     int32_t cell, H, E, umax;
     const void* fn;
@@ -32,6 +49,8 @@ struct Variant {
 const Variant* variants(int32_t* n);
 // Cluster-replica specialisations (vpps_cluster.cu); Variant.umax holds the cluster size.
 const Variant* cluster_variants(int32_t* n);
+// Dataflow specialisations (vpps_dataflow.cu); Variant.umax holds the group size.
+const Variant* df_variants(int32_t* n);
 // dW = Σ g xᵀ per weight matrix from the recorded operands, fused SGD when mode == 1.
 // Also forms the leaf input gradient dX[tok] += W_iouᵀ g_leaf when d_inputs is not null.  Node lists are
 // grouped by replica group (offsets int_off / leaf_off, n_grp + 1 entries); with `early` the kernel is a

@@ -20,13 +20,13 @@ def _vpps():
     return vpps
 
 
-def run_case(cell, H, E, C, graphs, V, seed=0, want_dx=True, sgd=None, groups=1, cluster=0):
+def run_case(cell, H, E, C, graphs, V, seed=0, want_dx=True, sgd=None, groups=1, cluster=0, dataflow=False):
     vpps = _vpps()
     rng = np.random.default_rng(seed)
     shapes = vpps.param_shapes(cell, H, E, C)
     P = synth.init_params(shapes, rng)
     X = synth.input_table(rng, V, E)
-    m = vpps.Model(cell, H, E, C, device=0, groups=groups, cluster=cluster)
+    m = vpps.Model(cell, H, E, C, device=0, groups=groups, cluster=cluster, dataflow=dataflow)
     dev = torch.device("cuda:0")
     params = torch.zeros(m.n_floats, dtype=torch.float32, device=dev)
     grads = torch.full_like(params, float("nan"))
@@ -50,9 +50,9 @@ def rel(a, b):
     return float(np.abs(np.asarray(a, np.float64) - b).max() / max(np.abs(b).max(), 1e-30))
 
 
-def check(cell, H, E, C, graphs, V, seed=0, want_dx=True, groups=1, cluster=0):
+def check(cell, H, E, C, graphs, V, seed=0, want_dx=True, groups=1, cluster=0, dataflow=False):
     m, P, X, loss, params, grads, dX = run_case(cell, H, E, C, graphs, V, seed, want_dx, groups=groups,
-                                                cluster=cluster)
+                                                cluster=cluster, dataflow=dataflow)
     lo, Go, dXo = M.forward_backward(cell, P, X, graphs, H)
     assert abs(loss - lo) <= TOL * abs(lo), (loss, lo)
     gv = m.views(grads.cpu())
@@ -90,17 +90,57 @@ def test_binary_target_cluster_replicas(b):
     check("binary", 256, 256, 5, synth.config_batch("tgt", b), 4096, seed=11 + b, cluster=16)
 
 
+@pytest.mark.parametrize("b", [0, 5, 9])
+def test_binary_target_dataflow_groups(b):
+    """Dataflow path: 16-CTA groups of a cooperative launch, epoch-tagged slots instead of barriers."""
+    check("binary", 256, 256, 5, synth.config_batch("tgt", b), 4096, seed=21 + b, cluster=16, dataflow=True)
+
+
+def test_dataflow_degenerate_and_repeated_passes():
+    check("binary", 256, 256, 5, [[((), 3, 2)]], 8, cluster=16, dataflow=True)           # one leaf
+    check("binary", 256, 256, 5, _trees(12, 3, (1, 9), 30, 5), 30, cluster=16, dataflow=True, want_dx=False)
+    t = [((), 0, 1), ((), 1, -1), ((0, 1), -1, 3), ((), 2, -1), ((2, 3), -1, 0)]           # inner labels
+    check("binary", 256, 256, 5, [t, t], 4, cluster=16, dataflow=True)
+
+
+def test_dataflow_epochs_across_passes():
+    """Tagged slots are reused by later passes (and by other scripts) without clearing."""
+    vpps = _vpps()
+    rng = np.random.default_rng(31)
+    H, C, V = 256, 5, 64
+    shapes = vpps.param_shapes("binary", H, H, C)
+    P = synth.init_params(shapes, rng)
+    m = vpps.Model("binary", H, H, C, cluster=16, dataflow=True)
+    params = torch.zeros(m.n_floats, device="cuda")
+    grads = torch.zeros_like(params)
+    for name, _ in shapes:
+        m.views(params)[name].copy_(torch.from_numpy(P[name]).float())
+    m.bind(params, grads)
+    X = torch.from_numpy(synth.input_table(rng, V, H)).float().cuda()
+    batches = [_trees(40 + i, 6, (2, 30), V, C) for i in range(3)]
+    scripts = [m.build_script(b) for b in batches]
+    for rep in range(2):
+        for b, s in zip(batches, scripts):
+            m.fwd_bwd(s, X)
+            lo, Go, _ = M.forward_backward("binary", P, X.cpu().double().numpy(), b, H)
+            assert abs(m.latest_loss() - lo) <= TOL * abs(lo)
+            gv = m.views(grads.cpu())
+            for name, _ in m.shapes:
+                assert rel(gv[name].numpy(), Go[name]) <= TOL, (rep, name)
+
+
 def test_cluster_degenerate_batches():
     check("binary", 256, 256, 5, [[((), 3, 2)]], 8, cluster=16)              # one leaf: most clusters idle
     check("binary", 256, 256, 5, _trees(12, 3, (1, 9), 30, 5), 30, cluster=16, want_dx=False)
 
 
-@pytest.mark.parametrize("groups,cluster", [(1, 0), (2, 0), (4, 0), (1, 16)])
-def test_fused_sgd_target_groups(groups, cluster):
+@pytest.mark.parametrize("groups,cluster,dataflow", [(1, 0, False), (2, 0, False), (4, 0, False), (1, 16, False),
+                                                     (1, 16, True)])
+def test_fused_sgd_target_groups(groups, cluster, dataflow):
     graphs = synth.config_batch("tgt", 4)
     lr, wd = 0.05, 1e-3
     m, P, X, loss, params, grads, dX = run_case("binary", 256, 256, 5, graphs, 4096, seed=6, sgd=(lr, wd),
-                                                groups=groups, cluster=cluster)
+                                                groups=groups, cluster=cluster, dataflow=dataflow)
     lo, Go, _ = M.forward_backward("binary", P, X, graphs, 256)
     Pn = M.sgd(P, Go, lr, wd)
     pv = m.views(params.cpu())

@@ -1,0 +1,67 @@
+"""Section clocks of the dataflow kernel (vpps_df) from its in-kernel trace (vpps_set_profile_buffer).
+
+    python tools/df_trace.py [--batch-idx 0] [--reps 3]
+
+Per CTA: span (globaltimer), batches executed and cycles per section (0 program decode, 1 staging issue,
+2 tag wait / data arrival, 3 forward, 4 cell-bwd, 5 transposed product, 6 heads, 7 other).  Prints the
+mean over CTAs, the slowest CTA and the per-group spans.
+"""
+import argparse
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--batch-idx", type=int, default=0)
+    ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--config", default="tgt")
+    args = ap.parse_args()
+    import torch
+    import synth
+    from paper_conf_micro_khorasanieas18_b200 import vpps
+    cfg = synth.CONFIGS[args.config]
+    cell, H, E, C, V = cfg["cell"], cfg["H"], cfg["E"], cfg["C"], cfg["V"]
+    rng = np.random.default_rng(0)
+    shapes = vpps.param_shapes(cell, H, E, C)
+    P = synth.init_params(shapes, rng)
+    m = vpps.Model(cell, H, E, C, cluster=16, dataflow=True)
+    params = torch.zeros(m.n_floats, device="cuda")
+    grads = torch.zeros_like(params)
+    for n, _ in shapes:
+        m.views(params)[n].copy_(torch.from_numpy(P[n]).float())
+    m.bind(params, grads)
+    X = torch.from_numpy(synth.input_table(rng, V, E)).float().cuda()
+    dX = torch.zeros_like(X)
+    s = m.build_script(synth.config_batch(args.config, args.batch_idx))
+    n_cta = m.plan_info()["n_cta"]
+    stride = 16
+    buf = torch.zeros((n_cta, stride), dtype=torch.int64, device="cuda")
+    m.set_profile_buffer(buf, stride)
+    for _ in range(args.reps):
+        m.fwd_bwd(s, X, dX)
+    torch.cuda.synchronize()
+    raw = buf.cpu().numpy().astype(np.float64)
+    t0 = raw[:, 0].min()
+    span = (raw[:, 1] - raw[:, 0]) / 1e3
+    names = ["program", "staging", "tag-wait", "forward", "cell-bwd", "transp", "heads", "other"]
+    secs = raw[:, 3:11]
+    print(f"{args.config} batch {args.batch_idx}: {n_cta} CTAs, span max {span.max():.1f} us "
+          f"(start skew {(raw[:, 0].max() - t0) / 1e3:.1f} us)")
+    groups = n_cta // 16
+    print("group spans (us): " + ", ".join(f"{(raw[g*16:(g+1)*16, 1].max() - t0) / 1e3:.1f}" for g in range(groups)))
+    print("batches per group: " + ", ".join(f"{int(raw[g*16, 2])}" for g in range(groups)))
+    mean = secs.mean(0)
+    slow = secs[np.argmax(raw[:, 1])]
+    tot = mean.sum()
+    print("section kcycles (mean | CTA that finished last):")
+    print("  " + ", ".join(f"{n} {a/1e3:.0f}k ({a/tot*100:.0f}%) | {b/1e3:.0f}k" for n, a, b in zip(names, mean, slow)))
+
+
+if __name__ == "__main__":
+    main()

@@ -22,6 +22,7 @@ def main():
     ap.add_argument("--groups", type=int, default=4)
     ap.add_argument("--config", default="tgt")
     ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--sync", choices=["dataflow", "cluster"], default="dataflow")
     args = ap.parse_args()
     import torch
     import synth
@@ -31,7 +32,7 @@ def main():
     rng = np.random.default_rng(0)
     shapes = vpps.param_shapes(cell, H, E, C)
     P = synth.init_params(shapes, rng)
-    m = vpps.Model(cell, H, E, C, groups=args.groups, cluster=args.cluster)
+    m = vpps.Model(cell, H, E, C, groups=args.groups, cluster=args.cluster, dataflow=args.sync == "dataflow")
     params = torch.zeros(m.n_floats, device="cuda")
     grads = torch.zeros_like(params)
     for n, _ in shapes:
@@ -60,7 +61,7 @@ def main():
     tot = 0.0
     print(f"{'kernel':70s} {'n':>4s} {'mean us':>9s}")
     for k, v in sorted(per.items(), key=lambda kv: -sum(kv[1])):
-        if "FillFunctor" in k and not args.no_flush and len(v) == args.steps:
+        if "FillFunc" in k and not args.no_flush and len(v) == args.steps:
             name = k + " (L2 flush, not in step)"
         else:
             name = k
