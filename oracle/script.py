@@ -26,7 +26,7 @@ def pre(op: str, length: int) -> int:
 def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 148, by_graph: bool = False):
     """Returns dict(words, pool_words, zero_words, loss_word, n_bar, levels, nodes).
 
-    by_graph: SPEC S5g — whole graphs are assigned to groups (min-load over graph MACs, batch order)
+    by_graph: SPEC S5g — whole graphs are assigned to groups (longest first, smallest estimated group time)
     instead of single nodes per level."""
     # S1/S2: super-graph node list
     nodes = []          # dict(kind, graph, cell(local), children(global ids), token, label, cellnode)
@@ -118,13 +118,25 @@ def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 14
         by_level[level[i]].append(i)
     graph_group = None
     if by_graph:
-        # S5g: whole graphs to the least-loaded group (graph cost = Σ node costs), batch order, ties lowest
-        gload = [0] * G
-        graph_group = []
-        for b in range(len(graphs)):
-            g = min(range(G), key=lambda x: (gload[x], x))
-            gload[g] += sum(cost(n) for n in nodes if n["graph"] == b)
-            graph_group.append(g)
+        # S5g: whole graphs, longest first (depth, then cell count, then batch index), each to the group
+        # whose estimated time after adding it is smallest (ties lowest); time of a group =
+        # Σ_levels (24 ceil(n_l / 16) + n_l), n_l = its cells at level l (batches of 16 per level)
+        hist = [[0] * (L + 1) for _ in range(len(graphs))]
+        for i, n in enumerate(nodes):
+            if n["kind"] != "HEAD":
+                hist[n["graph"]][level[i]] += 1
+        depth = [max((lv for lv in range(L + 1) if hist[b][lv]), default=0) for b in range(len(graphs))]
+        order = sorted(range(len(graphs)), key=lambda b: (-depth[b], -sum(hist[b]), b))
+        gh = [[0] * (L + 1) for _ in range(G)]
+
+        def est(h):
+            return sum(24 * ((x + 15) // 16) + x for x in h)
+
+        graph_group = [0] * len(graphs)
+        for b in order:
+            g = min(range(G), key=lambda x: (est([a + c for a, c in zip(gh[x], hist[b])]), x))
+            gh[g] = [a + c for a, c in zip(gh[g], hist[b])]
+            graph_group[b] = g
     phase_instrs = []            # per phase: per group list of words
     part = []
     for p in range(P):

@@ -192,18 +192,44 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     std::vector<std::vector<uint32_t>> body(G);
     std::vector<int64_t> load(G);
     std::vector<char> was_active(G, 0);
-    // S5g (cluster replicas): every graph goes whole to the least-loaded group, in batch order
+    // S5g (whole-graph replica groups): graphs longest first (depth, then cell count, then batch
+    // index), each to the group whose estimated time after adding it is smallest (ties: lowest group).
+    // A group's time is dominated by its per-level batches of <= 16 cells: est = Σ_l 24 ceil(n_l/16) + n_l.
     std::vector<int32_t> graph_group;
     if (plan.by_graph) {
-        std::vector<int64_t> gcost(b.n_graphs, 0);
-        for (int64_t i = 0; i < N; ++i) gcost[nodes[i].graph] += macs(i);
-        std::vector<int64_t> gload(G, 0);
-        graph_group.resize(b.n_graphs);
-        for (int32_t gi = 0; gi < b.n_graphs; ++gi) {
+        const int32_t NG = b.n_graphs;
+        std::vector<std::vector<int32_t>> hist(NG, std::vector<int32_t>(L + 1, 0));
+        std::vector<int32_t> depth(NG, 0), cells(NG, 0);
+        for (int64_t i = 0; i < N; ++i)
+            if (nodes[i].kind != K_HEAD) {
+                ++hist[nodes[i].graph][level[i]];
+                ++cells[nodes[i].graph];
+                depth[nodes[i].graph] = std::max(depth[nodes[i].graph], level[i]);
+            }
+        std::vector<int32_t> order(NG);
+        for (int32_t gi = 0; gi < NG; ++gi) order[gi] = gi;
+        std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t c) {
+            if (depth[a] != depth[c]) return depth[a] > depth[c];
+            return cells[a] > cells[c];
+        });
+        std::vector<std::vector<int32_t>> gh(G, std::vector<int32_t>(L + 1, 0));
+        auto est_with = [&](int32_t g, int32_t gi) {
+            int64_t t = 0;
+            for (int32_t l = 0; l <= L; ++l) {
+                const int64_t x = gh[g][l] + hist[gi][l];
+                t += 24 * ((x + 15) / 16) + x;
+            }
+            return t;
+        };
+        graph_group.resize(NG);
+        for (int32_t gi : order) {
             int32_t best = 0;
-            for (int32_t g = 1; g < G; ++g)
-                if (gload[g] < gload[best]) best = g;
-            gload[best] += gcost[gi];
+            int64_t best_t = est_with(0, gi);
+            for (int32_t g = 1; g < G; ++g) {
+                const int64_t t = est_with(g, gi);
+                if (t < best_t) { best = g; best_t = t; }
+            }
+            for (int32_t l = 0; l <= L; ++l) gh[best][l] += hist[gi][l];
             graph_group[gi] = best;
         }
     }

@@ -45,20 +45,15 @@ __device__ __forceinline__ u64 tagv(float v, uint32_t e) { return ((u64)e << 32)
 __device__ __forceinline__ void st_tag(u64* p, float v, uint32_t e) {
     asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(tagv(v, e)) : "memory");
 }
+// L1-bypassing poll of one slot (relaxed, gpu scope: always observes the L2 copy)
+__device__ __forceinline__ u64 ld_slot(const u64* p) {
+    u64 v;
+    asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
 __device__ __forceinline__ void st_tag4(u64* p, const float* v, uint32_t e) {
     asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(tagv(v[0], e)), "l"(tagv(v[1], e)) : "memory");
     asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p + 2), "l"(tagv(v[2], e)), "l"(tagv(v[3], e)) : "memory");
-}
-// value of a slot once it carries epoch e (spins; the producer is a co-resident CTA of the group)
-__device__ __forceinline__ float wait_tag(const u64* p, u64 seen, uint32_t e) {
-    while ((uint32_t)(seen >> 32) != e) {
-        __nanosleep(32);
-        asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(seen) : "l"(p) : "memory");
-    }
-    return __uint_as_float((uint32_t)seen);
-}
-__device__ __forceinline__ void cp_async8(void* dst, const void* src) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
 }
 
 template <int H, int E>
@@ -192,102 +187,110 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         const bool is_head = (op == HEAD_F || op == HEAD_B);
         if (is_head && !holds_head) { pos = next; continue; }
         ++nbatch;
+        uint64_t* bt = (prof && tid == 0 && nbatch <= 48 && P.prof_stride >= 16 + 5 * 48) ? prof + 16 + 5 * (nbatch - 1) : nullptr;
+        if (bt) { bt[0] = clock64(); bt[4] = op; }
+        int rounds = 0;
         mark(1);
         if (op == INT_F || is_head) {
-            // rows: [h_l; h_r] (INT_F) or h of the labelled node (heads): tagged HX slots of internal
-            // children -> u64 scratch, leaf records (written by the leaf GEMM) -> xs directly
+            // rows [h_l; h_r] (INT_F) or h of the labelled node (heads), one half row (H values) per
+            // (node, side).  Internal children: H tagged slots = H/2 16-byte pieces -> u64 scratch; leaf
+            // children (leaf GEMM output): H floats = H/4 pieces straight into xs.  Half rows are spread
+            // over the block NTH / (H/2) at a time with shift-only index math.
+            constexpr int PPR = H / 2;                     // pieces per tagged half row
+            constexpr int RPP = NTH / PPR;                 // half rows per pass
             const int A = op == INT_F ? 2 : 1;
-            const int q16 = H / 4;                          // 16-byte pieces per half row of floats
-            for (int i = tid; i < nb * A * q16; i += NTH) {
-                const int n = i / (A * q16), rem = i - n * (A * q16), half = rem / q16, c = (rem - half * q16) * 4;
+            const int rows = nb * A;
+            const int pr = tid % PPR, rsub = tid / PPR;
+            uint32_t my_tagged = 0;                        // bit p: pass p's half row is tagged
+            for (int r = rsub, p = 0; r < rows; r += RPP, ++p) {
+                const int n = A == 2 ? r >> 1 : r, half = A == 2 ? r & 1 : 0;
                 const uint32_t* e = ent + n * sz;
-                const uint32_t rec = op == INT_F ? e[2 + 2 * half] : e[1];
                 const uint32_t hx = op == INT_F ? e[3 + 2 * half] : (op == HEAD_F ? e[3] : e[4]);
                 if (hx == NONE) {
-                    cp_async16(xs + n * KP + half * H + c, pool + rec + c, 16u);
+                    if (pr < H / 4) cp_async16(xs + n * KP + half * H + 4 * pr, pool + (op == INT_F ? e[2 + 2 * half] : e[1]) + 4 * pr, 16u);
                 } else {
-                    const u64* src = HX + (int64_t)hx * H + c;
-                    u64* dst = tbuf + n * KP + half * H + c;
-                    cp_async16(dst, src, 16u);
-                    cp_async16(dst + 2, src + 2, 16u);
+                    cp_async16(tbuf + n * KP + half * H + 2 * pr, HX + (int64_t)hx * H + 2 * pr, 16u);
+                    my_tagged |= 1u << p;
                 }
             }
-            if (op == INT_F) {                              // c_l, c_r of this CTA's units (own records)
-                for (int i = tid; i < nb * UM * 2; i += NTH) {
-                    const int n = i / (UM * 2), rem = i - n * (UM * 2), uu = rem >> 1, k = rem & 1;
-                    const uint32_t* e = ent + n * sz;
-                    cp_async4(cin + (n * UM + uu) * CINMAX + k, pool + e[2 + 2 * k] + H + lc * UM + uu, 4u);
-                }
-            }
-            cp_async_wait_all();
-            __syncthreads();
-            mark(2);
-            // tagged columns: check the epoch, wait for late producers, convert to floats
-            for (int i = tid; i < nb * A * (H / 2); i += NTH) {
-                const int n = i / (A * (H / 2)), rem = i - n * (A * (H / 2)), half = rem / (H / 2);
-                const int c = (rem - half * (H / 2)) * 2;
-                const uint32_t* e = ent + n * sz;
-                const uint32_t hx = op == INT_F ? e[3 + 2 * half] : (op == HEAD_F ? e[3] : e[4]);
-                if (hx == NONE) continue;
-                const u64* t = tbuf + n * KP + half * H + c;
-                const u64* g = HX + (int64_t)hx * H + c;
-                xs[n * KP + half * H + c] = wait_tag(g, t[0], ep);
-                xs[n * KP + half * H + c + 1] = wait_tag(g + 1, t[1], ep);
-            }
-            __syncthreads();
-        } else {
-            // backward: dh = Σ_k PART[parent][lc][k][side*U + u] (+ HD) -> u64 scratch [n][k][U], [n][16][U]
-            for (int i = tid; i < nb * (NCL + 1) * (UM / 2); i += NTH) {
-                const int n = i / ((NCL + 1) * (UM / 2)), rem = i - n * ((NCL + 1) * (UM / 2));
-                const int k = rem / (UM / 2), c = (rem - k * (UM / 2)) * 2;
-                const uint32_t* e = ent + n * sz;
-                const uint32_t dsrc = e[2], hd = e[3];
-                const u64* src = nullptr;
-                if (k < NCL) {
-                    if (dsrc != NONE)
-                        src = PART + ((((int64_t)(dsrc >> 1) * NCL + lc) * NCL + k) * 2 + (dsrc & 1)) * UM + c;
-                } else if (hd != NONE) {
-                    src = HD + (int64_t)hd * H + lc * UM + c;
-                }
-                if (src) cp_async16(tbuf + (n * (NCL + 1) + k) * UM + c, src, 16u);
-            }
-            // own operands: dc (adj + H), c i o u (fl fr) (rec + H..), c_l c_r (children's records)
-            const int ncin = op == INT_B ? 10 : 6;
-            for (int i = tid; i < nb * UM * (ncin - 1); i += NTH) {
-                const int n = i / (UM * (ncin - 1)), rem = i - n * (UM * (ncin - 1));
-                const int uu = rem / (ncin - 1), k = 1 + rem - uu * (ncin - 1);
-                const uint32_t* e = ent + n * sz;
-                const int jj = lc * UM + uu;
-                const float* src;
-                if (k == 1) src = pool + e[1] + H + jj;
-                else if (k < 8) src = pool + e[0] + (k - 1) * H + jj;
-                else src = pool + (k == 8 ? e[5] : e[7]) + H + jj;
-                cp_async4(cin + (n * UM + uu) * CINMAX + k, src, 4u);
-            }
-            cp_async_wait_all();
-            __syncthreads();
-            mark(2);
-            {   // thread (n = tid / U, u = tid % U): the 16 partials (+ head) in fixed order
+            if (op == INT_F && tid < nb * UM) {            // c_l, c_r of this CTA's units (own records)
                 const int n = tid / UM, uu = tid % UM;
-                if (n < nb) {
-                    const uint32_t* e = ent + n * sz;
-                    const uint32_t dsrc = e[2], hd = e[3];
-                    float dh = 0.f;
-                    if (dsrc != NONE) {
-                        const u64* g = PART + (((int64_t)(dsrc >> 1) * NCL + lc) * NCL * 2 + (dsrc & 1)) * UM + uu;
-#pragma unroll 4
-                        for (int k = 0; k < NCL; ++k)
-                            dh += wait_tag(g + (int64_t)k * 2 * UM, tbuf[(n * (NCL + 1) + k) * UM + uu], ep);
+                const uint32_t* e = ent + n * sz;
+                cp_async4(cin + tid * CINMAX, pool + e[2] + H + lc * UM + uu, 4u);
+                cp_async4(cin + tid * CINMAX + 1, pool + e[4] + H + lc * UM + uu, 4u);
+            }
+            cp_async_wait_all();
+            __syncthreads();
+            if (bt) bt[1] = clock64();
+            mark(2);
+            // check the epochs, convert fresh pieces; re-fetch pieces of producers that were still behind
+            while (true) {
+                int stale = 0;
+                for (int r = rsub, p = 0; r < rows; r += RPP, ++p) {
+                    if (!(my_tagged >> p & 1u)) continue;
+                    const int n = A == 2 ? r >> 1 : r, half = A == 2 ? r & 1 : 0;
+                    const int o = n * KP + half * H + 2 * pr;
+                    const u64 a = tbuf[o], b = tbuf[o + 1];
+                    if ((uint32_t)(a >> 32) == ep && (uint32_t)(b >> 32) == ep) {
+                        *reinterpret_cast<float2*>(xs + o) = make_float2(__uint_as_float((uint32_t)a), __uint_as_float((uint32_t)b));
+                        my_tagged &= ~(1u << p);
+                    } else {
+                        const uint32_t* e = ent + n * sz;
+                        const uint32_t hx = op == INT_F ? e[3 + 2 * half] : (op == HEAD_F ? e[3] : e[4]);
+                        cp_async16(tbuf + o, HX + (int64_t)hx * H + 2 * pr, 16u);
+                        ++stale;
                     }
-                    if (hd != NONE) {
-                        const u64* g = HD + (int64_t)hd * H + lc * UM + uu;
-                        dh += wait_tag(g, tbuf[(n * (NCL + 1) + NCL) * UM + uu], ep);
-                    }
-                    cin[(n * UM + uu) * CINMAX] = dh;
                 }
+                if (__syncthreads_count(stale) == 0) break;
+                ++rounds;
+                cp_async_wait_all();
+            }
+        } else {
+            // backward, thread (n = tid / U, u = tid % U): dh = Σ_k PART[parent][lc][k][side][u] (+ HD), its
+            // own 17 slots polled with L1-bypassing relaxed loads; own operands dc (adj + H), c i o u
+            // (fl fr), c_l c_r by cp.async
+            const int n = tid / UM, uu = tid % UM, jj = lc * UM + uu;
+            const bool act = n < nb;
+            const uint32_t* e = ent + (act ? n : 0) * sz;
+            const uint32_t dsrc = act ? e[2] : NONE, hd = act ? e[3] : NONE;
+            if (act) {
+                float* cv = cin + tid * CINMAX;
+                cp_async4(cv + 1, pool + e[1] + H + jj, 4u);
+                const int nrec = op == INT_B ? 6 : 4;
+                for (int k = 0; k < nrec; ++k) cp_async4(cv + 2 + k, pool + e[0] + (k + 1) * H + jj, 4u);
+                if (op == INT_B) {
+                    cp_async4(cv + 8, pool + e[5] + H + jj, 4u);
+                    cp_async4(cv + 9, pool + e[7] + H + jj, 4u);
+                }
+            }
+            const u64* psrc = dsrc != NONE ? PART + ((((int64_t)(dsrc >> 1) * NCL + lc) * NCL) * 2 + (dsrc & 1)) * UM + uu : nullptr;
+            const u64* hsrc = hd != NONE ? HD + (int64_t)hd * H + jj : nullptr;
+            u64 v[NCL + 1];
+            const u64 none = (u64)ep << 32;                // an absent source reads as a current 0
+#pragma unroll
+            for (int k = 0; k < NCL; ++k) v[k] = psrc ? ld_slot(psrc + k * 2 * UM) : none;
+            v[NCL] = hsrc ? ld_slot(hsrc) : none;
+            cp_async_wait_all();
+            if (bt) bt[1] = clock64();
+            mark(2);
+            while (true) {
+                bool stale = false;
+#pragma unroll
+                for (int k = 0; k < NCL; ++k)
+                    if ((uint32_t)(v[k] >> 32) != ep) { stale = true; v[k] = ld_slot(psrc + k * 2 * UM); }
+                if ((uint32_t)(v[NCL] >> 32) != ep) { stale = true; v[NCL] = ld_slot(hsrc); }
+                if (!stale) break;
+                ++rounds;
+            }
+            if (act) {
+                float dh = 0.f;
+#pragma unroll
+                for (int k = 0; k <= NCL; ++k) dh += __uint_as_float((uint32_t)v[k]);
+                cin[tid * CINMAX] = dh;
             }
             __syncthreads();
         }
+        if (bt) { bt[2] = clock64(); bt[4] |= (uint64_t)rounds << 8; }
 
         mark(is_head ? 6 : (op == INT_F ? 3 : 4));
         if (is_head) {            // loss heads (L42) on the CTA holding W_out
@@ -489,6 +492,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             }
         }
         __syncthreads();
+        if (bt) bt[3] = clock64();
         pos = next;
     }
     mark(7);

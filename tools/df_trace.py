@@ -21,6 +21,7 @@ def main():
     ap.add_argument("--batch-idx", type=int, default=0)
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--config", default="tgt")
+    ap.add_argument("--batches", action="store_true", help="per-batch timeline of the last CTA's group")
     args = ap.parse_args()
     import torch
     import synth
@@ -40,7 +41,7 @@ def main():
     dX = torch.zeros_like(X)
     s = m.build_script(synth.config_batch(args.config, args.batch_idx))
     n_cta = m.plan_info()["n_cta"]
-    stride = 16
+    stride = 16 + 5 * 48
     buf = torch.zeros((n_cta, stride), dtype=torch.int64, device="cuda")
     m.set_profile_buffer(buf, stride)
     for _ in range(args.reps):
@@ -61,6 +62,21 @@ def main():
     tot = mean.sum()
     print("section kcycles (mean | CTA that finished last):")
     print("  " + ", ".join(f"{n} {a/1e3:.0f}k ({a/tot*100:.0f}%) | {b/1e3:.0f}k" for n, a, b in zip(names, mean, slow)))
+    if args.batches:
+        last = int(np.argmax(raw[:, 1]))
+        g0 = (last // 16) * 16
+        ops = {0x21: "LEAF_B", 0x22: "INT_F", 0x23: "INT_B", 0x40: "HEAD_F", 0x41: "HEAD_B"}
+        print(f"per-batch cycles of group {last // 16} (CTA {g0} | CTA {last}): issue->staged, staged->fresh "
+              f"(retry rounds), compute, batch end relative to CTA {g0}")
+        nbt = int(raw[last, 2])
+        for cta in (g0,):
+            b = raw[cta, 16:16 + 5 * 48].reshape(48, 5)
+            bl = raw[last, 16:16 + 5 * 48].reshape(48, 5)
+            for k in range(min(nbt, 48)):
+                op = int(b[k, 4]) & 0xFF
+                r = int(b[k, 4]) >> 8
+                print(f"  {k:3d} {ops.get(op, hex(op)):7s} stage {b[k,1]-b[k,0]:6.0f} wait {b[k,2]-b[k,1]:6.0f} ({r} rnd)"
+                      f" compute {b[k,3]-b[k,2]:6.0f} | end skew vs last CTA {bl[k,3]-b[k,3]:7.0f}")
 
 
 if __name__ == "__main__":
