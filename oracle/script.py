@@ -120,7 +120,7 @@ def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 14
     if by_graph:
         # S5g: whole graphs, longest first (depth, then cell count, then batch index), each to the group
         # whose estimated time after adding it is smallest (ties lowest); time of a group =
-        # Σ_levels (24 ceil(n_l / 16) + n_l), n_l = its cells at level l (batches of 16 per level)
+        # Σ_levels (2 ceil(n_l / 16) + n_l), n_l = its cells at level l (batches of 16 per level)
         hist = [[0] * (L + 1) for _ in range(len(graphs))]
         for i, n in enumerate(nodes):
             if n["kind"] != "HEAD":
@@ -130,7 +130,7 @@ def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 14
         gh = [[0] * (L + 1) for _ in range(G)]
 
         def est(h):
-            return sum(24 * ((x + 15) // 16) + x for x in h)
+            return sum(2 * ((x + 15) // 16) + x for x in h)
 
         graph_group = [0] * len(graphs)
         for b in order:

@@ -194,7 +194,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     std::vector<char> was_active(G, 0);
     // S5g (whole-graph replica groups): graphs longest first (depth, then cell count, then batch
     // index), each to the group whose estimated time after adding it is smallest (ties: lowest group).
-    // A group's time is dominated by its per-level batches of <= 16 cells: est = Σ_l 24 ceil(n_l/16) + n_l.
+    // A group's time: per-level batches of <= 16 cells plus per-cell work: est = Σ_l 2 ceil(n_l/16) + n_l.
     std::vector<int32_t> graph_group;
     if (plan.by_graph) {
         const int32_t NG = b.n_graphs;
@@ -213,11 +213,12 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
             return cells[a] > cells[c];
         });
         std::vector<std::vector<int32_t>> gh(G, std::vector<int32_t>(L + 1, 0));
+        constexpr int64_t kBatch = 2;   // per-batch overhead in units of one cell (measured sweep)
         auto est_with = [&](int32_t g, int32_t gi) {
             int64_t t = 0;
             for (int32_t l = 0; l <= L; ++l) {
                 const int64_t x = gh[g][l] + hist[gi][l];
-                t += 24 * ((x + 15) / 16) + x;
+                t += kBatch * ((x + 15) / 16) + x;
             }
             return t;
         };

@@ -14,6 +14,7 @@
 //   HD[node][H]          the loss head's contribution to a labelled node's dh
 // The epoch is the pass counter, so slots never need clearing.  Without hardware clusters the groups
 // are ordinary co-resident CTAs of a cooperative launch: 9 groups on 144 SMs instead of 7 clusters.
+#include <type_traits>
 #include "vpps_kernel.cuh"
 #include "dev_common.cuh"
 
@@ -354,10 +355,13 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         } else if (op == INT_F) {
             // ---- forward of internal cells: matvec from registers (L123), 4 nodes at a time; the unit's
             //      16 lanes reduce with a transposed butterfly; the lane holding node n's gates updates it ----
-            for (int n0 = 0; n0 < nb; n0 += 4) {
-                float2 a[4][5];
+            // groups of NN in {4, 2, 1} nodes: the unit's 16 lanes reduce NN partial sums with a transposed
+            // butterfly, after which lane 16/NN * m holds node m's gates
+            auto fwd_group = [&](auto nnc, int n0) {
+                constexpr int NN = decltype(nnc)::value;
+                float2 a[NN][5];
 #pragma unroll
-                for (int n = 0; n < 4; ++n)
+                for (int n = 0; n < NN; ++n)
 #pragma unroll
                     for (int o = 0; o < 5; ++o) a[n][o] = make_float2(0.f, 0.f);
 #pragma unroll
@@ -365,7 +369,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                     const int col0 = LB::CG * (tu + TU * t);
                     const int of = col0 < H ? 3 : 4;
 #pragma unroll
-                    for (int n = 0; n < 4; ++n) {
+                    for (int n = 0; n < NN; ++n) {
                         float xv[LB::CG];
                         lds<LB::CG>(xs + (n0 + n) * KP + col0, xv);
 #pragma unroll
@@ -383,11 +387,28 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 }
                 float g5[5];
 #pragma unroll
-                for (int o = 0; o < 5; ++o)
-                    g5[o] = treduce4_16(a[0][o].x + a[0][o].y, a[1][o].x + a[1][o].y, a[2][o].x + a[2][o].y,
-                                        a[3][o].x + a[3][o].y, gl);
-                const int n = n0 + (gl >> 2);
-                if ((gl & 3) == 0 && n < nb) {
+                for (int o = 0; o < 5; ++o) {
+                    if constexpr (NN == 4) {
+                        g5[o] = treduce4_16(a[0][o].x + a[0][o].y, a[1][o].x + a[1][o].y, a[2][o].x + a[2][o].y,
+                                            a[3][o].x + a[3][o].y, gl);
+                    } else if constexpr (NN == 2) {
+                        const bool b3 = gl & 8;
+                        const float v0 = a[0][o].x + a[0][o].y, v1 = a[1][o].x + a[1][o].y;
+                        float k = b3 ? v1 : v0;
+                        k += __shfl_xor_sync(FULLMASK, b3 ? v0 : v1, 8);
+                        k += __shfl_xor_sync(FULLMASK, k, 4);
+                        k += __shfl_xor_sync(FULLMASK, k, 2);
+                        g5[o] = k + __shfl_xor_sync(FULLMASK, k, 1);
+                    } else {
+                        float k = a[0][o].x + a[0][o].y;
+#pragma unroll
+                        for (int d = 8; d >= 1; d >>= 1) k += __shfl_xor_sync(FULLMASK, k, d);
+                        g5[o] = k;
+                    }
+                }
+                constexpr int SPAN = 16 / NN;
+                const int n = n0 + gl / SPAN;
+                if (gl % SPAN == 0 && n < nb) {
                     const uint32_t* e = ent + n * sz;
                     const uint32_t rec = e[0];
                     const float* b = bias + u * 4;
@@ -405,7 +426,11 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                     pool[rec + 5 * H + j] = fl;
                     pool[rec + 6 * H + j] = fr;
                 }
-            }
+            };
+            int n0 = 0;
+            for (; n0 + 2 < nb; n0 += 4) fwd_group(std::integral_constant<int, 4>{}, n0);
+            if (nb - n0 == 2) fwd_group(std::integral_constant<int, 2>{}, n0);
+            else if (nb - n0 == 1) fwd_group(std::integral_constant<int, 1>{}, n0);
         } else {
             // ---- backward: cell backward by thread (unit u, node gl); gate gradients recorded for the dW
             //      GEMM (L185) and broadcast to the unit's lanes ----
@@ -448,6 +473,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
 #pragma unroll
                     for (int dn = 0; dn < NC; ++dn) {
                         const int n = n0 + dn;
+                        if (n >= nb) break;
                         float gr[5];
 #pragma unroll
                         for (int r = 0; r < 5; ++r) gr[r] = __shfl_sync(FULLMASK, g[r], src | (n & 15));
