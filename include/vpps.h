@@ -109,6 +109,8 @@ typedef struct {
     int64_t n_heads;
     double flops;         /* algorithmic FLOPs of the pass (2/MAC; fwd, dW, dX/dh)     */
     double act_bytes;     /* algorithmic activation bytes read+written by the pass     */
+    int64_t blob_words;   /* words copied host->device per pass: the script words plus the device-side
+                             node lists and dataflow program (the one H2D copy of L169)  */
 } vpps_script_info;
 
 /* ---- model (vpps::handle hndl(model)) -------------------------------------- */

@@ -315,6 +315,7 @@ vpps_status vpps_script_info_get(vpps_script s, vpps_script_info* info) {
     info->n_heads = s->s.n_heads;
     info->flops = s->s.flops;
     info->act_bytes = s->s.act_bytes;
+    info->blob_words = (int64_t)s->s.blob.size();
     return VPPS_OK;
 }
 

@@ -7,6 +7,7 @@ into exceptions.  There is no CPU fallback: if libvpps.so is missing, importing 
 from __future__ import annotations
 
 import ctypes as ct
+import itertools
 import os
 
 import numpy as np
@@ -47,7 +48,7 @@ class _Info(ct.Structure):
     _fields_ = [("n_words", ct.c_int64), ("pool_words", ct.c_int64), ("zero_words", ct.c_int64),
                 ("loss_word", ct.c_int64), ("n_barriers", ct.c_int32), ("n_levels", ct.c_int32),
                 ("n_nodes", ct.c_int64), ("n_heads", ct.c_int64), ("flops", ct.c_double),
-                ("act_bytes", ct.c_double)]
+                ("act_bytes", ct.c_double), ("blob_words", ct.c_int64)]
 
 
 def _load():
@@ -147,16 +148,56 @@ def paper_choose_cps(mats, n_sm, tb=256, rpw=1, pack_rows=True):
 
 def to_csr(graphs):
     """Graphs as lists of (children, token, label) -> CSR int32 arrays of vpps_batch."""
-    gp, cp, ch, tok, lab = [0], [0], [], [], []
-    for g in graphs:
-        for (c, t, l) in g:
-            ch.extend(c)
-            cp.append(len(ch))
-            tok.append(t)
-            lab.append(l)
-        gp.append(len(tok))
-    as32 = lambda a: np.ascontiguousarray(np.asarray(a, dtype=np.int32))
-    return as32(gp), as32(cp), as32(ch if ch else [0]), as32(tok), as32(lab)
+    nodes = [n for g in graphs for n in g]
+    nn = len(nodes)
+    gp = np.zeros(len(graphs) + 1, np.int32)
+    np.cumsum(np.fromiter((len(g) for g in graphs), np.int32, len(graphs)), out=gp[1:])
+    cp = np.zeros(nn + 1, np.int32)
+    np.cumsum(np.fromiter((len(n[0]) for n in nodes), np.int32, nn), out=cp[1:])
+    ch = np.fromiter(itertools.chain.from_iterable(n[0] for n in nodes), np.int32, int(cp[-1]))
+    tok = np.fromiter((n[1] for n in nodes), np.int32, nn)
+    lab = np.fromiter((n[2] for n in nodes), np.int32, nn)
+    return gp, cp, ch if ch.size else np.zeros(1, np.int32), tok, lab
+
+
+class CsrBatch:
+    """A batch in the CSR form of vpps_batch (include/vpps.h): graph_ptr, child_ptr, children, token, label."""
+
+    def __init__(self, graph_ptr, child_ptr, children, token, label):
+        as32 = lambda a: np.ascontiguousarray(np.asarray(a, dtype=np.int32))
+        self.arrays = (as32(graph_ptr), as32(child_ptr), as32(children), as32(token), as32(label))
+
+    @classmethod
+    def from_graphs(cls, graphs):
+        return cls(*to_csr(graphs))
+
+
+def prefetch_scripts(model: "Model", batches, depth: int = 3):
+    """Yield model.build_script(b) for b in batches, built `depth` ahead on a background thread (the C++
+    builder runs without the GIL), so host script generation overlaps the device pass."""
+    import queue
+    import threading
+    q = queue.Queue(maxsize=depth)
+    done = object()
+
+    def work():
+        try:
+            for b in batches:
+                q.put(model.build_script(b))
+        except BaseException as e:   # surface builder errors in the consumer
+            q.put(e)
+        q.put(done)
+
+    th = threading.Thread(target=work, daemon=True)
+    th.start()
+    while True:
+        item = q.get()
+        if item is done:
+            break
+        if isinstance(item, BaseException):
+            raise item
+        yield item
+    th.join()
 
 
 class Script:
@@ -236,8 +277,11 @@ class Model:
         return dict(n_cta=a.value, n_g=b.value, n_act=c.value, umax=d.value)
 
     def build_script(self, graphs) -> Script:
-        gp, cp, ch, tok, lab = to_csr(graphs)
-        b = _Batch(len(graphs), gp.ctypes.data, cp.ctypes.data, ch.ctypes.data, tok.ctypes.data, lab.ctypes.data)
+        """graphs: a list of graphs (lists of (children, token, label)) or a CsrBatch (to_csr output, the
+        form a data loader hands over: no per-node Python work)."""
+        csr = graphs if isinstance(graphs, CsrBatch) else CsrBatch(*to_csr(graphs))
+        gp, cp, ch, tok, lab = csr.arrays
+        b = _Batch(len(gp) - 1, gp.ctypes.data, cp.ctypes.data, ch.ctypes.data, tok.ctypes.data, lab.ctypes.data)
         h = ct.c_void_p()
         _check(_lib.vpps_build_script(self._h, ct.byref(b), ct.byref(h)))
         return Script(self, h)
