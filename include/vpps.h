@@ -111,6 +111,9 @@ typedef struct {
     double act_bytes;     /* algorithmic activation bytes read+written by the pass     */
     int64_t blob_words;   /* words copied host->device per pass: the script words plus the device-side
                              node lists and dataflow program (the one H2D copy of L169)  */
+    double kernel_flops;  /* algorithmic FLOPs of the replica-group kernel of the binary cluster /
+                             dataflow paths (internal-cell matvecs and transposed products, 32 H^2
+                             per cell, and the loss heads); the rest of `flops` runs in the GEMMs */
 } vpps_script_info;
 
 /* ---- model (vpps::handle hndl(model)) -------------------------------------- */
@@ -183,6 +186,12 @@ vpps_status vpps_sync_get_latest_loss(vpps_model m, float* loss);
  * ev_before immediately before and ev_after immediately after the persistent kernel on the
  * launching stream, so the kernel's own duration can be timed without the pool memsets. */
 vpps_status vpps_set_timing_events(vpps_model m, void* ev_before, void* ev_after);
+
+/* Measurement hook for the replica-group kernel alone (cluster / dataflow paths): ev_before and ev_after
+ * are recorded immediately around vpps_cl / vpps_df only.  The records sit between programmatically
+ * dependent launches, so while set the neighbouring GEMMs no longer overlap that kernel: use it for a
+ * separate timing pass.  NULL clears. */
+vpps_status vpps_set_kernel_events(vpps_model m, void* ev_before, void* ev_after);
 
 /* In-kernel phase trace (measurement only): when buf != NULL (dev, >= n_cta*stride uint64), every
  * later launch writes per CTA, from %globaltimer (ns): [0] start of interpretation, [1] end, and for

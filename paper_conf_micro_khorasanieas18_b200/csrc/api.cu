@@ -59,6 +59,7 @@ struct vpps_model_s {
     cudaEvent_t ev[2] = {nullptr, nullptr};
     int64_t passes = 0;
     cudaEvent_t t_before = nullptr, t_after = nullptr;
+    cudaEvent_t k_before = nullptr, k_after = nullptr;   // around the replica-group kernel only
     uint64_t* prof = nullptr;
     int64_t prof_stride = 0;
     int32_t cluster = 0;                // > 1: cluster-replica path (vpps_cluster.cu)
@@ -316,6 +317,7 @@ vpps_status vpps_script_info_get(vpps_script s, vpps_script_info* info) {
     info->flops = s->s.flops;
     info->act_bytes = s->s.act_bytes;
     info->blob_words = (int64_t)s->s.blob.size();
+    info->kernel_flops = s->s.kernel_flops;
     return VPPS_OK;
 }
 
@@ -449,7 +451,9 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         const float* W_iou = m->params + m->offsets[0];
         launch_leaf_fwd(W_iou, m->params + m->offsets[5], inputs, m->pool, leaf_list, (int32_t)s->s.n_leaf,
                         m->plan.H, m->plan.E, st);
+        if (m->k_before) CK(cudaEventRecord(m->k_before, st));
         CK(cudaLaunchKernelExC(&cfg, m->var->fn, dargs));
+        if (m->k_after) CK(cudaEventRecord(m->k_after, st));
         const int32_t n_grp = (int32_t)s->s.int_off.size() - 1;
         std::vector<int32_t> order(n_grp);
         for (int32_t g = 0; g < n_grp; ++g) order[g] = g;
@@ -487,7 +491,9 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         // level 0 (all leaves share W_iou on their word vectors) as one dense GEMM + cell pass
         launch_leaf_fwd(W_iou, m->params + m->offsets[5], inputs, m->pool, leaf_list, (int32_t)s->s.n_leaf,
                         m->plan.H, m->plan.E, st);
+        if (m->k_before) CK(cudaEventRecord(m->k_before, st));
         CK(cudaLaunchKernelExC(&cfg, m->var->fn, args));
+        if (m->k_after) CK(cudaEventRecord(m->k_after, st));
         // dW of the weight matrices from the recorded operands and dX of the leaves
         // = W_iouᵀ g_leaf (words are inputs) in one launch; SGD in mode 1.  Groups whose
         // cluster should finish first (fewest levels, then fewest nodes) get the lowest tile indices.
@@ -559,6 +565,13 @@ vpps_status vpps_set_timing_events(vpps_model m, void* ev_before, void* ev_after
     if (!m) return fail(VPPS_E_INVALID, "null model");
     m->t_before = (cudaEvent_t)ev_before;
     m->t_after = (cudaEvent_t)ev_after;
+    return VPPS_OK;
+}
+
+vpps_status vpps_set_kernel_events(vpps_model m, void* ev_before, void* ev_after) {
+    if (!m) return fail(VPPS_E_INVALID, "null model");
+    m->k_before = (cudaEvent_t)ev_before;
+    m->k_after = (cudaEvent_t)ev_after;
     return VPPS_OK;
 }
 

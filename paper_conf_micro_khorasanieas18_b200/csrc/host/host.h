@@ -66,6 +66,7 @@ struct Script {
     int64_t df_off = -1, n_hx = 0, n_part = 0, n_hd = 0;
     int64_t df_hx = 0, df_part = 0, df_hd = 0, df_words = 0;
     double flops = 0.0, act_bytes = 0.0;
+    double kernel_flops = 0.0;   // binary whole-graph paths: FLOPs of the replica-group kernel alone
 };
 
 // Returns 0 on success, -4 (graph error) or -1 (invalid) with a message.

@@ -287,6 +287,14 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     }
     s.flops = flops;
     s.act_bytes = abytes;
+    // replica-group kernel of the binary whole-graph paths: per internal cell the recurrent matvec and
+    // its transpose (2 x 8 H^2 MACs), per head the logits, dW_out and dh (3 C H MACs); leaves and dW are
+    // GEMMs outside it
+    s.kernel_flops = 0.0;
+    for (const Node& n : nodes) {
+        if (n.kind == K_INT) s.kernel_flops += 2.0 * 16.0 * (double)H * (double)H;
+        else if (n.kind == K_HEAD) s.kernel_flops += 2.0 * 3.0 * (double)C * (double)H;
+    }
     // device blob: the words, then the operand lists of the per-matrix gradient GEMM (binary cells)
     // (grouped by replica group when graphs are assigned whole, S5g: the GEMM tiles of a group can then
     // start as soon as that group's cluster has finished)

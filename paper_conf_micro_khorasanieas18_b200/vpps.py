@@ -48,7 +48,7 @@ class _Info(ct.Structure):
     _fields_ = [("n_words", ct.c_int64), ("pool_words", ct.c_int64), ("zero_words", ct.c_int64),
                 ("loss_word", ct.c_int64), ("n_barriers", ct.c_int32), ("n_levels", ct.c_int32),
                 ("n_nodes", ct.c_int64), ("n_heads", ct.c_int64), ("flops", ct.c_double),
-                ("act_bytes", ct.c_double), ("blob_words", ct.c_int64)]
+                ("act_bytes", ct.c_double), ("blob_words", ct.c_int64), ("kernel_flops", ct.c_double)]
 
 
 def _load():
@@ -76,6 +76,7 @@ def _load():
         "vpps_sync_get_latest_loss": [VP, P(F)],
         "vpps_pool_ptr": [VP, P(VP), P(I64)],
         "vpps_set_timing_events": [VP, VP, VP],
+        "vpps_set_kernel_events": [VP, VP, VP],
         "vpps_set_profile_buffer": [VP, VP, I64],
         "vpps_destroy_script": [VP],
         "vpps_destroy_model": [VP],
@@ -312,6 +313,11 @@ class Model:
     def set_timing_events(self, before, after):
         """torch.cuda.Event pair recorded around every later kernel launch (None clears)."""
         _check(_lib.vpps_set_timing_events(self._h, ct.c_void_p(before.cuda_event) if before else None,
+                                           ct.c_void_p(after.cuda_event) if after else None))
+
+    def set_kernel_events(self, before, after):
+        """torch.cuda.Event pair recorded around the replica-group kernel alone (None clears)."""
+        _check(_lib.vpps_set_kernel_events(self._h, ct.c_void_p(before.cuda_event) if before else None,
                                            ct.c_void_p(after.cuda_event) if after else None))
 
     def set_profile_buffer(self, buf=None, stride=0):
