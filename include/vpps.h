@@ -198,6 +198,10 @@ vpps_status vpps_set_kernel_events(vpps_model m, void* ev_before, void* ev_after
  * barrier b: [2+3b] signal, [3+3b] wait begin, [4+3b] wait end.  stride >= 2 + 3*(n_barriers+1). */
 vpps_status vpps_set_profile_buffer(vpps_model m, uint64_t* buf, int64_t stride);
 
+/* Measurement hook (dataflow path): when buf != NULL (dev, >= 5 x gradient-GEMM items uint64), every
+ * later pass writes per item of the gradient GEMM (group, item, start ns, end ns, SM id). */
+vpps_status vpps_set_gemm_trace(vpps_model m, uint64_t* buf);
+
 /* Device pointer of the model's activation pool (SPEC §S7 layout of the last script run). */
 vpps_status vpps_pool_ptr(vpps_model m, float** pool, int64_t* pool_words);
 

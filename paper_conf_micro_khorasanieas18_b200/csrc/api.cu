@@ -55,17 +55,19 @@ struct vpps_model_s {
     float* grads = nullptr;
     float* pool = nullptr;
     int64_t pool_cap = 0, last_pool_words = 0;
-    float* h_loss = nullptr;            // pinned [2]
+    float* h_loss = nullptr;            // pinned [2] (mapped on the cluster / dataflow paths)
+    float* d_loss_map = nullptr;        // device view of h_loss (kernel writes the loss directly)
     cudaEvent_t ev[2] = {nullptr, nullptr};
     int64_t passes = 0;
     cudaEvent_t t_before = nullptr, t_after = nullptr;
     cudaEvent_t k_before = nullptr, k_after = nullptr;   // around the replica-group kernel only
+    uint64_t* gemm_trace = nullptr;                      // measurement: gradient GEMM item stamps
     uint64_t* prof = nullptr;
     int64_t prof_stride = 0;
     int32_t cluster = 0;                // > 1: cluster-replica path (vpps_cluster.cu)
-    int32_t* done = nullptr;            // cluster path: per-group completion counters [kMaxGroups]
+    int32_t* done = nullptr;            // per-group completion counters [kMaxGroups] + GEMM claim counters [kMaxGroups]
     bool dataflow = false;              // groups of co-resident CTAs synchronised by tagged slots (vpps_df)
-    uint32_t epoch = 0;                 // dataflow pass counter (slot tags)
+    uint32_t* d_epoch = nullptr;        // dataflow pass counter on the device (slot tags), advanced per pass
     static constexpr int kMaxGroups = 16;
     // Pre-allocated staging ring for per-batch scripts: a pinned host buffer and a
     // device buffer per slot; a slot is reused once the kernel that last read it has finished.
@@ -194,8 +196,12 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     if (m->cluster && m->plan.n_g != m->cluster) return fail(VPPS_E_INVALID, "groups x cluster must equal n_sm");
     if (m->cluster && !m->plan_only) {
         if (m->plan.G > vpps_model_s::kMaxGroups) return fail(VPPS_E_NOFIT, "more than 16 cluster replicas");
-        CK(cudaMalloc(&m->done, vpps_model_s::kMaxGroups * sizeof(int32_t)));
-        CK(cudaMallocHost(&m->h_loss, 2 * sizeof(float)));
+        CK(cudaMalloc(&m->done, 4 * vpps_model_s::kMaxGroups * sizeof(int32_t)));   // done, claim, fin/tail
+        CK(cudaMemset(m->done, 0, 4 * vpps_model_s::kMaxGroups * sizeof(int32_t)));
+        CK(cudaMalloc(&m->d_epoch, sizeof(uint32_t)));
+        CK(cudaMemset(m->d_epoch, 0, sizeof(uint32_t)));
+        CK(cudaHostAlloc(&m->h_loss, 2 * sizeof(float), cudaHostAllocMapped));
+        CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&m->d_loss_map), m->h_loss, 0));
         m->h_loss[0] = m->h_loss[1] = 0.f;
         CK(cudaEventCreateWithFlags(&m->ev[0], cudaEventDisableTiming));
         CK(cudaEventCreateWithFlags(&m->ev[1], cudaEventDisableTiming));
@@ -385,10 +391,15 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         vpps_status r = stage_script(m, s, st, &ring_slot, &dwords);
         if (r != VPPS_OK) return r;
     }
-    CK(cudaMemsetAsync(m->pool, 0, s->s.zero_words * sizeof(float), st));
-    if (m->plan.G > 1 || m->cluster) CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));
-    if (m->cluster) CK(cudaMemsetAsync(m->done, 0, vpps_model_s::kMaxGroups * sizeof(int32_t), st));
-    if (d_inputs) CK(cudaMemsetAsync(d_inputs, 0, (size_t)n_rows * m->plan.E * sizeof(float), st));
+    // per-pass clearing: the cluster / dataflow paths fold it into the leaf kernel (no memset calls)
+    float* zero_ptr[4] = {m->pool, m->grads, reinterpret_cast<float*>(m->done), d_inputs};
+    const int64_t zero_n[4] = {s->s.zero_words, m->n_floats, 4 * vpps_model_s::kMaxGroups,
+                               d_inputs ? n_rows * m->plan.E : 0};
+    if (!m->cluster) {
+        CK(cudaMemsetAsync(m->pool, 0, s->s.zero_words * sizeof(float), st));
+        if (m->plan.G > 1) CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));
+        if (d_inputs) CK(cudaMemsetAsync(d_inputs, 0, (size_t)n_rows * m->plan.E * sizeof(float), st));
+    }
     KParams kp{};
     kp.params = m->params;
     kp.grads = m->grads;
@@ -413,9 +424,9 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     void* args[] = {&kp};
     if (m->t_before) CK(cudaEventRecord(m->t_before, st));
     if (m->dataflow) {
-        // leaf GEMM -> vpps_df (cooperative: the groups' CTAs must be co-resident because consumers
-        // spin on producers; programmatic dependent: weight prologue overlaps the leaf tail) -> gradient
-        // GEMM (programmatic dependent, per-group completion counters) -> SGD
+        // leaf GEMM (also clears the pass's accumulators, advances the pass counter) -> vpps_df
+        // (cooperative: the groups' CTAs must be co-resident because consumers spin on producers) ->
+        // gradient GEMM (programmatic dependent, per-group completion counters) -> SGD
         DfParams dp{};
         dp.params = m->params;
         dp.grads = m->grads;
@@ -424,8 +435,7 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         dp.df_off = s->s.df_off;
         for (size_t i = 0; i < m->offsets.size() && i < 8; ++i) dp.off[i] = m->offsets[i];
         dp.C = m->plan.C;
-        dp.epoch = ++m->epoch;
-        if (dp.epoch == 0) dp.epoch = ++m->epoch;      // 0 is the value of never-written slots
+        dp.epoch = m->d_epoch;
         dp.loss_word = s->s.loss_word;
         dp.df_hx = s->s.df_hx;
         dp.df_part = s->s.df_part;
@@ -438,19 +448,17 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         cudaLaunchAttribute attr[2];
         attr[0].id = cudaLaunchAttributeCooperative;
         attr[0].val.cooperative = 1;
-        attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-        attr[1].val.programmaticStreamSerializationAllowed = 1;
         cfg.gridDim = dim3(m->plan.n_cta);
         cfg.blockDim = dim3(256);
         cfg.dynamicSmemBytes = m->smem;
         cfg.stream = st;
         cfg.attrs = attr;
-        cfg.numAttrs = 2;
+        cfg.numAttrs = 1;       // ordinary stream order after the leaf kernel (which clears `done`)
         const uint32_t* lists = dwords + s->s.words.size();
         const uint32_t* leaf_list = lists + 3 * s->s.n_int;
         const float* W_iou = m->params + m->offsets[0];
         launch_leaf_fwd(W_iou, m->params + m->offsets[5], inputs, m->pool, leaf_list, (int32_t)s->s.n_leaf,
-                        m->plan.H, m->plan.E, st);
+                        m->plan.H, m->plan.E, zero_ptr, zero_n, m->d_epoch, st);
         if (m->k_before) CK(cudaEventRecord(m->k_before, st));
         CK(cudaLaunchKernelExC(&cfg, m->var->fn, dargs));
         if (m->k_after) CK(cudaEventRecord(m->k_after, st));
@@ -463,13 +471,14 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         });
         launch_dw_gemm(m->pool, inputs, d_inputs, m->params, m->grads, lists, leaf_list, n_grp, s->s.int_off.data(),
                        s->s.leaf_off.data(), order.data(), m->done, m->cluster, true, m->plan.H, m->plan.E,
-                       m->offsets.data(), m->n_floats, mode, lr, wd, st);
+                       m->offsets.data(), m->n_floats, mode, lr, wd, st, m->gemm_trace,
+                       m->pool + s->s.loss_word, m->d_loss_map + (m->passes & 1));
         CK(cudaGetLastError());
     } else if (m->cluster) {
         // one cluster per replica group; clusters never wait on each other (graphs are whole per group).
-        // Launch order: leaf GEMM -> vpps_cl (programmatic dependent: weight prologue overlaps the leaf
-        // tail, griddepcontrol.wait before level 1) -> gradient GEMM (programmatic dependent: a group's
-        // tiles start when its cluster's 16 CTAs have counted themselves done) -> SGD.
+        // Launch order: leaf GEMM (also clears the pass's accumulators) -> vpps_cl -> gradient GEMM
+        // (programmatic dependent: a group's tiles start when its cluster's 16 CTAs have counted
+        // themselves done) -> SGD.
         kp.done = m->done;
         cudaLaunchConfig_t cfg = {};
         cudaLaunchAttribute attr[2];
@@ -477,20 +486,18 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         attr[0].val.clusterDim.x = m->cluster;
         attr[0].val.clusterDim.y = 1;
         attr[0].val.clusterDim.z = 1;
-        attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-        attr[1].val.programmaticStreamSerializationAllowed = 1;
         cfg.gridDim = dim3(m->plan.n_cta);
         cfg.blockDim = dim3(256);
         cfg.dynamicSmemBytes = m->smem;
         cfg.stream = st;
         cfg.attrs = attr;
-        cfg.numAttrs = 2;
+        cfg.numAttrs = 1;       // ordinary stream order after the leaf kernel (which clears `done`)
         const uint32_t* lists = dwords + s->s.words.size();
         const uint32_t* leaf_list = lists + 3 * s->s.n_int;
         const float* W_iou = m->params + m->offsets[0];
         // level 0 (all leaves share W_iou on their word vectors) as one dense GEMM + cell pass
         launch_leaf_fwd(W_iou, m->params + m->offsets[5], inputs, m->pool, leaf_list, (int32_t)s->s.n_leaf,
-                        m->plan.H, m->plan.E, st);
+                        m->plan.H, m->plan.E, zero_ptr, zero_n, nullptr, st);
         if (m->k_before) CK(cudaEventRecord(m->k_before, st));
         CK(cudaLaunchKernelExC(&cfg, m->var->fn, args));
         if (m->k_after) CK(cudaEventRecord(m->k_after, st));
@@ -506,7 +513,8 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         });
         launch_dw_gemm(m->pool, inputs, d_inputs, m->params, m->grads, lists, leaf_list, n_grp, s->s.int_off.data(),
                        s->s.leaf_off.data(), order.data(), m->done, m->cluster, true, m->plan.H, m->plan.E,
-                       m->offsets.data(), m->n_floats, mode, lr, wd, st);
+                       m->offsets.data(), m->n_floats, mode, lr, wd, st, nullptr,
+                       m->pool + s->s.loss_word, m->d_loss_map + (m->passes & 1));
         CK(cudaGetLastError());
     } else {
         CK(cudaLaunchCooperativeKernel(m->var->fn, dim3(m->plan.n_cta), dim3(256), args, m->smem, st));
@@ -517,7 +525,8 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         m->ring[ring_slot].used = true;
     }
     const int slot = (int)(m->passes & 1);
-    CK(cudaMemcpyAsync(m->h_loss + slot, m->pool + s->s.loss_word, sizeof(float), cudaMemcpyDeviceToHost, st));
+    if (!m->cluster)   // (the cluster / dataflow gradient kernel writes the loss into mapped h_loss itself)
+        CK(cudaMemcpyAsync(m->h_loss + slot, m->pool + s->s.loss_word, sizeof(float), cudaMemcpyDeviceToHost, st));
     CK(cudaEventRecord(m->ev[slot], st));
     ++m->passes;
     return VPPS_OK;
@@ -575,6 +584,12 @@ vpps_status vpps_set_kernel_events(vpps_model m, void* ev_before, void* ev_after
     return VPPS_OK;
 }
 
+vpps_status vpps_set_gemm_trace(vpps_model m, uint64_t* buf) {
+    if (!m) return fail(VPPS_E_INVALID, "null model");
+    m->gemm_trace = buf;
+    return VPPS_OK;
+}
+
 vpps_status vpps_set_profile_buffer(vpps_model m, uint64_t* buf, int64_t stride) {
     if (!m) return fail(VPPS_E_INVALID, "null model");
     m->prof = buf;
@@ -599,7 +614,8 @@ void vpps_destroy_model(vpps_model m) {
     if (!m) return;
     if (m->pool) cudaFree(m->pool);
     if (m->done) cudaFree(m->done);
-    if (m->h_loss) cudaFreeHost(m->h_loss);
+    if (m->d_epoch) cudaFree(m->d_epoch);
+    if (m->h_loss) cudaFreeHost(m->h_loss);   // (cudaHostAlloc'd or cudaMallocHost'd: both freed here)
     for (cudaEvent_t e : m->ev)
         if (e) cudaEventDestroy(e);
     for (auto& sl : m->ring) {

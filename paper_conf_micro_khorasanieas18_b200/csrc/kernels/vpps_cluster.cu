@@ -9,6 +9,8 @@
 // the paper's gradient-accumulation strategy (L185, §III-C2): it records the outer-product operands
 // (the gate gradients, next to the activations already in the pool) and one GEMM per weight matrix
 // (vpps_dw_gemm below) forms dW = Σ g xᵀ afterwards, fused with the SGD update (L129, L197).
+#include <algorithm>
+#include <cstdlib>
 #include "vpps_kernel.cuh"
 #include "dev_common.cuh"
 
@@ -599,85 +601,92 @@ struct GemmParams {
     int64_t off[8];
     const float* w_iou;          // W_iou (params), for the leaf input gradient
     float* d_inputs;             // dX, or nullptr
-    const int32_t* done;         // per-group completion counters written by vpps_cl (nullptr: no wait)
-    int32_t done_target;         // CTAs per cluster
+    const int32_t* done;         // per-group completion counters written by vpps_cl / vpps_df (nullptr: no wait)
+    int32_t* claim;              // per-group work-claim counters (zeroed per pass), used with `done`
+    int32_t done_target;         // CTAs per group
     int32_t n_grp;
-    int32_t grp[16];             // groups in processing order (clusters expected to finish first go first)
+    int32_t grp[16];             // groups in processing order (groups expected to finish first go first)
     int32_t int_off[17], leaf_off[17];
-    int32_t items[16];           // work items of grp[q]
+    int32_t items[16];           // work items of group g (indexed by group)
+    int32_t static_items;        // 1: one CTA per item (waiting on its group) instead of persistent claiming
+    uint64_t* trace;             // measurement only: per claimed item (group, item, start ns, end ns, smid)
+    // fused tail (persistent mode): once every item is finished (counter fin == total_items) the CTAs
+    // apply SGD to the flat parameters in claimed chunks (mode 1) and one CTA copies the summed loss to
+    // mapped host memory (loss_dst, may be null)
+    int32_t* fin;
+    int32_t* tail_claim;
+    int32_t total_items;
+    int32_t mode;
+    float* params;
+    int64_t n_floats;
+    float lr, wd;
+    const float* loss_src;
+    float* loss_dst;
 };
 
 constexpr int TM = 128;          // tile rows (gate-gradient rows)
 constexpr int TN = 64;           // tile cols (input columns)
-constexpr int KS = 16;           // nodes per pipeline stage
+
 constexpr int KCH = 96;          // nodes per work item (split-K)
-constexpr int NST = 3;           // cp.async pipeline stages
 
 // work items of one group: job m = 0 dU_iou, 1 dU_fl, 2 dU_fr, 3 dW_iou (split-K over the group's nodes),
 // 4 leaf dX (split-K over the 3H gate rows)
-__host__ __device__ inline int job_items(int m, int n_int, int n_leaf, int H, int E, bool dx);
 
 // leaf input gradient dX[tok_l] += Σ_r g_l[r] W_iou[r][:] (word vectors are inputs of the
-// leaves).  Tile 64 leaves x 64 columns, split-K over the 3H gate rows in chunks of DXK, 4 x 4 per thread;
-// the leaf gate gradients are staged row-major ([leaf][k], stride 20: conflict-free column reads).
-constexpr int DXM = 64, DXN = 64, DXK = 128, DXS = 20;
+// leaves).  Tile 64 leaves x 64 columns, split-K over the 3H gate rows in chunks of DXK, 4 x 4 per thread.
+// The item stages all of its operands with one batch of cp.async (one L2 round trip): the leaf gate
+// gradients row-major ([leaf][k], stride DXS ≡ 4 mod 32: conflict-free column reads) and DXK rows of W_iou.
+constexpr int DXM = 64, DXN = 64, DXK = 128, DXS = DXK + 4;
+constexpr size_t DW_SMEM = 4 * (size_t)((KCH * TM + KCH * TN) > (DXM * DXS + DXK * DXN) ? (KCH * TM + KCH * TN)
+                                                                                          : (DXM * DXS + DXK * DXN));
 __device__ __forceinline__ void leaf_dx_tile(const GemmParams& P, const uint32_t* leaf_nodes, int n_leaf, int b,
-                                             float* As, float* Bs) {
+                                             float* sm, uint32_t* idx) {
     const int tid = threadIdx.x, H = P.H, E = P.E;
     const int tiles_c = E / DXN, tiles_r = (n_leaf + DXM - 1) / DXM;
     const int kc = b / (tiles_r * tiles_c), t = b - kc * (tiles_r * tiles_c);
     const int r0 = (t / tiles_c) * DXM, c0 = (t % tiles_c) * DXN;
-    const int k0 = kc * DXK, k1 = min(3 * H, k0 + DXK);
+    const int k0 = kc * DXK, nk = min(3 * H, k0 + DXK) - k0;
+    float* As = sm;                      // [DXM][DXS]
+    float* Bs = sm + DXM * DXS;          // [DXK][DXN]
+    if (tid < DXM) {
+        const int row = r0 + tid;
+        idx[2 * tid] = row < n_leaf ? leaf_nodes[2 * row] : 0xFFFFFFFFu;
+        idx[2 * tid + 1] = row < n_leaf ? leaf_nodes[2 * row + 1] : 0u;
+    }
+    __syncthreads();
+    for (int e = tid; e < DXM * (DXK / 4); e += 256) {
+        const int l = e / (DXK / 4), p = (e % (DXK / 4)) * 4;
+        const uint32_t rec = idx[2 * l];
+        const bool ok = rec != 0xFFFFFFFFu && p < nk;
+        cp_async16(As + l * DXS + p, ok ? P.pool + rec + 5 * H + k0 + p : P.pool, ok ? 16u : 0u);
+    }
+    for (int e = tid; e < nk * (DXN / 4); e += 256) {
+        const int k = e / (DXN / 4), p = (e % (DXN / 4)) * 4;
+        cp_async16(Bs + k * DXN + p, P.w_iou + (int64_t)(k0 + k) * E + c0 + p, 16u);
+    }
+    cp_async_wait_all();
+    __syncthreads();
     const int ty = tid / 16, tx = tid % 16;          // leaves r0 + ty + 16a, columns c0 + 4tx .. +3
     float2 acc2[4][2];
 #pragma unroll
     for (int a = 0; a < 4; ++a) acc2[a][0] = acc2[a][1] = make_float2(0.f, 0.f);
-    auto stage = [&](int s, int buf) {
-        {
-            const int l = tid / 4, piece = (tid % 4) * 4, row = r0 + l;
-            const float* src = row < n_leaf ? P.pool + leaf_nodes[2 * row] + 5 * H + k0 + s * KS + piece : nullptr;
-            cp_async16(As + buf * DXM * DXS + l * DXS + piece, src ? src : P.pool, src ? 16u : 0u);
-        }
-        {
-            const int k = tid / 16, piece = (tid % 16) * 4;
-            cp_async16(Bs + buf * KS * TN + k * TN + piece, P.w_iou + (int64_t)(k0 + s * KS + k) * E + c0 + piece, 16u);
-        }
-        asm volatile("cp.async.commit_group;" ::: "memory");
-    };
-    const int steps = (k1 - k0) / KS;
-    stage(0, 0);
-    if (steps > 1) stage(1, 1);
-    for (int s = 0; s < steps; ++s) {
-        if (s + 2 < steps) {
-            stage(s + 2, (s + 2) % NST);
-            asm volatile("cp.async.wait_group 2;" ::: "memory");
-        } else if (s + 1 < steps) {
-            asm volatile("cp.async.wait_group 1;" ::: "memory");
-        } else {
-            asm volatile("cp.async.wait_group 0;" ::: "memory");
-        }
-        __syncthreads();
-        const float* A = As + (s % NST) * DXM * DXS;
-        const float* B = Bs + (s % NST) * KS * TN;
+#pragma unroll 4
+    for (int k = 0; k < nk; ++k) {
+        const float4 bv = *reinterpret_cast<const float4*>(Bs + k * DXN + tx * 4);
+        const float2 b01 = make_float2(bv.x, bv.y), b23 = make_float2(bv.z, bv.w);
 #pragma unroll
-        for (int k = 0; k < KS; ++k) {
-            const float4 bv = *reinterpret_cast<const float4*>(B + k * TN + tx * 4);
-            const float2 b01 = make_float2(bv.x, bv.y), b23 = make_float2(bv.z, bv.w);
-#pragma unroll
-            for (int a = 0; a < 4; ++a) {
-                const float av = A[(ty + 16 * a) * DXS + k];
-                const float2 aa = make_float2(av, av);
-                acc2[a][0] = __ffma2_rn(aa, b01, acc2[a][0]);
-                acc2[a][1] = __ffma2_rn(aa, b23, acc2[a][1]);
-            }
+        for (int a = 0; a < 4; ++a) {
+            const float av = As[(ty + 16 * a) * DXS + k];
+            const float2 aa = make_float2(av, av);
+            acc2[a][0] = __ffma2_rn(aa, b01, acc2[a][0]);
+            acc2[a][1] = __ffma2_rn(aa, b23, acc2[a][1]);
         }
-        __syncthreads();
     }
 #pragma unroll
     for (int a = 0; a < 4; ++a) {
-        const int row = r0 + ty + 16 * a;
+        const int l = ty + 16 * a;
         const float v[4] = {acc2[a][0].x, acc2[a][0].y, acc2[a][1].x, acc2[a][1].y};
-        if (row < n_leaf) red_add<4>(P.d_inputs + (int64_t)leaf_nodes[2 * row + 1] * E + c0 + tx * 4, v);
+        if (r0 + l < n_leaf) red_add<4>(P.d_inputs + (int64_t)idx[2 * l + 1] * E + c0 + tx * 4, v);
     }
 }
 
@@ -692,19 +701,15 @@ __host__ __device__ inline int job_items(int m, int n_int, int n_leaf, int H, in
     }
 }
 
-__global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
-    __shared__ __align__(16) float Gs[NST][KS][TM];
-    __shared__ __align__(16) float Xs[NST][KS][TN];
+// One work item of group g: item i -> (job m, local index b).  dW tiles: 128 gate rows x 64 input columns
+// over the item's <= KCH nodes, all operand rows staged by one batch of cp.async after the node record
+// offsets are read once into shared memory; 8 x 4 FFMA2 per thread; partial tile added to grads.
+__device__ __forceinline__ void dw_item(const GemmParams& P, int g, int i, float* sm, uint32_t* idx) {
     const int tid = threadIdx.x, H = P.H, E = P.E;
-    // item -> (group g, job m, local index b)
-    int b = blockIdx.x, q = 0;
-    while (q < P.n_grp && b >= P.items[q]) { b -= P.items[q]; ++q; }
-    if (q == P.n_grp) return;
-    const int g = P.grp[q];
     const int n_int = P.int_off[g + 1] - P.int_off[g], n_leaf = P.leaf_off[g + 1] - P.leaf_off[g];
     const uint32_t* int_nodes = P.int_nodes + 3 * P.int_off[g];
     const uint32_t* leaf_nodes = P.leaf_nodes + 2 * P.leaf_off[g];
-    int m = 0;
+    int m = 0, b = i;
     while (m < 5) {
         const int n = job_items(m, n_int, n_leaf, H, E, P.d_inputs != nullptr);
         if (b < n) break;
@@ -712,98 +717,187 @@ __global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
         ++m;
     }
     if (m == 5) return;
-    // launched early (programmatic dependent launch): wait until every CTA of this group's cluster is done
-    if (P.done) {
-        if (tid == 0) {
-            uint32_t v;
-            while (true) {
-                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(P.done + g) : "memory");
-                if ((int)v >= P.done_target) break;
-                __nanosleep(200);
-            }
-        }
-        __syncthreads();
-    }
-    if (m == 4) { leaf_dx_tile(P, leaf_nodes, n_leaf, b, &Gs[0][0][0], &Xs[0][0][0]); return; }
+    if (m == 4) { leaf_dx_tile(P, leaf_nodes, n_leaf, b, sm, idx); return; }
     const int rows = (m == 0 || m == 3) ? 3 * H : H;
     const int cols = m == 0 ? 2 * H : (m == 3 ? E : H);
     const int K = m == 3 ? n_leaf : n_int;
     const int tiles_r = rows / TM, tiles_c = cols / TN;
     const int kc = b / (tiles_r * tiles_c), t = b - kc * (tiles_r * tiles_c);
     const int r0 = (t / tiles_c) * TM, c0 = (t % tiles_c) * TN;
-    const int k0 = kc * KCH, k1 = min(K, k0 + KCH);
+    const int k0 = kc * KCH, nk = min(K, k0 + KCH) - k0;
     const int goff = m == 0 ? 7 * H : (m == 1 ? 10 * H : (m == 2 ? 11 * H : 5 * H));
+    float* Gs = sm;                      // [KCH][TM]
+    float* Xs = sm + KCH * TM;           // [KCH][TN]
+    // node operands: idx[3k] = g row base, idx[3k+1] / idx[3k+2] = x row bases (left / right or token)
+    if (tid < nk) {
+        const int node = k0 + tid;
+        if (m == 3) {
+            idx[3 * tid] = leaf_nodes[2 * node];
+            idx[3 * tid + 1] = leaf_nodes[2 * node + 1];
+        } else {
+            idx[3 * tid] = int_nodes[3 * node];
+            idx[3 * tid + 1] = int_nodes[3 * node + 1];
+            idx[3 * tid + 2] = int_nodes[3 * node + 2];
+        }
+    }
+    __syncthreads();
+    for (int e = tid; e < nk * (TM / 4); e += 256) {
+        const int k = e / (TM / 4), p = (e % (TM / 4)) * 4;
+        cp_async16(Gs + k * TM + p, P.pool + idx[3 * k] + goff + r0 + p, 16u);
+    }
+    for (int e = tid; e < nk * (TN / 4); e += 256) {
+        const int k = e / (TN / 4), p = (e % (TN / 4)) * 4, c = c0 + p;
+        const float* src;
+        if (m == 3) src = P.inputs + (int64_t)idx[3 * k + 1] * E + c;
+        else if (m == 0) src = c < H ? P.pool + idx[3 * k + 1] + c : P.pool + idx[3 * k + 2] + (c - H);
+        else src = P.pool + idx[3 * k + (m == 1 ? 1 : 2)] + c;
+        cp_async16(Xs + k * TN + p, src, 16u);
+    }
+    cp_async_wait_all();
+    __syncthreads();
     const int ty = tid / 16, tx = tid % 16;        // rows ty*8 .. +7, cols tx*4 .. +3
     float2 acc[8][2];
 #pragma unroll
     for (int a = 0; a < 8; ++a) acc[a][0] = acc[a][1] = make_float2(0.f, 0.f);
-    // stage: KS nodes x 128 rows of g (2 x 16 B per thread) and KS nodes x 64 cols of x (16 B per thread)
-    auto stage = [&](int s, int buf) {
+#pragma unroll 4
+    for (int k = 0; k < nk; ++k) {
+        const float4 g0 = *reinterpret_cast<const float4*>(Gs + k * TM + ty * 8);
+        const float4 g1 = *reinterpret_cast<const float4*>(Gs + k * TM + ty * 8 + 4);
+        const float4 xv = *reinterpret_cast<const float4*>(Xs + k * TN + tx * 4);
+        const float ga[8] = {g0.x, g0.y, g0.z, g0.w, g1.x, g1.y, g1.z, g1.w};
+        const float2 x01 = make_float2(xv.x, xv.y), x23 = make_float2(xv.z, xv.w);
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
-            const int e = tid + h * 256, k = e / 32, piece = (e % 32) * 4;
-            const int node = k0 + s * KS + k;
-            const float* src = nullptr;
-            if (node < k1) {
-                const uint32_t rec = m == 3 ? leaf_nodes[2 * node] : int_nodes[3 * node];
-                src = P.pool + rec + goff + r0 + piece;
-            }
-            cp_async16(&Gs[buf][k][piece], src ? src : P.pool, src ? 16u : 0u);
+        for (int a = 0; a < 8; ++a) {
+            const float2 gg = make_float2(ga[a], ga[a]);
+            acc[a][0] = __ffma2_rn(gg, x01, acc[a][0]);
+            acc[a][1] = __ffma2_rn(gg, x23, acc[a][1]);
         }
-        {
-            const int k = tid / 16, piece = (tid % 16) * 4;
-            const int node = k0 + s * KS + k;
-            const float* src = nullptr;
-            if (node < k1) {
-                const int c = c0 + piece;
-                if (m == 3) {
-                    src = P.inputs + (int64_t)leaf_nodes[2 * node + 1] * E + c;
-                } else {
-                    const uint32_t xl = int_nodes[3 * node + 1], xr = int_nodes[3 * node + 2];
-                    if (m == 0) src = c < H ? P.pool + xl + c : P.pool + xr + (c - H);
-                    else src = P.pool + (m == 1 ? xl : xr) + c;
-                }
-            }
-            cp_async16(&Xs[buf][k][piece], src ? src : P.pool, src ? 16u : 0u);
-        }
-        asm volatile("cp.async.commit_group;" ::: "memory");
-    };
-    const int steps = (k1 - k0 + KS - 1) / KS;
-    if (steps <= 0) return;
-    stage(0, 0);
-    if (steps > 1) stage(1, 1);
-    for (int s = 0; s < steps; ++s) {
-        if (s + 2 < steps) {
-            stage(s + 2, (s + 2) % NST);
-            asm volatile("cp.async.wait_group 2;" ::: "memory");
-        } else if (s + 1 < steps) {
-            asm volatile("cp.async.wait_group 1;" ::: "memory");
-        } else {
-            asm volatile("cp.async.wait_group 0;" ::: "memory");
-        }
-        __syncthreads();
-        const int buf = s % NST;
-#pragma unroll
-        for (int k = 0; k < KS; ++k) {
-            const float4 g0 = *reinterpret_cast<const float4*>(&Gs[buf][k][ty * 8]);
-            const float4 g1 = *reinterpret_cast<const float4*>(&Gs[buf][k][ty * 8 + 4]);
-            const float4 xv = *reinterpret_cast<const float4*>(&Xs[buf][k][tx * 4]);
-            const float ga[8] = {g0.x, g0.y, g0.z, g0.w, g1.x, g1.y, g1.z, g1.w};
-            const float2 x01 = make_float2(xv.x, xv.y), x23 = make_float2(xv.z, xv.w);
-#pragma unroll
-            for (int a = 0; a < 8; ++a) {
-                const float2 gg = make_float2(ga[a], ga[a]);
-                acc[a][0] = __ffma2_rn(gg, x01, acc[a][0]);
-                acc[a][1] = __ffma2_rn(gg, x23, acc[a][1]);
-            }
-        }
-        __syncthreads();
     }
     float* base = P.grads + P.off[m == 3 ? 0 : m + 1];
 #pragma unroll
     for (int a = 0; a < 8; ++a) {
         const float v[4] = {acc[a][0].x, acc[a][0].y, acc[a][1].x, acc[a][1].y};
+#ifdef VPPS_EXP_STORE
+        *reinterpret_cast<float4*>(base + (int64_t)(r0 + ty * 8 + a) * cols + c0 + tx * 4) = make_float4(v[0], v[1], v[2], v[3]);
+#else
         red_add<4>(base + (int64_t)(r0 + ty * 8 + a) * cols + c0 + tx * 4, v);
+#endif
+    }
+}
+
+// Persistent CTAs claim work items only from groups whose CTAs have all counted themselves done (no CTA
+// ever sits on an SM waiting for a group that is still running); groups are scanned in the host's order.
+// Without counters (P.done == nullptr) item = blockIdx.x over the groups in order.
+__global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
+    extern __shared__ __align__(16) float dsm[];
+    __shared__ uint32_t idx[3 * KCH];
+    __shared__ int pick[3];
+    const int tid = threadIdx.x;
+    if (!P.done || P.static_items) {
+        // one item per CTA in the host's group order; with counters, wait for the item's group first
+        int b = blockIdx.x;
+        for (int q = 0; q < P.n_grp; ++q) {
+            const int g = P.grp[q];
+            if (b < P.items[g]) {
+                if (P.done) {
+                    if (tid == 0) {
+                        uint32_t v;
+                        while (true) {
+                            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(P.done + g) : "memory");
+                            if ((int)v >= P.done_target) break;
+                            __nanosleep(200);
+                        }
+                    }
+                    __syncthreads();
+                }
+                dw_item(P, g, b, dsm, idx);
+                return;
+            }
+            b -= P.items[g];
+        }
+        return;
+    }
+    while (true) {
+        if (tid < 32) {
+            // lane q looks at group grp[q] (all groups in one parallel round trip); the first eligible
+            // group in order is claimed, retrying further groups if its items ran out meanwhile
+            const int lane = tid;
+            const int g = lane < P.n_grp ? P.grp[lane] : -1;
+            uint32_t c = 0, d = 0;
+            if (g >= 0) {
+                asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(c) : "l"(P.claim + g) : "memory");
+                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(d) : "l"(P.done + g) : "memory");
+            }
+            const bool left = g >= 0 && (int)c < P.items[g];
+            unsigned ready = __ballot_sync(FULLMASK, left && (int)d >= P.done_target);
+            int got_g = -1, got_i = -1;
+            while (ready && got_g < 0) {
+                const int q = __ffs(ready) - 1;
+                int i = 0;
+                if (lane == q) i = atomicAdd(P.claim + g, 1);
+                i = __shfl_sync(FULLMASK, i, q);
+                const int gq = __shfl_sync(FULLMASK, g, q);
+                if (i < P.items[gq]) { got_g = gq; got_i = i; }
+                ready &= ready - 1;
+            }
+            const unsigned any_left = __ballot_sync(FULLMASK, left);
+            if (lane == 0) { pick[0] = got_g; pick[1] = got_i; pick[2] = any_left != 0; }
+        }
+        __syncthreads();
+        const int g = pick[0], i = pick[1], rem = pick[2];
+        __syncthreads();
+        if (g >= 0) {
+            const uint64_t t0 = P.trace ? gtimer() : 0;
+            dw_item(P, g, i, dsm, idx);
+            __threadfence();
+            __syncthreads();
+            if (tid == 0) atomicAdd(P.fin, 1);
+            if (P.trace && tid == 0) {
+                int k = 0;
+                for (int q = 0; q < g; ++q) k += P.items[q];
+                uint64_t* o = P.trace + 5 * (k + i);
+                uint32_t smid;
+                asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+                o[0] = (uint64_t)g; o[1] = (uint64_t)i; o[2] = t0; o[3] = gtimer(); o[4] = smid;
+            }
+            continue;
+        }
+        if (!rem) break;
+        __nanosleep(500);
+    }
+    // ---- fused tail: SGD over the flat parameters (L129, L197) and the loss read-back (L199) ----
+    if (tid == 0) {
+        uint32_t f;
+        while (true) {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(f) : "l"(P.fin) : "memory");
+            if ((int)f >= P.total_items) break;
+            __nanosleep(200);
+        }
+    }
+    __syncthreads();
+    constexpr int64_t CH = 16384;                          // floats per claimed chunk
+    const int64_t n_chunks = P.mode == 1 ? (P.n_floats + CH - 1) / CH : 0;
+    while (true) {
+        if (tid == 0) pick[0] = atomicAdd(P.tail_claim, 1);
+        __syncthreads();
+        const int64_t c = pick[0];
+        __syncthreads();
+        if (c == 0 && P.loss_dst && tid == 0) {
+            const float l = *reinterpret_cast<const volatile float*>(P.loss_src);
+            *reinterpret_cast<volatile float*>(P.loss_dst) = l;
+        }
+        if (c >= n_chunks) break;
+        const int64_t lo = c * CH, hi = min(P.n_floats, lo + CH);
+        float4* p4 = reinterpret_cast<float4*>(P.params + lo);
+        const float4* g4 = reinterpret_cast<const float4*>(P.grads + lo);
+        const float lr = P.lr, wd = P.wd;
+        for (int64_t k = tid; k < (hi - lo) / 4; k += 256) {
+            float4 a = p4[k];
+            const float4 b = g4[k];
+            a.x -= lr * (b.x + wd * a.x); a.y -= lr * (b.y + wd * a.y);
+            a.z -= lr * (b.z + wd * a.z); a.w -= lr * (b.w + wd * a.w);
+            p4[k] = a;
+        }
     }
 }
 
@@ -824,11 +918,12 @@ const Variant* cluster_variants(int32_t* n) {
 
 void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, float* params, float* grads,
                     const uint32_t* int_nodes, const uint32_t* leaf_nodes, int32_t n_grp, const int32_t* int_off,
-                    const int32_t* leaf_off, const int32_t* order, const int32_t* done, int32_t done_target,
+                    const int32_t* leaf_off, const int32_t* order, int32_t* done, int32_t done_target,
                     bool early, int32_t H, int32_t E, const int64_t* off, int64_t n_floats, int32_t mode, float lr,
-                    float wd, cudaStream_t s) {
+                    float wd, cudaStream_t s, uint64_t* trace, const float* loss_src, float* loss_dst) {
     using namespace dev::cl;
     GemmParams g{};
+    g.trace = trace;
     g.pool = pool; g.inputs = inputs; g.grads = grads;
     g.int_nodes = int_nodes; g.leaf_nodes = leaf_nodes;
     g.H = H; g.E = E;
@@ -836,6 +931,16 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, flo
     g.w_iou = params + off[0];
     g.d_inputs = d_inputs;
     g.done = done;
+    g.claim = done ? done + 16 : nullptr;
+    g.fin = done ? done + 32 : nullptr;
+    g.tail_claim = done ? done + 33 : nullptr;
+    g.mode = mode;
+    g.params = params;
+    g.n_floats = n_floats;
+    g.lr = lr;
+    g.wd = wd;
+    g.loss_src = loss_src;
+    g.loss_dst = loss_dst;
     g.done_target = done_target;
     g.n_grp = n_grp;
     int items = 0;
@@ -845,23 +950,35 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, flo
         const int ni = int_off[gi + 1] - int_off[gi], nl = leaf_off[gi + 1] - leaf_off[gi];
         int n = 0;
         for (int m = 0; m < 5; ++m) n += job_items(m, ni, nl, H, E, d_inputs != nullptr);
-        g.items[q] = n;
+        g.items[gi] = n;
         items += n;
     }
     for (int i = 0; i <= n_grp; ++i) { g.int_off[i] = int_off[i]; g.leaf_off[i] = leaf_off[i]; }
+    g.total_items = items;
+    static const int stat = getenv("VPPS_DW_STATIC") ? atoi(getenv("VPPS_DW_STATIC")) : 0;   // TEMP A/B
+    const bool fused_tail = done && !stat && items > 0 && (n_floats % 4) == 0;
     if (items > 0) {
         cudaLaunchConfig_t cfg = {};
         cudaLaunchAttribute attr[1];
         attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
         attr[0].val.programmaticStreamSerializationAllowed = 1;
-        cfg.gridDim = dim3(items);
+        g.static_items = stat;
+        cfg.gridDim = dim3(done && !stat ? std::min(items, 148 * 3) : items);   // persistent when claiming
         cfg.blockDim = dim3(256);
+        cfg.dynamicSmemBytes = DW_SMEM;
+        static bool attr_set = false;
+        if (!attr_set) {
+            cudaFuncSetAttribute(vpps_dw_gemm, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DW_SMEM);
+            attr_set = true;
+        }
         cfg.stream = s;
         cfg.attrs = attr;
         cfg.numAttrs = early ? 1 : 0;
         cudaLaunchKernelEx(&cfg, vpps_dw_gemm, g);
     }
+    if (fused_tail) return;                                            // SGD + loss inside the kernel
     if (mode == 1) launch_sgd(params, grads, n_floats, lr, wd, s);   // W -= lr (dW + wd W), every parameter
+    if (loss_dst) cudaMemcpyAsync(loss_dst, loss_src, sizeof(float), cudaMemcpyDeviceToDevice, s);
 }
 
 }  // namespace vpps

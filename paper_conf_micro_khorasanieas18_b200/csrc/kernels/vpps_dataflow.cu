@@ -98,7 +98,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     const int grp = blockIdx.x / NCL, lc = blockIdx.x % NCL;
     float* pool = P.pool;
     const int64_t* off = P.off;
-    const uint32_t ep = P.epoch;
+    uint32_t ep = 0;
     u64* HX = reinterpret_cast<u64*>(pool + P.df_hx);
     u64* PART = reinterpret_cast<u64*>(pool + P.df_part);
     u64* HD = reinterpret_cast<u64*>(pool + P.df_hd);
@@ -157,8 +157,9 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             sec_last = now;
         }
     };
-    // the leaf records (vpps_leaf_fwd, the preceding grid) are complete and visible from here on
+    // the leaf records and the pass counter (vpps_leaf_fwd, the preceding grid) are visible from here on
     asm volatile("griddepcontrol.wait;" ::: "memory");
+    ep = *P.epoch;
     __syncthreads();
     if (prof && tid == 0) { prof[0] = gtimer(); sec_last = clock64(); }
 

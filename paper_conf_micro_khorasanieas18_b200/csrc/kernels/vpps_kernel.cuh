@@ -31,7 +31,7 @@ struct DfParams {
     int64_t df_off;
     int64_t off[8];
     int32_t C;
-    uint32_t epoch;             // pass counter (>= 1): tag of every slot written by this pass
+    const uint32_t* epoch;      // device pass counter (advanced by the leaf kernel): tag of this pass's slots
     int64_t loss_word;
     int64_t df_hx, df_part, df_hd;   // word offsets of the tagged regions in the pool
     uint64_t* prof;
@@ -54,16 +54,23 @@ const Variant* df_variants(int32_t* n);
 // dW = Σ g xᵀ per weight matrix from the recorded operands, fused SGD when mode == 1.
 // Also forms the leaf input gradient dX[tok] += W_iouᵀ g_leaf when d_inputs is not null.  Node lists are
 // grouped by replica group (offsets int_off / leaf_off, n_grp + 1 entries); with `early` the kernel is a
-// programmatic dependent launch of vpps_cl and each group's tiles wait for done[group] >= done_target.
+// programmatic dependent launch of vpps_cl / vpps_df; persistent CTAs claim a group's tiles (counters
+// done[16 + group], zeroed per pass) once done[group] >= done_target.
 void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, float* params, float* grads,
                     const uint32_t* int_nodes, const uint32_t* leaf_nodes, int32_t n_grp, const int32_t* int_off,
-                    const int32_t* leaf_off, const int32_t* order, const int32_t* done, int32_t done_target,
+                    const int32_t* leaf_off, const int32_t* order, int32_t* done, int32_t done_target,
                     bool early, int32_t H, int32_t E, const int64_t* off, int64_t n_floats, int32_t mode, float lr,
-                    float wd, cudaStream_t s);
+                    float wd, cudaStream_t s, uint64_t* trace = nullptr, const float* loss_src = nullptr,
+                    float* loss_dst = nullptr);
+// (with completion counters the kernel also applies the SGD update and copies *loss_src to loss_dst, a
+//  device-visible pointer to mapped host memory, after the last item; otherwise separate launches do)
 // Leaf level of the binary cell as one GEMM + fused cell (vpps_leaf.cu): records h, c, i, o, u of every
 // leaf before the cluster kernel.
+// It also zeroes up to 4 float ranges (zero_ptr[r], zero_n[r] floats, multiples of 4; nullptr = unused)
+// and advances the device pass counter `epoch` (if not null): the per-pass clearing without memset calls.
 void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float* pool, const uint32_t* leaves,
-                     int32_t n_leaf, int32_t H, int32_t E, cudaStream_t s);
+                     int32_t n_leaf, int32_t H, int32_t E, float* const* zero_ptr, const int64_t* zero_n,
+                     uint32_t* epoch, cudaStream_t s);
 // Elementwise SGD on the flat buffer (K3): p -= lr * (g + wd * p).
 void launch_sgd(float* p, const float* g, int64_t n, float lr, float wd, cudaStream_t s);
 

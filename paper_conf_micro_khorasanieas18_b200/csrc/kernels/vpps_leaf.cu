@@ -14,6 +14,7 @@
 // of 32; each thread owns 4 leaves x 2 units x 3 gates and reads 16-byte K slices.
 // The input-table gradient dX = W_iouᵀ g_leaf is a job of the gradient GEMM (vpps_dw_gemm, vpps_cluster.cu).
 // Requires E <= KMAX and H % 32 == 0 (the cluster variants are H = E = 256).
+#include <algorithm>
 #include "vpps_kernel.cuh"
 #include "dev_common.cuh"
 
@@ -28,19 +29,40 @@ constexpr int KMAX = 256;       // E <= KMAX: the whole K range is staged at onc
 constexpr int KS = KMAX + 4;    // row stride in floats (≡ 4 mod 32: conflict-free 16-byte column reads)
 constexpr size_t SMEM = (size_t)(LM + 3 * LU) * KS * sizeof(float);
 
+// Per-pass clearing folded into the leaf kernel (it runs first in the pass): up to 4 float ranges
+// (multiples of 4 floats) are zeroed by a grid-stride loop, and the device pass counter is advanced.
+struct PassClear {
+    float* ptr[4];
+    int64_t n[4];
+    uint32_t* epoch;     // dataflow pass counter (tags of this pass), or nullptr
+};
+
 template <int E>
 __global__ void __launch_bounds__(NT, 3) vpps_leaf_fwd(const float* __restrict__ W, const float* __restrict__ b,
                                                        const float* __restrict__ inputs, float* pool,
-                                                       const uint32_t* __restrict__ leaves, int n_leaf, int H) {
+                                                       const uint32_t* __restrict__ leaves, int n_leaf, int H,
+                                                       const PassClear pc) {
     static_assert(E <= KMAX && E % 16 == 0, "leaf GEMM: E <= 256");
     extern __shared__ __align__(16) float lsm[];
     __shared__ uint32_t lrec[LM], ltok[LM];
     float* As = lsm;                 // [16 leaves][KS]: x rows
     float* Bs = lsm + LM * KS;       // [48 rows][KS]: W_iou rows g*H + j0 + uu, row index g*16 + uu
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");   // vpps_cl may start its weight prologue
     const int tid = threadIdx.x;
+    if (pc.epoch && blockIdx.x == 0 && tid == 0) {
+        uint32_t e = *pc.epoch + 1;
+        *pc.epoch = e ? e : 1u;                                   // 0 marks never-written slots
+    }
+    {
+        const int64_t stride = (int64_t)gridDim.x * NT;
+        for (int r = 0; r < 4; ++r) {
+            float4* p = reinterpret_cast<float4*>(pc.ptr[r]);
+            const int64_t n4 = pc.ptr[r] ? pc.n[r] / 4 : 0;
+            for (int64_t i = (int64_t)blockIdx.x * NT + tid; i < n4; i += stride) p[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+    }
     const int tiles_u = H / LU;
     const int l0 = (blockIdx.x / tiles_u) * LM, j0 = (blockIdx.x % tiles_u) * LU;
+    if (l0 >= n_leaf) return;                                      // clearing-only CTA
     if (tid < LM) {
         const int l = l0 + tid;
         lrec[tid] = l < n_leaf ? leaves[2 * l] : 0u;
@@ -126,16 +148,20 @@ __global__ void __launch_bounds__(NT, 3) vpps_leaf_fwd(const float* __restrict__
 }  // namespace dev
 
 void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float* pool, const uint32_t* leaves,
-                     int32_t n_leaf, int32_t H, int32_t E, cudaStream_t s) {
+                     int32_t n_leaf, int32_t H, int32_t E, float* const* zero_ptr, const int64_t* zero_n,
+                     uint32_t* epoch, cudaStream_t s) {
     using namespace dev::leaf;
-    if (n_leaf <= 0 || E != 256 || H % LU) return;   // the cluster variants are H = E = 256 (api.cu checks)
+    if (E != 256 || H % LU) return;   // the cluster / dataflow variants are H = E = 256 (api.cu checks)
     static bool attr = false;
     if (!attr) {
         cudaFuncSetAttribute(vpps_leaf_fwd<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
         attr = true;
     }
-    const int tiles = ((n_leaf + LM - 1) / LM) * (H / LU);
-    vpps_leaf_fwd<256><<<tiles, NT, SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H);
+    PassClear pc{};
+    for (int r = 0; r < 4; ++r) { pc.ptr[r] = zero_ptr ? zero_ptr[r] : nullptr; pc.n[r] = zero_ptr ? zero_n[r] : 0; }
+    pc.epoch = epoch;
+    const int tiles = std::max(((n_leaf + LM - 1) / LM) * (H / LU), 148);
+    vpps_leaf_fwd<256><<<tiles, NT, SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
 }
 
 }  // namespace vpps

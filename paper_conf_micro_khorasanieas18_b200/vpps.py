@@ -77,6 +77,7 @@ def _load():
         "vpps_pool_ptr": [VP, P(VP), P(I64)],
         "vpps_set_timing_events": [VP, VP, VP],
         "vpps_set_kernel_events": [VP, VP, VP],
+        "vpps_set_gemm_trace": [VP, VP],
         "vpps_set_profile_buffer": [VP, VP, I64],
         "vpps_destroy_script": [VP],
         "vpps_destroy_model": [VP],
@@ -225,7 +226,7 @@ class Script:
         _check(_lib.vpps_upload_script(self._h, _stream_ptr(stream)))
 
     def __del__(self):
-        if getattr(self, "_h", None):
+        if getattr(self, "_h", None) and _lib is not None:   # _lib is None during interpreter shutdown
             _lib.vpps_destroy_script(self._h)
             self._h = None
 
@@ -320,6 +321,10 @@ class Model:
         _check(_lib.vpps_set_kernel_events(self._h, ct.c_void_p(before.cuda_event) if before else None,
                                            ct.c_void_p(after.cuda_event) if after else None))
 
+    def set_gemm_trace(self, buf=None):
+        """int64 CUDA tensor [items, 5] receiving (group, item, start ns, end ns, smid) per GEMM item."""
+        _check(_lib.vpps_set_gemm_trace(self._h, ct.c_void_p(buf.data_ptr()) if buf is not None else None))
+
     def set_profile_buffer(self, buf=None, stride=0):
         """int64 CUDA tensor [n_cta, stride] receiving the in-kernel globaltimer trace (None clears)."""
         _check(_lib.vpps_set_profile_buffer(self._h, ct.c_void_p(buf.data_ptr()) if buf is not None else None,
@@ -332,6 +337,6 @@ class Model:
         return p.value, n.value
 
     def __del__(self):
-        if getattr(self, "_h", None):
+        if getattr(self, "_h", None) and _lib is not None:
             _lib.vpps_destroy_model(self._h)
             self._h = None

@@ -44,10 +44,14 @@ def main():
     stride = 16 + 5 * 48
     buf = torch.zeros((n_cta, stride), dtype=torch.int64, device="cuda")
     m.set_profile_buffer(buf, stride)
+    gt = torch.zeros((4096, 5), dtype=torch.int64, device="cuda")
+    m.set_gemm_trace(gt)
     for _ in range(args.reps):
         m.fwd_bwd(s, X, dX)
     torch.cuda.synchronize()
     raw = buf.cpu().numpy().astype(np.float64)
+    gtr = gt.cpu().numpy().astype(np.float64)
+    gtr = gtr[gtr[:, 3] > 0]
     t0 = raw[:, 0].min()
     span = (raw[:, 1] - raw[:, 0]) / 1e3
     names = ["program", "staging", "tag-wait", "forward", "cell-bwd", "transp", "heads", "other"]
@@ -57,6 +61,18 @@ def main():
     groups = n_cta // 16
     print("group spans (us): " + ", ".join(f"{(raw[g*16:(g+1)*16, 1].max() - t0) / 1e3:.1f}" for g in range(groups)))
     print("batches per group: " + ", ".join(f"{int(raw[g*16, 2])}" for g in range(groups)))
+    if len(gtr):
+        gend = [(raw[g*16:(g+1)*16, 1].max() - t0) / 1e3 for g in range(groups)]
+        st = (gtr[:, 2] - t0) / 1e3
+        en = (gtr[:, 3] - t0) / 1e3
+        print(f"gradient GEMM: {len(gtr)} items, first start {st.min():.1f} us, last end {en.max():.1f} us, "
+              f"mean item {np.mean(en - st):.2f} us, SMs used {len(set(gtr[:, 4]))}")
+        for g in range(groups):
+            sel = gtr[:, 0] == g
+            if sel.any():
+                print(f"  group {g}: done {gend[g]:.1f} us; its {int(sel.sum())} items run {st[sel].min():.1f}-{en[sel].max():.1f} us")
+        kern_end = (raw[:, 1].max() - t0) / 1e3
+        print(f"  items finished before the last group ended: {(en <= kern_end).mean()*100:.0f} %")
     mean = secs.mean(0)
     slow = secs[np.argmax(raw[:, 1])]
     tot = mean.sum()

@@ -54,6 +54,23 @@ def main():
                 flush.zero_()
             m.fwd_bwd_sgd(scripts[i % 16], X, dX, lr=1e-3, weight_decay=0.0)
         torch.cuda.synchronize()
+    # timeline of the last few steps: kernel start / end relative to the step's first kernel (us)
+    evs = sorted([e for e in prof.events() if e.device_type == torch.autograd.DeviceType.CUDA],
+                 key=lambda e: e.time_range.start)
+    steps, cur = [], []
+    for e in evs:
+        if "leaf_fwd" in e.name and cur:
+            steps.append(cur)
+            cur = []
+        if "FillFunc" not in e.name:
+            cur.append(e)
+    if cur:
+        steps.append(cur)
+    for st in steps[-3:]:
+        t0 = st[0].time_range.start
+        print("step timeline (us): " + "; ".join(
+            f"{e.name.split('(')[0].split('::')[-1][:18]} {e.time_range.start - t0:.1f}-{e.time_range.end - t0:.1f}"
+            for e in st))
     per = collections.defaultdict(list)
     for e in prof.events():
         if e.device_type == torch.autograd.DeviceType.CUDA:
