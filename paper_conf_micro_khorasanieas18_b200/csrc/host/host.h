@@ -16,7 +16,7 @@ enum Op : uint32_t {
     OP_LSTM_F = 0x10, OP_LSTM_B = 0x11,
     OP_LEAF_F = 0x20, OP_LEAF_B = 0x21, OP_INT_F = 0x22, OP_INT_B = 0x23,
     OP_CS_F = 0x30, OP_CS_B = 0x31,
-    OP_HEAD_F = 0x40, OP_HEAD_B = 0x41,
+    OP_HEAD_F = 0x40, OP_HEAD_B = 0x41, OP_HEAD_FB = 0x42,   // HEAD_FB: dataflow program only
 };
 
 struct Shape { int32_t rows, cols; };

@@ -364,8 +364,9 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
         };
         std::vector<std::vector<uint32_t>> prog(G);
         auto emit_batches = [&](int32_t g, uint32_t op, const std::vector<int64_t>& list) {
-            for (size_t b0 = 0; b0 < list.size(); b0 += 16) {
-                const size_t nb = std::min<size_t>(16, list.size() - b0);
+            const size_t cap = op == OP_LEAF_B ? 64 : 16;   // leaf backward needs no shared staging
+            for (size_t b0 = 0; b0 < list.size(); b0 += cap) {
+                const size_t nb = std::min<size_t>(cap, list.size() - b0);
                 std::vector<uint32_t>& w = prog[g];
                 w.push_back(op | (uint32_t)(nb << 8));
                 for (size_t k = b0; k < b0 + nb; ++k) {
@@ -375,11 +376,8 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
                         case OP_INT_F:
                             w.insert(w.end(), {rec[i], hx[i], rec[ch[0]], hx[ch[0]], rec[ch[1]], hx[ch[1]]});
                             break;
-                        case OP_HEAD_F:
-                            w.insert(w.end(), {rec[i], rec[ch[0]], (uint32_t)nodes[i].label, hx[ch[0]]});
-                            break;
-                        case OP_HEAD_B:
-                            w.insert(w.end(), {rec[i], rec[ch[0]], (uint32_t)nodes[i].label, hd[ch[0]], hx[ch[0]]});
+                        case OP_HEAD_FB:
+                            w.insert(w.end(), {rec[i], rec[ch[0]], (uint32_t)nodes[i].label, hx[ch[0]], hd[ch[0]]});
                             break;
                         case OP_INT_B:
                             w.insert(w.end(), {rec[i], adj[i], dsrc(i), hd[i], pp[i], rec[ch[0]], adj[ch[0]],
@@ -401,17 +399,15 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
                     else if (nodes[i].kind == K_HEAD) lists[1].push_back(i);
                 }
                 emit_batches(g, OP_INT_F, lists[0]);
-                emit_batches(g, OP_HEAD_F, lists[1]);
+                emit_batches(g, OP_HEAD_FB, lists[1]);   // head forward + backward (dz needs only p)
             }
             for (int32_t lv = L; lv >= 0; --lv) {
                 for (auto& l : lists) l.clear();
                 for (int64_t i : at_level[lv]) {
                     if (graph_group[nodes[i].graph] != g) continue;
-                    if (nodes[i].kind == K_HEAD) lists[2].push_back(i);
-                    else if (nodes[i].kind == K_INT) lists[3].push_back(i);
+                    if (nodes[i].kind == K_INT) lists[3].push_back(i);
                     else if (nodes[i].kind == K_LEAF) lists[4].push_back(i);
                 }
-                emit_batches(g, OP_HEAD_B, lists[2]);
                 emit_batches(g, OP_INT_B, lists[3]);
                 emit_batches(g, OP_LEAF_B, lists[4]);
             }

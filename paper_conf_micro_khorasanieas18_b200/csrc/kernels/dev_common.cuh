@@ -8,6 +8,11 @@ namespace dev {
 constexpr uint32_t FULLMASK = 0xFFFFFFFFu;
 
 __device__ __forceinline__ float sigm(float x) { return 1.0f / (1.0f + expf(-x)); }
+// Latency-short forms for the critical path of the dataflow / leaf kernels: MUFU.EX2-based exp and the
+// approximate divide (a few ulp; the parity bar is 1e-4 relative, SURVEY R-22).  tanh x = 1 - 2/(1+e^{2x})
+// saturates correctly at both ends (e^{2x} -> inf gives 1, -> 0 gives -1).
+__device__ __forceinline__ float fsigm(float x) { return __fdividef(1.0f, 1.0f + __expf(-x)); }
+__device__ __forceinline__ float ftanh(float x) { return 1.0f - __fdividef(2.0f, 1.0f + __expf(2.0f * x)); }
 __device__ __forceinline__ float4 ld4cg(const float* p) { return __ldcg(reinterpret_cast<const float4*>(p)); }
 __device__ __forceinline__ float4 f4zero() { return make_float4(0.f, 0.f, 0.f, 0.f); }
 

@@ -973,7 +973,8 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, flo
         }
         cfg.stream = s;
         cfg.attrs = attr;
-        cfg.numAttrs = early ? 1 : 0;
+        static const bool no_pdl = getenv("VPPS_DW_NOPDL") != nullptr;   // measurement only: no overlap
+        cfg.numAttrs = early && !no_pdl ? 1 : 0;
         cudaLaunchKernelEx(&cfg, vpps_dw_gemm, g);
     }
     if (fused_tail) return;                                            // SGD + loss inside the kernel

@@ -25,19 +25,23 @@ namespace df {
 constexpr int NTH = 256;
 constexpr int NCL = 16;        // CTAs per group
 constexpr int CHUNK = 4096;    // program words staged in shared memory
-constexpr int NB = 16;         // nodes per batch
+constexpr int NB = 16;         // nodes per batch (LEAF_B: up to NBL)
+constexpr int NBL = 64;        // leaves per LEAF_B batch (no shared staging: one (unit, leaf) pair per thread pass)
+constexpr int MAXB = 1 + (NB * 9 > NBL * 4 ? NB * 9 : NBL * 4);   // words of the largest batch
 constexpr int NC = 2;          // nodes per transposed-product chunk
 constexpr int ZC = 32;         // classes per head (C <= 32)
 constexpr int CINMAX = 10;
 constexpr uint32_t NONE = 0xFFFFFFFFu;
-enum : uint32_t { LEAF_B = 0x21, INT_F = 0x22, INT_B = 0x23, HEAD_F = 0x40, HEAD_B = 0x41 };
+// HEAD_FB: the loss head's forward and backward in one batch (L42: softmax-NLL; dz = p - onehot needs
+// nothing but the head's own forward), emitted at the labelled cell's forward level
+enum : uint32_t { LEAF_B = 0x21, INT_F = 0x22, INT_B = 0x23, HEAD_FB = 0x42 };
 
 __device__ __forceinline__ int entry_words(uint32_t op) {
     switch (op) {
         case INT_F: return 6;    // rec, hx, rec_l, hx_l, rec_r, hx_r
         case INT_B: return 9;    // rec, adj, dsrc, hd, pp, rec_l, adj_l, rec_r, adj_r
-        case HEAD_B: return 5;   // rec, rec_c, label, hd_c, hx_c
-        default: return 4;       // HEAD_F: rec, rec_c, label, hx_c | LEAF_B: rec, adj, dsrc, hd
+        case HEAD_FB: return 5;  // rec, rec_c, label, hx_c, hd_c
+        default: return 4;       // LEAF_B: rec, adj, dsrc, hd
     }
 }
 
@@ -46,10 +50,12 @@ __device__ __forceinline__ u64 tagv(float v, uint32_t e) { return ((u64)e << 32)
 __device__ __forceinline__ void st_tag(u64* p, float v, uint32_t e) {
     asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(tagv(v, e)) : "memory");
 }
-// L1-bypassing poll of one slot (relaxed, gpu scope: always observes the L2 copy)
+// L1-bypassing poll of one slot: an L2-cached (.cg) 8-byte load of an aligned slot that producers write
+// with one 8-byte store, so value and epoch arrive together.  (Strong ld.relaxed.gpu loads issue one at
+// a time: 17 of them took ~3.6K cycles where these pipeline like ordinary loads.)
 __device__ __forceinline__ u64 ld_slot(const u64* p) {
     u64 v;
-    asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    asm volatile("ld.global.cg.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
 __device__ __forceinline__ void st_tag4(u64* p, const float* v, uint32_t e) {
@@ -64,6 +70,9 @@ struct DCfg {
     static_assert(H % NCL == 0 && TU == 16, "dataflow kernel: 16 units per CTA, 16 threads per unit");
     using LB = Lay<2 * H, TU>;                     // internal bundle rows (i, o, u of U_iou; f) over [h_l; h_r]
     static constexpr int KP = LB::KP;              // 2H
+    // column granule t of a thread covers h_l iff t < TH, for every thread of the unit (compile-time split)
+    static constexpr int TH = H / (LB::CG * TU);
+    static_assert(H % (LB::CG * TU) == 0, "h_l / h_r boundary on a granule-round boundary");
     static constexpr int O_X = CHUNK;                               // xs [NB][KP] floats
     static constexpr int O_DXB = O_X + NB * KP;                     // dxb [UM][NC][KP] floats / u64 scratch
     static constexpr int O_CIN = O_DXB + UM * NC * KP;
@@ -133,7 +142,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         for (int i = tid; i < C * H; i += NTH) { Wo[i] = __ldg(P.params + off[4] + i); dWo[i] = 0.f; }
         for (int i = tid; i < C; i += NTH) { bo[i] = __ldg(P.params + off[7] + i); dbo[i] = 0.f; }
     }
-    float dbacc[4] = {0.f, 0.f, 0.f, 0.f};
+    float dbacc[4] = {0.f, 0.f, 0.f, 0.f};   // bias gradients of unit j (thread (u, gl) mapping)
+    float dbleaf[3] = {0.f, 0.f, 0.f};       // ... of unit lc * UM + tid % UM (LEAF_B mapping)
     uint64_t* prof = P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
     // section clocks (trace only): 0 program, 1 staging, 2 tag wait, 3 forward, 4 cell-bwd, 5 transposed,
     // 6 heads, 7 other
@@ -177,8 +187,9 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     if (s0 < s1) refill(s0);
     uint32_t pos = s0;
     int nbatch = 0;
+    int xdone = 0;            // fine stamps taken (trace only)
     while (pos < s1) {
-        if (pos + 1 + NB * 9 > cbase + CHUNK && cbase + CHUNK < s1) refill(pos);
+        if (pos + MAXB > cbase + CHUNK && cbase + CHUNK < s1) refill(pos);
         mark(0);
         const uint32_t hdr = chunk[pos - cbase];
         const uint32_t op = hdr & 0xFF;
@@ -186,13 +197,71 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         const int sz = entry_words(op);
         const uint32_t* ent = chunk + (pos - cbase) + 1;
         const uint32_t next = pos + 1 + nb * sz;
-        const bool is_head = (op == HEAD_F || op == HEAD_B);
+        const bool is_head = op == HEAD_FB;
         if (is_head && !holds_head) { pos = next; continue; }
         ++nbatch;
         uint64_t* bt = (prof && tid == 0 && nbatch <= 48 && P.prof_stride >= 16 + 5 * 48) ? prof + 16 + 5 * (nbatch - 1) : nullptr;
         if (bt) { bt[0] = clock64(); bt[4] = op; }
         int rounds = 0;
+        // fine stamps (trace only, tid 0, first single-node batch of each kind): prof[256 + k]
+        uint64_t* xst = (prof && tid == 0 && P.prof_stride >= 288) ? prof + 256 : nullptr;
+        const bool stF = xst && op == INT_F && nb == 1 && !(xdone & 1);
+        const bool stB = xst && op == INT_B && nb == 1 && !(xdone & 2);
+        const bool stL = xst && op == LEAF_B && !(xdone & 4);
+        xdone |= (stF ? 1 : 0) | (stB ? 2 : 0) | (stL ? 4 : 0);
+        XST(stF, 16);
+        XST(stB, 22);
+#define XST(f, k) do { if (f) xst[k] = clock64(); } while (0)
         mark(1);
+        if (op == LEAF_B) {
+            // leaf backward, thread (leaf tid / U + 16 p, unit tid % U): consecutive threads read consecutive
+            // units of the same slot row (coalesced), own operands and the 17 dh slots straight into
+            // registers, cell backward, gate gradients to the record for the W_iou / dX GEMM (L185)
+            const int uu = tid % UM, jj = lc * UM + uu;
+            for (int n = tid / UM; n < nb; n += NTH / UM) {
+                const uint32_t* e = ent + n * sz;
+                const uint32_t rec = e[0], dsrc = e[2], hd = e[3];
+                const float dc = __ldcg(pool + e[1] + H + jj), c = __ldcg(pool + rec + H + jj);
+                const float i = __ldcg(pool + rec + 2 * H + jj), o = __ldcg(pool + rec + 3 * H + jj);
+                const float uv = __ldcg(pool + rec + 4 * H + jj);
+                const u64* psrc = dsrc != NONE ? PART + ((((int64_t)(dsrc >> 1) * NCL + lc) * NCL) * 2 + (dsrc & 1)) * UM + uu : nullptr;
+                const u64* hsrc = hd != NONE ? HD + (int64_t)hd * H + jj : nullptr;
+                const u64 none = (u64)ep << 32;
+                u64 v[NCL + 1];
+#pragma unroll
+                for (int k = 0; k < NCL; ++k) v[k] = psrc ? ld_slot(psrc + k * 2 * UM) : none;
+                v[NCL] = hsrc ? ld_slot(hsrc) : none;
+                XST(stL && n == tid / UM, 12);
+                while (true) {
+                    bool stale = false;
+#pragma unroll
+                    for (int k = 0; k < NCL; ++k)
+                        if ((uint32_t)(v[k] >> 32) != ep) { stale = true; v[k] = ld_slot(psrc + k * 2 * UM); }
+                    if ((uint32_t)(v[NCL] >> 32) != ep) { stale = true; v[NCL] = ld_slot(hsrc); }
+                    if (!stale) break;
+                    ++rounds;
+                }
+                XST(stL && n == tid / UM, 13);
+                float dh = 0.f;
+#pragma unroll
+                for (int k = 0; k <= NCL; ++k) dh += __uint_as_float((uint32_t)v[k]);
+                const float th = ftanh(c);
+                const float chat = dc + dh * o * (1.f - th * th);
+                const float g0 = chat * uv * i * (1.f - i), g1 = dh * th * o * (1.f - o), g2 = chat * i * (1.f - uv * uv);
+                pool[rec + 5 * H + jj] = g0;
+                pool[rec + 6 * H + jj] = g1;
+                pool[rec + 7 * H + jj] = g2;
+                dbleaf[0] += g0; dbleaf[1] += g1; dbleaf[2] += g2;
+                XST(stL && n == tid / UM, 14);
+            }
+            XST(stL, 15);
+            if (bt) { bt[1] = bt[2] = clock64(); bt[4] |= (uint64_t)rounds << 8; }
+            mark(4);
+            __syncthreads();
+            if (bt) bt[3] = clock64();
+            pos = next;
+            continue;
+        }
         if (op == INT_F || is_head) {
             // rows [h_l; h_r] (INT_F) or h of the labelled node (heads), one half row (H values) per
             // (node, side).  Internal children: H tagged slots = H/2 16-byte pieces -> u64 scratch; leaf
@@ -207,7 +276,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             for (int r = rsub, p = 0; r < rows; r += RPP, ++p) {
                 const int n = A == 2 ? r >> 1 : r, half = A == 2 ? r & 1 : 0;
                 const uint32_t* e = ent + n * sz;
-                const uint32_t hx = op == INT_F ? e[3 + 2 * half] : (op == HEAD_F ? e[3] : e[4]);
+                const uint32_t hx = op == INT_F ? e[3 + 2 * half] : e[3];
                 if (hx == NONE) {
                     if (pr < H / 4) cp_async16(xs + n * KP + half * H + 4 * pr, pool + (op == INT_F ? e[2 + 2 * half] : e[1]) + 4 * pr, 16u);
                 } else {
@@ -215,6 +284,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                     my_tagged |= 1u << p;
                 }
             }
+            XST(stF, 17);
             if (op == INT_F && tid < nb * UM) {            // c_l, c_r of this CTA's units (own records)
                 const int n = tid / UM, uu = tid % UM;
                 const uint32_t* e = ent + n * sz;
@@ -222,7 +292,9 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 cp_async4(cin + tid * CINMAX + 1, pool + e[4] + H + lc * UM + uu, 4u);
             }
             cp_async_wait_all();
+            XST(stF, 18);
             __syncthreads();
+            XST(stF, 19);
             if (bt) bt[1] = clock64();
             mark(2);
             // check the epochs, convert fresh pieces; re-fetch pieces of producers that were still behind
@@ -238,11 +310,12 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                         my_tagged &= ~(1u << p);
                     } else {
                         const uint32_t* e = ent + n * sz;
-                        const uint32_t hx = op == INT_F ? e[3 + 2 * half] : (op == HEAD_F ? e[3] : e[4]);
+                        const uint32_t hx = op == INT_F ? e[3 + 2 * half] : e[3];
                         cp_async16(tbuf + o, HX + (int64_t)hx * H + 2 * pr, 16u);
                         ++stale;
                     }
                 }
+                XST(stF && rounds == 0, 20);
                 if (__syncthreads_count(stale) == 0) break;
                 ++rounds;
                 cp_async_wait_all();
@@ -272,7 +345,9 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
 #pragma unroll
             for (int k = 0; k < NCL; ++k) v[k] = psrc ? ld_slot(psrc + k * 2 * UM) : none;
             v[NCL] = hsrc ? ld_slot(hsrc) : none;
+            XST(stB, 23);
             cp_async_wait_all();
+            XST(stB, 24);
             if (bt) bt[1] = clock64();
             mark(2);
             while (true) {
@@ -290,68 +365,68 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 for (int k = 0; k <= NCL; ++k) dh += __uint_as_float((uint32_t)v[k]);
                 cin[tid * CINMAX] = dh;
             }
+            XST(stB, 25);
             __syncthreads();
+            XST(stB, 26);
         }
         if (bt) { bt[2] = clock64(); bt[4] |= (uint64_t)rounds << 8; }
 
         mark(is_head ? 6 : (op == INT_F ? 3 : 4));
         if (is_head) {            // loss heads (L42) on the CTA holding W_out
             constexpr int KPH = KP;
-            if (op == HEAD_F) {
-                for (int pi = warp; pi < nb * C; pi += NTH / 32) {
-                    const int n = pi / C, c = pi - n * C;
-                    float s = 0.f;
-                    for (int k = 4 * lane; k < H; k += 128) {
-                        const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
-                        const float4 h4 = *reinterpret_cast<const float4*>(xs + n * KPH + k);
-                        s += w4.x * h4.x + w4.y * h4.y + w4.z * h4.z + w4.w * h4.w;
-                    }
-                    s = warp_sum(s);
-                    if (lane == 0) zs[n * ZC + c] = s + bo[c];
+            // forward: logits z = W_out h + b_out, softmax-NLL (L42); backward: dz = p - onehot(y),
+            // dW_out += dz h^T, db_out += dz, dh = W_out^T dz -> HD slots of the labelled cell
+            for (int pi = warp; pi < nb * C; pi += NTH / 32) {
+                const int n = pi / C, c = pi - n * C;
+                float s = 0.f;
+                for (int k = 4 * lane; k < H; k += 128) {
+                    const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                    const float4 h4 = *reinterpret_cast<const float4*>(xs + n * KPH + k);
+                    s += w4.x * h4.x + w4.y * h4.y + w4.z * h4.z + w4.w * h4.w;
                 }
-                __syncthreads();
-                for (int n = warp; n < nb; n += NTH / 32) {
-                    const uint32_t* e = ent + n * sz;
-                    const float zl = lane < C ? zs[n * ZC + lane] : -INFINITY;
-                    const float m = warp_max(zl);
-                    const float lse = m + logf(warp_sum(lane < C ? expf(zl - m) : 0.f));
-                    if (lane < C) pool[e[0] + lane] = expf(zl - lse);
-                    const float zy = __shfl_sync(FULLMASK, zl, (int)e[2]);
-                    if (lane == 0) {
-                        pool[e[0] + C] = lse - zy;
-                        atomicAdd(pool + P.loss_word, lse - zy);   // aggregated loss node (L205)
-                    }
+                s = warp_sum(s);
+                if (lane == 0) zs[n * ZC + c] = s + bo[c];
+            }
+            __syncthreads();
+            for (int n = warp; n < nb; n += NTH / 32) {
+                const uint32_t* e = ent + n * sz;
+                const float zl = lane < C ? zs[n * ZC + lane] : -INFINITY;
+                const float m = warp_max(zl);
+                const float lse = m + logf(warp_sum(lane < C ? expf(zl - m) : 0.f));
+                const float p = expf(zl - lse);
+                if (lane < C) {
+                    pool[e[0] + lane] = p;
+                    zs[n * ZC + lane] = p - (lane == (int)e[2] ? 1.f : 0.f);
                 }
-            } else {
-                for (int i = tid; i < nb * C; i += NTH) {
-                    const int n = i / C, c = i - n * C;
-                    const uint32_t* e = ent + n * sz;
-                    zs[n * ZC + c] = pool[e[0] + c] - (c == (int)e[2] ? 1.f : 0.f);
+                const float zy = __shfl_sync(FULLMASK, zl, (int)e[2]);
+                if (lane == 0) {
+                    pool[e[0] + C] = lse - zy;
+                    atomicAdd(pool + P.loss_word, lse - zy);   // aggregated loss node (L205)
                 }
-                __syncthreads();
-                for (int c = tid; c < C; c += NTH) {
-                    float s = 0.f;
-                    for (int n = 0; n < nb; ++n) s += zs[n * ZC + c];
-                    dbo[c] += s;
+            }
+            __syncthreads();
+            for (int c = tid; c < C; c += NTH) {
+                float s = 0.f;
+                for (int n = 0; n < nb; ++n) s += zs[n * ZC + c];
+                dbo[c] += s;
+            }
+            for (int i = tid; i < C * H; i += NTH) {
+                const int c = i / H, k = i - c * H;
+                float s = 0.f;
+                for (int n = 0; n < nb; ++n) s = fmaf(zs[n * ZC + c], xs[n * KPH + k], s);
+                dWo[i] += s;
+            }
+            for (int i = tid; i < nb * (H / 4); i += NTH) {   // dh of the labelled node -> HD slots
+                const int n = i / (H / 4), k = (i - n * (H / 4)) * 4;
+                float v4[4] = {0.f, 0.f, 0.f, 0.f};
+                for (int c = 0; c < C; ++c) {
+                    const float dzc = zs[n * ZC + c];
+                    const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                    v4[0] = fmaf(w4.x, dzc, v4[0]); v4[1] = fmaf(w4.y, dzc, v4[1]);
+                    v4[2] = fmaf(w4.z, dzc, v4[2]); v4[3] = fmaf(w4.w, dzc, v4[3]);
                 }
-                for (int i = tid; i < C * H; i += NTH) {
-                    const int c = i / H, k = i - c * H;
-                    float s = 0.f;
-                    for (int n = 0; n < nb; ++n) s = fmaf(zs[n * ZC + c], xs[n * KPH + k], s);
-                    dWo[i] += s;
-                }
-                for (int i = tid; i < nb * (H / 4); i += NTH) {   // dh of the labelled node -> HD slots
-                    const int n = i / (H / 4), k = (i - n * (H / 4)) * 4;
-                    float v4[4] = {0.f, 0.f, 0.f, 0.f};
-                    for (int c = 0; c < C; ++c) {
-                        const float dzc = zs[n * ZC + c];
-                        const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
-                        v4[0] = fmaf(w4.x, dzc, v4[0]); v4[1] = fmaf(w4.y, dzc, v4[1]);
-                        v4[2] = fmaf(w4.z, dzc, v4[2]); v4[3] = fmaf(w4.w, dzc, v4[3]);
-                    }
-                    const uint32_t hd = ent[n * sz + 3];
-                    if (hd != NONE) st_tag4(HD + (int64_t)hd * H + k, v4, ep);
-                }
+                const uint32_t hd = ent[n * sz + 4];
+                if (hd != NONE) st_tag4(HD + (int64_t)hd * H + k, v4, ep);
             }
         } else if (op == INT_F) {
             // ---- forward of internal cells: matvec from registers (L123), 4 nodes at a time; the unit's
@@ -360,6 +435,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             // butterfly, after which lane 16/NN * m holds node m's gates
             auto fwd_group = [&](auto nnc, int n0) {
                 constexpr int NN = decltype(nnc)::value;
+                XST(stF, 0);
                 float2 a[NN][5];
 #pragma unroll
                 for (int n = 0; n < NN; ++n)
@@ -368,7 +444,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
 #pragma unroll
                 for (int t = 0; t < LB::NT; ++t) {
                     const int col0 = LB::CG * (tu + TU * t);
-                    const int of = col0 < H ? 3 : 4;
+                    constexpr int of0 = 3;                  // granules t < T::TH read h_l (U_fl), the rest h_r (U_fr)
 #pragma unroll
                     for (int n = 0; n < NN; ++n) {
                         float xv[LB::CG];
@@ -380,12 +456,11 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
 #pragma unroll
                             for (int r = 0; r < 3; ++r)
                                 a[n][r] = __ffma2_rn(make_float2(wb[r][k], wb[r][k + 1]), x2, a[n][r]);
-                            const float2 f2 = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), x2, make_float2(0.f, 0.f));
-                            if (of == 3) { a[n][3].x += f2.x; a[n][3].y += f2.y; }
-                            else { a[n][4].x += f2.x; a[n][4].y += f2.y; }
+                            a[n][of0 + (t >= T::TH)] = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), x2, a[n][of0 + (t >= T::TH)]);
                         }
                     }
                 }
+                XST(stF, 1);
                 float g5[5];
 #pragma unroll
                 for (int o = 0; o < 5; ++o) {
@@ -407,6 +482,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                         g5[o] = k;
                     }
                 }
+                XST(stF, 2);
                 constexpr int SPAN = 16 / NN;
                 const int n = n0 + gl / SPAN;
                 if (gl % SPAN == 0 && n < nb) {
@@ -414,10 +490,10 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                     const uint32_t rec = e[0];
                     const float* b = bias + u * 4;
                     const float* cv = cin + (n * UM + u) * CINMAX;
-                    const float i = sigm(g5[0] + b[0]), o = sigm(g5[1] + b[1]), uv = tanhf(g5[2] + b[2]);
-                    const float fl = sigm(g5[3] + b[3]), fr = sigm(g5[4] + b[3]);
+                    const float i = fsigm(g5[0] + b[0]), o = fsigm(g5[1] + b[1]), uv = ftanh(g5[2] + b[2]);
+                    const float fl = fsigm(g5[3] + b[3]), fr = fsigm(g5[4] + b[3]);
                     const float c = i * uv + fl * cv[0] + fr * cv[1];
-                    const float h = o * tanhf(c);
+                    const float h = o * ftanh(c);
                     if (e[1] != NONE) st_tag(HX + (int64_t)e[1] * H + j, h, ep);   // read by the whole group
                     pool[rec + j] = h;                                              // the rest: this CTA, GEMMs
                     pool[rec + H + j] = c;
@@ -427,6 +503,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                     pool[rec + 5 * H + j] = fl;
                     pool[rec + 6 * H + j] = fr;
                 }
+                XST(stF, 3);
             };
             int n0 = 0;
             for (; n0 + 2 < nb; n0 += 4) fwd_group(std::integral_constant<int, 4>{}, n0);
@@ -436,13 +513,14 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             // ---- backward: cell backward by thread (unit u, node gl); gate gradients recorded for the dW
             //      GEMM (L185) and broadcast to the unit's lanes ----
             const bool kindB = op == INT_B;
+            XST(stB, 5);
             float g[5] = {0.f, 0.f, 0.f, 0.f, 0.f};
             if (gl < nb) {
                 const uint32_t* e = ent + gl * sz;
                 const uint32_t rec = e[0];
                 const float* cv = cin + (gl * UM + u) * CINMAX;
                 const float dh = cv[0], dc = cv[1], c = cv[2], i = cv[3], o = cv[4], uv = cv[5];
-                const float th = tanhf(c);
+                const float th = ftanh(c);
                 const float chat = dc + dh * o * (1.f - th * th);
                 g[0] = chat * uv * i * (1.f - i);
                 g[1] = dh * th * o * (1.f - o);
@@ -466,6 +544,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 dbacc[0] += g[0]; dbacc[1] += g[1]; dbacc[2] += g[2]; dbacc[3] += g[3] + g[4];
             }
             mark(5);
+            XST(stB, 6);
             // transposed products (L94, fn4): per node, this CTA's partial dx = Σ_r W[r] g_r over all 2H
             // columns; the 16 unit slices are summed in shared memory and published as tagged PART slots
             if (kindB) {
@@ -482,7 +561,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
 #pragma unroll
                         for (int t = 0; t < LB::NT; ++t) {
                             const int col0 = LB::CG * (tu + TU * t);
-                            const float gf = col0 < H ? gr[3] : gr[4];
+                            const float gf = t < T::TH ? gr[3] : gr[4];
                             float dx[LB::CG];
 #pragma unroll
                             for (int q = 0; q < LB::CG; q += 2) {
@@ -498,7 +577,9 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                             sts_granule<LB::CG>(drow + col0, dx, n < nb);
                         }
                     }
+                    XST(stB, 7);
                     __syncthreads();
+                    XST(stB, 8);
                     constexpr int q4 = KP / 4;
                     for (int i = tid; i < NC * q4; i += NTH) {
                         const int dn = i / q4, c = (i - dn * q4) * 4, n = n0 + dn;
@@ -514,11 +595,15 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                         const uint32_t pp = ent[n * sz + 4];
                         st_tag4(PART + ((((int64_t)pp * NCL + m) * NCL + lc) * 2 + side) * UM + (jj - m * UM), s, ep);
                     }
+                    XST(stB, 9);
                     __syncthreads();
+                    XST(stB, 10);
                 }
             }
         }
         __syncthreads();
+        XST(stF, 4);
+        XST(stB, 11);
         if (bt) bt[3] = clock64();
         pos = next;
     }
@@ -540,6 +625,12 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
 #pragma unroll
         for (int k = 0; k < 3; ++k) atomicAdd(P.grads + off[5] + k * H + j, dbacc[k]);
         atomicAdd(P.grads + off[6] + j, dbacc[3]);
+    }
+#pragma unroll
+    for (int k = 0; k < 3; ++k) dbleaf[k] += __shfl_xor_sync(FULLMASK, dbleaf[k], 16);   // lanes l, l^16: same unit
+    if (lane < 16) {
+#pragma unroll
+        for (int k = 0; k < 3; ++k) atomicAdd(P.grads + off[5] + k * H + lc * UM + lane, dbleaf[k]);
     }
     if (holds_head) {
         __syncthreads();

@@ -133,10 +133,10 @@ __global__ void __launch_bounds__(NT, 3) vpps_leaf_fwd(const float* __restrict__
 #pragma unroll
     for (int c = 0; c < 2; ++c) {
         const int j = j0 + up + 8 * c;
-        const float ig = sigm(pre[0][c] + __ldg(b + j)), og = sigm(pre[1][c] + __ldg(b + H + j));
-        const float ug = tanhf(pre[2][c] + __ldg(b + 2 * H + j));
+        const float ig = fsigm(pre[0][c] + __ldg(b + j)), og = fsigm(pre[1][c] + __ldg(b + H + j));
+        const float ug = ftanh(pre[2][c] + __ldg(b + 2 * H + j));
         const float cc = ig * ug;
-        r[j] = og * tanhf(cc);
+        r[j] = og * ftanh(cc);
         r[H + j] = cc;
         r[2 * H + j] = ig;
         r[3 * H + j] = og;

@@ -41,12 +41,15 @@ def main():
     dX = torch.zeros_like(X)
     s = m.build_script(synth.config_batch(args.config, args.batch_idx))
     n_cta = m.plan_info()["n_cta"]
-    stride = 16 + 5 * 48
+    stride = 16 + 5 * 48 + 32
     buf = torch.zeros((n_cta, stride), dtype=torch.int64, device="cuda")
     m.set_profile_buffer(buf, stride)
     gt = torch.zeros((4096, 5), dtype=torch.int64, device="cuda")
     m.set_gemm_trace(gt)
-    for _ in range(args.reps):
+    for r in range(args.reps):
+        if r == args.reps - 1:
+            torch.cuda.synchronize()
+            buf.zero_()
         m.fwd_bwd(s, X, dX)
     torch.cuda.synchronize()
     raw = buf.cpu().numpy().astype(np.float64)
@@ -81,7 +84,7 @@ def main():
     if args.batches:
         last = int(np.argmax(raw[:, 1]))
         g0 = (last // 16) * 16
-        ops = {0x21: "LEAF_B", 0x22: "INT_F", 0x23: "INT_B", 0x40: "HEAD_F", 0x41: "HEAD_B"}
+        ops = {0x21: "LEAF_B", 0x22: "INT_F", 0x23: "INT_B", 0x42: "HEAD_FB"}
         print(f"per-batch cycles of group {last // 16} (CTA {g0} | CTA {last}): issue->staged, staged->fresh "
               f"(retry rounds), compute, batch end relative to CTA {g0}")
         nbt = int(raw[last, 2])
@@ -93,6 +96,22 @@ def main():
                 r = int(b[k, 4]) >> 8
                 print(f"  {k:3d} {ops.get(op, hex(op)):7s} stage {b[k,1]-b[k,0]:6.0f} wait {b[k,2]-b[k,1]:6.0f} ({r} rnd)"
                       f" compute {b[k,3]-b[k,2]:6.0f} | end skew vs last CTA {bl[k,3]-b[k,3]:7.0f}")
+            x = raw[cta, 256:288]
+            if x[0] > 0:
+                print("  INT_F nb=1 compute: fma %.0f, reduce %.0f, cell+stores %.0f, end barrier %.0f" %
+                      (x[1] - x[0], x[2] - x[1], x[3] - x[2], x[4] - x[3]))
+            if x[16] > 0:
+                print("  INT_F nb=1 staging: issue %.0f, cp.async wait %.0f, bar %.0f, check %.0f, bar_count %.0f" %
+                      (x[17] - x[16], x[18] - x[17], x[19] - x[18], x[20] - x[19], x[0] - x[20]))
+            if x[22] > 0:
+                print("  INT_B nb=1 staging: issue %.0f, cp.async wait %.0f, poll %.0f, bar %.0f" %
+                      (x[23] - x[22], x[24] - x[23], x[25] - x[24], x[26] - x[25]))
+            if x[5] > 0:
+                print("  INT_B nb=1 compute: cell-bwd %.0f, tmv+sts %.0f, bar %.0f, reduce+st %.0f, bar %.0f, end bar %.0f" %
+                      (x[6] - x[5], x[7] - x[6], x[8] - x[7], x[9] - x[8], x[10] - x[9], x[11] - x[10]))
+            if x[12] > 0:
+                print("  LEAF_B iter0: poll %.0f, compute+stores %.0f; loop total from iter0 issue %.0f" %
+                      (x[13] - x[12], x[14] - x[13], x[15] - x[12]))
 
 
 if __name__ == "__main__":
