@@ -209,9 +209,9 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         const bool stB = xst && op == INT_B && nb == 1 && !(xdone & 2);
         const bool stL = xst && op == LEAF_B && !(xdone & 4);
         xdone |= (stF ? 1 : 0) | (stB ? 2 : 0) | (stL ? 4 : 0);
+#define XST(f, k) do { if (f) xst[k] = clock64(); } while (0)
         XST(stF, 16);
         XST(stB, 22);
-#define XST(f, k) do { if (f) xst[k] = clock64(); } while (0)
         mark(1);
         if (op == LEAF_B) {
             // leaf backward, thread (leaf tid / U + 16 p, unit tid % U): consecutive threads read consecutive
