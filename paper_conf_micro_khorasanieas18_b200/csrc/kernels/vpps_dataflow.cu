@@ -58,6 +58,9 @@ __device__ __forceinline__ u64 ld_slot(const u64* p) {
     asm volatile("ld.global.cg.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
+__device__ __forceinline__ void ld_slot2(const u64* p, u64& a, u64& b) {
+    asm volatile("ld.global.cg.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
 __device__ __forceinline__ void st_tag4(u64* p, const float* v, uint32_t e) {
     asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(tagv(v[0], e)), "l"(tagv(v[1], e)) : "memory");
     asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p + 2), "l"(tagv(v[2], e)), "l"(tagv(v[3], e)) : "memory");
@@ -273,6 +276,59 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             const int rows = nb * A;
             const int pr = tid % PPR, rsub = tid / PPR;
             uint32_t my_tagged = 0;                        // bit p: pass p's half row is tagged
+            if (rows <= 4 * RPP) {
+                // small batch (<= 4 passes per thread): tagged pieces straight into registers, checked and
+                // converted there — one L2 round trip and one barrier
+                u64 ta[4], tb[4];
+#pragma unroll
+                for (int p = 0; p < 4; ++p) {
+                    const int r = rsub + p * RPP;
+                    if (r >= rows) break;
+                    const int n = A == 2 ? r >> 1 : r, half = A == 2 ? r & 1 : 0;
+                    const uint32_t* e = ent + n * sz;
+                    const uint32_t hx = op == INT_F ? e[3 + 2 * half] : e[3];
+                    if (hx == NONE) {
+                        if (pr < H / 4) cp_async16(xs + n * KP + half * H + 4 * pr, pool + (op == INT_F ? e[2 + 2 * half] : e[1]) + 4 * pr, 16u);
+                    } else {
+                        ld_slot2(HX + (int64_t)hx * H + 2 * pr, ta[p], tb[p]);
+                        my_tagged |= 1u << p;
+                    }
+                }
+                XST(stF, 17);
+                if (op == INT_F && tid < nb * UM) {        // c_l, c_r of this CTA's units (own records)
+                    const int n = tid / UM, uu = tid % UM;
+                    const uint32_t* e = ent + n * sz;
+                    cp_async4(cin + tid * CINMAX, pool + e[2] + H + lc * UM + uu, 4u);
+                    cp_async4(cin + tid * CINMAX + 1, pool + e[4] + H + lc * UM + uu, 4u);
+                }
+                cp_async_wait_all();
+                XST(stF, 18);
+                XST(stF, 19);
+                if (bt) bt[1] = clock64();
+                mark(2);
+                while (true) {
+                    int stale = 0;
+#pragma unroll
+                    for (int p = 0; p < 4; ++p) {
+                        if (!(my_tagged >> p & 1u)) continue;
+                        const int r = rsub + p * RPP;
+                        const int n = A == 2 ? r >> 1 : r, half = A == 2 ? r & 1 : 0;
+                        const int o = n * KP + half * H + 2 * pr;
+                        if ((uint32_t)(ta[p] >> 32) == ep && (uint32_t)(tb[p] >> 32) == ep) {
+                            *reinterpret_cast<float2*>(xs + o) = make_float2(__uint_as_float((uint32_t)ta[p]), __uint_as_float((uint32_t)tb[p]));
+                            my_tagged &= ~(1u << p);
+                        } else {
+                            const uint32_t* e = ent + n * sz;
+                            const uint32_t hx = op == INT_F ? e[3 + 2 * half] : e[3];
+                            ld_slot2(HX + (int64_t)hx * H + 2 * pr, ta[p], tb[p]);
+                            ++stale;
+                        }
+                    }
+                    XST(stF && rounds == 0, 20);
+                    if (__syncthreads_count(stale) == 0) break;
+                    ++rounds;
+                }
+            } else {
             for (int r = rsub, p = 0; r < rows; r += RPP, ++p) {
                 const int n = A == 2 ? r >> 1 : r, half = A == 2 ? r & 1 : 0;
                 const uint32_t* e = ent + n * sz;
@@ -284,7 +340,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                     my_tagged |= 1u << p;
                 }
             }
-            XST(stF, 17);
             if (op == INT_F && tid < nb * UM) {            // c_l, c_r of this CTA's units (own records)
                 const int n = tid / UM, uu = tid % UM;
                 const uint32_t* e = ent + n * sz;
@@ -292,9 +347,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 cp_async4(cin + tid * CINMAX + 1, pool + e[4] + H + lc * UM + uu, 4u);
             }
             cp_async_wait_all();
-            XST(stF, 18);
             __syncthreads();
-            XST(stF, 19);
             if (bt) bt[1] = clock64();
             mark(2);
             // check the epochs, convert fresh pieces; re-fetch pieces of producers that were still behind
@@ -315,10 +368,10 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                         ++stale;
                     }
                 }
-                XST(stF && rounds == 0, 20);
                 if (__syncthreads_count(stale) == 0) break;
                 ++rounds;
                 cp_async_wait_all();
+            }
             }
         } else {
             // backward, thread (n = tid / U, u = tid % U): dh = Σ_k PART[parent][lc][k][side][u] (+ HD), its

@@ -186,6 +186,14 @@ def test_lstm_h256_small_vocab():
     check("lstm", 256, 256, 16, graphs, 16, seed=9)
 
 
+@pytest.mark.parametrize("batch", [1, 4, 16, 64])
+def test_lstm_config3_batch_sweep(batch):
+    """Config 3 (LSTM LM, H = E = 256, sentences of 5-60 tokens, batch 1/4/16/64) with the GPU reading of
+    the vocabulary (R-31: V = C = 32 symbols, the head held in one CTA's shared memory)."""
+    graphs = synth.config_batch("c3", 0, batch=batch, V=32, C=32)
+    check("lstm", 256, 256, 32, graphs, 32, seed=30 + batch)
+
+
 def test_fused_sgd_update():
     graphs = _trees(6, 4, (1, 9), 20, 5)
     lr, wd = 0.05, 1e-3
