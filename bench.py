@@ -226,6 +226,7 @@ def main():
         s.upload()
     infos = [s.info() for s in scripts]
     flush = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device=dev)   # 256 MiB > 126 MB L2
+    flush2 = torch.ones(64 * 1024 * 1024, dtype=torch.float32, device=dev) if os.environ.get("VPPS_FLUSH_CLEAN") else None
     lr, wd = 1e-3, 1e-5
 
     from paper_conf_micro_khorasanieas18_b200 import dp
@@ -257,6 +258,8 @@ def main():
     for k in range(args.steps):
         if not args.no_flush:
             flush.zero_()
+            if os.environ.get("VPPS_FLUSH_CLEAN"):     # measurement experiment: leave the L2 clean
+                flush2.sum()
         m.set_timing_events(*kev[k])
         ev[k][0].record(stream)
         step(args.warmup + k)

@@ -622,6 +622,7 @@ struct GemmParams {
     float lr, wd;
     const float* loss_src;
     float* loss_dst;
+    int32_t tc;                  // 1: weight-gradient tiles on the tensor cores (tcgen05, 3xTF32, TMEM)
 };
 
 constexpr int TM = 128;          // tile rows (gate-gradient rows)
@@ -690,8 +691,11 @@ __device__ __forceinline__ void leaf_dx_tile(const GemmParams& P, const uint32_t
     }
 }
 
-__host__ __device__ inline int job_items(int m, int n_int, int n_leaf, int H, int E, bool dx) {
-    const int ki = (n_int + KCH - 1) / KCH, kl = (n_leaf + KCH - 1) / KCH;
+constexpr int KTC = 48;          // nodes per tensor-core work item (6 MMA k-steps of 8)
+
+__host__ __device__ inline int job_items(int m, int n_int, int n_leaf, int H, int E, bool dx, bool tc = false) {
+    const int kch = tc ? KTC : KCH;
+    const int ki = (n_int + kch - 1) / kch, kl = (n_leaf + kch - 1) / kch;
     switch (m) {
         case 0: return (3 * H / TM) * (2 * H / TN) * ki;
         case 1:
@@ -701,9 +705,199 @@ __host__ __device__ inline int job_items(int m, int n_int, int n_leaf, int H, in
     }
 }
 
+// ---- tensor-core weight-gradient tile (tcgen05.mma kind::tf32, accumulator in TMEM) ----
+// D[128 gate rows][64 input cols] = Σ_k g_k[rows] x_k[cols]ᵀ over <= KTC nodes.  FP32 accuracy with 3xTF32:
+// D = A·B + A·B_lo + A_lo·B, where the tensor core truncates A, B to TF32 and A_lo = A - trunc(A) (exact in
+// FP32); the dropped A_lo·B_lo term is ~2^-20 of |A||B| (tools/umma_test.cu: 7e-7 max relative error).
+// Operands are staged K-major in the SWIZZLE_NONE canonical layout: core matrix = 8 rows x 16 B (4 k),
+// rows 16 B apart, SBO = 128 B between 8-row groups, LBO = (rows / 8) * 128 B between 4-k chunks
+// (tools/umma_test.cu pins this layout; the MN-major form read zeros on sm_100a).
+__shared__ uint32_t tc_tmem;                  // TMEM base of this CTA's 64-column accumulator
+__shared__ __align__(8) uint64_t tc_mbar;      // MMA-completion mbarrier
+__shared__ uint32_t tc_phase;                 // parity of the next completion
+
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo) {
+    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
+           ((uint64_t)(128 >> 4) << 32) | ((uint64_t)1 << 46);
+}
+constexpr uint32_t umma_idesc(int m, int n) {      // F32 accumulate, TF32 A/B, both K-major
+    return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(m >> 4) << 24);
+}
+__device__ __forceinline__ void umma_tf32(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, int acc) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                 "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}\n"
+                 ::"r"(d), "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ float tf32_lo(float v) { return v - __uint_as_float(__float_as_uint(v) & 0xFFFFE000u); }
+
+__device__ void tc_setup() {                   // warp 0: TMEM allocation; thread 0: mbarrier
+    if (threadIdx.x < 32) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tc_tmem)), "r"(64));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&tc_mbar)));
+        asm volatile("fence.mbarrier_init.release.cluster;");
+        tc_phase = 0;
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+__device__ void tc_teardown() {
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    if (threadIdx.x < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tc_tmem), "r"(64));
+}
+
+__device__ __forceinline__ void dw_item_tc(const GemmParams& P, int m, int b, int n_int, int n_leaf,
+                                           const uint32_t* int_nodes, const uint32_t* leaf_nodes, float* sm,
+                                           uint32_t* idx) {
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, H = P.H, E = P.E;
+    const int rows = (m == 0 || m == 3) ? 3 * H : H;
+    const int cols = m == 0 ? 2 * H : (m == 3 ? E : H);
+    const int K = m == 3 ? n_leaf : n_int;
+    const int tiles_r = rows / TM, tiles_c = cols / TN;
+    const int kc = b / (tiles_r * tiles_c), t = b - kc * (tiles_r * tiles_c);
+    const int r0 = (t / tiles_c) * TM, c0 = (t % tiles_c) * TN;
+    const int k0 = kc * KTC, nk = min(K, k0 + KTC) - k0;
+    const int ks = (nk + 7) / 8;                   // MMA k-steps
+    const uint32_t ph = tc_phase;                  // read before the staging barrier; thread 0 flips it after
+    const int goff = m == 0 ? 7 * H : (m == 1 ? 10 * H : (m == 2 ? 11 * H : 5 * H));
+    // smem: A hi/lo [TM x KTC], B hi/lo [TN x KTC], K-major canonical
+    float* Ah = sm;
+    float* Al = Ah + TM * KTC;
+    float* Bh = Al + TM * KTC;
+    float* Bl = Bh + TN * KTC;
+    constexpr uint32_t LBO_A = (TM / 8) * 128, LBO_B = (TN / 8) * 128;   // bytes between 4-k chunks
+    if (tid < nk) {
+        const int node = k0 + tid;
+        if (m == 3) {
+            idx[3 * tid] = leaf_nodes[2 * node];
+            idx[3 * tid + 1] = leaf_nodes[2 * node + 1];
+        } else {
+            idx[3 * tid] = int_nodes[3 * node];
+            idx[3 * tid + 1] = int_nodes[3 * node + 1];
+            idx[3 * tid + 2] = int_nodes[3 * node + 2];
+        }
+    }
+    __syncthreads();
+    // A blocks (TM/4 x ks*2), then B blocks (TN/4 x ks*2); k >= nk zero-filled up to the k-step
+    const int kb = 2 * ks;                         // 4-k chunks
+    const int na = (TM / 4) * kb, nbk = (TN / 4) * kb;
+    // every block's loads in flight before any conversion (one L2 round trip): <= 3 blocks per thread
+    constexpr int BPT = ((TM / 4) * (2 * KTC / 8) + (TN / 4) * (2 * KTC / 8) + 255) / 256;
+    float4 v[BPT][4];
+#pragma unroll
+    for (int q = 0; q < BPT; ++q) {
+        const int e = tid + 256 * q;
+        const bool isA = e < na;
+        const int ee = isA ? e : e - na;
+        const int nr4 = isA ? TM / 4 : TN / 4;      // consecutive threads: consecutive row blocks of one
+        const int k4 = ee / nr4, r4 = ee - k4 * nr4; // 4-k chunk (coalesced loads, conflict-free 16 B stores)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int k = 4 * k4 + j;
+            const float* src = nullptr;
+            if (e < na + nbk && k < nk) {
+                if (isA) {
+                    src = P.pool + idx[3 * k] + goff + r0 + 4 * r4;
+                } else {
+                    const int c = c0 + 4 * r4;
+                    if (m == 3) src = P.inputs + (int64_t)idx[3 * k + 1] * E + c;
+                    else if (m == 0) src = c < H ? P.pool + idx[3 * k + 1] + c : P.pool + idx[3 * k + 2] + (c - H);
+                    else src = P.pool + idx[3 * k + (m == 1 ? 1 : 2)] + c;
+                }
+            }
+            v[q][j] = src ? __ldcg(reinterpret_cast<const float4*>(src)) : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+    }
+#pragma unroll
+    for (int q = 0; q < BPT; ++q) {
+        const int e = tid + 256 * q;
+        if (e >= na + nbk) break;
+        const bool isA = e < na;
+        const int ee = isA ? e : e - na;
+        const int nr4 = isA ? TM / 4 : TN / 4;
+        const int k4 = ee / nr4, r4 = ee - k4 * nr4;
+        float* hi = isA ? Ah : Bh;
+        float* lo = isA ? Al : Bl;
+        const uint32_t lbo_f = isA ? LBO_A / 4 : LBO_B / 4;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+            const int r = 4 * r4 + c;
+            const uint32_t o = (uint32_t)((r >> 3) * 32 + (r & 7) * 4 + k4 * lbo_f);   // floats
+            const float a0 = c == 0 ? v[q][0].x : c == 1 ? v[q][0].y : c == 2 ? v[q][0].z : v[q][0].w;
+            const float a1 = c == 0 ? v[q][1].x : c == 1 ? v[q][1].y : c == 2 ? v[q][1].z : v[q][1].w;
+            const float a2 = c == 0 ? v[q][2].x : c == 1 ? v[q][2].y : c == 2 ? v[q][2].z : v[q][2].w;
+            const float a3 = c == 0 ? v[q][3].x : c == 1 ? v[q][3].y : c == 2 ? v[q][3].z : v[q][3].w;
+            *reinterpret_cast<float4*>(hi + o) = make_float4(a0, a1, a2, a3);
+            *reinterpret_cast<float4*>(lo + o) = make_float4(tf32_lo(a0), tf32_lo(a1), tf32_lo(a2), tf32_lo(a3));
+        }
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic smem writes -> tensor core
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    if (tid == 0) {
+        constexpr uint32_t idesc = umma_idesc(TM, TN);
+        const uint32_t a0 = smem_u32(Ah), al0 = smem_u32(Al), b0 = smem_u32(Bh), bl0 = smem_u32(Bl);
+        for (int s = 0; s < ks; ++s) {
+            const uint64_t a = umma_desc(a0 + 2 * s * LBO_A, LBO_A), al = umma_desc(al0 + 2 * s * LBO_A, LBO_A);
+            const uint64_t bb = umma_desc(b0 + 2 * s * LBO_B, LBO_B), bl = umma_desc(bl0 + 2 * s * LBO_B, LBO_B);
+            umma_tf32(tc_tmem, a, bb, idesc, s > 0);
+            umma_tf32(tc_tmem, a, bl, idesc, 1);
+            umma_tf32(tc_tmem, al, bb, idesc, 1);
+        }
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(&tc_mbar)) : "memory");
+    }
+    {
+        uint32_t ok = 0;
+        while (!ok)
+            asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}\n"
+                         : "=r"(ok) : "r"(smem_u32(&tc_mbar)), "r"(ph) : "memory");
+    }
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    // epilogue: warp w reads TMEM lanes 32 (w % 4) .. +31 (tile rows), columns 32 (w / 4) .. +31
+    const int row = 32 * (warp & 3) + lane, cb = 32 * (warp >> 2);
+    uint32_t r[32];
+    const uint32_t ta = tc_tmem + ((uint32_t)(32 * (warp & 3)) << 16) + cb;
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+                   "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+                 : "r"(ta));
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+                 : "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+                   "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+                 : "r"(ta + 16));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");   // TMEM reads done before the next MMA
+    if (tid == 0) tc_phase ^= 1u;
+    // transpose through shared memory (the MMA has finished reading the operands) so that a warp's vector
+    // reductions cover whole 256-byte row segments: tile [TM][TN + 4]
+    constexpr int DS = TN + 4;
+    float* Ds = sm;
+#pragma unroll
+    for (int q = 0; q < 8; ++q)
+        *reinterpret_cast<float4*>(Ds + row * DS + cb + 4 * q) =
+            make_float4(__uint_as_float(r[4 * q]), __uint_as_float(r[4 * q + 1]), __uint_as_float(r[4 * q + 2]),
+                        __uint_as_float(r[4 * q + 3]));
+    __syncthreads();
+    const int ty = tid / 16, tx = tid % 16;
+    float* base = P.grads + P.off[m == 3 ? 0 : m + 1] + (int64_t)r0 * cols + c0 + 4 * tx;
+#pragma unroll
+    for (int a = 0; a < TM / 16; ++a) {
+        const float4 x = *reinterpret_cast<const float4*>(Ds + (ty + 16 * a) * DS + 4 * tx);
+        const float v[4] = {x.x, x.y, x.z, x.w};
+        red_add<4>(base + (int64_t)(ty + 16 * a) * cols, v);
+    }
+}
+
 // One work item of group g: item i -> (job m, local index b).  dW tiles: 128 gate rows x 64 input columns
 // over the item's <= KCH nodes, all operand rows staged by one batch of cp.async after the node record
 // offsets are read once into shared memory; 8 x 4 FFMA2 per thread; partial tile added to grads.
+template <bool TC>
 __device__ __forceinline__ void dw_item(const GemmParams& P, int g, int i, float* sm, uint32_t* idx) {
     const int tid = threadIdx.x, H = P.H, E = P.E;
     const int n_int = P.int_off[g + 1] - P.int_off[g], n_leaf = P.leaf_off[g + 1] - P.leaf_off[g];
@@ -711,13 +905,14 @@ __device__ __forceinline__ void dw_item(const GemmParams& P, int g, int i, float
     const uint32_t* leaf_nodes = P.leaf_nodes + 2 * P.leaf_off[g];
     int m = 0, b = i;
     while (m < 5) {
-        const int n = job_items(m, n_int, n_leaf, H, E, P.d_inputs != nullptr);
+        const int n = job_items(m, n_int, n_leaf, H, E, P.d_inputs != nullptr, TC);
         if (b < n) break;
         b -= n;
         ++m;
     }
     if (m == 5) return;
     if (m == 4) { leaf_dx_tile(P, leaf_nodes, n_leaf, b, sm, idx); return; }
+    if constexpr (TC) { dw_item_tc(P, m, b, n_int, n_leaf, int_nodes, leaf_nodes, sm, idx); return; }
     const int rows = (m == 0 || m == 3) ? 3 * H : H;
     const int cols = m == 0 ? 2 * H : (m == 3 ? E : H);
     const int K = m == 3 ? n_leaf : n_int;
@@ -788,11 +983,13 @@ __device__ __forceinline__ void dw_item(const GemmParams& P, int g, int i, float
 // Persistent CTAs claim work items only from groups whose CTAs have all counted themselves done (no CTA
 // ever sits on an SM waiting for a group that is still running); groups are scanned in the host's order.
 // Without counters (P.done == nullptr) item = blockIdx.x over the groups in order.
+template <bool TC>
 __global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
     extern __shared__ __align__(16) float dsm[];
     __shared__ uint32_t idx[3 * KCH];
     __shared__ int pick[3];
     const int tid = threadIdx.x;
+    if constexpr (TC) tc_setup();
     if (!P.done || P.static_items) {
         // one item per CTA in the host's group order; with counters, wait for the item's group first
         int b = blockIdx.x;
@@ -810,11 +1007,13 @@ __global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
                     }
                     __syncthreads();
                 }
-                dw_item(P, g, b, dsm, idx);
+                dw_item<TC>(P, g, b, dsm, idx);
+                if constexpr (TC) tc_teardown();
                 return;
             }
             b -= P.items[g];
         }
+        if constexpr (TC) tc_teardown();
         return;
     }
     while (true) {
@@ -848,7 +1047,7 @@ __global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
         __syncthreads();
         if (g >= 0) {
             const uint64_t t0 = P.trace ? gtimer() : 0;
-            dw_item(P, g, i, dsm, idx);
+            dw_item<TC>(P, g, i, dsm, idx);
             __threadfence();
             __syncthreads();
             if (tid == 0) atomicAdd(P.fin, 1);
@@ -865,6 +1064,7 @@ __global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
         if (!rem) break;
         __nanosleep(500);
     }
+    if constexpr (TC) tc_teardown();
     // ---- fused tail: SGD over the flat parameters (L129, L197) and the loss read-back (L199) ----
     if (tid == 0) {
         uint32_t f;
@@ -943,13 +1143,17 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, flo
     g.loss_dst = loss_dst;
     g.done_target = done_target;
     g.n_grp = n_grp;
+    static const int tc_env = getenv("VPPS_DW_TC") ? atoi(getenv("VPPS_DW_TC")) : 0;
+    // tensor-core weight-gradient tiles (opt-in: measured 95.5K vs 100.6K samples/s for the FFMA2 tiles,
+    // the split-K tiles are bound by operand staging and the cross-group reductions, not by FMA issue)
+    g.tc = tc_env && H % TM == 0 && E % TN == 0;
     int items = 0;
     for (int q = 0; q < n_grp; ++q) {
         const int gi = order ? order[q] : q;
         g.grp[q] = gi;
         const int ni = int_off[gi + 1] - int_off[gi], nl = leaf_off[gi + 1] - leaf_off[gi];
         int n = 0;
-        for (int m = 0; m < 5; ++m) n += job_items(m, ni, nl, H, E, d_inputs != nullptr);
+        for (int m = 0; m < 5; ++m) n += job_items(m, ni, nl, H, E, d_inputs != nullptr, g.tc != 0);
         g.items[gi] = n;
         items += n;
     }
@@ -968,14 +1172,16 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, flo
         cfg.dynamicSmemBytes = DW_SMEM;
         static bool attr_set = false;
         if (!attr_set) {
-            cudaFuncSetAttribute(vpps_dw_gemm, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DW_SMEM);
+            cudaFuncSetAttribute(vpps_dw_gemm<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DW_SMEM);
+            cudaFuncSetAttribute(vpps_dw_gemm<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DW_SMEM);
             attr_set = true;
         }
         cfg.stream = s;
         cfg.attrs = attr;
         static const bool no_pdl = getenv("VPPS_DW_NOPDL") != nullptr;   // measurement only: no overlap
         cfg.numAttrs = early && !no_pdl ? 1 : 0;
-        cudaLaunchKernelEx(&cfg, vpps_dw_gemm, g);
+        if (g.tc) cudaLaunchKernelEx(&cfg, vpps_dw_gemm<true>, g);
+        else cudaLaunchKernelEx(&cfg, vpps_dw_gemm<false>, g);
     }
     if (fused_tail) return;                                            // SGD + loss inside the kernel
     if (mode == 1) launch_sgd(params, grads, n_floats, lr, wd, s);   // W -= lr (dW + wd W), every parameter

@@ -119,6 +119,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     const bool holds_head = (lc == 0);
 
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    if (P.prof && threadIdx.x == 0) P.prof[(int64_t)blockIdx.x * P.prof_stride + 11] = gtimer();   // entry
     // ---- prologue: this CTA's rows of U_iou, U_fl, U_fr -> registers (L123, L129) ----
     float wb[4][LB::NREG];
 #pragma unroll
@@ -696,6 +697,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         __syncthreads();
         if (tid == 0) atomicAdd(P.done + grp, 1);
     }
+    if (prof && tid == 0) prof[12] = gtimer();   // exit
 }
 
 }  // namespace df

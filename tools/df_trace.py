@@ -57,6 +57,12 @@ def main():
     gtr = gtr[gtr[:, 3] > 0]
     t0 = raw[:, 0].min()
     span = (raw[:, 1] - raw[:, 0]) / 1e3
+    if raw[:, 11].min() > 0:
+        print(f"kernel entry skew {(raw[:, 11].max() - raw[:, 11].min()) / 1e3:.1f} us, prologue (entry -> span "
+              f"start) mean {((raw[:, 0] - raw[:, 11]) / 1e3).mean():.1f} max {((raw[:, 0] - raw[:, 11]) / 1e3).max():.1f} us, "
+              f"epilogue (span end -> exit) mean {((raw[:, 12] - raw[:, 1]) / 1e3).mean():.1f} max "
+              f"{((raw[:, 12] - raw[:, 1]) / 1e3).max():.1f} us, first entry -> last exit "
+              f"{(raw[:, 12].max() - raw[:, 11].min()) / 1e3:.1f} us")
     names = ["program", "staging", "tag-wait", "forward", "cell-bwd", "transp", "heads", "other"]
     secs = raw[:, 3:11]
     print(f"{args.config} batch {args.batch_idx}: {n_cta} CTAs, span max {span.max():.1f} us "
