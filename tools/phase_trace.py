@@ -25,12 +25,18 @@ def main():
     ap.add_argument("--quiet", action="store_true")
     ap.add_argument("--sections", action="store_true")
     ap.add_argument("--cluster", type=int, default=0)
+    ap.add_argument("--vocab", type=int, default=0, help="override V = C (e.g. 32 for the config-3 GPU reading)")
+    ap.add_argument("--batch", type=int, default=0)
     args = ap.parse_args()
     import torch
     import synth
     from paper_conf_micro_khorasanieas18_b200 import vpps
     cfg = synth.CONFIGS[args.config]
     cell, H, E, C, V = cfg["cell"], cfg["H"], cfg["E"], cfg["C"], cfg["V"]
+    over = {}
+    if args.vocab:
+        C = V = args.vocab
+        over = {"V": V, "C": C}
     rng = np.random.default_rng(0)
     shapes = vpps.param_shapes(cell, H, E, C)
     P = synth.init_params(shapes, rng)
@@ -42,7 +48,7 @@ def main():
     m.bind(params, grads)
     X = torch.from_numpy(synth.input_table(rng, V, E)).float().cuda()
     dX = torch.zeros_like(X)
-    graphs = synth.config_batch(args.config, args.batch_idx)
+    graphs = synth.config_batch(args.config, args.batch_idx, batch=args.batch or None, **over)
     s = m.build_script(graphs)
     info = s.info()
     nbar = info["n_barriers"]
