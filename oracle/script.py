@@ -114,8 +114,12 @@ def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 14
     # S4/S5: phases and min-load group assignment
     P = 2 * L + 2
     by_level = [[] for _ in range(L + 1)]
+    for i in range(len(nodes)):                  # S4 (R-13): cells first, then heads, ascending global id
+        if nodes[i]["kind"] != "HEAD":
+            by_level[level[i]].append(i)
     for i in range(len(nodes)):
-        by_level[level[i]].append(i)
+        if nodes[i]["kind"] == "HEAD":
+            by_level[level[i]].append(i)
     graph_group = None
     if by_graph:
         # S5g: whole graphs, longest first (depth, then cell count, then batch index), each to the group

@@ -186,7 +186,12 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     // ---- S4-S6: phases, min-load groups, signal/wait ------------------------------------------
     const int32_t G = plan.G, P = 2 * L + 2;
     std::vector<std::vector<int64_t>> at_level(L + 1);
-    for (int64_t i = 0; i < N; ++i) at_level[level[i]].push_back(i);   // ascending global id
+    // S4 (reading R-13): cells before heads, each in ascending global id — consecutive same-opcode
+    // instructions form one batch in the kernels (an LM level alternates cell / head otherwise)
+    for (int64_t i = 0; i < N; ++i)
+        if (nodes[i].kind != K_HEAD) at_level[level[i]].push_back(i);
+    for (int64_t i = 0; i < N; ++i)
+        if (nodes[i].kind == K_HEAD) at_level[level[i]].push_back(i);
     std::vector<std::vector<uint32_t>> streams(G);
     std::vector<uint32_t> targets(n_bar + 1, 0);
     std::vector<std::vector<uint32_t>> body(G);

@@ -113,7 +113,8 @@ struct Cfg {
     static constexpr int ITER2 = (NB * UMAX * CINMAX + NTH - 1) / NTH;
     static_assert(UMAX * NB <= NTH && NB <= 32 && 32 % NB == 0, "one (unit, node) pair per thread");
     static_assert(KPMAX >= H, "head rows are staged in the input rows");
-    static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 2 * C + 8); }
+    static constexpr int HP = H + 4;          // W_out row stride in shared memory (conflict-free rows)
+    static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + C * HP + C * H + 2 * C + 8); }
 };
 
 __device__ __forceinline__ float sigm(float x) { return 1.0f / (1.0f + expf(-x)); }
@@ -366,7 +367,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
     float* dxb = sm + T::O_DXB;
     const int C = P.C;
     float* Wo = sm + T::O_HEAD;
-    float* dWo = Wo + C * H;
+    constexpr int HP = T::HP;
+    float* dWo = Wo + C * HP;                  // W_out rows at stride HP, dW_out dense
     float* bo = dWo + C * H;
     float* dbo = bo + C;
 
@@ -436,7 +438,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
     }
     const int wout_m = LS ? 2 : 4, bout_m = LS ? 4 : 7;
     if (holds_head) {
-        for (int i = tid; i < C * H; i += NTH) { Wo[i] = __ldg(P.params + off[wout_m] + i); dWo[i] = 0.f; }
+        for (int i = tid; i < C * H; i += NTH) { Wo[(i / H) * HP + i % H] = __ldg(P.params + off[wout_m] + i); dWo[i] = 0.f; }
         for (int i = tid; i < C; i += NTH) { bo[i] = __ldg(P.params + off[bout_m] + i); dbo[i] = 0.f; }
     }
 
@@ -636,16 +638,17 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
             mark(6);
             if (holds_head) {
                 if (op == OP_HEAD_F) {
-                    for (int pi = warp; pi < nb * C; pi += NTH / 32) {      // z[n][c], one warp per pair
-                        const int n = pi / C, c = pi - n * C;
-                        float s = 0.f;
-                        for (int k = 4 * lane; k < H; k += 128) {
-                            const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                    for (int pi = tid; pi < nb * C; pi += NTH) {            // z[n][c], one thread per pair:
+                        const int n = pi / C, c = pi - n * C;                   // h row broadcast, W_out rows
+                        float4 a = make_float4(0.f, 0.f, 0.f, 0.f);             // at stride HP (no conflicts)
+#pragma unroll 8
+                        for (int k = 0; k < H; k += 4) {
+                            const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * HP + k);
                             const float4 h4 = *reinterpret_cast<const float4*>(xs + n * KP + k);
-                            s += w4.x * h4.x + w4.y * h4.y + w4.z * h4.z + w4.w * h4.w;
+                            a.x = fmaf(w4.x, h4.x, a.x); a.y = fmaf(w4.y, h4.y, a.y);
+                            a.z = fmaf(w4.z, h4.z, a.z); a.w = fmaf(w4.w, h4.w, a.w);
                         }
-                        s = warp_sum(s);
-                        if (lane == 0) zs[n * ZC + c] = s + bo[c];
+                        zs[n * ZC + c] = (a.x + a.y) + (a.z + a.w) + bo[c];
                     }
                     __syncthreads();
                     for (int n = warp; n < nb; n += NTH / 32) {             // softmax-NLL, one warp per head
@@ -686,7 +689,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
                         float v4[4] = {0.f, 0.f, 0.f, 0.f};
                         for (int c = 0; c < C; ++c) {
                             const float dzc = zs[n * ZC + c];
-                            const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                            const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * HP + k);
                             v4[0] = fmaf(w4.x, dzc, v4[0]); v4[1] = fmaf(w4.y, dzc, v4[1]);
                             v4[2] = fmaf(w4.z, dzc, v4[2]); v4[3] = fmaf(w4.w, dzc, v4[3]);
                         }
@@ -1090,7 +1093,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
             if (jj < H) f((LS || k < 3) ? off[bias_m0] + k * H + jj : off[6] + jj, bias[tid], dbias[tid]);
         }
         if (holds_head) {
-            for (int i = tid; i < C * H; i += NTH) f(off[wout_m] + i, Wo[i], dWo[i]);
+            for (int i = tid; i < C * H; i += NTH) f(off[wout_m] + i, Wo[(i / H) * HP + i % H], dWo[i]);
             for (int i = tid; i < C; i += NTH) f(off[bout_m] + i, bo[i], dbo[i]);
         }
     };
