@@ -1143,9 +1143,12 @@ static const Variant kVariants[] = {
     VPPS_VARIANT(dev::CELL_BINARY, 128, 128, 1),
     VPPS_VARIANT(dev::CELL_BINARY, 32, 32, 1),
     VPPS_VARIANT(dev::CELL_CHILDSUM, 128, 128, 1),  // config 2
+    VPPS_VARIANT(dev::CELL_CHILDSUM, 128, 128, 2),  // ... G = 2 replica groups of 74 CTAs
+    VPPS_VARIANT(dev::CELL_CHILDSUM, 128, 128, 4),  // ... G = 4 replica groups of 37 CTAs
     VPPS_VARIANT(dev::CELL_CHILDSUM, 32, 32, 1),
     VPPS_VARIANT(dev::CELL_LSTM, 32, 32, 1),        // config 1
-    VPPS_VARIANT(dev::CELL_LSTM, 256, 256, 2),
+    VPPS_VARIANT(dev::CELL_LSTM, 256, 256, 2),      // config 3, G = 1
+    VPPS_VARIANT(dev::CELL_LSTM, 256, 256, 4),      // ... G = 2 (an LM level's loss heads split over 2 holders)
 };
 
 const Variant* variants(int32_t* n) {

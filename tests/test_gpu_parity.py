@@ -194,6 +194,17 @@ def test_lstm_config3_batch_sweep(batch):
     check("lstm", 256, 256, 32, graphs, 32, seed=30 + batch)
 
 
+@pytest.mark.parametrize("cell,H,groups", [("lstm", 256, 2), ("childsum", 128, 2), ("childsum", 128, 4)])
+def test_grid_replica_groups(cell, H, groups):
+    """Replica groups (R-28) of the grid kernel for configs 2 and 3: nodes split over G groups by the
+    min-load rule, gradients summed across groups in the epilogue."""
+    if cell == "lstm":
+        graphs = synth.config_batch("c3", 1, batch=16, V=32, C=32)
+        check("lstm", H, H, 32, graphs, 32, seed=40 + groups, groups=groups)
+    else:
+        check("childsum", H, H, 5, synth.config_batch("c2", 1), 4096, seed=50 + groups, groups=groups)
+
+
 def test_fused_sgd_update():
     graphs = _trees(6, 4, (1, 9), 20, 5)
     lr, wd = 0.05, 1e-3

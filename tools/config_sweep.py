@@ -26,6 +26,9 @@ CASES = [
     ("c3 LSTM-LM H256 B4 (V=C=32)", "c3", "lstm", 256, 256, 32, 32, 4, {}, {"V": 32, "C": 32}),
     ("c3 LSTM-LM H256 B16 (V=C=32)", "c3", "lstm", 256, 256, 32, 32, 16, {}, {"V": 32, "C": 32}),
     ("c3 LSTM-LM H256 B64 (V=C=32)", "c3", "lstm", 256, 256, 32, 32, 64, {}, {"V": 32, "C": 32}),
+    ("c2 child-sum H128 B16 G4", "c2", "childsum", 128, 128, 5, 4096, 16, {"groups": 4}, {}),
+    ("c3 LSTM-LM H256 B16 G2", "c3", "lstm", 256, 256, 32, 32, 16, {"groups": 2}, {"V": 32, "C": 32}),
+    ("c3 LSTM-LM H256 B64 G2", "c3", "lstm", 256, 256, 32, 32, 64, {"groups": 2}, {"V": 32, "C": 32}),
     ("tgt binary H256 B1 (dataflow)", "tgt", "binary", 256, 256, 5, 4096, 1, {"cluster": 16, "dataflow": True}, {}),
     ("tgt binary H256 B4 (dataflow)", "tgt", "binary", 256, 256, 5, 4096, 4, {"cluster": 16, "dataflow": True}, {}),
     ("tgt binary H256 B16 (dataflow)", "tgt", "binary", 256, 256, 5, 4096, 16, {"cluster": 16, "dataflow": True}, {}),
