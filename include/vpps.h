@@ -84,6 +84,12 @@ typedef struct {
                             cooperative launch (floor(n_sm / 16) groups) and the signal/wait of L165
                             is replaced by epoch-tagged 64-bit slots that consumers poll (vpps_df);
                             0 = barrier synchronisation. */
+    int32_t level;       /* binary cell only.  1: level-synchronous GEMM path — per level one dense
+                            product of the gathered children rows with the weights (PAPER L185's
+                            concatenation applied to every matrix use; weights L2-resident, plain
+                            FP32 SGEMM), fused cell / head / scatter kernels, dW as one GEMM per
+                            matrix.  0 = auto: chosen when no register-resident specialisation
+                            exists for (H, E) (config 5: H = E = 1024); -1 = never. */
 } vpps_options;
 
 /* A batch of graphs in CSR form (the super-graph of L205 is built from it).

@@ -69,6 +69,7 @@ struct vpps_model_s {
     bool dataflow = false;              // groups of co-resident CTAs synchronised by tagged slots (vpps_df)
     uint32_t* d_epoch = nullptr;        // dataflow pass counter on the device (slot tags), advanced per pass
     static constexpr int kMaxGroups = 16;
+    void* level = nullptr;              // level-synchronous path context (cuBLAS handle, work buffers)
     // Pre-allocated staging ring for per-batch scripts: a pinned host buffer and a
     // device buffer per slot; a slot is reused once the kernel that last read it has finished.
     struct Slot {
@@ -211,6 +212,21 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
         const Variant* v = variants(&nv);
         for (int32_t i = 0; i < nv; ++i)
             if (v[i].cell == cell && v[i].H == H && v[i].E == E && v[i].umax == m->plan.umax) m->var = &v[i];
+        const bool want_level = cell == CELL_BINARY && (o.level > 0 || (o.level == 0 && !m->var));
+        if (o.level > 0 && cell != CELL_BINARY) return fail(VPPS_E_INVALID, "the level path is built for the binary cell");
+        if (want_level) {
+            // level-synchronous GEMM path (vpps_level.cu): no register-resident specialisation needed
+            m->var = nullptr;
+            m->plan.level = true;
+            m->level = level_ctx_create();
+            if (!m->level) return fail(VPPS_E_CUDA, "cuBLAS initialisation failed");
+            CK(cudaMallocHost(&m->h_loss, 2 * sizeof(float)));
+            m->h_loss[0] = m->h_loss[1] = 0.f;
+            CK(cudaEventCreateWithFlags(&m->ev[0], cudaEventDisableTiming));
+            CK(cudaEventCreateWithFlags(&m->ev[1], cudaEventDisableTiming));
+            *out = m.release();
+            return VPPS_OK;
+        }
         if (!m->var)
             return fail(VPPS_E_NOFIT, "no kernel specialisation for cell " + std::to_string(cell) + " H=" +
                                           std::to_string(H) + " E=" + std::to_string(E) +
@@ -474,6 +490,15 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
                        m->offsets.data(), m->n_floats, mode, lr, wd, st, m->gemm_trace,
                        m->pool + s->s.loss_word, m->d_loss_map + (m->passes & 1));
         CK(cudaGetLastError());
+    } else if (m->plan.level) {
+        if (s->s.lv_int < 0) return fail(VPPS_E_INVALID, "script was not built for the level path");
+        CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));   // (memset above: G > 1 only)
+        const int rc = level_pass(m->level, m->params, m->offsets.data(), m->grads, m->pool, inputs, d_inputs, dwords,
+                                  s->s.lv_int, s->s.lv_leaf, s->s.lv_head, s->s.lv_start.data(),
+                                  (int32_t)s->s.lv_start.size() - 2, s->s.lv_n_int, s->s.lv_n_leaf, s->s.lv_n_head,
+                                  m->plan.H, m->plan.E, m->plan.C, s->s.loss_word, st);
+        if (rc != 0) return fail(VPPS_E_CUDA, "level pass failed (code " + std::to_string(rc) + ")");
+        if (mode == 1) launch_sgd(m->params, m->grads, m->n_floats, lr, wd, st);
     } else if (m->cluster) {
         // one cluster per replica group; clusters never wait on each other (graphs are whole per group).
         // Launch order: leaf GEMM (also clears the pass's accumulators) -> vpps_cl -> gradient GEMM
@@ -612,6 +637,7 @@ void vpps_destroy_script(vpps_script s) {
 
 void vpps_destroy_model(vpps_model m) {
     if (!m) return;
+    if (m->level) level_ctx_destroy(m->level);
     if (m->pool) cudaFree(m->pool);
     if (m->done) cudaFree(m->done);
     if (m->d_epoch) cudaFree(m->d_epoch);

@@ -34,6 +34,7 @@ struct Plan {
     int32_t cell, H, E, C;
     int32_t n_cta, n_g, n_act, umax, G;
     bool by_graph = false;   // SPEC S5g: whole graphs assigned to groups (cluster replicas)
+    bool level = false;      // level-synchronous GEMM path (binary cell, weights L2-resident)
     std::vector<int32_t> table;   // rows of 8 int32
 };
 bool unit_plan(int32_t cell, int32_t H, int32_t E, int32_t C, int32_t n_sm, int32_t cps, int32_t G,
@@ -67,6 +68,12 @@ struct Script {
     int64_t df_hx = 0, df_part = 0, df_hd = 0, df_words = 0;
     double flops = 0.0, act_bytes = 0.0;
     double kernel_flops = 0.0;   // binary whole-graph paths: FLOPs of the replica-group kernel alone
+    // level-synchronous path (Plan::level): blob word offsets of the internal-node list sorted by level
+    // (rec, rec_l, rec_r, adj, adj_l, adj_r), the leaf list (rec, adj, token) and the head list
+    // (rec, rec_c, adj_c, label); lv_start[l] = first internal node of level l (l = 1 .. L+1)
+    int64_t lv_int = -1, lv_leaf = -1, lv_head = -1;
+    int64_t lv_n_int = 0, lv_n_leaf = 0, lv_n_head = 0;
+    std::vector<int32_t> lv_start;
 };
 
 // Returns 0 on success, -4 (graph error) or -1 (invalid) with a message.

@@ -337,6 +337,38 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     }
     s.leaf_off[n_grp] = (int32_t)s.n_leaf;
 
+    // ---- level-synchronous lowering of the binary cell (Plan::level): per-level node lists ------
+    s.lv_int = s.lv_leaf = s.lv_head = -1;
+    s.lv_n_int = s.lv_n_leaf = s.lv_n_head = 0;
+    s.lv_start.clear();
+    if (plan.level && plan.cell == CELL_BINARY) {
+        s.lv_int = (int64_t)s.blob.size();
+        s.lv_start.assign(L + 2, 0);
+        for (int32_t lv = 1; lv <= L + 1; ++lv) {
+            s.lv_start[lv] = (int32_t)s.lv_n_int;
+            if (lv > L) break;
+            for (int64_t i : at_level[lv]) {
+                if (nodes[i].kind != K_INT) continue;
+                const int32_t* ch = kids.data() + nodes[i].ch_begin;
+                s.blob.insert(s.blob.end(), {rec[i], rec[ch[0]], rec[ch[1]], adj[i], adj[ch[0]], adj[ch[1]]});
+                ++s.lv_n_int;
+            }
+        }
+        s.lv_leaf = (int64_t)s.blob.size();
+        for (int64_t i = 0; i < N; ++i)
+            if (nodes[i].kind == K_LEAF) {
+                s.blob.insert(s.blob.end(), {rec[i], adj[i], (uint32_t)nodes[i].token});
+                ++s.lv_n_leaf;
+            }
+        s.lv_head = (int64_t)s.blob.size();
+        for (int64_t i = 0; i < N; ++i)
+            if (nodes[i].kind == K_HEAD) {
+                const int32_t* ch = kids.data() + nodes[i].ch_begin;
+                s.blob.insert(s.blob.end(), {rec[i], rec[ch[0]], adj[ch[0]], (uint32_t)nodes[i].label});
+                ++s.lv_n_head;
+            }
+    }
+
     // ---- dataflow lowering of the binary cell for whole-graph groups (vpps_df) ------------------
     // Per group: batches of <= 16 nodes of one opcode, forward levels 1..L then backward levels L..0
     // (level 0 leaves run as a GEMM before the kernel).  Cross-CTA values live in epoch-tagged 64-bit

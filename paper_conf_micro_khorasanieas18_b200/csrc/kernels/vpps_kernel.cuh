@@ -73,5 +73,12 @@ void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float*
                      uint32_t* epoch, cudaStream_t s);
 // Elementwise SGD on the flat buffer (K3): p -= lr * (g + wd * p).
 void launch_sgd(float* p, const float* g, int64_t n, float lr, float wd, cudaStream_t s);
+// Level-synchronous path (vpps_level.cu): context (cuBLAS handle + work buffers) and one training pass.
+void* level_ctx_create();
+void level_ctx_destroy(void* ctx);
+int level_pass(void* ctx, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
+               float* d_inputs, const uint32_t* d_blob, int64_t lv_int, int64_t lv_leaf, int64_t lv_head,
+               const int32_t* lv_start, int32_t L, int64_t n_int, int64_t n_leaf, int64_t n_head, int32_t H,
+               int32_t E, int32_t C, int64_t loss_word, cudaStream_t s);
 
 }  // namespace vpps

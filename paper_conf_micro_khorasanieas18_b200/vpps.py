@@ -36,7 +36,7 @@ class _Opset(ct.Structure):
 class _Options(ct.Structure):
     _fields_ = [("n_sm", ct.c_int32), ("ctas_per_sm", ct.c_int32), ("groups", ct.c_int32),
                 ("device", ct.c_int32), ("plan_only", ct.c_int32), ("cluster", ct.c_int32),
-                ("dataflow", ct.c_int32)]
+                ("dataflow", ct.c_int32), ("level", ct.c_int32)]
 
 
 class _Batch(ct.Structure):
@@ -235,12 +235,12 @@ class Model:
     """vpps_define_model + vpps_bind_buffers (PAPER L191: `vpps::handle hndl(model)`)."""
 
     def __init__(self, cell: str, H: int, E: int, C: int, device: int = 0, n_sm: int = 0, groups: int = 1,
-                 plan_only: bool = False, cluster: int = 0, dataflow: bool = False):
+                 plan_only: bool = False, cluster: int = 0, dataflow: bool = False, level: int = 0):
         self.cell, self.H, self.E, self.C = cell, H, E, C
         self.shapes = param_shapes(cell, H, E, C)
         sh = (_Shape * len(self.shapes))(*[_Shape(s[0], s[1] if len(s) == 2 else 1) for _, s in self.shapes])
         ops = _Opset(CELLS[cell], E, H, C)
-        opt = _Options(n_sm, 1, groups, device, int(plan_only), cluster, int(dataflow))
+        opt = _Options(n_sm, 1, groups, device, int(plan_only), cluster, int(dataflow), int(level))
         h = ct.c_void_p()
         _check(_lib.vpps_define_model(sh, len(self.shapes), ct.byref(ops), ct.byref(opt), ct.byref(h)))
         self._h = h

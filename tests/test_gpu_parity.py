@@ -20,13 +20,13 @@ def _vpps():
     return vpps
 
 
-def run_case(cell, H, E, C, graphs, V, seed=0, want_dx=True, sgd=None, groups=1, cluster=0, dataflow=False):
+def run_case(cell, H, E, C, graphs, V, seed=0, want_dx=True, sgd=None, groups=1, cluster=0, dataflow=False, level=0):
     vpps = _vpps()
     rng = np.random.default_rng(seed)
     shapes = vpps.param_shapes(cell, H, E, C)
     P = synth.init_params(shapes, rng)
     X = synth.input_table(rng, V, E)
-    m = vpps.Model(cell, H, E, C, device=0, groups=groups, cluster=cluster, dataflow=dataflow)
+    m = vpps.Model(cell, H, E, C, device=0, groups=groups, cluster=cluster, dataflow=dataflow, level=level)
     dev = torch.device("cuda:0")
     params = torch.zeros(m.n_floats, dtype=torch.float32, device=dev)
     grads = torch.full_like(params, float("nan"))
@@ -50,9 +50,9 @@ def rel(a, b):
     return float(np.abs(np.asarray(a, np.float64) - b).max() / max(np.abs(b).max(), 1e-30))
 
 
-def check(cell, H, E, C, graphs, V, seed=0, want_dx=True, groups=1, cluster=0, dataflow=False):
+def check(cell, H, E, C, graphs, V, seed=0, want_dx=True, groups=1, cluster=0, dataflow=False, level=0):
     m, P, X, loss, params, grads, dX = run_case(cell, H, E, C, graphs, V, seed, want_dx, groups=groups,
-                                                cluster=cluster, dataflow=dataflow)
+                                                cluster=cluster, dataflow=dataflow, level=level)
     lo, Go, dXo = M.forward_backward(cell, P, X, graphs, H)
     assert abs(loss - lo) <= TOL * abs(lo), (loss, lo)
     gv = m.views(grads.cpu())
@@ -203,6 +203,41 @@ def test_grid_replica_groups(cell, H, groups):
         check("lstm", H, H, 32, graphs, 32, seed=40 + groups, groups=groups)
     else:
         check("childsum", H, H, 5, synth.config_batch("c2", 1), 4096, seed=50 + groups, groups=groups)
+
+
+def test_level_path_target_batch():
+    """Level-synchronous GEMM path (vpps_level.cu) on the target config's shapes (H = E = 256)."""
+    check("binary", 256, 256, 5, synth.config_batch("tgt", 2), 4096, seed=61, level=1)
+
+
+def test_level_path_degenerate():
+    check("binary", 64, 64, 5, [[((), 3, 2)]], 8, level=1)                                # one labelled leaf
+    check("binary", 64, 32, 7, _trees(5, 3, (1, 9), 30, 7), 30, level=1, want_dx=False)
+    g = [((), 1, -1), ((), 0, -1), ((0, 1), -1, 3), ((), 2, -1), ((2, 3), -1, 1)]      # inner labels
+    check("binary", 64, 64, 5, [g], 4, level=1)
+
+
+def test_level_path_config5_small():
+    """Config 5's cell size (binary Tree-LSTM H = E = 1024) on a few small trees: the level path is what
+    define_model picks automatically when no register-resident specialisation exists."""
+    graphs = synth.config_batch("c5", 0, batch=3, leaves=(3, 9))
+    check("binary", 1024, 1024, 5, graphs, 4096, seed=62)
+
+
+def test_level_path_config5_full_batch_additivity():
+    """Config 5 at its full per-GPU size (64 SST-shaped trees, H = E = 1024), where the FP64 oracle is too
+    slow: the summed loss and every gradient are additive over a split of the batch (SURVEY c.5 batch
+    invariant, the property the DP all-reduce relies on), and the full batch's loss is finite."""
+    vpps = _vpps()
+    graphs = synth.config_batch("c5", 0)
+    res = []
+    for part in (graphs, graphs[:32], graphs[32:]):
+        _, _, _, loss, params, grads, dX = run_case("binary", 1024, 1024, 5, part, 4096, seed=63)
+        res.append((loss, grads.double().cpu().numpy(), dX.double().cpu().numpy()))
+    (l0, g0, x0), (l1, g1, x1), (l2, g2, x2) = res
+    assert np.isfinite(l0) and abs(l0 - (l1 + l2)) <= 1e-4 * abs(l0), (l0, l1 + l2)
+    assert rel(g1 + g2, g0) <= 1e-4
+    assert rel(x1 + x2, x0) <= 1e-4
 
 
 def test_fused_sgd_update():
