@@ -52,7 +52,10 @@ typedef struct vpps_script_s* vpps_script; /* owns one batch's encoded words (ho
 typedef enum {
     VPPS_CELL_LSTM = 0,
     VPPS_CELL_TREE_BINARY = 1,
-    VPPS_CELL_TREE_CHILDSUM = 2
+    VPPS_CELL_TREE_CHILDSUM = 2,
+    VPPS_CELL_BILSTM_TAGGER = 3   /* M2: forward + backward LSTM (i, f, o, g), per
+                                     position m = tanh(W_mlp [h→; h←] + b_mlp), tag head z = W_tag m +
+                                     b_tag; runs on the level-synchronous path (C <= 32 tags) */
 } vpps_cell;
 
 typedef struct {
@@ -60,12 +63,14 @@ typedef struct {
     int32_t E;    /* input (word-vector) length                           */
     int32_t H;    /* hidden length                                        */
     int32_t C;    /* classes of the softmax-NLL head          */
+    int32_t mlp;  /* BiLSTM tagger MLP width M (256); ignored by the other cells */
 } vpps_opset;
 
 /* Parameter shapes, matrices first then biases (bias = {n, 1}), in exactly this order:
  *   LSTM:          W 4H×E, U 4H×H, W_out C×H, b 4H, b_out C
  *   TREE_BINARY:   W_iou 3H×E, U_iou 3H×2H, U_fl H×H, U_fr H×H, W_out C×H, b_iou 3H, b_f H, b_out C
- *   TREE_CHILDSUM: W_iou 3H×E, W_f H×E, U_iou 3H×H, U_f H×H, W_out C×H, b_iou 3H, b_f H, b_out C */
+ *   TREE_CHILDSUM: W_iou 3H×E, W_f H×E, U_iou 3H×H, U_f H×H, W_out C×H, b_iou 3H, b_f H, b_out C
+ *   BILSTM_TAGGER: Wf 4H×E, Uf 4H×H, Wb 4H×E, Ub 4H×H, W_mlp M×2H, W_tag C×M, bf 4H, bb 4H, b_mlp M, b_tag C */
 typedef struct {
     int32_t rows, cols;
 } vpps_shape;

@@ -32,8 +32,11 @@ vpps_status cuda_fail(cudaError_t e, const char* what) {
         if (_e != cudaSuccess) return cuda_fail(_e, #call);    \
     } while (0)
 
-std::vector<Shape> expected_shapes(int32_t cell, int32_t H, int32_t E, int32_t C) {
+std::vector<Shape> expected_shapes(int32_t cell, int32_t H, int32_t E, int32_t C, int32_t M = 0) {
     switch (cell) {
+        case CELL_BILSTM:
+            return {{4 * H, E}, {4 * H, H}, {4 * H, E}, {4 * H, H}, {M, 2 * H}, {C, M},
+                    {4 * H, 1}, {4 * H, 1}, {M, 1}, {C, 1}};
         case CELL_LSTM: return {{4 * H, E}, {4 * H, H}, {C, H}, {4 * H, 1}, {C, 1}};
         case CELL_BINARY: return {{3 * H, E}, {3 * H, 2 * H}, {H, H}, {H, H}, {C, H}, {3 * H, 1}, {H, 1}, {C, 1}};
         case CELL_CHILDSUM: return {{3 * H, E}, {H, E}, {3 * H, H}, {H, H}, {C, H}, {3 * H, 1}, {H, 1}, {C, 1}};
@@ -110,9 +113,10 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     *out = nullptr;
     vpps_options o{};
     if (opt) o = *opt;
-    const int32_t cell = ops->cell, H = ops->H, E = ops->E, C = ops->C;
-    if (cell < 0 || cell > 2 || H <= 0 || E <= 0 || C <= 0) return fail(VPPS_E_INVALID, "bad op set");
-    std::vector<Shape> want = expected_shapes(cell, H, E, C);
+    const int32_t cell = ops->cell, H = ops->H, E = ops->E, C = ops->C, Mw = ops->mlp;
+    if (cell < 0 || cell > 3 || H <= 0 || E <= 0 || C <= 0) return fail(VPPS_E_INVALID, "bad op set");
+    if (cell == CELL_BILSTM && Mw <= 0) return fail(VPPS_E_INVALID, "BiLSTM tagger needs mlp > 0");
+    std::vector<Shape> want = expected_shapes(cell, H, E, C, Mw);
     if ((int32_t)want.size() != n_params) return fail(VPPS_E_INVALID, "wrong number of parameters for the op set");
     for (int32_t i = 0; i < n_params; ++i)
         if (params[i].rows != want[i].rows || params[i].cols != want[i].cols)
@@ -132,6 +136,30 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     }
     m->n_floats = cur;
     int32_t n_sm = o.n_sm;
+    if (cell == CELL_BILSTM) {
+        // M2 runs on the level-synchronous path only (vpps_level.cu): no partition plan
+        if (o.cluster > 1 || o.dataflow || o.level < 0) return fail(VPPS_E_INVALID, "BiLSTM tagger: level path only");
+        if (C > 32) return fail(VPPS_E_NOFIT, "tag head supports C <= 32 in v1");
+        if (H % 4 || E % 4) return fail(VPPS_E_INVALID, "H and E must be multiples of 4");
+        m->plan.cell = cell; m->plan.H = H; m->plan.E = E; m->plan.C = C; m->plan.mlp = Mw;
+        m->plan.n_cta = m->plan.n_g = m->plan.n_act = m->plan.umax = m->plan.G = 1;
+        m->plan.level = true;
+        if (!m->plan_only) {
+            m->device = o.device;
+            CK(cudaSetDevice(o.device));
+            cudaDeviceProp prop;
+            CK(cudaGetDeviceProperties(&prop, o.device));
+            if (prop.major != 10) return fail(VPPS_E_INVALID, "libvpps is built for sm_100a (B200) only");
+            m->level = level_ctx_create();
+            if (!m->level) return fail(VPPS_E_CUDA, "cuBLAS initialisation failed");
+            CK(cudaMallocHost(&m->h_loss, 2 * sizeof(float)));
+            m->h_loss[0] = m->h_loss[1] = 0.f;
+            CK(cudaEventCreateWithFlags(&m->ev[0], cudaEventDisableTiming));
+            CK(cudaEventCreateWithFlags(&m->ev[1], cudaEventDisableTiming));
+        }
+        *out = m.release();
+        return VPPS_OK;
+    }
     m->cluster = o.cluster > 1 ? o.cluster : 0;
     m->dataflow = m->cluster && o.dataflow;
     if (!m->plan_only) {
@@ -313,7 +341,8 @@ vpps_status vpps_build_script(vpps_model m, const vpps_batch* batch, vpps_script
     BatchIn b{batch->n_graphs, batch->graph_ptr, batch->child_ptr, batch->children, batch->token, batch->label};
     std::string err;
     // the input table's row count is not known here; token range is re-checked against it at run time
-    const int rc = build_script(m->plan, b, INT64_MAX, &s->s, &err);
+    const int rc = m->plan.cell == CELL_BILSTM ? build_tagger_script(m->plan, b, INT64_MAX, &s->s, &err)
+                                               : build_script(m->plan, b, INT64_MAX, &s->s, &err);
     if (rc != 0) return fail(rc == -4 ? VPPS_E_GRAPH : VPPS_E_INVALID, err);
     *out = s.release();
     return VPPS_OK;
@@ -490,6 +519,14 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
                        m->offsets.data(), m->n_floats, mode, lr, wd, st, m->gemm_trace,
                        m->pool + s->s.loss_word, m->d_loss_map + (m->passes & 1));
         CK(cudaGetLastError());
+    } else if (m->plan.level && m->plan.cell == CELL_BILSTM) {
+        CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));   // incl. padding
+        const int rc = tagger_pass(m->level, m->params, m->offsets.data(), m->grads, m->pool, inputs, d_inputs, dwords,
+                                   s->s.tg_tok, s->s.tg_lab, s->s.tg_fpos, s->s.tg_bpos, s->s.tg_start.data(),
+                                   (int32_t)s->s.tg_start.size() - 1, s->s.tg_T, m->plan.H, m->plan.E, m->plan.C,
+                                   m->plan.mlp, s->s.loss_word, st);
+        if (rc != 0) return fail(VPPS_E_CUDA, "tagger pass failed (code " + std::to_string(rc) + ")");
+        if (mode == 1) launch_sgd(m->params, m->grads, m->n_floats, lr, wd, st);
     } else if (m->plan.level) {
         if (s->s.lv_int < 0) return fail(VPPS_E_INVALID, "script was not built for the level path");
         CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));   // (memset above: G > 1 only)

@@ -9,7 +9,7 @@ namespace vpps {
 
 constexpr uint32_t NONE = 0xFFFFFFFFu;
 
-enum Cell : int32_t { CELL_LSTM = 0, CELL_BINARY = 1, CELL_CHILDSUM = 2 };
+enum Cell : int32_t { CELL_LSTM = 0, CELL_BINARY = 1, CELL_CHILDSUM = 2, CELL_BILSTM = 3 };
 
 enum Op : uint32_t {
     OP_S = 0x01, OP_W = 0x02,
@@ -32,6 +32,7 @@ int32_t paper_choose_cps(const std::vector<Shape>& mats, int32_t n_sm, int32_t t
 // ---- SPEC P1: unit-bundle plan --------------------------------------------------------------
 struct Plan {
     int32_t cell, H, E, C;
+    int32_t mlp = 0;         // BiLSTM tagger MLP width (256)
     int32_t n_cta, n_g, n_act, umax, G;
     bool by_graph = false;   // SPEC S5g: whole graphs assigned to groups (cluster replicas)
     bool level = false;      // level-synchronous GEMM path (binary cell, weights L2-resident)
@@ -74,9 +75,16 @@ struct Script {
     int64_t lv_int = -1, lv_leaf = -1, lv_head = -1;
     int64_t lv_n_int = 0, lv_n_leaf = 0, lv_n_head = 0;
     std::vector<int32_t> lv_start;
+    // BiLSTM tagger (CELL_BILSTM, level path): T positions (sentences concatenated), blob offsets of
+    // tok[T], lab[T], the forward step lists fpos[T] (positions of step t: sentences longer than t, in
+    // batch order, starting at fstart[t]) and the backward step lists bpos[T] (position len-1-t)
+    int64_t tg_T = 0, tg_tok = -1, tg_lab = -1, tg_fpos = -1, tg_bpos = -1;
+    std::vector<int32_t> tg_start;   // [maxlen + 1]
 };
 
 // Returns 0 on success, -4 (graph error) or -1 (invalid) with a message.
 int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Script* out, std::string* err);
+// BiLSTM tagger batches (chains: node t has child t-1 and a token; labels are tags < C).
+int build_tagger_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Script* out, std::string* err);
 
 }  // namespace vpps

@@ -1,0 +1,68 @@
+// Batch lowering of the BiLSTM tagger (M2; the NER tagger of Table III) for the
+// level-synchronous path: sentences are concatenated into T positions; time step t of the forward LSTM
+// runs position t of every sentence longer than t, step t of the backward LSTM position len-1-t (the
+// paper's level sort, L139, of the two chains).  The loss is the sum over labelled positions (L205).
+#include <algorithm>
+#include "host.h"
+
+namespace vpps {
+
+int build_tagger_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Script* out, std::string* err) {
+    if (b.n_graphs < 0 || (b.n_graphs > 0 && (!b.graph_ptr || !b.child_ptr || !b.token || !b.label))) {
+        *err = "null batch array";
+        return -1;
+    }
+    Script& s = *out;
+    s = Script{};
+    std::vector<int32_t> off(b.n_graphs + 1, 0), len(b.n_graphs, 0);
+    for (int32_t g = 0; g < b.n_graphs; ++g) {
+        const int32_t first = b.graph_ptr[g], last = b.graph_ptr[g + 1];
+        if (last < first) { *err = "graph_ptr not monotone"; return -4; }
+        for (int32_t v = first; v < last; ++v) {
+            const int32_t t = v - first, c0 = b.child_ptr[v], c1 = b.child_ptr[v + 1];
+            const bool ok = (t == 0 && c1 == c0) || (t > 0 && c1 == c0 + 1 && b.children[c0] == t - 1);
+            if (!ok) { *err = "BiLSTM tagger: node t has the single child t-1"; return -4; }
+            if (b.token[v] < 0 || b.token[v] >= n_input_rows) { *err = "token out of range"; return -4; }
+            if (b.label[v] < -1 || b.label[v] >= plan.C) { *err = "label out of range"; return -4; }
+            s.max_token = std::max<int64_t>(s.max_token, b.token[v]);
+            s.n_heads += b.label[v] >= 0;
+        }
+        len[g] = last - first;
+        off[g + 1] = off[g] + len[g];
+    }
+    const int32_t T = off[b.n_graphs];
+    const int32_t maxlen = b.n_graphs ? *std::max_element(len.begin(), len.end()) : 0;
+    s.tg_T = T;
+    s.n_nodes = T;
+    s.n_levels = maxlen;
+    s.tg_tok = (int64_t)s.blob.size();
+    for (int32_t g = 0; g < b.n_graphs; ++g)
+        for (int32_t t = 0; t < len[g]; ++t) s.blob.push_back((uint32_t)b.token[b.graph_ptr[g] + t]);
+    s.tg_lab = (int64_t)s.blob.size();
+    for (int32_t g = 0; g < b.n_graphs; ++g)
+        for (int32_t t = 0; t < len[g]; ++t) s.blob.push_back((uint32_t)b.label[b.graph_ptr[g] + t]);
+    s.tg_start.assign(maxlen + 1, 0);
+    s.tg_fpos = (int64_t)s.blob.size();
+    int32_t k = 0;
+    for (int32_t t = 0; t < maxlen; ++t) {
+        s.tg_start[t] = k;
+        for (int32_t g = 0; g < b.n_graphs; ++g)
+            if (len[g] > t) { s.blob.push_back((uint32_t)(off[g] + t)); ++k; }
+    }
+    s.tg_start[maxlen] = k;
+    s.tg_bpos = (int64_t)s.blob.size();
+    for (int32_t t = 0; t < maxlen; ++t)
+        for (int32_t g = 0; g < b.n_graphs; ++g)
+            if (len[g] > t) s.blob.push_back((uint32_t)(off[g] + len[g] - 1 - t));
+    // pool: the loss word only (the tagger's activations live in the path's work buffers)
+    s.loss_word = 0;
+    s.zero_words = 32;
+    s.pool_words = 32;
+    // algorithmic FLOPs: per position and direction 24H(E+H); per labelled position the
+    // MLP (2 x 2H x M x 3) and the tag head (2 x M x C x 3)
+    const double H = plan.H, E = plan.E, C = plan.C, M = plan.mlp;
+    s.flops = (double)T * 2.0 * 24.0 * H * (E + H) + (double)s.n_heads * (12.0 * H * M + 6.0 * M * C);
+    return 0;
+}
+
+}  // namespace vpps

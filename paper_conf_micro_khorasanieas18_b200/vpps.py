@@ -15,7 +15,7 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libvpps.so")
 
-CELLS = {"lstm": 0, "binary": 1, "childsum": 2}
+CELLS = {"lstm": 0, "binary": 1, "childsum": 2, "bilstm": 3}
 STATUS = {0: "OK", -1: "INVALID", -2: "NOFIT", -3: "CUDA", -4: "GRAPH", -5: "STATE", -6: "NOMEM"}
 
 
@@ -30,7 +30,7 @@ class _Shape(ct.Structure):
 
 
 class _Opset(ct.Structure):
-    _fields_ = [("cell", ct.c_int32), ("E", ct.c_int32), ("H", ct.c_int32), ("C", ct.c_int32)]
+    _fields_ = [("cell", ct.c_int32), ("E", ct.c_int32), ("H", ct.c_int32), ("C", ct.c_int32), ("mlp", ct.c_int32)]
 
 
 class _Options(ct.Structure):
@@ -111,8 +111,12 @@ def _stream_ptr(stream):
     return ct.c_void_p(stream.cuda_stream)
 
 
-def param_shapes(cell: str, H: int, E: int, C: int):
+def param_shapes(cell: str, H: int, E: int, C: int, mlp: int = 256):
     """Parameter order of vpps_define_model (include/vpps.h); bias shapes are (n,)."""
+    if cell == "bilstm":
+        return [("Wf", (4 * H, E)), ("Uf", (4 * H, H)), ("Wb", (4 * H, E)), ("Ub", (4 * H, H)),
+                ("W_mlp", (mlp, 2 * H)), ("W_tag", (C, mlp)),
+                ("bf", (4 * H,)), ("bb", (4 * H,)), ("b_mlp", (mlp,)), ("b_tag", (C,))]
     if cell == "lstm":
         return [("W", (4 * H, E)), ("U", (4 * H, H)), ("W_out", (C, H)), ("b", (4 * H,)), ("b_out", (C,))]
     if cell == "binary":
@@ -235,11 +239,12 @@ class Model:
     """vpps_define_model + vpps_bind_buffers (PAPER L191: `vpps::handle hndl(model)`)."""
 
     def __init__(self, cell: str, H: int, E: int, C: int, device: int = 0, n_sm: int = 0, groups: int = 1,
-                 plan_only: bool = False, cluster: int = 0, dataflow: bool = False, level: int = 0):
+                 plan_only: bool = False, cluster: int = 0, dataflow: bool = False, level: int = 0,
+                 mlp: int = 256):
         self.cell, self.H, self.E, self.C = cell, H, E, C
-        self.shapes = param_shapes(cell, H, E, C)
+        self.shapes = param_shapes(cell, H, E, C, mlp)
         sh = (_Shape * len(self.shapes))(*[_Shape(s[0], s[1] if len(s) == 2 else 1) for _, s in self.shapes])
-        ops = _Opset(CELLS[cell], E, H, C)
+        ops = _Opset(CELLS[cell], E, H, C, mlp)
         opt = _Options(n_sm, 1, groups, device, int(plan_only), cluster, int(dataflow), int(level))
         h = ct.c_void_p()
         _check(_lib.vpps_define_model(sh, len(self.shapes), ct.byref(ops), ct.byref(opt), ct.byref(h)))

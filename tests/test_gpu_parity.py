@@ -20,13 +20,14 @@ def _vpps():
     return vpps
 
 
-def run_case(cell, H, E, C, graphs, V, seed=0, want_dx=True, sgd=None, groups=1, cluster=0, dataflow=False, level=0):
+def run_case(cell, H, E, C, graphs, V, seed=0, want_dx=True, sgd=None, groups=1, cluster=0, dataflow=False, level=0,
+             mlp=256):
     vpps = _vpps()
     rng = np.random.default_rng(seed)
-    shapes = vpps.param_shapes(cell, H, E, C)
+    shapes = vpps.param_shapes(cell, H, E, C, mlp)
     P = synth.init_params(shapes, rng)
     X = synth.input_table(rng, V, E)
-    m = vpps.Model(cell, H, E, C, device=0, groups=groups, cluster=cluster, dataflow=dataflow, level=level)
+    m = vpps.Model(cell, H, E, C, device=0, groups=groups, cluster=cluster, dataflow=dataflow, level=level, mlp=mlp)
     dev = torch.device("cuda:0")
     params = torch.zeros(m.n_floats, dtype=torch.float32, device=dev)
     grads = torch.full_like(params, float("nan"))
@@ -50,9 +51,9 @@ def rel(a, b):
     return float(np.abs(np.asarray(a, np.float64) - b).max() / max(np.abs(b).max(), 1e-30))
 
 
-def check(cell, H, E, C, graphs, V, seed=0, want_dx=True, groups=1, cluster=0, dataflow=False, level=0):
+def check(cell, H, E, C, graphs, V, seed=0, want_dx=True, groups=1, cluster=0, dataflow=False, level=0, mlp=256):
     m, P, X, loss, params, grads, dX = run_case(cell, H, E, C, graphs, V, seed, want_dx, groups=groups,
-                                                cluster=cluster, dataflow=dataflow, level=level)
+                                                cluster=cluster, dataflow=dataflow, level=level, mlp=mlp)
     lo, Go, dXo = M.forward_backward(cell, P, X, graphs, H)
     assert abs(loss - lo) <= TOL * abs(lo), (loss, lo)
     gv = m.views(grads.cpu())
@@ -233,6 +234,32 @@ def test_level_path_config5_full_batch_additivity():
     res = []
     for part in (graphs, graphs[:32], graphs[32:]):
         _, _, _, loss, params, grads, dX = run_case("binary", 1024, 1024, 5, part, 4096, seed=63)
+        res.append((loss, grads.double().cpu().numpy(), dX.double().cpu().numpy()))
+    (l0, g0, x0), (l1, g1, x1), (l2, g2, x2) = res
+    assert np.isfinite(l0) and abs(l0 - (l1 + l2)) <= 1e-4 * abs(l0), (l0, l1 + l2)
+    assert rel(g1 + g2, g0) <= 1e-4
+    assert rel(x1 + x2, x0) <= 1e-4
+
+
+def test_tagger_small():
+    """BiLSTM tagger (M2, config 4's model) on the level path: small sizes, ragged sentence lengths."""
+    rng = np.random.default_rng(70)
+    graphs = synth.tagger_batch(rng, 3, (1, 8), 50, 9)
+    check("bilstm", 32, 32, 9, graphs, 50, seed=71, mlp=16)
+
+
+def test_tagger_config4_shapes():
+    """Config 4's sizes (H = E = 512, MLP 256, 9 tags) on a few short sentences."""
+    graphs = synth.config_batch("c4", 0, batch=4, lengths=(3, 12))
+    check("bilstm", 512, 512, 9, graphs, 4096, seed=72, mlp=256)
+
+
+def test_tagger_config4_full_batch_additivity():
+    """Config 4 at its full size (16 sentences of 5-60 tokens): loss and gradients additive over a split."""
+    graphs = synth.config_batch("c4", 1)
+    res = []
+    for part in (graphs, graphs[:8], graphs[8:]):
+        _, _, _, loss, params, grads, dX = run_case("bilstm", 512, 512, 9, part, 4096, seed=73, mlp=256)
         res.append((loss, grads.double().cpu().numpy(), dX.double().cpu().numpy()))
     (l0, g0, x0), (l1, g1, x1), (l2, g2, x2) = res
     assert np.isfinite(l0) and abs(l0 - (l1 + l2)) <= 1e-4 * abs(l0), (l0, l1 + l2)
