@@ -136,12 +136,12 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     }
     m->n_floats = cur;
     int32_t n_sm = o.n_sm;
-    if (cell == CELL_BILSTM) {
-        // M2 runs on the level-synchronous path only (vpps_level.cu): no partition plan
-        if (o.cluster > 1 || o.dataflow || o.level < 0) return fail(VPPS_E_INVALID, "BiLSTM tagger: level path only");
-        if (C > 32) return fail(VPPS_E_NOFIT, "tag head supports C <= 32 in v1");
+    if (cell == CELL_BILSTM || (cell == CELL_LSTM && (o.level > 0 || (o.level == 0 && C > 32)))) {
+        // M2 runs on the level-synchronous path only (vpps_level.cu), and so does an LSTM LM whose
+        // vocabulary head exceeds one CTA's shared memory (config 3 at V = 1000): no partition plan
+        if (o.cluster > 1 || o.dataflow || o.level < 0) return fail(VPPS_E_INVALID, "this op set runs on the level path only");
         if (H % 4 || E % 4) return fail(VPPS_E_INVALID, "H and E must be multiples of 4");
-        m->plan.cell = cell; m->plan.H = H; m->plan.E = E; m->plan.C = C; m->plan.mlp = Mw;
+        m->plan.cell = cell; m->plan.H = H; m->plan.E = E; m->plan.C = C; m->plan.mlp = cell == CELL_BILSTM ? Mw : 0;
         m->plan.n_cta = m->plan.n_g = m->plan.n_act = m->plan.umax = m->plan.G = 1;
         m->plan.level = true;
         if (!m->plan_only) {
@@ -341,8 +341,9 @@ vpps_status vpps_build_script(vpps_model m, const vpps_batch* batch, vpps_script
     BatchIn b{batch->n_graphs, batch->graph_ptr, batch->child_ptr, batch->children, batch->token, batch->label};
     std::string err;
     // the input table's row count is not known here; token range is re-checked against it at run time
-    const int rc = m->plan.cell == CELL_BILSTM ? build_tagger_script(m->plan, b, INT64_MAX, &s->s, &err)
-                                               : build_script(m->plan, b, INT64_MAX, &s->s, &err);
+    const bool chains = m->plan.level && (m->plan.cell == CELL_BILSTM || m->plan.cell == CELL_LSTM);
+    const int rc = chains ? build_tagger_script(m->plan, b, INT64_MAX, &s->s, &err)
+                          : build_script(m->plan, b, INT64_MAX, &s->s, &err);
     if (rc != 0) return fail(rc == -4 ? VPPS_E_GRAPH : VPPS_E_INVALID, err);
     *out = s.release();
     return VPPS_OK;
@@ -519,12 +520,19 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
                        m->offsets.data(), m->n_floats, mode, lr, wd, st, m->gemm_trace,
                        m->pool + s->s.loss_word, m->d_loss_map + (m->passes & 1));
         CK(cudaGetLastError());
-    } else if (m->plan.level && m->plan.cell == CELL_BILSTM) {
+    } else if (m->plan.level && (m->plan.cell == CELL_BILSTM || m->plan.cell == CELL_LSTM)) {
+        if (s->s.tg_tok < 0) return fail(VPPS_E_INVALID, "script was not built for the level path");
         CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));   // incl. padding
-        const int rc = tagger_pass(m->level, m->params, m->offsets.data(), m->grads, m->pool, inputs, d_inputs, dwords,
+        const bool bi = m->plan.cell == CELL_BILSTM;
+        const int64_t* o6 = m->offsets.data();
+        // (Wf, Uf, Wb, Ub, W_mlp, W_tag, bf, bb, b_mlp, b_tag); the LM: (W, U, -, -, -, W_out, b, -, -, b_out)
+        const int64_t off10[10] = {o6[0], o6[1], bi ? o6[2] : -1, bi ? o6[3] : -1, bi ? o6[4] : -1,
+                                   bi ? o6[5] : o6[2], bi ? o6[6] : o6[3], bi ? o6[7] : -1, bi ? o6[8] : -1,
+                                   bi ? o6[9] : o6[4]};
+        const int rc = tagger_pass(m->level, m->params, off10, m->grads, m->pool, inputs, d_inputs, dwords,
                                    s->s.tg_tok, s->s.tg_lab, s->s.tg_fpos, s->s.tg_bpos, s->s.tg_start.data(),
                                    (int32_t)s->s.tg_start.size() - 1, s->s.tg_T, m->plan.H, m->plan.E, m->plan.C,
-                                   m->plan.mlp, s->s.loss_word, st);
+                                   bi ? m->plan.mlp : 0, bi ? 2 : 1, s->s.loss_word, st);
         if (rc != 0) return fail(VPPS_E_CUDA, "tagger pass failed (code " + std::to_string(rc) + ")");
         if (mode == 1) launch_sgd(m->params, m->grads, m->n_floats, lr, wd, st);
     } else if (m->plan.level) {

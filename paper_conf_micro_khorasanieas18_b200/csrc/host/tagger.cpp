@@ -1,5 +1,5 @@
-// Batch lowering of the BiLSTM tagger (M2; the NER tagger of Table III) for the
-// level-synchronous path: sentences are concatenated into T positions; time step t of the forward LSTM
+// Batch lowering of LSTM chains for the level-synchronous path: the BiLSTM tagger (M2; PAPER L265, L281:
+// the NER tagger of Table III) and the LSTM LM with a large vocabulary (config 3): sentences are concatenated into T positions; time step t of the forward LSTM
 // runs position t of every sentence longer than t, step t of the backward LSTM position len-1-t (the
 // paper's level sort, L139, of the two chains).  The loss is the sum over labelled positions (L205).
 #include <algorithm>
@@ -61,7 +61,10 @@ int build_tagger_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows
     // algorithmic FLOPs: per position and direction 24H(E+H); per labelled position the
     // MLP (2 x 2H x M x 3) and the tag head (2 x M x C x 3)
     const double H = plan.H, E = plan.E, C = plan.C, M = plan.mlp;
-    s.flops = (double)T * 2.0 * 24.0 * H * (E + H) + (double)s.n_heads * (12.0 * H * M + 6.0 * M * C);
+    if (plan.cell == CELL_BILSTM)
+        s.flops = (double)T * 2.0 * 24.0 * H * (E + H) + (double)s.n_heads * (12.0 * H * M + 6.0 * M * C);
+    else   // LSTM LM: one direction, head on h
+        s.flops = (double)T * 24.0 * H * (E + H) + (double)s.n_heads * 6.0 * C * H;
     return 0;
 }
 

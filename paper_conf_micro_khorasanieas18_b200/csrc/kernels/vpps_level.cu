@@ -224,17 +224,17 @@ __global__ void tg_gather_x(const float* __restrict__ inputs, const uint32_t* __
 
 // rows of h_prev for the positions of one step: HH[pos + dp][d H .. d H + H)
 __global__ void tg_gather_hprev(const float* __restrict__ HH, const uint32_t* __restrict__ pos, int n, int dp, int d,
-                                int H, float* __restrict__ Hp) {
+                                int H, int HW, float* __restrict__ Hp) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)n * H) return;
     const int r = (int)(t / H), j = (int)(t % H);
-    Hp[t] = HH[(int64_t)((int)pos[r] + dp) * 2 * H + d * H + j];
+    Hp[t] = HH[(int64_t)((int)pos[r] + dp) * HW + d * H + j];
 }
 
 // LSTM step (M1, gates i f o g): a = P[pos] + Zs[r] (recurrent, absent at t = 0) + b
 __global__ void tg_cell(const float* __restrict__ P, const float* __restrict__ Zs, const float* __restrict__ b,
-                        const uint32_t* __restrict__ pos, int n, int dp, bool first, int d, int H, float* HH, float* Cd,
-                        float* Gd) {
+                        const uint32_t* __restrict__ pos, int n, int dp, bool first, int d, int H, int HW, float* HH,
+                        float* Cd, float* Gd) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)n * H) return;
     const int r = (int)(t / H), j = (int)(t % H);
@@ -246,7 +246,7 @@ __global__ void tg_cell(const float* __restrict__ P, const float* __restrict__ Z
     const float i = sigm(a[0]), f = sigm(a[1]), o = sigm(a[2]), g = tanhf(a[3]);
     const float cp = first ? 0.f : Cd[(p + dp) * H + j];
     const float c = f * cp + i * g;
-    HH[p * 2 * H + d * H + j] = o * tanhf(c);
+    HH[p * HW + d * H + j] = o * tanhf(c);
     Cd[p * H + j] = c;
     float* gr = Gd + p * 4 * H;
     gr[j] = i; gr[H + j] = f; gr[2 * H + j] = o; gr[3 * H + j] = g;
@@ -258,19 +258,24 @@ __global__ void tg_tanh_bias(float* A, const float* __restrict__ b, int64_t n, i
     if (t < n) A[t] = tanhf(A[t] + b[t % M]);
 }
 
-// tag head per position (warp per position, C <= 32): softmax-NLL of labelled positions -> loss, dZ
+// softmax-NLL head per position (warp per position, any C): labelled positions add their NLL to the loss
+// (L205) and get dZ = p - onehot(y); unlabelled positions get dZ = 0
 __global__ void tg_softmax(const float* __restrict__ Z, const float* __restrict__ b_tag, const uint32_t* __restrict__ lab,
                            int T, int C, float* dZ, float* loss) {
     const int w = (int)(((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5), lane = threadIdx.x & 31;
     if (w >= T) return;
     const int y = (int)lab[w];
-    const float z = lane < C ? Z[(int64_t)w * C + lane] + b_tag[lane] : -INFINITY;
-    if (y < 0) { if (lane < C) dZ[(int64_t)w * C + lane] = 0.f; return; }
-    const float m = warp_max(z);
-    const float lse = m + logf(warp_sum(lane < C ? expf(z - m) : 0.f));
-    const float zy = __shfl_sync(FULLMASK, z, y);
-    if (lane < C) dZ[(int64_t)w * C + lane] = expf(z - lse) - (lane == y ? 1.f : 0.f);
-    if (lane == 0) atomicAdd(loss, lse - zy);
+    const float* z = Z + (int64_t)w * C;
+    float* dz = dZ + (int64_t)w * C;
+    if (y < 0) { for (int c = lane; c < C; c += 32) dz[c] = 0.f; return; }
+    float m = -INFINITY;
+    for (int c = lane; c < C; c += 32) m = fmaxf(m, z[c] + b_tag[c]);
+    m = warp_max(m);
+    float se = 0.f;
+    for (int c = lane; c < C; c += 32) se += expf(z[c] + b_tag[c] - m);
+    const float lse = m + logf(warp_sum(se));
+    for (int c = lane; c < C; c += 32) dz[c] = expf(z[c] + b_tag[c] - lse) - (c == y ? 1.f : 0.f);
+    if (lane == 0) atomicAdd(loss, lse - (z[y] + b_tag[y]));
 }
 
 // dA = dM (1 - m^2) in place
@@ -281,14 +286,14 @@ __global__ void tg_dtanh(float* dM, const float* __restrict__ Mm, int64_t n) {
 
 // LSTM step backward (c.2b M1): dh = dHH[pos] (head) + dHr[pos] (from the next step), dc = dCr[pos];
 // γ -> Gam[pos] and the step buffer Gs[r]; dc_prev -> dCr[pos + dp]
-__global__ void tg_cell_bwd(const uint32_t* __restrict__ pos, int n, int dp, bool first, int d, int H,
+__global__ void tg_cell_bwd(const uint32_t* __restrict__ pos, int n, int dp, bool first, int d, int H, int HW,
                             const float* __restrict__ dHH, const float* __restrict__ dHr, float* dCr,
                             const float* __restrict__ Cd, const float* __restrict__ Gd, float* Gam, float* Gs) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)n * H) return;
     const int r = (int)(t / H), j = (int)(t % H);
     const int64_t p = pos[r];
-    const float dh = dHH[p * 2 * H + d * H + j] + dHr[p * H + j], dc = dCr[p * H + j];
+    const float dh = dHH[p * HW + d * H + j] + dHr[p * H + j], dc = dCr[p * H + j];
     const float* gr = Gd + p * 4 * H;
     const float i = gr[j], f = gr[H + j], o = gr[2 * H + j], g = gr[3 * H + j];
     const float c = Cd[p * H + j], cp = first ? 0.f : Cd[(p + dp) * H + j];
@@ -311,11 +316,11 @@ __global__ void tg_scatter_dh(const float* __restrict__ Dh, const uint32_t* __re
 
 // Hp_all[p] = h of p's predecessor in direction d (zeros at the chain start), for dU = Γᵀ Hp_all
 __global__ void tg_hprev_all(const float* __restrict__ HH, const uint32_t* __restrict__ pos, int n, int dp, int d,
-                             int H, float* Hp) {
+                             int H, int HW, float* Hp) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)n * H) return;
     const int r = (int)(t / H), j = (int)(t % H);
-    Hp[(int64_t)pos[r] * H + j] = HH[((int64_t)pos[r] + dp) * 2 * H + d * H + j];
+    Hp[(int64_t)pos[r] * H + j] = HH[((int64_t)pos[r] + dp) * HW + d * H + j];
 }
 
 __global__ void tg_scatter_dx(const float* __restrict__ DX, const uint32_t* __restrict__ tok, int T, int E, float* dX) {
@@ -484,8 +489,12 @@ int level_pass(void* ctx_, const float* params, const int64_t* off, float* grads
 int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
                 float* d_inputs, const uint32_t* d_blob, int64_t tg_tok, int64_t tg_lab, int64_t tg_fpos,
                 int64_t tg_bpos, const int32_t* start, int32_t maxlen, int64_t T, int32_t H, int32_t E, int32_t C,
-                int32_t Mw, int64_t loss_word, cudaStream_t s) {
+                int32_t Mw, int32_t dirs, int64_t loss_word, cudaStream_t s) {
+    // off: parameter offsets (Wf, Uf, Wb, Ub, W_mlp, W_tag, bf, bb, b_mlp, b_tag); dirs = 1 is the LSTM LM
+    // (M1: W, U, -, -, -, W_out, b, -, -, b_out; the head reads h directly), Mw = 0 without the MLP
     using namespace dev::lv;
+    const int HW = dirs * H;
+    const bool has_mlp = Mw > 0;
     LevelCtx* c = static_cast<LevelCtx*>(ctx_);
     TaggerBufs& tb = c->tg;
     cublasSetStream(c->blas, s);
@@ -493,49 +502,59 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
     float** bufs[24] = {&tb.X, &tb.Pf, &tb.Pb, &tb.HH, &tb.Cf, &tb.Cb, &tb.Gf, &tb.Gb, &tb.Hp, &tb.Zs, &tb.Mm, &tb.Z,
                         &tb.dZ, &tb.dM, &tb.dHH, &tb.dHf, &tb.dHb, &tb.dCf, &tb.dCb, &tb.Gamf, &tb.Gamb, &tb.Gs, &tb.Dh,
                         &tb.DX};
-    const int64_t need[24] = {Tn * E, Tn * 4 * H, Tn * 4 * H, Tn * 2 * H, Tn * H, Tn * H, Tn * 4 * H, Tn * 4 * H,
-                              Tn * H, Tn * 4 * H, Tn * Mw, Tn * C, Tn * C, Tn * Mw, Tn * 2 * H, Tn * H, Tn * H,
-                              Tn * H, Tn * H, Tn * 4 * H, Tn * 4 * H, Tn * 4 * H, Tn * H, Tn * E};
+    const int64_t Kh = has_mlp ? Mw : HW;         // width of the head's input
+    const int64_t need[24] = {Tn * E, Tn * 4 * H, Tn * 4 * H, Tn * HW, Tn * H, Tn * H, Tn * 4 * H, Tn * 4 * H,
+                              Tn * H, Tn * 4 * H, Tn * std::max<int64_t>(Mw, 1), Tn * C, Tn * C, Tn * Kh, Tn * HW,
+                              Tn * H, Tn * H, Tn * H, Tn * H, Tn * 4 * H, Tn * 4 * H, Tn * 4 * H, Tn * H, Tn * E};
     for (int k = 0; k < 24; ++k)
         if (!grow(bufs[k], &tb.cap[k], need[k])) return (int)cudaErrorMemoryAllocation;
-    const float *Wf = params + off[0], *Uf = params + off[1], *Wb = params + off[2], *Ub = params + off[3];
-    const float *Wm = params + off[4], *Wt = params + off[5], *bf = params + off[6], *bb = params + off[7];
-    const float *bm = params + off[8], *bt = params + off[9];
+    auto P_ = [&](int k) -> const float* { return off[k] >= 0 ? params + off[k] : nullptr; };
+    const float *Wf = P_(0), *Uf = P_(1), *Wb = P_(2), *Ub = P_(3), *Wm = P_(4), *Wt = P_(5), *bf = P_(6),
+                *bb = P_(7), *bm = P_(8), *bt = P_(9);
     const uint32_t *tok = d_blob + tg_tok, *lab = d_blob + tg_lab, *fpos = d_blob + tg_fpos, *bpos = d_blob + tg_bpos;
     cublasStatus_t st;
 #define BL(call) do { st = (call); if (st != CUBLAS_STATUS_SUCCESS) return 1000 + (int)st; } while (0)
     if (T == 0) return 0;
     tg_gather_x<<<nblk(T * (E / 4)), 256, 0, s>>>(inputs, tok, (int)T, E, tb.X);
     BL(gemm_rm(c->blas, false, true, (int)T, 4 * H, E, tb.X, E, Wf, E, tb.Pf, 4 * H, 0.f));
-    BL(gemm_rm(c->blas, false, true, (int)T, 4 * H, E, tb.X, E, Wb, E, tb.Pb, 4 * H, 0.f));
+    if (dirs > 1) BL(gemm_rm(c->blas, false, true, (int)T, 4 * H, E, tb.X, E, Wb, E, tb.Pb, 4 * H, 0.f));
     // forward over the time steps, both directions (independent chains)
     for (int32_t t = 0; t < maxlen; ++t) {
         const int32_t r0 = start[t], n = start[t + 1] - r0;
-        for (int d = 0; d < 2; ++d) {
+        for (int d = 0; d < dirs; ++d) {
             const uint32_t* pos = (d == 0 ? fpos : bpos) + r0;
             const int dp = d == 0 ? -1 : 1;
             const float* U = d == 0 ? Uf : Ub;
             if (t > 0) {
-                tg_gather_hprev<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.HH, pos, n, dp, d, H, tb.Hp);
+                tg_gather_hprev<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.HH, pos, n, dp, d, H, HW, tb.Hp);
                 BL(gemm_rm(c->blas, false, true, n, 4 * H, H, tb.Hp, H, U, H, tb.Zs, 4 * H, 0.f));
             }
             tg_cell<<<nblk((int64_t)n * H), 256, 0, s>>>(d == 0 ? tb.Pf : tb.Pb, tb.Zs, d == 0 ? bf : bb, pos, n, dp,
-                                                           t == 0, d, H, tb.HH, d == 0 ? tb.Cf : tb.Cb,
+                                                           t == 0, d, H, HW, tb.HH, d == 0 ? tb.Cf : tb.Cb,
                                                            d == 0 ? tb.Gf : tb.Gb);
         }
     }
-    // MLP + tag head over all positions (MLP 256), forward and backward
-    BL(gemm_rm(c->blas, false, true, (int)T, Mw, 2 * H, tb.HH, 2 * H, Wm, 2 * H, tb.Mm, Mw, 0.f));
-    tg_tanh_bias<<<nblk(T * Mw), 256, 0, s>>>(tb.Mm, bm, T * Mw, Mw);
-    BL(gemm_rm(c->blas, false, true, (int)T, C, Mw, tb.Mm, Mw, Wt, Mw, tb.Z, C, 0.f));
+    // head over all positions: BiLSTM tagger m = tanh(W_mlp [h→; h←] + b_mlp) (MLP 256), then
+    // z = W_tag m + b_tag; LSTM LM z = W_out h + b_out (L42); forward and backward
+    const float* Hin = tb.HH;
+    if (has_mlp) {
+        BL(gemm_rm(c->blas, false, true, (int)T, Mw, HW, tb.HH, HW, Wm, HW, tb.Mm, Mw, 0.f));
+        tg_tanh_bias<<<nblk(T * Mw), 256, 0, s>>>(tb.Mm, bm, T * Mw, Mw);
+        Hin = tb.Mm;
+    }
+    BL(gemm_rm(c->blas, false, true, (int)T, C, (int)Kh, Hin, (int)Kh, Wt, (int)Kh, tb.Z, C, 0.f));
     tg_softmax<<<nblk(T * 32), 256, 0, s>>>(tb.Z, bt, lab, (int)T, C, tb.dZ, pool + loss_word);
-    BL(gemm_rm(c->blas, true, false, C, Mw, (int)T, tb.dZ, C, tb.Mm, Mw, grads + off[5], Mw, 0.f));
+    BL(gemm_rm(c->blas, true, false, C, (int)Kh, (int)T, tb.dZ, C, Hin, (int)Kh, grads + off[5], (int)Kh, 0.f));
     colsum<<<nblk(C), 256, 0, s>>>(tb.dZ, (int)T, C, grads + off[9]);
-    BL(gemm_rm(c->blas, false, false, (int)T, Mw, C, tb.dZ, C, Wt, Mw, tb.dM, Mw, 0.f));
-    tg_dtanh<<<nblk(T * Mw), 256, 0, s>>>(tb.dM, tb.Mm, T * Mw);
-    BL(gemm_rm(c->blas, true, false, Mw, 2 * H, (int)T, tb.dM, Mw, tb.HH, 2 * H, grads + off[4], 2 * H, 0.f));
-    colsum<<<nblk(Mw), 256, 0, s>>>(tb.dM, (int)T, Mw, grads + off[8]);
-    BL(gemm_rm(c->blas, false, false, (int)T, 2 * H, Mw, tb.dM, Mw, Wm, 2 * H, tb.dHH, 2 * H, 0.f));
+    if (has_mlp) {
+        BL(gemm_rm(c->blas, false, false, (int)T, Mw, C, tb.dZ, C, Wt, Mw, tb.dM, Mw, 0.f));
+        tg_dtanh<<<nblk(T * Mw), 256, 0, s>>>(tb.dM, tb.Mm, T * Mw);
+        BL(gemm_rm(c->blas, true, false, Mw, HW, (int)T, tb.dM, Mw, tb.HH, HW, grads + off[4], HW, 0.f));
+        colsum<<<nblk(Mw), 256, 0, s>>>(tb.dM, (int)T, Mw, grads + off[8]);
+        BL(gemm_rm(c->blas, false, false, (int)T, HW, Mw, tb.dM, Mw, Wm, HW, tb.dHH, HW, 0.f));
+    } else {
+        BL(gemm_rm(c->blas, false, false, (int)T, HW, C, tb.dZ, C, Wt, HW, tb.dHH, HW, 0.f));
+    }
     // backward through both LSTMs, last step first
     cudaMemsetAsync(tb.dHf, 0, T * H * sizeof(float), s);
     cudaMemsetAsync(tb.dHb, 0, T * H * sizeof(float), s);
@@ -543,11 +562,11 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
     cudaMemsetAsync(tb.dCb, 0, T * H * sizeof(float), s);
     for (int32_t t = maxlen - 1; t >= 0; --t) {
         const int32_t r0 = start[t], n = start[t + 1] - r0;
-        for (int d = 0; d < 2; ++d) {
+        for (int d = 0; d < dirs; ++d) {
             const uint32_t* pos = (d == 0 ? fpos : bpos) + r0;
             const int dp = d == 0 ? -1 : 1;
             float* dHr = d == 0 ? tb.dHf : tb.dHb;
-            tg_cell_bwd<<<nblk((int64_t)n * H), 256, 0, s>>>(pos, n, dp, t == 0, d, H, tb.dHH, dHr, d == 0 ? tb.dCf : tb.dCb,
+            tg_cell_bwd<<<nblk((int64_t)n * H), 256, 0, s>>>(pos, n, dp, t == 0, d, H, HW, tb.dHH, dHr, d == 0 ? tb.dCf : tb.dCb,
                                                                d == 0 ? tb.Cf : tb.Cb, d == 0 ? tb.Gf : tb.Gb,
                                                                d == 0 ? tb.Gamf : tb.Gamb, tb.Gs);
             if (t > 0) {
@@ -557,14 +576,14 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
         }
     }
     // weight gradients: dW = Γᵀ X, dU = Γᵀ H_prev (zeros at chain starts), db = Σ Γ; dX = Γf Wf + Γb Wb
-    for (int d = 0; d < 2; ++d) {
+    for (int d = 0; d < dirs; ++d) {
         float* Gam = d == 0 ? tb.Gamf : tb.Gamb;
         const uint32_t* pos = d == 0 ? fpos : bpos;
         const int dp = d == 0 ? -1 : 1;
         cudaMemsetAsync(tb.Hp, 0, T * H * sizeof(float), s);
         if (maxlen > 1) {
             const int32_t n = start[maxlen] - start[1];
-            tg_hprev_all<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.HH, pos + start[1], n, dp, d, H, tb.Hp);
+            tg_hprev_all<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.HH, pos + start[1], n, dp, d, H, HW, tb.Hp);
         }
         BL(gemm_rm(c->blas, true, false, 4 * H, E, (int)T, Gam, 4 * H, tb.X, E, grads + off[d == 0 ? 0 : 2], E, 0.f));
         BL(gemm_rm(c->blas, true, false, 4 * H, H, (int)T, Gam, 4 * H, tb.Hp, H, grads + off[d == 0 ? 1 : 3], H, 0.f));
@@ -572,7 +591,7 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
     }
     if (d_inputs) {
         BL(gemm_rm(c->blas, false, false, (int)T, E, 4 * H, tb.Gamf, 4 * H, Wf, E, tb.DX, E, 0.f));
-        BL(gemm_rm(c->blas, false, false, (int)T, E, 4 * H, tb.Gamb, 4 * H, Wb, E, tb.DX, E, 1.f));
+        if (dirs > 1) BL(gemm_rm(c->blas, false, false, (int)T, E, 4 * H, tb.Gamb, 4 * H, Wb, E, tb.DX, E, 1.f));
         tg_scatter_dx<<<nblk(T * E), 256, 0, s>>>(tb.DX, tok, (int)T, E, d_inputs);
     }
 #undef BL

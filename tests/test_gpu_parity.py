@@ -267,6 +267,27 @@ def test_tagger_config4_full_batch_additivity():
     assert rel(x1 + x2, x0) <= 1e-4
 
 
+@pytest.mark.parametrize("batch", [1, 4])
+def test_lstm_lm_config3_vocab1000(batch):
+    """Config 3 as BASELINE states it (LSTM LM H = 256, V = 1000 next-token head, R-25): the vocabulary head
+    exceeds one CTA's shared memory, so define_model takes the level path (head as a dense product)."""
+    graphs = synth.config_batch("c3", 2, batch=batch, lengths=(5, 20))
+    check("lstm", 256, 256, 1000, graphs, 1000, seed=80 + batch)
+
+
+def test_lstm_lm_config3_full_batch_additivity():
+    graphs = synth.config_batch("c3", 3, batch=64)
+    res = []
+    for part in (graphs, graphs[:32], graphs[32:]):
+        m, _, _, loss, params, grads, dX = run_case("lstm", 256, 256, 1000, part, 1000, seed=84)
+        gv = m.views(grads.cpu())
+        res.append((loss, np.concatenate([gv[n].double().numpy().ravel() for n, _ in m.shapes]), dX.double().cpu().numpy()))
+    (l0, g0, x0), (l1, g1, x1), (l2, g2, x2) = res
+    assert np.isfinite(l0) and abs(l0 - (l1 + l2)) <= 1e-4 * abs(l0), (l0, l1 + l2)
+    assert rel(g1 + g2, g0) <= 1e-4
+    assert rel(x1 + x2, x0) <= 1e-4
+
+
 def test_fused_sgd_update():
     graphs = _trees(6, 4, (1, 9), 20, 5)
     lr, wd = 0.05, 1e-3
