@@ -141,8 +141,17 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
         // vocabulary head exceeds one CTA's shared memory (config 3 at V = 1000): no partition plan
         if (o.cluster > 1 || o.dataflow || o.level < 0) return fail(VPPS_E_INVALID, "this op set runs on the level path only");
         if (H % 4 || E % 4) return fail(VPPS_E_INVALID, "H and E must be multiples of 4");
-        m->plan.cell = cell; m->plan.H = H; m->plan.E = E; m->plan.C = C; m->plan.mlp = cell == CELL_BILSTM ? Mw : 0;
-        m->plan.n_cta = m->plan.n_g = m->plan.n_act = m->plan.umax = m->plan.G = 1;
+        if (cell == CELL_LSTM) {
+            // the partition plan (SPEC P1) stays defined for the op set (a bit-exact artifact) even though
+            // the level path does not place weights by it
+            std::string perr;
+            if (!unit_plan(cell, H, E, C, n_sm ? n_sm : 148, o.ctas_per_sm, o.groups, &m->plan, &perr))
+                return fail(perr.rfind("NOFIT", 0) == 0 ? VPPS_E_NOFIT : VPPS_E_INVALID, perr);
+        } else {
+            m->plan.cell = cell; m->plan.H = H; m->plan.E = E; m->plan.C = C;
+            m->plan.n_cta = m->plan.n_g = m->plan.n_act = m->plan.umax = m->plan.G = 1;
+        }
+        m->plan.mlp = cell == CELL_BILSTM ? Mw : 0;
         m->plan.level = true;
         if (!m->plan_only) {
             m->device = o.device;
@@ -342,8 +351,29 @@ vpps_status vpps_build_script(vpps_model m, const vpps_batch* batch, vpps_script
     std::string err;
     // the input table's row count is not known here; token range is re-checked against it at run time
     const bool chains = m->plan.level && (m->plan.cell == CELL_BILSTM || m->plan.cell == CELL_LSTM);
-    const int rc = chains ? build_tagger_script(m->plan, b, INT64_MAX, &s->s, &err)
-                          : build_script(m->plan, b, INT64_MAX, &s->s, &err);
+    int rc = 0;
+    if (chains && m->plan.cell == CELL_LSTM) {
+        // LSTM LM on the level path: the SPEC script (words, pool plan: a bit-exact artifact of the op set)
+        // plus the chain lists of the level path appended to the upload blob
+        Plan spec = m->plan;
+        spec.level = false;
+        rc = build_script(spec, b, INT64_MAX, &s->s, &err);
+        Script t;
+        if (rc == 0) rc = build_tagger_script(m->plan, b, INT64_MAX, &t, &err);
+        if (rc == 0) {
+            const int64_t shift = (int64_t)s->s.blob.size();
+            s->s.blob.insert(s->s.blob.end(), t.blob.begin(), t.blob.end());
+            s->s.tg_T = t.tg_T;
+            s->s.tg_tok = t.tg_tok + shift;
+            s->s.tg_lab = t.tg_lab + shift;
+            s->s.tg_fpos = t.tg_fpos + shift;
+            s->s.tg_bpos = t.tg_bpos + shift;
+            s->s.tg_start = t.tg_start;
+        }
+    } else {
+        rc = chains ? build_tagger_script(m->plan, b, INT64_MAX, &s->s, &err)
+                    : build_script(m->plan, b, INT64_MAX, &s->s, &err);
+    }
     if (rc != 0) return fail(rc == -4 ? VPPS_E_GRAPH : VPPS_E_INVALID, err);
     *out = s.release();
     return VPPS_OK;
