@@ -1075,7 +1075,10 @@ __global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
         }
     }
     __syncthreads();
-    constexpr int64_t CH = 16384;                          // floats per claimed chunk
+    // chunks of 4 float4 per thread with every load in flight before the first store (a strided
+    // load-update-store loop is one L2 round trip per iteration: params may alias grads for the compiler)
+    constexpr int CV = 4;                                  // float4 per thread per chunk
+    constexpr int64_t CH = 4 * CV * 256;                   // floats per claimed chunk
     const int64_t n_chunks = P.mode == 1 ? (P.n_floats + CH - 1) / CH : 0;
     while (true) {
         if (tid == 0) pick[0] = atomicAdd(P.tail_claim, 1);
@@ -1087,16 +1090,23 @@ __global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
             *reinterpret_cast<volatile float*>(P.loss_dst) = l;
         }
         if (c >= n_chunks) break;
-        const int64_t lo = c * CH, hi = min(P.n_floats, lo + CH);
+        const int64_t lo = c * CH, n4 = (min(P.n_floats, lo + CH) - lo) / 4;
         float4* p4 = reinterpret_cast<float4*>(P.params + lo);
         const float4* g4 = reinterpret_cast<const float4*>(P.grads + lo);
         const float lr = P.lr, wd = P.wd;
-        for (int64_t k = tid; k < (hi - lo) / 4; k += 256) {
-            float4 a = p4[k];
-            const float4 b = g4[k];
-            a.x -= lr * (b.x + wd * a.x); a.y -= lr * (b.y + wd * a.y);
-            a.z -= lr * (b.z + wd * a.z); a.w -= lr * (b.w + wd * a.w);
-            p4[k] = a;
+        float4 a[CV], b[CV];
+#pragma unroll
+        for (int q = 0; q < CV; ++q) {
+            const int64_t k = tid + 256 * q;
+            if (k < n4) { a[q] = __ldcg(p4 + k); b[q] = __ldcg(g4 + k); }
+        }
+#pragma unroll
+        for (int q = 0; q < CV; ++q) {
+            const int64_t k = tid + 256 * q;
+            if (k >= n4) break;
+            a[q].x -= lr * (b[q].x + wd * a[q].x); a[q].y -= lr * (b[q].y + wd * a[q].y);
+            a[q].z -= lr * (b[q].z + wd * a[q].z); a[q].w -= lr * (b[q].w + wd * a[q].w);
+            p4[k] = a[q];
         }
     }
 }

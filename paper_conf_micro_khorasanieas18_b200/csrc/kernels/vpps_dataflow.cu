@@ -28,7 +28,7 @@ constexpr int CHUNK = 4096;    // program words staged in shared memory
 constexpr int NB = 16;         // nodes per batch (LEAF_B: up to NBL)
 constexpr int NBL = 64;        // leaves per LEAF_B batch (no shared staging: one (unit, leaf) pair per thread pass)
 constexpr int MAXB = 1 + (NB * 9 > NBL * 4 ? NB * 9 : NBL * 4);   // words of the largest batch
-constexpr int NC = 2;          // nodes per transposed-product chunk
+constexpr int NC = 2;          // nodes per transposed-product chunk (two chunk buffers; 4 measured slower)
 constexpr int ZC = 32;         // classes per head (C <= 32)
 constexpr int CINMAX = 10;
 constexpr uint32_t NONE = 0xFFFFFFFFu;
@@ -77,12 +77,13 @@ struct DCfg {
     static constexpr int TH = H / (LB::CG * TU);
     static_assert(H % (LB::CG * TU) == 0, "h_l / h_r boundary on a granule-round boundary");
     static constexpr int O_X = CHUNK;                               // xs [NB][KP] floats
-    static constexpr int O_DXB = O_X + NB * KP;                     // dxb [UM][NC][KP] floats / u64 scratch
-    static constexpr int O_CIN = O_DXB + UM * NC * KP;
+    static constexpr int O_DXB = O_X + NB * KP;                     // dxb [2][NTH/32][NC][KP] floats / u64 scratch
+    static constexpr int DXB = 2 * (NTH / 32) * NC * KP;           // two buffers of 8 warp slices
+    static constexpr int O_CIN = O_DXB + DXB;
     static constexpr int O_BIAS = O_CIN + NB * UM * CINMAX;
     static constexpr int O_ZS = O_BIAS + UM * 4;
     static constexpr int O_HEAD = O_ZS + NB * ZC;
-    static_assert(UM * NC * KP >= 2 * NB * KP && UM * NC * KP >= 2 * NB * NCL * 2 * UM, "u64 staging fits in dxb");
+    static_assert(DXB >= 2 * NB * KP && DXB >= 2 * NB * NCL * 2 * UM, "u64 staging fits in dxb");
     static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 2 * C + 8); }
 };
 
@@ -212,10 +213,12 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         const bool stF = xst && op == INT_F && nb == 1 && !(xdone & 1);
         const bool stB = xst && op == INT_B && nb == 1 && !(xdone & 2);
         const bool stL = xst && op == LEAF_B && !(xdone & 4);
-        xdone |= (stF ? 1 : 0) | (stB ? 2 : 0) | (stL ? 4 : 0);
+        const bool stBB = xst && op == INT_B && nb >= 12 && !(xdone & 8);     // first big backward batch
+        xdone |= (stF ? 1 : 0) | (stB ? 2 : 0) | (stL ? 4 : 0) | (stBB ? 8 : 0);
 #define XST(f, k) do { if (f) xst[k] = clock64(); } while (0)
         XST(stF, 16);
         XST(stB, 22);
+        XST(stBB, 27);
         mark(1);
         if (op == LEAF_B) {
             // leaf backward, thread (leaf tid / U + 16 p, unit tid % U): consecutive threads read consecutive
@@ -422,6 +425,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             XST(stB, 25);
             __syncthreads();
             XST(stB, 26);
+            XST(stBB, 28);
         }
         if (bt) { bt[2] = clock64(); bt[4] |= (uint64_t)rounds << 8; }
 
@@ -599,11 +603,20 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             }
             mark(5);
             XST(stB, 6);
+            XST(stBB, 29);
             // transposed products (L94, fn4): per node, this CTA's partial dx = Σ_r W[r] g_r over all 2H
-            // columns; the 16 unit slices are summed in shared memory and published as tagged PART slots
+            // columns.  The two units of a warp are pre-summed with one shuffle exchange (lane l keeps the
+            // even or odd granules of the pair, l ^ 16 the others), the 8 warp slices are summed in shared
+            // memory and published as tagged PART slots.  Chunks of NC nodes alternate between two
+            // buffers, so one barrier per chunk separates a chunk's stores from its reduction and the
+            // reduction of chunk c overlaps the products of chunk c + 1.
             if (kindB) {
+                constexpr int NW = NTH / 32;
                 const int src = lane & 16;
-                for (int n0 = 0; n0 < nb; n0 += NC) {
+                const bool hi = lane & 16;
+                int cbuf = 0;
+                for (int n0 = 0; n0 < nb; n0 += NC, cbuf ^= 1) {
+                    float* buf = dxb + cbuf * (NW * NC * KP);
 #pragma unroll
                     for (int dn = 0; dn < NC; ++dn) {
                         const int n = n0 + dn;
@@ -611,24 +624,35 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                         float gr[5];
 #pragma unroll
                         for (int r = 0; r < 5; ++r) gr[r] = __shfl_sync(FULLMASK, g[r], src | (n & 15));
-                        float* drow = dxb + (u * NC + dn) * KP;
+                        float* drow = buf + (warp * NC + dn) * KP;
 #pragma unroll
-                        for (int t = 0; t < LB::NT; ++t) {
-                            const int col0 = LB::CG * (tu + TU * t);
-                            const float gf = t < T::TH ? gr[3] : gr[4];
-                            float dx[LB::CG];
+                        for (int t = 0; t < LB::NT; t += 2) {
+                            // granules t, t + 1; lanes < 16 keep granule t, lanes >= 16 granule t + 1 (the
+                            // partner lane l ^ 16 holds the same columns of the warp's other unit)
+                            float dx[2][LB::CG];
 #pragma unroll
-                            for (int q = 0; q < LB::CG; q += 2) {
-                                const int k = t * LB::CG + q;
-                                float2 d = __ffma2_rn(make_float2(wb[0][k], wb[0][k + 1]), make_float2(gr[0], gr[0]),
-                                                      make_float2(0.f, 0.f));
-                                d = __ffma2_rn(make_float2(wb[1][k], wb[1][k + 1]), make_float2(gr[1], gr[1]), d);
-                                d = __ffma2_rn(make_float2(wb[2][k], wb[2][k + 1]), make_float2(gr[2], gr[2]), d);
-                                d = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), make_float2(gf, gf), d);
-                                dx[q] = d.x;
-                                dx[q + 1] = d.y;
+                            for (int h = 0; h < 2; ++h) {
+                                const float gf = t + h < T::TH ? gr[3] : gr[4];
+#pragma unroll
+                                for (int q = 0; q < LB::CG; q += 2) {
+                                    const int k = (t + h) * LB::CG + q;
+                                    float2 d = __ffma2_rn(make_float2(wb[0][k], wb[0][k + 1]), make_float2(gr[0], gr[0]),
+                                                          make_float2(0.f, 0.f));
+                                    d = __ffma2_rn(make_float2(wb[1][k], wb[1][k + 1]), make_float2(gr[1], gr[1]), d);
+                                    d = __ffma2_rn(make_float2(wb[2][k], wb[2][k + 1]), make_float2(gr[2], gr[2]), d);
+                                    d = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), make_float2(gf, gf), d);
+                                    dx[h][q] = d.x;
+                                    dx[h][q + 1] = d.y;
+                                }
                             }
-                            sts_granule<LB::CG>(drow + col0, dx, n < nb);
+                            float kv[LB::CG];
+#pragma unroll
+                            for (int q = 0; q < LB::CG; ++q) {
+                                const float send = hi ? dx[0][q] : dx[1][q];
+                                kv[q] = (hi ? dx[1][q] : dx[0][q]) + __shfl_xor_sync(FULLMASK, send, 16);
+                            }
+                            const int col0 = LB::CG * (tu + TU * (t + (hi ? 1 : 0)));
+                            sts_granule<LB::CG>(drow + col0, kv, true);
                         }
                     }
                     XST(stB, 7);
@@ -638,26 +662,27 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                     for (int i = tid; i < NC * q4; i += NTH) {
                         const int dn = i / q4, c = (i - dn * q4) * 4, n = n0 + dn;
                         if (n >= nb) continue;
-                        float s[4] = {0.f, 0.f, 0.f, 0.f};
+                        float s4[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
-                        for (int uu = 0; uu < UM; ++uu) {
-                            const float4 x = *reinterpret_cast<const float4*>(dxb + (uu * NC + dn) * KP + c);
-                            s[0] += x.x; s[1] += x.y; s[2] += x.z; s[3] += x.w;
+                        for (int w = 0; w < NW; ++w) {
+                            const float4 x = *reinterpret_cast<const float4*>(buf + (w * NC + dn) * KP + c);
+                            s4[0] += x.x; s4[1] += x.y; s4[2] += x.z; s4[3] += x.w;
                         }
                         // column c: child side = c / H, unit jj = c % H, owner CTA m = jj / U, slot jj % U
                         const int side = c >= H, jj = c - side * H, m = jj / UM;
                         const uint32_t pp = ent[n * sz + 4];
-                        st_tag4(PART + ((((int64_t)pp * NCL + m) * NCL + lc) * 2 + side) * UM + (jj - m * UM), s, ep);
+                        st_tag4(PART + ((((int64_t)pp * NCL + m) * NCL + lc) * 2 + side) * UM + (jj - m * UM), s4, ep);
                     }
                     XST(stB, 9);
-                    __syncthreads();
                     XST(stB, 10);
                 }
+                XST(stBB, 30);
             }
         }
         __syncthreads();
         XST(stF, 4);
         XST(stB, 11);
+        XST(stBB, 31);
         if (bt) bt[3] = clock64();
         pos = next;
     }

@@ -115,6 +115,9 @@ def main():
             if x[5] > 0:
                 print("  INT_B nb=1 compute: cell-bwd %.0f, tmv+sts %.0f, bar %.0f, reduce+st %.0f, bar %.0f, end bar %.0f" %
                       (x[6] - x[5], x[7] - x[6], x[8] - x[7], x[9] - x[8], x[10] - x[9], x[11] - x[10]))
+            if x[27] > 0:
+                print("  INT_B big batch: staging %.0f, cell-bwd %.0f, transposed chunks %.0f, end bar %.0f" %
+                      (x[28] - x[27], x[29] - x[28], x[30] - x[29], x[31] - x[30]))
             if x[12] > 0:
                 print("  LEAF_B iter0: poll %.0f, compute+stores %.0f; loop total from iter0 issue %.0f" %
                       (x[13] - x[12], x[14] - x[13], x[15] - x[12]))
