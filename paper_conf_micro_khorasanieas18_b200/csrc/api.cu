@@ -528,8 +528,13 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         cfg.blockDim = dim3(256);
         cfg.dynamicSmemBytes = m->smem;
         cfg.stream = st;
+        // programmatic dependent of the leaf kernel: its launch overlaps the leaf grid's tail; the kernel
+        // executes griddepcontrol.wait before it reads the leaf records, the pass counter or `done`
+        static const bool no_pdl_df = getenv("VPPS_DF_NOPDL") != nullptr;   // measurement only
+        attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        attr[1].val.programmaticStreamSerializationAllowed = 1;
         cfg.attrs = attr;
-        cfg.numAttrs = 1;       // ordinary stream order after the leaf kernel (which clears `done`)
+        cfg.numAttrs = no_pdl_df ? 1 : 2;
         const uint32_t* lists = dwords + s->s.words.size();
         const uint32_t* leaf_list = lists + 3 * s->s.n_int;
         const float* W_iou = m->params + m->offsets[0];

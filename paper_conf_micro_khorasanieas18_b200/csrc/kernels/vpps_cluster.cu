@@ -1016,6 +1016,8 @@ __global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
         if constexpr (TC) tc_teardown();
         return;
     }
+    // (claiming the group's next item ahead, while the current one runs, was measured slower: at the
+    // end the last group's items pile up on the CTAs that claimed ahead)
     while (true) {
         if (tid < 32) {
             // lane q looks at group grp[q] (all groups in one parallel round trip); the first eligible
@@ -1048,9 +1050,10 @@ __global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
         if (g >= 0) {
             const uint64_t t0 = P.trace ? gtimer() : 0;
             dw_item<TC>(P, g, i, dsm, idx);
-            __threadfence();
+            // the item's reductions into grads / dX are ordered before the count by the barrier and
+            // thread 0's release (cumulative), as the SGD tail acquires `fin`
             __syncthreads();
-            if (tid == 0) atomicAdd(P.fin, 1);
+            if (tid == 0) asm volatile("red.release.gpu.global.add.s32 [%0], 1;" ::"l"(P.fin) : "memory");
             if (P.trace && tid == 0) {
                 int k = 0;
                 for (int q = 0; q < g; ++q) k += P.items[q];

@@ -119,7 +119,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     const int j = lc * UM + u;                                  // hidden unit of this thread (blocked)
     const bool holds_head = (lc == 0);
 
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     if (P.prof && threadIdx.x == 0) P.prof[(int64_t)blockIdx.x * P.prof_stride + 11] = gtimer();   // entry
     // ---- prologue: this CTA's rows of U_iou, U_fl, U_fr -> registers (L123, L129) ----
     float wb[4][LB::NREG];
@@ -174,6 +173,10 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     };
     // the leaf records and the pass counter (vpps_leaf_fwd, the preceding grid) are visible from here on
     asm volatile("griddepcontrol.wait;" ::: "memory");
+    // the gradient GEMM (programmatic dependent of this grid) may launch from here on: it reads the
+    // `done` / claim counters the leaf grid cleared, which is complete and visible once every CTA of this
+    // grid has passed the wait above
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     ep = *P.epoch;
     __syncthreads();
     if (prof && tid == 0) { prof[0] = gtimer(); sec_last = clock64(); }

@@ -64,6 +64,9 @@ __global__ void __launch_bounds__(NT + NTC, 1) vpps_leaf_fwd(const float* __rest
     float* As = lsm;                 // [64 leaves][KS]: x rows
     float* Bs = lsm + LM * KS;       // [48 rows][KS]: W_iou rows g*H + j0 + uu, row index g*16 + uu
     const int tid = threadIdx.x;
+    // the dataflow kernel may be scheduled as SMs free up (it waits for this grid with griddepcontrol.wait
+    // before reading anything written here)
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     const bool pf = g_leaf_prof_on && tid == 0 && blockIdx.x < 1024;
     uint64_t* pst = g_leaf_prof + blockIdx.x * 8;
     if (pf) pst[0] = gtimer();
@@ -81,6 +84,7 @@ __global__ void __launch_bounds__(NT + NTC, 1) vpps_leaf_fwd(const float* __rest
             const int64_t n4 = pc.ptr[r] ? pc.n[r] / 4 : 0;
             for (int64_t i = (int64_t)blockIdx.x * NTC + (tid - NT); i < n4; i += stride) p[i] = make_float4(0.f, 0.f, 0.f, 0.f);
         }
+        if (g_leaf_prof_on && tid == NT && blockIdx.x < 1024) g_leaf_prof[blockIdx.x * 8 + 6] = gtimer();
         return;
     }
     if (work) {

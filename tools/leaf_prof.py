@@ -48,9 +48,9 @@ def main():
         work = b[:, 2] > 0
         rel = (b - t0) / 1e3
         print(f"step {step}: CTAs {len(b)}, working {work.sum()}")
-        names = ["entry", "issued+cleared", "K0 landed", "K3 landed", "FMA done", "exit"]
+        names = ["entry", "issued", "K0 landed", "K3 landed", "FMA done", "exit", "clear done"]
         for k, nm in enumerate(names):
-            sel = rel[work, k] if k >= 2 else rel[:, k]
+            sel = rel[work, k] if 2 <= k <= 5 else rel[:, k]
             print(f"  {nm:15s} min {sel.min():6.2f} mean {sel.mean():6.2f} max {sel.max():6.2f} us")
         b[:] = 0
         buf[:] = 0
