@@ -108,7 +108,7 @@ class ClockSampler:
                 "samples": len(self.sm), "source": "nvml" if self.nvml else "nvidia-smi"}
 
 
-PROFILE_TAG = "r02"     # profiles/<tag>_ncu_summary.json: ncu capture of the kernels this bench times
+PROFILE_TAG = "r03"     # profiles/<tag>_ncu_summary.json: ncu capture of the kernels this bench times
 
 
 def make_batches(rank: int, batch: int):
@@ -304,13 +304,13 @@ def main():
     # ---- end to end through the public API: host script build + one H2D copy + kernel + loss D2H ----
     e2e_steps = min(args.steps, 200)
     h2d = 0
+    csr = [vpps.CsrBatch.from_graphs(g) for g in batches]   # the data loader's output: CSR batches (API input)
     if dist:
         dist.barrier()
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    csr = [vpps.CsrBatch.from_graphs(g) for g in batches]   # the data loader's output format (CSR)
-    # host: super-graph, levels, schedule, encode — built a few batches ahead on a background thread
-    for k, s in enumerate(vpps.prefetch_scripts(m, (csr[k % N_BATCHES] for k in range(e2e_steps)))):
+    # host: super-graph, levels, schedule, encode — built a few batches ahead by 3 background workers
+    for k, s in enumerate(vpps.prefetch_scripts(m, (csr[k % N_BATCHES] for k in range(e2e_steps)), workers=3)):
         h2d += s.info()["blob_words"] * 4            # staged by the call below: one pinned H2D copy (L169)
         if world == 1:
             m.fwd_bwd_sgd(s, inputs, d_inputs, lr=lr, weight_decay=wd)
@@ -341,13 +341,15 @@ def main():
         else:
             dom_avg_ms, dom_avg_flops, achieved = kern_ms / args.steps, avg_flops, step_tflops
         w_once = 4 * sum(int(np.prod(s)) for _, s in shapes if len(s) == 2)
-        traffic = None
+        traffic = inpipe = None
         prof = os.path.join(ROOT, "profiles", f"{PROFILE_TAG}_ncu_summary.json")
         if os.path.exists(prof):
             try:
-                traffic = json.load(open(prof)).get("dram_bytes_per_launch")
+                pj = json.load(open(prof))
+                traffic = pj.get("dram_bytes_per_launch")
+                inpipe = pj.get("in_pipeline")
             except Exception:
-                traffic = None
+                traffic = inpipe = None
         line = {
             "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": step_ms / args.steps, "higher_is_better": True,
@@ -370,11 +372,18 @@ def main():
                          "step_kernels_ms": kern_ms / args.steps, "step_flops": avg_flops,
                          "step_tflops": step_tflops,
                          "peak_note": "FP32 FFMA: 148 SM x 128 lanes x 2 FLOP x sm_max_mhz (derived, DESIGN.md)"},
-            "dram": {"weights_once_bytes": w_once, "dram_bytes_per_pass": traffic,
-                     "source": f"profiles/{PROFILE_TAG}_ncu_summary.json (ncu --set full, dominant kernel)" if traffic else None},
+            "dram": {"weights_once_bytes": w_once,
+                     "dominant_kernel_cold_bytes": traffic,
+                     "pass_read_bytes_in_pipeline": inpipe["pass_dram_read_bytes"] if inpipe else None,
+                     "pass_read_vs_weights_once": (inpipe["pass_dram_read_bytes"] / w_once) if inpipe else None,
+                     "pass_write_bytes_in_pipeline": inpipe["pass_dram_write_bytes"] if inpipe else None,
+                     "note": "cold: ncu --set full of the dominant kernel (caches flushed per replay); in pipeline: "
+                             "ncu --cache-control none over bench steps, all kernels of a pass (writes include "
+                             "evictions of the L2-flush buffer's dirty lines)",
+                     "source": f"profiles/{PROFILE_TAG}_ncu_summary.json" if traffic else None},
             "e2e": {"value": e2e_steps * args.batch * world / e2e_s, "unit": "samples/s",
                     "h2d_bytes_per_step": h2d // e2e_steps, "d2h_bytes_per_step": 4,
-                    "includes": "host script build from CSR batches (background thread, 3 ahead) + pinned H2D copy + kernels (+ all-reduce) + loss D2H (stale-loss read)"},
+                    "includes": "per step: host script build from the step's CSR batch (3 builder threads, 4 ahead) + pinned H2D copy of the script + kernels (+ all-reduce) + loss D2H (stale-loss read); CSR batches are the data loader's output, made before the timed region"},
             "clocks": clk,
         }
         if world == 1 and not args.no_cpu_baseline:

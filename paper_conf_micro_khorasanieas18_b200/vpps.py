@@ -178,32 +178,25 @@ class CsrBatch:
         return cls(*to_csr(graphs))
 
 
-def prefetch_scripts(model: "Model", batches, depth: int = 3):
-    """Yield model.build_script(b) for b in batches, built `depth` ahead on a background thread (the C++
-    builder runs without the GIL), so host script generation overlaps the device pass."""
-    import queue
-    import threading
-    q = queue.Queue(maxsize=depth)
-    done = object()
-
-    def work():
-        try:
-            for b in batches:
-                q.put(model.build_script(b))
-        except BaseException as e:   # surface builder errors in the consumer
-            q.put(e)
-        q.put(done)
-
-    th = threading.Thread(target=work, daemon=True)
-    th.start()
-    while True:
-        item = q.get()
-        if item is done:
-            break
-        if isinstance(item, BaseException):
-            raise item
-        yield item
-    th.join()
+def prefetch_scripts(model: "Model", batches, depth: int = 4, workers: int = 3):
+    """Yield model.build_script(b) for b in batches, in order, built up to `depth` ahead by `workers`
+    background threads (the C++ builder runs without the GIL), so host script generation
+    overlaps the device passes: one builder takes ~200 us per 16-tree batch, longer than a device step."""
+    import collections
+    from concurrent.futures import ThreadPoolExecutor
+    it = iter(batches)
+    with ThreadPoolExecutor(max_workers=max(1, workers)) as ex:
+        pend = collections.deque()
+        for b in it:
+            pend.append(ex.submit(model.build_script, b))
+            if len(pend) >= depth:
+                break
+        while pend:
+            s = pend.popleft().result()      # re-raises a builder error in the consumer
+            for b in it:
+                pend.append(ex.submit(model.build_script, b))
+                break
+            yield s
 
 
 class Script:

@@ -78,6 +78,24 @@ def main():
                                          "share_of_step": (sum(v) / tot if k != "FillFunctor" else None)}
                                      for k, v in per.items()}
         shutil.copy(launches, os.path.join(out_dir, f"{tag}_launches.csv"))
+    # in-pipeline DRAM (ncu --cache-control none over a bench run, L2 flush kernel between steps): what a
+    # real pass reads from / writes to DRAM; writes include evictions of the flush buffer's dirty lines
+    inpipe = os.path.join(ROOT, "gpurun_out", f"dram_inpipe_{tag}.csv")
+    if os.path.exists(inpipe):
+        lrows = [r for r in csv.DictReader(l for l in open(inpipe) if not l.startswith("=="))]
+        per = collections.defaultdict(lambda: collections.defaultdict(list))
+        for r in lrows:
+            v = float(r["Metric Value"]) * SCALE.get(r.get("Metric Unit", "byte"), 1.0)
+            per[short(r["Kernel Name"])][r["Metric Name"]].append(v)
+        ip = {k: {m: sum(l) / len(l) for m, l in d.items()} | {"launches": len(next(iter(d.values())))}
+              for k, d in per.items()}
+        pass_k = [k for k in ip if k != "FillFunctor"]
+        summary["in_pipeline"] = {
+            "capture": "ncu --cache-control none --clock-control none (bench steps, 256 MiB L2 flush between steps)",
+            "kernels": ip,
+            "pass_dram_read_bytes": sum(ip[k].get("dram__bytes_read.sum", 0.0) for k in pass_k),
+            "pass_dram_write_bytes": sum(ip[k].get("dram__bytes_write.sum", 0.0) for k in pass_k)}
+        shutil.copy(inpipe, os.path.join(out_dir, f"{tag}_dram_inpipe.csv"))
     with open(os.path.join(out_dir, f"{tag}_ncu_summary.json"), "w") as f:
         json.dump(summary, f, indent=1)
     details = subprocess.run(["ncu", "-i", rep, "--page", "details"], capture_output=True, text=True).stdout
