@@ -192,6 +192,215 @@ __global__ void __launch_bounds__(NT + NTC, 1) vpps_leaf_fwd(const float* __rest
     if (pf) pst[5] = gtimer();
 }
 
+
+// ---- tensor-core variant (opt-in, VPPS_LEAF_TC=1): the leaf GEMM as tcgen05.mma kind::tf32 with a 3xTF32 split ----
+// D[128 leaves][48 rows] = Σ_k x[leaf][k] W_iou[row][k]: both operands are K-major as they lie in memory
+// (embedding rows, W_iou rows), so each thread stages 16-byte k-pieces through registers, splitting
+// v = hi + lo (hi = v truncated to TF32, lo = v - hi exact in FP32) into the SWIZZLE_NONE canonical layout
+// (core matrix = 8 rows x 16 B; rows 16 B apart, SBO = 128 B between 8-row groups, LBO = (rows/8)*128 B
+// between 4-k chunks; the layout tools/umma_test.cu pins).  D = A·B + A·B_lo + A_lo·B (the dropped
+// A_lo·B_lo is ~2^-22 relative: FP32 accuracy, parity bar 1e-4) accumulates in TMEM (48 of 64 columns).
+// K runs in 4 chunks of 64 through two smem buffers: the MMAs of chunk c (issued by one thread, completion
+// on an mbarrier) overlap the global loads and conversion of chunk c + 1.  Epilogue: tcgen05.ld of the
+// i, o, u columns of 8 units per thread (warp w: TMEM lanes 32(w&3).., units 8(w>>2)..), cell, 16-byte
+// record stores.  Tile count for the TGT batch (~450 leaves): 4 x 16 = 64 CTAs; the CTAs behind the tiles
+// (the leftover SMs, at least 32) do the per-pass clearing.
+constexpr int TL = 128;                 // leaves per tile (UMMA M)
+constexpr int TR = 3 * LU;              // W_iou rows per tile (UMMA N = 48)
+constexpr int KC = 64;                  // K per chunk
+constexpr int NCH = KMAX / KC;
+static_assert(NCH == 4, "chunk / mbarrier phase sequence below assumes 4 chunks");
+constexpr int A_F = TL * KC, B_F = TR * KC;          // floats per hi (or lo) copy
+constexpr int BUF_F = 2 * A_F + 2 * B_F;
+constexpr size_t TC_SMEM = (size_t)2 * BUF_F * sizeof(float);
+constexpr uint32_t LBO_A = (TL / 8) * 128, LBO_B = (TR / 8) * 128;   // bytes between 4-k chunks
+
+__device__ __forceinline__ uint64_t lf_desc(uint32_t saddr, uint32_t lbo) {
+    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
+           ((uint64_t)(128 >> 4) << 32) | ((uint64_t)1 << 46);
+}
+constexpr uint32_t lf_idesc(int m, int n) {      // F32 accumulate, TF32 A/B, both K-major
+    return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(m >> 4) << 24);
+}
+__device__ __forceinline__ void lf_mma(uint32_t d, uint64_t a, uint64_t b, int acc) {
+    constexpr uint32_t idesc = lf_idesc(TL, TR);
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                 "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}\n"
+                 ::"r"(d), "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void lf_wait(uint32_t mbar, uint32_t parity) {
+    uint32_t ok = 0;
+    while (!ok)
+        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}\n"
+                     : "=r"(ok) : "r"(mbar), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void split_store(float* hi, float* lo, uint32_t off, const float4 v) {
+    const float4 h = make_float4(__uint_as_float(__float_as_uint(v.x) & 0xFFFFE000u), __uint_as_float(__float_as_uint(v.y) & 0xFFFFE000u),
+                                 __uint_as_float(__float_as_uint(v.z) & 0xFFFFE000u), __uint_as_float(__float_as_uint(v.w) & 0xFFFFE000u));
+    *reinterpret_cast<float4*>(hi + off) = h;
+    *reinterpret_cast<float4*>(lo + off) = make_float4(v.x - h.x, v.y - h.y, v.z - h.z, v.w - h.w);
+}
+#define LF_LD8(r, addr)                                                                                        \
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"                     \
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]) \
+                 : "r"(addr))
+
+__global__ void __launch_bounds__(NT, 1) vpps_leaf_fwd_tc(const float* __restrict__ W, const float* __restrict__ b,
+                                                        const float* __restrict__ inputs, float* pool,
+                                                        const uint32_t* __restrict__ leaves, int n_leaf, int H,
+                                                        int tiles, const PassClear pc) {
+    extern __shared__ __align__(128) float tsm[];
+    __shared__ uint32_t tmem_base;
+    __shared__ __align__(8) uint64_t mbar[2];
+    __shared__ float bias_s[3 * LU];
+    const int tid = threadIdx.x;
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    const bool pf = g_leaf_prof_on && tid == 0 && blockIdx.x < 1024;
+    uint64_t* pst = g_leaf_prof + blockIdx.x * 8;
+    if (pf) pst[0] = gtimer();
+    if ((int)blockIdx.x >= tiles) {
+        // clearing CTAs (the GEMM tiles never wait for the per-pass clearing) and the pass counter
+        const int cb = blockIdx.x - tiles, ncb = gridDim.x - tiles;
+        if (pc.epoch && cb == 0 && tid == 0) {
+            uint32_t e = *pc.epoch + 1;
+            *pc.epoch = e ? e : 1u;                               // 0 marks never-written slots
+        }
+        const int64_t stride = (int64_t)ncb * NT;
+        for (int r = 0; r < 4; ++r) {
+            float4* p = reinterpret_cast<float4*>(pc.ptr[r]);
+            const int64_t n4 = pc.ptr[r] ? pc.n[r] / 4 : 0;
+            for (int64_t i = (int64_t)cb * NT + tid; i < n4; i += stride) p[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+        if (pf) pst[6] = gtimer();
+        return;
+    }
+    const int tiles_u = H / LU;
+    const int l0 = (blockIdx.x / tiles_u) * TL, j0 = (blockIdx.x % tiles_u) * LU;
+    const int warp = tid >> 5, lane = tid & 31;
+    if (warp == 0) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base)), "r"(64));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    if (tid == 32) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&mbar[0])));
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&mbar[1])));
+        asm volatile("fence.mbarrier_init.release.cluster;");
+    }
+    if (tid >= 64 && tid < 64 + 3 * LU) {                          // b_iou of the tile's units
+        const int k = tid - 64;
+        bias_s[k] = __ldg(b + (k / LU) * H + j0 + k % LU);
+    }
+    // epilogue leaf of this thread (TMEM lane 32 (w & 3) + lane): its record offset, fetched early
+    const int eq = warp & 3, eh = warp >> 2, eli = 32 * eq + lane;
+    const uint32_t erec = l0 + eli < n_leaf ? __ldg(leaves + 2 * (l0 + eli)) : 0u;
+    // staging: A row (leaf l0 + (tid & 127)), pieces k4 = ak0 + 2p (p < 8); B pieces e = tid + 256p:
+    // row e % 48, k4 = e / 48.  Two chunks of registers in flight.
+    const int ar = tid & (TL - 1), ak0 = tid >> 7;
+    const uint32_t tok = l0 + ar < n_leaf ? __ldg(leaves + 2 * (l0 + ar) + 1) : 0xFFFFFFFFu;
+    const float* arow = tok != 0xFFFFFFFFu ? inputs + (int64_t)tok * KMAX : nullptr;
+    const float* brow[3];
+    int bk4[3];
+#pragma unroll
+    for (int p = 0; p < 3; ++p) {
+        const int e = tid + NT * p, r = e % TR;
+        bk4[p] = e / TR;
+        brow[p] = W + (int64_t)((r / LU) * H + j0 + r % LU) * KMAX;
+    }
+    float4 ra[2][8], rb[2][3];
+    auto load = [&](int c, int set) {
+#pragma unroll
+        for (int p = 0; p < 8; ++p)
+            ra[set][p] = arow ? __ldg(reinterpret_cast<const float4*>(arow + c * KC + 4 * (ak0 + 2 * p))) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+        for (int p = 0; p < 3; ++p) rb[set][p] = __ldg(reinterpret_cast<const float4*>(brow[p] + c * KC + 4 * bk4[p]));
+    };
+    load(0, 0);
+    load(1, 1);
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem = tmem_base;
+    if (pf) pst[1] = gtimer();
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+        const int set = c & 1;
+        float* buf = tsm + set * BUF_F;
+        float* Ah = buf;
+        float* Al = Ah + A_F;
+        float* Bh = Al + A_F;
+        float* Bl = Bh + B_F;
+        if (c >= 2) lf_wait(smem_u32(&mbar[set]), 0);             // the MMAs of chunk c - 2 have read the buffer
+#pragma unroll
+        for (int p = 0; p < 8; ++p) {
+            const int k4 = ak0 + 2 * p;
+            split_store(Ah, Al, (uint32_t)((ar >> 3) * 32 + (ar & 7) * 4 + k4 * (LBO_A / 4)), ra[set][p]);
+        }
+#pragma unroll
+        for (int p = 0; p < 3; ++p) {
+            const int e = tid + NT * p, r = e % TR;
+            split_store(Bh, Bl, (uint32_t)((r >> 3) * 32 + (r & 7) * 4 + bk4[p] * (LBO_B / 4)), rb[set][p]);
+        }
+        if (c + 2 < NCH) load(c + 2, set);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic smem writes -> tensor core
+        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        __syncthreads();
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        if (c == 0 && pf) pst[2] = gtimer();
+        if (tid == 0) {
+            const uint32_t a0 = smem_u32(Ah), al0 = smem_u32(Al), b0 = smem_u32(Bh), bl0 = smem_u32(Bl);
+#pragma unroll
+            for (int s = 0; s < KC / 8; ++s) {
+                const uint64_t a = lf_desc(a0 + 2 * s * LBO_A, LBO_A), al = lf_desc(al0 + 2 * s * LBO_A, LBO_A);
+                const uint64_t bb = lf_desc(b0 + 2 * s * LBO_B, LBO_B), bl = lf_desc(bl0 + 2 * s * LBO_B, LBO_B);
+                lf_mma(tmem, a, bb, c > 0 || s > 0);
+                lf_mma(tmem, a, bl, 1);
+                lf_mma(tmem, al, bb, 1);
+            }
+            asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                         ::"r"(smem_u32(&mbar[set])) : "memory");
+        }
+    }
+    if (pf) pst[3] = gtimer();
+    lf_wait(smem_u32(&mbar[1]), 1);                                // chunk 3 (and every earlier MMA) done
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    if (pf) pst[4] = gtimer();
+    // epilogue: warp w reads TMEM lanes 32 (w & 3) .. +31 (leaves), the i / o / u columns of units 8 (w >> 2) .. +7
+    {
+        const uint32_t ta = tmem + ((uint32_t)(32 * eq) << 16) + 8 * eh;
+        uint32_t gi[8], go[8], gu[8];
+        LF_LD8(gi, ta);
+        LF_LD8(go, ta + LU);
+        LF_LD8(gu, ta + 2 * LU);
+        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+        if (l0 + eli < n_leaf) {
+            const int jb = j0 + 8 * eh;
+            float* r = pool + erec;
+            float hv[8], cv[8], iv[8], ov[8], uv[8];
+#pragma unroll
+            for (int t = 0; t < 8; ++t) {
+                const int u = 8 * eh + t;
+                const float ig = fsigm(__uint_as_float(gi[t]) + bias_s[u]);
+                const float og = fsigm(__uint_as_float(go[t]) + bias_s[LU + u]);
+                const float ug = ftanh(__uint_as_float(gu[t]) + bias_s[2 * LU + u]);
+                const float cc = ig * ug;
+                hv[t] = og * ftanh(cc); cv[t] = cc; iv[t] = ig; ov[t] = og; uv[t] = ug;
+            }
+#pragma unroll
+            for (int t = 0; t < 8; t += 4) {
+                *reinterpret_cast<float4*>(r + jb + t) = make_float4(hv[t], hv[t + 1], hv[t + 2], hv[t + 3]);
+                *reinterpret_cast<float4*>(r + H + jb + t) = make_float4(cv[t], cv[t + 1], cv[t + 2], cv[t + 3]);
+                *reinterpret_cast<float4*>(r + 2 * H + jb + t) = make_float4(iv[t], iv[t + 1], iv[t + 2], iv[t + 3]);
+                *reinterpret_cast<float4*>(r + 3 * H + jb + t) = make_float4(ov[t], ov[t + 1], ov[t + 2], ov[t + 3]);
+                *reinterpret_cast<float4*>(r + 4 * H + jb + t) = make_float4(uv[t], uv[t + 1], uv[t + 2], uv[t + 3]);
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(64));
+    if (pf) pst[5] = gtimer();
+}
+
 }  // namespace leaf
 }  // namespace dev
 
@@ -208,16 +417,28 @@ void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float*
     static bool attr = false;
     if (!attr) {
         cudaFuncSetAttribute(vpps_leaf_fwd<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+        cudaFuncSetAttribute(vpps_leaf_fwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TC_SMEM);
         attr = true;
     }
     PassClear pc{};
     static const int exp_ = getenv("VPPS_LEAF_EXP") ? atoi(getenv("VPPS_LEAF_EXP")) : 0;   // measurement only
+    // VPPS_LEAF_TC=1: the tensor-core variant (parity-green; measured slower than the FFMA tiles, 17.5 vs
+    // 12.3 us per TGT pass: the register-transit staging of the hi / lo split and the first TMEM allocation
+    // sit on its critical path)
+    static const bool simt = !(getenv("VPPS_LEAF_TC") && atoi(getenv("VPPS_LEAF_TC")) != 0);
     for (int r = 0; r < 4; ++r) { pc.ptr[r] = zero_ptr ? zero_ptr[r] : nullptr; pc.n[r] = zero_ptr ? zero_n[r] : 0; }
     if (exp_ & 1) for (int r = 0; r < 4; ++r) if (r != 2) pc.n[r] = 0;     // no clearing (but the counters)
     if (exp_ & 2) n_leaf = 0;                                                // clearing only
     pc.epoch = epoch;
-    const int tiles = std::max(((n_leaf + LM - 1) / LM) * (H / LU), 148);
-    vpps_leaf_fwd<256><<<tiles, NT + NTC, SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
+    if (simt) {
+        const int tiles = std::max(((n_leaf + LM - 1) / LM) * (H / LU), 148);
+        vpps_leaf_fwd<256><<<tiles, NT + NTC, SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
+    } else {
+        // GEMM tiles first, then clearing CTAs: the SMs left over (at least 32 CTAs)
+        const int tiles = ((n_leaf + TL - 1) / TL) * (H / LU);
+        const int grid = tiles + std::max(148 - tiles, 32);
+        vpps_leaf_fwd_tc<<<grid, NT, TC_SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H, tiles, pc);
+    }
 }
 
 }  // namespace vpps

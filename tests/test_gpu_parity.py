@@ -345,3 +345,19 @@ def test_errors_are_loud():
     s = m.build_script(_trees(1, 2, (1, 5), 8, 5))
     with pytest.raises(vpps.VppsError):                   # buffers not bound
         m.fwd_bwd(s, torch.zeros(8, 32, device="cuda"))
+
+
+@pytest.mark.parametrize("env", ["VPPS_LEAF_TC", "VPPS_DW_TC"])
+def test_tensor_core_variants_subprocess(env):
+    """The opt-in tensor-core leaf GEMM / gradient GEMM (tcgen05 kind::tf32, 3xTF32 split) on the dataflow
+    path against the oracle.  The switches are read once per process, so each runs in a child process."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = ("import sys; sys.path.insert(0, %r); sys.path.insert(0, %r); import test_gpu_parity as t; "
+            "t.check('binary', 256, 256, 5, t._trees(3, 16, (5, 50), 4096, 5), 4096, cluster=16, dataflow=True); "
+            "print('ok')" % (root, os.path.join(root, "tests")))
+    r = subprocess.run([sys.executable, "-c", code], env={**os.environ, env: "1"}, capture_output=True, text=True,
+                       timeout=600)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stdout + r.stderr
