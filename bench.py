@@ -171,6 +171,42 @@ def cpu_baseline(batches, budget_s=12.0):
             "sample": f"{n} trees of the bench batches in {dt:.1f} s (FP64 NumPy, BLAS threads = 1)"}
 
 
+def _oracle_trees(args_):
+    """Worker of cpu_baseline_all_cores: trees (b, i) of the bench batches through the FP64 oracle."""
+    idx, budget_s = args_
+    from threadpoolctl import threadpool_limits
+    from oracle import models as M
+    rng = np.random.default_rng(0)
+    P = synth.init_params(M.param_shapes("binary", H, E, C), rng)
+    X = synth.input_table(rng, V, E)
+    batches = make_batches(0, 16)
+    n, t0 = 0, time.perf_counter()
+    with threadpool_limits(limits=1):
+        for b, i in idx:
+            M.forward_backward("binary", P, X, [batches[b][i]], H)
+            n += 1
+            if time.perf_counter() - t0 > budget_s:
+                break
+    return n
+
+
+def cpu_baseline_all_cores(batches, budget_s=8.0):
+    """The same oracle across every host core (one process per core, trees split round-robin)."""
+    import multiprocessing as mp
+    cores = len(os.sched_getaffinity(0))
+    trees = [(b, i) for b in range(len(batches)) for i in range(len(batches[b]))]
+    work = [(trees[r::cores], budget_s) for r in range(cores)]
+    ctx = mp.get_context("spawn")
+    with ctx.Pool(cores) as pool:
+        pool.map(_oracle_trees, [([trees[0]], 1.0)] * cores)      # warm the workers (imports)
+        t0 = time.perf_counter()
+        n = sum(pool.map(_oracle_trees, work))
+        dt = time.perf_counter() - t0
+    return {"value": n / dt, "unit": "samples/s", "cores": cores, "kind": "oracle",
+            "sample": f"{n} trees of the bench batches in {dt:.1f} s on {cores} processes (FP64 NumPy, "
+                      f"BLAS threads = 1 each)"}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -266,6 +302,8 @@ def main():
         ev[k][1].record(stream)
         flops += infos[(args.warmup + k) % N_BATCHES]["flops"]
     m.set_timing_events(None, None)
+    # north_star roofline per batch: T = max(F / P_fp32, (2 W_once + A) / BW_HBM), averaged over the timed
+    # batches (F, A: the script's algorithmic FLOPs and activation bytes)
     torch.cuda.synchronize()
     clk = clocks.stop()
     step_ms = sum(a.elapsed_time(b) for a, b in ev)
@@ -332,6 +370,14 @@ def main():
         pk = peaks()
         mhz = clk.get("sm_mhz") or pk.get("sm_max_mhz", 1965.0)
         peak = fp32_peak_tflops(pk.get("sm_max_mhz", 1965.0))
+        try:
+            bw_hbm = float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"]) * 1e9
+        except Exception:
+            bw_hbm = 7.7e12                                  # B200_PROFILING.md fallback
+        w_once_b = 4 * sum(int(np.prod(s)) for _, s in shapes)
+        t_roof = [max(inf["flops"] / (peak * 1e12), (2 * w_once_b + inf["act_bytes"]) / bw_hbm)
+                  for inf in (infos[(args.warmup + k) % N_BATCHES] for k in range(args.steps))]
+        t_roof_mean = float(np.mean(t_roof))
         avg_flops = flops / args.steps
         step_tflops = avg_flops / (kern_ms / args.steps / 1e3) / 1e12
         if dom_n:
@@ -371,7 +417,12 @@ def main():
                          "kernel_ms": dom_avg_ms, "flops_per_launch": dom_avg_flops,
                          "step_kernels_ms": kern_ms / args.steps, "step_flops": avg_flops,
                          "step_tflops": step_tflops,
-                         "peak_note": "FP32 FFMA: 148 SM x 128 lanes x 2 FLOP x sm_max_mhz (derived, DESIGN.md)"},
+                         "peak_note": "FP32 FFMA: 148 SM x 128 lanes x 2 FLOP x sm_max_mhz (derived, DESIGN.md)",
+                         "north_star": {"t_roofline_us": 1e6 * t_roof_mean,
+                                        "t_measured_us": 1e3 * step_ms / args.steps,
+                                        "frac": 1e6 * t_roof_mean / (1e3 * step_ms / args.steps),
+                                        "definition": "max(F / P_fp32, (2 W_once + A) / BW_hbm) per batch, "
+                                                      "mean over the timed batches, / measured step time"}},
             "dram": {"weights_once_bytes": w_once,
                      "dominant_kernel_cold_bytes": traffic,
                      "pass_read_bytes_in_pipeline": inpipe["pass_dram_read_bytes"] if inpipe else None,
@@ -388,6 +439,7 @@ def main():
         }
         if world == 1 and not args.no_cpu_baseline:
             line["cpu_baseline"] = cpu_baseline(batches)
+            line["cpu_baseline_all_cores"] = cpu_baseline_all_cores(batches)
         print(json.dumps(line), flush=True)
     if dist:
         dist.destroy_process_group()
