@@ -1021,7 +1021,9 @@ __global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
     while (true) {
         if (tid < 32) {
             // lane q looks at group grp[q] (all groups in one parallel round trip); the first eligible
-            // group in order is claimed, retrying further groups if its items ran out meanwhile
+            // group in order is claimed, retrying further groups if its items ran out meanwhile (claiming
+            // the newest group first was measured neutral: at the last group's completion every CTA is
+            // still busy with earlier items)
             const int lane = tid;
             const int g = lane < P.n_grp ? P.grp[lane] : -1;
             uint32_t c = 0, d = 0;
@@ -1078,6 +1080,7 @@ __global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
         }
     }
     __syncthreads();
+    const uint64_t t_tail = P.trace ? gtimer() : 0;
     // chunks of 4 float4 per thread with every load in flight before the first store (a strided
     // load-update-store loop is one L2 round trip per iteration: params may alias grads for the compiler)
     constexpr int CV = 4;                                  // float4 per thread per chunk
@@ -1111,6 +1114,12 @@ __global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
             a[q].z -= lr * (b[q].z + wd * a[q].z); a[q].w -= lr * (b[q].w + wd * a[q].w);
             p4[k] = a[q];
         }
+    }
+    if (P.trace && tid == 0 && blockIdx.x < 1000) {   // tail stamps (measurement): rows 3000 + CTA
+        uint32_t smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        uint64_t* o = P.trace + 5 * (3000 + blockIdx.x);
+        o[0] = 99; o[1] = blockIdx.x; o[2] = t_tail; o[3] = gtimer(); o[4] = smid;
     }
 }
 

@@ -22,6 +22,7 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--config", default="tgt")
     ap.add_argument("--batches", action="store_true", help="per-batch timeline of the last CTA's group")
+    ap.add_argument("--sgd", action="store_true", help="fused SGD step (the bench mode)")
     args = ap.parse_args()
     import torch
     import synth
@@ -50,10 +51,15 @@ def main():
         if r == args.reps - 1:
             torch.cuda.synchronize()
             buf.zero_()
-        m.fwd_bwd(s, X, dX)
+        if args.sgd:
+            m.fwd_bwd_sgd(s, X, dX, lr=1e-3)
+        else:
+            m.fwd_bwd(s, X, dX)
     torch.cuda.synchronize()
     raw = buf.cpu().numpy().astype(np.float64)
     gtr = gt.cpu().numpy().astype(np.float64)
+    tail = gtr[3000:][gtr[3000:, 0] == 99]
+    gtr = gtr[:3000]
     gtr = gtr[gtr[:, 3] > 0]
     t0 = raw[:, 0].min()
     span = (raw[:, 1] - raw[:, 0]) / 1e3
@@ -74,6 +80,10 @@ def main():
         gend = [(raw[g*16:(g+1)*16, 1].max() - t0) / 1e3 for g in range(groups)]
         st = (gtr[:, 2] - t0) / 1e3
         en = (gtr[:, 3] - t0) / 1e3
+        if len(tail):
+            ts, te = (tail[:, 2] - t0) / 1e3, (tail[:, 3] - t0) / 1e3
+            print(f"gradient GEMM tail ({len(tail)} CTAs): fin seen {ts.min():.1f}-{ts.max():.1f} us, "
+                  f"SGD + exit {te.min():.1f}-{te.max():.1f} us")
         print(f"gradient GEMM: {len(gtr)} items, first start {st.min():.1f} us, last end {en.max():.1f} us, "
               f"mean item {np.mean(en - st):.2f} us, SMs used {len(set(gtr[:, 4]))}")
         for g in range(groups):
