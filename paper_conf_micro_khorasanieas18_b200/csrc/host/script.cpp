@@ -9,6 +9,13 @@
 #include <algorithm>
 #include <cstring>
 #include "host.h"
+#ifdef VPPS_HOST_PHASES   // measurement build (tools/host_breakdown.py): per-phase host times
+#include <chrono>
+double vpps_host_phase_us[8];
+#define PHASE(k) do { const double _n = std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now().time_since_epoch()).count(); if (k > 0) vpps_host_phase_us[k - 1] += _n - _t0; _t0 = _n; } while (0)
+#else
+#define PHASE(k) do { } while (0)
+#endif
 
 namespace vpps {
 namespace {
@@ -33,6 +40,10 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
         *err = "null batch array";
         return -1;
     }
+#ifdef VPPS_HOST_PHASES
+    double _t0 = 0;
+#endif
+    PHASE(0);
     // ---- S1/S2: super-graph (cells in given order, then heads of labelled cells) -----------------
     std::vector<Node> nodes;
     std::vector<int32_t> kids;
@@ -84,6 +95,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     const int64_t N = (int64_t)nodes.size();
     if (N == 0) { *err = "empty batch"; return -4; }
 
+    PHASE(1);
     // ---- S3: level = maximum depth from the sources (L139) --------------------------------------
     std::vector<int32_t> level(N, 0);
     int32_t L = 0;
@@ -117,6 +129,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     }
     if (cursor >= (int64_t)NONE) { *err = "pool exceeds 2^32 words (16 GiB, L159)"; return -1; }
 
+    PHASE(2);
     // ---- per-node cost (MACs; L167 "relatively higher load" for cached-matrix ops) and FLOPs -----
     auto macs = [&](int64_t i) -> int64_t {
         const Node& n = nodes[i];
@@ -183,6 +196,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
         }
     };
 
+    PHASE(3);
     // ---- S4-S6: phases, min-load groups, signal/wait ------------------------------------------
     const int32_t G = plan.G, P = 2 * L + 2;
     std::vector<std::vector<int64_t>> at_level(L + 1);
@@ -268,6 +282,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
         }
     }
 
+    PHASE(4);
     // ---- header: [G, n_bar, prefix sums], streams, barrier targets (L169) ---------------------
     Script& s = *out;
     s.words.clear();
@@ -337,6 +352,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     }
     s.leaf_off[n_grp] = (int32_t)s.n_leaf;
 
+    PHASE(5);
     // ---- level-synchronous lowering of the binary cell (Plan::level): per-level node lists ------
     s.lv_int = s.lv_leaf = s.lv_head = -1;
     s.lv_n_int = s.lv_n_leaf = s.lv_n_head = 0;
@@ -369,6 +385,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
             }
     }
 
+    PHASE(6);
     // ---- dataflow lowering of the binary cell for whole-graph groups (vpps_df) ------------------
     // Per group: batches of <= 16 nodes of one opcode, forward levels 1..L then backward levels L..0
     // (level 0 leaves run as a GEMM before the kernel).  Cross-CTA values live in epoch-tagged 64-bit
@@ -463,6 +480,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
         s.df_hd = cur;   cur = align32(cur + 2 * H * s.n_hd);
         s.df_words = cur - s.pool_words;
     }
+    PHASE(7);
     return 0;
 }
 
