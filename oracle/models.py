@@ -14,6 +14,10 @@ L321) and the readings of SURVEY.md §8(c) c.2 / DESIGN.md "Readings" (R-1 … R
   M3  child-sum Tree-LSTM ([5] eqs. 2-8), stacked (i, o, u)
   M4  binary Tree-LSTM ([5] eqs. 9-14, N = 2, words at leaves only, diagonal forget couplings),
       matrices W_iou 3H×E, U_iou 3H×2H, U_fl H×H, U_fr H×H, W_out C×H  (11H²+5H at E=H: Tab.I)
+  M5  GRU step (Cho et al.; the variation L21 names; reading R-34): gates
+      stacked (r, z, n), a_x = W x + b_i, a_h = U h_prev + b_h,
+      r = σ(a_x[r] + a_h[r]), z = σ(a_x[z] + a_h[z]), n = tanh(a_x[n] + r ⊙ a_h[n]),
+      h = (1 − z) ⊙ n + z ⊙ h_prev
   head: z = W_out h + b_out, ℓ = −log softmax(z)[y]  ("negative softmax log likelihood", L42)
 
 Everything is float64, node by node, in the graph's own order for the forward pass and in
@@ -24,7 +28,7 @@ from __future__ import annotations
 
 import numpy as np
 
-CELLS = ("lstm", "binary", "childsum", "bilstm")
+CELLS = ("lstm", "binary", "childsum", "bilstm", "gru")
 
 
 def param_shapes(cell: str, H: int, E: int, C: int, M: int = 256):
@@ -40,6 +44,9 @@ def param_shapes(cell: str, H: int, E: int, C: int, M: int = 256):
     if cell == "childsum":
         return [("W_iou", (3 * H, E)), ("W_f", (H, E)), ("U_iou", (3 * H, H)), ("U_f", (H, H)),
                 ("W_out", (C, H)), ("b_iou", (3 * H,)), ("b_f", (H,)), ("b_out", (C,))]
+    if cell == "gru":
+        return [("W", (3 * H, E)), ("U", (3 * H, H)), ("W_out", (C, H)),
+                ("b_i", (3 * H,)), ("b_h", (3 * H,)), ("b_out", (C,))]
     if cell == "bilstm":
         return [("Wf", (4 * H, E)), ("Uf", (4 * H, H)), ("Wb", (4 * H, E)), ("Ub", (4 * H, H)),
                 ("W_mlp", (M, 2 * H)), ("W_tag", (C, M)),
@@ -127,6 +134,63 @@ def _lstm_graph(P, G, X, dX, nodes, H):
         if ch:
             dh[ch[0]] += dhp
             dc[ch[0]] += dcp
+    return loss
+
+
+# ----------------------------------------------------------------------------------------
+# M5: GRU step (gate order r, z, n; the reset gate multiplies U_n h_prev + b_hn, reading R-34)
+# ----------------------------------------------------------------------------------------
+def gru_step(W, U, b_i, b_h, x, h_prev):
+    H = U.shape[1]
+    ax = W @ x + b_i
+    ah = U @ h_prev + b_h
+    r = sigmoid(ax[0:H] + ah[0:H])
+    z = sigmoid(ax[H:2 * H] + ah[H:2 * H])
+    n = np.tanh(ax[2 * H:3 * H] + r * ah[2 * H:3 * H])
+    h = (1.0 - z) * n + z * h_prev
+    return dict(r=r, z=z, n=n, hn=ah[2 * H:3 * H], h=h, x=x, h_prev=h_prev)
+
+
+def gru_step_backward(W, U, s, dh):
+    """Returns (γ_x, γ_h, dx, dh_prev): γ_x the gradient of a_x = W x + b_i, γ_h that of a_h = U h + b_h."""
+    r, z, n = s["r"], s["z"], s["n"]
+    dn = dh * (1.0 - z)
+    dz = dh * (s["h_prev"] - n)
+    dan = dn * (1.0 - n * n)                 # pre-activation of n
+    dr = dan * s["hn"]
+    dar = dr * r * (1.0 - r)
+    daz = dz * z * (1.0 - z)
+    gam_x = np.concatenate([dar, daz, dan])
+    gam_h = np.concatenate([dar, daz, dan * r])
+    return gam_x, gam_h, W.T @ gam_x, U.T @ gam_h + dh * z
+
+
+def _gru_graph(P, G, X, dX, nodes, H):
+    """One GRU chain (node t's single child is t-1). Returns the graph's loss."""
+    n = len(nodes)
+    st = [None] * n
+    loss = 0.0
+    heads = {}
+    for t, (ch, tok, lab) in enumerate(nodes):
+        hp = st[ch[0]]["h"] if ch else np.zeros(H)
+        st[t] = gru_step(P["W"], P["U"], P["b_i"], P["b_h"], X[tok], hp)
+        if lab >= 0:
+            l, p = head_forward(P, st[t]["h"], lab)
+            loss += l
+            heads[t] = p
+    dh = [np.zeros(H) for _ in range(n)]
+    for t in range(n - 1, -1, -1):
+        ch, tok, lab = nodes[t]
+        if lab >= 0:
+            dh[t] += head_backward(P, G, st[t]["h"], heads[t], lab)
+        gx, gh, dx, dhp = gru_step_backward(P["W"], P["U"], st[t], dh[t])
+        G["W"] += np.outer(gx, st[t]["x"])
+        G["U"] += np.outer(gh, st[t]["h_prev"])
+        G["b_i"] += gx
+        G["b_h"] += gh
+        dX[tok] += dx
+        if ch:
+            dh[ch[0]] += dhp
     return loss
 
 
@@ -294,7 +358,7 @@ def _bilstm_graph(P, G, X, dX, nodes, H):
 
 
 _GRAPH_FN = {"lstm": _lstm_graph, "binary": _binary_graph, "childsum": _childsum_graph,
-             "bilstm": _bilstm_graph}
+             "bilstm": _bilstm_graph, "gru": _gru_graph}
 
 
 def validate(cell: str, graphs, n_tokens: int, n_classes: int):
@@ -307,7 +371,7 @@ def validate(cell: str, graphs, n_tokens: int, n_classes: int):
                 raise ValueError("token/label out of range")
             if cell == "binary" and not ((len(ch) == 0 and tok >= 0) or (len(ch) == 2 and tok < 0)):
                 raise ValueError("binary Tree-LSTM: leaves carry a token, internal nodes have 2 children")
-            if cell in ("lstm", "bilstm") and (len(ch) > 1 or tok < 0 or (ch and ch[0] != v - 1)):
+            if cell in ("lstm", "bilstm", "gru") and (len(ch) > 1 or tok < 0 or (ch and ch[0] != v - 1)):
                 raise ValueError("LSTM chain: node t has child t-1 and a token")
         parents = [0] * len(nodes)
         for ch, _, _ in nodes:
@@ -350,6 +414,8 @@ def flop_count(cell: str, graphs, H: int, E: int, C: int, want_dx: bool = True, 
                 f += 2 * 3 * (3 * H * H + k * H * H) if k else 0
             elif cell == "lstm":
                 f += 2 * (4 * H * E) * kx + 2 * 3 * 4 * H * H * (1 if ch else 0)
+            elif cell == "gru":
+                f += 2 * (3 * H * E) * kx + 2 * 3 * 3 * H * H * (1 if ch else 0)
             if lab >= 0 and cell != "bilstm":
                 f += 2 * 3 * C * H
     return f

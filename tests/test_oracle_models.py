@@ -82,6 +82,52 @@ def test_fd_bilstm():
     _fd_check("bilstm", [g1, g2], H=2, E=2, C=3, V=3, M_=3)
 
 
+def test_fd_gru():
+    g1 = [((), 0, 1), ((0,), 2, -1), ((1,), 1, 0)]
+    g2 = [((), 1, 2), ((0,), 1, 1)]
+    _fd_check("gru", [g1, g2], H=3, E=2, C=3, V=3)
+
+
+def test_gru_equals_torch_grucell():
+    """M5 (reading R-34) == torch.nn.GRUCell in float64: torch stacks (r, z, n) in weight_ih / weight_hh
+    with separate biases and applies the reset gate to W_hn h + b_hn, as the oracle does — a swapped gate,
+    a reset applied before U_n, or a wrong sign of the (1 - z) / z interpolation fails this."""
+    H, E, C, V = 5, 4, 6, 7
+    P = _params("gru", H, E, C, 3)
+    P = {k: v * 2.0 for k, v in P.items()}
+    rng = np.random.default_rng(4)
+    X = rng.uniform(-1, 1, (V, E))
+    nodes = synth.chain(rng, 6, V, lm=True)
+    loss, G, dX = M.forward_backward("gru", P, X, [nodes], H)
+    cell = torch.nn.GRUCell(E, H, dtype=torch.float64)
+    with torch.no_grad():
+        cell.weight_ih.copy_(torch.tensor(P["W"])); cell.weight_hh.copy_(torch.tensor(P["U"]))
+        cell.bias_ih.copy_(torch.tensor(P["b_i"])); cell.bias_hh.copy_(torch.tensor(P["b_h"]))
+    Wo = torch.tensor(P["W_out"], requires_grad=True)
+    bo = torch.tensor(P["b_out"], requires_grad=True)
+    toks = [t for (_, t, _) in nodes]
+    Xt = torch.tensor(np.array([X[t] for t in toks]), requires_grad=True)
+    h = torch.zeros(1, H, dtype=torch.float64)
+    ref = torch.zeros((), dtype=torch.float64)
+    for t, (_, _, lab) in enumerate(nodes):
+        h = cell(Xt[t:t + 1], h)
+        if lab >= 0:
+            ref = ref + torch.nn.functional.cross_entropy((h[0] @ Wo.T + bo)[None], torch.tensor([lab]),
+                                                          reduction="sum")
+    ref.backward()
+    assert abs(loss - ref.item()) < 1e-12
+    np.testing.assert_allclose(G["W"], cell.weight_ih.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(G["U"], cell.weight_hh.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(G["b_i"], cell.bias_ih.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(G["b_h"], cell.bias_hh.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(G["W_out"], Wo.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(G["b_out"], bo.grad.numpy(), atol=1e-12)
+    dXref = np.zeros_like(X)
+    for t, tok in enumerate(toks):
+        dXref[tok] += Xt.grad.numpy()[t]
+    np.testing.assert_allclose(dX, dXref, atol=1e-12)
+
+
 def _torch_lstm_chain(Wih, Whh, b, xs, Wout, bout, labels):
     """Reference with torch.nn.LSTMCell (gate order i, f, g, o) + cross_entropy(sum)."""
     H = Whh.shape[1]
@@ -234,13 +280,13 @@ def test_childsum_chain_equals_lstm():
     np.testing.assert_allclose(dX3, dX1, atol=1e-12)
 
 
-@pytest.mark.parametrize("cell", ["binary", "childsum", "lstm"])
+@pytest.mark.parametrize("cell", ["binary", "childsum", "lstm", "gru"])
 def test_batch_order_and_linearity(cell):
     H, E, C, V = 4, 4, 5, 50
     P = _params(cell, H, E, C, 10)
     rng = np.random.default_rng(11)
     X = rng.uniform(-1, 1, (V, E))
-    if cell == "lstm":
+    if cell in ("lstm", "gru"):
         graphs = [synth.chain(rng, int(rng.integers(2, 6)), C) for _ in range(4)]
     else:
         graphs = synth.tree_batch(rng, 4, (2, 7), V, C)
