@@ -38,6 +38,7 @@ std::vector<Shape> expected_shapes(int32_t cell, int32_t H, int32_t E, int32_t C
             return {{4 * H, E}, {4 * H, H}, {4 * H, E}, {4 * H, H}, {M, 2 * H}, {C, M},
                     {4 * H, 1}, {4 * H, 1}, {M, 1}, {C, 1}};
         case CELL_LSTM: return {{4 * H, E}, {4 * H, H}, {C, H}, {4 * H, 1}, {C, 1}};
+        case CELL_GRU: return {{3 * H, E}, {3 * H, H}, {C, H}, {3 * H, 1}, {3 * H, 1}, {C, 1}};
         case CELL_BINARY: return {{3 * H, E}, {3 * H, 2 * H}, {H, H}, {H, H}, {C, H}, {3 * H, 1}, {H, 1}, {C, 1}};
         case CELL_CHILDSUM: return {{3 * H, E}, {H, E}, {3 * H, H}, {H, H}, {C, H}, {3 * H, 1}, {H, 1}, {C, 1}};
     }
@@ -114,7 +115,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     vpps_options o{};
     if (opt) o = *opt;
     const int32_t cell = ops->cell, H = ops->H, E = ops->E, C = ops->C, Mw = ops->mlp;
-    if (cell < 0 || cell > 3 || H <= 0 || E <= 0 || C <= 0) return fail(VPPS_E_INVALID, "bad op set");
+    if (cell < 0 || cell > 4 || H <= 0 || E <= 0 || C <= 0) return fail(VPPS_E_INVALID, "bad op set");
     if (cell == CELL_BILSTM && Mw <= 0) return fail(VPPS_E_INVALID, "BiLSTM tagger needs mlp > 0");
     std::vector<Shape> want = expected_shapes(cell, H, E, C, Mw);
     if ((int32_t)want.size() != n_params) return fail(VPPS_E_INVALID, "wrong number of parameters for the op set");
@@ -136,9 +137,9 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     }
     m->n_floats = cur;
     int32_t n_sm = o.n_sm;
-    if (cell == CELL_BILSTM || (cell == CELL_LSTM && (o.level > 0 || (o.level == 0 && C > 32)))) {
-        // M2 runs on the level-synchronous path only (vpps_level.cu), and so does an LSTM LM whose
-        // vocabulary head exceeds one CTA's shared memory (config 3 at V = 1000): no partition plan
+    if (cell == CELL_BILSTM || cell == CELL_GRU || (cell == CELL_LSTM && (o.level > 0 || (o.level == 0 && C > 32)))) {
+        // M2 and M5 (GRU) run on the level-synchronous path only (vpps_level.cu), and so does an LSTM LM
+        // whose vocabulary head exceeds one CTA's shared memory (config 3 at V = 1000): no partition plan
         if (o.cluster > 1 || o.dataflow || o.level < 0) return fail(VPPS_E_INVALID, "this op set runs on the level path only");
         if (H % 4 || E % 4) return fail(VPPS_E_INVALID, "H and E must be multiples of 4");
         if (cell == CELL_LSTM) {
@@ -350,7 +351,8 @@ vpps_status vpps_build_script(vpps_model m, const vpps_batch* batch, vpps_script
     BatchIn b{batch->n_graphs, batch->graph_ptr, batch->child_ptr, batch->children, batch->token, batch->label};
     std::string err;
     // the input table's row count is not known here; token range is re-checked against it at run time
-    const bool chains = m->plan.level && (m->plan.cell == CELL_BILSTM || m->plan.cell == CELL_LSTM);
+    const bool chains = m->plan.level && (m->plan.cell == CELL_BILSTM || m->plan.cell == CELL_LSTM ||
+                                          m->plan.cell == CELL_GRU);
     int rc = 0;
     if (chains && m->plan.cell == CELL_LSTM) {
         // LSTM LM on the level path: the SPEC script (words, pool plan: a bit-exact artifact of the op set)
@@ -555,6 +557,15 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
                        m->offsets.data(), m->n_floats, mode, lr, wd, st, m->gemm_trace,
                        m->pool + s->s.loss_word, m->d_loss_map + (m->passes & 1));
         CK(cudaGetLastError());
+    } else if (m->plan.level && m->plan.cell == CELL_GRU) {
+        if (s->s.tg_tok < 0) return fail(VPPS_E_INVALID, "script was not built for the level path");
+        CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));
+        const int rc = gru_pass(m->level, m->params, m->offsets.data(), m->grads, m->pool, inputs, d_inputs, dwords,
+                                s->s.tg_tok, s->s.tg_lab, s->s.tg_fpos, s->s.tg_start.data(),
+                                (int32_t)s->s.tg_start.size() - 1, s->s.tg_T, m->plan.H, m->plan.E, m->plan.C,
+                                s->s.loss_word, st);
+        if (rc != 0) return fail(VPPS_E_CUDA, "GRU pass failed (code " + std::to_string(rc) + ")");
+        if (mode == 1) launch_sgd(m->params, m->grads, m->n_floats, lr, wd, st);
     } else if (m->plan.level && (m->plan.cell == CELL_BILSTM || m->plan.cell == CELL_LSTM)) {
         if (s->s.tg_tok < 0) return fail(VPPS_E_INVALID, "script was not built for the level path");
         CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));   // incl. padding

@@ -21,7 +21,7 @@ int build_tagger_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows
         for (int32_t v = first; v < last; ++v) {
             const int32_t t = v - first, c0 = b.child_ptr[v], c1 = b.child_ptr[v + 1];
             const bool ok = (t == 0 && c1 == c0) || (t > 0 && c1 == c0 + 1 && b.children[c0] == t - 1);
-            if (!ok) { *err = "BiLSTM tagger: node t has the single child t-1"; return -4; }
+            if (!ok) { *err = "chain: node t has the single child t-1"; return -4; }
             if (b.token[v] < 0 || b.token[v] >= n_input_rows) { *err = "token out of range"; return -4; }
             if (b.label[v] < -1 || b.label[v] >= plan.C) { *err = "label out of range"; return -4; }
             s.max_token = std::max<int64_t>(s.max_token, b.token[v]);
@@ -63,6 +63,8 @@ int build_tagger_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows
     const double H = plan.H, E = plan.E, C = plan.C, M = plan.mlp;
     if (plan.cell == CELL_BILSTM)
         s.flops = (double)T * 2.0 * 24.0 * H * (E + H) + (double)s.n_heads * (12.0 * H * M + 6.0 * M * C);
+    else if (plan.cell == CELL_GRU)   // GRU chains: 3 gates, one direction, head on h
+        s.flops = (double)T * 18.0 * H * (E + H) + (double)s.n_heads * 6.0 * C * H;
     else   // LSTM LM: one direction, head on h
         s.flops = (double)T * 24.0 * H * (E + H) + (double)s.n_heads * 6.0 * C * H;
     return 0;

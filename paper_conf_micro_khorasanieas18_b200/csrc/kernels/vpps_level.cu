@@ -329,6 +329,66 @@ __global__ void tg_scatter_dx(const float* __restrict__ DX, const uint32_t* __re
     atomicAdd(dX + (int64_t)tok[t / E] * E + t % E, DX[t]);
 }
 
+
+// ---- GRU chains (M5, reading R-34): gates (r, z, n); a_x = W x + b_i (Px = X Wᵀ over all positions),
+//      a_h = U h_prev + b_h (Zs = H_prev Uᵀ per step); the reset gate multiplies a_h[n] ----
+// forward step: Gd[p] = (r, z, n, a_h[n]) for the backward
+__global__ void gru_cell(const float* __restrict__ Px, const float* __restrict__ Zs, const float* __restrict__ b_i,
+                         const float* __restrict__ b_h, const uint32_t* __restrict__ pos, int n, int dp, bool first,
+                         int H, float* HH, float* Gd) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= (int64_t)n * H) return;
+    const int r = (int)(t / H), j = (int)(t % H);
+    const int64_t p = pos[r];
+    const float* px = Px + p * 3 * H;
+    const float* zs = Zs + (int64_t)r * 3 * H;
+    const float ahr = b_h[j] + (first ? 0.f : zs[j]);
+    const float ahz = b_h[H + j] + (first ? 0.f : zs[H + j]);
+    const float ahn = b_h[2 * H + j] + (first ? 0.f : zs[2 * H + j]);
+    const float rg = sigm(px[j] + b_i[j] + ahr);
+    const float zg = sigm(px[H + j] + b_i[H + j] + ahz);
+    const float ng = tanhf(px[2 * H + j] + b_i[2 * H + j] + rg * ahn);
+    const float hp = first ? 0.f : HH[(p + dp) * H + j];
+    HH[p * H + j] = (1.f - zg) * ng + zg * hp;
+    float* g = Gd + p * 4 * H;
+    g[j] = rg; g[H + j] = zg; g[2 * H + j] = ng; g[3 * H + j] = ahn;
+}
+
+// backward step: dh = dHH[p] (head) + dHr[p] (successor); γ_x -> Gx[p], γ_h -> Gh[p] and the step buffer
+// Gs[r]; the direct term dh ⊙ z of dh_prev -> Ez[r]
+__global__ void gru_cell_bwd(const uint32_t* __restrict__ pos, int n, int dp, bool first, int H,
+                             const float* __restrict__ dHH, const float* __restrict__ dHr,
+                             const float* __restrict__ HH, const float* __restrict__ Gd, float* Gx, float* Gh,
+                             float* Gs, float* Ez) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= (int64_t)n * H) return;
+    const int r = (int)(t / H), j = (int)(t % H);
+    const int64_t p = pos[r];
+    const float dh = dHH[p * H + j] + dHr[p * H + j];
+    const float* g = Gd + p * 4 * H;
+    const float rg = g[j], zg = g[H + j], ng = g[2 * H + j], ahn = g[3 * H + j];
+    const float hp = first ? 0.f : HH[(p + dp) * H + j];
+    const float dan = dh * (1.f - zg) * (1.f - ng * ng);
+    const float dar = dan * ahn * rg * (1.f - rg);
+    const float daz = dh * (hp - ng) * zg * (1.f - zg);
+    float* gx = Gx + p * 3 * H;
+    float* gh = Gh + p * 3 * H;
+    float* gs = Gs + (int64_t)r * 3 * H;
+    gx[j] = dar; gx[H + j] = daz; gx[2 * H + j] = dan;
+    gh[j] = dar; gh[H + j] = daz; gh[2 * H + j] = dan * rg;
+    gs[j] = dar; gs[H + j] = daz; gs[2 * H + j] = dan * rg;
+    Ez[t] = dh * zg;
+}
+
+// dHr[pos + dp] = Dh[r] + Ez[r]: the step's dh_prev = Γ_h U + dh ⊙ z
+__global__ void gru_scatter_dh(const float* __restrict__ Dh, const float* __restrict__ Ez, const uint32_t* __restrict__ pos,
+                               int n, int dp, int H, float* dHr) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= (int64_t)n * H) return;
+    const int r = (int)(t / H), j = (int)(t % H);
+    dHr[((int64_t)pos[r] + dp) * H + j] = Dh[t] + Ez[t];
+}
+
 // out[c] = Σ_r A[r][c] (+= when accumulate)
 __global__ void colsum(const float* __restrict__ A, int rows, int cols, float* out) {
     const int c = blockIdx.x * blockDim.x + threadIdx.x;
@@ -592,6 +652,81 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
     if (d_inputs) {
         BL(gemm_rm(c->blas, false, false, (int)T, E, 4 * H, tb.Gamf, 4 * H, Wf, E, tb.DX, E, 0.f));
         if (dirs > 1) BL(gemm_rm(c->blas, false, false, (int)T, E, 4 * H, tb.Gamb, 4 * H, Wb, E, tb.DX, E, 1.f));
+        tg_scatter_dx<<<nblk(T * E), 256, 0, s>>>(tb.DX, tok, (int)T, E, d_inputs);
+    }
+#undef BL
+    return (int)cudaGetLastError();
+}
+
+
+// GRU chains (M5) on the level-synchronous path: the LSTM LM's organisation (input projections and the
+// head as dense products over all positions, one recurrent product per time step, dW / dU / dX as GEMMs)
+// with the GRU cell.  off: (W, U, W_out, b_i, b_h, b_out).
+int gru_pass(void* ctx_, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
+             float* d_inputs, const uint32_t* d_blob, int64_t tg_tok, int64_t tg_lab, int64_t tg_fpos,
+             const int32_t* start, int32_t maxlen, int64_t T, int32_t H, int32_t E, int32_t C, int64_t loss_word,
+             cudaStream_t s) {
+    using namespace dev::lv;
+    LevelCtx* c = static_cast<LevelCtx*>(ctx_);
+    TaggerBufs& tb = c->tg;
+    cublasSetStream(c->blas, s);
+    const int64_t Tn = std::max<int64_t>(T, 1);
+    // X, Px (Pf), HH, Gd (Gf), Hp, Zs, Z, dZ, dHH, dHr (dHf), Gx (Gamf), Gh (Gamb), Gs, Dh, Ez (Cf), DX
+    float** bufs[16] = {&tb.X, &tb.Pf, &tb.HH, &tb.Gf, &tb.Hp, &tb.Zs, &tb.Z, &tb.dZ, &tb.dHH, &tb.dHf, &tb.Gamf,
+                        &tb.Gamb, &tb.Gs, &tb.Dh, &tb.Cf, &tb.DX};
+    int64_t* caps[16] = {&tb.cap[0], &tb.cap[1], &tb.cap[3], &tb.cap[6], &tb.cap[8], &tb.cap[9], &tb.cap[11],
+                         &tb.cap[12], &tb.cap[14], &tb.cap[15], &tb.cap[19], &tb.cap[20], &tb.cap[21], &tb.cap[22],
+                         &tb.cap[4], &tb.cap[23]};
+    const int64_t need[16] = {Tn * E, Tn * 3 * H, Tn * H, Tn * 4 * H, Tn * H, Tn * 3 * H, Tn * C, Tn * C, Tn * H,
+                              Tn * H, Tn * 3 * H, Tn * 3 * H, Tn * 3 * H, Tn * H, Tn * H, Tn * E};
+    for (int k = 0; k < 16; ++k)
+        if (!grow(bufs[k], caps[k], need[k])) return (int)cudaErrorMemoryAllocation;
+    const float *W = params + off[0], *U = params + off[1], *Wo = params + off[2], *b_i = params + off[3],
+                *b_h = params + off[4], *bo = params + off[5];
+    const uint32_t *tok = d_blob + tg_tok, *lab = d_blob + tg_lab, *fpos = d_blob + tg_fpos;
+    cublasStatus_t st;
+#define BL(call) do { st = (call); if (st != CUBLAS_STATUS_SUCCESS) return 1000 + (int)st; } while (0)
+    if (T == 0) return 0;
+    tg_gather_x<<<nblk(T * (E / 4)), 256, 0, s>>>(inputs, tok, (int)T, E, tb.X);
+    BL(gemm_rm(c->blas, false, true, (int)T, 3 * H, E, tb.X, E, W, E, tb.Pf, 3 * H, 0.f));
+    for (int32_t t = 0; t < maxlen; ++t) {
+        const int32_t r0 = start[t], n = start[t + 1] - r0;
+        const uint32_t* pos = fpos + r0;
+        if (t > 0) {
+            tg_gather_hprev<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.HH, pos, n, -1, 0, H, H, tb.Hp);
+            BL(gemm_rm(c->blas, false, true, n, 3 * H, H, tb.Hp, H, U, H, tb.Zs, 3 * H, 0.f));
+        }
+        gru_cell<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.Pf, tb.Zs, b_i, b_h, pos, n, -1, t == 0, H, tb.HH, tb.Gf);
+    }
+    // head on h (L42): z = W_out h + b_out, softmax-NLL on labelled positions, dW_out, db_out, dh
+    BL(gemm_rm(c->blas, false, true, (int)T, C, H, tb.HH, H, Wo, H, tb.Z, C, 0.f));
+    tg_softmax<<<nblk(T * 32), 256, 0, s>>>(tb.Z, bo, lab, (int)T, C, tb.dZ, pool + loss_word);
+    BL(gemm_rm(c->blas, true, false, C, H, (int)T, tb.dZ, C, tb.HH, H, grads + off[2], H, 0.f));
+    colsum<<<nblk(C), 256, 0, s>>>(tb.dZ, (int)T, C, grads + off[5]);
+    BL(gemm_rm(c->blas, false, false, (int)T, H, C, tb.dZ, C, Wo, H, tb.dHH, H, 0.f));
+    cudaMemsetAsync(tb.dHf, 0, T * H * sizeof(float), s);
+    for (int32_t t = maxlen - 1; t >= 0; --t) {
+        const int32_t r0 = start[t], n = start[t + 1] - r0;
+        const uint32_t* pos = fpos + r0;
+        gru_cell_bwd<<<nblk((int64_t)n * H), 256, 0, s>>>(pos, n, -1, t == 0, H, tb.dHH, tb.dHf, tb.HH, tb.Gf,
+                                                           tb.Gamf, tb.Gamb, tb.Gs, tb.Cf);
+        if (t > 0) {
+            BL(gemm_rm(c->blas, false, false, n, H, 3 * H, tb.Gs, 3 * H, U, H, tb.Dh, H, 0.f));
+            gru_scatter_dh<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.Dh, tb.Cf, pos, n, -1, H, tb.dHf);
+        }
+    }
+    // dW = Γ_xᵀ X, dU = Γ_hᵀ H_prev (zeros at chain starts), db_i = Σ Γ_x, db_h = Σ Γ_h; dX = Γ_x W
+    cudaMemsetAsync(tb.Hp, 0, T * H * sizeof(float), s);
+    if (maxlen > 1) {
+        const int32_t n = start[maxlen] - start[1];
+        tg_hprev_all<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.HH, fpos + start[1], n, -1, 0, H, H, tb.Hp);
+    }
+    BL(gemm_rm(c->blas, true, false, 3 * H, E, (int)T, tb.Gamf, 3 * H, tb.X, E, grads + off[0], E, 0.f));
+    BL(gemm_rm(c->blas, true, false, 3 * H, H, (int)T, tb.Gamb, 3 * H, tb.Hp, H, grads + off[1], H, 0.f));
+    colsum<<<nblk(3 * H), 256, 0, s>>>(tb.Gamf, (int)T, 3 * H, grads + off[3]);
+    colsum<<<nblk(3 * H), 256, 0, s>>>(tb.Gamb, (int)T, 3 * H, grads + off[4]);
+    if (d_inputs) {
+        BL(gemm_rm(c->blas, false, false, (int)T, E, 3 * H, tb.Gamf, 3 * H, W, E, tb.DX, E, 0.f));
         tg_scatter_dx<<<nblk(T * E), 256, 0, s>>>(tb.DX, tok, (int)T, E, d_inputs);
     }
 #undef BL

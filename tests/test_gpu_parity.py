@@ -361,3 +361,24 @@ def test_tensor_core_variants_subprocess(env):
     r = subprocess.run([sys.executable, "-c", code], env={**os.environ, env: "1"}, capture_output=True, text=True,
                        timeout=600)
     assert r.returncode == 0 and "ok" in r.stdout, r.stdout + r.stderr
+
+
+def test_gru_small():
+    """M5 GRU chains (reading R-34) on the level path, config-1 shapes (H = E = 32, 4 sequences of 2-5)."""
+    graphs = synth.config_batch("c1", 1)
+    check("gru", 32, 32, 16, graphs, 16, seed=41)
+
+
+@pytest.mark.parametrize("batch", [1, 4, 16])
+def test_gru_lm_h256_vocab1000(batch):
+    """GRU language model at config-3 shapes (H = E = 256, V = C = 1000, sentences of 5-60 tokens)."""
+    graphs = synth.config_batch("c3", 4, batch=batch, lengths=(5, 40))
+    check("gru", 256, 256, 1000, graphs, 1000, seed=90 + batch)
+
+
+def test_gru_degenerate_chains():
+    """Single-token chains, unlabelled positions and a repeated token (dX accumulation)."""
+    g1 = [([], 3, 2)]
+    g2 = [([], 1, -1), ([0], 1, -1), ([1], 1, 4)]
+    g3 = [([], 0, 1), ([0], 5, -1)]
+    check("gru", 32, 32, 8, [g1, g2, g3], 8, seed=43)
