@@ -410,7 +410,9 @@ def main():
                                 else "fused fwd-bwd-sgd, 1 kernel") + ("" if world == 1 else ", NCCL all-reduce before SGD"),
                        "l2": "no flush" if args.no_flush else "flushed (256 MiB write) before every timed step",
                        "batches": f"{N_BATCHES} distinct pre-built scripts cycled"},
-            "gpu_launches": args.steps * (4 if args.cluster else (1 if world == 1 else 2)),
+            # leaf GEMM + vpps_df + gradient GEMM (SGD fused in its tail at N = 1; a separate sgd_kernel after
+            # the all-reduce at N > 1); the grid path: one fused kernel (+ sgd_kernel at N > 1)
+            "gpu_launches": args.steps * ((3 if world == 1 else 4) if args.cluster else (1 if world == 1 else 2)),
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "kernel": ("vpps_df" if args.sync == "dataflow" else "vpps_cl") if args.cluster else "vpps_fb",
