@@ -18,6 +18,8 @@ L321) and the readings of SURVEY.md §8(c) c.2 / DESIGN.md "Readings" (R-1 … R
       stacked (r, z, n), a_x = W x + b_i, a_h = U h_prev + b_h,
       r = σ(a_x[r] + a_h[r]), z = σ(a_x[z] + a_h[z]), n = tanh(a_x[n] + r ⊙ a_h[n]),
       h = (1 − z) ⊙ n + z ⊙ h_prev
+  M6  RvNN (Socher-style recursive net with untied leaf / internal weights; reading R-35):
+      leaf h = tanh(W_leaf x + b_leaf), internal h = tanh(W_int [h_l; h_r] + b_int)
   head: z = W_out h + b_out, ℓ = −log softmax(z)[y]  ("negative softmax log likelihood", L42)
 
 Everything is float64, node by node, in the graph's own order for the forward pass and in
@@ -28,7 +30,7 @@ from __future__ import annotations
 
 import numpy as np
 
-CELLS = ("lstm", "binary", "childsum", "bilstm", "gru")
+CELLS = ("lstm", "binary", "childsum", "bilstm", "gru", "rvnn")
 
 
 def param_shapes(cell: str, H: int, E: int, C: int, M: int = 256):
@@ -44,6 +46,9 @@ def param_shapes(cell: str, H: int, E: int, C: int, M: int = 256):
     if cell == "childsum":
         return [("W_iou", (3 * H, E)), ("W_f", (H, E)), ("U_iou", (3 * H, H)), ("U_f", (H, H)),
                 ("W_out", (C, H)), ("b_iou", (3 * H,)), ("b_f", (H,)), ("b_out", (C,))]
+    if cell == "rvnn":
+        return [("W_leaf", (H, E)), ("W_int", (H, 2 * H)), ("W_out", (C, H)),
+                ("b_leaf", (H,)), ("b_int", (H,)), ("b_out", (C,))]
     if cell == "gru":
         return [("W", (3 * H, E)), ("U", (3 * H, H)), ("W_out", (C, H)),
                 ("b_i", (3 * H,)), ("b_h", (3 * H,)), ("b_out", (C,))]
@@ -191,6 +196,44 @@ def _gru_graph(P, G, X, dX, nodes, H):
         dX[tok] += dx
         if ch:
             dh[ch[0]] += dhp
+    return loss
+
+
+# ----------------------------------------------------------------------------------------
+# M6: RvNN (untied leaf / internal transformations, reading R-35)
+# ----------------------------------------------------------------------------------------
+def _rvnn_graph(P, G, X, dX, nodes, H):
+    """One binary tree: leaves carry a token, internal nodes two children. Returns the graph's loss."""
+    n = len(nodes)
+    h = [None] * n
+    loss = 0.0
+    heads = {}
+    for v, (ch, tok, lab) in enumerate(nodes):
+        if not ch:
+            h[v] = np.tanh(P["W_leaf"] @ X[tok] + P["b_leaf"])
+        else:
+            h[v] = np.tanh(P["W_int"] @ np.concatenate([h[ch[0]], h[ch[1]]]) + P["b_int"])
+        if lab >= 0:
+            l, p = head_forward(P, h[v], lab)
+            loss += l
+            heads[v] = p
+    dh = [np.zeros(H) for _ in range(n)]
+    for v in range(n - 1, -1, -1):
+        ch, tok, lab = nodes[v]
+        if lab >= 0:
+            dh[v] += head_backward(P, G, h[v], heads[v], lab)
+        g = dh[v] * (1.0 - h[v] * h[v])              # pre-activation gradient
+        if not ch:
+            G["W_leaf"] += np.outer(g, X[tok])
+            G["b_leaf"] += g
+            dX[tok] += P["W_leaf"].T @ g
+        else:
+            x = np.concatenate([h[ch[0]], h[ch[1]]])
+            G["W_int"] += np.outer(g, x)
+            G["b_int"] += g
+            dx = P["W_int"].T @ g
+            dh[ch[0]] += dx[:H]
+            dh[ch[1]] += dx[H:]
     return loss
 
 
@@ -358,7 +401,7 @@ def _bilstm_graph(P, G, X, dX, nodes, H):
 
 
 _GRAPH_FN = {"lstm": _lstm_graph, "binary": _binary_graph, "childsum": _childsum_graph,
-             "bilstm": _bilstm_graph, "gru": _gru_graph}
+             "bilstm": _bilstm_graph, "gru": _gru_graph, "rvnn": _rvnn_graph}
 
 
 def validate(cell: str, graphs, n_tokens: int, n_classes: int):
@@ -369,7 +412,7 @@ def validate(cell: str, graphs, n_tokens: int, n_classes: int):
                 raise ValueError("children must precede their parent")
             if not (-1 <= tok < n_tokens) or not (-1 <= lab < n_classes):
                 raise ValueError("token/label out of range")
-            if cell == "binary" and not ((len(ch) == 0 and tok >= 0) or (len(ch) == 2 and tok < 0)):
+            if cell in ("binary", "rvnn") and not ((len(ch) == 0 and tok >= 0) or (len(ch) == 2 and tok < 0)):
                 raise ValueError("binary Tree-LSTM: leaves carry a token, internal nodes have 2 children")
             if cell in ("lstm", "bilstm", "gru") and (len(ch) > 1 or tok < 0 or (ch and ch[0] != v - 1)):
                 raise ValueError("LSTM chain: node t has child t-1 and a token")
@@ -414,6 +457,8 @@ def flop_count(cell: str, graphs, H: int, E: int, C: int, want_dx: bool = True, 
                 f += 2 * 3 * (3 * H * H + k * H * H) if k else 0
             elif cell == "lstm":
                 f += 2 * (4 * H * E) * kx + 2 * 3 * 4 * H * H * (1 if ch else 0)
+            elif cell == "rvnn":
+                f += (2 * H * E * kx) if not ch else 2 * 3 * H * 2 * H
             elif cell == "gru":
                 f += 2 * (3 * H * E) * kx + 2 * 3 * 3 * H * H * (1 if ch else 0)
             if lab >= 0 and cell != "bilstm":

@@ -88,6 +88,58 @@ def test_fd_gru():
     _fd_check("gru", [g1, g2], H=3, E=2, C=3, V=3)
 
 
+def test_fd_rvnn():
+    g1 = [((), 0, -1), ((), 1, -1), ((0, 1), -1, -1), ((), 2, -1), ((2, 3), -1, 1)]
+    g2 = [((), 1, -1), ((), 1, -1), ((0, 1), -1, 2)]
+    _fd_check("rvnn", [g1, g2], H=3, E=2, C=3, V=3)
+
+
+def test_rvnn_left_comb_equals_torch_rnncell():
+    """M6 on a left-comb tree == torch.nn.RNNCell over the leaf outputs (reading R-35): internal node k has
+    the previous node on the left and leaf k on the right, so h_k = tanh(W_hh h_{k-1} + W_ih z_k + b) with
+    W_int = [W_hh | W_ih] and z_k = tanh(W_leaf x_k + b_leaf) (torch Linear + tanh); the first state is the
+    leftmost leaf's output.  Swapped halves of W_int, a wrong child order or a dropped tanh' fail this."""
+    H, E, C, V, n = 4, 3, 5, 6, 5
+    P = {k: v * 2.0 for k, v in _params("rvnn", H, E, C, 7).items()}
+    rng = np.random.default_rng(8)
+    X = rng.uniform(-1, 1, (V, E))
+    toks = [int(t) for t in rng.integers(0, V, n)]
+    nodes = [((), toks[0], -1)]
+    prev = 0
+    for k in range(1, n):
+        nodes.append(((), toks[k], -1))
+        nodes.append(((prev, len(nodes) - 1), -1, -1))
+        prev = len(nodes) - 1
+    nodes[-1] = (nodes[-1][0], -1, 3)
+    loss, G, dX = M.forward_backward("rvnn", P, X, [nodes], H)
+    leaf = torch.nn.Linear(E, H, dtype=torch.float64)
+    cell = torch.nn.RNNCell(H, H, nonlinearity="tanh", dtype=torch.float64)
+    with torch.no_grad():
+        leaf.weight.copy_(torch.tensor(P["W_leaf"])); leaf.bias.copy_(torch.tensor(P["b_leaf"]))
+        cell.weight_hh.copy_(torch.tensor(P["W_int"][:, :H])); cell.weight_ih.copy_(torch.tensor(P["W_int"][:, H:]))
+        cell.bias_ih.copy_(torch.tensor(P["b_int"])); cell.bias_hh.zero_()
+    Wo = torch.tensor(P["W_out"], requires_grad=True)
+    bo = torch.tensor(P["b_out"], requires_grad=True)
+    Xt = torch.tensor(np.array([X[t] for t in toks]), requires_grad=True)
+    z = torch.tanh(leaf(Xt))
+    h = z[0:1]
+    for k in range(1, n):
+        h = cell(z[k:k + 1], h)
+    ref = torch.nn.functional.cross_entropy((h[0] @ Wo.T + bo)[None], torch.tensor([3]), reduction="sum")
+    ref.backward()
+    assert abs(loss - ref.item()) < 1e-12
+    np.testing.assert_allclose(G["W_int"], np.concatenate([cell.weight_hh.grad.numpy(), cell.weight_ih.grad.numpy()], 1),
+                               atol=1e-12)
+    np.testing.assert_allclose(G["b_int"], cell.bias_ih.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(G["W_leaf"], leaf.weight.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(G["b_leaf"], leaf.bias.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(G["W_out"], Wo.grad.numpy(), atol=1e-12)
+    dXref = np.zeros_like(X)
+    for k, t in enumerate(toks):
+        dXref[t] += Xt.grad.numpy()[k]
+    np.testing.assert_allclose(dX, dXref, atol=1e-12)
+
+
 def test_gru_equals_torch_grucell():
     """M5 (reading R-34) == torch.nn.GRUCell in float64: torch stacks (r, z, n) in weight_ih / weight_hh
     with separate biases and applies the reset gate to W_hn h + b_hn, as the oracle does — a swapped gate,
@@ -280,7 +332,7 @@ def test_childsum_chain_equals_lstm():
     np.testing.assert_allclose(dX3, dX1, atol=1e-12)
 
 
-@pytest.mark.parametrize("cell", ["binary", "childsum", "lstm", "gru"])
+@pytest.mark.parametrize("cell", ["binary", "childsum", "lstm", "gru", "rvnn"])
 def test_batch_order_and_linearity(cell):
     H, E, C, V = 4, 4, 5, 50
     P = _params(cell, H, E, C, 10)
