@@ -56,11 +56,15 @@ typedef enum {
     VPPS_CELL_BILSTM_TAGGER = 3,  /* M2: forward + backward LSTM (i, f, o, g), per
                                      position m = tanh(W_mlp [h→; h←] + b_mlp), tag head z = W_tag m +
                                      b_tag; runs on the level-synchronous path (C <= 32 tags) */
-    VPPS_CELL_GRU = 4             /* M5 (the variation PAPER L21 names; DESIGN reading R-34): chains,
+    VPPS_CELL_GRU = 4,            /* M5 (the variation PAPER L21 names; DESIGN reading R-34): chains,
                                      gates (r, z, n), parameters W 3H×E, U 3H×H, W_out C×H, b_i 3H,
                                      b_h 3H, b_out C; r = σ(W_r x + b_ir + U_r h + b_hr), z likewise,
                                      n = tanh(W_n x + b_in + r ⊙ (U_n h + b_hn)), h' = (1−z) n + z h;
                                      head on labelled positions; level-synchronous path */
+    VPPS_CELL_RVNN = 5            /* M6 (DESIGN reading R-35): binary trees, untied weights
+                                     W_leaf H×E, W_int H×2H, W_out C×H, b_leaf H, b_int H, b_out C;
+                                     leaf h = tanh(W_leaf x + b_leaf), internal h = tanh(W_int [h_l; h_r]
+                                     + b_int); level-synchronous path */
 } vpps_cell;
 
 typedef struct {

@@ -68,6 +68,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
                 kids.push_back(base + ch);
             }
             switch (plan.cell) {
+                case CELL_RVNN:
                 case CELL_BINARY:
                     if (nch == 0 && tok >= 0) nd.kind = K_LEAF;
                     else if (nch == 2 && tok < 0) nd.kind = K_INT;
@@ -144,7 +145,10 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     };
     double flops = 0.0, abytes = 0.0;
     for (int64_t i = 0; i < N; ++i) {
-        flops += 6.0 * (double)macs(i);   // forward, weight gradient, input/hidden gradient (2 FLOP/MAC)
+        if (plan.cell == CELL_RVNN)       // M6: leaf H×E, internal H×2H, head C×H
+            flops += 6.0 * (double)(nodes[i].kind == K_LEAF ? H * E : nodes[i].kind == K_INT ? 2 * H * H : C * H);
+        else
+            flops += 6.0 * (double)macs(i);   // forward, weight gradient, input/hidden gradient (2 FLOP/MAC)
         const Node& n = nodes[i];
         const double nc = n.ch_count;
         double kin = 0, recsz = 0;
@@ -357,7 +361,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     s.lv_int = s.lv_leaf = s.lv_head = -1;
     s.lv_n_int = s.lv_n_leaf = s.lv_n_head = 0;
     s.lv_start.clear();
-    if (plan.level && plan.cell == CELL_BINARY) {
+    if (plan.level && (plan.cell == CELL_BINARY || plan.cell == CELL_RVNN)) {
         s.lv_int = (int64_t)s.blob.size();
         s.lv_start.assign(L + 2, 0);
         for (int32_t lv = 1; lv <= L + 1; ++lv) {

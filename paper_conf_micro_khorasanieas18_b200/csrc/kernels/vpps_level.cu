@@ -389,6 +389,29 @@ __global__ void gru_scatter_dh(const float* __restrict__ Dh, const float* __rest
     dHr[((int64_t)pos[r] + dp) * H + j] = Dh[t] + Ez[t];
 }
 
+
+// ---- RvNN (M6, reading R-35): leaf h = tanh(W_leaf x + b_leaf), internal h = tanh(W_int [h_l; h_r] + b_int);
+//      records keep h at offset 0, adjoints dh at adj + 0 ----
+// h = tanh(Z + b) -> pool[rec]; rows of a node list with record offsets at nodes[stride * r]
+__global__ void rv_cell(const float* __restrict__ Z, const float* __restrict__ b, const uint32_t* __restrict__ nodes,
+                        int stride, int n, int H, float* pool) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= (int64_t)n * H) return;
+    const int r = (int)(t / H), j = (int)(t % H);
+    pool[nodes[(int64_t)stride * r] + j] = tanhf(Z[t] + b[j]);
+}
+
+// g = dh (1 - h²) -> G rows (dh from the adjoint block nodes[stride r + adj_word])
+__global__ void rv_bwd(const uint32_t* __restrict__ nodes, int stride, int adj_word, int n, int H,
+                       const float* __restrict__ pool, float* __restrict__ G) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= (int64_t)n * H) return;
+    const int r = (int)(t / H), j = (int)(t % H);
+    const uint32_t* e = nodes + (int64_t)stride * r;
+    const float h = __ldcg(pool + e[0] + j), dh = __ldcg(pool + e[adj_word] + j);
+    G[t] = dh * (1.f - h * h);
+}
+
 // out[c] = Σ_r A[r][c] (+= when accumulate)
 __global__ void colsum(const float* __restrict__ A, int rows, int cols, float* out) {
     const int c = blockIdx.x * blockDim.x + threadIdx.x;
@@ -728,6 +751,73 @@ int gru_pass(void* ctx_, const float* params, const int64_t* off, float* grads, 
     if (d_inputs) {
         BL(gemm_rm(c->blas, false, false, (int)T, E, 3 * H, tb.Gamf, 3 * H, W, E, tb.DX, E, 0.f));
         tg_scatter_dx<<<nblk(T * E), 256, 0, s>>>(tb.DX, tok, (int)T, E, d_inputs);
+    }
+#undef BL
+    return (int)cudaGetLastError();
+}
+
+
+// RvNN (M6) on the level-synchronous path: leaves as one GEMM, every internal level as one gathered product,
+// dW_int / dW_leaf as one GEMM each over the concatenated nodes (L185).  off: (W_leaf, W_int, W_out,
+// b_leaf, b_int, b_out).  Buffers: X_leaf [n_leaf E], X_int [n_int 2H], Z, G_int [n_int H], G_leaf, DX.
+int rvnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
+              float* d_inputs, const uint32_t* d_blob, int64_t lv_int, int64_t lv_leaf, int64_t lv_head,
+              const int32_t* lv_start, int32_t L, int64_t n_int, int64_t n_leaf, int64_t n_head, int32_t H,
+              int32_t E, int32_t C, int64_t loss_word, cudaStream_t s) {
+    using namespace dev::lv;
+    LevelCtx* c = static_cast<LevelCtx*>(ctx_);
+    cublasSetStream(c->blas, s);
+    if (!grow(&c->b.X_leaf, &c->cap_X_leaf, std::max<int64_t>(n_leaf * E, 4)) ||
+        !grow(&c->b.X_int, &c->cap_X_int, std::max<int64_t>(n_int * 2 * H, 4)) ||
+        !grow(&c->b.Z, &c->cap_Z, std::max<int64_t>(std::max(n_leaf, n_int) * H, 4)) ||
+        !grow(&c->b.G_int, &c->cap_G_int, std::max<int64_t>(n_int * H, 4)) ||
+        !grow(&c->b.G_leaf, &c->cap_G_leaf, std::max<int64_t>(n_leaf * H, 4)) ||
+        !grow(&c->b.DX, &c->cap_DX, std::max<int64_t>(std::max<int64_t>(n_int * 2 * H, n_leaf * E), 4)))
+        return (int)cudaErrorMemoryAllocation;
+    const float *W_leaf = params + off[0], *W_int = params + off[1], *W_out = params + off[2];
+    const float *b_leaf = params + off[3], *b_int = params + off[4], *b_out = params + off[5];
+    const uint32_t* ints = d_blob + lv_int;      // (rec, rec_l, rec_r, adj, adj_l, adj_r) per internal node
+    const uint32_t* leaves = d_blob + lv_leaf;   // (rec, adj, token) per leaf
+    const uint32_t* hl = d_blob + lv_head;
+    float *Xl = c->b.X_leaf, *Xi = c->b.X_int, *Z = c->b.Z, *Gi = c->b.G_int, *Gl = c->b.G_leaf, *DX = c->b.DX;
+    cublasStatus_t st = CUBLAS_STATUS_SUCCESS;
+#define BL(call) do { st = (call); if (st != CUBLAS_STATUS_SUCCESS) return 1000 + (int)st; } while (0)
+    if (n_leaf > 0) {
+        gather_leaf<<<nblk(n_leaf * (E / 4)), 256, 0, s>>>(inputs, leaves, (int)n_leaf, E, Xl);
+        BL(gemm_rm(c->blas, false, true, (int)n_leaf, H, E, Xl, E, W_leaf, E, Z, H, 0.f));
+        rv_cell<<<nblk(n_leaf * H), 256, 0, s>>>(Z, b_leaf, leaves, 3, (int)n_leaf, H, pool);
+    }
+    for (int32_t l = 1; l <= L; ++l) {
+        const int64_t r0 = lv_start[l], n = lv_start[l + 1] - r0;
+        if (n <= 0) continue;
+        float* X = Xi + r0 * 2 * H;
+        gather_int<<<nblk(n * (2 * H / 4)), 256, 0, s>>>(pool, ints + 6 * r0, (int)n, H, X);
+        BL(gemm_rm(c->blas, false, true, (int)n, H, 2 * H, X, 2 * H, W_int, 2 * H, Z, H, 0.f));
+        rv_cell<<<nblk(n * H), 256, 0, s>>>(Z, b_int, ints + 6 * r0, 6, (int)n, H, pool);
+    }
+    if (n_head > 0)
+        heads<<<(unsigned)n_head, 256, C * sizeof(float), s>>>(W_out, b_out, hl, H, C, pool, loss_word, grads + off[2],
+                                                             grads + off[5]);
+    for (int32_t l = L; l >= 1; --l) {
+        const int64_t r0 = lv_start[l], n = lv_start[l + 1] - r0;
+        if (n <= 0) continue;
+        float* G = Gi + r0 * H;
+        rv_bwd<<<nblk(n * H), 256, 0, s>>>(ints + 6 * r0, 6, 3, (int)n, H, pool, G);
+        BL(gemm_rm(c->blas, false, false, (int)n, 2 * H, H, G, H, W_int, 2 * H, DX, 2 * H, 0.f));
+        scatter_dh<<<nblk(n * 2 * H), 256, 0, s>>>(DX, ints + 6 * r0, (int)n, H, pool);
+    }
+    if (n_leaf > 0) {
+        rv_bwd<<<nblk(n_leaf * H), 256, 0, s>>>(leaves, 3, 1, (int)n_leaf, H, pool, Gl);
+        if (d_inputs) {
+            BL(gemm_rm(c->blas, false, false, (int)n_leaf, E, H, Gl, H, W_leaf, E, DX, E, 0.f));
+            scatter_dx<<<nblk(n_leaf * E), 256, 0, s>>>(DX, leaves, (int)n_leaf, E, d_inputs);
+        }
+        BL(gemm_rm(c->blas, true, false, H, E, (int)n_leaf, Gl, H, Xl, E, grads + off[0], E, 0.f));
+        colsum<<<nblk(H), 256, 0, s>>>(Gl, (int)n_leaf, H, grads + off[3]);
+    }
+    if (n_int > 0) {
+        BL(gemm_rm(c->blas, true, false, H, 2 * H, (int)n_int, Gi, H, Xi, 2 * H, grads + off[1], 2 * H, 0.f));
+        colsum<<<nblk(H), 256, 0, s>>>(Gi, (int)n_int, H, grads + off[4]);
     }
 #undef BL
     return (int)cudaGetLastError();

@@ -382,3 +382,20 @@ def test_gru_degenerate_chains():
     g2 = [([], 1, -1), ([0], 1, -1), ([1], 1, 4)]
     g3 = [([], 0, 1), ([0], 5, -1)]
     check("gru", 32, 32, 8, [g1, g2, g3], 8, seed=43)
+
+
+def test_rvnn_small():
+    """M6 RvNN (reading R-35, untied leaf / internal weights) on the level path, small trees."""
+    check("rvnn", 32, 32, 5, _trees(61, 6, (1, 9), 16, 5), 16, seed=61)
+
+
+@pytest.mark.parametrize("b", [0, 1])
+def test_rvnn_paper_size(b):
+    """RvNN at the paper's size (Fig. 12: hidden and embedding 512) on SST-shaped trees, batch 16."""
+    check("rvnn", 512, 512, 5, synth.config_batch("tgt", 20 + b), 4096, seed=62 + b)
+
+
+def test_rvnn_labels_on_inner_nodes_and_single_leaves():
+    g1 = [([], 1, 2)]                                           # a single labelled leaf
+    g2 = [([], 0, -1), ([], 3, 1), ([0, 1], -1, 4), ([], 3, -1), ([2, 3], -1, 0)]
+    check("rvnn", 64, 64, 5, [g1, g2] + _trees(64, 3, (2, 12), 8, 5), 8, seed=64)
