@@ -399,3 +399,12 @@ def test_rvnn_labels_on_inner_nodes_and_single_leaves():
     g1 = [([], 1, 2)]                                           # a single labelled leaf
     g2 = [([], 0, -1), ([], 3, 1), ([0, 1], -1, 4), ([], 3, -1), ([2, 3], -1, 0)]
     check("rvnn", 64, 64, 5, [g1, g2] + _trees(64, 3, (2, 12), 8, 5), 8, seed=64)
+
+
+@pytest.mark.parametrize("batch", [1, 4, 64])
+def test_dataflow_batch_sweep(batch):
+    """The bench's path (dataflow groups) at batch 1 / 4 / 64 (BASELINE's TGT batch sweep): at 64 trees a
+    group runs ~7 trees, so its program spans several shared-memory chunks (refills) and its slots regions
+    are the largest the bench sees."""
+    check("binary", 256, 256, 5, synth.config_batch("tgt", 40 + batch, batch=batch), 4096, seed=70 + batch,
+          cluster=16, dataflow=True)
