@@ -20,6 +20,9 @@ L321) and the readings of SURVEY.md §8(c) c.2 / DESIGN.md "Readings" (R-1 … R
       h = (1 − z) ⊙ n + z ⊙ h_prev
   M6  RvNN (Socher-style recursive net with untied leaf / internal weights; reading R-35):
       leaf h = tanh(W_leaf x + b_leaf), internal h = tanh(W_int [h_l; h_r] + b_int)
+  M7  TD-RNN (reading R-36): a DAG over a sentence — level 0 the embeddings themselves
+      (h = x, E = H), node i of level k: h = tanh(W [h_i; h_{i+1}] + b) over level k−1 (one composition
+      function; inner nodes have two parents), the softmax head on the labelled top node
   head: z = W_out h + b_out, ℓ = −log softmax(z)[y]  ("negative softmax log likelihood", L42)
 
 Everything is float64, node by node, in the graph's own order for the forward pass and in
@@ -30,7 +33,7 @@ from __future__ import annotations
 
 import numpy as np
 
-CELLS = ("lstm", "binary", "childsum", "bilstm", "gru", "rvnn")
+CELLS = ("lstm", "binary", "childsum", "bilstm", "gru", "rvnn", "tdrnn")
 
 
 def param_shapes(cell: str, H: int, E: int, C: int, M: int = 256):
@@ -46,6 +49,8 @@ def param_shapes(cell: str, H: int, E: int, C: int, M: int = 256):
     if cell == "childsum":
         return [("W_iou", (3 * H, E)), ("W_f", (H, E)), ("U_iou", (3 * H, H)), ("U_f", (H, H)),
                 ("W_out", (C, H)), ("b_iou", (3 * H,)), ("b_f", (H,)), ("b_out", (C,))]
+    if cell == "tdrnn":
+        return [("W", (H, 2 * H)), ("W_out", (C, H)), ("b", (H,)), ("b_out", (C,))]
     if cell == "rvnn":
         return [("W_leaf", (H, E)), ("W_int", (H, 2 * H)), ("W_out", (C, H)),
                 ("b_leaf", (H,)), ("b_int", (H,)), ("b_out", (C,))]
@@ -238,6 +243,37 @@ def _rvnn_graph(P, G, X, dX, nodes, H):
 
 
 # ----------------------------------------------------------------------------------------
+# M7: TD-RNN (reading R-36): leaves are the embeddings, one composition function, shared children
+# ----------------------------------------------------------------------------------------
+def _tdrnn_graph(P, G, X, dX, nodes, H):
+    n = len(nodes)
+    h = [None] * n
+    loss = 0.0
+    heads = {}
+    for v, (ch, tok, lab) in enumerate(nodes):
+        h[v] = X[tok].copy() if not ch else np.tanh(P["W"] @ np.concatenate([h[ch[0]], h[ch[1]]]) + P["b"])
+        if lab >= 0:
+            l, p = head_forward(P, h[v], lab)
+            loss += l
+            heads[v] = p
+    dh = [np.zeros(H) for _ in range(n)]
+    for v in range(n - 1, -1, -1):         # every parent of v comes after v: its dh is complete here
+        ch, tok, lab = nodes[v]
+        if lab >= 0:
+            dh[v] += head_backward(P, G, h[v], heads[v], lab)
+        if not ch:
+            dX[tok] += dh[v]
+            continue
+        g = dh[v] * (1.0 - h[v] * h[v])
+        G["W"] += np.outer(g, np.concatenate([h[ch[0]], h[ch[1]]]))
+        G["b"] += g
+        dx = P["W"].T @ g
+        dh[ch[0]] += dx[:H]
+        dh[ch[1]] += dx[H:]
+    return loss
+
+
+# ----------------------------------------------------------------------------------------
 # M4: binary Tree-LSTM ([5] eqs. 9-14 with N = 2; stacked rows [i; o; u])
 # ----------------------------------------------------------------------------------------
 def _binary_graph(P, G, X, dX, nodes, H):
@@ -401,7 +437,7 @@ def _bilstm_graph(P, G, X, dX, nodes, H):
 
 
 _GRAPH_FN = {"lstm": _lstm_graph, "binary": _binary_graph, "childsum": _childsum_graph,
-             "bilstm": _bilstm_graph, "gru": _gru_graph, "rvnn": _rvnn_graph}
+             "bilstm": _bilstm_graph, "gru": _gru_graph, "rvnn": _rvnn_graph, "tdrnn": _tdrnn_graph}
 
 
 def validate(cell: str, graphs, n_tokens: int, n_classes: int):
@@ -412,7 +448,7 @@ def validate(cell: str, graphs, n_tokens: int, n_classes: int):
                 raise ValueError("children must precede their parent")
             if not (-1 <= tok < n_tokens) or not (-1 <= lab < n_classes):
                 raise ValueError("token/label out of range")
-            if cell in ("binary", "rvnn") and not ((len(ch) == 0 and tok >= 0) or (len(ch) == 2 and tok < 0)):
+            if cell in ("binary", "rvnn", "tdrnn") and not ((len(ch) == 0 and tok >= 0) or (len(ch) == 2 and tok < 0)):
                 raise ValueError("binary Tree-LSTM: leaves carry a token, internal nodes have 2 children")
             if cell in ("lstm", "bilstm", "gru") and (len(ch) > 1 or tok < 0 or (ch and ch[0] != v - 1)):
                 raise ValueError("LSTM chain: node t has child t-1 and a token")
@@ -420,7 +456,7 @@ def validate(cell: str, graphs, n_tokens: int, n_classes: int):
         for ch, _, _ in nodes:
             for k in ch:
                 parents[k] += 1
-        if any(p > 1 for p in parents):
+        if cell != "tdrnn" and any(p > 1 for p in parents):      # TD-RNN is a DAG (R-36)
             raise ValueError("a node may have at most one parent")
 
 
@@ -457,6 +493,8 @@ def flop_count(cell: str, graphs, H: int, E: int, C: int, want_dx: bool = True, 
                 f += 2 * 3 * (3 * H * H + k * H * H) if k else 0
             elif cell == "lstm":
                 f += 2 * (4 * H * E) * kx + 2 * 3 * 4 * H * H * (1 if ch else 0)
+            elif cell == "tdrnn":
+                f += 0 if not ch else 2 * 3 * H * 2 * H
             elif cell == "rvnn":
                 f += (2 * H * E * kx) if not ch else 2 * 3 * H * 2 * H
             elif cell == "gru":

@@ -80,6 +80,28 @@ def tagger_batch(rng, batch: int, lengths=(5, 60), vocab=4096, n_tags=9):
             for _ in range(batch)]
 
 
+def td_pyramid(rng: np.random.Generator, length: int, vocab: int, n_classes: int):
+    """A TD-RNN graph over a sentence of `length` tokens (reading R-36): level 0 the tokens,
+    node i of level k composes nodes i and i+1 of level k-1 (each inner node of a level below the top has
+    two parents), the single top node carries the sentence label.  Nodes are listed level by level."""
+    toks = rng.integers(0, vocab, size=length)
+    nodes = [((), int(t), -1) for t in toks]
+    prev = list(range(length))
+    for _ in range(1, length):
+        cur = []
+        for i in range(len(prev) - 1):
+            nodes.append(((prev[i], prev[i + 1]), -1, -1))
+            cur.append(len(nodes) - 1)
+        prev = cur
+    top = prev[0]
+    nodes[top] = (nodes[top][0], nodes[top][1], int(rng.integers(0, n_classes)))
+    return nodes
+
+
+def td_batch(rng, batch: int, lengths=(5, 30), vocab=4096, n_classes=5):
+    return [td_pyramid(rng, int(rng.integers(lengths[0], lengths[1] + 1)), vocab, n_classes) for _ in range(batch)]
+
+
 def init_params(shapes, rng: np.random.Generator, dtype=np.float64):
     """shapes: ordered list of (name, shape). Glorot-uniform for 2-D, U(-0.1, 0.1) for 1-D."""
     out = {}

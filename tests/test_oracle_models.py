@@ -140,6 +140,47 @@ def test_rvnn_left_comb_equals_torch_rnncell():
     np.testing.assert_allclose(dX, dXref, atol=1e-12)
 
 
+def test_fd_tdrnn():
+    rng = np.random.default_rng(3)
+    g1 = synth.td_pyramid(rng, 4, 3, 3)
+    g2 = synth.td_pyramid(rng, 3, 3, 3)
+    _fd_check("tdrnn", [g1, g2], H=2, E=2, C=3, V=3)
+
+
+def test_tdrnn_pyramid_equals_torch_conv1d():
+    """M7 (reading R-36) == repeated torch conv1d with kernel 2 (+ tanh) until one position remains: the
+    composition W [h_i; h_{i+1}] + b is a kernel-2 convolution with taps W[:, :H], W[:, H:].  The oracle
+    walks the DAG node by node and accumulates each shared child's dh from both parents; a dropped parent,
+    swapped taps or a wrong tanh' fail this (loss, dW, db, dW_out and dX to 1e-12 in float64)."""
+    H, C, V = 4, 5, 9
+    P = {k: v * 1.5 for k, v in _params("tdrnn", H, H, C, 5).items()}
+    rng = np.random.default_rng(6)
+    X = rng.uniform(-1, 1, (V, H))
+    graphs = [synth.td_pyramid(rng, n, V, C) for n in (6, 1, 3)]
+    loss, G, dX = M.forward_backward("tdrnn", P, X, graphs, H)
+    W = torch.tensor(P["W"], requires_grad=True)
+    b = torch.tensor(P["b"], requires_grad=True)
+    Wo = torch.tensor(P["W_out"], requires_grad=True)
+    bo = torch.tensor(P["b_out"], requires_grad=True)
+    Xt = torch.tensor(X, requires_grad=True)
+    ker = torch.stack([W[:, :H], W[:, H:]], dim=2)          # [H_out, H_in, 2]
+    ref = torch.zeros((), dtype=torch.float64)
+    for nodes in graphs:
+        toks = [t for (ch, t, _) in nodes if not ch]
+        e = Xt[toks].T[None]                                # [1, H, n]
+        while e.shape[2] > 1:
+            e = torch.tanh(torch.nn.functional.conv1d(e, ker, b))
+        y = [lab for (_, _, lab) in nodes if lab >= 0][0]
+        ref = ref + torch.nn.functional.cross_entropy((e[0, :, 0] @ Wo.T + bo)[None], torch.tensor([y]), reduction="sum")
+    ref.backward()
+    assert abs(loss - ref.item()) < 1e-12
+    np.testing.assert_allclose(G["W"], W.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(G["b"], b.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(G["W_out"], Wo.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(G["b_out"], bo.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(dX, Xt.grad.numpy(), atol=1e-12)
+
+
 def test_gru_equals_torch_grucell():
     """M5 (reading R-34) == torch.nn.GRUCell in float64: torch stacks (r, z, n) in weight_ih / weight_hh
     with separate biases and applies the reset gate to W_hn h + b_hn, as the oracle does — a swapped gate,
