@@ -61,10 +61,14 @@ typedef enum {
                                      b_h 3H, b_out C; r = σ(W_r x + b_ir + U_r h + b_hr), z likewise,
                                      n = tanh(W_n x + b_in + r ⊙ (U_n h + b_hn)), h' = (1−z) n + z h;
                                      head on labelled positions; level-synchronous path */
-    VPPS_CELL_RVNN = 5            /* M6 (DESIGN reading R-35): binary trees, untied weights
+    VPPS_CELL_RVNN = 5,           /* M6 (DESIGN reading R-35): binary trees, untied weights
                                      W_leaf H×E, W_int H×2H, W_out C×H, b_leaf H, b_int H, b_out C;
                                      leaf h = tanh(W_leaf x + b_leaf), internal h = tanh(W_int [h_l; h_r]
                                      + b_int); level-synchronous path */
+    VPPS_CELL_TDRNN = 6           /* M7 (DESIGN reading R-36): DAGs — leaves are the input
+                                     rows themselves (E = H), every inner node h = tanh(W [h_a; h_b] + b)
+                                     with W H×2H, b H, and a node may feed two parents; W_out C×H, b_out C;
+                                     level-synchronous path */
 } vpps_cell;
 
 typedef struct {

@@ -64,11 +64,15 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
             for (int32_t k = c0; k < c1; ++k) {
                 const int32_t ch = b.children[k];
                 if (ch < 0 || ch >= local) { *err = "children must precede their parent"; return -4; }
-                if (++parents_seen[ch] > 1) { *err = "a node may have at most one parent"; return -4; }
+                if (++parents_seen[ch] > 1 && plan.cell != CELL_TDRNN) {   // TD-RNN graphs are DAGs (R-36)
+                    *err = "a node may have at most one parent";
+                    return -4;
+                }
                 kids.push_back(base + ch);
             }
             switch (plan.cell) {
                 case CELL_RVNN:
+                case CELL_TDRNN:
                 case CELL_BINARY:
                     if (nch == 0 && tok >= 0) nd.kind = K_LEAF;
                     else if (nch == 2 && tok < 0) nd.kind = K_INT;
@@ -147,6 +151,8 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     for (int64_t i = 0; i < N; ++i) {
         if (plan.cell == CELL_RVNN)       // M6: leaf H×E, internal H×2H, head C×H
             flops += 6.0 * (double)(nodes[i].kind == K_LEAF ? H * E : nodes[i].kind == K_INT ? 2 * H * H : C * H);
+        else if (plan.cell == CELL_TDRNN)   // M7: no leaf transform, inner H×2H, head C×H
+            flops += 6.0 * (double)(nodes[i].kind == K_LEAF ? 0 : nodes[i].kind == K_INT ? 2 * H * H : C * H);
         else
             flops += 6.0 * (double)macs(i);   // forward, weight gradient, input/hidden gradient (2 FLOP/MAC)
         const Node& n = nodes[i];
@@ -361,7 +367,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     s.lv_int = s.lv_leaf = s.lv_head = -1;
     s.lv_n_int = s.lv_n_leaf = s.lv_n_head = 0;
     s.lv_start.clear();
-    if (plan.level && (plan.cell == CELL_BINARY || plan.cell == CELL_RVNN)) {
+    if (plan.level && (plan.cell == CELL_BINARY || plan.cell == CELL_RVNN || plan.cell == CELL_TDRNN)) {
         s.lv_int = (int64_t)s.blob.size();
         s.lv_start.assign(L + 2, 0);
         for (int32_t lv = 1; lv <= L + 1; ++lv) {

@@ -412,6 +412,35 @@ __global__ void rv_bwd(const uint32_t* __restrict__ nodes, int stride, int adj_w
     G[t] = dh * (1.f - h * h);
 }
 
+
+// ---- TD-RNN (M7, reading R-36): leaves copy their input row; shared children take dh from two parents ----
+__global__ void td_leaf(const float* __restrict__ inputs, const uint32_t* __restrict__ leaf, int n, int H, float* pool) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= (int64_t)n * H) return;
+    const int r = (int)(t / H), j = (int)(t % H);
+    const uint32_t* e = leaf + 3 * r;
+    pool[e[0] + j] = e[2] == NONE ? 0.f : __ldg(inputs + (int64_t)e[2] * H + j);
+}
+
+// children's dh += DX rows with atomics (a child may have a second parent in the same level)
+__global__ void scatter_dh_shared(const float* __restrict__ DX, const uint32_t* __restrict__ nodes, int n, int H,
+                                  float* pool) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= (int64_t)n * 2 * H) return;
+    const int r = (int)(t / (2 * H)), c = (int)(t % (2 * H));
+    const uint32_t* e = nodes + 6 * r;
+    atomicAdd(c < H ? pool + e[4] + c : pool + e[5] + (c - H), DX[t]);
+}
+
+// dX[token] += dh of each leaf (its adjoint block)
+__global__ void td_leaf_dx(const uint32_t* __restrict__ leaf, int n, int H, const float* __restrict__ pool, float* dX) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= (int64_t)n * H) return;
+    const int r = (int)(t / H), j = (int)(t % H);
+    const uint32_t* e = leaf + 3 * r;
+    if (e[2] != NONE) atomicAdd(dX + (int64_t)e[2] * H + j, __ldcg(pool + e[1] + j));
+}
+
 // out[c] = Σ_r A[r][c] (+= when accumulate)
 __global__ void colsum(const float* __restrict__ A, int rows, int cols, float* out) {
     const int c = blockIdx.x * blockDim.x + threadIdx.x;
@@ -818,6 +847,59 @@ int rvnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads,
     if (n_int > 0) {
         BL(gemm_rm(c->blas, true, false, H, 2 * H, (int)n_int, Gi, H, Xi, 2 * H, grads + off[1], 2 * H, 0.f));
         colsum<<<nblk(H), 256, 0, s>>>(Gi, (int)n_int, H, grads + off[4]);
+    }
+#undef BL
+    return (int)cudaGetLastError();
+}
+
+
+// TD-RNN (M7) on the level-synchronous path: level k of every sentence's pyramid as one gathered product;
+// a child of two parents of the same level receives both dh contributions atomically.  off: (W, W_out, b,
+// b_out).  E == H.
+int tdrnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
+               float* d_inputs, const uint32_t* d_blob, int64_t lv_int, int64_t lv_leaf, int64_t lv_head,
+               const int32_t* lv_start, int32_t L, int64_t n_int, int64_t n_leaf, int64_t n_head, int32_t H,
+               int32_t E, int32_t C, int64_t loss_word, cudaStream_t s) {
+    using namespace dev::lv;
+    (void)E;
+    LevelCtx* c = static_cast<LevelCtx*>(ctx_);
+    cublasSetStream(c->blas, s);
+    if (!grow(&c->b.X_int, &c->cap_X_int, std::max<int64_t>(n_int * 2 * H, 4)) ||
+        !grow(&c->b.Z, &c->cap_Z, std::max<int64_t>(n_int * H, 4)) ||
+        !grow(&c->b.G_int, &c->cap_G_int, std::max<int64_t>(n_int * H, 4)) ||
+        !grow(&c->b.DX, &c->cap_DX, std::max<int64_t>(n_int * 2 * H, 4)))
+        return (int)cudaErrorMemoryAllocation;
+    const float *W = params + off[0], *W_out = params + off[1], *b = params + off[2], *b_out = params + off[3];
+    const uint32_t* ints = d_blob + lv_int;
+    const uint32_t* leaves = d_blob + lv_leaf;
+    const uint32_t* hl = d_blob + lv_head;
+    float *Xi = c->b.X_int, *Z = c->b.Z, *Gi = c->b.G_int, *DX = c->b.DX;
+    cublasStatus_t st = CUBLAS_STATUS_SUCCESS;
+#define BL(call) do { st = (call); if (st != CUBLAS_STATUS_SUCCESS) return 1000 + (int)st; } while (0)
+    if (n_leaf > 0) td_leaf<<<nblk(n_leaf * H), 256, 0, s>>>(inputs, leaves, (int)n_leaf, H, pool);
+    for (int32_t l = 1; l <= L; ++l) {
+        const int64_t r0 = lv_start[l], n = lv_start[l + 1] - r0;
+        if (n <= 0) continue;
+        float* X = Xi + r0 * 2 * H;
+        gather_int<<<nblk(n * (2 * H / 4)), 256, 0, s>>>(pool, ints + 6 * r0, (int)n, H, X);
+        BL(gemm_rm(c->blas, false, true, (int)n, H, 2 * H, X, 2 * H, W, 2 * H, Z, H, 0.f));
+        rv_cell<<<nblk(n * H), 256, 0, s>>>(Z, b, ints + 6 * r0, 6, (int)n, H, pool);
+    }
+    if (n_head > 0)
+        heads<<<(unsigned)n_head, 256, C * sizeof(float), s>>>(W_out, b_out, hl, H, C, pool, loss_word, grads + off[1],
+                                                             grads + off[3]);
+    for (int32_t l = L; l >= 1; --l) {
+        const int64_t r0 = lv_start[l], n = lv_start[l + 1] - r0;
+        if (n <= 0) continue;
+        float* G = Gi + r0 * H;
+        rv_bwd<<<nblk(n * H), 256, 0, s>>>(ints + 6 * r0, 6, 3, (int)n, H, pool, G);
+        BL(gemm_rm(c->blas, false, false, (int)n, 2 * H, H, G, H, W, 2 * H, DX, 2 * H, 0.f));
+        scatter_dh_shared<<<nblk(n * 2 * H), 256, 0, s>>>(DX, ints + 6 * r0, (int)n, H, pool);
+    }
+    if (n_leaf > 0 && d_inputs) td_leaf_dx<<<nblk(n_leaf * H), 256, 0, s>>>(leaves, (int)n_leaf, H, pool, d_inputs);
+    if (n_int > 0) {
+        BL(gemm_rm(c->blas, true, false, H, 2 * H, (int)n_int, Gi, H, Xi, 2 * H, grads + off[0], 2 * H, 0.f));
+        colsum<<<nblk(H), 256, 0, s>>>(Gi, (int)n_int, H, grads + off[2]);
     }
 #undef BL
     return (int)cudaGetLastError();

@@ -15,7 +15,7 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libvpps.so")
 
-CELLS = {"lstm": 0, "binary": 1, "childsum": 2, "bilstm": 3, "gru": 4, "rvnn": 5}
+CELLS = {"lstm": 0, "binary": 1, "childsum": 2, "bilstm": 3, "gru": 4, "rvnn": 5, "tdrnn": 6}
 STATUS = {0: "OK", -1: "INVALID", -2: "NOFIT", -3: "CUDA", -4: "GRAPH", -5: "STATE", -6: "NOMEM"}
 
 
@@ -119,6 +119,8 @@ def param_shapes(cell: str, H: int, E: int, C: int, mlp: int = 256):
                 ("bf", (4 * H,)), ("bb", (4 * H,)), ("b_mlp", (mlp,)), ("b_tag", (C,))]
     if cell == "lstm":
         return [("W", (4 * H, E)), ("U", (4 * H, H)), ("W_out", (C, H)), ("b", (4 * H,)), ("b_out", (C,))]
+    if cell == "tdrnn":
+        return [("W", (H, 2 * H)), ("W_out", (C, H)), ("b", (H,)), ("b_out", (C,))]
     if cell == "rvnn":
         return [("W_leaf", (H, E)), ("W_int", (H, 2 * H)), ("W_out", (C, H)), ("b_leaf", (H,)), ("b_int", (H,)),
                 ("b_out", (C,))]

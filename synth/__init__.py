@@ -126,8 +126,10 @@ CONFIGS = {
     "c4": dict(cell="bilstm", H=512, E=512, C=9, V=4096, batch=16, lengths=(5, 60), mlp=256),
     "c5": dict(cell="binary", H=1024, E=1024, C=5, V=4096, batch=64, leaves=(5, 50)),
     "tgt": dict(cell="binary", H=256, E=256, C=5, V=4096, batch=16, leaves=(5, 50)),
+    # paper's other workloads (Fig. 12: hidden = embedding = 512), SST-length sentences
+    "tdrnn": dict(cell="tdrnn", H=512, E=512, C=5, V=4096, batch=16, lengths=(5, 30)),
 }
-_CONFIG_IDS = {"c1": 1, "c2": 2, "c3": 3, "c4": 4, "c5": 5, "tgt": 6}
+_CONFIG_IDS = {"c1": 1, "c2": 2, "c3": 3, "c4": 4, "c5": 5, "tgt": 6, "tdrnn": 7}
 
 
 def config_batch(name: str, batch_idx: int, batch: int | None = None, **over):
@@ -138,6 +140,8 @@ def config_batch(name: str, batch_idx: int, batch: int | None = None, **over):
     rng = rng_for(_CONFIG_IDS[name], batch_idx)
     if cfg["cell"] in ("binary", "childsum"):
         return tree_batch(rng, b, cfg["leaves"], cfg["V"], cfg["C"])
+    if cfg["cell"] == "tdrnn":
+        return td_batch(rng, b, cfg["lengths"], cfg["V"], cfg["C"])
     if cfg["cell"] == "lstm":
         return [chain(rng, int(rng.integers(cfg["lengths"][0], cfg["lengths"][1] + 1)), cfg["V"], lm=True)
                 for _ in range(b)]

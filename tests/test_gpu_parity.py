@@ -408,3 +408,17 @@ def test_dataflow_batch_sweep(batch):
     are the largest the bench sees."""
     check("binary", 256, 256, 5, synth.config_batch("tgt", 40 + batch, batch=batch), 4096, seed=70 + batch,
           cluster=16, dataflow=True)
+
+
+def test_tdrnn_small():
+    """M7 TD-RNN (reading R-36): pyramids over sentences — every inner node below the top has two parents,
+    so a level's backward scatters two dh contributions into one child; includes a one-token sentence."""
+    rng = np.random.default_rng(71)
+    graphs = [synth.td_pyramid(rng, n, 16, 5) for n in (7, 1, 4, 12, 2)]
+    check("tdrnn", 32, 32, 5, graphs, 16, seed=71)
+
+
+def test_tdrnn_paper_size():
+    """TD-RNN at the paper's size (Fig. 12: hidden and embedding 512), SST-length sentences."""
+    graphs = synth.td_batch(np.random.default_rng(72), 4, lengths=(5, 20), vocab=4096)
+    check("tdrnn", 512, 512, 5, graphs, 4096, seed=72)

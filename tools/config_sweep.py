@@ -38,6 +38,7 @@ CASES = [
     ("GRU-LM H256 V1000 B64 (level path)", "c3", "gru", 256, 256, 1000, 1000, 64, {}, {}),
     ("RvNN H512 B16 (level path)", "tgt", "rvnn", 512, 512, 5, 4096, 16, {}, {}),
     ("RvNN H512 B64 (level path)", "tgt", "rvnn", 512, 512, 5, 4096, 64, {}, {}),
+    ("TD-RNN H512 B16 (level path)", "tdrnn", "tdrnn", 512, 512, 5, 4096, 16, {}, {}),
     ("c4 BiLSTM tagger H512 B16 (level path)", "c4", "bilstm", 512, 512, 9, 4096, 16, {"mlp": 256}, {}),
     ("c5 binary H1024 B64 (level path)", "c5", "binary", 1024, 1024, 5, 4096, 64, {}, {}),
     ("tgt binary H256 B16 (level path)", "tgt", "binary", 256, 256, 5, 4096, 16, {"level": 1}, {}),
@@ -101,7 +102,7 @@ def main():
         rec = {"case": label, "ms_per_step": round(ms, 4), "samples_per_s": round(B / ms * 1e3, 1),
                "nodes_per_s": round(nn / ms * 1e3, 1), "gflop_per_step": round(f / 1e9, 4),
                "tflops": round(f / ms / 1e9, 3), "frac_fp32_peak": round(f / (ms * 1e-3) / peak, 4),
-               "kernel": "vpps_df + GEMMs" if opts.get("dataflow") else ("level GEMMs" if (opts.get("level") or H > 256 or cell in ("bilstm", "gru", "rvnn") or C > 32) else "vpps_fb (grid)")}
+               "kernel": "vpps_df + GEMMs" if opts.get("dataflow") else ("level GEMMs" if (opts.get("level") or H > 256 or cell in ("bilstm", "gru", "rvnn", "tdrnn") or C > 32) else "vpps_fb (grid)")}
         lines.append(rec)
         print(json.dumps(rec), flush=True)
         del m
