@@ -23,6 +23,8 @@ L321) and the readings of SURVEY.md §8(c) c.2 / DESIGN.md "Readings" (R-1 … R
   M7  TD-RNN (reading R-36): a DAG over a sentence — level 0 the embeddings themselves
       (h = x, E = H), node i of level k: h = tanh(W [h_i; h_{i+1}] + b) over level k−1 (one composition
       function; inner nodes have two parents), the softmax head on the labelled top node
+  M8  TD-LSTM (reading R-37): M4's binary Tree-LSTM cell on the TD-RNN pyramid DAG (leaves are
+      M4 leaf cells on the tokens; shared children accumulate dh and dc from both parents)
   head: z = W_out h + b_out, ℓ = −log softmax(z)[y]  ("negative softmax log likelihood", L42)
 
 Everything is float64, node by node, in the graph's own order for the forward pass and in
@@ -33,7 +35,7 @@ from __future__ import annotations
 
 import numpy as np
 
-CELLS = ("lstm", "binary", "childsum", "bilstm", "gru", "rvnn", "tdrnn")
+CELLS = ("lstm", "binary", "childsum", "bilstm", "gru", "rvnn", "tdrnn", "tdlstm")
 
 
 def param_shapes(cell: str, H: int, E: int, C: int, M: int = 256):
@@ -43,7 +45,7 @@ def param_shapes(cell: str, H: int, E: int, C: int, M: int = 256):
     if cell == "lstm":
         return [("W", (4 * H, E)), ("U", (4 * H, H)), ("W_out", (C, H)),
                 ("b", (4 * H,)), ("b_out", (C,))]
-    if cell == "binary":
+    if cell in ("binary", "tdlstm"):
         return [("W_iou", (3 * H, E)), ("U_iou", (3 * H, 2 * H)), ("U_fl", (H, H)), ("U_fr", (H, H)),
                 ("W_out", (C, H)), ("b_iou", (3 * H,)), ("b_f", (H,)), ("b_out", (C,))]
     if cell == "childsum":
@@ -437,7 +439,8 @@ def _bilstm_graph(P, G, X, dX, nodes, H):
 
 
 _GRAPH_FN = {"lstm": _lstm_graph, "binary": _binary_graph, "childsum": _childsum_graph,
-             "bilstm": _bilstm_graph, "gru": _gru_graph, "rvnn": _rvnn_graph, "tdrnn": _tdrnn_graph}
+             "bilstm": _bilstm_graph, "gru": _gru_graph, "rvnn": _rvnn_graph, "tdrnn": _tdrnn_graph,
+             "tdlstm": _binary_graph}   # M4's reverse pass accumulates dh / dc (+=): correct on DAGs
 
 
 def validate(cell: str, graphs, n_tokens: int, n_classes: int):
@@ -448,7 +451,7 @@ def validate(cell: str, graphs, n_tokens: int, n_classes: int):
                 raise ValueError("children must precede their parent")
             if not (-1 <= tok < n_tokens) or not (-1 <= lab < n_classes):
                 raise ValueError("token/label out of range")
-            if cell in ("binary", "rvnn", "tdrnn") and not ((len(ch) == 0 and tok >= 0) or (len(ch) == 2 and tok < 0)):
+            if cell in ("binary", "rvnn", "tdrnn", "tdlstm") and not ((len(ch) == 0 and tok >= 0) or (len(ch) == 2 and tok < 0)):
                 raise ValueError("binary Tree-LSTM: leaves carry a token, internal nodes have 2 children")
             if cell in ("lstm", "bilstm", "gru") and (len(ch) > 1 or tok < 0 or (ch and ch[0] != v - 1)):
                 raise ValueError("LSTM chain: node t has child t-1 and a token")
@@ -456,7 +459,7 @@ def validate(cell: str, graphs, n_tokens: int, n_classes: int):
         for ch, _, _ in nodes:
             for k in ch:
                 parents[k] += 1
-        if cell != "tdrnn" and any(p > 1 for p in parents):      # TD-RNN is a DAG (R-36)
+        if cell not in ("tdrnn", "tdlstm") and any(p > 1 for p in parents):   # TD graphs are DAGs (R-36/37)
             raise ValueError("a node may have at most one parent")
 
 
@@ -484,7 +487,7 @@ def flop_count(cell: str, graphs, H: int, E: int, C: int, want_dx: bool = True, 
     kx = 3 if want_dx else 2
     for nodes in graphs:
         for ch, tok, lab in nodes:
-            if cell == "binary":
+            if cell in ("binary", "tdlstm"):
                 f += (2 * 3 * H * E * kx) if not ch else 2 * 3 * (3 * H * 2 * H + 2 * H * H)
             elif cell == "childsum":
                 k = len(ch)

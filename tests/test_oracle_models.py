@@ -181,6 +181,45 @@ def test_tdrnn_pyramid_equals_torch_conv1d():
     np.testing.assert_allclose(dX, Xt.grad.numpy(), atol=1e-12)
 
 
+def _unshare(nodes):
+    """Tree expansion of a DAG: every use of a shared node gets its own copy of its sub-DAG."""
+    out = []
+
+    def emit(v):
+        ch, tok, lab = nodes[v]
+        kids = tuple(emit(k) for k in ch)
+        out.append((kids, tok, -1))
+        return len(out) - 1
+
+    top = [v for v, (_, _, lab) in enumerate(nodes) if lab >= 0][0]
+    root = emit(top)
+    out[root] = (out[root][0], out[root][1], nodes[top][2])
+    return out
+
+
+def test_tdlstm_dag_equals_its_tree_expansion():
+    """M8 (reading R-37): the binary Tree-LSTM on a TD pyramid DAG equals M4 on the DAG's tree expansion
+    (each shared node duplicated per use) — loss, every weight gradient and dX are sums over the copies, so a
+    shared child that kept only one parent's dh or dc fails this.  M4 itself is pinned against torch LSTMCell
+    (test_binary_comb_equals_torch_lstmcell)."""
+    H, E, C, V = 3, 2, 4, 6
+    P = _params("binary", H, E, C, 13)
+    rng = np.random.default_rng(14)
+    X = rng.uniform(-1, 1, (V, E))
+    dags = [synth.td_pyramid(rng, n, V, C) for n in (4, 2, 5)]
+    l1, G1, dX1 = M.forward_backward("tdlstm", P, X, dags, H)
+    l2, G2, dX2 = M.forward_backward("binary", P, X, [_unshare(g) for g in dags], H)
+    assert abs(l1 - l2) < 1e-12
+    for k in G1:
+        np.testing.assert_allclose(G1[k], G2[k], atol=1e-12)
+    np.testing.assert_allclose(dX1, dX2, atol=1e-12)
+
+
+def test_fd_tdlstm():
+    rng = np.random.default_rng(15)
+    _fd_check("tdlstm", [synth.td_pyramid(rng, 3, 3, 3), synth.td_pyramid(rng, 2, 3, 3)], H=2, E=2, C=3, V=3)
+
+
 def test_gru_equals_torch_grucell():
     """M5 (reading R-34) == torch.nn.GRUCell in float64: torch stacks (r, z, n) in weight_ih / weight_hh
     with separate biases and applies the reset gate to W_hn h + b_hn, as the oracle does — a swapped gate,
