@@ -65,10 +65,13 @@ typedef enum {
                                      W_leaf H×E, W_int H×2H, W_out C×H, b_leaf H, b_int H, b_out C;
                                      leaf h = tanh(W_leaf x + b_leaf), internal h = tanh(W_int [h_l; h_r]
                                      + b_int); level-synchronous path */
-    VPPS_CELL_TDRNN = 6           /* M7 (DESIGN reading R-36): DAGs — leaves are the input
+    VPPS_CELL_TDRNN = 6,          /* M7 (DESIGN reading R-36): DAGs — leaves are the input
                                      rows themselves (E = H), every inner node h = tanh(W [h_a; h_b] + b)
                                      with W H×2H, b H, and a node may feed two parents; W_out C×H, b_out C;
                                      level-synchronous path */
+    VPPS_CELL_TDLSTM = 7          /* M8 (DESIGN reading R-37): TREE_BINARY's cell and
+                                     parameters on TD pyramid DAGs (a node may feed two parents, its dh and
+                                     dc accumulate from both); level-synchronous path */
 } vpps_cell;
 
 typedef struct {

@@ -41,7 +41,8 @@ std::vector<Shape> expected_shapes(int32_t cell, int32_t H, int32_t E, int32_t C
         case CELL_GRU: return {{3 * H, E}, {3 * H, H}, {C, H}, {3 * H, 1}, {3 * H, 1}, {C, 1}};
         case CELL_RVNN: return {{H, E}, {H, 2 * H}, {C, H}, {H, 1}, {H, 1}, {C, 1}};
         case CELL_TDRNN: return {{H, 2 * H}, {C, H}, {H, 1}, {C, 1}};
-        case CELL_BINARY: return {{3 * H, E}, {3 * H, 2 * H}, {H, H}, {H, H}, {C, H}, {3 * H, 1}, {H, 1}, {C, 1}};
+        case CELL_BINARY:
+        case CELL_TDLSTM: return {{3 * H, E}, {3 * H, 2 * H}, {H, H}, {H, H}, {C, H}, {3 * H, 1}, {H, 1}, {C, 1}};
         case CELL_CHILDSUM: return {{3 * H, E}, {H, E}, {3 * H, H}, {H, H}, {C, H}, {3 * H, 1}, {H, 1}, {C, 1}};
     }
     return {};
@@ -117,7 +118,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     vpps_options o{};
     if (opt) o = *opt;
     const int32_t cell = ops->cell, H = ops->H, E = ops->E, C = ops->C, Mw = ops->mlp;
-    if (cell < 0 || cell > 6 || H <= 0 || E <= 0 || C <= 0) return fail(VPPS_E_INVALID, "bad op set");
+    if (cell < 0 || cell > 7 || H <= 0 || E <= 0 || C <= 0) return fail(VPPS_E_INVALID, "bad op set");
     if (cell == CELL_TDRNN && E != H) return fail(VPPS_E_INVALID, "TD-RNN: the leaves are the input rows (E == H)");
     if (cell == CELL_BILSTM && Mw <= 0) return fail(VPPS_E_INVALID, "BiLSTM tagger needs mlp > 0");
     std::vector<Shape> want = expected_shapes(cell, H, E, C, Mw);
@@ -140,7 +141,8 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     }
     m->n_floats = cur;
     int32_t n_sm = o.n_sm;
-    if (cell == CELL_BILSTM || cell == CELL_GRU || cell == CELL_RVNN || cell == CELL_TDRNN || (cell == CELL_LSTM && (o.level > 0 || (o.level == 0 && C > 32)))) {
+    if (cell == CELL_BILSTM || cell == CELL_GRU || cell == CELL_RVNN || cell == CELL_TDRNN || cell == CELL_TDLSTM ||
+        (cell == CELL_LSTM && (o.level > 0 || (o.level == 0 && C > 32)))) {
         // M2 and M5 (GRU) run on the level-synchronous path only (vpps_level.cu), and so does an LSTM LM
         // whose vocabulary head exceeds one CTA's shared memory (config 3 at V = 1000): no partition plan
         if (o.cluster > 1 || o.dataflow || o.level < 0) return fail(VPPS_E_INVALID, "this op set runs on the level path only");
@@ -587,10 +589,20 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     } else if (m->plan.level) {
         if (s->s.lv_int < 0) return fail(VPPS_E_INVALID, "script was not built for the level path");
         CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));   // (memset above: G > 1 only)
-        const int rc = (m->plan.cell == CELL_RVNN ? rvnn_pass : m->plan.cell == CELL_TDRNN ? tdrnn_pass : level_pass)(
-            m->level, m->params, m->offsets.data(), m->grads, m->pool, inputs, d_inputs, dwords, s->s.lv_int,
-            s->s.lv_leaf, s->s.lv_head, s->s.lv_start.data(), (int32_t)s->s.lv_start.size() - 2, s->s.lv_n_int,
-            s->s.lv_n_leaf, s->s.lv_n_head, m->plan.H, m->plan.E, m->plan.C, s->s.loss_word, st);
+        const int32_t Lv = (int32_t)s->s.lv_start.size() - 2;
+        const int rc =
+            m->plan.cell == CELL_RVNN
+                ? rvnn_pass(m->level, m->params, m->offsets.data(), m->grads, m->pool, inputs, d_inputs, dwords,
+                            s->s.lv_int, s->s.lv_leaf, s->s.lv_head, s->s.lv_start.data(), Lv, s->s.lv_n_int,
+                            s->s.lv_n_leaf, s->s.lv_n_head, m->plan.H, m->plan.E, m->plan.C, s->s.loss_word, st)
+            : m->plan.cell == CELL_TDRNN
+                ? tdrnn_pass(m->level, m->params, m->offsets.data(), m->grads, m->pool, inputs, d_inputs, dwords,
+                             s->s.lv_int, s->s.lv_leaf, s->s.lv_head, s->s.lv_start.data(), Lv, s->s.lv_n_int,
+                             s->s.lv_n_leaf, s->s.lv_n_head, m->plan.H, m->plan.E, m->plan.C, s->s.loss_word, st)
+                : level_pass(m->level, m->params, m->offsets.data(), m->grads, m->pool, inputs, d_inputs, dwords,
+                             s->s.lv_int, s->s.lv_leaf, s->s.lv_head, s->s.lv_start.data(), Lv, s->s.lv_n_int,
+                             s->s.lv_n_leaf, s->s.lv_n_head, m->plan.H, m->plan.E, m->plan.C, s->s.loss_word, st,
+                             m->plan.cell == CELL_TDLSTM);
         if (rc != 0) return fail(VPPS_E_CUDA, "level pass failed (code " + std::to_string(rc) + ")");
         if (mode == 1) launch_sgd(m->params, m->grads, m->n_floats, lr, wd, st);
     } else if (m->cluster) {

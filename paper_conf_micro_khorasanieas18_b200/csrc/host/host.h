@@ -9,7 +9,7 @@ namespace vpps {
 
 constexpr uint32_t NONE = 0xFFFFFFFFu;
 
-enum Cell : int32_t { CELL_LSTM = 0, CELL_BINARY = 1, CELL_CHILDSUM = 2, CELL_BILSTM = 3, CELL_GRU = 4, CELL_RVNN = 5, CELL_TDRNN = 6 };
+enum Cell : int32_t { CELL_LSTM = 0, CELL_BINARY = 1, CELL_CHILDSUM = 2, CELL_BILSTM = 3, CELL_GRU = 4, CELL_RVNN = 5, CELL_TDRNN = 6, CELL_TDLSTM = 7 };
 
 enum Op : uint32_t {
     OP_S = 0x01, OP_W = 0x02,

@@ -64,7 +64,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
             for (int32_t k = c0; k < c1; ++k) {
                 const int32_t ch = b.children[k];
                 if (ch < 0 || ch >= local) { *err = "children must precede their parent"; return -4; }
-                if (++parents_seen[ch] > 1 && plan.cell != CELL_TDRNN) {   // TD-RNN graphs are DAGs (R-36)
+                if (++parents_seen[ch] > 1 && plan.cell != CELL_TDRNN && plan.cell != CELL_TDLSTM) {   // TD DAGs (R-36/37)
                     *err = "a node may have at most one parent";
                     return -4;
                 }
@@ -73,6 +73,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
             switch (plan.cell) {
                 case CELL_RVNN:
                 case CELL_TDRNN:
+                case CELL_TDLSTM:
                 case CELL_BINARY:
                     if (nch == 0 && tok >= 0) nd.kind = K_LEAF;
                     else if (nch == 2 && tok < 0) nd.kind = K_INT;
@@ -367,7 +368,8 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     s.lv_int = s.lv_leaf = s.lv_head = -1;
     s.lv_n_int = s.lv_n_leaf = s.lv_n_head = 0;
     s.lv_start.clear();
-    if (plan.level && (plan.cell == CELL_BINARY || plan.cell == CELL_RVNN || plan.cell == CELL_TDRNN)) {
+    if (plan.level && (plan.cell == CELL_BINARY || plan.cell == CELL_RVNN || plan.cell == CELL_TDRNN ||
+                       plan.cell == CELL_TDLSTM)) {
         s.lv_int = (int64_t)s.blob.size();
         s.lv_start.assign(L + 2, 0);
         for (int32_t lv = 1; lv <= L + 1; ++lv) {

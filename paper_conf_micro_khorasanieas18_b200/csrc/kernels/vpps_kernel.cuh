@@ -79,7 +79,7 @@ void level_ctx_destroy(void* ctx);
 int level_pass(void* ctx, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
                float* d_inputs, const uint32_t* d_blob, int64_t lv_int, int64_t lv_leaf, int64_t lv_head,
                const int32_t* lv_start, int32_t L, int64_t n_int, int64_t n_leaf, int64_t n_head, int32_t H,
-               int32_t E, int32_t C, int64_t loss_word, cudaStream_t s);
+               int32_t E, int32_t C, int64_t loss_word, cudaStream_t s, bool shared = false);
 int rvnn_pass(void* ctx, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
               float* d_inputs, const uint32_t* d_blob, int64_t lv_int, int64_t lv_leaf, int64_t lv_head,
               const int32_t* lv_start, int32_t L, int64_t n_int, int64_t n_leaf, int64_t n_head, int32_t H,

@@ -137,7 +137,8 @@ __global__ void heads(const float* __restrict__ Wo, const float* __restrict__ bo
 
 // internal cell backward (c.2b): given dh, dc (adj) -> gate gradients g = [g_i g_o g_u g_fl g_fr] into the
 // record and the level's G rows; the children's dc (each child has this node as its only parent)
-__global__ void int_bwd(const uint32_t* __restrict__ nodes, int n, int H, float* pool, float* __restrict__ G) {
+__global__ void int_bwd(const uint32_t* __restrict__ nodes, int n, int H, float* pool, float* __restrict__ G,
+                        bool shared = false) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)n * H) return;
     const int r = (int)(t / H), j = (int)(t % H);
@@ -155,8 +156,13 @@ __global__ void int_bwd(const uint32_t* __restrict__ nodes, int n, int H, float*
     float* Gr = G + (int64_t)r * 5 * H;
 #pragma unroll
     for (int k = 0; k < 5; ++k) { gr[k * H + j] = g[k]; Gr[k * H + j] = g[k]; }
-    pool[e[4] + H + j] = chat * fl;
-    pool[e[5] + H + j] = chat * fr;
+    if (shared) {             // TD-LSTM (R-37): a child may have two parents in the level
+        atomicAdd(pool + e[4] + H + j, chat * fl);
+        atomicAdd(pool + e[5] + H + j, chat * fr);
+    } else {
+        pool[e[4] + H + j] = chat * fl;
+        pool[e[5] + H + j] = chat * fr;
+    }
 }
 
 // children's dh += DX rows (left half -> child l, right half -> child r); unique parent: plain adds
@@ -522,7 +528,8 @@ static inline unsigned nblk(int64_t n, int t = 256) { return (unsigned)((n + t -
 int level_pass(void* ctx_, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
                float* d_inputs, const uint32_t* d_blob, int64_t lv_int, int64_t lv_leaf, int64_t lv_head,
                const int32_t* lv_start, int32_t L, int64_t n_int, int64_t n_leaf, int64_t n_head, int32_t H,
-               int32_t E, int32_t C, int64_t loss_word, cudaStream_t s) {
+               int32_t E, int32_t C, int64_t loss_word, cudaStream_t s, bool shared) {
+    // shared: TD-LSTM DAGs (R-37) — children's dh and dc accumulate atomically (two parents per level)
     using namespace dev::lv;
     LevelCtx* c = static_cast<LevelCtx*>(ctx_);
     cublasSetStream(c->blas, s);
@@ -573,12 +580,13 @@ int level_pass(void* ctx_, const float* params, const int64_t* off, float* grads
         const int64_t r0 = lv_start[l], n = lv_start[l + 1] - r0;
         if (n <= 0) continue;
         float* G = Gi + r0 * 5 * H;
-        int_bwd<<<nblk(n * H), 256, 0, s>>>(ints + 6 * r0, (int)n, H, pool, G);
+        int_bwd<<<nblk(n * H), 256, 0, s>>>(ints + 6 * r0, (int)n, H, pool, G, shared);
         // [dh_l; dh_r] = U_iouᵀ g_iou, dh_l += U_flᵀ g_fl, dh_r += U_frᵀ g_fr
         BL(gemm_rm(c->blas, false, false, (int)n, 2 * H, 3 * H, G, 5 * H, U_iou, 2 * H, DX, 2 * H, 0.f));
         BL(gemm_rm(c->blas, false, false, (int)n, H, H, G + 3 * H, 5 * H, U_fl, H, DX, 2 * H, 1.f));
         BL(gemm_rm(c->blas, false, false, (int)n, H, H, G + 4 * H, 5 * H, U_fr, H, DX + H, 2 * H, 1.f));
-        scatter_dh<<<nblk(n * 2 * H), 256, 0, s>>>(DX, ints + 6 * r0, (int)n, H, pool);
+        if (shared) scatter_dh_shared<<<nblk(n * 2 * H), 256, 0, s>>>(DX, ints + 6 * r0, (int)n, H, pool);
+        else scatter_dh<<<nblk(n * 2 * H), 256, 0, s>>>(DX, ints + 6 * r0, (int)n, H, pool);
     }
     if (n_leaf > 0) {
         leaf_bwd<<<nblk(n_leaf * H), 256, 0, s>>>(leaves, (int)n_leaf, H, pool, Gl);

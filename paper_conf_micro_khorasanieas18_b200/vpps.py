@@ -15,7 +15,7 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libvpps.so")
 
-CELLS = {"lstm": 0, "binary": 1, "childsum": 2, "bilstm": 3, "gru": 4, "rvnn": 5, "tdrnn": 6}
+CELLS = {"lstm": 0, "binary": 1, "childsum": 2, "bilstm": 3, "gru": 4, "rvnn": 5, "tdrnn": 6, "tdlstm": 7}
 STATUS = {0: "OK", -1: "INVALID", -2: "NOFIT", -3: "CUDA", -4: "GRAPH", -5: "STATE", -6: "NOMEM"}
 
 
@@ -127,7 +127,7 @@ def param_shapes(cell: str, H: int, E: int, C: int, mlp: int = 256):
     if cell == "gru":
         return [("W", (3 * H, E)), ("U", (3 * H, H)), ("W_out", (C, H)), ("b_i", (3 * H,)), ("b_h", (3 * H,)),
                 ("b_out", (C,))]
-    if cell == "binary":
+    if cell in ("binary", "tdlstm"):
         return [("W_iou", (3 * H, E)), ("U_iou", (3 * H, 2 * H)), ("U_fl", (H, H)), ("U_fr", (H, H)),
                 ("W_out", (C, H)), ("b_iou", (3 * H,)), ("b_f", (H,)), ("b_out", (C,))]
     if cell == "childsum":

@@ -422,3 +422,11 @@ def test_tdrnn_paper_size():
     """TD-RNN at the paper's size (Fig. 12: hidden and embedding 512), SST-length sentences."""
     graphs = synth.td_batch(np.random.default_rng(72), 4, lengths=(5, 20), vocab=4096)
     check("tdrnn", 512, 512, 5, graphs, 4096, seed=72)
+
+
+def test_tdlstm_small_and_paper_size():
+    """M8 TD-LSTM (reading R-37): the binary Tree-LSTM cell on TD pyramids (shared children: dh and dc from
+    two parents per level, accumulated atomically) — small shapes and the paper's H = E = 256."""
+    rng = np.random.default_rng(81)
+    check("tdlstm", 32, 32, 5, [synth.td_pyramid(rng, n, 16, 5) for n in (6, 1, 3, 9)], 16, seed=81)
+    check("tdlstm", 256, 256, 5, synth.td_batch(np.random.default_rng(82), 4, lengths=(5, 20)), 4096, seed=82)

@@ -39,6 +39,7 @@ CASES = [
     ("RvNN H512 B16 (level path)", "tgt", "rvnn", 512, 512, 5, 4096, 16, {}, {}),
     ("RvNN H512 B64 (level path)", "tgt", "rvnn", 512, 512, 5, 4096, 64, {}, {}),
     ("TD-RNN H512 B16 (level path)", "tdrnn", "tdrnn", 512, 512, 5, 4096, 16, {}, {}),
+    ("TD-LSTM H256 B16 (level path)", "tdrnn", "tdlstm", 256, 256, 5, 4096, 16, {}, {}),
     ("c4 BiLSTM tagger H512 B16 (level path)", "c4", "bilstm", 512, 512, 9, 4096, 16, {"mlp": 256}, {}),
     ("c5 binary H1024 B64 (level path)", "c5", "binary", 1024, 1024, 5, 4096, 64, {}, {}),
     ("tgt binary H256 B16 (level path)", "tgt", "binary", 256, 256, 5, 4096, 16, {"level": 1}, {}),
@@ -102,7 +103,7 @@ def main():
         rec = {"case": label, "ms_per_step": round(ms, 4), "samples_per_s": round(B / ms * 1e3, 1),
                "nodes_per_s": round(nn / ms * 1e3, 1), "gflop_per_step": round(f / 1e9, 4),
                "tflops": round(f / ms / 1e9, 3), "frac_fp32_peak": round(f / (ms * 1e-3) / peak, 4),
-               "kernel": "vpps_df + GEMMs" if opts.get("dataflow") else ("level GEMMs" if (opts.get("level") or H > 256 or cell in ("bilstm", "gru", "rvnn", "tdrnn") or C > 32) else "vpps_fb (grid)")}
+               "kernel": "vpps_df + GEMMs" if opts.get("dataflow") else ("level GEMMs" if (opts.get("level") or H > 256 or cell in ("bilstm", "gru", "rvnn", "tdrnn", "tdlstm") or C > 32) else "vpps_fb (grid)")}
         lines.append(rec)
         print(json.dumps(rec), flush=True)
         del m
