@@ -491,11 +491,18 @@ struct TaggerBufs {
           *Gb = nullptr, *Hp = nullptr, *Zs = nullptr, *Mm = nullptr, *Z = nullptr, *dZ = nullptr, *dM = nullptr,
           *dHH = nullptr, *dHf = nullptr, *dHb = nullptr, *dCf = nullptr, *dCb = nullptr, *Gamf = nullptr,
           *Gamb = nullptr, *Gs = nullptr, *Dh = nullptr, *DX = nullptr;
+    float *Hp2 = nullptr, *Zs2 = nullptr, *Gs2 = nullptr, *Dh2 = nullptr;   // second direction's step buffers
     int64_t cap[24] = {0};
+    int64_t cap2[4] = {0};
 };
 
 struct LevelCtx {
     cublasHandle_t blas = nullptr;
+    // BiLSTM tagger: the backward-direction chain runs on a second stream (its own cuBLAS handle), joined
+    // by events — the two directions are independent until the head
+    cublasHandle_t blas2 = nullptr;
+    cudaStream_t s2 = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     LevelBufs b;
     TaggerBufs tg;
     int64_t cap_X_leaf = 0, cap_X_int = 0, cap_Z = 0, cap_G_int = 0, cap_G_leaf = 0, cap_DX = 0;
@@ -504,6 +511,16 @@ struct LevelCtx {
 void* level_ctx_create() {
     LevelCtx* c = new LevelCtx;
     if (cublasCreate(&c->blas) != CUBLAS_STATUS_SUCCESS) { delete c; return nullptr; }
+    if (cublasCreate(&c->blas2) != CUBLAS_STATUS_SUCCESS ||
+        cudaStreamCreateWithFlags(&c->s2, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming) != cudaSuccess) {
+        cublasDestroy(c->blas);
+        delete c;
+        return nullptr;
+    }
+    cublasSetMathMode(c->blas2, CUBLAS_PEDANTIC_MATH);
+    cublasSetStream(c->blas2, c->s2);
     cublasSetMathMode(c->blas, CUBLAS_PEDANTIC_MATH);     // plain FP32 (no TF32, no emulation)
     return c;
 }
@@ -512,11 +529,15 @@ void level_ctx_destroy(void* p) {
     LevelCtx* c = static_cast<LevelCtx*>(p);
     if (!c) return;
     if (c->blas) cublasDestroy(c->blas);
+    if (c->blas2) cublasDestroy(c->blas2);
+    if (c->s2) cudaStreamDestroy(c->s2);
+    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+    if (c->ev_join) cudaEventDestroy(c->ev_join);
     float* bufs[] = {c->b.X_leaf, c->b.X_int, c->b.Z, c->b.G_int, c->b.G_leaf, c->b.DX};
     for (float* q : bufs) if (q) cudaFree(q);
     TaggerBufs& t = c->tg;
     float* tbufs[] = {t.X, t.Pf, t.Pb, t.HH, t.Cf, t.Cb, t.Gf, t.Gb, t.Hp, t.Zs, t.Mm, t.Z, t.dZ, t.dM, t.dHH, t.dHf,
-                      t.dHb, t.dCf, t.dCb, t.Gamf, t.Gamb, t.Gs, t.Dh, t.DX};
+                      t.dHb, t.dCf, t.dCb, t.Gamf, t.Gamb, t.Gs, t.Dh, t.DX, t.Hp2, t.Zs2, t.Gs2, t.Dh2};
     for (float* q : tbufs) if (q) cudaFree(q);
     delete c;
 }
@@ -628,6 +649,12 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
                               Tn * H, Tn * H, Tn * H, Tn * H, Tn * 4 * H, Tn * 4 * H, Tn * 4 * H, Tn * H, Tn * E};
     for (int k = 0; k < 24; ++k)
         if (!grow(bufs[k], &tb.cap[k], need[k])) return (int)cudaErrorMemoryAllocation;
+    if (dirs > 1) {
+        float** b2[4] = {&tb.Hp2, &tb.Zs2, &tb.Gs2, &tb.Dh2};
+        const int64_t n2[4] = {Tn * H, Tn * 4 * H, Tn * 4 * H, Tn * H};
+        for (int k = 0; k < 4; ++k)
+            if (!grow(b2[k], &tb.cap2[k], n2[k])) return (int)cudaErrorMemoryAllocation;
+    }
     auto P_ = [&](int k) -> const float* { return off[k] >= 0 ? params + off[k] : nullptr; };
     const float *Wf = P_(0), *Uf = P_(1), *Wb = P_(2), *Ub = P_(3), *Wm = P_(4), *Wt = P_(5), *bf = P_(6),
                 *bb = P_(7), *bm = P_(8), *bt = P_(9);
@@ -638,21 +665,34 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
     tg_gather_x<<<nblk(T * (E / 4)), 256, 0, s>>>(inputs, tok, (int)T, E, tb.X);
     BL(gemm_rm(c->blas, false, true, (int)T, 4 * H, E, tb.X, E, Wf, E, tb.Pf, 4 * H, 0.f));
     if (dirs > 1) BL(gemm_rm(c->blas, false, true, (int)T, 4 * H, E, tb.X, E, Wb, E, tb.Pb, 4 * H, 0.f));
-    // forward over the time steps, both directions (independent chains)
+    // forward over the time steps; the two directions are independent chains: the backward one runs on
+    // the second stream (its own h_prev / recurrent-product buffers), joined before the head
+    if (dirs > 1) {
+        cudaEventRecord(c->ev_fork, s);
+        cudaStreamWaitEvent(c->s2, c->ev_fork, 0);
+    }
     for (int32_t t = 0; t < maxlen; ++t) {
         const int32_t r0 = start[t], n = start[t + 1] - r0;
         for (int d = 0; d < dirs; ++d) {
             const uint32_t* pos = (d == 0 ? fpos : bpos) + r0;
             const int dp = d == 0 ? -1 : 1;
             const float* U = d == 0 ? Uf : Ub;
+            cudaStream_t sd = d == 0 ? s : c->s2;
+            cublasHandle_t hd = d == 0 ? c->blas : c->blas2;
+            float* Hp = d == 0 ? tb.Hp : tb.Hp2;
+            float* Zs = d == 0 ? tb.Zs : tb.Zs2;
             if (t > 0) {
-                tg_gather_hprev<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.HH, pos, n, dp, d, H, HW, tb.Hp);
-                BL(gemm_rm(c->blas, false, true, n, 4 * H, H, tb.Hp, H, U, H, tb.Zs, 4 * H, 0.f));
+                tg_gather_hprev<<<nblk((int64_t)n * H), 256, 0, sd>>>(tb.HH, pos, n, dp, d, H, HW, Hp);
+                BL(gemm_rm(hd, false, true, n, 4 * H, H, Hp, H, U, H, Zs, 4 * H, 0.f));
             }
-            tg_cell<<<nblk((int64_t)n * H), 256, 0, s>>>(d == 0 ? tb.Pf : tb.Pb, tb.Zs, d == 0 ? bf : bb, pos, n, dp,
-                                                           t == 0, d, H, HW, tb.HH, d == 0 ? tb.Cf : tb.Cb,
-                                                           d == 0 ? tb.Gf : tb.Gb);
+            tg_cell<<<nblk((int64_t)n * H), 256, 0, sd>>>(d == 0 ? tb.Pf : tb.Pb, Zs, d == 0 ? bf : bb, pos, n, dp,
+                                                            t == 0, d, H, HW, tb.HH, d == 0 ? tb.Cf : tb.Cb,
+                                                            d == 0 ? tb.Gf : tb.Gb);
         }
+    }
+    if (dirs > 1) {
+        cudaEventRecord(c->ev_join, c->s2);
+        cudaStreamWaitEvent(s, c->ev_join, 0);
     }
     // head over all positions: BiLSTM tagger m = tanh(W_mlp [h→; h←] + b_mlp) (MLP 256), then
     // z = W_tag m + b_tag; LSTM LM z = W_out h + b_out (L42); forward and backward
@@ -680,20 +720,32 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
     cudaMemsetAsync(tb.dHb, 0, T * H * sizeof(float), s);
     cudaMemsetAsync(tb.dCf, 0, T * H * sizeof(float), s);
     cudaMemsetAsync(tb.dCb, 0, T * H * sizeof(float), s);
+    if (dirs > 1) {
+        cudaEventRecord(c->ev_fork, s);
+        cudaStreamWaitEvent(c->s2, c->ev_fork, 0);
+    }
     for (int32_t t = maxlen - 1; t >= 0; --t) {
         const int32_t r0 = start[t], n = start[t + 1] - r0;
         for (int d = 0; d < dirs; ++d) {
             const uint32_t* pos = (d == 0 ? fpos : bpos) + r0;
             const int dp = d == 0 ? -1 : 1;
             float* dHr = d == 0 ? tb.dHf : tb.dHb;
-            tg_cell_bwd<<<nblk((int64_t)n * H), 256, 0, s>>>(pos, n, dp, t == 0, d, H, HW, tb.dHH, dHr, d == 0 ? tb.dCf : tb.dCb,
-                                                               d == 0 ? tb.Cf : tb.Cb, d == 0 ? tb.Gf : tb.Gb,
-                                                               d == 0 ? tb.Gamf : tb.Gamb, tb.Gs);
+            cudaStream_t sd = d == 0 ? s : c->s2;
+            cublasHandle_t hd = d == 0 ? c->blas : c->blas2;
+            float* Gs = d == 0 ? tb.Gs : tb.Gs2;
+            float* Dh = d == 0 ? tb.Dh : tb.Dh2;
+            tg_cell_bwd<<<nblk((int64_t)n * H), 256, 0, sd>>>(pos, n, dp, t == 0, d, H, HW, tb.dHH, dHr, d == 0 ? tb.dCf : tb.dCb,
+                                                                d == 0 ? tb.Cf : tb.Cb, d == 0 ? tb.Gf : tb.Gb,
+                                                                d == 0 ? tb.Gamf : tb.Gamb, Gs);
             if (t > 0) {
-                BL(gemm_rm(c->blas, false, false, n, H, 4 * H, tb.Gs, 4 * H, d == 0 ? Uf : Ub, H, tb.Dh, H, 0.f));
-                tg_scatter_dh<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.Dh, pos, n, dp, H, dHr);
+                BL(gemm_rm(hd, false, false, n, H, 4 * H, Gs, 4 * H, d == 0 ? Uf : Ub, H, Dh, H, 0.f));
+                tg_scatter_dh<<<nblk((int64_t)n * H), 256, 0, sd>>>(Dh, pos, n, dp, H, dHr);
             }
         }
+    }
+    if (dirs > 1) {
+        cudaEventRecord(c->ev_join, c->s2);
+        cudaStreamWaitEvent(s, c->ev_join, 0);
     }
     // weight gradients: dW = Γᵀ X, dU = Γᵀ H_prev (zeros at chain starts), db = Σ Γ; dX = Γf Wf + Γb Wb
     for (int d = 0; d < dirs; ++d) {
