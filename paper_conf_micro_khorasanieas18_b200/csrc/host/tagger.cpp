@@ -41,18 +41,24 @@ int build_tagger_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows
     s.tg_lab = (int64_t)s.blob.size();
     for (int32_t g = 0; g < b.n_graphs; ++g)
         for (int32_t t = 0; t < len[g]; ++t) s.blob.push_back((uint32_t)b.label[b.graph_ptr[g] + t]);
+    // step lists with the sentences longest first: the sentences still running at step t are then a prefix
+    // of those at step t-1, so row r of step t continues row r of step t-1 (the device reads h_prev and the
+    // successor's dh as row-aligned step blocks, without gathers or scatters)
+    std::vector<int32_t> order(b.n_graphs);
+    for (int32_t g = 0; g < b.n_graphs; ++g) order[g] = g;
+    std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t c) { return len[a] > len[c]; });
     s.tg_start.assign(maxlen + 1, 0);
     s.tg_fpos = (int64_t)s.blob.size();
     int32_t k = 0;
     for (int32_t t = 0; t < maxlen; ++t) {
         s.tg_start[t] = k;
-        for (int32_t g = 0; g < b.n_graphs; ++g)
+        for (int32_t g : order)
             if (len[g] > t) { s.blob.push_back((uint32_t)(off[g] + t)); ++k; }
     }
     s.tg_start[maxlen] = k;
     s.tg_bpos = (int64_t)s.blob.size();
     for (int32_t t = 0; t < maxlen; ++t)
-        for (int32_t g = 0; g < b.n_graphs; ++g)
+        for (int32_t g : order)
             if (len[g] > t) s.blob.push_back((uint32_t)(off[g] + len[g] - 1 - t));
     // pool: the loss word only (the tagger's activations live in the path's work buffers)
     s.loss_word = 0;

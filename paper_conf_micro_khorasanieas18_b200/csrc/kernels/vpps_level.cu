@@ -240,7 +240,7 @@ __global__ void tg_gather_hprev(const float* __restrict__ HH, const uint32_t* __
 // LSTM step (M1, gates i f o g): a = P[pos] + Zs[r] (recurrent, absent at t = 0) + b
 __global__ void tg_cell(const float* __restrict__ P, const float* __restrict__ Zs, const float* __restrict__ b,
                         const uint32_t* __restrict__ pos, int n, int dp, bool first, int d, int H, int HW, float* HH,
-                        float* Cd, float* Gd) {
+                        float* Cd, float* Gd, float* HS) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)n * H) return;
     const int r = (int)(t / H), j = (int)(t % H);
@@ -252,7 +252,9 @@ __global__ void tg_cell(const float* __restrict__ P, const float* __restrict__ Z
     const float i = sigm(a[0]), f = sigm(a[1]), o = sigm(a[2]), g = tanhf(a[3]);
     const float cp = first ? 0.f : Cd[(p + dp) * H + j];
     const float c = f * cp + i * g;
-    HH[p * HW + d * H + j] = o * tanhf(c);
+    const float h = o * tanhf(c);
+    HH[p * HW + d * H + j] = h;
+    HS[t] = h;                        // step-major copy: the next step's recurrent product reads it in place
     Cd[p * H + j] = c;
     float* gr = Gd + p * 4 * H;
     gr[j] = i; gr[H + j] = f; gr[2 * H + j] = o; gr[3 * H + j] = g;
@@ -293,13 +295,14 @@ __global__ void tg_dtanh(float* dM, const float* __restrict__ Mm, int64_t n) {
 // LSTM step backward (c.2b M1): dh = dHH[pos] (head) + dHr[pos] (from the next step), dc = dCr[pos];
 // γ -> Gam[pos] and the step buffer Gs[r]; dc_prev -> dCr[pos + dp]
 __global__ void tg_cell_bwd(const uint32_t* __restrict__ pos, int n, int dp, bool first, int d, int H, int HW,
-                            const float* __restrict__ dHH, const float* __restrict__ dHr, float* dCr,
+                            const float* __restrict__ dHH, const float* __restrict__ DhN, int n_next, float* dCr,
                             const float* __restrict__ Cd, const float* __restrict__ Gd, float* Gam, float* Gs) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)n * H) return;
     const int r = (int)(t / H), j = (int)(t % H);
     const int64_t p = pos[r];
-    const float dh = dHH[p * HW + d * H + j] + dHr[p * H + j], dc = dCr[p * H + j];
+    // recurrent dh: row r of the successor step's Γ Uᵀ block (the successor step has n_next <= n rows)
+    const float dh = dHH[p * HW + d * H + j] + (r < n_next ? DhN[t] : 0.f), dc = dCr[p * H + j];
     const float* gr = Gd + p * 4 * H;
     const float i = gr[j], f = gr[H + j], o = gr[2 * H + j], g = gr[3 * H + j];
     const float c = Cd[p * H + j], cp = first ? 0.f : Cd[(p + dp) * H + j];
@@ -341,7 +344,7 @@ __global__ void tg_scatter_dx(const float* __restrict__ DX, const uint32_t* __re
 // forward step: Gd[p] = (r, z, n, a_h[n]) for the backward
 __global__ void gru_cell(const float* __restrict__ Px, const float* __restrict__ Zs, const float* __restrict__ b_i,
                          const float* __restrict__ b_h, const uint32_t* __restrict__ pos, int n, int dp, bool first,
-                         int H, float* HH, float* Gd) {
+                         int H, float* HH, float* Gd, float* HS) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)n * H) return;
     const int r = (int)(t / H), j = (int)(t % H);
@@ -355,7 +358,9 @@ __global__ void gru_cell(const float* __restrict__ Px, const float* __restrict__
     const float zg = sigm(px[H + j] + b_i[H + j] + ahz);
     const float ng = tanhf(px[2 * H + j] + b_i[2 * H + j] + rg * ahn);
     const float hp = first ? 0.f : HH[(p + dp) * H + j];
-    HH[p * H + j] = (1.f - zg) * ng + zg * hp;
+    const float h = (1.f - zg) * ng + zg * hp;
+    HH[p * H + j] = h;
+    HS[t] = h;                        // step-major copy for the next step's recurrent product
     float* g = Gd + p * 4 * H;
     g[j] = rg; g[H + j] = zg; g[2 * H + j] = ng; g[3 * H + j] = ahn;
 }
@@ -363,14 +368,16 @@ __global__ void gru_cell(const float* __restrict__ Px, const float* __restrict__
 // backward step: dh = dHH[p] (head) + dHr[p] (successor); γ_x -> Gx[p], γ_h -> Gh[p] and the step buffer
 // Gs[r]; the direct term dh ⊙ z of dh_prev -> Ez[r]
 __global__ void gru_cell_bwd(const uint32_t* __restrict__ pos, int n, int dp, bool first, int H,
-                             const float* __restrict__ dHH, const float* __restrict__ dHr,
+                             const float* __restrict__ dHH, const float* __restrict__ DhN,
+                             const float* __restrict__ EzN, int n_next,
                              const float* __restrict__ HH, const float* __restrict__ Gd, float* Gx, float* Gh,
                              float* Gs, float* Ez) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)n * H) return;
     const int r = (int)(t / H), j = (int)(t % H);
     const int64_t p = pos[r];
-    const float dh = dHH[p * H + j] + dHr[p * H + j];
+    // recurrent dh from the successor step's row r: Γ_h U + dh ⊙ z of that step
+    const float dh = dHH[p * H + j] + (r < n_next ? DhN[t] + EzN[t] : 0.f);
     const float* g = Gd + p * 4 * H;
     const float rg = g[j], zg = g[H + j], ng = g[2 * H + j], ahn = g[3 * H + j];
     const float hp = first ? 0.f : HH[(p + dp) * H + j];
@@ -492,8 +499,10 @@ struct TaggerBufs {
           *dHH = nullptr, *dHf = nullptr, *dHb = nullptr, *dCf = nullptr, *dCb = nullptr, *Gamf = nullptr,
           *Gamb = nullptr, *Gs = nullptr, *Dh = nullptr, *DX = nullptr;
     float *Hp2 = nullptr, *Zs2 = nullptr, *Gs2 = nullptr, *Dh2 = nullptr;   // second direction's step buffers
+    float *HS0 = nullptr, *HS1 = nullptr, *DhB0 = nullptr, *DhB1 = nullptr, *EzB = nullptr;   // step-major h, 2nd Dh
     int64_t cap[24] = {0};
     int64_t cap2[4] = {0};
+    int64_t cap3[5] = {0};
 };
 
 struct LevelCtx {
@@ -537,7 +546,8 @@ void level_ctx_destroy(void* p) {
     for (float* q : bufs) if (q) cudaFree(q);
     TaggerBufs& t = c->tg;
     float* tbufs[] = {t.X, t.Pf, t.Pb, t.HH, t.Cf, t.Cb, t.Gf, t.Gb, t.Hp, t.Zs, t.Mm, t.Z, t.dZ, t.dM, t.dHH, t.dHf,
-                      t.dHb, t.dCf, t.dCb, t.Gamf, t.Gamb, t.Gs, t.Dh, t.DX, t.Hp2, t.Zs2, t.Gs2, t.Dh2};
+                      t.dHb, t.dCf, t.dCb, t.Gamf, t.Gamb, t.Gs, t.Dh, t.DX, t.Hp2, t.Zs2, t.Gs2, t.Dh2,
+                      t.HS0, t.HS1, t.DhB0, t.DhB1, t.EzB};
     for (float* q : tbufs) if (q) cudaFree(q);
     delete c;
 }
@@ -649,6 +659,12 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
                               Tn * H, Tn * H, Tn * H, Tn * H, Tn * 4 * H, Tn * 4 * H, Tn * 4 * H, Tn * H, Tn * E};
     for (int k = 0; k < 24; ++k)
         if (!grow(bufs[k], &tb.cap[k], need[k])) return (int)cudaErrorMemoryAllocation;
+    {
+        float** b3[5] = {&tb.HS0, &tb.HS1, &tb.DhB0, &tb.DhB1, &tb.EzB};
+        const int64_t n3[5] = {Tn * H, dirs > 1 ? Tn * H : 4, Tn * H, dirs > 1 ? Tn * H : 4, 4};
+        for (int k = 0; k < 5; ++k)
+            if (!grow(b3[k], &tb.cap3[k], n3[k])) return (int)cudaErrorMemoryAllocation;
+    }
     if (dirs > 1) {
         float** b2[4] = {&tb.Hp2, &tb.Zs2, &tb.Gs2, &tb.Dh2};
         const int64_t n2[4] = {Tn * H, Tn * 4 * H, Tn * 4 * H, Tn * H};
@@ -679,15 +695,13 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
             const float* U = d == 0 ? Uf : Ub;
             cudaStream_t sd = d == 0 ? s : c->s2;
             cublasHandle_t hd = d == 0 ? c->blas : c->blas2;
-            float* Hp = d == 0 ? tb.Hp : tb.Hp2;
+            float* HS = d == 0 ? tb.HS0 : tb.HS1;        // step-major h of this direction
             float* Zs = d == 0 ? tb.Zs : tb.Zs2;
-            if (t > 0) {
-                tg_gather_hprev<<<nblk((int64_t)n * H), 256, 0, sd>>>(tb.HH, pos, n, dp, d, H, HW, Hp);
-                BL(gemm_rm(hd, false, true, n, 4 * H, H, Hp, H, U, H, Zs, 4 * H, 0.f));
-            }
+            if (t > 0)   // h_prev of row r = row r of the previous step's block (longest-first step lists)
+                BL(gemm_rm(hd, false, true, n, 4 * H, H, HS + (int64_t)start[t - 1] * H, H, U, H, Zs, 4 * H, 0.f));
             tg_cell<<<nblk((int64_t)n * H), 256, 0, sd>>>(d == 0 ? tb.Pf : tb.Pb, Zs, d == 0 ? bf : bb, pos, n, dp,
                                                             t == 0, d, H, HW, tb.HH, d == 0 ? tb.Cf : tb.Cb,
-                                                            d == 0 ? tb.Gf : tb.Gb);
+                                                            d == 0 ? tb.Gf : tb.Gb, HS + (int64_t)r0 * H);
         }
     }
     if (dirs > 1) {
@@ -729,18 +743,17 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
         for (int d = 0; d < dirs; ++d) {
             const uint32_t* pos = (d == 0 ? fpos : bpos) + r0;
             const int dp = d == 0 ? -1 : 1;
-            float* dHr = d == 0 ? tb.dHf : tb.dHb;
             cudaStream_t sd = d == 0 ? s : c->s2;
             cublasHandle_t hd = d == 0 ? c->blas : c->blas2;
             float* Gs = d == 0 ? tb.Gs : tb.Gs2;
-            float* Dh = d == 0 ? tb.Dh : tb.Dh2;
-            tg_cell_bwd<<<nblk((int64_t)n * H), 256, 0, sd>>>(pos, n, dp, t == 0, d, H, HW, tb.dHH, dHr, d == 0 ? tb.dCf : tb.dCb,
-                                                                d == 0 ? tb.Cf : tb.Cb, d == 0 ? tb.Gf : tb.Gb,
-                                                                d == 0 ? tb.Gamf : tb.Gamb, Gs);
-            if (t > 0) {
-                BL(gemm_rm(hd, false, false, n, H, 4 * H, Gs, 4 * H, d == 0 ? Uf : Ub, H, Dh, H, 0.f));
-                tg_scatter_dh<<<nblk((int64_t)n * H), 256, 0, sd>>>(Dh, pos, n, dp, H, dHr);
-            }
+            // Γ Uᵀ of step t goes to one buffer and is read by step t-1, whose product goes to the other
+            float* DhW = (t & 1) ? (d == 0 ? tb.Dh : tb.Dh2) : (d == 0 ? tb.DhB0 : tb.DhB1);
+            const float* DhR = (t & 1) ? (d == 0 ? tb.DhB0 : tb.DhB1) : (d == 0 ? tb.Dh : tb.Dh2);
+            const int32_t n_next = t + 1 < maxlen ? start[t + 2] - start[t + 1] : 0;
+            tg_cell_bwd<<<nblk((int64_t)n * H), 256, 0, sd>>>(pos, n, dp, t == 0, d, H, HW, tb.dHH, DhR, n_next,
+                                                                d == 0 ? tb.dCf : tb.dCb, d == 0 ? tb.Cf : tb.Cb,
+                                                                d == 0 ? tb.Gf : tb.Gb, d == 0 ? tb.Gamf : tb.Gamb, Gs);
+            if (t > 0) BL(gemm_rm(hd, false, false, n, H, 4 * H, Gs, 4 * H, d == 0 ? Uf : Ub, H, DhW, H, 0.f));
         }
     }
     if (dirs > 1) {
@@ -793,6 +806,8 @@ int gru_pass(void* ctx_, const float* params, const int64_t* off, float* grads, 
                               Tn * H, Tn * 3 * H, Tn * 3 * H, Tn * 3 * H, Tn * H, Tn * H, Tn * E};
     for (int k = 0; k < 16; ++k)
         if (!grow(bufs[k], caps[k], need[k])) return (int)cudaErrorMemoryAllocation;
+    if (!grow(&tb.HS0, &tb.cap3[0], Tn * H) || !grow(&tb.DhB0, &tb.cap3[2], Tn * H) || !grow(&tb.EzB, &tb.cap3[4], Tn * H))
+        return (int)cudaErrorMemoryAllocation;
     const float *W = params + off[0], *U = params + off[1], *Wo = params + off[2], *b_i = params + off[3],
                 *b_h = params + off[4], *bo = params + off[5];
     const uint32_t *tok = d_blob + tg_tok, *lab = d_blob + tg_lab, *fpos = d_blob + tg_fpos;
@@ -804,11 +819,10 @@ int gru_pass(void* ctx_, const float* params, const int64_t* off, float* grads, 
     for (int32_t t = 0; t < maxlen; ++t) {
         const int32_t r0 = start[t], n = start[t + 1] - r0;
         const uint32_t* pos = fpos + r0;
-        if (t > 0) {
-            tg_gather_hprev<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.HH, pos, n, -1, 0, H, H, tb.Hp);
-            BL(gemm_rm(c->blas, false, true, n, 3 * H, H, tb.Hp, H, U, H, tb.Zs, 3 * H, 0.f));
-        }
-        gru_cell<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.Pf, tb.Zs, b_i, b_h, pos, n, -1, t == 0, H, tb.HH, tb.Gf);
+        if (t > 0)   // h_prev of row r = row r of the previous step's block (longest-first step lists)
+            BL(gemm_rm(c->blas, false, true, n, 3 * H, H, tb.HS0 + (int64_t)start[t - 1] * H, H, U, H, tb.Zs, 3 * H, 0.f));
+        gru_cell<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.Pf, tb.Zs, b_i, b_h, pos, n, -1, t == 0, H, tb.HH, tb.Gf,
+                                                       tb.HS0 + (int64_t)r0 * H);
     }
     // head on h (L42): z = W_out h + b_out, softmax-NLL on labelled positions, dW_out, db_out, dh
     BL(gemm_rm(c->blas, false, true, (int)T, C, H, tb.HH, H, Wo, H, tb.Z, C, 0.f));
@@ -820,12 +834,15 @@ int gru_pass(void* ctx_, const float* params, const int64_t* off, float* grads, 
     for (int32_t t = maxlen - 1; t >= 0; --t) {
         const int32_t r0 = start[t], n = start[t + 1] - r0;
         const uint32_t* pos = fpos + r0;
-        gru_cell_bwd<<<nblk((int64_t)n * H), 256, 0, s>>>(pos, n, -1, t == 0, H, tb.dHH, tb.dHf, tb.HH, tb.Gf,
-                                                           tb.Gamf, tb.Gamb, tb.Gs, tb.Cf);
-        if (t > 0) {
-            BL(gemm_rm(c->blas, false, false, n, H, 3 * H, tb.Gs, 3 * H, U, H, tb.Dh, H, 0.f));
-            gru_scatter_dh<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.Dh, tb.Cf, pos, n, -1, H, tb.dHf);
-        }
+        // Γ_h U and dh ⊙ z of step t go to one buffer pair, read by step t-1 (row-aligned)
+        float* DhW = (t & 1) ? tb.Dh : tb.DhB0;
+        float* EzW = (t & 1) ? tb.Cf : tb.EzB;
+        const float* DhR = (t & 1) ? tb.DhB0 : tb.Dh;
+        const float* EzR = (t & 1) ? tb.EzB : tb.Cf;
+        const int32_t n_next = t + 1 < maxlen ? start[t + 2] - start[t + 1] : 0;
+        gru_cell_bwd<<<nblk((int64_t)n * H), 256, 0, s>>>(pos, n, -1, t == 0, H, tb.dHH, DhR, EzR, n_next, tb.HH,
+                                                           tb.Gf, tb.Gamf, tb.Gamb, tb.Gs, EzW);
+        if (t > 0) BL(gemm_rm(c->blas, false, false, n, H, 3 * H, tb.Gs, 3 * H, U, H, DhW, H, 0.f));
     }
     // dW = Γ_xᵀ X, dU = Γ_hᵀ H_prev (zeros at chain starts), db_i = Σ Γ_x, db_h = Σ Γ_h; dX = Γ_x W
     cudaMemsetAsync(tb.Hp, 0, T * H * sizeof(float), s);

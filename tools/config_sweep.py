@@ -55,6 +55,7 @@ def main():
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--only", default=None, help="run the cases whose label contains this substring")
     args = ap.parse_args()
     import torch
     import synth
@@ -63,6 +64,8 @@ def main():
     peak = 148 * 128 * 2 * mhz * 1e6
     lines = []
     for label, cfg, cell, H, E, C, V, B, opts, over in CASES:
+        if args.only and args.only not in label:
+            continue
         rng = np.random.default_rng(0)
         shapes = vpps.param_shapes(cell, H, E, C, opts.get("mlp", 256))
         P = synth.init_params(shapes, rng)
