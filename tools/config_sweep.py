@@ -3,7 +3,7 @@ the graded bench line is bench.py's target config).
 
     python tools/config_sweep.py [--steps 50] [--warmup 5] [--out FILE]
 
-Per case: 16 distinct pre-built, device-resident scripts cycled, fused forward + backward + SGD
+Per case: 16 distinct pre-built, device-resident scripts cycled (each run once untimed first), fused forward + backward + SGD
 (vpps_fwd_bwd_sgd), device time per step from CUDA events around the timed steps (no L2 flush: these are
 steady-state numbers), samples/s, nodes/s and the algorithmic FLOP rate (SURVEY §8(d) F counted by the host
 from the script) against the FP32 FFMA peak.
@@ -53,7 +53,9 @@ CASES = [
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--steps", type=int, default=50)
-    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=16,
+                    help="untimed passes; >= 16 runs every script once, so work buffers that grow with the "
+                         "largest script are allocated before the timed region")
     ap.add_argument("--out", default=None)
     ap.add_argument("--only", default=None, help="run the cases whose label contains this substring")
     args = ap.parse_args()
