@@ -548,7 +548,10 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         launch_leaf_fwd(W_iou, m->params + m->offsets[5], inputs, m->pool, leaf_list, (int32_t)s->s.n_leaf,
                         m->plan.H, m->plan.E, zero_ptr, zero_n, m->d_epoch, st);
         if (m->k_before) CK(cudaEventRecord(m->k_before, st));
-        CK(cudaLaunchKernelExC(&cfg, m->var->fn, dargs));
+        const void* dfn = m->prof ? df_prof_fn(m->var->fn) : m->var->fn;
+        if (!dfn) return fail(VPPS_E_STATE, "no trace-enabled dataflow kernel for this variant");
+        if (m->prof) CK(cudaFuncSetAttribute(dfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)m->smem));
+        CK(cudaLaunchKernelExC(&cfg, dfn, dargs));
         if (m->k_after) CK(cudaEventRecord(m->k_after, st));
         const int32_t n_grp = (int32_t)s->s.int_off.size() - 1;
         std::vector<int32_t> order(n_grp);

@@ -87,7 +87,9 @@ struct DCfg {
     static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 2 * C + 8); }
 };
 
-template <int H, int E>
+// PROF = false (the production instantiation): every trace stamp, section clock and per-batch record folds
+// away at compile time (prof is a constant nullptr); PROF = true when vpps_set_profile_buffer is active
+template <int H, int E, bool PROF>
 __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     using T = DCfg<H, E>;
     using LB = typename T::LB;
@@ -119,7 +121,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     const int j = lc * UM + u;                                  // hidden unit of this thread (blocked)
     const bool holds_head = (lc == 0);
 
-    if (P.prof && threadIdx.x == 0) P.prof[(int64_t)blockIdx.x * P.prof_stride + 11] = gtimer();   // entry
+    if (PROF && P.prof && threadIdx.x == 0) P.prof[(int64_t)blockIdx.x * P.prof_stride + 11] = gtimer();   // entry
     // ---- prologue: this CTA's rows of U_iou, U_fl, U_fr -> registers (L123, L129) ----
     float wb[4][LB::NREG];
 #pragma unroll
@@ -148,7 +150,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     }
     float dbacc[4] = {0.f, 0.f, 0.f, 0.f};   // bias gradients of unit j (thread (u, gl) mapping)
     float dbleaf[3] = {0.f, 0.f, 0.f};       // ... of unit lc * UM + tid % UM (LEAF_B mapping)
-    uint64_t* prof = P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
+    uint64_t* prof = PROF && P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
     // section clocks (trace only): 0 program, 1 staging, 2 tag wait, 3 forward, 4 cell-bwd, 5 transposed,
     // 6 heads, 7 other
     uint64_t sec[8] = {0, 0, 0, 0, 0, 0, 0, 0};
@@ -171,17 +173,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             sec_last = now;
         }
     };
-    // the leaf records and the pass counter (vpps_leaf_fwd, the preceding grid) are visible from here on
-    asm volatile("griddepcontrol.wait;" ::: "memory");
-    // the gradient GEMM (programmatic dependent of this grid) may launch from here on: it reads the
-    // `done` / claim counters the leaf grid cleared, which is complete and visible once every CTA of this
-    // grid has passed the wait above
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-    ep = *P.epoch;
-    __syncthreads();
-    if (prof && tid == 0) { prof[0] = gtimer(); sec_last = clock64(); }
-
-    // ---- program of this group: batches [op | nb << 8, nb entries] ----
+    // ---- program of this group: batches [op | nb << 8, nb entries].  The script was copied before the
+    //      leaf grid ran, so its first chunk loads while that grid drains (before griddepcontrol.wait) ----
     const uint32_t* S_ = P.script + P.df_off;
     const uint32_t G = S_[0];
     const uint32_t s0 = 2 + G + S_[1 + grp], s1 = 2 + G + S_[2 + grp];
@@ -193,6 +186,15 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         cbase = from;
     };
     if (s0 < s1) refill(s0);
+    // the leaf records and the pass counter (vpps_leaf_fwd, the preceding grid) are visible from here on
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    // the gradient GEMM (programmatic dependent of this grid) may launch from here on: it reads the
+    // `done` / claim counters the leaf grid cleared, which is complete and visible once every CTA of this
+    // grid has passed the wait above
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    ep = *P.epoch;
+    __syncthreads();
+    if (prof && tid == 0) { prof[0] = gtimer(); sec_last = clock64(); }
     uint32_t pos = s0;
     int nbatch = 0;
     int xdone = 0;            // fine stamps taken (trace only)
@@ -732,11 +734,17 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
 }  // namespace dev
 
 #define VPPS_DF_VARIANT(H, E) \
-    {1, H, E, 16, (const void*)&dev::df::vpps_df<H, E>, &dev::df::DCfg<H, E>::smem_bytes}
+    {1, H, E, 16, (const void*)&dev::df::vpps_df<H, E, false>, &dev::df::DCfg<H, E>::smem_bytes}
 
 static const Variant kDfVariants[] = {
     VPPS_DF_VARIANT(256, 256),    // target: binary Tree-LSTM H = E = 256, groups of 16 CTAs
 };
+
+// the profiling instantiation of a dataflow variant (same shared memory, in-kernel trace enabled)
+const void* df_prof_fn(const void* fn) {
+    if (fn == (const void*)&dev::df::vpps_df<256, 256, false>) return (const void*)&dev::df::vpps_df<256, 256, true>;
+    return nullptr;
+}
 
 const Variant* df_variants(int32_t* n) {
     *n = (int32_t)(sizeof(kDfVariants) / sizeof(kDfVariants[0]));
