@@ -32,7 +32,7 @@ def test_abi_exports_every_declared_symbol():
 
 
 def test_param_shapes_agree_with_oracle(vpps):
-    for cell in ("lstm", "binary", "childsum"):
+    for cell in ("lstm", "binary", "childsum", "gru", "rvnn", "tdlstm"):
         a = [(n, tuple(s)) for n, s in vpps.param_shapes(cell, 8, 4, 3)]
         b = [(n, tuple(s)) for n, s in M.param_shapes(cell, 8, 4, 3)]
         assert a == b
@@ -166,3 +166,23 @@ def test_nofit_and_bad_shapes(vpps):
     with pytest.raises(vpps.VppsError) as e:
         vpps.Model("binary", 4096, 4096, 5, n_sm=148, plan_only=True)
     assert e.value.status == -2
+
+
+def test_widened_cells_host_side(vpps):
+    """The NEXT-3 cells (GRU, RvNN, TD-RNN, TD-LSTM) on the host side: op sets accepted in plan-only mode,
+    scripts built, the DAG rule applied only to the TD cells, and the TD-RNN's E == H requirement."""
+    rng = np.random.default_rng(5)
+    assert vpps.param_shapes("tdrnn", 8, 8, 3) == M.param_shapes("tdrnn", 8, 8, 3)
+    gru = vpps.Model("gru", 8, 12, 5, plan_only=True)
+    info = gru.build_script([synth.chain(rng, 6, 5), synth.chain(rng, 1, 5)]).info()
+    assert info["n_levels"] == 6 and info["flops"] > 0
+    rv = vpps.Model("rvnn", 8, 12, 5, plan_only=True)
+    rv.build_script(synth.tree_batch(rng, 3, (1, 6), 8, 5))
+    dag = synth.td_pyramid(rng, 5, 8, 5)                       # inner nodes with two parents
+    td = vpps.Model("tdrnn", 8, 8, 5, plan_only=True)
+    assert td.build_script([dag]).info()["n_levels"] == 5
+    vpps.Model("tdlstm", 8, 8, 5, plan_only=True).build_script([dag])
+    with pytest.raises(vpps.VppsError):
+        rv.build_script([dag])                                  # shared children only in the TD cells
+    with pytest.raises(vpps.VppsError):
+        vpps.Model("tdrnn", 8, 12, 5, plan_only=True)           # leaves are the input rows: E == H
