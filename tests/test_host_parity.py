@@ -180,7 +180,7 @@ def test_widened_cells_host_side(vpps):
     rv.build_script(synth.tree_batch(rng, 3, (1, 6), 8, 5))
     dag = synth.td_pyramid(rng, 5, 8, 5)                       # inner nodes with two parents
     td = vpps.Model("tdrnn", 8, 8, 5, plan_only=True)
-    assert td.build_script([dag]).info()["n_levels"] == 5
+    assert td.build_script([dag]).info()["n_levels"] == 6           # 5 pyramid levels + the head
     vpps.Model("tdlstm", 8, 8, 5, plan_only=True).build_script([dag])
     with pytest.raises(vpps.VppsError):
         rv.build_script([dag])                                  # shared children only in the TD cells
