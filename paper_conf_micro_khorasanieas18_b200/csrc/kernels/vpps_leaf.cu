@@ -43,6 +43,7 @@ constexpr size_t SMEM = (size_t)(LM + 3 * LU) * KS * sizeof(float);
 // (multiples of 4 floats) are zeroed by a grid-stride loop, and the device pass counter is advanced.
 __device__ uint64_t g_leaf_prof[1024 * 8];   // measurement only (VPPS_LEAF_PROF): per-CTA phase stamps
 __device__ int g_leaf_prof_on;
+static int h_leaf_prof_on = 0;   // host copy: selects the trace-enabled instantiation (PROF = true)
 
 // barrier of the NT GEMM threads only (the clearing warps never join it)
 __device__ __forceinline__ void gemm_sync() { asm volatile("bar.sync 1, %0;" ::"n"(NT) : "memory"); }
@@ -53,7 +54,7 @@ struct PassClear {
     uint32_t* epoch;     // dataflow pass counter (tags of this pass), or nullptr
 };
 
-template <int E>
+template <int E, bool PROF>
 __global__ void __launch_bounds__(NT + NTC, 1) vpps_leaf_fwd(const float* __restrict__ W, const float* __restrict__ b,
                                                        const float* __restrict__ inputs, float* pool,
                                                        const uint32_t* __restrict__ leaves, int n_leaf, int H,
@@ -67,7 +68,8 @@ __global__ void __launch_bounds__(NT + NTC, 1) vpps_leaf_fwd(const float* __rest
     // the dataflow kernel may be scheduled as SMs free up (it waits for this grid with griddepcontrol.wait
     // before reading anything written here)
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-    const bool pf = g_leaf_prof_on && tid == 0 && blockIdx.x < 1024;
+    // production instantiation: no trace (the flag load and the stamps fold away)
+    const bool pf = PROF && tid == 0 && blockIdx.x < 1024 && g_leaf_prof_on;
     uint64_t* pst = g_leaf_prof + blockIdx.x * 8;
     if (pf) pst[0] = gtimer();
     if (pc.epoch && blockIdx.x == 0 && tid == 0) {
@@ -84,7 +86,7 @@ __global__ void __launch_bounds__(NT + NTC, 1) vpps_leaf_fwd(const float* __rest
             const int64_t n4 = pc.ptr[r] ? pc.n[r] / 4 : 0;
             for (int64_t i = (int64_t)blockIdx.x * NTC + (tid - NT); i < n4; i += stride) p[i] = make_float4(0.f, 0.f, 0.f, 0.f);
         }
-        if (g_leaf_prof_on && tid == NT && blockIdx.x < 1024) g_leaf_prof[blockIdx.x * 8 + 6] = gtimer();
+        if (PROF && tid == NT && blockIdx.x < 1024 && g_leaf_prof_on) g_leaf_prof[blockIdx.x * 8 + 6] = gtimer();
         return;
     }
     if (work) {
@@ -406,6 +408,7 @@ __global__ void __launch_bounds__(NT, 1) vpps_leaf_fwd_tc(const float* __restric
 
 extern "C" int vpps_leaf_prof(int on, uint64_t* out) {   // measurement tool hook (not in vpps.h)
     if (out) return (int)cudaMemcpyFromSymbol(out, dev::leaf::g_leaf_prof, sizeof(uint64_t) * 1024 * 8);
+    dev::leaf::h_leaf_prof_on = on;
     return (int)cudaMemcpyToSymbol(dev::leaf::g_leaf_prof_on, &on, sizeof(int));
 }
 
@@ -416,7 +419,8 @@ void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float*
     if (E != KMAX || H % LU) return;   // the cluster / dataflow variants are H = E = 256 (api.cu checks)
     static bool attr = false;
     if (!attr) {
-        cudaFuncSetAttribute(vpps_leaf_fwd<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+        cudaFuncSetAttribute(vpps_leaf_fwd<256, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+        cudaFuncSetAttribute(vpps_leaf_fwd<256, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
         cudaFuncSetAttribute(vpps_leaf_fwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TC_SMEM);
         attr = true;
     }
@@ -432,7 +436,8 @@ void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float*
     pc.epoch = epoch;
     if (simt) {
         const int tiles = std::max(((n_leaf + LM - 1) / LM) * (H / LU), 148);
-        vpps_leaf_fwd<256><<<tiles, NT + NTC, SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
+        if (h_leaf_prof_on) vpps_leaf_fwd<256, true><<<tiles, NT + NTC, SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
+        else vpps_leaf_fwd<256, false><<<tiles, NT + NTC, SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
     } else {
         // GEMM tiles first, then clearing CTAs: the SMs left over (at least 32 CTAs)
         const int tiles = ((n_leaf + TL - 1) / TL) * (H / LU);
