@@ -82,7 +82,10 @@ struct DCfg {
     static constexpr int O_CIN = O_DXB + DXB;
     static constexpr int O_BIAS = O_CIN + NB * UM * CINMAX;
     static constexpr int O_ZS = O_BIAS + UM * 4;
-    static constexpr int O_HEAD = O_ZS + NB * ZC;
+    // second staging buffers: consecutive batches alternate, so a batch needs no closing barrier
+    static constexpr int O_X2 = O_ZS + NB * ZC;
+    static constexpr int O_CIN2 = O_X2 + NB * KP;
+    static constexpr int O_HEAD = O_CIN2 + NB * UM * CINMAX;
     static_assert(DXB >= 2 * NB * KP && DXB >= 2 * NB * NCL * 2 * UM, "u64 staging fits in dxb");
     static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 2 * C + 8); }
 };
@@ -101,6 +104,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     float* dxb = sm + T::O_DXB;
     u64* tbuf = reinterpret_cast<u64*>(sm + T::O_DXB);     // tagged staging (aliases dxb)
     float* cin = sm + T::O_CIN;
+    int cbuf = 0;                                          // transposed-product buffer, alternating across batches
     float* bias = sm + T::O_BIAS;
     float* zs = sm + T::O_ZS;
     const int C = P.C;
@@ -210,6 +214,10 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         const bool is_head = op == HEAD_FB;
         if (is_head && !holds_head) { pos = next; continue; }
         ++nbatch;
+        // staging buffers of this batch: the other pair than the previous batch's (a thread still computing
+        // that batch reads only those); batch b+2 reuses them after batch b+1's staging barrier
+        xs = sm + ((nbatch & 1) ? T::O_X : T::O_X2);
+        cin = sm + ((nbatch & 1) ? T::O_CIN : T::O_CIN2);
         uint64_t* bt = (prof && tid == 0 && nbatch <= 48 && P.prof_stride >= 16 + 5 * 48) ? prof + 16 + 5 * (nbatch - 1) : nullptr;
         if (bt) { bt[0] = clock64(); bt[4] = op; }
         int rounds = 0;
@@ -619,7 +627,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 constexpr int NW = NTH / 32;
                 const int src = lane & 16;
                 const bool hi = lane & 16;
-                int cbuf = 0;
                 for (int n0 = 0; n0 < nb; n0 += NC, cbuf ^= 1) {
                     float* buf = dxb + cbuf * (NW * NC * KP);
 #pragma unroll
@@ -684,7 +691,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 XST(stBB, 30);
             }
         }
-        __syncthreads();
+        // (no closing barrier: the next batch stages into the other buffers, and every cross-batch reuse
+        //  of shared memory is ordered by a staging or refill barrier in between)
         XST(stF, 4);
         XST(stB, 11);
         XST(stBB, 31);
