@@ -71,7 +71,7 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, flo
 // and advances the device pass counter `epoch` (if not null): the per-pass clearing without memset calls.
 void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float* pool, const uint32_t* leaves,
                      int32_t n_leaf, int32_t H, int32_t E, float* const* zero_ptr, const int64_t* zero_n,
-                     uint32_t* epoch, cudaStream_t s);
+                     uint32_t* epoch, cudaStream_t s, const void* prefetch = nullptr, int64_t prefetch_bytes = 0);
 // Elementwise SGD on the flat buffer (K3): p -= lr * (g + wd * p).
 void launch_sgd(float* p, const float* g, int64_t n, float lr, float wd, cudaStream_t s);
 // Level-synchronous path (vpps_level.cu): context (cuBLAS handle + work buffers) and one training pass.

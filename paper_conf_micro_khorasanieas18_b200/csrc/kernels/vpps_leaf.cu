@@ -52,6 +52,8 @@ struct PassClear {
     float* ptr[4];
     int64_t n[4];
     uint32_t* epoch;     // dataflow pass counter (tags of this pass), or nullptr
+    const char* pf;      // bytes to pull into L2 for the next kernel (the dataflow kernel's weights), or nullptr
+    int64_t pf_bytes;
 };
 
 template <int E, bool PROF>
@@ -86,6 +88,10 @@ __global__ void __launch_bounds__(NT + NTC, 1) vpps_leaf_fwd(const float* __rest
             const int64_t n4 = pc.ptr[r] ? pc.n[r] / 4 : 0;
             for (int64_t i = (int64_t)blockIdx.x * NTC + (tid - NT); i < n4; i += stride) p[i] = make_float4(0.f, 0.f, 0.f, 0.f);
         }
+        // pull the dataflow kernel's recurrent weights into L2 meanwhile: its prologue (registers of every
+        // CTA, after this grid's CTAs have left the SMs) then reads L2 instead of DRAM
+        for (int64_t i = (int64_t)blockIdx.x * NTC + (tid - NT); i < pc.pf_bytes / 128; i += stride)
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(pc.pf + i * 128));
         if (PROF && tid == NT && blockIdx.x < 1024 && g_leaf_prof_on) g_leaf_prof[blockIdx.x * 8 + 6] = gtimer();
         return;
     }
@@ -414,7 +420,7 @@ extern "C" int vpps_leaf_prof(int on, uint64_t* out) {   // measurement tool hoo
 
 void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float* pool, const uint32_t* leaves,
                      int32_t n_leaf, int32_t H, int32_t E, float* const* zero_ptr, const int64_t* zero_n,
-                     uint32_t* epoch, cudaStream_t s) {
+                     uint32_t* epoch, cudaStream_t s, const void* prefetch, int64_t prefetch_bytes) {
     using namespace dev::leaf;
     if (E != KMAX || H % LU) return;   // the cluster / dataflow variants are H = E = 256 (api.cu checks)
     static bool attr = false;
@@ -434,6 +440,8 @@ void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float*
     if (exp_ & 1) for (int r = 0; r < 4; ++r) if (r != 2) pc.n[r] = 0;     // no clearing (but the counters)
     if (exp_ & 2) n_leaf = 0;                                                // clearing only
     pc.epoch = epoch;
+    pc.pf = static_cast<const char*>(prefetch);
+    pc.pf_bytes = prefetch ? prefetch_bytes : 0;
     if (simt) {
         const int tiles = std::max(((n_leaf + LM - 1) / LM) * (H / LU), 148);
         if (h_leaf_prof_on) vpps_leaf_fwd<256, true><<<tiles, NT + NTC, SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
