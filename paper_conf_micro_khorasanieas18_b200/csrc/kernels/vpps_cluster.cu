@@ -671,16 +671,24 @@ __device__ __forceinline__ void leaf_dx_tile(const GemmParams& P, const uint32_t
     float2 acc2[4][2];
 #pragma unroll
     for (int a = 0; a < 4; ++a) acc2[a][0] = acc2[a][1] = make_float2(0.f, 0.f);
-#pragma unroll 4
-    for (int k = 0; k < nk; ++k) {
-        const float4 bv = *reinterpret_cast<const float4*>(Bs + k * DXN + tx * 4);
-        const float2 b01 = make_float2(bv.x, bv.y), b23 = make_float2(bv.z, bv.w);
+    // 4 k per step: one LDS.128 per leaf (its 4 gate gradients) and one per k of W_iou (4 columns)
+    // (nk is a multiple of 4: chunks of DXK = 128 of the 3H gate rows)
+#pragma unroll 2
+    for (int k = 0; k < nk; k += 4) {
+        float4 av[4];
 #pragma unroll
-        for (int a = 0; a < 4; ++a) {
-            const float av = As[(ty + 16 * a) * DXS + k];
-            const float2 aa = make_float2(av, av);
-            acc2[a][0] = __ffma2_rn(aa, b01, acc2[a][0]);
-            acc2[a][1] = __ffma2_rn(aa, b23, acc2[a][1]);
+        for (int a = 0; a < 4; ++a) av[a] = *reinterpret_cast<const float4*>(As + (ty + 16 * a) * DXS + k);
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            const float4 bv = *reinterpret_cast<const float4*>(Bs + (k + q) * DXN + tx * 4);
+            const float2 b01 = make_float2(bv.x, bv.y), b23 = make_float2(bv.z, bv.w);
+#pragma unroll
+            for (int a = 0; a < 4; ++a) {
+                const float g = q == 0 ? av[a].x : q == 1 ? av[a].y : q == 2 ? av[a].z : av[a].w;
+                const float2 aa = make_float2(g, g);
+                acc2[a][0] = __ffma2_rn(aa, b01, acc2[a][0]);
+                acc2[a][1] = __ffma2_rn(aa, b23, acc2[a][1]);
+            }
         }
     }
 #pragma unroll
