@@ -476,17 +476,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 }
             }
             __syncthreads();
-            for (int c = tid; c < C; c += NTH) {
-                float s = 0.f;
-                for (int n = 0; n < nb; ++n) s += zs[n * ZC + c];
-                dbo[c] += s;
-            }
-            for (int i = tid; i < C * H; i += NTH) {
-                const int c = i / H, k = i - c * H;
-                float s = 0.f;
-                for (int n = 0; n < nb; ++n) s = fmaf(zs[n * ZC + c], xs[n * KPH + k], s);
-                dWo[i] += s;
-            }
+            // the labelled cell's dh first: the group's CTAs wait on these HD slots; the head's own
+            // parameter gradients follow off the critical path
             for (int i = tid; i < nb * (H / 4); i += NTH) {   // dh of the labelled node -> HD slots
                 const int n = i / (H / 4), k = (i - n * (H / 4)) * 4;
                 float v4[4] = {0.f, 0.f, 0.f, 0.f};
@@ -498,6 +489,17 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 }
                 const uint32_t hd = ent[n * sz + 4];
                 if (hd != NONE) st_tag4(HD + (int64_t)hd * H + k, v4, ep);
+            }
+            for (int c = tid; c < C; c += NTH) {
+                float s = 0.f;
+                for (int n = 0; n < nb; ++n) s += zs[n * ZC + c];
+                dbo[c] += s;
+            }
+            for (int i = tid; i < C * H; i += NTH) {
+                const int c = i / H, k = i - c * H;
+                float s = 0.f;
+                for (int n = 0; n < nb; ++n) s = fmaf(zs[n * ZC + c], xs[n * KPH + k], s);
+                dWo[i] += s;
             }
         } else if (op == INT_F) {
             // ---- forward of internal cells: matvec from registers (L123), 4 nodes at a time; the unit's
