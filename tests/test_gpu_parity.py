@@ -430,3 +430,9 @@ def test_tdlstm_small_and_paper_size():
     rng = np.random.default_rng(81)
     check("tdlstm", 32, 32, 5, [synth.td_pyramid(rng, n, 16, 5) for n in (6, 1, 3, 9)], 16, seed=81)
     check("tdlstm", 256, 256, 5, synth.td_batch(np.random.default_rng(82), 4, lengths=(5, 20)), 4096, seed=82)
+
+
+def test_tdrnn_config_batch():
+    """TD-RNN at the sweep's full configuration (16 pyramids over sentences of 5-30 tokens, H = E = 512):
+    the whole batch against the oracle."""
+    check("tdrnn", 512, 512, 5, synth.config_batch("tdrnn", 3), 4096, seed=73)
