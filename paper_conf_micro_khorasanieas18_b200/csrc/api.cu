@@ -655,7 +655,10 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
                        m->pool + s->s.loss_word, m->d_loss_map + (m->passes & 1));
         CK(cudaGetLastError());
     } else {
-        CK(cudaLaunchCooperativeKernel(m->var->fn, dim3(m->plan.n_cta), dim3(256), args, m->smem, st));
+        const void* gfn = m->prof ? fb_prof_fn(m->var->fn) : m->var->fn;
+        if (!gfn) return fail(VPPS_E_STATE, "no trace-enabled grid kernel for this variant");
+        if (m->prof) CK(cudaFuncSetAttribute(gfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)m->smem));
+        CK(cudaLaunchCooperativeKernel(gfn, dim3(m->plan.n_cta), dim3(256), args, m->smem, st));
     }
     if (m->t_after) CK(cudaEventRecord(m->t_after, st));
     if (ring_slot >= 0) {

@@ -338,7 +338,9 @@ __device__ __forceinline__ const float* cin_src(uint32_t op, const uint32_t* I, 
     }
 }
 
-template <int CELL, int H, int E, int UMAX>
+// PROF = false: the production instantiation (the barrier / section trace folds away, prof is a constant
+// nullptr); PROF = true only with a profile buffer (vpps_set_profile_buffer)
+template <int CELL, int H, int E, int UMAX, bool PROF>
 __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
     using T = Cfg<CELL, H, E, UMAX>;
     using LA = typename T::LA;
@@ -442,7 +444,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_fb(const KParams P) {
         for (int i = tid; i < C; i += NTH) { bo[i] = __ldg(P.params + off[bout_m] + i); dbo[i] = 0.f; }
     }
 
-    uint64_t* prof = P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
+    uint64_t* prof = PROF && P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
     // section clocks (thread 0, trace only): 0 decode, 1 staging, 2 matvec, 3 cell, 4 cell-bwd,
     // 5 outer/transposed, 6 heads, 7 signal, 8 wait, 9 other
     uint64_t sec[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
@@ -1134,22 +1136,32 @@ __global__ void sgd_kernel(float* __restrict__ p, const float* __restrict__ g, i
 }  // namespace dev
 
 #define VPPS_VARIANT(CELL, H, E, U) \
-    {CELL, H, E, U, (const void*)&dev::vpps_fb<CELL, H, E, U>, &dev::Cfg<CELL, H, E, U>::smem_bytes}
+    {CELL, H, E, U, (const void*)&dev::vpps_fb<CELL, H, E, U, false>, &dev::Cfg<CELL, H, E, U>::smem_bytes}
+#define VPPS_PROF_PAIR(CELL, H, E, U) \
+    {(const void*)&dev::vpps_fb<CELL, H, E, U, false>, (const void*)&dev::vpps_fb<CELL, H, E, U, true>}
+#define VPPS_FB_LIST(X) \
+    X(dev::CELL_BINARY, 256, 256, 2),    /* target: binary Tree-LSTM H = E = 256 on 148 SMs, G = 1 */ \
+    X(dev::CELL_BINARY, 256, 256, 4),    /* ... G = 2 replica groups of 74 CTAs */ \
+    X(dev::CELL_BINARY, 256, 256, 8),    /* ... G = 4 replica groups of 37 CTAs */ \
+    X(dev::CELL_BINARY, 128, 128, 1), \
+    X(dev::CELL_BINARY, 32, 32, 1), \
+    X(dev::CELL_CHILDSUM, 128, 128, 1),  /* config 2 */ \
+    X(dev::CELL_CHILDSUM, 128, 128, 2),  /* ... G = 2 replica groups of 74 CTAs */ \
+    X(dev::CELL_CHILDSUM, 128, 128, 4),  /* ... G = 4 replica groups of 37 CTAs */ \
+    X(dev::CELL_CHILDSUM, 32, 32, 1), \
+    X(dev::CELL_LSTM, 32, 32, 1),        /* config 1 */ \
+    X(dev::CELL_LSTM, 256, 256, 2),      /* config 3, G = 1 */ \
+    X(dev::CELL_LSTM, 256, 256, 4)       /* ... G = 2 (an LM level's loss heads split over 2 holders) */
 
-static const Variant kVariants[] = {
-    VPPS_VARIANT(dev::CELL_BINARY, 256, 256, 2),    // target: binary Tree-LSTM H = E = 256 on 148 SMs, G = 1
-    VPPS_VARIANT(dev::CELL_BINARY, 256, 256, 4),    // ... G = 2 replica groups of 74 CTAs
-    VPPS_VARIANT(dev::CELL_BINARY, 256, 256, 8),    // ... G = 4 replica groups of 37 CTAs
-    VPPS_VARIANT(dev::CELL_BINARY, 128, 128, 1),
-    VPPS_VARIANT(dev::CELL_BINARY, 32, 32, 1),
-    VPPS_VARIANT(dev::CELL_CHILDSUM, 128, 128, 1),  // config 2
-    VPPS_VARIANT(dev::CELL_CHILDSUM, 128, 128, 2),  // ... G = 2 replica groups of 74 CTAs
-    VPPS_VARIANT(dev::CELL_CHILDSUM, 128, 128, 4),  // ... G = 4 replica groups of 37 CTAs
-    VPPS_VARIANT(dev::CELL_CHILDSUM, 32, 32, 1),
-    VPPS_VARIANT(dev::CELL_LSTM, 32, 32, 1),        // config 1
-    VPPS_VARIANT(dev::CELL_LSTM, 256, 256, 2),      // config 3, G = 1
-    VPPS_VARIANT(dev::CELL_LSTM, 256, 256, 4),      // ... G = 2 (an LM level's loss heads split over 2 holders)
-};
+static const Variant kVariants[] = {VPPS_FB_LIST(VPPS_VARIANT)};
+static const void* const kProfPairs[][2] = {VPPS_FB_LIST(VPPS_PROF_PAIR)};
+
+// the trace-enabled instantiation of a grid-kernel variant (same shared memory)
+const void* fb_prof_fn(const void* fn) {
+    for (const auto& pr : kProfPairs)
+        if (pr[0] == fn) return pr[1];
+    return nullptr;
+}
 
 const Variant* variants(int32_t* n) {
     *n = (int32_t)(sizeof(kVariants) / sizeof(kVariants[0]));
