@@ -25,6 +25,10 @@ L321) and the readings of SURVEY.md §8(c) c.2 / DESIGN.md "Readings" (R-1 … R
       function; inner nodes have two parents), the softmax head on the labelled top node
   M8  TD-LSTM (reading R-37): M4's binary Tree-LSTM cell on the TD-RNN pyramid DAG (leaves are
       M4 leaf cells on the tokens; shared children accumulate dh and dc from both parents)
+  M9  BiLSTMwChar (PAPER L267; reading R-38): M2 where the embedding of a rare word is [h→_c(last char);
+      h←_c(first char)] of a character BiLSTM (hidden E/2 per direction, char embeddings C_emb of
+      length Ec = 64, L281) over the word's spelling; a node is (children, tok, label, chars) and a
+      non-empty `chars` marks the word rare (its row of X is not read)
   head: z = W_out h + b_out, ℓ = −log softmax(z)[y]  ("negative softmax log likelihood", L42)
 
 Everything is float64, node by node, in the graph's own order for the forward pass and in
@@ -35,10 +39,10 @@ from __future__ import annotations
 
 import numpy as np
 
-CELLS = ("lstm", "binary", "childsum", "bilstm", "gru", "rvnn", "tdrnn", "tdlstm")
+CELLS = ("lstm", "binary", "childsum", "bilstm", "gru", "rvnn", "tdrnn", "tdlstm", "bilstmchar")
 
 
-def param_shapes(cell: str, H: int, E: int, C: int, M: int = 256):
+def param_shapes(cell: str, H: int, E: int, C: int, M: int = 256, Ec: int = 64, Vc: int = 64):
     """Ordered (name, shape) list of a model's parameters: matrices first, then biases.
 
     This is the parameter order of the C ABI (include/vpps.h, vpps_define_model)."""
@@ -63,6 +67,16 @@ def param_shapes(cell: str, H: int, E: int, C: int, M: int = 256):
         return [("Wf", (4 * H, E)), ("Uf", (4 * H, H)), ("Wb", (4 * H, E)), ("Ub", (4 * H, H)),
                 ("W_mlp", (M, 2 * H)), ("W_tag", (C, M)),
                 ("bf", (4 * H,)), ("bb", (4 * H,)), ("b_mlp", (M,)), ("b_tag", (C,))]
+    if cell == "bilstmchar":      # M2 + the character BiLSTM (hidden Hc = E/2 per direction, R-38)
+        if E % 2:
+            raise ValueError("BiLSTMwChar: E must be even ([h→_c; h←_c] is the rare word's embedding)")
+        Hc = E // 2
+        return [("Wf", (4 * H, E)), ("Uf", (4 * H, H)), ("Wb", (4 * H, E)), ("Ub", (4 * H, H)),
+                ("W_mlp", (M, 2 * H)), ("W_tag", (C, M)),
+                ("C_emb", (Vc, Ec)), ("Wcf", (4 * Hc, Ec)), ("Ucf", (4 * Hc, Hc)), ("Wcb", (4 * Hc, Ec)),
+                ("Ucb", (4 * Hc, Hc)),
+                ("bf", (4 * H,)), ("bb", (4 * H,)), ("b_mlp", (M,)), ("b_tag", (C,)),
+                ("bcf", (4 * Hc,)), ("bcb", (4 * Hc,))]
     raise ValueError(cell)
 
 
@@ -397,21 +411,30 @@ def _childsum_graph(P, G, X, dX, nodes, H):
 # M2: BiLSTM tagger ([25] via L265, L281): positions t = 0..n-1 of a chain
 # ----------------------------------------------------------------------------------------
 def _bilstm_graph(P, G, X, dX, nodes, H):
+    toks = [nd[1] for nd in nodes]
+    loss, dxs = _bilstm_core(P, G, [X[k] for k in toks], nodes, H)
+    for t, k in enumerate(toks):
+        dX[k] += dxs[t]
+    return loss
+
+
+def _bilstm_core(P, G, xs, nodes, H):
+    """M2 over the word vectors xs[t]: summed loss, parameter gradients into G, returns dL/dxs[t]."""
     n = len(nodes)
-    toks = [tok for (_, tok, _) in nodes]
     sf, sb = [None] * n, [None] * n
     h, c = np.zeros(H), np.zeros(H)
     for t in range(n):
-        sf[t] = lstm_step(P["Wf"], P["Uf"], P["bf"], X[toks[t]], h, c)
+        sf[t] = lstm_step(P["Wf"], P["Uf"], P["bf"], xs[t], h, c)
         h, c = sf[t]["h"], sf[t]["c"]
     h, c = np.zeros(H), np.zeros(H)
     for t in range(n - 1, -1, -1):
-        sb[t] = lstm_step(P["Wb"], P["Ub"], P["bb"], X[toks[t]], h, c)
+        sb[t] = lstm_step(P["Wb"], P["Ub"], P["bb"], xs[t], h, c)
         h, c = sb[t]["h"], sb[t]["c"]
     loss = 0.0
     dhf = [np.zeros(H) for _ in range(n)]
     dhb = [np.zeros(H) for _ in range(n)]
-    for t, (_, _, lab) in enumerate(nodes):
+    for t, nd in enumerate(nodes):
+        lab = nd[2]
         if lab < 0:
             continue
         hcat = np.concatenate([sf[t]["h"], sb[t]["h"]])
@@ -425,39 +448,97 @@ def _bilstm_graph(P, G, X, dX, nodes, H):
         dcat = P["W_mlp"].T @ da
         dhf[t] += dcat[:H]
         dhb[t] += dcat[H:]
+    dxs = [None] * n
     dh, dc = np.zeros(H), np.zeros(H)
     for t in range(n - 1, -1, -1):
         gam, dx, dh, dc = lstm_step_backward(P["Wf"], P["Uf"], sf[t], dhf[t] + dh, dc)
         G["Wf"] += np.outer(gam, sf[t]["x"]); G["Uf"] += np.outer(gam, sf[t]["h_prev"]); G["bf"] += gam
-        dX[toks[t]] += dx
+        dxs[t] = dx
     dh, dc = np.zeros(H), np.zeros(H)
     for t in range(n):
         gam, dx, dh, dc = lstm_step_backward(P["Wb"], P["Ub"], sb[t], dhb[t] + dh, dc)
         G["Wb"] += np.outer(gam, sb[t]["x"]); G["Ub"] += np.outer(gam, sb[t]["h_prev"]); G["bb"] += gam
-        dX[toks[t]] += dx
+        dxs[t] = dxs[t] + dx
+    return loss, dxs
+
+
+def _char_encode(P, chars):
+    """M9 character BiLSTM over one word's spelling: returns [h→(last); h←(first)] and the
+    recorded steps of both directions."""
+    Hc = P["Ucf"].shape[1]
+    n = len(chars)
+    sf, sb = [None] * n, [None] * n
+    h, c = np.zeros(Hc), np.zeros(Hc)
+    for t in range(n):
+        sf[t] = lstm_step(P["Wcf"], P["Ucf"], P["bcf"], P["C_emb"][chars[t]], h, c)
+        h, c = sf[t]["h"], sf[t]["c"]
+    h, c = np.zeros(Hc), np.zeros(Hc)
+    for t in range(n - 1, -1, -1):
+        sb[t] = lstm_step(P["Wcb"], P["Ucb"], P["bcb"], P["C_emb"][chars[t]], h, c)
+        h, c = sb[t]["h"], sb[t]["c"]
+    return np.concatenate([sf[n - 1]["h"], sb[0]["h"]]), (sf, sb)
+
+
+def _char_backward(P, G, chars, rec, drep):
+    """Reverse of _char_encode: dL/drep enters at the forward direction's last step and the backward
+    direction's last-processed (first-char) step only."""
+    Hc = P["Ucf"].shape[1]
+    sf, sb = rec
+    n = len(chars)
+    dh, dc = drep[:Hc].copy(), np.zeros(Hc)
+    for t in range(n - 1, -1, -1):
+        gam, dx, dh, dc = lstm_step_backward(P["Wcf"], P["Ucf"], sf[t], dh, dc)
+        G["Wcf"] += np.outer(gam, sf[t]["x"]); G["Ucf"] += np.outer(gam, sf[t]["h_prev"]); G["bcf"] += gam
+        G["C_emb"][chars[t]] += dx
+    dh, dc = drep[Hc:].copy(), np.zeros(Hc)
+    for t in range(n):
+        gam, dx, dh, dc = lstm_step_backward(P["Wcb"], P["Ucb"], sb[t], dh, dc)
+        G["Wcb"] += np.outer(gam, sb[t]["x"]); G["Ucb"] += np.outer(gam, sb[t]["h_prev"]); G["bcb"] += gam
+        G["C_emb"][chars[t]] += dx
+
+
+def _bilstmchar_graph(P, G, X, dX, nodes, H):
+    """M9: rare words (non-empty chars) take the character BiLSTM's output as their embedding."""
+    xs, recs = [], []
+    for nd in nodes:
+        chars = nd[3] if len(nd) > 3 else ()
+        if chars:
+            rep, rec = _char_encode(P, chars)
+            xs.append(rep); recs.append(rec)
+        else:
+            xs.append(X[nd[1]]); recs.append(None)
+    loss, dxs = _bilstm_core(P, G, xs, nodes, H)
+    for t, nd in enumerate(nodes):
+        if recs[t] is None:
+            dX[nd[1]] += dxs[t]
+        else:
+            _char_backward(P, G, nd[3], recs[t], dxs[t])
     return loss
 
 
 _GRAPH_FN = {"lstm": _lstm_graph, "binary": _binary_graph, "childsum": _childsum_graph,
              "bilstm": _bilstm_graph, "gru": _gru_graph, "rvnn": _rvnn_graph, "tdrnn": _tdrnn_graph,
-             "tdlstm": _binary_graph}   # M4's reverse pass accumulates dh / dc (+=): correct on DAGs
+             "tdlstm": _binary_graph, "bilstmchar": _bilstmchar_graph}   # M4's reverse pass accumulates dh / dc (+=): correct on DAGs
 
 
-def validate(cell: str, graphs, n_tokens: int, n_classes: int):
+def validate(cell: str, graphs, n_tokens: int, n_classes: int, n_chars: int = 0):
     """Structural rules of the op sets (readings R-4, R-26); raises ValueError."""
     for nodes in graphs:
-        for v, (ch, tok, lab) in enumerate(nodes):
+        for v, nd in enumerate(nodes):
+            ch, tok, lab = nd[:3]
+            if len(nd) > 3 and (cell != "bilstmchar" or any(not (0 <= k < n_chars) for k in nd[3])):
+                raise ValueError("a character spelling needs cell 'bilstmchar' and ids in [0, n_chars)")
             if any(not (0 <= k < v) for k in ch):
                 raise ValueError("children must precede their parent")
             if not (-1 <= tok < n_tokens) or not (-1 <= lab < n_classes):
                 raise ValueError("token/label out of range")
             if cell in ("binary", "rvnn", "tdrnn", "tdlstm") and not ((len(ch) == 0 and tok >= 0) or (len(ch) == 2 and tok < 0)):
                 raise ValueError("binary Tree-LSTM: leaves carry a token, internal nodes have 2 children")
-            if cell in ("lstm", "bilstm", "gru") and (len(ch) > 1 or tok < 0 or (ch and ch[0] != v - 1)):
+            if cell in ("lstm", "bilstm", "gru", "bilstmchar") and (len(ch) > 1 or tok < 0 or (ch and ch[0] != v - 1)):
                 raise ValueError("LSTM chain: node t has child t-1 and a token")
         parents = [0] * len(nodes)
-        for ch, _, _ in nodes:
-            for k in ch:
+        for nd in nodes:
+            for k in nd[0]:
                 parents[k] += 1
         if cell not in ("tdrnn", "tdlstm") and any(p > 1 for p in parents):   # TD graphs are DAGs (R-36/37)
             raise ValueError("a node may have at most one parent")
@@ -486,7 +567,8 @@ def flop_count(cell: str, graphs, H: int, E: int, C: int, want_dx: bool = True, 
     f = 0
     kx = 3 if want_dx else 2
     for nodes in graphs:
-        for ch, tok, lab in nodes:
+        for nd in nodes:
+            ch, tok, lab = nd[:3]
             if cell in ("binary", "tdlstm"):
                 f += (2 * 3 * H * E * kx) if not ch else 2 * 3 * (3 * H * 2 * H + 2 * H * H)
             elif cell == "childsum":

@@ -118,6 +118,31 @@ def input_table(rng: np.random.Generator, n_rows: int, dim: int, dtype=np.float6
     return rng.uniform(-0.1, 0.1, size=(n_rows, dim)).astype(dtype)
 
 
+def spelling(word: int, n_chars: int = 64, lengths=(2, 12)):
+    """Deterministic synthetic spelling of a word id (BiLSTMwChar): a length in `lengths` and
+    character ids in [0, n_chars), drawn from a generator seeded by the word id alone, so every occurrence
+    of a word is spelled the same way."""
+    r = np.random.default_rng(np.random.SeedSequence([0x5EED, int(word)]))
+    n = int(r.integers(lengths[0], lengths[1] + 1))
+    return tuple(int(c) for c in r.integers(0, n_chars, size=n))
+
+
+def char_tagger_batch(rng, batch: int, lengths=(5, 60), vocab=4096, n_tags=9, n_chars=64, rare_from=None):
+    """BiLSTMwChar sentences (reading R-38): tagger chains whose word ids follow a Zipf-like law (WikiNER-
+    style frequencies); ids >= rare_from (default: the top quarter of the vocabulary, the words seen fewer
+    than 5 times in a corpus of this law) are rare and carry their spelling as a fourth node field."""
+    rare_from = (3 * vocab) // 4 if rare_from is None else rare_from
+    out = []
+    for _ in range(batch):
+        n = int(rng.integers(lengths[0], lengths[1] + 1))
+        toks = np.minimum((rng.pareto(1.0, size=n) * vocab / 64).astype(np.int64), vocab - 1)
+        labs = rng.integers(0, n_tags, size=n)
+        out.append([((t - 1,) if t > 0 else (), int(toks[t]), int(labs[t]),
+                     spelling(int(toks[t]), n_chars) if toks[t] >= rare_from else ())
+                    for t in range(n)])
+    return out
+
+
 # BASELINE.json configs (SURVEY §8 "Configs"); 'tgt' is the north_star target.
 CONFIGS = {
     "c1": dict(cell="lstm", H=32, E=32, C=16, V=16, batch=4, lengths=(2, 5)),
@@ -128,8 +153,11 @@ CONFIGS = {
     "tgt": dict(cell="binary", H=256, E=256, C=5, V=4096, batch=16, leaves=(5, 50)),
     # paper's other workloads (Fig. 12: hidden = embedding = 512), SST-length sentences
     "tdrnn": dict(cell="tdrnn", H=512, E=512, C=5, V=4096, batch=16, lengths=(5, 30)),
+    # BiLSTMwChar (Fig. 12: hidden = embedding = 256, MLP 256, character embedding 64), WikiNER-length sentences
+    "bilstmchar": dict(cell="bilstmchar", H=256, E=256, C=9, V=4096, batch=16, lengths=(5, 60), mlp=256,
+                       Ec=64, Vc=64),
 }
-_CONFIG_IDS = {"c1": 1, "c2": 2, "c3": 3, "c4": 4, "c5": 5, "tgt": 6, "tdrnn": 7}
+_CONFIG_IDS = {"c1": 1, "c2": 2, "c3": 3, "c4": 4, "c5": 5, "tgt": 6, "tdrnn": 7, "bilstmchar": 8}
 
 
 def config_batch(name: str, batch_idx: int, batch: int | None = None, **over):
@@ -140,6 +168,8 @@ def config_batch(name: str, batch_idx: int, batch: int | None = None, **over):
     rng = rng_for(_CONFIG_IDS[name], batch_idx)
     if cfg["cell"] in ("binary", "childsum"):
         return tree_batch(rng, b, cfg["leaves"], cfg["V"], cfg["C"])
+    if cfg["cell"] == "bilstmchar":
+        return char_tagger_batch(rng, b, cfg["lengths"], cfg["V"], cfg["C"], cfg["Vc"])
     if cfg["cell"] == "tdrnn":
         return td_batch(rng, b, cfg["lengths"], cfg["V"], cfg["C"])
     if cfg["cell"] == "lstm":

@@ -24,14 +24,14 @@ from oracle import models as M
 GOLD = os.path.join(os.path.dirname(__file__), "golden")
 
 
-def _params(cell, H, E, C, seed=0, M_=4):
+def _params(cell, H, E, C, seed=0, M_=4, **kw):
     rng = np.random.default_rng(seed)
-    return synth.init_params(M.param_shapes(cell, H, E, C, M_), rng)
+    return synth.init_params(M.param_shapes(cell, H, E, C, M_, **kw), rng)
 
 
-def _fd_check(cell, graphs, H, E, C, V, M_=4, eps=1e-6, tol=1e-7):
+def _fd_check(cell, graphs, H, E, C, V, M_=4, eps=1e-6, tol=1e-7, **kw):
     rng = np.random.default_rng(1)
-    P = _params(cell, H, E, C, 2, M_)
+    P = _params(cell, H, E, C, 2, M_, **kw)
     # larger weights so that every gate is away from saturation-free linear regime
     P = {k: v * 3.0 for k, v in P.items()}
     X = rng.uniform(-1, 1, size=(V, E))
@@ -213,6 +213,105 @@ def test_tdlstm_dag_equals_its_tree_expansion():
     for k in G1:
         np.testing.assert_allclose(G1[k], G2[k], atol=1e-12)
     np.testing.assert_allclose(dX1, dX2, atol=1e-12)
+
+
+def test_fd_bilstmchar():
+    """M9: every parameter incl. the character BiLSTM and C_emb, and X (rare positions must not touch X:
+    word 1 is spelled at every occurrence in g1, so X[1] gets only g2's plain occurrence)."""
+    g1 = [((), 0, 1, ()), ((0,), 1, -1, (2, 0, 1)), ((1,), 2, 0, ()), ((2,), 1, 2, (2, 0, 1))]
+    g2 = [((), 1, 2, ()), ((0,), 2, 1, (1,))]
+    _fd_check("bilstmchar", [g1, g2], H=2, E=4, C=3, V=3, M_=3, Ec=2, Vc=3)
+
+
+def _torch_bilstm(Wf, Uf, bf, Wb, Ub, bb, H):
+    lstm = torch.nn.LSTM(Wf.shape[1], H, bidirectional=True, dtype=torch.float64)
+    with torch.no_grad():
+        lstm.weight_ih_l0.copy_(torch.tensor(_ifog_to_torch(Wf, H)))
+        lstm.weight_hh_l0.copy_(torch.tensor(_ifog_to_torch(Uf, H)))
+        lstm.bias_ih_l0.copy_(torch.tensor(_ifog_to_torch(bf, H))); lstm.bias_hh_l0.zero_()
+        lstm.weight_ih_l0_reverse.copy_(torch.tensor(_ifog_to_torch(Wb, H)))
+        lstm.weight_hh_l0_reverse.copy_(torch.tensor(_ifog_to_torch(Ub, H)))
+        lstm.bias_ih_l0_reverse.copy_(torch.tensor(_ifog_to_torch(bb, H))); lstm.bias_hh_l0_reverse.zero_()
+    return lstm
+
+
+def test_bilstmchar_equals_torch():
+    """M9 == torch: nn.LSTM(bidirectional) over each rare word's characters, its final states h_n
+    (forward after the last char, backward after the first) as the word vector, then M2 as nn.LSTM +
+    Linear/tanh/Linear + cross-entropy; gradients by autograd (pins R-38's wiring: which final state,
+    which half of the word vector, C_emb accumulation over repeated characters)."""
+    H, E, C, V, Mh, Ec, Vc = 3, 4, 5, 6, 7, 3, 4
+    P = _params("bilstmchar", H, E, C, 11, Mh, Ec=Ec, Vc=Vc)
+    rng = np.random.default_rng(12)
+    X = rng.uniform(-1, 1, (V, E))
+    nodes = [((), 0, 1, ()), ((0,), 4, 2, (1, 3, 1, 0)), ((1,), 2, -1, ()), ((2,), 5, 0, (2,)),
+             ((3,), 3, 4, ())]
+    loss, G, dX = M.forward_backward("bilstmchar", P, X, [nodes], H)
+    Hc = E // 2
+    clstm = _torch_bilstm(P["Wcf"], P["Ucf"], P["bcf"], P["Wcb"], P["Ucb"], P["bcb"], Hc)
+    wlstm = _torch_bilstm(P["Wf"], P["Uf"], P["bf"], P["Wb"], P["Ub"], P["bb"], H)
+    mlp = torch.nn.Linear(2 * H, Mh, dtype=torch.float64)
+    tag = torch.nn.Linear(Mh, C, dtype=torch.float64)
+    with torch.no_grad():
+        mlp.weight.copy_(torch.tensor(P["W_mlp"])); mlp.bias.copy_(torch.tensor(P["b_mlp"]))
+        tag.weight.copy_(torch.tensor(P["W_tag"])); tag.bias.copy_(torch.tensor(P["b_tag"]))
+    cemb = torch.tensor(P["C_emb"], requires_grad=True)
+    Xt = torch.tensor(X, requires_grad=True)
+    rows = []
+    for (_, tok, _, chars) in nodes:
+        if chars:
+            _, (hn, _) = clstm(cemb[list(chars)][:, None, :])
+            rows.append(torch.cat([hn[0, 0], hn[1, 0]]))
+        else:
+            rows.append(Xt[tok])
+    out, _ = wlstm(torch.stack(rows)[:, None, :])
+    z = tag(torch.tanh(mlp(out[:, 0, :])))
+    keep = [t for t, nd in enumerate(nodes) if nd[2] >= 0]
+    lt = torch.nn.functional.cross_entropy(z[keep], torch.tensor([nodes[t][2] for t in keep]), reduction="sum")
+    lt.backward()
+    assert abs(loss - lt.item()) < 1e-12
+    np.testing.assert_allclose(G["C_emb"], cemb.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(dX, Xt.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(_ifog_to_torch(G["Wcf"], Hc), clstm.weight_ih_l0.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(_ifog_to_torch(G["Ucb"], Hc), clstm.weight_hh_l0_reverse.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(_ifog_to_torch(G["bcb"], Hc), clstm.bias_ih_l0_reverse.grad.numpy(), atol=1e-12)
+    np.testing.assert_allclose(_ifog_to_torch(G["Wb"], H), wlstm.weight_ih_l0_reverse.grad.numpy(), atol=1e-12)
+
+
+def test_bilstmchar_without_rare_words_is_bilstm():
+    """Special case: with no spelled word M9 is M2 exactly, and the character parameters get zero gradient."""
+    H, E, C, V = 4, 6, 5, 9
+    P = _params("bilstmchar", H, E, C, 13, 5, Ec=3, Vc=5)
+    rng = np.random.default_rng(14)
+    X = rng.uniform(-1, 1, (V, E))
+    graphs = synth.tagger_batch(rng, 3, (2, 6), V, C)
+    l9, G9, dX9 = M.forward_backward("bilstmchar", P, X, [[nd + ((),) for nd in g] for g in graphs], H)
+    P2 = {k: P[k] for k, _ in M.param_shapes("bilstm", H, E, C, 5)}
+    l2, G2, dX2 = M.forward_backward("bilstm", P2, X, graphs, H)
+    assert l9 == l2
+    for k in P2:
+        np.testing.assert_array_equal(G9[k], G2[k])
+    np.testing.assert_array_equal(dX9, dX2)
+    for k in ("C_emb", "Wcf", "Ucf", "Wcb", "Ucb", "bcf", "bcb"):
+        assert not G9[k].any()
+
+
+def test_bilstmchar_synthetic_batch():
+    """Input recipe (R-38): spellings are a function of the word id; validation accepts the batch and
+    rejects spellings outside the character set or on another cell."""
+    g = synth.config_batch("bilstmchar", 0, batch=32)
+    spelled = {}
+    for nodes in g:
+        for nd in nodes:
+            if nd[3]:
+                assert spelled.setdefault(nd[1], nd[3]) == nd[3]
+                assert 2 <= len(nd[3]) <= 12
+    assert spelled
+    M.validate("bilstmchar", g, 4096, 9, n_chars=64)
+    with pytest.raises(ValueError):
+        M.validate("bilstmchar", g, 4096, 9, n_chars=8 if max(max(s) for s in spelled.values()) >= 8 else 0)
+    with pytest.raises(ValueError):
+        M.validate("bilstm", g, 4096, 9, n_chars=64)
 
 
 def test_fd_tdlstm():
