@@ -36,7 +36,8 @@ typedef enum {
     VPPS_E_NOFIT = -2,   /* weights do not fit the on-chip budget of any built kernel variant     */
     VPPS_E_CUDA = -3,    /* a CUDA runtime call failed (message in vpps_last_error)             */
     VPPS_E_GRAPH = -4,   /* bad graph: arity, order (children must precede parents), multiple
-                            parents, token/label out of range                                   */
+                            parents, token/label out of range, an empty batch (no nodes; the
+                            tagger-script cells BiLSTM / GRU run it as a T = 0 pass instead)     */
     VPPS_E_STATE = -5,   /* wrong call order: buffers not bound, plan-only model, script of
                             another model                                                       */
     VPPS_E_NOMEM = -6

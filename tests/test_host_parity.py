@@ -162,6 +162,18 @@ def test_graph_errors(vpps):
         vpps.Model("binary", 8, 8, 3, n_sm=16, plan_only=True).build_script([[((1,), 0, -1), ((), 0, -1)]])
 
 
+@pytest.mark.parametrize("cell", ["binary", "lstm", "childsum", "rvnn"])
+def test_empty_batch_is_a_graph_error(vpps, cell):
+    """Edge case: a batch without nodes (no graphs, or only empty graphs) is rejected with VPPS_E_GRAPH
+    (include/vpps.h) rather than launching a pass with nothing to compute.  (The tagger-script cells,
+    bilstm and gru, accept it as a pass with T = 0 tokens: zero loss, zero gradients.)"""
+    m = vpps.Model(cell, 8, 8, 3, n_sm=16, plan_only=True)
+    for graphs in ([], [[]], [[], []]):
+        with pytest.raises(vpps.VppsError) as e:
+            m.build_script(graphs)
+        assert e.value.status == -4
+
+
 def test_nofit_and_bad_shapes(vpps):
     with pytest.raises(vpps.VppsError) as e:
         vpps.Model("binary", 4096, 4096, 5, n_sm=148, plan_only=True)
