@@ -248,6 +248,13 @@ def test_tagger_small():
     check("bilstm", 32, 32, 9, graphs, 50, seed=71, mlp=16)
 
 
+def test_tagger_empty_sentences_in_batch():
+    """Edge case: empty sentences mixed into a batch (ragged down to length 0) change nothing."""
+    rng = np.random.default_rng(74)
+    graphs = synth.tagger_batch(rng, 2, (1, 6), 50, 9)
+    check("bilstm", 32, 32, 9, [[]] + graphs[:1] + [[]] + graphs[1:], 50, seed=75, mlp=16)
+
+
 def test_tagger_config4_shapes():
     """Config 4's sizes (H = E = 512, MLP 256, 9 tags) on a few short sentences."""
     graphs = synth.config_batch("c4", 0, batch=4, lengths=(3, 12))
