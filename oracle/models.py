@@ -567,6 +567,14 @@ def flop_count(cell: str, graphs, H: int, E: int, C: int, want_dx: bool = True, 
     f = 0
     kx = 3 if want_dx else 2
     for nodes in graphs:
+        if cell == "bilstm":
+            # M2 (L265, L281): per position and direction the input product (W x) and, after the first
+            # step of that direction, the recurrent product (U h); per labelled position the MLP over
+            # [h_fwd; h_bwd] (M x 2H) and the tag head (C x M); no MLP or head where there is no label
+            n = len(nodes)
+            f += 2 * (2 * 4 * H * E * kx * n + 2 * 3 * 4 * H * H * max(n - 1, 0))
+            f += sum(2 * 3 * (M * 2 * H + C * M) for nd in nodes if nd[2] >= 0)
+            continue
         for nd in nodes:
             ch, tok, lab = nd[:3]
             if cell in ("binary", "tdlstm"):

@@ -64,15 +64,20 @@ int build_tagger_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows
     s.loss_word = 0;
     s.zero_words = 32;
     s.pool_words = 32;
-    // algorithmic FLOPs: per position and direction 24H(E+H); per labelled position the
-    // MLP (2 x 2H x M x 3) and the tag head (2 x M x C x 3)
+    // algorithmic FLOPs (oracle.models.flop_count): per position and direction the input
+    // product W x (fwd, dW, dx: 3 x 2 FLOP per MAC), after a direction's first step the recurrent product
+    // U h; per labelled position the MLP (2H x M) and the tag head (M x C) of the tagger, the head (H x C)
+    // of the LM / GRU
+    int32_t S = 0;
+    for (int32_t g = 0; g < b.n_graphs; ++g) S += len[g] > 0;
     const double H = plan.H, E = plan.E, C = plan.C, M = plan.mlp;
+    const double Tt = T, Tr = (double)T - S;   // positions with a predecessor in a direction
     if (plan.cell == CELL_BILSTM)
-        s.flops = (double)T * 2.0 * 24.0 * H * (E + H) + (double)s.n_heads * (12.0 * H * M + 6.0 * M * C);
+        s.flops = 2.0 * (Tt * 24.0 * H * E + Tr * 24.0 * H * H) + (double)s.n_heads * (12.0 * H * M + 6.0 * M * C);
     else if (plan.cell == CELL_GRU)   // GRU chains: 3 gates, one direction, head on h
-        s.flops = (double)T * 18.0 * H * (E + H) + (double)s.n_heads * 6.0 * C * H;
+        s.flops = Tt * 18.0 * H * E + Tr * 18.0 * H * H + (double)s.n_heads * 6.0 * C * H;
     else   // LSTM LM: one direction, head on h
-        s.flops = (double)T * 24.0 * H * (E + H) + (double)s.n_heads * 6.0 * C * H;
+        s.flops = Tt * 24.0 * H * E + Tr * 24.0 * H * H + (double)s.n_heads * 6.0 * C * H;
     return 0;
 }
 

@@ -198,3 +198,15 @@ def test_widened_cells_host_side(vpps):
         rv.build_script([dag])                                  # shared children only in the TD cells
     with pytest.raises(vpps.VppsError):
         vpps.Model("tdrnn", 8, 12, 5, plan_only=True)           # leaves are the input rows: E == H
+
+
+@pytest.mark.parametrize("cell", ["bilstm", "gru", "lstm"])
+def test_chain_script_flops_equal_oracle_count(vpps, cell):
+    """The level path's chain scripts (tagger.cpp) report the oracle's algorithmic FLOP count (SURVEY
+    §8(d)), ragged lengths including one-token and empty sentences."""
+    H, E, C = 8, 12, 5
+    rng = np.random.default_rng(31)
+    graphs = synth.tagger_batch(rng, 5, (1, 9), 20, C) + [[]]
+    m = vpps.Model(cell, H, E, C, plan_only=True, mlp=6, level=1 if cell == "lstm" else 0)
+    info = m.build_script(graphs).info()
+    assert info["flops"] == M.flop_count(cell, graphs, H, E, C, M=6)

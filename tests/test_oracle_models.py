@@ -585,3 +585,71 @@ def test_validate_rules():
     with pytest.raises(ValueError):
         M.validate("binary", [[((), -1, 1)]], 5, 5)                     # leaf without a word
     M.validate("childsum", [[((), -1, -1), ((0,), 2, 1)]], 5, 5)
+
+
+def _torch_chain_flops(P, xs, H, fwd_only_dir=False):
+    """FLOPs that torch.utils.flop_counter counts for forward + backward of the M1/M2 definitions written
+    with plain linear maps (the first step of a direction has no recurrent product: h_0 = 0)."""
+    import torch
+    from torch.utils.flop_counter import FlopCounterMode
+    T = {k: torch.tensor(v, requires_grad=True) for k, v in P.items()}
+    x = torch.tensor(np.stack(xs), requires_grad=True)
+    lin = torch.nn.functional.linear
+
+    def run(W, U, b, order):
+        h = c = None
+        out = {}
+        for t in order:
+            a = lin(x[t], W, b) if h is None else lin(x[t], W, b) + lin(h, U)
+            i, f, o, g = torch.sigmoid(a[:H]), torch.sigmoid(a[H:2 * H]), torch.sigmoid(a[2 * H:3 * H]), torch.tanh(a[3 * H:])
+            c = i * g if c is None else f * c + i * g
+            h = o * torch.tanh(c)
+            out[t] = h
+        return out
+    return T, x, run, lin, FlopCounterMode
+
+
+def test_flop_count_bilstm_equals_torch_flop_counter():
+    """flop_count('bilstm') (M2, L265/L281) against torch's own FLOP counter over forward + backward of the
+    tagger written with plain linear maps: 2 FLOP per MAC for the forward product, dW and dx / dh."""
+    import torch
+    H, E, C, Mh = 3, 4, 5, 6
+    P = _params("bilstm", H, E, C, 21, Mh)
+    rng = np.random.default_rng(22)
+    for n, labels in ((5, [1, -1, 2, 0, -1]), (1, [3]), (4, [-1, -1, -1, 1])):
+        xs = [rng.standard_normal(E) for _ in range(n)]
+        T, x, run, lin, FC = _torch_chain_flops(P, xs, H)
+        with FC(display=False) as fc:
+            hf = run(T["Wf"], T["Uf"], T["bf"], range(n))
+            hb = run(T["Wb"], T["Ub"], T["bb"], range(n - 1, -1, -1))
+            loss = 0
+            for t, y in enumerate(labels):
+                if y < 0:
+                    continue
+                m = torch.tanh(lin(torch.cat([hf[t], hb[t]]), T["W_mlp"], T["b_mlp"]))
+                z = lin(m, T["W_tag"], T["b_tag"])
+                loss = loss + torch.nn.functional.cross_entropy(z[None], torch.tensor([y]))
+            # every position runs its backward step (as in the oracle and the device), also a trailing
+            # unlabelled one whose gradient is zero: tie all states into the loss with weight 0
+            loss = loss + 0 * sum(h.sum() for h in list(hf.values()) + list(hb.values()))
+            loss.backward()
+        nodes = [((t - 1,) if t else (), 0, y) for t, y in enumerate(labels)]
+        assert M.flop_count("bilstm", [nodes], H, E, C, M=Mh) == fc.get_total_flops()
+    assert M.flop_count("bilstm", [], H, E, C, M=Mh) == 0
+
+
+def test_flop_count_lstm_equals_torch_flop_counter():
+    import torch
+    H, E, C = 3, 4, 5
+    P = _params("lstm", H, E, C, 23)
+    rng = np.random.default_rng(24)
+    labels = [2, -1, 4, 0]
+    xs = [rng.standard_normal(E) for _ in labels]
+    T, x, run, lin, FC = _torch_chain_flops(P, xs, H)
+    with FC(display=False) as fc:
+        hs = run(T["W"], T["U"], T["b"], range(len(labels)))
+        loss = sum(torch.nn.functional.cross_entropy(lin(hs[t], T["W_out"], T["b_out"])[None], torch.tensor([y]))
+                   for t, y in enumerate(labels) if y >= 0)
+        loss.backward()
+    nodes = [((t - 1,) if t else (), 0, y) for t, y in enumerate(labels)]
+    assert M.flop_count("lstm", [nodes], H, E, C) == fc.get_total_flops()
