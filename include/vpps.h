@@ -92,6 +92,16 @@ typedef struct {
     int32_t rows, cols;
 } vpps_shape;
 
+/* Device-memory callbacks (PyTorch supplies device memory): the library takes its
+ * activation pool, per-slot script buffers and level-path work buffers through them.  `stream` is the
+ * cudaStream_t of the call that needs the memory: an allocation is used on it in stream order, and a
+ * buffer is handed to free once no later work on that stream reads it (stream-ordered, like
+ * cudaMallocAsync / cudaFreeAsync, so growing the pool never synchronises the device).  alloc returns
+ * NULL on failure (-> VPPS_E_NOMEM).  Both NULL = cudaMallocAsync / cudaFreeAsync on `stream`.  The
+ * Python binding passes torch's caching allocator. */
+typedef void* (*vpps_alloc_fn)(size_t bytes, void* stream, void* ctx);
+typedef void (*vpps_free_fn)(void* ptr, void* stream, void* ctx);
+
 typedef struct {
     int32_t n_sm;        /* SMs to spread the weights over; 0 = all SMs of `device`            */
     int32_t ctas_per_sm; /* 1 (0 = auto = 1)                                                   */
@@ -112,6 +122,9 @@ typedef struct {
                             FP32 SGEMM), fused cell / head / scatter kernels, dW as one GEMM per
                             matrix.  0 = auto: chosen when no register-resident specialisation
                             exists for (H, E) (config 5: H = E = 1024); -1 = never. */
+    vpps_alloc_fn alloc; /* device allocator for library-owned buffers (see above); NULL = default */
+    vpps_free_fn free;
+    void* alloc_ctx;     /* passed back to alloc / free                                         */
 } vpps_options;
 
 /* A batch of graphs in CSR form (the super-graph of L205 is built from it).
@@ -181,7 +194,14 @@ int32_t vpps_paper_choose_cps(const vpps_shape* mats, int32_t n_mats, int32_t n_
  * L141/L167, signal/wait L165, pool plan L159) and stages the words in pinned host memory.
  * The batch arrays are deep-copied; the caller may free them on return. */
 vpps_status vpps_build_script(vpps_model m, const vpps_batch* batch, vpps_script* out);
+/* The SPEC words (SPEC_SCRIPT.md §E).  A dataflow model's scripts leave them out of the device blob (its
+ * kernels never read them); they are built here on first request (same batch, same result). */
 vpps_status vpps_script_words(vpps_script s, const uint32_t** words /*host*/, int64_t* n_words);
+/* The whole device upload blob (host copy; SPEC_SCRIPT.md §D/§L): [words ‖] the device lowerings.
+ * *lists_off = blob offset of the device lowering (0 when the words are left out), *df_off = offset of
+ * the dataflow program or -1.  Pointer valid until the script is destroyed. */
+vpps_status vpps_script_blob(vpps_script s, const uint32_t** blob /*host*/, int64_t* n_words,
+                             int64_t* lists_off, int64_t* df_off);
 vpps_status vpps_script_info_get(vpps_script s, vpps_script_info* info);
 /* Asynchronous H2D copy of the script (one copy).  vpps_fwd_bwd* upload a script
  * automatically on first use; call this to move the copy out of the timed kernel region. */

@@ -178,4 +178,100 @@ def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 14
         words += s
     words += targets
     return dict(words=[w & 0xFFFFFFFF for w in words], pool_words=pool_words, zero_words=zero_words,
-                loss_word=z_loss, n_bar=n_bar, levels=level, nodes=nodes, rec=rec, adj=adj)
+                loss_word=z_loss, n_bar=n_bar, levels=level, nodes=nodes, rec=rec, adj=adj, L=L,
+                graph_group=graph_group, G=G, H=H)
+
+
+DF_OP = dict(LEAF_B=0x21, INT_F=0x22, INT_B=0x23, HEAD_FB=0x42)
+
+
+def device_lowering(ref):
+    """SPEC_SCRIPT.md §D, step by step: the binary cell's device lowering for whole-graph groups (S5g) —
+    the gradient GEMM's node lists (L185: one GEMM per matrix over the concatenated operands) and the
+    dataflow program of the replica-group kernel (the per-group instruction streams of L141-167 with
+    per-node slots in place of the signal/wait of L165).  `ref` is build(..., by_graph=True) of a binary
+    batch.  Returns dict(lists: the blob after the SPEC words, df_off: offset of the program inside it,
+    n_hx, n_part, n_hd, df_hx, df_part, df_hd, df_words)."""
+    nodes, level, rec, adj = ref["nodes"], ref["levels"], ref["rec"], ref["adj"]
+    G, L, H, gg = ref["G"], ref["L"], ref["H"], ref["graph_group"]
+    NONE_ = NONE
+    group = [gg[n["graph"]] for n in nodes]
+    # INT list (rec, rec_l, rec_r) and LEAF list (rec, token), grouped by group, ascending global id
+    out = []
+    for g in range(G):
+        for i, n in enumerate(nodes):
+            if n["kind"] == "INT" and group[i] == g:
+                out += [rec[i], rec[n["children"][0]], rec[n["children"][1]]]
+    for g in range(G):
+        for i, n in enumerate(nodes):
+            if n["kind"] == "LEAF" and group[i] == g:
+                out += [rec[i], n["token"]]
+    # slots in ascending global id: hx (internal cell with a parent or a head), pp (internal cell),
+    # hd (cell with a head); dsrc = pp(parent) << 1 | side
+    parent, side, head_of = {}, {}, {}
+    for i, n in enumerate(nodes):
+        if n["kind"] == "INT":
+            for sd, c in enumerate(n["children"]):
+                parent[c], side[c] = i, sd
+        elif n["kind"] == "HEAD":
+            head_of[n["children"][0]] = i
+    hx, pp, hd = {}, {}, {}
+    for i, n in enumerate(nodes):
+        if n["kind"] == "INT" and (i in parent or i in head_of):
+            hx[i] = len(hx)
+        if n["kind"] == "INT":
+            pp[i] = len(pp)
+        if i in head_of:
+            hd[i] = len(hd)
+
+    def dsrc(i):
+        return (pp[parent[i]] << 1 | side[i]) if i in parent else NONE_
+
+    def entry(op, i):
+        n = nodes[i]
+        if op == "INT_F":
+            l, r = n["children"]
+            return [rec[i], hx.get(i, NONE_), rec[l], hx.get(l, NONE_), rec[r], hx.get(r, NONE_)]
+        if op == "HEAD_FB":
+            c = n["children"][0]
+            return [rec[i], rec[c], n["label"], hx.get(c, NONE_), hd.get(c, NONE_)]
+        if op == "INT_B":
+            l, r = n["children"]
+            return [rec[i], adj[i], dsrc(i), hd.get(i, NONE_), pp[i], rec[l], adj[l], rec[r], adj[r]]
+        return [rec[i], adj[i], dsrc(i), hd.get(i, NONE_)]          # LEAF_B
+
+    def batches(op, ids):
+        cap = 64 if op == "LEAF_B" else 16
+        w = []
+        for b0 in range(0, len(ids), cap):
+            chunk = ids[b0:b0 + cap]
+            w.append(DF_OP[op] | (len(chunk) << 8))
+            for i in chunk:
+                w += entry(op, i)
+        return w
+
+    progs = []
+    for g in range(G):
+        w = []
+        mine = [i for i in range(len(nodes)) if group[i] == g]
+        for lv in range(1, L + 1):                 # forward levels: cells, then the heads of that level
+            w += batches("INT_F", [i for i in mine if level[i] == lv and nodes[i]["kind"] == "INT"])
+            w += batches("HEAD_FB", [i for i in mine if level[i] == lv and nodes[i]["kind"] == "HEAD"])
+        for lv in range(L, -1, -1):                # backward levels in reverse (L167)
+            w += batches("INT_B", [i for i in mine if level[i] == lv and nodes[i]["kind"] == "INT"])
+            w += batches("LEAF_B", [i for i in mine if level[i] == lv and nodes[i]["kind"] == "LEAF"])
+        progs.append(w)
+    df_off = len(out)
+    pre = [0]
+    for w in progs:
+        pre.append(pre[-1] + len(w))
+    out += [G] + pre
+    for w in progs:
+        out += w
+    # tagged regions behind the SPEC pool: 64-bit slots (2 words), each region aligned to 32 words
+    df_hx = _a32(ref["pool_words"])
+    df_part = _a32(df_hx + 2 * H * len(hx))
+    df_hd = _a32(df_part + 2 * 32 * H * len(pp))
+    end = _a32(df_hd + 2 * H * len(hd))
+    return dict(lists=[x & 0xFFFFFFFF for x in out], df_off=df_off, n_hx=len(hx), n_part=len(pp), n_hd=len(hd),
+                df_hx=df_hx, df_part=df_part, df_hd=df_hd, df_words=end - ref["pool_words"])

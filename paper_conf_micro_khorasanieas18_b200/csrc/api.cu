@@ -51,6 +51,7 @@ std::vector<Shape> expected_shapes(int32_t cell, int32_t H, int32_t E, int32_t C
 
 struct vpps_model_s {
     Plan plan;
+    DevAlloc alloc;                     // device memory of library-owned buffers (vpps_options callbacks)
     std::vector<Shape> shapes;
     std::vector<int64_t> offsets;
     int64_t n_floats = 0;
@@ -94,6 +95,9 @@ struct vpps_model_s {
 struct vpps_script_s {
     vpps_model model = nullptr;
     Script s;
+    // dataflow models build the SPEC words on request only (Plan::skip_words): the batch is kept for that
+    bool words_pending = false;
+    std::vector<int32_t> b_gp, b_cp, b_ch, b_tok, b_lab;
     uint32_t* d_words = nullptr;   // dedicated device copy after vpps_upload_script (resident script)
     bool uploaded = false;
 };
@@ -133,6 +137,10 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     std::unique_ptr<vpps_model_s> m(new (std::nothrow) vpps_model_s);
     if (!m) return fail(VPPS_E_NOMEM, "out of host memory");
     m->plan_only = o.plan_only != 0;
+    if ((o.alloc == nullptr) != (o.free == nullptr)) return fail(VPPS_E_INVALID, "alloc and free callbacks go together");
+    m->alloc.alloc_fn = o.alloc;
+    m->alloc.free_fn = o.free;
+    m->alloc.ctx = o.alloc_ctx;
     m->shapes = want;
     int64_t cur = 0;
     for (const Shape& s : want) {
@@ -165,7 +173,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
             cudaDeviceProp prop;
             CK(cudaGetDeviceProperties(&prop, o.device));
             if (prop.major != 10) return fail(VPPS_E_INVALID, "libvpps is built for sm_100a (B200) only");
-            m->level = level_ctx_create();
+            m->level = level_ctx_create(&m->alloc);
             if (!m->level) return fail(VPPS_E_CUDA, "cuBLAS initialisation failed");
             CK(cudaMallocHost(&m->h_loss, 2 * sizeof(float)));
             m->h_loss[0] = m->h_loss[1] = 0.f;
@@ -237,9 +245,12 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     if (!unit_plan(cell, H, E, C, n_sm, o.ctas_per_sm, o.groups, &m->plan, &err))
         return fail(err.rfind("NOFIT", 0) == 0 ? VPPS_E_NOFIT : VPPS_E_INVALID, err);
     m->plan.by_graph = m->cluster != 0;
+    m->plan.skip_words = m->dataflow;   // vpps_df reads only the device lowering (SPEC §D)
     if (m->cluster && m->plan.n_g != m->cluster) return fail(VPPS_E_INVALID, "groups x cluster must equal n_sm");
     if (m->cluster && !m->plan_only) {
         if (m->plan.G > vpps_model_s::kMaxGroups) return fail(VPPS_E_NOFIT, "more than 16 cluster replicas");
+        CK(setup_leaf_attrs());        // per device (this model's), after cudaSetDevice above
+        CK(setup_dw_gemm_attrs());
         CK(cudaMalloc(&m->done, 4 * vpps_model_s::kMaxGroups * sizeof(int32_t)));   // done, claim, fin/tail
         CK(cudaMemset(m->done, 0, 4 * vpps_model_s::kMaxGroups * sizeof(int32_t)));
         CK(cudaMalloc(&m->d_epoch, sizeof(uint32_t)));
@@ -261,7 +272,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
             // level-synchronous GEMM path (vpps_level.cu): no register-resident specialisation needed
             m->var = nullptr;
             m->plan.level = true;
-            m->level = level_ctx_create();
+            m->level = level_ctx_create(&m->alloc);
             if (!m->level) return fail(VPPS_E_CUDA, "cuBLAS initialisation failed");
             CK(cudaMallocHost(&m->h_loss, 2 * sizeof(float)));
             m->h_loss[0] = m->h_loss[1] = 0.f;
@@ -380,6 +391,16 @@ vpps_status vpps_build_script(vpps_model m, const vpps_batch* batch, vpps_script
     } else {
         rc = chains ? build_tagger_script(m->plan, b, INT64_MAX, &s->s, &err)
                     : build_script(m->plan, b, INT64_MAX, &s->s, &err);
+        if (rc == 0 && !chains && m->plan.skip_words && b.n_graphs > 0) {
+            // the SPEC words are built on request (vpps_script_words): keep a copy of the batch
+            const int32_t nn = b.graph_ptr[b.n_graphs];
+            s->b_gp.assign(b.graph_ptr, b.graph_ptr + b.n_graphs + 1);
+            s->b_cp.assign(b.child_ptr, b.child_ptr + nn + 1);
+            s->b_ch.assign(b.children, b.children + b.child_ptr[nn]);
+            s->b_tok.assign(b.token, b.token + nn);
+            s->b_lab.assign(b.label, b.label + nn);
+            s->words_pending = true;
+        }
     }
     if (rc != 0) return fail(rc == -4 ? VPPS_E_GRAPH : VPPS_E_INVALID, err);
     *out = s.release();
@@ -388,8 +409,28 @@ vpps_status vpps_build_script(vpps_model m, const vpps_batch* batch, vpps_script
 
 vpps_status vpps_script_words(vpps_script s, const uint32_t** words, int64_t* n) {
     if (!s || !words || !n) return fail(VPPS_E_INVALID, "null argument");
+    if (s->words_pending) {
+        Plan spec = s->model->plan;
+        spec.skip_words = false;
+        BatchIn b{(int32_t)s->b_gp.size() - 1, s->b_gp.data(), s->b_cp.data(), s->b_ch.data(), s->b_tok.data(),
+                  s->b_lab.data()};
+        Script t;
+        std::string err;
+        if (build_script(spec, b, INT64_MAX, &t, &err) != 0) return fail(VPPS_E_GRAPH, err);
+        s->s.words.swap(t.words);
+        s->words_pending = false;
+    }
     *words = s->s.words.data();
     *n = (int64_t)s->s.words.size();
+    return VPPS_OK;
+}
+
+vpps_status vpps_script_blob(vpps_script s, const uint32_t** blob, int64_t* n, int64_t* lists_off, int64_t* df_off) {
+    if (!s || !blob || !n) return fail(VPPS_E_INVALID, "null argument");
+    *blob = s->s.blob.data();
+    *n = (int64_t)s->s.blob.size();
+    if (lists_off) *lists_off = s->s.lists_off;
+    if (df_off) *df_off = s->s.df_off;
     return VPPS_OK;
 }
 
@@ -433,11 +474,17 @@ static vpps_status stage_script(vpps_model m, vpps_script s, cudaStream_t st, in
     if (!sl.done) CK(cudaEventCreateWithFlags(&sl.done, cudaEventDisableTiming));
     if (sl.used) CK(cudaEventSynchronize(sl.done));
     if (n > sl.cap) {
+        // (the slot's last reader has finished: event above; the pinned staging is library-owned, §8(b))
         if (sl.h) CK(cudaFreeHost(sl.h));
-        if (sl.d) CK(cudaFree(sl.d));
-        sl.cap = n + n / 2 + 1024;
-        CK(cudaMallocHost(&sl.h, sl.cap * sizeof(uint32_t)));
-        CK(cudaMalloc(&sl.d, sl.cap * sizeof(uint32_t)));
+        m->alloc.put(sl.d, st);
+        sl.h = nullptr;
+        sl.d = nullptr;
+        sl.cap = 0;
+        const size_t cap = n + n / 2 + 1024;
+        CK(cudaMallocHost(&sl.h, cap * sizeof(uint32_t)));
+        sl.d = static_cast<uint32_t*>(m->alloc.get(cap * sizeof(uint32_t), st));
+        if (!sl.d) return fail(VPPS_E_NOMEM, "script slot allocation failed");
+        sl.cap = cap;
     }
     std::memcpy(sl.h, s->s.blob.data(), n * sizeof(uint32_t));
     CK(cudaMemcpyAsync(sl.d, sl.h, n * sizeof(uint32_t), cudaMemcpyHostToDevice, st));
@@ -456,17 +503,30 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     if (s->s.max_token >= n_rows) return fail(VPPS_E_GRAPH, "token out of range of the input table");
     if (((uintptr_t)inputs | (uintptr_t)d_inputs) & 15) return fail(VPPS_E_INVALID, "input tables must be 16-byte aligned");
     cudaStream_t st = (cudaStream_t)stream_;
+    // every check before anything is queued (a failed call leaves no staged copy or pool change behind)
+    if (m->dataflow && s->s.df_off < 0) return fail(VPPS_E_INVALID, "script has no dataflow program (binary cell only)");
+    if (m->prof && !m->dataflow &&
+        m->prof_stride < 2 + 3 * (int64_t)(s->s.n_bar + 1) + 10 * (int64_t)(s->s.n_bar + 2))
+        return fail(VPPS_E_INVALID, "profile buffer stride too small for this script");
+    if (m->prof && m->dataflow && m->prof_stride < 11) return fail(VPPS_E_INVALID, "profile buffer stride < 11");
+    if (m->prof && m->dataflow && !df_prof_fn(m->var->fn))
+        return fail(VPPS_E_STATE, "no trace-enabled dataflow kernel for this variant");
+    if (m->prof && !m->dataflow && !m->cluster && !m->plan.level && !fb_prof_fn(m->var->fn))
+        return fail(VPPS_E_STATE, "no trace-enabled grid kernel for this variant");
     CK(cudaSetDevice(m->device));
     const int64_t need = s->s.pool_words + (m->dataflow ? s->s.df_words : 0);
     if (need > m->pool_cap) {
-        if (m->pool) { CK(cudaStreamSynchronize(st)); CK(cudaFree(m->pool)); m->pool = nullptr; }
+        // stream-ordered growth through the model's allocator: no device synchronisation inside the pass
+        m->alloc.put(m->pool, st);
+        m->pool = nullptr;
+        m->pool_cap = 0;
         const int64_t cap = need + need / 4 + 1024;
-        CK(cudaMalloc(&m->pool, cap * sizeof(float)));
+        m->pool = static_cast<float*>(m->alloc.get((size_t)cap * sizeof(float), st));
+        if (!m->pool) return fail(VPPS_E_NOMEM, "activation pool allocation failed");
         // tagged slots (dataflow) must never carry a live epoch before they are written: zero once
         CK(cudaMemsetAsync(m->pool, 0, cap * sizeof(float), st));
         m->pool_cap = cap;
     }
-    if (m->dataflow && s->s.df_off < 0) return fail(VPPS_E_INVALID, "script has no dataflow program (binary cell only)");
     m->last_pool_words = s->s.pool_words;
     int ring_slot = -1;
     const uint32_t* dwords = s->d_words;
@@ -499,9 +559,6 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     kp.loss_word = s->s.loss_word;
     kp.lr = lr;
     kp.wd = wd;
-    if (m->prof && !m->dataflow && m->prof_stride < 2 + 3 * (int64_t)(s->s.n_bar + 1) + 10 * (int64_t)(s->s.n_bar + 2))
-        return fail(VPPS_E_INVALID, "profile buffer stride too small for this script");
-    if (m->prof && m->dataflow && m->prof_stride < 11) return fail(VPPS_E_INVALID, "profile buffer stride < 11");
     kp.prof = m->prof;
     kp.prof_stride = m->prof_stride;
     void* args[] = {&kp};
@@ -542,7 +599,7 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         attr[1].val.programmaticStreamSerializationAllowed = 1;
         cfg.attrs = attr;
         cfg.numAttrs = no_pdl_df ? 1 : 2;
-        const uint32_t* lists = dwords + s->s.words.size();
+        const uint32_t* lists = dwords + s->s.lists_off;
         const uint32_t* leaf_list = lists + 3 * s->s.n_int;
         const float* W_iou = m->params + m->offsets[0];
         // U_iou, U_fl, U_fr, W_out and the biases (contiguous after W_iou in the flat layout) are pulled into
@@ -553,7 +610,6 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
                         pf_floats * (int64_t)sizeof(float));
         if (m->k_before) CK(cudaEventRecord(m->k_before, st));
         const void* dfn = m->prof ? df_prof_fn(m->var->fn) : m->var->fn;
-        if (!dfn) return fail(VPPS_E_STATE, "no trace-enabled dataflow kernel for this variant");
         if (m->prof) CK(cudaFuncSetAttribute(dfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)m->smem));
         CK(cudaLaunchKernelExC(&cfg, dfn, dargs));
         if (m->k_after) CK(cudaEventRecord(m->k_after, st));
@@ -630,7 +686,7 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         cfg.stream = st;
         cfg.attrs = attr;
         cfg.numAttrs = 1;       // ordinary stream order after the leaf kernel (which clears `done`)
-        const uint32_t* lists = dwords + s->s.words.size();
+        const uint32_t* lists = dwords + s->s.lists_off;
         const uint32_t* leaf_list = lists + 3 * s->s.n_int;
         const float* W_iou = m->params + m->offsets[0];
         // level 0 (all leaves share W_iou on their word vectors) as one dense GEMM + cell pass
@@ -656,7 +712,6 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         CK(cudaGetLastError());
     } else {
         const void* gfn = m->prof ? fb_prof_fn(m->var->fn) : m->var->fn;
-        if (!gfn) return fail(VPPS_E_STATE, "no trace-enabled grid kernel for this variant");
         if (m->prof) CK(cudaFuncSetAttribute(gfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)m->smem));
         CK(cudaLaunchCooperativeKernel(gfn, dim3(m->plan.n_cta), dim3(256), args, m->smem, st));
     }
@@ -753,8 +808,10 @@ void vpps_destroy_script(vpps_script s) {
 
 void vpps_destroy_model(vpps_model m) {
     if (!m) return;
+    for (cudaEvent_t e : m->ev)            // the last passes (the pool's last readers) have finished
+        if (e) cudaEventSynchronize(e);
     if (m->level) level_ctx_destroy(m->level);
-    if (m->pool) cudaFree(m->pool);
+    if (m->pool) m->alloc.put(m->pool, nullptr);
     if (m->done) cudaFree(m->done);
     if (m->d_epoch) cudaFree(m->d_epoch);
     if (m->h_loss) cudaFreeHost(m->h_loss);   // (cudaHostAlloc'd or cudaMallocHost'd: both freed here)
@@ -763,7 +820,7 @@ void vpps_destroy_model(vpps_model m) {
     for (auto& sl : m->ring) {
         if (sl.done) cudaEventSynchronize(sl.done), cudaEventDestroy(sl.done);
         if (sl.h) cudaFreeHost(sl.h);
-        if (sl.d) cudaFree(sl.d);
+        if (sl.d) m->alloc.put(sl.d, nullptr);
     }
     delete m;
 }

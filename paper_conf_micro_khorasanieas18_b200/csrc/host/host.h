@@ -36,6 +36,8 @@ struct Plan {
     int32_t n_cta, n_g, n_act, umax, G;
     bool by_graph = false;   // SPEC S5g: whole graphs assigned to groups (cluster replicas)
     bool level = false;      // level-synchronous GEMM path (binary cell, weights L2-resident)
+    bool skip_words = false; // dataflow models: the SPEC words (S4-S6, §E) are not built with the device
+                             // lowering (its kernels never read them); vpps_script_words builds them on demand
     std::vector<int32_t> table;   // rows of 8 int32
 };
 bool unit_plan(int32_t cell, int32_t H, int32_t E, int32_t C, int32_t n_sm, int32_t cps, int32_t G,
@@ -59,6 +61,7 @@ struct Script {
     // device upload blob = words ‖ (rec, rec_l, rec_r) per internal node ‖ (rec, token) per leaf; the node
     // lists drive the gradient GEMM of the cluster path.  Not part of the SPEC words.
     std::vector<uint32_t> blob;
+    int64_t lists_off = 0;   // blob offset of the INT list (= words.size(), 0 when the words are skipped)
     int64_t n_int = 0, n_leaf = 0;
     // per replica group g (S5g plans; one group otherwise): its internal / leaf nodes are list entries
     // [int_off[g], int_off[g+1]) / [leaf_off[g], leaf_off[g+1]); node count and deepest level

@@ -264,7 +264,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
             graph_group[gi] = best;
         }
     }
-    for (int32_t p = 0; p < P; ++p) {
+    for (int32_t p = 0; p < P && !plan.skip_words; ++p) {
         const bool fwd = p <= L;
         const int32_t lv = fwd ? p : 2 * L + 1 - p;
         for (int32_t g = 0; g < G; ++g) { body[g].clear(); load[g] = 0; }
@@ -297,13 +297,15 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     // ---- header: [G, n_bar, prefix sums], streams, barrier targets (L169) ---------------------
     Script& s = *out;
     s.words.clear();
-    s.words.push_back((uint32_t)G);
-    s.words.push_back((uint32_t)n_bar);
-    uint32_t run = 0;
-    s.words.push_back(0);
-    for (int32_t g = 0; g < G; ++g) { run += (uint32_t)streams[g].size(); s.words.push_back(run); }
-    for (int32_t g = 0; g < G; ++g) s.words.insert(s.words.end(), streams[g].begin(), streams[g].end());
-    s.words.insert(s.words.end(), targets.begin(), targets.end());
+    if (!plan.skip_words) {
+        s.words.push_back((uint32_t)G);
+        s.words.push_back((uint32_t)n_bar);
+        uint32_t run = 0;
+        s.words.push_back(0);
+        for (int32_t g = 0; g < G; ++g) { run += (uint32_t)streams[g].size(); s.words.push_back(run); }
+        for (int32_t g = 0; g < G; ++g) s.words.insert(s.words.end(), streams[g].begin(), streams[g].end());
+        s.words.insert(s.words.end(), targets.begin(), targets.end());
+    }
     s.pool_words = cursor;
     s.zero_words = zero_words;
     s.loss_word = loss_word;
@@ -330,6 +332,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
     // (grouped by replica group when graphs are assigned whole, S5g: the GEMM tiles of a group can then
     // start as soon as that group's cluster has finished)
     s.blob = s.words;
+    s.lists_off = (int64_t)s.blob.size();
     s.n_int = s.n_leaf = 0;
     const int32_t n_grp = plan.by_graph ? G : 1;
     auto group_of = [&](int64_t i) { return plan.by_graph ? graph_group[nodes[i].graph] : 0; };

@@ -1200,12 +1200,6 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, flo
         cfg.gridDim = dim3(done && !stat ? std::min(items, 148 * 3) : items);   // persistent when claiming
         cfg.blockDim = dim3(256);
         cfg.dynamicSmemBytes = DW_SMEM;
-        static bool attr_set = false;
-        if (!attr_set) {
-            cudaFuncSetAttribute(vpps_dw_gemm<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DW_SMEM);
-            cudaFuncSetAttribute(vpps_dw_gemm<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DW_SMEM);
-            attr_set = true;
-        }
         cfg.stream = s;
         cfg.attrs = attr;
         static const bool no_pdl = getenv("VPPS_DW_NOPDL") != nullptr;   // measurement only: no overlap
@@ -1216,6 +1210,15 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, flo
     if (fused_tail) return;                                            // SGD + loss inside the kernel
     if (mode == 1) launch_sgd(params, grads, n_floats, lr, wd, s);   // W -= lr (dW + wd W), every parameter
     if (loss_dst) cudaMemcpyAsync(loss_dst, loss_src, sizeof(float), cudaMemcpyDeviceToDevice, s);
+}
+
+// per-device launch attributes of the gradient GEMM (vpps_define_model calls this after cudaSetDevice)
+cudaError_t setup_dw_gemm_attrs() {
+    using namespace dev::cl;
+    cudaError_t e = cudaFuncSetAttribute(vpps_dw_gemm<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DW_SMEM);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(vpps_dw_gemm<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DW_SMEM);
+    return e;
 }
 
 }  // namespace vpps

@@ -39,6 +39,24 @@ struct DfParams {
     int32_t* done;              // per-group completion counters, or nullptr
 };
 
+// Device allocations of library-owned buffers (include/vpps.h vpps_alloc_fn / vpps_free_fn): the caller's
+// callbacks, or stream-ordered cudaMallocAsync / cudaFreeAsync when they are NULL.
+struct DevAlloc {
+    void* (*alloc_fn)(size_t bytes, void* stream, void* ctx) = nullptr;
+    void (*free_fn)(void* p, void* stream, void* ctx) = nullptr;
+    void* ctx = nullptr;
+    void* get(size_t bytes, cudaStream_t s) const {
+        if (alloc_fn) return alloc_fn(bytes, (void*)s, ctx);
+        void* p = nullptr;
+        return cudaMallocAsync(&p, bytes, s) == cudaSuccess ? p : nullptr;
+    }
+    void put(void* p, cudaStream_t s) const {
+        if (!p) return;
+        if (free_fn) free_fn(p, (void*)s, ctx);
+        else cudaFreeAsync(p, s);
+    }
+};
+
 struct Variant {
     int32_t cell, H, E, umax;
     const void* fn;
@@ -73,10 +91,13 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, flo
 void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float* pool, const uint32_t* leaves,
                      int32_t n_leaf, int32_t H, int32_t E, float* const* zero_ptr, const int64_t* zero_n,
                      uint32_t* epoch, cudaStream_t s, const void* prefetch = nullptr, int64_t prefetch_bytes = 0);
+// Per-device function attributes (dynamic shared memory) of the gradient GEMM and the leaf kernels.
+cudaError_t setup_dw_gemm_attrs();
+cudaError_t setup_leaf_attrs();
 // Elementwise SGD on the flat buffer (K3): p -= lr * (g + wd * p).
 void launch_sgd(float* p, const float* g, int64_t n, float lr, float wd, cudaStream_t s);
 // Level-synchronous path (vpps_level.cu): context (cuBLAS handle + work buffers) and one training pass.
-void* level_ctx_create();
+void* level_ctx_create(const DevAlloc* alloc);
 void level_ctx_destroy(void* ctx);
 int level_pass(void* ctx, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
                float* d_inputs, const uint32_t* d_blob, int64_t lv_int, int64_t lv_leaf, int64_t lv_head,

@@ -423,13 +423,6 @@ void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float*
                      uint32_t* epoch, cudaStream_t s, const void* prefetch, int64_t prefetch_bytes) {
     using namespace dev::leaf;
     if (E != KMAX || H % LU) return;   // the cluster / dataflow variants are H = E = 256 (api.cu checks)
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(vpps_leaf_fwd<256, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
-        cudaFuncSetAttribute(vpps_leaf_fwd<256, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
-        cudaFuncSetAttribute(vpps_leaf_fwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TC_SMEM);
-        attr = true;
-    }
     PassClear pc{};
     static const int exp_ = getenv("VPPS_LEAF_EXP") ? atoi(getenv("VPPS_LEAF_EXP")) : 0;   // measurement only
     // VPPS_LEAF_TC=1: the tensor-core variant (parity-green; measured slower than the FFMA tiles, 17.5 vs
@@ -452,6 +445,15 @@ void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float*
         const int grid = tiles + std::max(148 - tiles, 32);
         vpps_leaf_fwd_tc<<<grid, NT, TC_SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H, tiles, pc);
     }
+}
+
+// per-device launch attributes of the leaf kernels (vpps_define_model calls this after cudaSetDevice)
+cudaError_t setup_leaf_attrs() {
+    using namespace dev::leaf;
+    cudaError_t e = cudaFuncSetAttribute(vpps_leaf_fwd<256, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(vpps_leaf_fwd<256, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(vpps_leaf_fwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TC_SMEM);
+    return e;
 }
 
 }  // namespace vpps

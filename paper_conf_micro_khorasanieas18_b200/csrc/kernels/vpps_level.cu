@@ -483,15 +483,19 @@ struct LevelBufs {
     int64_t cap_leaf = 0, cap_int = 0;
 };
 
-static bool grow(float** p, int64_t* cap, int64_t need) {
+// work buffers grow geometrically through the model's device allocator (stream-ordered: no device sync)
+static bool grow_buf(const DevAlloc* a, cudaStream_t s, float** p, int64_t* cap, int64_t need) {
     if (need <= *cap) return true;
-    if (*p) cudaFree(*p);
+    a->put(*p, s);
     *p = nullptr;
+    *cap = 0;
     const int64_t c = need + need / 4 + 1024;
-    if (cudaMalloc(p, c * sizeof(float)) != cudaSuccess) return false;
+    *p = static_cast<float*>(a->get((size_t)c * sizeof(float), s));
+    if (!*p) return false;
     *cap = c;
     return true;
 }
+#define grow(...) grow_buf(&c->alloc, s, __VA_ARGS__)
 
 struct TaggerBufs {
     float *X = nullptr, *Pf = nullptr, *Pb = nullptr, *HH = nullptr, *Cf = nullptr, *Cb = nullptr, *Gf = nullptr,
@@ -506,6 +510,7 @@ struct TaggerBufs {
 };
 
 struct LevelCtx {
+    DevAlloc alloc;
     cublasHandle_t blas = nullptr;
     // BiLSTM tagger: the backward-direction chain runs on a second stream (its own cuBLAS handle), joined
     // by events — the two directions are independent until the head
@@ -517,8 +522,9 @@ struct LevelCtx {
     int64_t cap_X_leaf = 0, cap_X_int = 0, cap_Z = 0, cap_G_int = 0, cap_G_leaf = 0, cap_DX = 0;
 };
 
-void* level_ctx_create() {
+void* level_ctx_create(const DevAlloc* alloc) {
     LevelCtx* c = new LevelCtx;
+    c->alloc = *alloc;
     if (cublasCreate(&c->blas) != CUBLAS_STATUS_SUCCESS) { delete c; return nullptr; }
     if (cublasCreate(&c->blas2) != CUBLAS_STATUS_SUCCESS ||
         cudaStreamCreateWithFlags(&c->s2, cudaStreamNonBlocking) != cudaSuccess ||
@@ -543,12 +549,12 @@ void level_ctx_destroy(void* p) {
     if (c->ev_fork) cudaEventDestroy(c->ev_fork);
     if (c->ev_join) cudaEventDestroy(c->ev_join);
     float* bufs[] = {c->b.X_leaf, c->b.X_int, c->b.Z, c->b.G_int, c->b.G_leaf, c->b.DX};
-    for (float* q : bufs) if (q) cudaFree(q);
+    for (float* q : bufs) c->alloc.put(q, nullptr);
     TaggerBufs& t = c->tg;
     float* tbufs[] = {t.X, t.Pf, t.Pb, t.HH, t.Cf, t.Cb, t.Gf, t.Gb, t.Hp, t.Zs, t.Mm, t.Z, t.dZ, t.dM, t.dHH, t.dHf,
                       t.dHb, t.dCf, t.dCb, t.Gamf, t.Gamb, t.Gs, t.Dh, t.DX, t.Hp2, t.Zs2, t.Gs2, t.Dh2,
                       t.HS0, t.HS1, t.DhB0, t.DhB1, t.EzB};
-    for (float* q : tbufs) if (q) cudaFree(q);
+    for (float* q : tbufs) c->alloc.put(q, nullptr);
     delete c;
 }
 

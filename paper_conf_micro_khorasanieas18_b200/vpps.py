@@ -33,10 +33,34 @@ class _Opset(ct.Structure):
     _fields_ = [("cell", ct.c_int32), ("E", ct.c_int32), ("H", ct.c_int32), ("C", ct.c_int32), ("mlp", ct.c_int32)]
 
 
+_ALLOC_FN = ct.CFUNCTYPE(ct.c_void_p, ct.c_size_t, ct.c_void_p, ct.c_void_p)
+_FREE_FN = ct.CFUNCTYPE(None, ct.c_void_p, ct.c_void_p, ct.c_void_p)
+
+
 class _Options(ct.Structure):
     _fields_ = [("n_sm", ct.c_int32), ("ctas_per_sm", ct.c_int32), ("groups", ct.c_int32),
                 ("device", ct.c_int32), ("plan_only", ct.c_int32), ("cluster", ct.c_int32),
-                ("dataflow", ct.c_int32), ("level", ct.c_int32)]
+                ("dataflow", ct.c_int32), ("level", ct.c_int32),
+                ("alloc", _ALLOC_FN), ("free", _FREE_FN), ("alloc_ctx", ct.c_void_p)]
+
+
+def _torch_allocator(device: int):
+    """vpps_alloc_fn / vpps_free_fn over torch's caching allocator (include/vpps.h): PyTorch supplies the
+    library's device memory (north_star).  Returns the two ctypes callbacks (keep them alive)."""
+    import torch
+
+    def alloc(nbytes, stream, _ctx):
+        try:
+            return torch.cuda.caching_allocator_alloc(int(nbytes), device, stream or 0)
+        except Exception:            # out of memory -> NULL -> VPPS_E_NOMEM
+            return None
+
+    def free(ptr, _stream, _ctx):
+        try:
+            torch.cuda.caching_allocator_delete(ptr)
+        except Exception:            # interpreter shutdown: torch already torn down
+            pass
+    return _ALLOC_FN(alloc), _FREE_FN(free)
 
 
 class _Batch(ct.Structure):
@@ -67,6 +91,7 @@ def _load():
         "vpps_paper_choose_cps": [P(_Shape), I32, I32, I32, I32, I32],
         "vpps_build_script": [VP, P(_Batch), P(VP)],
         "vpps_script_words": [VP, P(P(ct.c_uint32)), P(I64)],
+        "vpps_script_blob": [VP, P(P(ct.c_uint32)), P(I64), P(I64), P(I64)],
         "vpps_script_info_get": [VP, P(_Info)],
         "vpps_upload_script": [VP, VP],
         "vpps_fwd_bwd": [VP, VP, VP, I64, VP, VP],
@@ -222,6 +247,15 @@ class Script:
         _check(_lib.vpps_script_words(self._h, ct.byref(p), ct.byref(n)))
         return np.ctypeslib.as_array(p, shape=(n.value,)).copy() if n.value else np.zeros(0, np.uint32)
 
+    def blob(self):
+        """(device upload blob as uint32 array, offset of the device lowering, offset of the dataflow
+        program or -1) — SPEC_SCRIPT.md §D."""
+        p = ct.POINTER(ct.c_uint32)()
+        n, lo, do = ct.c_int64(), ct.c_int64(), ct.c_int64()
+        _check(_lib.vpps_script_blob(self._h, ct.byref(p), ct.byref(n), ct.byref(lo), ct.byref(do)))
+        arr = np.ctypeslib.as_array(p, shape=(n.value,)).copy() if n.value else np.zeros(0, np.uint32)
+        return arr, lo.value, do.value
+
     def info(self) -> dict:
         i = _Info()
         _check(_lib.vpps_script_info_get(self._h, ct.byref(i)))
@@ -241,12 +275,17 @@ class Model:
 
     def __init__(self, cell: str, H: int, E: int, C: int, device: int = 0, n_sm: int = 0, groups: int = 1,
                  plan_only: bool = False, cluster: int = 0, dataflow: bool = False, level: int = 0,
-                 mlp: int = 256):
+                 mlp: int = 256, allocator: str = "torch"):
+        """allocator: "torch" (the library's device buffers come from torch's caching allocator) or
+        "cuda" (the library's default, stream-ordered cudaMallocAsync)."""
         self.cell, self.H, self.E, self.C = cell, H, E, C
         self.shapes = param_shapes(cell, H, E, C, mlp)
         sh = (_Shape * len(self.shapes))(*[_Shape(s[0], s[1] if len(s) == 2 else 1) for _, s in self.shapes])
         ops = _Opset(CELLS[cell], E, H, C, mlp)
-        opt = _Options(n_sm, 1, groups, device, int(plan_only), cluster, int(dataflow), int(level))
+        self._alloc_cbs = _torch_allocator(device) if (allocator == "torch" and not plan_only) else \
+            (_ALLOC_FN(), _FREE_FN())
+        opt = _Options(n_sm, 1, groups, device, int(plan_only), cluster, int(dataflow), int(level),
+                       self._alloc_cbs[0], self._alloc_cbs[1], None)
         h = ct.c_void_p()
         _check(_lib.vpps_define_model(sh, len(self.shapes), ct.byref(ops), ct.byref(opt), ct.byref(h)))
         self._h = h

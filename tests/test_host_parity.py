@@ -210,3 +210,29 @@ def test_chain_script_flops_equal_oracle_count(vpps, cell):
     m = vpps.Model(cell, H, E, C, plan_only=True, mlp=6, level=1 if cell == "lstm" else 0)
     info = m.build_script(graphs).info()
     assert info["flops"] == M.flop_count(cell, graphs, H, E, C, M=6)
+
+
+@pytest.mark.parametrize("G", [1, 3, 9])
+@pytest.mark.parametrize("dataflow", [True, False])
+def test_device_lowering_bit_exact(vpps, G, dataflow):
+    """SPEC_SCRIPT.md §D: the gradient GEMM's node lists and the dataflow program that vpps_df executes
+    (batches, entries, slot numbering) are bit-identical to oracle/script.py::device_lowering, on
+    SST-shaped batches of 1 / 4 / 16 / 64 trees, degenerate ones (a lone labelled leaf, labels on inner
+    nodes) and the bench's TGT batches.  A dataflow model leaves the SPEC words out of the blob and still
+    returns them, bit-exact, on request."""
+    H, E, C = 256, 256, 5
+    m = vpps.Model("binary", H, E, C, n_sm=16 * G, groups=G, cluster=16, dataflow=dataflow, plan_only=True)
+    rng = np.random.default_rng(200 + G)
+    inner = [((), 0, 1), ((), 1, -1), ((0, 1), -1, 3), ((), 2, -1), ((2, 3), -1, 0)]
+    batches = [synth.tree_batch(rng, b, (1, 50), 64, C) for b in (1, 4, 16, 64)]
+    batches += [[[((), 3, 2)]], [inner, inner], synth.config_batch("tgt", 0), synth.config_batch("tgt", 7)]
+    for graphs in batches:
+        s = m.build_script(graphs)
+        blob, lists_off, df_off = s.blob()
+        ref = oscript.build("binary", graphs, H, E, C, G=G, n_act=m.plan_info()["n_act"], by_graph=True)
+        low = oscript.device_lowering(ref)
+        assert lists_off == (0 if dataflow else len(ref["words"]))
+        assert np.array_equal(blob[lists_off:], np.array(low["lists"], dtype=np.uint32))
+        assert df_off - lists_off == low["df_off"]
+        assert np.array_equal(s.words(), np.array(ref["words"], dtype=np.uint32))    # (lazy when dataflow)
+        assert s.info()["n_words"] == len(ref["words"])

@@ -163,3 +163,62 @@ def test_pool_records_do_not_overlap():
     spans.sort()
     assert all(a[1] <= b[0] for a, b in zip(spans, spans[1:]))
     assert s["loss_word"] >= s["n_bar"] + 1
+
+
+def test_device_lowering_invariants():
+    """oracle device_lowering (SPEC §D) against what the schedule must guarantee (L139/L141/L167): every
+    internal cell is computed once forward (after its children) and once backward (after its parent), every
+    leaf once backward, every head once, each group only touches its own graphs, and the slot numbers are
+    distinct."""
+    import synth
+    rng = np.random.default_rng(3)
+    for G in (1, 4):
+        graphs = synth.tree_batch(rng, 12, (1, 30), 40, 5)
+        graphs.append([((), 0, 1), ((), 1, -1), ((0, 1), -1, 3), ((), 2, -1), ((2, 3), -1, 0)])
+        ref = script.build("binary", graphs, 16, 16, 5, G=G, n_act=16, by_graph=True)
+        low = script.device_lowering(ref)
+        w = low["lists"][low["df_off"]:]
+        assert w[0] == G
+        pre = w[1:G + 2]
+        rec_id = {r: i for i, r in enumerate(ref["rec"])}
+        seen_f, seen_b, heads, hx_seen, pp_seen = {}, {}, set(), set(), set()
+        t = 0
+        for g in range(G):
+            pos, end = G + 2 + pre[g], G + 2 + pre[g + 1]
+            while pos < end:
+                op, nb = w[pos] & 0xFF, w[pos] >> 8
+                sz = {0x22: 6, 0x42: 5, 0x23: 9, 0x21: 4}[op]
+                assert 1 <= nb <= (64 if op == 0x21 else 16)
+                for k in range(nb):
+                    e = w[pos + 1 + k * sz: pos + 1 + (k + 1) * sz]
+                    i = rec_id[e[0]]
+                    node = ref["nodes"][i]
+                    assert ref["graph_group"][node["graph"]] == g
+                    t += 1
+                    if op == 0x22:
+                        assert i not in seen_f
+                        for c in node["children"]:
+                            assert ref["nodes"][c]["kind"] == "LEAF" or c in seen_f
+                        seen_f[i] = t
+                        if e[1] != script.NONE:
+                            assert e[1] not in hx_seen
+                            hx_seen.add(e[1])
+                    elif op == 0x42:
+                        assert rec_id[e[1]] == node["children"][0] and (ref["nodes"][rec_id[e[1]]]["kind"] == "LEAF"
+                                                                         or rec_id[e[1]] in seen_f)
+                        heads.add(i)
+                    else:
+                        assert i not in seen_b
+                        if e[2] != script.NONE:       # dsrc: the parent's PART slot, already backward
+                            par = [p for p, n in enumerate(ref["nodes"]) if i in n["children"] and n["kind"] == "INT"]
+                            assert par and par[0] in seen_b
+                        seen_b[i] = t
+                        if op == 0x23:
+                            assert e[4] not in pp_seen
+                            pp_seen.add(e[4])
+                pos += 1 + nb * sz
+        n_int = sum(n["kind"] == "INT" for n in ref["nodes"])
+        n_leaf = sum(n["kind"] == "LEAF" for n in ref["nodes"])
+        n_head = sum(n["kind"] == "HEAD" for n in ref["nodes"])
+        assert len(seen_f) == n_int and len(seen_b) == n_int + n_leaf and len(heads) == n_head
+        assert len(pp_seen) == n_int == low["n_part"] and len(hx_seen) == low["n_hx"]
