@@ -494,3 +494,31 @@ def test_tdrnn_config_batch():
     """TD-RNN at the sweep's full configuration (16 pyramids over sentences of 5-30 tokens, H = E = 512):
     the whole batch against the oracle."""
     check("tdrnn", 512, 512, 5, synth.config_batch("tdrnn", 3), 4096, seed=73)
+
+
+def _golden(case):
+    import os
+    return np.load(os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", f"full_{case}.npz"))
+
+
+@pytest.mark.parametrize("case,cell,H,C,V,mlp,cfg,b,batch,seed", [
+    ("c5", "binary", 1024, 5, 4096, 256, "c5", 0, None, 63),
+    ("c4", "bilstm", 512, 9, 4096, 256, "c4", 1, None, 73),
+    ("c3", "lstm", 256, 1000, 1000, 256, "c3", 3, 64, 84)])
+def test_full_size_against_oracle_golden(case, cell, H, C, V, mlp, cfg, b, batch, seed):
+    """BASELINE.json configs 5, 4, 3 at their full sizes (64 trees at H = 1024; 16 sentences of 5-60 tokens
+    at H = 512; 64 sentences at H = 256, V = 1000) in the configuration define_model picks, against the
+    FP64 oracle: the loss, and 2048 sampled entries of every gradient and of dX (tests/golden/full_*.npz,
+    written by tools/make_golden.py from oracle/ and synth/ only) within 1e-4 of the tensor's max |value|
+    (R-22)."""
+    g = _golden(case)
+    graphs = synth.config_batch(cfg, b, batch=batch)
+    m, P, X, loss, params, grads, dX = run_case(cell, H, H, C, graphs, V, seed=seed, mlp=mlp)
+    assert abs(loss - float(g["loss"])) <= TOL * abs(float(g["loss"])), (loss, float(g["loss"]))
+    gv = m.views(grads.cpu())
+    for name, _ in m.shapes:
+        flat = gv[name].double().numpy().ravel()
+        idx, val, mx = g[f"{name}__idx"], g[f"{name}__val"], float(g[f"{name}__max"])
+        assert np.abs(flat[idx] - val).max() <= TOL * mx, name
+    dflat = dX.cpu().double().numpy().ravel()
+    assert np.abs(dflat[g["dX__idx"]] - g["dX__val"]).max() <= TOL * float(g["dX__max"]), "dX"

@@ -653,3 +653,23 @@ def test_flop_count_lstm_equals_torch_flop_counter():
         loss.backward()
     nodes = [((t - 1,) if t else (), 0, y) for t, y in enumerate(labels)]
     assert M.flop_count("lstm", [nodes], H, E, C) == fc.get_total_flops()
+
+
+def test_full_size_golden_regenerates():
+    """tests/golden/full_c3.npz is what tools/make_golden.py (oracle/ + synth/ only) writes: recompute the
+    config-3 case (64 sentences, H = 256, V = 1000) and compare every stored value bit for bit."""
+    import importlib.util
+    import os
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    spec = importlib.util.spec_from_file_location("make_golden", os.path.join(root, "tools", "make_golden.py"))
+    mg = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mg)
+    g = np.load(os.path.join(root, "tests", "golden", "full_c3.npz"))
+    graphs, P, X = mg.inputs("c3")
+    loss, G, dX = M.forward_backward("lstm", P, X, graphs, 256)
+    assert abs(loss - float(g["loss"])) <= 1e-9 * abs(loss)
+    for k in G:
+        flat = G[k].ravel()
+        np.testing.assert_allclose(flat[g[f"{k}__idx"]], g[f"{k}__val"], rtol=1e-9, atol=1e-12)
+        assert abs(np.abs(flat).max() - float(g[f"{k}__max"])) <= 1e-9 * float(g[f"{k}__max"])
+    np.testing.assert_allclose(dX.ravel()[g["dX__idx"]], g["dX__val"], rtol=1e-9, atol=1e-12)
