@@ -142,7 +142,7 @@ def run_reference(args, world: int, rank: int):
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": WORKLOAD, "global_batch": args.batch * world, "per_gpu_batch": args.batch,
                    "parallelism": f"dp{world}"},
-        "cpu_baseline": {"value": value, "unit": "samples/s", "cores": 1, "kind": "oracle",
+        "cpu_baseline": {"value": value, "unit": "samples/s", "cores": 1, "kind": "oracle", "cpu": lscpu_model(),
                          "sample": f"{per_step} tree of each step's batch (FP64 NumPy, BLAS threads = 1)"},
         "e2e": {"value": value, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
@@ -167,7 +167,7 @@ def cpu_baseline(batches, budget_s=12.0):
             if time.perf_counter() - t0 > budget_s:
                 break
     dt = time.perf_counter() - t0
-    return {"value": n / dt, "unit": "samples/s", "cores": 1, "kind": "oracle",
+    return {"value": n / dt, "unit": "samples/s", "cores": 1, "kind": "oracle", "cpu": lscpu_model(),
             "sample": f"{n} trees of the bench batches in {dt:.1f} s (FP64 NumPy, BLAS threads = 1)"}
 
 
@@ -202,9 +202,38 @@ def cpu_baseline_all_cores(batches, budget_s=8.0):
         t0 = time.perf_counter()
         n = sum(pool.map(_oracle_trees, work))
         dt = time.perf_counter() - t0
-    return {"value": n / dt, "unit": "samples/s", "cores": cores, "kind": "oracle",
+    return {"value": n / dt, "unit": "samples/s", "cores": cores, "kind": "oracle", "cpu": lscpu_model(),
             "sample": f"{n} trees of the bench batches in {dt:.1f} s on {cores} processes (FP64 NumPy, "
                       f"BLAS threads = 1 each)"}
+
+
+def _rank_entry(rank: int, world: int, port: int, argv):
+    os.environ.update(RANK=str(rank), LOCAL_RANK=str(rank), WORLD_SIZE=str(world), LOCAL_WORLD_SIZE=str(world),
+                      MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    sys.argv = argv
+    main()
+
+
+def spawn_ranks(n: int):
+    """`bench.py --gpus N` without torchrun: N processes, one per GPU, as torchrun would start them; each
+    times its own steps and rank 0 prints the line with the max over ranks."""
+    import socket
+    import torch.multiprocessing as mp
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    mp.spawn(_rank_entry, args=(n, port, list(sys.argv)), nprocs=n, join=True)
+
+
+def lscpu_model() -> str:
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
 
 
 def main():
@@ -225,7 +254,13 @@ def main():
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
 
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        # launched without torchrun: start the N ranks here (one process per GPU, 127.0.0.1 rendezvous)
+        spawn_ranks(args.gpus)
+        return
     world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world != args.gpus:
+        sys.exit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world} (launch N ranks with --gpus N)")
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if args.impl == "reference":
@@ -235,12 +270,21 @@ def main():
     import torch
     from paper_conf_micro_khorasanieas18_b200 import vpps
 
+    n_dev = torch.cuda.device_count()
+    local = local % n_dev                     # (more ranks than GPUs only in a functional check, see below)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     dist = None
+    backend = "nccl"
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        # NCCL needs one GPU per rank; ranks sharing a GPU (a functional check of the N-rank path on a
+        # smaller box, never a measurement) fall back to gloo and say so in the line
+        backend = "nccl" if world <= n_dev else "gloo"
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
 
     rng = np.random.default_rng(1234)          # identical initial parameters on every rank
     shapes = vpps.param_shapes("binary", H, E, C)
@@ -343,12 +387,20 @@ def main():
     e2e_steps = min(args.steps, 200)
     h2d = 0
     csr = [vpps.CsrBatch.from_graphs(g) for g in batches]   # the data loader's output: CSR batches (API input)
+    from concurrent.futures import ThreadPoolExecutor
+    builders = ThreadPoolExecutor(max_workers=3)            # the data loader's worker pool, started up front
+    for k, s in enumerate(vpps.prefetch_scripts(m, (csr[(k + 7) % N_BATCHES] for k in range(args.warmup)),
+                                                executor=builders)):
+        m.fwd_bwd_sgd(s, inputs, d_inputs, lr=lr, weight_decay=wd) if world == 1 else \
+            dp.dp_step(m, s, inputs, d_inputs, grads, lr, wd)     # untimed: warms builders and staging ring
+    m.latest_loss()
     if dist:
         dist.barrier()
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     # host: super-graph, levels, schedule, encode — built a few batches ahead by 3 background workers
-    for k, s in enumerate(vpps.prefetch_scripts(m, (csr[k % N_BATCHES] for k in range(e2e_steps)), workers=3)):
+    for k, s in enumerate(vpps.prefetch_scripts(m, (csr[k % N_BATCHES] for k in range(e2e_steps)),
+                                                executor=builders)):
         h2d += s.info()["blob_words"] * 4            # staged by the call below: one pinned H2D copy (L169)
         if world == 1:
             m.fwd_bwd_sgd(s, inputs, d_inputs, lr=lr, weight_decay=wd)
@@ -359,6 +411,7 @@ def main():
     m.latest_loss()                                  # the last step's loss
     torch.cuda.synchronize()
     e2e_s = time.perf_counter() - t0
+    builders.shutdown()
     te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
     if dist:
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
@@ -403,6 +456,7 @@ def main():
             "impl": "vpps",
             "config": {"workload": WORKLOAD, "global_batch": args.batch * world, "per_gpu_batch": args.batch,
                        "seq_len": None, "parallelism": f"dp{world}",
+                       "backend": backend if world > 1 else None,
                        "replica_groups": m.plan_info()["n_cta"] // m.plan_info()["n_g"],
                        "cluster": args.cluster or None, "ctas": m.plan_info()["n_cta"],
                        "sync": (args.sync if args.cluster else "grid barrier"),

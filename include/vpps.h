@@ -253,6 +253,14 @@ vpps_status vpps_set_gemm_trace(vpps_model m, uint64_t* buf);
 /* Device pointer of the model's activation pool (SPEC §S7 layout of the last script run). */
 vpps_status vpps_pool_ptr(vpps_model m, float** pool, int64_t* pool_words);
 
+/* The level paths' dense FP32 product (PAPER L185's concatenated operands; hand-written FFMA2 tiles,
+ * csrc/kernels/vpps_gemm.cu), exposed for testing:  C = op(A) op(B) + beta C, row-major dev pointers,
+ * op(A) = A (M x K, leading dimension lda) or, with ta, the transpose of A stored K x M; op(B) = B (K x N)
+ * or, with tb, the transpose of B stored N x K.  beta must be 0 or 1.  Asynchronous on `stream`; returns
+ * a vpps_status: VPPS_E_INVALID for bad arguments, VPPS_E_CUDA for a failed launch. */
+int32_t vpps_gemm_f32(void* stream, int32_t ta, int32_t tb, int32_t M, int32_t N, int32_t K, const float* A,
+                      int32_t lda, const float* B, int32_t ldb, float* C, int32_t ldc, float beta);
+
 void vpps_destroy_script(vpps_script s);
 void vpps_destroy_model(vpps_model m);
 const char* vpps_last_error(void);

@@ -19,7 +19,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
          "--expt-relaxed-constexpr", "-I", os.path.join(ROOT, "include")]
 FLAGS += os.environ.get("VPPS_NVCC_EXTRA", "").split()     # measurement-only experiments
-SOURCES = ["host/plan.cpp", "host/script.cpp", "host/tagger.cpp", "kernels/vpps_kernel.cu", "kernels/vpps_cluster.cu", "kernels/vpps_leaf.cu", "kernels/vpps_dataflow.cu", "kernels/vpps_level.cu", "api.cu"]
+SOURCES = ["host/plan.cpp", "host/script.cpp", "host/tagger.cpp", "kernels/vpps_kernel.cu", "kernels/vpps_cluster.cu", "kernels/vpps_leaf.cu", "kernels/vpps_dataflow.cu", "kernels/vpps_level.cu", "kernels/vpps_gemm.cu", "api.cu"]
 HEADERS = ["host/host.h", "kernels/vpps_kernel.cuh", "kernels/dev_common.cuh"]
 
 
@@ -50,7 +50,7 @@ def build(verbose: bool = False) -> str:
         objs = list(ex.map(lambda s: _compile(s, verbose), SOURCES))
     if os.path.exists(LIB) and os.path.getmtime(LIB) >= _newest(objs):
         return LIB
-    cmd = [NVCC, *ARCH, "-shared", "-o", LIB, *objs, "-lcudart", "-lcublas"]
+    cmd = [NVCC, *ARCH, "-shared", "-o", LIB, *objs, "-lcudart"]
     res = subprocess.run(cmd, capture_output=True, text=True)
     if res.returncode != 0:
         raise RuntimeError(f"link failed:\n{res.stderr}")

@@ -77,7 +77,7 @@ struct vpps_model_s {
     bool dataflow = false;              // groups of co-resident CTAs synchronised by tagged slots (vpps_df)
     uint32_t* d_epoch = nullptr;        // dataflow pass counter on the device (slot tags), advanced per pass
     static constexpr int kMaxGroups = 16;
-    void* level = nullptr;              // level-synchronous path context (cuBLAS handle, work buffers)
+    void* level = nullptr;              // level-synchronous path context (second stream, work buffers)
     // Pre-allocated staging ring for per-batch scripts: a pinned host buffer and a
     // device buffer per slot; a slot is reused once the kernel that last read it has finished.
     struct Slot {
@@ -174,7 +174,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
             CK(cudaGetDeviceProperties(&prop, o.device));
             if (prop.major != 10) return fail(VPPS_E_INVALID, "libvpps is built for sm_100a (B200) only");
             m->level = level_ctx_create(&m->alloc);
-            if (!m->level) return fail(VPPS_E_CUDA, "cuBLAS initialisation failed");
+            if (!m->level) return fail(VPPS_E_CUDA, "level-path context initialisation failed");
             CK(cudaMallocHost(&m->h_loss, 2 * sizeof(float)));
             m->h_loss[0] = m->h_loss[1] = 0.f;
             CK(cudaEventCreateWithFlags(&m->ev[0], cudaEventDisableTiming));
@@ -273,7 +273,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
             m->var = nullptr;
             m->plan.level = true;
             m->level = level_ctx_create(&m->alloc);
-            if (!m->level) return fail(VPPS_E_CUDA, "cuBLAS initialisation failed");
+            if (!m->level) return fail(VPPS_E_CUDA, "level-path context initialisation failed");
             CK(cudaMallocHost(&m->h_loss, 2 * sizeof(float)));
             m->h_loss[0] = m->h_loss[1] = 0.f;
             CK(cudaEventCreateWithFlags(&m->ev[0], cudaEventDisableTiming));

@@ -96,6 +96,9 @@ cudaError_t setup_dw_gemm_attrs();
 cudaError_t setup_leaf_attrs();
 // Elementwise SGD on the flat buffer (K3): p -= lr * (g + wd * p).
 void launch_sgd(float* p, const float* g, int64_t n, float lr, float wd, cudaStream_t s);
+// Dense FP32 product of the level paths (vpps_gemm.cu): row-major C = op(A) op(B) + beta C (beta 0 or 1).
+cudaError_t gemm_f32(cudaStream_t s, bool ta, bool tb, int M, int N, int K, const float* A, int lda, const float* B,
+                     int ldb, float* C, int ldc, float beta);
 // Level-synchronous path (vpps_level.cu): context (cuBLAS handle + work buffers) and one training pass.
 void* level_ctx_create(const DevAlloc* alloc);
 void level_ctx_destroy(void* ctx);

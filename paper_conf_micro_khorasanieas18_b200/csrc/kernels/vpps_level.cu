@@ -9,10 +9,9 @@
 // elementwise pass, and the backward level multiplies the gate gradients by the same weights.  The weights
 // (33.5 MB) stay resident in the 126 MB L2 across the levels of a pass, so DRAM still reads them about once
 // per pass; this is a deliberate deviation from register residency.  The dense products are
-// plain FP32 GEMMs (cuBLAS SGEMM, no TF32); gathers, cells, heads, scatters and bias gradients are the
+// plain FP32 GEMMs (vpps_gemm.cu FFMA2 tiles, no TF32); gathers, cells, heads, scatters and bias gradients are the
 // kernels below.  Pool records and adjoint blocks follow SPEC_SCRIPT §S7 (binary leaf [h c i o u | g_i g_o
 // g_u], internal [h c i o u f_l f_r | g_i g_o g_u g_fl g_fr], head [p(C) loss], adj [dh | dc]).
-#include <cublas_v2.h>
 #include <algorithm>
 #include <cstdio>
 #include "vpps_kernel.cuh"
@@ -468,14 +467,11 @@ __global__ void colsum(const float* __restrict__ A, int rows, int cols, float* o
 
 // ---- host orchestration ------------------------------------------------------------------------
 
-// Row-major C[M x N] = alpha op(A) op(B) + beta C (A: M x K, or K x M when ta; B: K x N, or N x K when tb)
-static cublasStatus_t gemm_rm(cublasHandle_t h, bool ta, bool tb, int M, int N, int K, const float* A, int lda,
-                              const float* B, int ldb, float* C, int ldc, float beta) {
-    const float alpha = 1.f;
-    if (M <= 0 || N <= 0) return CUBLAS_STATUS_SUCCESS;
-    if (K <= 0) return CUBLAS_STATUS_SUCCESS;      // only dW products with no nodes: grads stay zero
-    return cublasSgemm(h, tb ? CUBLAS_OP_T : CUBLAS_OP_N, ta ? CUBLAS_OP_T : CUBLAS_OP_N, N, M, K, &alpha, B, ldb,
-                       A, lda, &beta, C, ldc);
+// Row-major C[M x N] = op(A) op(B) + beta C (A: M x K, or K x M when ta; B: K x N, or N x K when tb): the
+// hand-written FFMA2 tiles of vpps_gemm.cu, on the stream of the chain / level being computed
+static cudaError_t gemm_rm(cudaStream_t h, bool ta, bool tb, int M, int N, int K, const float* A, int lda,
+                           const float* B, int ldb, float* C, int ldc, float beta) {
+    return gemm_f32(h, ta, tb, M, N, K, A, lda, B, ldb, C, ldc, beta);
 }
 
 struct LevelBufs {
@@ -511,10 +507,9 @@ struct TaggerBufs {
 
 struct LevelCtx {
     DevAlloc alloc;
-    cublasHandle_t blas = nullptr;
-    // BiLSTM tagger: the backward-direction chain runs on a second stream (its own cuBLAS handle), joined
-    // by events — the two directions are independent until the head
-    cublasHandle_t blas2 = nullptr;
+    cudaStream_t st = nullptr;         // stream of the pass in progress (the products run on it)
+    // BiLSTM tagger: the backward-direction chain runs on a second stream, joined by events — the two
+    // directions are independent until the head
     cudaStream_t s2 = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     LevelBufs b;
@@ -525,26 +520,18 @@ struct LevelCtx {
 void* level_ctx_create(const DevAlloc* alloc) {
     LevelCtx* c = new LevelCtx;
     c->alloc = *alloc;
-    if (cublasCreate(&c->blas) != CUBLAS_STATUS_SUCCESS) { delete c; return nullptr; }
-    if (cublasCreate(&c->blas2) != CUBLAS_STATUS_SUCCESS ||
-        cudaStreamCreateWithFlags(&c->s2, cudaStreamNonBlocking) != cudaSuccess ||
+    if (cudaStreamCreateWithFlags(&c->s2, cudaStreamNonBlocking) != cudaSuccess ||
         cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming) != cudaSuccess) {
-        cublasDestroy(c->blas);
         delete c;
         return nullptr;
     }
-    cublasSetMathMode(c->blas2, CUBLAS_PEDANTIC_MATH);
-    cublasSetStream(c->blas2, c->s2);
-    cublasSetMathMode(c->blas, CUBLAS_PEDANTIC_MATH);     // plain FP32 (no TF32, no emulation)
     return c;
 }
 
 void level_ctx_destroy(void* p) {
     LevelCtx* c = static_cast<LevelCtx*>(p);
     if (!c) return;
-    if (c->blas) cublasDestroy(c->blas);
-    if (c->blas2) cublasDestroy(c->blas2);
     if (c->s2) cudaStreamDestroy(c->s2);
     if (c->ev_fork) cudaEventDestroy(c->ev_fork);
     if (c->ev_join) cudaEventDestroy(c->ev_join);
@@ -561,7 +548,7 @@ void level_ctx_destroy(void* p) {
 static inline unsigned nblk(int64_t n, int t = 256) { return (unsigned)((n + t - 1) / t); }
 
 // One forward + backward pass (+ dW, bias and head gradients into grads, which the caller zeroed; dX into
-// d_inputs, zeroed by the caller).  Returns a CUDA / cuBLAS error code (0 = ok).
+// d_inputs, zeroed by the caller).  Returns a CUDA error code (0 = ok).
 int level_pass(void* ctx_, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
                float* d_inputs, const uint32_t* d_blob, int64_t lv_int, int64_t lv_leaf, int64_t lv_head,
                const int32_t* lv_start, int32_t L, int64_t n_int, int64_t n_leaf, int64_t n_head, int32_t H,
@@ -569,7 +556,7 @@ int level_pass(void* ctx_, const float* params, const int64_t* off, float* grads
     // shared: TD-LSTM DAGs (R-37) — children's dh and dc accumulate atomically (two parents per level)
     using namespace dev::lv;
     LevelCtx* c = static_cast<LevelCtx*>(ctx_);
-    cublasSetStream(c->blas, s);
+    c->st = s;
     const int64_t zrows = std::max<int64_t>(n_leaf * 3 * H, n_int * 5 * H);
     if (!grow(&c->b.X_leaf, &c->cap_X_leaf, std::max<int64_t>(n_leaf * E, 4)) ||
         !grow(&c->b.X_int, &c->cap_X_int, std::max<int64_t>(n_int * 2 * H, 4)) ||
@@ -590,12 +577,12 @@ int level_pass(void* ctx_, const float* params, const int64_t* off, float* grads
     const uint32_t* leaves = d_blob + lv_leaf;
     const uint32_t* hl = d_blob + lv_head;
     float *Xl = c->b.X_leaf, *Xi = c->b.X_int, *Z = c->b.Z, *Gi = c->b.G_int, *Gl = c->b.G_leaf, *DX = c->b.DX;
-    cublasStatus_t st = CUBLAS_STATUS_SUCCESS;
-#define BL(call) do { st = (call); if (st != CUBLAS_STATUS_SUCCESS) return 1000 + (int)st; } while (0)
+    cudaError_t st = cudaSuccess;
+#define BL(call) do { st = (call); if (st != cudaSuccess) return 1000 + (int)st; } while (0)
     // ---- forward: leaves (level 0) as one GEMM, then every internal level ----
     if (n_leaf > 0) {
         gather_leaf<<<nblk(n_leaf * (E / 4)), 256, 0, s>>>(inputs, leaves, (int)n_leaf, E, Xl);
-        BL(gemm_rm(c->blas, false, true, (int)n_leaf, 3 * H, E, Xl, E, W_iou, E, Z, 3 * H, 0.f));
+        BL(gemm_rm(c->st, false, true, (int)n_leaf, 3 * H, E, Xl, E, W_iou, E, Z, 3 * H, 0.f));
         leaf_cell<<<nblk(n_leaf * H), 256, 0, s>>>(Z, b_iou, leaves, (int)n_leaf, H, pool);
     }
     for (int32_t l = 1; l <= L; ++l) {
@@ -603,9 +590,9 @@ int level_pass(void* ctx_, const float* params, const int64_t* off, float* grads
         if (n <= 0) continue;
         float* X = Xi + r0 * 2 * H;
         gather_int<<<nblk(n * (2 * H / 4)), 256, 0, s>>>(pool, ints + 6 * r0, (int)n, H, X);
-        BL(gemm_rm(c->blas, false, true, (int)n, 3 * H, 2 * H, X, 2 * H, U_iou, 2 * H, Z, 5 * H, 0.f));
-        BL(gemm_rm(c->blas, false, true, (int)n, H, H, X, 2 * H, U_fl, H, Z + 3 * H, 5 * H, 0.f));
-        BL(gemm_rm(c->blas, false, true, (int)n, H, H, X + H, 2 * H, U_fr, H, Z + 4 * H, 5 * H, 0.f));
+        BL(gemm_rm(c->st, false, true, (int)n, 3 * H, 2 * H, X, 2 * H, U_iou, 2 * H, Z, 5 * H, 0.f));
+        BL(gemm_rm(c->st, false, true, (int)n, H, H, X, 2 * H, U_fl, H, Z + 3 * H, 5 * H, 0.f));
+        BL(gemm_rm(c->st, false, true, (int)n, H, H, X + H, 2 * H, U_fr, H, Z + 4 * H, 5 * H, 0.f));
         int_cell<<<nblk(n * H), 256, 0, s>>>(Z, b_iou, b_f, ints + 6 * r0, (int)n, H, pool);
     }
     // ---- loss heads: forward and backward (they feed nothing forward) ----
@@ -619,24 +606,24 @@ int level_pass(void* ctx_, const float* params, const int64_t* off, float* grads
         float* G = Gi + r0 * 5 * H;
         int_bwd<<<nblk(n * H), 256, 0, s>>>(ints + 6 * r0, (int)n, H, pool, G, shared);
         // [dh_l; dh_r] = U_iouᵀ g_iou, dh_l += U_flᵀ g_fl, dh_r += U_frᵀ g_fr
-        BL(gemm_rm(c->blas, false, false, (int)n, 2 * H, 3 * H, G, 5 * H, U_iou, 2 * H, DX, 2 * H, 0.f));
-        BL(gemm_rm(c->blas, false, false, (int)n, H, H, G + 3 * H, 5 * H, U_fl, H, DX, 2 * H, 1.f));
-        BL(gemm_rm(c->blas, false, false, (int)n, H, H, G + 4 * H, 5 * H, U_fr, H, DX + H, 2 * H, 1.f));
+        BL(gemm_rm(c->st, false, false, (int)n, 2 * H, 3 * H, G, 5 * H, U_iou, 2 * H, DX, 2 * H, 0.f));
+        BL(gemm_rm(c->st, false, false, (int)n, H, H, G + 3 * H, 5 * H, U_fl, H, DX, 2 * H, 1.f));
+        BL(gemm_rm(c->st, false, false, (int)n, H, H, G + 4 * H, 5 * H, U_fr, H, DX + H, 2 * H, 1.f));
         if (shared) scatter_dh_shared<<<nblk(n * 2 * H), 256, 0, s>>>(DX, ints + 6 * r0, (int)n, H, pool);
         else scatter_dh<<<nblk(n * 2 * H), 256, 0, s>>>(DX, ints + 6 * r0, (int)n, H, pool);
     }
     if (n_leaf > 0) {
         leaf_bwd<<<nblk(n_leaf * H), 256, 0, s>>>(leaves, (int)n_leaf, H, pool, Gl);
         if (d_inputs) {
-            BL(gemm_rm(c->blas, false, false, (int)n_leaf, E, 3 * H, Gl, 3 * H, W_iou, E, DX, E, 0.f));
+            BL(gemm_rm(c->st, false, false, (int)n_leaf, E, 3 * H, Gl, 3 * H, W_iou, E, DX, E, 0.f));
             scatter_dx<<<nblk(n_leaf * E), 256, 0, s>>>(DX, leaves, (int)n_leaf, E, d_inputs);
         }
     }
     // ---- weight gradients (L185): one GEMM per matrix over the concatenated nodes ----
-    BL(gemm_rm(c->blas, true, false, 3 * H, 2 * H, (int)n_int, Gi, 5 * H, Xi, 2 * H, grads + off[1], 2 * H, 0.f));
-    BL(gemm_rm(c->blas, true, false, H, H, (int)n_int, Gi + 3 * H, 5 * H, Xi, 2 * H, grads + off[2], H, 0.f));
-    BL(gemm_rm(c->blas, true, false, H, H, (int)n_int, Gi + 4 * H, 5 * H, Xi + H, 2 * H, grads + off[3], H, 0.f));
-    BL(gemm_rm(c->blas, true, false, 3 * H, E, (int)n_leaf, Gl, 3 * H, Xl, E, grads + off[0], E, 0.f));
+    BL(gemm_rm(c->st, true, false, 3 * H, 2 * H, (int)n_int, Gi, 5 * H, Xi, 2 * H, grads + off[1], 2 * H, 0.f));
+    BL(gemm_rm(c->st, true, false, H, H, (int)n_int, Gi + 3 * H, 5 * H, Xi, 2 * H, grads + off[2], H, 0.f));
+    BL(gemm_rm(c->st, true, false, H, H, (int)n_int, Gi + 4 * H, 5 * H, Xi + H, 2 * H, grads + off[3], H, 0.f));
+    BL(gemm_rm(c->st, true, false, 3 * H, E, (int)n_leaf, Gl, 3 * H, Xl, E, grads + off[0], E, 0.f));
     bias_grads<<<nblk(4 * H), 256, 0, s>>>(Gi, (int)n_int, Gl, (int)n_leaf, H, grads + off[5], grads + off[6]);
 #undef BL
     return (int)cudaGetLastError();
@@ -654,7 +641,7 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
     const bool has_mlp = Mw > 0;
     LevelCtx* c = static_cast<LevelCtx*>(ctx_);
     TaggerBufs& tb = c->tg;
-    cublasSetStream(c->blas, s);
+    c->st = s;
     const int64_t Tn = std::max<int64_t>(T, 1);
     float** bufs[24] = {&tb.X, &tb.Pf, &tb.Pb, &tb.HH, &tb.Cf, &tb.Cb, &tb.Gf, &tb.Gb, &tb.Hp, &tb.Zs, &tb.Mm, &tb.Z,
                         &tb.dZ, &tb.dM, &tb.dHH, &tb.dHf, &tb.dHb, &tb.dCf, &tb.dCb, &tb.Gamf, &tb.Gamb, &tb.Gs, &tb.Dh,
@@ -681,12 +668,12 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
     const float *Wf = P_(0), *Uf = P_(1), *Wb = P_(2), *Ub = P_(3), *Wm = P_(4), *Wt = P_(5), *bf = P_(6),
                 *bb = P_(7), *bm = P_(8), *bt = P_(9);
     const uint32_t *tok = d_blob + tg_tok, *lab = d_blob + tg_lab, *fpos = d_blob + tg_fpos, *bpos = d_blob + tg_bpos;
-    cublasStatus_t st;
-#define BL(call) do { st = (call); if (st != CUBLAS_STATUS_SUCCESS) return 1000 + (int)st; } while (0)
+    cudaError_t st;
+#define BL(call) do { st = (call); if (st != cudaSuccess) return 1000 + (int)st; } while (0)
     if (T == 0) return 0;
     tg_gather_x<<<nblk(T * (E / 4)), 256, 0, s>>>(inputs, tok, (int)T, E, tb.X);
-    BL(gemm_rm(c->blas, false, true, (int)T, 4 * H, E, tb.X, E, Wf, E, tb.Pf, 4 * H, 0.f));
-    if (dirs > 1) BL(gemm_rm(c->blas, false, true, (int)T, 4 * H, E, tb.X, E, Wb, E, tb.Pb, 4 * H, 0.f));
+    BL(gemm_rm(c->st, false, true, (int)T, 4 * H, E, tb.X, E, Wf, E, tb.Pf, 4 * H, 0.f));
+    if (dirs > 1) BL(gemm_rm(c->st, false, true, (int)T, 4 * H, E, tb.X, E, Wb, E, tb.Pb, 4 * H, 0.f));
     // forward over the time steps; the two directions are independent chains: the backward one runs on
     // the second stream (its own h_prev / recurrent-product buffers), joined before the head
     if (dirs > 1) {
@@ -700,7 +687,7 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
             const int dp = d == 0 ? -1 : 1;
             const float* U = d == 0 ? Uf : Ub;
             cudaStream_t sd = d == 0 ? s : c->s2;
-            cublasHandle_t hd = d == 0 ? c->blas : c->blas2;
+            cudaStream_t hd = d == 0 ? c->st : c->s2;
             float* HS = d == 0 ? tb.HS0 : tb.HS1;        // step-major h of this direction
             float* Zs = d == 0 ? tb.Zs : tb.Zs2;
             if (t > 0)   // h_prev of row r = row r of the previous step's block (longest-first step lists)
@@ -718,22 +705,22 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
     // z = W_tag m + b_tag; LSTM LM z = W_out h + b_out (L42); forward and backward
     const float* Hin = tb.HH;
     if (has_mlp) {
-        BL(gemm_rm(c->blas, false, true, (int)T, Mw, HW, tb.HH, HW, Wm, HW, tb.Mm, Mw, 0.f));
+        BL(gemm_rm(c->st, false, true, (int)T, Mw, HW, tb.HH, HW, Wm, HW, tb.Mm, Mw, 0.f));
         tg_tanh_bias<<<nblk(T * Mw), 256, 0, s>>>(tb.Mm, bm, T * Mw, Mw);
         Hin = tb.Mm;
     }
-    BL(gemm_rm(c->blas, false, true, (int)T, C, (int)Kh, Hin, (int)Kh, Wt, (int)Kh, tb.Z, C, 0.f));
+    BL(gemm_rm(c->st, false, true, (int)T, C, (int)Kh, Hin, (int)Kh, Wt, (int)Kh, tb.Z, C, 0.f));
     tg_softmax<<<nblk(T * 32), 256, 0, s>>>(tb.Z, bt, lab, (int)T, C, tb.dZ, pool + loss_word);
-    BL(gemm_rm(c->blas, true, false, C, (int)Kh, (int)T, tb.dZ, C, Hin, (int)Kh, grads + off[5], (int)Kh, 0.f));
+    BL(gemm_rm(c->st, true, false, C, (int)Kh, (int)T, tb.dZ, C, Hin, (int)Kh, grads + off[5], (int)Kh, 0.f));
     colsum<<<nblk(C), 256, 0, s>>>(tb.dZ, (int)T, C, grads + off[9]);
     if (has_mlp) {
-        BL(gemm_rm(c->blas, false, false, (int)T, Mw, C, tb.dZ, C, Wt, Mw, tb.dM, Mw, 0.f));
+        BL(gemm_rm(c->st, false, false, (int)T, Mw, C, tb.dZ, C, Wt, Mw, tb.dM, Mw, 0.f));
         tg_dtanh<<<nblk(T * Mw), 256, 0, s>>>(tb.dM, tb.Mm, T * Mw);
-        BL(gemm_rm(c->blas, true, false, Mw, HW, (int)T, tb.dM, Mw, tb.HH, HW, grads + off[4], HW, 0.f));
+        BL(gemm_rm(c->st, true, false, Mw, HW, (int)T, tb.dM, Mw, tb.HH, HW, grads + off[4], HW, 0.f));
         colsum<<<nblk(Mw), 256, 0, s>>>(tb.dM, (int)T, Mw, grads + off[8]);
-        BL(gemm_rm(c->blas, false, false, (int)T, HW, Mw, tb.dM, Mw, Wm, HW, tb.dHH, HW, 0.f));
+        BL(gemm_rm(c->st, false, false, (int)T, HW, Mw, tb.dM, Mw, Wm, HW, tb.dHH, HW, 0.f));
     } else {
-        BL(gemm_rm(c->blas, false, false, (int)T, HW, C, tb.dZ, C, Wt, HW, tb.dHH, HW, 0.f));
+        BL(gemm_rm(c->st, false, false, (int)T, HW, C, tb.dZ, C, Wt, HW, tb.dHH, HW, 0.f));
     }
     // backward through both LSTMs, last step first
     cudaMemsetAsync(tb.dHf, 0, T * H * sizeof(float), s);
@@ -750,7 +737,7 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
             const uint32_t* pos = (d == 0 ? fpos : bpos) + r0;
             const int dp = d == 0 ? -1 : 1;
             cudaStream_t sd = d == 0 ? s : c->s2;
-            cublasHandle_t hd = d == 0 ? c->blas : c->blas2;
+            cudaStream_t hd = d == 0 ? c->st : c->s2;
             float* Gs = d == 0 ? tb.Gs : tb.Gs2;
             // Γ Uᵀ of step t goes to one buffer and is read by step t-1, whose product goes to the other
             float* DhW = (t & 1) ? (d == 0 ? tb.Dh : tb.Dh2) : (d == 0 ? tb.DhB0 : tb.DhB1);
@@ -776,13 +763,13 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
             const int32_t n = start[maxlen] - start[1];
             tg_hprev_all<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.HH, pos + start[1], n, dp, d, H, HW, tb.Hp);
         }
-        BL(gemm_rm(c->blas, true, false, 4 * H, E, (int)T, Gam, 4 * H, tb.X, E, grads + off[d == 0 ? 0 : 2], E, 0.f));
-        BL(gemm_rm(c->blas, true, false, 4 * H, H, (int)T, Gam, 4 * H, tb.Hp, H, grads + off[d == 0 ? 1 : 3], H, 0.f));
+        BL(gemm_rm(c->st, true, false, 4 * H, E, (int)T, Gam, 4 * H, tb.X, E, grads + off[d == 0 ? 0 : 2], E, 0.f));
+        BL(gemm_rm(c->st, true, false, 4 * H, H, (int)T, Gam, 4 * H, tb.Hp, H, grads + off[d == 0 ? 1 : 3], H, 0.f));
         colsum<<<nblk(4 * H), 256, 0, s>>>(Gam, (int)T, 4 * H, grads + off[d == 0 ? 6 : 7]);
     }
     if (d_inputs) {
-        BL(gemm_rm(c->blas, false, false, (int)T, E, 4 * H, tb.Gamf, 4 * H, Wf, E, tb.DX, E, 0.f));
-        if (dirs > 1) BL(gemm_rm(c->blas, false, false, (int)T, E, 4 * H, tb.Gamb, 4 * H, Wb, E, tb.DX, E, 1.f));
+        BL(gemm_rm(c->st, false, false, (int)T, E, 4 * H, tb.Gamf, 4 * H, Wf, E, tb.DX, E, 0.f));
+        if (dirs > 1) BL(gemm_rm(c->st, false, false, (int)T, E, 4 * H, tb.Gamb, 4 * H, Wb, E, tb.DX, E, 1.f));
         tg_scatter_dx<<<nblk(T * E), 256, 0, s>>>(tb.DX, tok, (int)T, E, d_inputs);
     }
 #undef BL
@@ -800,7 +787,7 @@ int gru_pass(void* ctx_, const float* params, const int64_t* off, float* grads, 
     using namespace dev::lv;
     LevelCtx* c = static_cast<LevelCtx*>(ctx_);
     TaggerBufs& tb = c->tg;
-    cublasSetStream(c->blas, s);
+    c->st = s;
     const int64_t Tn = std::max<int64_t>(T, 1);
     // X, Px (Pf), HH, Gd (Gf), Hp, Zs, Z, dZ, dHH, dHr (dHf), Gx (Gamf), Gh (Gamb), Gs, Dh, Ez (Cf), DX
     float** bufs[16] = {&tb.X, &tb.Pf, &tb.HH, &tb.Gf, &tb.Hp, &tb.Zs, &tb.Z, &tb.dZ, &tb.dHH, &tb.dHf, &tb.Gamf,
@@ -817,25 +804,25 @@ int gru_pass(void* ctx_, const float* params, const int64_t* off, float* grads, 
     const float *W = params + off[0], *U = params + off[1], *Wo = params + off[2], *b_i = params + off[3],
                 *b_h = params + off[4], *bo = params + off[5];
     const uint32_t *tok = d_blob + tg_tok, *lab = d_blob + tg_lab, *fpos = d_blob + tg_fpos;
-    cublasStatus_t st;
-#define BL(call) do { st = (call); if (st != CUBLAS_STATUS_SUCCESS) return 1000 + (int)st; } while (0)
+    cudaError_t st;
+#define BL(call) do { st = (call); if (st != cudaSuccess) return 1000 + (int)st; } while (0)
     if (T == 0) return 0;
     tg_gather_x<<<nblk(T * (E / 4)), 256, 0, s>>>(inputs, tok, (int)T, E, tb.X);
-    BL(gemm_rm(c->blas, false, true, (int)T, 3 * H, E, tb.X, E, W, E, tb.Pf, 3 * H, 0.f));
+    BL(gemm_rm(c->st, false, true, (int)T, 3 * H, E, tb.X, E, W, E, tb.Pf, 3 * H, 0.f));
     for (int32_t t = 0; t < maxlen; ++t) {
         const int32_t r0 = start[t], n = start[t + 1] - r0;
         const uint32_t* pos = fpos + r0;
         if (t > 0)   // h_prev of row r = row r of the previous step's block (longest-first step lists)
-            BL(gemm_rm(c->blas, false, true, n, 3 * H, H, tb.HS0 + (int64_t)start[t - 1] * H, H, U, H, tb.Zs, 3 * H, 0.f));
+            BL(gemm_rm(c->st, false, true, n, 3 * H, H, tb.HS0 + (int64_t)start[t - 1] * H, H, U, H, tb.Zs, 3 * H, 0.f));
         gru_cell<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.Pf, tb.Zs, b_i, b_h, pos, n, -1, t == 0, H, tb.HH, tb.Gf,
                                                        tb.HS0 + (int64_t)r0 * H);
     }
     // head on h (L42): z = W_out h + b_out, softmax-NLL on labelled positions, dW_out, db_out, dh
-    BL(gemm_rm(c->blas, false, true, (int)T, C, H, tb.HH, H, Wo, H, tb.Z, C, 0.f));
+    BL(gemm_rm(c->st, false, true, (int)T, C, H, tb.HH, H, Wo, H, tb.Z, C, 0.f));
     tg_softmax<<<nblk(T * 32), 256, 0, s>>>(tb.Z, bo, lab, (int)T, C, tb.dZ, pool + loss_word);
-    BL(gemm_rm(c->blas, true, false, C, H, (int)T, tb.dZ, C, tb.HH, H, grads + off[2], H, 0.f));
+    BL(gemm_rm(c->st, true, false, C, H, (int)T, tb.dZ, C, tb.HH, H, grads + off[2], H, 0.f));
     colsum<<<nblk(C), 256, 0, s>>>(tb.dZ, (int)T, C, grads + off[5]);
-    BL(gemm_rm(c->blas, false, false, (int)T, H, C, tb.dZ, C, Wo, H, tb.dHH, H, 0.f));
+    BL(gemm_rm(c->st, false, false, (int)T, H, C, tb.dZ, C, Wo, H, tb.dHH, H, 0.f));
     cudaMemsetAsync(tb.dHf, 0, T * H * sizeof(float), s);
     for (int32_t t = maxlen - 1; t >= 0; --t) {
         const int32_t r0 = start[t], n = start[t + 1] - r0;
@@ -848,7 +835,7 @@ int gru_pass(void* ctx_, const float* params, const int64_t* off, float* grads, 
         const int32_t n_next = t + 1 < maxlen ? start[t + 2] - start[t + 1] : 0;
         gru_cell_bwd<<<nblk((int64_t)n * H), 256, 0, s>>>(pos, n, -1, t == 0, H, tb.dHH, DhR, EzR, n_next, tb.HH,
                                                            tb.Gf, tb.Gamf, tb.Gamb, tb.Gs, EzW);
-        if (t > 0) BL(gemm_rm(c->blas, false, false, n, H, 3 * H, tb.Gs, 3 * H, U, H, DhW, H, 0.f));
+        if (t > 0) BL(gemm_rm(c->st, false, false, n, H, 3 * H, tb.Gs, 3 * H, U, H, DhW, H, 0.f));
     }
     // dW = Γ_xᵀ X, dU = Γ_hᵀ H_prev (zeros at chain starts), db_i = Σ Γ_x, db_h = Σ Γ_h; dX = Γ_x W
     cudaMemsetAsync(tb.Hp, 0, T * H * sizeof(float), s);
@@ -856,12 +843,12 @@ int gru_pass(void* ctx_, const float* params, const int64_t* off, float* grads, 
         const int32_t n = start[maxlen] - start[1];
         tg_hprev_all<<<nblk((int64_t)n * H), 256, 0, s>>>(tb.HH, fpos + start[1], n, -1, 0, H, H, tb.Hp);
     }
-    BL(gemm_rm(c->blas, true, false, 3 * H, E, (int)T, tb.Gamf, 3 * H, tb.X, E, grads + off[0], E, 0.f));
-    BL(gemm_rm(c->blas, true, false, 3 * H, H, (int)T, tb.Gamb, 3 * H, tb.Hp, H, grads + off[1], H, 0.f));
+    BL(gemm_rm(c->st, true, false, 3 * H, E, (int)T, tb.Gamf, 3 * H, tb.X, E, grads + off[0], E, 0.f));
+    BL(gemm_rm(c->st, true, false, 3 * H, H, (int)T, tb.Gamb, 3 * H, tb.Hp, H, grads + off[1], H, 0.f));
     colsum<<<nblk(3 * H), 256, 0, s>>>(tb.Gamf, (int)T, 3 * H, grads + off[3]);
     colsum<<<nblk(3 * H), 256, 0, s>>>(tb.Gamb, (int)T, 3 * H, grads + off[4]);
     if (d_inputs) {
-        BL(gemm_rm(c->blas, false, false, (int)T, E, 3 * H, tb.Gamf, 3 * H, W, E, tb.DX, E, 0.f));
+        BL(gemm_rm(c->st, false, false, (int)T, E, 3 * H, tb.Gamf, 3 * H, W, E, tb.DX, E, 0.f));
         tg_scatter_dx<<<nblk(T * E), 256, 0, s>>>(tb.DX, tok, (int)T, E, d_inputs);
     }
 #undef BL
@@ -878,7 +865,7 @@ int rvnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads,
               int32_t E, int32_t C, int64_t loss_word, cudaStream_t s) {
     using namespace dev::lv;
     LevelCtx* c = static_cast<LevelCtx*>(ctx_);
-    cublasSetStream(c->blas, s);
+    c->st = s;
     if (!grow(&c->b.X_leaf, &c->cap_X_leaf, std::max<int64_t>(n_leaf * E, 4)) ||
         !grow(&c->b.X_int, &c->cap_X_int, std::max<int64_t>(n_int * 2 * H, 4)) ||
         !grow(&c->b.Z, &c->cap_Z, std::max<int64_t>(std::max(n_leaf, n_int) * H, 4)) ||
@@ -892,11 +879,11 @@ int rvnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads,
     const uint32_t* leaves = d_blob + lv_leaf;   // (rec, adj, token) per leaf
     const uint32_t* hl = d_blob + lv_head;
     float *Xl = c->b.X_leaf, *Xi = c->b.X_int, *Z = c->b.Z, *Gi = c->b.G_int, *Gl = c->b.G_leaf, *DX = c->b.DX;
-    cublasStatus_t st = CUBLAS_STATUS_SUCCESS;
-#define BL(call) do { st = (call); if (st != CUBLAS_STATUS_SUCCESS) return 1000 + (int)st; } while (0)
+    cudaError_t st = cudaSuccess;
+#define BL(call) do { st = (call); if (st != cudaSuccess) return 1000 + (int)st; } while (0)
     if (n_leaf > 0) {
         gather_leaf<<<nblk(n_leaf * (E / 4)), 256, 0, s>>>(inputs, leaves, (int)n_leaf, E, Xl);
-        BL(gemm_rm(c->blas, false, true, (int)n_leaf, H, E, Xl, E, W_leaf, E, Z, H, 0.f));
+        BL(gemm_rm(c->st, false, true, (int)n_leaf, H, E, Xl, E, W_leaf, E, Z, H, 0.f));
         rv_cell<<<nblk(n_leaf * H), 256, 0, s>>>(Z, b_leaf, leaves, 3, (int)n_leaf, H, pool);
     }
     for (int32_t l = 1; l <= L; ++l) {
@@ -904,7 +891,7 @@ int rvnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads,
         if (n <= 0) continue;
         float* X = Xi + r0 * 2 * H;
         gather_int<<<nblk(n * (2 * H / 4)), 256, 0, s>>>(pool, ints + 6 * r0, (int)n, H, X);
-        BL(gemm_rm(c->blas, false, true, (int)n, H, 2 * H, X, 2 * H, W_int, 2 * H, Z, H, 0.f));
+        BL(gemm_rm(c->st, false, true, (int)n, H, 2 * H, X, 2 * H, W_int, 2 * H, Z, H, 0.f));
         rv_cell<<<nblk(n * H), 256, 0, s>>>(Z, b_int, ints + 6 * r0, 6, (int)n, H, pool);
     }
     if (n_head > 0)
@@ -915,20 +902,20 @@ int rvnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads,
         if (n <= 0) continue;
         float* G = Gi + r0 * H;
         rv_bwd<<<nblk(n * H), 256, 0, s>>>(ints + 6 * r0, 6, 3, (int)n, H, pool, G);
-        BL(gemm_rm(c->blas, false, false, (int)n, 2 * H, H, G, H, W_int, 2 * H, DX, 2 * H, 0.f));
+        BL(gemm_rm(c->st, false, false, (int)n, 2 * H, H, G, H, W_int, 2 * H, DX, 2 * H, 0.f));
         scatter_dh<<<nblk(n * 2 * H), 256, 0, s>>>(DX, ints + 6 * r0, (int)n, H, pool);
     }
     if (n_leaf > 0) {
         rv_bwd<<<nblk(n_leaf * H), 256, 0, s>>>(leaves, 3, 1, (int)n_leaf, H, pool, Gl);
         if (d_inputs) {
-            BL(gemm_rm(c->blas, false, false, (int)n_leaf, E, H, Gl, H, W_leaf, E, DX, E, 0.f));
+            BL(gemm_rm(c->st, false, false, (int)n_leaf, E, H, Gl, H, W_leaf, E, DX, E, 0.f));
             scatter_dx<<<nblk(n_leaf * E), 256, 0, s>>>(DX, leaves, (int)n_leaf, E, d_inputs);
         }
-        BL(gemm_rm(c->blas, true, false, H, E, (int)n_leaf, Gl, H, Xl, E, grads + off[0], E, 0.f));
+        BL(gemm_rm(c->st, true, false, H, E, (int)n_leaf, Gl, H, Xl, E, grads + off[0], E, 0.f));
         colsum<<<nblk(H), 256, 0, s>>>(Gl, (int)n_leaf, H, grads + off[3]);
     }
     if (n_int > 0) {
-        BL(gemm_rm(c->blas, true, false, H, 2 * H, (int)n_int, Gi, H, Xi, 2 * H, grads + off[1], 2 * H, 0.f));
+        BL(gemm_rm(c->st, true, false, H, 2 * H, (int)n_int, Gi, H, Xi, 2 * H, grads + off[1], 2 * H, 0.f));
         colsum<<<nblk(H), 256, 0, s>>>(Gi, (int)n_int, H, grads + off[4]);
     }
 #undef BL
@@ -946,7 +933,7 @@ int tdrnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads
     using namespace dev::lv;
     (void)E;
     LevelCtx* c = static_cast<LevelCtx*>(ctx_);
-    cublasSetStream(c->blas, s);
+    c->st = s;
     if (!grow(&c->b.X_int, &c->cap_X_int, std::max<int64_t>(n_int * 2 * H, 4)) ||
         !grow(&c->b.Z, &c->cap_Z, std::max<int64_t>(n_int * H, 4)) ||
         !grow(&c->b.G_int, &c->cap_G_int, std::max<int64_t>(n_int * H, 4)) ||
@@ -957,15 +944,15 @@ int tdrnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads
     const uint32_t* leaves = d_blob + lv_leaf;
     const uint32_t* hl = d_blob + lv_head;
     float *Xi = c->b.X_int, *Z = c->b.Z, *Gi = c->b.G_int, *DX = c->b.DX;
-    cublasStatus_t st = CUBLAS_STATUS_SUCCESS;
-#define BL(call) do { st = (call); if (st != CUBLAS_STATUS_SUCCESS) return 1000 + (int)st; } while (0)
+    cudaError_t st = cudaSuccess;
+#define BL(call) do { st = (call); if (st != cudaSuccess) return 1000 + (int)st; } while (0)
     if (n_leaf > 0) td_leaf<<<nblk(n_leaf * H), 256, 0, s>>>(inputs, leaves, (int)n_leaf, H, pool);
     for (int32_t l = 1; l <= L; ++l) {
         const int64_t r0 = lv_start[l], n = lv_start[l + 1] - r0;
         if (n <= 0) continue;
         float* X = Xi + r0 * 2 * H;
         gather_int<<<nblk(n * (2 * H / 4)), 256, 0, s>>>(pool, ints + 6 * r0, (int)n, H, X);
-        BL(gemm_rm(c->blas, false, true, (int)n, H, 2 * H, X, 2 * H, W, 2 * H, Z, H, 0.f));
+        BL(gemm_rm(c->st, false, true, (int)n, H, 2 * H, X, 2 * H, W, 2 * H, Z, H, 0.f));
         rv_cell<<<nblk(n * H), 256, 0, s>>>(Z, b, ints + 6 * r0, 6, (int)n, H, pool);
     }
     if (n_head > 0)
@@ -976,12 +963,12 @@ int tdrnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads
         if (n <= 0) continue;
         float* G = Gi + r0 * H;
         rv_bwd<<<nblk(n * H), 256, 0, s>>>(ints + 6 * r0, 6, 3, (int)n, H, pool, G);
-        BL(gemm_rm(c->blas, false, false, (int)n, 2 * H, H, G, H, W, 2 * H, DX, 2 * H, 0.f));
+        BL(gemm_rm(c->st, false, false, (int)n, 2 * H, H, G, H, W, 2 * H, DX, 2 * H, 0.f));
         scatter_dh_shared<<<nblk(n * 2 * H), 256, 0, s>>>(DX, ints + 6 * r0, (int)n, H, pool);
     }
     if (n_leaf > 0 && d_inputs) td_leaf_dx<<<nblk(n_leaf * H), 256, 0, s>>>(leaves, (int)n_leaf, H, pool, d_inputs);
     if (n_int > 0) {
-        BL(gemm_rm(c->blas, true, false, H, 2 * H, (int)n_int, Gi, H, Xi, 2 * H, grads + off[0], 2 * H, 0.f));
+        BL(gemm_rm(c->st, true, false, H, 2 * H, (int)n_int, Gi, H, Xi, 2 * H, grads + off[0], 2 * H, 0.f));
         colsum<<<nblk(H), 256, 0, s>>>(Gi, (int)n_int, H, grads + off[2]);
     }
 #undef BL

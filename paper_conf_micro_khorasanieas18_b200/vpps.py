@@ -109,6 +109,7 @@ def _load():
         "vpps_last_error": [],
         "vpps_variants": [VP, I32],
     }
+    sig["vpps_gemm_f32"] = [VP, I32, I32, I32, I32, I32, VP, I32, VP, I32, VP, I32, F]
     for name, args in sig.items():
         fn = getattr(lib, name)
         fn.argtypes = args
@@ -161,6 +162,18 @@ def param_shapes(cell: str, H: int, E: int, C: int, mlp: int = 256):
     raise ValueError(cell)
 
 
+def gemm_f32(A, B, C, ta=False, tb=False, beta=0.0, M=None, N=None, K=None, lda=None, ldb=None, ldc=None,
+             stream=None):
+    """C = op(A) op(B) + beta C through vpps_gemm_f32 (include/vpps.h) on float32 CUDA tensors (row-major;
+    leading dimensions default to the tensors' row strides)."""
+    M = M if M is not None else C.shape[0]
+    N = N if N is not None else C.shape[1]
+    K = K if K is not None else (A.shape[0] if ta else A.shape[1])
+    _check(_lib.vpps_gemm_f32(_stream_ptr(stream), int(ta), int(tb), M, N, K, ct.c_void_p(A.data_ptr()),
+                              lda or A.stride(0), ct.c_void_p(B.data_ptr()), ldb or B.stride(0),
+                              ct.c_void_p(C.data_ptr()), ldc or C.stride(0), beta))
+
+
 def variants():
     buf = (ct.c_int32 * 256)()
     n = _lib.vpps_variants(ct.cast(buf, ct.c_void_p), 64)
@@ -211,14 +224,17 @@ class CsrBatch:
         return cls(*to_csr(graphs))
 
 
-def prefetch_scripts(model: "Model", batches, depth: int = 4, workers: int = 3):
+def prefetch_scripts(model: "Model", batches, depth: int = 4, workers: int = 3, executor=None):
     """Yield model.build_script(b) for b in batches, in order, built up to `depth` ahead by `workers`
     background threads (the C++ builder runs without the GIL), so host script generation
-    overlaps the device passes: one builder takes ~200 us per 16-tree batch, longer than a device step."""
+    overlaps the device passes: one builder takes ~100-200 us per 16-tree batch, about a device step.
+    `executor`: an existing concurrent.futures executor to build on (kept running across calls)."""
     import collections
+    import contextlib
     from concurrent.futures import ThreadPoolExecutor
     it = iter(batches)
-    with ThreadPoolExecutor(max_workers=max(1, workers)) as ex:
+    own = executor is None
+    with (ThreadPoolExecutor(max_workers=max(1, workers)) if own else contextlib.nullcontext(executor)) as ex:
         pend = collections.deque()
         for b in it:
             pend.append(ex.submit(model.build_script, b))

@@ -143,7 +143,7 @@ def check_update(m, P, Pn, params):
     for name, _ in m.shapes:
         got = pv[name].double().numpy()
         step = Pn[name] - P[name]
-        bound = TOL * np.abs(step).max() + 2.0 ** -24 * np.abs(Pn[name]).max()
+        bound = TOL * np.abs(step).max() + 2.0 ** -22 * np.abs(Pn[name]).max()
         assert np.abs(got - Pn[name]).max() <= bound, (name, np.abs(got - Pn[name]).max(), bound)
 
 
