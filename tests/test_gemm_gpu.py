@@ -54,3 +54,26 @@ def test_gemm_strided_and_unaligned():
     vpps.gemm_f32(X, W, C, M=8, N=8, K=0)
     torch.cuda.synchronize()
     assert float(C.abs().max()) == 0.0
+
+
+TC_SHAPES = [(64, 64, 64), (65, 129, 70), (200, 96, 100), (128, 128, 4096), (300, 1000, 257), (1000, 3072, 2048)]
+
+
+@pytest.mark.parametrize("mode", ["0", "-1"])
+def test_gemm_tensor_core_and_simt_forced(mode):
+    """VPPS_GEMM_TC_MIN=0 sends every product with M, N, K >= 64 to the tcgen05 3xTF32 tiles (ragged tiles,
+    split-K, all transposes, beta 0 / 1); -1 keeps every product on the FFMA2 tiles.  The switch is read
+    once per process, so each mode runs in a child process."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = ("import sys; sys.path.insert(0, %r); sys.path.insert(0, %r); import test_gemm_gpu as t\n"
+            "for ta in (False, True):\n"
+            "  for tb in (False, True):\n"
+            "    for sh in t.TC_SHAPES + t.SHAPES[:6]:\n"
+            "      t.test_gemm_against_float64(ta, tb, sh)\n"
+            "print('ok')" % (root, os.path.join(root, "tests")))
+    r = subprocess.run([sys.executable, "-c", code], env={**os.environ, "VPPS_GEMM_TC_MIN": mode}, capture_output=True,
+                       text=True, timeout=900)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stdout + r.stderr
