@@ -57,6 +57,7 @@ struct vpps_model_s {
     int64_t n_floats = 0;
     bool plan_only = true;
     int device = 0;
+    int32_t sms = 148;                  // SM count of the device (persistent GEMM grids)
     const Variant* var = nullptr;
     size_t smem = 0;
     float* params = nullptr;
@@ -193,6 +194,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
         if (prop.major != 10) return fail(VPPS_E_INVALID, "libvpps is built for sm_100a (B200) only");
         if (n_sm == 0) n_sm = prop.multiProcessorCount;
         if (n_sm > prop.multiProcessorCount) return fail(VPPS_E_INVALID, "n_sm exceeds the device's SM count");
+        m->sms = prop.multiProcessorCount;
     } else if (n_sm == 0) {
         n_sm = m->cluster ? m->cluster * o.groups : 148;
     }
@@ -620,10 +622,21 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
             if (s->s.grp_levels[a] != s->s.grp_levels[b]) return s->s.grp_levels[a] < s->s.grp_levels[b];
             return s->s.grp_nodes[a] < s->s.grp_nodes[b];
         });
-        launch_dw_gemm(m->pool, inputs, d_inputs, m->params, m->grads, lists, leaf_list, n_grp, s->s.int_off.data(),
-                       s->s.leaf_off.data(), order.data(), m->done, m->cluster, true, m->plan.H, m->plan.E,
-                       m->offsets.data(), m->n_floats, mode, lr, wd, st, m->gemm_trace,
-                       m->pool + s->s.loss_word, m->d_loss_map + (m->passes & 1));
+        // weight gradients (L185) + leaf dX after the pass: tensor-core tiles over every node of the batch
+        // (vpps_dwtc.cu), SGD fused in their tail at N = 1; VPPS_DW_ITEMS=1 (measurement) keeps the FFMA2
+        // per-group items that overlap the slowest groups instead
+        static const bool dw_items = getenv("VPPS_DW_ITEMS") && atoi(getenv("VPPS_DW_ITEMS")) != 0;
+        if (dw_items || m->gemm_trace) {
+            launch_dw_gemm(m->pool, inputs, d_inputs, m->params, m->grads, lists, leaf_list, n_grp, s->s.int_off.data(),
+                           s->s.leaf_off.data(), order.data(), m->done, m->cluster, true, m->plan.H, m->plan.E,
+                           m->offsets.data(), m->n_floats, mode, lr, wd, st, m->gemm_trace,
+                           m->pool + s->s.loss_word, m->d_loss_map + (m->passes & 1));
+        } else if (!launch_dw_tc(m->pool, inputs, d_inputs, m->params, m->grads, lists, leaf_list, (int32_t)s->s.n_int,
+                                 (int32_t)s->s.n_leaf, m->plan.H, m->plan.E, m->offsets.data(), m->n_floats,
+                                 m->done + 32, mode, lr, wd, st, m->pool + s->s.loss_word,
+                                 m->d_loss_map + (m->passes & 1), m->sms)) {
+            return fail(VPPS_E_CUDA, "gradient GEMM launch failed");
+        }
         CK(cudaGetLastError());
     } else if (m->plan.level && m->plan.cell == CELL_GRU) {
         if (s->s.tg_tok < 0) return fail(VPPS_E_INVALID, "script was not built for the level path");

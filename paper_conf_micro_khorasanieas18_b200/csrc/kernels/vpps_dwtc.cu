@@ -1,0 +1,321 @@
+// Weight gradients of the binary Tree-LSTM's dataflow path on the tensor cores ("concatenate all
+// the left hand side and all the right hand side tensors that participate in the outer-product for each
+// weight matrix, and use dense matrix-matrix multiplication"), after vpps_df, over every node of the batch:
+//   p0  dU_iou [3H x 2H] = Σ_int  g_iou [h_l; h_r]ᵀ     A(m, k) = pool[rec_k + 7H + m], B(k, n) = h_l / h_r of k
+//   p1  dU_fl  [H x H]   = Σ_int  g_fl h_lᵀ             A = pool[rec_k + 10H + m],      B = pool[rec_l(k) + n]
+//   p2  dU_fr  [H x H]   = Σ_int  g_fr h_rᵀ             A = pool[rec_k + 11H + m],      B = pool[rec_r(k) + n]
+//   p3  dW_iou [3H x E]  = Σ_leaf g x_tokᵀ              A = pool[rec_k + 5H + m],       B = inputs[tok_k E + n]
+//   p4  dX[tok_m] += g_leaf(m)ᵀ W_iou  [leaves x E]     A(m, k) = pool[rec_m + 5H + k], B(k, n) = W_iou[k E + n]
+// (operands gathered row by row through the node lists while they are staged; tc_common.cuh's 128 x 128
+// 3xTF32 tiles).  Work items = (product, 128 x 128 tile, K range); K is split so that the items of all
+// products fill one wave of persistent CTAs; partial tiles are added into grads / dX (cleared by the leaf
+// kernel) with red.global.add.v4.  Then, as in the FFMA2 gradient GEMM it replaces, the CTAs apply the SGD
+// update (L129, L197) once every item is counted, and one CTA copies the summed loss to mapped host memory.
+#include <algorithm>
+#include <atomic>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "dev_common.cuh"
+#include "tc_common.cuh"
+#include "vpps_kernel.cuh"
+
+namespace vpps {
+namespace dev {
+namespace dwtc {
+using namespace tcc;
+
+constexpr int NP = 5;
+
+struct Params {
+    const float* pool;
+    const float* inputs;
+    const float* w_iou;
+    float* grads;
+    float* d_inputs;                 // dX or nullptr (p4 skipped)
+    const uint32_t* ints;            // n_int x (rec, rec_l, rec_r)
+    const uint32_t* leaves;          // n_leaf x (rec, token)
+    int32_t n_int, n_leaf, H, E;
+    int64_t off[8];
+    int32_t tm[NP], tn[NP], splits[NP], ksplit[NP], K[NP], M[NP], N[NP];
+    int32_t first[NP + 1];           // item prefix over the products
+    int32_t total;
+    // tail
+    int32_t* fin;
+    int32_t* tail_claim;
+    int32_t mode;
+    float* params;
+    int64_t n_floats;
+    float lr, wd;
+    const float* loss_src;
+    float* loss_dst;
+};
+
+// the row pointer of element (row r, k) of a K-contiguous operand, or of (k, row r) of a row-contiguous one
+struct Op {
+    const float* base;   // element address = base + (per-row or per-k offset) + (k or r)
+};
+
+__device__ __forceinline__ const float* a_ptr(const Params& P, int p, int r, int k) {
+    // A(m = r, k): p0..p3 row-contiguous in m for a fixed node k; p4 K-contiguous for a fixed leaf r
+    const int H = P.H;
+    switch (p) {
+        case 0: return P.pool + P.ints[3 * k] + 7 * H + r;
+        case 1: return P.pool + P.ints[3 * k] + 10 * H + r;
+        case 2: return P.pool + P.ints[3 * k] + 11 * H + r;
+        case 3: return P.pool + P.leaves[2 * k] + 5 * H + r;
+        default: return P.pool + P.leaves[2 * r] + 5 * H + k;
+    }
+}
+__device__ __forceinline__ const float* b_ptr(const Params& P, int p, int k, int n) {
+    // B(k, n): row-contiguous in n for a fixed k in every product
+    const int H = P.H;
+    switch (p) {
+        case 0: return n < H ? P.pool + P.ints[3 * k + 1] + n : P.pool + P.ints[3 * k + 2] + (n - H);
+        case 1: return P.pool + P.ints[3 * k + 1] + n;
+        case 2: return P.pool + P.ints[3 * k + 2] + n;
+        case 3: return P.inputs + (int64_t)P.leaves[2 * k + 1] * P.E + n;
+        default: return P.w_iou + (int64_t)k * P.E + n;
+    }
+}
+
+// stage loads of one chunk: A is K-contiguous only in p4; B is always row-contiguous (in n)
+__device__ __forceinline__ void load_a(const Params& P, int p, int m0, int M, int k0, int ke, float4 (&v)[4]) {
+    const bool kc = p == 4;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        int r, k;
+        piece_rk(kc, q, r, k);
+        const int gr = m0 + r, gk = k0 + k;
+        float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (kc) {
+            if (gr < M) {
+                const float* src = a_ptr(P, p, gr, gk);
+                if (gk + 3 < ke) x = __ldcg(reinterpret_cast<const float4*>(src));
+                else {
+                    if (gk < ke) x.x = __ldcg(src);
+                    if (gk + 1 < ke) x.y = __ldcg(src + 1);
+                    if (gk + 2 < ke) x.z = __ldcg(src + 2);
+                }
+            }
+        } else if (gk < ke && gr < M) {       // M is a multiple of 4 (3H, H)
+            x = __ldcg(reinterpret_cast<const float4*>(a_ptr(P, p, gr, gk)));
+        }
+        v[q] = x;
+    }
+}
+__device__ __forceinline__ void load_b(const Params& P, int p, int n0, int N, int k0, int ke, float4 (&v)[4]) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        int r, k;
+        piece_rk(false, q, r, k);
+        const int gn = n0 + r, gk = k0 + k;
+        v[q] = (gk < ke && gn < N) ? __ldcg(reinterpret_cast<const float4*>(b_ptr(P, p, gk, gn)))
+                                   : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+}
+
+__global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
+    extern __shared__ __align__(128) float tsm[];
+    __shared__ uint32_t tmem_base;
+    __shared__ __align__(8) uint64_t mbar[2];
+    __shared__ int pick;
+    float* sm = reinterpret_cast<float*>((reinterpret_cast<uintptr_t>(tsm) + 127) & ~uintptr_t(127));
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    setup(&tmem_base, mbar);
+    const uint32_t tmem = tmem_base;
+    uint32_t phases = 0u;
+    // the records and node lists are complete once vpps_df (the primary grid) has finished
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    for (int it = blockIdx.x; it < P.total; it += gridDim.x) {
+        int p = 0;
+        while (it >= P.first[p + 1]) ++p;
+        const int local = it - P.first[p];
+        const int per_split = P.tm[p] * P.tn[p];
+        const int sp = local / per_split, t = local - sp * per_split;
+        const int m0 = (t / P.tn[p]) * BM, n0 = (t % P.tn[p]) * BN;
+        const int kb = sp * P.ksplit[p], ke = min(P.K[p], kb + P.ksplit[p]);
+        const int M = P.M[p], N = P.N[p];
+        const int nch = (ke - kb + BKC - 1) / BKC;
+        float4 ra[4], rb[4];
+        load_a(P, p, m0, M, kb, ke, ra);
+        load_b(P, p, n0, N, kb, ke, rb);
+        for (int c = 0; c < nch; ++c) {
+            const int st = c & 1;
+            float* Ah = sm + st * STAGE_F;
+            if (c >= 2) { mbar_wait(smem_u32(&mbar[st]), (phases >> st) & 1u); phases ^= 1u << st; }
+            if (p == 4) store_chunk<true>(Ah, Ah + OP_F, ra);
+            else store_chunk<false>(Ah, Ah + OP_F, ra);
+            store_chunk<false>(Ah + 2 * OP_F, Ah + 3 * OP_F, rb);
+            if (c + 1 < nch) {
+                load_a(P, p, m0, M, kb + (c + 1) * BKC, ke, ra);
+                load_b(P, p, n0, N, kb + (c + 1) * BKC, ke, rb);
+            }
+            issue_chunk(tmem, Ah, &mbar[st], c == 0);
+        }
+        // drain: the last commit covers every MMA of the item; both stages are then free for the next item
+        if (nch > 0) {
+            const int st = (nch - 1) & 1;
+            mbar_wait(smem_u32(&mbar[st]), (phases >> st) & 1u);
+            phases ^= 1u << st;
+            if (nch >= 2) {                       // the other stage's last completion was not waited for
+                const int so = st ^ 1;
+                mbar_wait(smem_u32(&mbar[so]), (phases >> so) & 1u);
+                phases ^= 1u << so;
+            }
+        }
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        if (nch > 0) {
+            const int row = m0 + 32 * (warp & 3) + lane, cb = 64 * (warp >> 2);
+            float* out;
+            int ld;
+            if (p == 4) {
+                out = row < M ? P.d_inputs + (int64_t)P.leaves[2 * row + 1] * P.E : nullptr;
+                ld = 0;
+            } else {
+                out = P.grads + P.off[p == 3 ? 0 : p + 1] + (int64_t)row * N;
+                ld = N;
+            }
+            (void)ld;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                uint32_t r[16];
+                load16(tmem, cb + 16 * q, r);
+                const int nb = n0 + cb + 16 * q;
+                if (row < M && out) {
+#pragma unroll
+                    for (int j = 0; j < 16; j += 4)
+                        if (nb + j < N) {     // N is a multiple of 4
+                            const float v[4] = {__uint_as_float(r[j]), __uint_as_float(r[j + 1]),
+                                                __uint_as_float(r[j + 2]), __uint_as_float(r[j + 3])};
+                            red_add<4>(out + nb + j, v);
+                        }
+                }
+            }
+        }
+        // every thread's TMEM reads (and the item's reductions) precede the next item's first MMA
+        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        __syncthreads();
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        if (tid == 0) asm volatile("red.release.gpu.global.add.s32 [%0], 1;" ::"l"(P.fin) : "memory");
+    }
+    teardown(tmem);
+    // ---- tail: SGD over the flat parameters once every item is counted (L129, L197), loss read-back (L199) ----
+    if (tid == 0) {
+        uint32_t f;
+        while (true) {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(f) : "l"(P.fin) : "memory");
+            if ((int)f >= P.total) break;
+            __nanosleep(100);
+        }
+    }
+    __syncthreads();
+    constexpr int CV = 4;
+    constexpr int64_t CH = 4 * CV * NT;
+    const int64_t n_chunks = P.mode == 1 ? (P.n_floats + CH - 1) / CH : 0;
+    while (true) {
+        if (tid == 0) pick = atomicAdd(P.tail_claim, 1);
+        __syncthreads();
+        const int64_t c = pick;
+        __syncthreads();
+        if (c == 0 && P.loss_dst && tid == 0) {
+            const float l = *reinterpret_cast<const volatile float*>(P.loss_src);
+            *reinterpret_cast<volatile float*>(P.loss_dst) = l;
+        }
+        if (c >= n_chunks) break;
+        const int64_t lo = c * CH, n4 = (min(P.n_floats, lo + CH) - lo) / 4;
+        float4* p4 = reinterpret_cast<float4*>(P.params + lo);
+        const float4* g4 = reinterpret_cast<const float4*>(P.grads + lo);
+        const float lr = P.lr, wd = P.wd;
+        float4 a[CV], b[CV];
+#pragma unroll
+        for (int q = 0; q < CV; ++q) {
+            const int64_t k = tid + NT * q;
+            if (k < n4) { a[q] = __ldcg(p4 + k); b[q] = __ldcg(g4 + k); }
+        }
+#pragma unroll
+        for (int q = 0; q < CV; ++q) {
+            const int64_t k = tid + NT * q;
+            if (k >= n4) break;
+            a[q].x -= lr * (b[q].x + wd * a[q].x); a[q].y -= lr * (b[q].y + wd * a[q].y);
+            a[q].z -= lr * (b[q].z + wd * a[q].z); a[q].w -= lr * (b[q].w + wd * a[q].w);
+            p4[k] = a[q];
+        }
+    }
+}
+
+}  // namespace dwtc
+}  // namespace dev
+
+// Host: products, tiles and K splits so that the items fill about one wave of 148 persistent CTAs.
+bool launch_dw_tc(const float* pool, const float* inputs, float* d_inputs, float* params, float* grads,
+                  const uint32_t* ints, const uint32_t* leaves, int32_t n_int, int32_t n_leaf, int32_t H, int32_t E,
+                  const int64_t* off, int64_t n_floats, int32_t* counters, int32_t mode, float lr, float wd,
+                  cudaStream_t s, const float* loss_src, float* loss_dst, int32_t n_sm) {
+    using namespace dev::dwtc;
+    using dev::tcc::BM;
+    using dev::tcc::BN;
+    using dev::tcc::BKC;
+    if ((H % 4) || (E % 4) || (n_floats % 4)) return false;
+    Params P{};
+    P.pool = pool; P.inputs = inputs; P.w_iou = params + off[0]; P.grads = grads; P.d_inputs = d_inputs;
+    P.ints = ints; P.leaves = leaves; P.n_int = n_int; P.n_leaf = n_leaf; P.H = H; P.E = E;
+    for (int i = 0; i < 8; ++i) P.off[i] = off[i];
+    const int Ms[NP] = {3 * H, H, H, 3 * H, n_leaf};
+    const int Ns[NP] = {2 * H, H, H, E, E};
+    const int Ks[NP] = {n_int, n_int, n_int, n_leaf, d_inputs ? 3 * H : 0};
+    int chunks_total = 0;
+    for (int p = 0; p < NP; ++p) {
+        P.M[p] = Ms[p]; P.N[p] = Ns[p]; P.K[p] = Ks[p];
+        P.tm[p] = (Ms[p] + BM - 1) / BM;
+        P.tn[p] = (Ns[p] + BN - 1) / BN;
+        if (Ms[p] <= 0 || Ks[p] <= 0) P.tm[p] = 0;
+        chunks_total += P.tm[p] * P.tn[p] * ((Ks[p] + BKC - 1) / BKC);
+    }
+    // smallest chunks-per-item target whose items fit one wave
+    int target = std::max(1, (chunks_total + n_sm - 1) / n_sm);
+    while (true) {
+        int items = 0;
+        for (int p = 0; p < NP; ++p) {
+            const int ch = (Ks[p] + BKC - 1) / BKC;
+            const int sp = P.tm[p] ? std::max(1, (ch + target - 1) / target) : 0;
+            items += P.tm[p] * P.tn[p] * sp;
+        }
+        if (items <= n_sm || target > 4096) break;
+        ++target;
+    }
+    P.first[0] = 0;
+    for (int p = 0; p < NP; ++p) {
+        const int ch = (Ks[p] + BKC - 1) / BKC;
+        int sp = P.tm[p] ? std::max(1, (ch + target - 1) / target) : 0;
+        P.ksplit[p] = sp ? ((ch + sp - 1) / sp) * BKC : 0;
+        P.splits[p] = sp ? (Ks[p] + P.ksplit[p] - 1) / P.ksplit[p] : 0;
+        P.first[p + 1] = P.first[p] + P.tm[p] * P.tn[p] * P.splits[p];
+    }
+    P.total = P.first[NP];
+    P.fin = counters;
+    P.tail_claim = counters + 1;
+    P.mode = mode; P.params = params; P.n_floats = n_floats; P.lr = lr; P.wd = wd;
+    P.loss_src = loss_src; P.loss_dst = loss_dst;
+    static std::atomic<uint64_t> attr_done{0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (!(attr_done.load() >> (dev & 63) & 1)) {
+        if (cudaFuncSetAttribute(vpps_dw_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dev::tcc::SMEM) != cudaSuccess)
+            return false;
+        attr_done.fetch_or(uint64_t(1) << (dev & 63));
+    }
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.gridDim = dim3(std::max(1, std::min(P.total, n_sm)));
+    cfg.blockDim = dim3(dev::tcc::NT);
+    cfg.dynamicSmemBytes = dev::tcc::SMEM;
+    cfg.stream = s;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, vpps_dw_tc, P) == cudaSuccess;
+}
+
+}  // namespace vpps

@@ -18,6 +18,7 @@
 #include <cuda_runtime.h>
 
 #include "dev_common.cuh"
+#include "tc_common.cuh"
 #include "vpps_kernel.cuh"
 
 namespace vpps {
@@ -167,52 +168,22 @@ sgemm(int M, int N, int K, const float* __restrict__ A, int lda, const float* __
     }
 }
 
-// ---- tensor-core tiles: tcgen05.mma kind::tf32 with a 3xTF32 split (FP32 accuracy) -------------------------
+// ---- tensor-core tiles: tcgen05.mma kind::tf32 with a 3xTF32 split (FP32 accuracy; tc_common.cuh) --------
 // Large products (the C5-sized level products and per-matrix gradient GEMMs: a level batches enough
-// same-parameter nodes to form a real dense GEMM, north_star) run on the 5th-gen tensor cores.
-// D[128 x 128] per CTA accumulates in TMEM (128 columns).  K runs in chunks of 32 through two shared-memory
-// stages; every thread stages its share of a chunk through registers — 16-byte global loads along the
-// operand's contiguous dimension, split v = hi + lo (hi = v truncated to TF32, lo = v - hi exact in FP32) and
-// stored in the K-major SWIZZLE_NONE canonical layout (core matrix 8 rows x 16 B, SBO 128 B between 8-row
-// groups; LBO = 2064 B between 4-k slices — 16 B of padding make both the 16-byte stores of K-contiguous
-// operands and the 4-byte transposing stores of M/N-contiguous ones bank-conflict free).  One thread issues
-// D += A·B + A·B_lo + A_lo·B per k-step of 8 (the dropped A_lo·B_lo is ~2^-22 relative) and commits to the
-// stage's mbarrier; the loads of chunk c + 1 are in flight while chunk c is converted and multiplied.
+// same-parameter nodes to form a real dense GEMM, north_star) run on the 5th-gen tensor cores: D[128 x 128]
+// per CTA in TMEM, K in chunks of 32 through two register-staged stages; the loads of chunk c + 1 are in
+// flight while chunk c is converted and multiplied.
 namespace tc {
-constexpr int BM = 128, BN = 128, BKC = 32, NT = 256;
-constexpr uint32_t LBO = (BM / 8) * 128 + 16;                 // bytes between 4-k slices (padded)
-constexpr int OP_F = (BKC / 4) * (LBO / 4);                    // floats of one operand copy (hi or lo)
-constexpr int STAGE_F = 4 * OP_F;                              // A hi, A lo, B hi, B lo
-constexpr size_t SMEM = (size_t)2 * STAGE_F * sizeof(float) + 128;
-static_assert(BM == BN, "one staging geometry for both operands");
+using namespace tcc;
 
-__device__ __forceinline__ uint64_t desc(uint32_t saddr) {
-    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)((LBO >> 4) & 0x3FFF) << 16) |
-           ((uint64_t)(128 >> 4) << 32) | ((uint64_t)1 << 46);
-}
-constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
-__device__ __forceinline__ void mma(uint32_t d, uint64_t a, uint64_t b, int acc) {
-    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-                 "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}\n"
-                 ::"r"(d), "l"(a), "l"(b), "r"(IDESC), "r"(acc));
-}
-__device__ __forceinline__ void mbar_wait(uint32_t mbar, uint32_t parity) {
-    uint32_t ok = 0;
-    while (!ok)
-        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}\n"
-                     : "=r"(ok) : "r"(mbar), "r"(parity) : "memory");
-}
-__device__ __forceinline__ float tf32_hi(float v) { return __uint_as_float(__float_as_uint(v) & 0xFFFFE000u); }
-
-// one operand's share of a chunk: 4 x 16-byte pieces per thread.  KC (contiguous along k): piece g = row
-// g / 8, k4 = g % 8; otherwise (contiguous along rows) lane = k, piece = 4 consecutive rows 4 (g / 32)
+// one operand's share of a chunk (piece_rk): 16-byte global loads along the operand's contiguous dimension
 template <bool KC>
 __device__ __forceinline__ void load_chunk(const float* __restrict__ X, int ld, int r0, int rmax, int k0, int kmax,
                                            float4 (&v)[4]) {
 #pragma unroll
     for (int p = 0; p < 4; ++p) {
-        const int g = threadIdx.x + NT * p;
-        const int r = KC ? g / 8 : 4 * (g / 32), k = KC ? 4 * (g % 8) : g % 32;
+        int r, k;
+        piece_rk(KC, p, r, k);
         const int gr = r0 + r, gk = k0 + k;
         float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
         if (KC) {
@@ -237,32 +208,6 @@ __device__ __forceinline__ void load_chunk(const float* __restrict__ X, int ld, 
         v[p] = x;
     }
 }
-// element (r, k) of a stage copy: float offset (k / 4) (LBO / 4) + (r / 8) 32 + (r % 8) 4 + k % 4
-template <bool KC>
-__device__ __forceinline__ void store_chunk(float* hi, float* lo, const float4 (&v)[4]) {
-#pragma unroll
-    for (int p = 0; p < 4; ++p) {
-        const int g = threadIdx.x + NT * p;
-        if (KC) {
-            const int r = g / 8, k4 = g % 8;
-            const int o = k4 * (LBO / 4) + (r >> 3) * 32 + (r & 7) * 4;
-            const float4 h = make_float4(tf32_hi(v[p].x), tf32_hi(v[p].y), tf32_hi(v[p].z), tf32_hi(v[p].w));
-            *reinterpret_cast<float4*>(hi + o) = h;
-            *reinterpret_cast<float4*>(lo + o) = make_float4(v[p].x - h.x, v[p].y - h.y, v[p].z - h.z, v[p].w - h.w);
-        } else {
-            const int r0 = 4 * (g / 32), k = g % 32;
-            const float e[4] = {v[p].x, v[p].y, v[p].z, v[p].w};
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-                const int r = r0 + q;
-                const int o = (k >> 2) * (LBO / 4) + (r >> 3) * 32 + (r & 7) * 4 + (k & 3);
-                const float h = tf32_hi(e[q]);
-                hi[o] = h;
-                lo[o] = e[q] - h;
-            }
-        }
-    }
-}
 
 template <bool TA, bool TB>
 __global__ void __launch_bounds__(NT, 1)
@@ -272,76 +217,41 @@ tc_sgemm(int M, int N, int K, const float* __restrict__ A, int lda, const float*
     __shared__ uint32_t tmem_base;
     __shared__ __align__(8) uint64_t mbar[2];
     float* sm = reinterpret_cast<float*>((reinterpret_cast<uintptr_t>(tsm) + 127) & ~uintptr_t(127));
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int m0 = blockIdx.y * BM, n0 = blockIdx.x * BN;
     const int kb = blockIdx.z * k_split, ke = min(K, kb + k_split);
     const int nch = (ke - kb + BKC - 1) / BKC;
-    if (warp == 0) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base)), "r"(BN));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-    }
-    if (tid == 32) {
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&mbar[0])));
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&mbar[1])));
-        asm volatile("fence.mbarrier_init.release.cluster;");
-    }
     float4 ra[4], rb[4];
     load_chunk<!TA>(A, lda, m0, M, kb, ke, ra);
     load_chunk<TB>(B, ldb, n0, N, kb, ke, rb);
-    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-    __syncthreads();
-    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    setup(&tmem_base, mbar);
     const uint32_t tmem = tmem_base;
     uint32_t phases = 0u;                          // bit st: parity of stage st's next completion
     for (int c = 0; c < nch; ++c) {
         const int st = c & 1;
         float* Ah = sm + st * STAGE_F;
-        float* Al = Ah + OP_F;
-        float* Bh = Al + OP_F;
-        float* Bl = Bh + OP_F;
         if (c >= 2) { mbar_wait(smem_u32(&mbar[st]), (phases >> st) & 1u); phases ^= 1u << st; }   // chunk c - 2 read it
-        store_chunk<!TA>(Ah, Al, ra);
-        store_chunk<TB>(Bh, Bl, rb);
+        store_chunk<!TA>(Ah, Ah + OP_F, ra);
+        store_chunk<TB>(Ah + 2 * OP_F, Ah + 3 * OP_F, rb);
         if (c + 1 < nch) {                        // next chunk's loads in flight during this chunk's MMAs
             load_chunk<!TA>(A, lda, m0, M, kb + (c + 1) * BKC, ke, ra);
             load_chunk<TB>(B, ldb, n0, N, kb + (c + 1) * BKC, ke, rb);
         }
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic smem writes -> tensor core
-        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-        __syncthreads();
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        if (tid == 0) {
-            const uint32_t a0 = smem_u32(Ah), al0 = smem_u32(Al), b0 = smem_u32(Bh), bl0 = smem_u32(Bl);
-#pragma unroll
-            for (int s = 0; s < BKC / 8; ++s) {
-                const uint32_t o = 2 * s * LBO;
-                mma(tmem, desc(a0 + o), desc(b0 + o), c > 0 || s > 0);
-                mma(tmem, desc(a0 + o), desc(bl0 + o), 1);
-                mma(tmem, desc(al0 + o), desc(b0 + o), 1);
-            }
-            asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
-                         ::"r"(smem_u32(&mbar[st])) : "memory");
-        }
+        issue_chunk(tmem, Ah, &mbar[st], c == 0);
     }
-    // the last commit covers every earlier MMA
-    if (nch > 0) {
+    if (nch > 0) {                                 // the last commit covers every earlier MMA
         const int st = (nch - 1) & 1;
         mbar_wait(smem_u32(&mbar[st]), (phases >> st) & 1u);
     }
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-    // epilogue: warp w reads TMEM lanes 32 (w & 3) .. (rows), columns 64 (w >> 2) .. +63
+    // epilogue: warp w holds rows 32 (w & 3) + lane, columns 64 (w >> 2) .. +63
     const int row = m0 + 32 * (warp & 3) + lane, cb = 64 * (warp >> 2);
     const bool split = gridDim.z > 1;
     const bool vec = (ldc & 3) == 0 && ((reinterpret_cast<uintptr_t>(C) & 15) == 0);
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
         uint32_t r[16];
-        const uint32_t ta = tmem + ((uint32_t)(32 * (warp & 3)) << 16) + cb + 16 * q;
-        asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-                     : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-                       "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
-                     : "r"(ta));
-        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+        load16(tmem, cb + 16 * q, r);
         if (nch == 0)
 #pragma unroll
             for (int j = 0; j < 16; ++j) r[j] = 0u;
@@ -371,9 +281,7 @@ tc_sgemm(int M, int N, int K, const float* __restrict__ A, int lda, const float*
             }
         }
     }
-    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-    __syncthreads();
-    if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(BN));
+    teardown(tmem);
 }
 
 template <bool TA, bool TB>

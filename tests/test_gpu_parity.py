@@ -405,10 +405,12 @@ def test_errors_are_loud():
         m.fwd_bwd(s, torch.zeros(8, 32, device="cuda"))
 
 
-@pytest.mark.parametrize("env", ["VPPS_LEAF_TC", "VPPS_DW_TC"])
+@pytest.mark.parametrize("env", ["VPPS_LEAF_TC", "VPPS_DW_ITEMS", "VPPS_DW_ITEMS+VPPS_DW_TC"])
 def test_tensor_core_variants_subprocess(env):
-    """The opt-in tensor-core leaf GEMM / gradient GEMM (tcgen05 kind::tf32, 3xTF32 split) on the dataflow
-    path against the oracle.  The switches are read once per process, so each runs in a child process."""
+    """The dataflow path's alternative kernels against the oracle: the opt-in tensor-core leaf GEMM, the
+    per-group FFMA2 gradient-GEMM items that overlap the slowest groups (VPPS_DW_ITEMS; the default is the
+    post-pass tensor-core GEMM of vpps_dwtc.cu) and their tcgen05 variant.  The switches are read once per
+    process, so each runs in a child process."""
     import os
     import subprocess
     import sys
@@ -416,8 +418,8 @@ def test_tensor_core_variants_subprocess(env):
     code = ("import sys; sys.path.insert(0, %r); sys.path.insert(0, %r); import test_gpu_parity as t; "
             "t.check('binary', 256, 256, 5, t._trees(3, 16, (5, 50), 4096, 5), 4096, cluster=16, dataflow=True); "
             "print('ok')" % (root, os.path.join(root, "tests")))
-    r = subprocess.run([sys.executable, "-c", code], env={**os.environ, env: "1"}, capture_output=True, text=True,
-                       timeout=600)
+    r = subprocess.run([sys.executable, "-c", code], env={**os.environ, **{e: "1" for e in env.split("+")}},
+                       capture_output=True, text=True, timeout=600)
     assert r.returncode == 0 and "ok" in r.stdout, r.stdout + r.stderr
 
 
