@@ -6,9 +6,9 @@
 //   p2  dU_fr  [H x H]   = Σ_int  g_fr h_rᵀ             A = pool[rec_k + 11H + m],      B = pool[rec_r(k) + n]
 //   p3  dW_iou [3H x E]  = Σ_leaf g x_tokᵀ              A = pool[rec_k + 5H + m],       B = inputs[tok_k E + n]
 //   p4  dX[tok_m] += g_leaf(m)ᵀ W_iou  [leaves x E]     A(m, k) = pool[rec_m + 5H + k], B(k, n) = W_iou[k E + n]
-// (operands gathered row by row through the node lists while they are staged; tc_common.cuh's 128 x 128
-// 3xTF32 tiles).  Work items = (product, 128 x 128 tile, K range); K is split so that the items of all
-// products fill one wave of persistent CTAs; partial tiles are added into grads / dX (cleared by the leaf
+// (operands gathered row by row through the node lists by cp.async into a raw ring two chunks deep, then
+// split into tc_common.cuh's 128 x 128 3xTF32 stages).  Work items = (product, 128 x 128 tile, K range); K is
+// split so that the items of all products fill one wave of persistent CTAs; partial tiles are added into grads / dX (cleared by the leaf
 // kernel) with red.global.add.v4.  Then, as in the FFMA2 gradient GEMM it replaces, the CTAs apply the SGD
 // update (L129, L197) once every item is counted, and one CTA copies the summed loss to mapped host memory.
 #include <algorithm>
@@ -51,67 +51,74 @@ struct Params {
     float* loss_dst;
 };
 
-// the row pointer of element (row r, k) of a K-contiguous operand, or of (k, row r) of a row-contiguous one
-struct Op {
-    const float* base;   // element address = base + (per-row or per-k offset) + (k or r)
-};
+// Staging: the operands are gathered node by node, so each chunk is first copied with 16-byte cp.async into
+// a raw shared-memory ring (two chunks ahead: no registers held across the L2 round trip) and then converted
+// into the canonical hi / lo stage of the tensor core.  Raw layouts: an operand contiguous along its rows
+// (every A but p4's, every B) as [32 k][RS] with RS = 132 (the conversion reads one k per lane: rows 132
+// floats apart hit distinct banks); p4's A (contiguous along k) as [128 rows][32 k].
+constexpr int RS = BM + 4;
+constexpr int RAW_F = BKC * RS;                 // floats of one raw operand chunk (>= 128 x 32)
+constexpr int KMAXI = 1024;                     // node offsets staged per item (host keeps K per item below)
+constexpr size_t SMEM_DW = tcc::SMEM + (size_t)2 * 2 * RAW_F * sizeof(float);
 
-__device__ __forceinline__ const float* a_ptr(const Params& P, int p, int r, int k) {
-    // A(m = r, k): p0..p3 row-contiguous in m for a fixed node k; p4 K-contiguous for a fixed leaf r
-    const int H = P.H;
-    switch (p) {
-        case 0: return P.pool + P.ints[3 * k] + 7 * H + r;
-        case 1: return P.pool + P.ints[3 * k] + 10 * H + r;
-        case 2: return P.pool + P.ints[3 * k] + 11 * H + r;
-        case 3: return P.pool + P.leaves[2 * k] + 5 * H + r;
-        default: return P.pool + P.leaves[2 * r] + 5 * H + k;
-    }
-}
-__device__ __forceinline__ const float* b_ptr(const Params& P, int p, int k, int n) {
-    // B(k, n): row-contiguous in n for a fixed k in every product
-    const int H = P.H;
-    switch (p) {
-        case 0: return n < H ? P.pool + P.ints[3 * k + 1] + n : P.pool + P.ints[3 * k + 2] + (n - H);
-        case 1: return P.pool + P.ints[3 * k + 1] + n;
-        case 2: return P.pool + P.ints[3 * k + 2] + n;
-        case 3: return P.inputs + (int64_t)P.leaves[2 * k + 1] * P.E + n;
-        default: return P.w_iou + (int64_t)k * P.E + n;
-    }
-}
-
-// stage loads of one chunk: A is K-contiguous only in p4; B is always row-contiguous (in n)
-__device__ __forceinline__ void load_a(const Params& P, int p, int m0, int M, int k0, int ke, float4 (&v)[4]) {
-    const bool kc = p == 4;
+// per-item operand offsets (floats, shared memory): element A(m, k) = abase + aoff[k] + m (p4: aoff[m] + k),
+// B(k, n) = bbase + boff[k] + n
+__device__ __forceinline__ void copy_chunk(const float* abase, const float* bbase, const uint32_t* aoff,
+                                           const uint32_t* boff, bool a_kc, int m0, int M, int n0, int N, int kc0,
+                                           int kb, int ke, float* rawA, float* rawB) {
+    const int tid = threadIdx.x;
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
-        int r, k;
-        piece_rk(kc, q, r, k);
-        const int gr = m0 + r, gk = k0 + k;
-        float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (kc) {
-            if (gr < M) {
-                const float* src = a_ptr(P, p, gr, gk);
-                if (gk + 3 < ke) x = __ldcg(reinterpret_cast<const float4*>(src));
-                else {
-                    if (gk < ke) x.x = __ldcg(src);
-                    if (gk + 1 < ke) x.y = __ldcg(src + 1);
-                    if (gk + 2 < ke) x.z = __ldcg(src + 2);
-                }
-            }
-        } else if (gk < ke && gr < M) {       // M is a multiple of 4 (3H, H)
-            x = __ldcg(reinterpret_cast<const float4*>(a_ptr(P, p, gr, gk)));
+        const int g = tid + NT * q;
+        if (a_kc) {                                    // [128 rows][32 k]: row g / 8, k 4 (g % 8)
+            const int r = g / 8, k = 4 * (g % 8), gr = m0 + r, gk = kc0 + k;
+            const bool ok = gr < M && gk < ke;
+            const float* src = ok ? abase + aoff[r] + gk : abase;
+            cp_async16(rawA + r * BKC + k, src, ok ? (gk + 3 < ke ? 16u : 4u * (ke - gk)) : 0u);
+        } else {                                       // [32 k][RS]: k g / 32, rows 4 (g % 32)
+            const int k = g / 32, r = 4 * (g % 32), gr = m0 + r, gk = kc0 + k;
+            const bool ok = gk < ke && gr < M;         // (M is a multiple of 4 here)
+            const float* src = ok ? abase + aoff[gk - kb] + gr : abase;
+            cp_async16(rawA + k * RS + r, src, ok ? 16u : 0u);
         }
-        v[q] = x;
+        {
+            const int k = g / 32, r = 4 * (g % 32), gn = n0 + r, gk = kc0 + k;
+            const bool ok = gk < ke && gn < N;
+            const float* src = ok ? bbase + boff[gk - kb] + gn : bbase;
+            cp_async16(rawB + k * RS + r, src, ok ? 16u : 0u);
+        }
     }
+    asm volatile("cp.async.commit_group;" ::: "memory");
 }
-__device__ __forceinline__ void load_b(const Params& P, int p, int n0, int N, int k0, int ke, float4 (&v)[4]) {
+
+// raw chunk -> canonical hi / lo copies (the layout of tc_common.cuh)
+__device__ __forceinline__ void convert_rows(const float* raw, float* hi, float* lo) {
+    // row-contiguous raw [32 k][RS]: lane = k, piece = rows 4 (g / 32) .. +3 (transposing 4-byte stores)
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
-        int r, k;
-        piece_rk(false, q, r, k);
-        const int gn = n0 + r, gk = k0 + k;
-        v[q] = (gk < ke && gn < N) ? __ldcg(reinterpret_cast<const float4*>(b_ptr(P, p, gk, gn)))
-                                   : make_float4(0.f, 0.f, 0.f, 0.f);
+        const int g = threadIdx.x + NT * q, k = g % 32, r0 = 4 * (g / 32);
+        const float4 v = *reinterpret_cast<const float4*>(raw + k * RS + r0);
+        const float e[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            const int r = r0 + t;
+            const int o = (k >> 2) * (LBO / 4) + (r >> 3) * 32 + (r & 7) * 4 + (k & 3);
+            const float h = tf32_hi(e[t]);
+            hi[o] = h;
+            lo[o] = e[t] - h;
+        }
+    }
+}
+__device__ __forceinline__ void convert_kc(const float* raw, float* hi, float* lo) {
+    // k-contiguous raw [128 rows][32 k]: piece = row g / 8, k 4 (g % 8) .. +3 (16-byte stores)
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        const int g = threadIdx.x + NT * q, r = g / 8, k4 = g % 8;
+        const float4 v = *reinterpret_cast<const float4*>(raw + r * BKC + 4 * k4);
+        const int o = k4 * (LBO / 4) + (r >> 3) * 32 + (r & 7) * 4;
+        const float4 h = make_float4(tf32_hi(v.x), tf32_hi(v.y), tf32_hi(v.z), tf32_hi(v.w));
+        *reinterpret_cast<float4*>(hi + o) = h;
+        *reinterpret_cast<float4*>(lo + o) = make_float4(v.x - h.x, v.y - h.y, v.z - h.z, v.w - h.w);
     }
 }
 
@@ -120,8 +127,11 @@ __global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
     __shared__ uint32_t tmem_base;
     __shared__ __align__(8) uint64_t mbar[2];
     __shared__ int pick;
-    float* sm = reinterpret_cast<float*>((reinterpret_cast<uintptr_t>(tsm) + 127) & ~uintptr_t(127));
+    __shared__ uint32_t aoff[KMAXI], boff[KMAXI];
+    float* canon = reinterpret_cast<float*>((reinterpret_cast<uintptr_t>(tsm) + 127) & ~uintptr_t(127));
+    float* raw = canon + 2 * STAGE_F;                 // 2 stages x (A, B)
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int H = P.H;
     setup(&tmem_base, mbar);
     const uint32_t tmem = tmem_base;
     uint32_t phases = 0u;
@@ -137,21 +147,49 @@ __global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
         const int kb = sp * P.ksplit[p], ke = min(P.K[p], kb + P.ksplit[p]);
         const int M = P.M[p], N = P.N[p];
         const int nch = (ke - kb + BKC - 1) / BKC;
-        float4 ra[4], rb[4];
-        load_a(P, p, m0, M, kb, ke, ra);
-        load_b(P, p, n0, N, kb, ke, rb);
+        const bool a_kc = p == 4;
+        // operand offsets of the item (node lists, PAPER L185's concatenated operands)
+        const float* abase = P.pool;
+        const float* bbase = p == 3 ? P.inputs : (p == 4 ? P.w_iou : P.pool);
+        if (a_kc) {
+            for (int r = tid; r < BM; r += NT) aoff[r] = m0 + r < M ? P.leaves[2 * (m0 + r)] + 5 * H : 0u;
+            for (int k = tid; k < ke - kb; k += NT) boff[k] = (uint32_t)(kb + k) * (uint32_t)P.E;
+        } else {
+            for (int k = tid; k < ke - kb; k += NT) {
+                const int node = kb + k;
+                if (p == 3) {
+                    aoff[k] = P.leaves[2 * node] + 5 * H;
+                    boff[k] = P.leaves[2 * node + 1] * (uint32_t)P.E;
+                } else {
+                    const uint32_t rec = P.ints[3 * node];
+                    aoff[k] = rec + (p == 0 ? 7 : (p == 1 ? 10 : 11)) * H;
+                    boff[k] = p == 1 || (p == 0 && n0 < H) ? P.ints[3 * node + 1]
+                                                           : P.ints[3 * node + 2] - (p == 0 ? H : 0);
+                }
+            }
+        }
+        __syncthreads();
+        // prologue: chunks 0 and 1 in flight
+        for (int c = 0; c < 2; ++c) {
+            if (c < nch)
+                copy_chunk(abase, bbase, aoff, boff, a_kc, m0, M, n0, N, kb + c * BKC, kb, ke, raw + c * 2 * RAW_F,
+                           raw + c * 2 * RAW_F + RAW_F);
+            else asm volatile("cp.async.commit_group;" ::: "memory");
+        }
         for (int c = 0; c < nch; ++c) {
             const int st = c & 1;
-            float* Ah = sm + st * STAGE_F;
+            float* rA = raw + st * 2 * RAW_F;
+            float* Ah = canon + st * STAGE_F;
+            asm volatile("cp.async.wait_group 1;" ::: "memory");      // this thread's copies of chunk c
+            __syncthreads();                                           // ... and everyone else's
             if (c >= 2) { mbar_wait(smem_u32(&mbar[st]), (phases >> st) & 1u); phases ^= 1u << st; }
-            if (p == 4) store_chunk<true>(Ah, Ah + OP_F, ra);
-            else store_chunk<false>(Ah, Ah + OP_F, ra);
-            store_chunk<false>(Ah + 2 * OP_F, Ah + 3 * OP_F, rb);
-            if (c + 1 < nch) {
-                load_a(P, p, m0, M, kb + (c + 1) * BKC, ke, ra);
-                load_b(P, p, n0, N, kb + (c + 1) * BKC, ke, rb);
-            }
-            issue_chunk(tmem, Ah, &mbar[st], c == 0);
+            if (a_kc) convert_kc(rA, Ah, Ah + OP_F);
+            else convert_rows(rA, Ah, Ah + OP_F);
+            convert_rows(rA + RAW_F, Ah + 2 * OP_F, Ah + 3 * OP_F);
+            issue_chunk(tmem, Ah, &mbar[st], c == 0);                 // (its barrier also frees raw stage st)
+            if (c + 2 < nch)
+                copy_chunk(abase, bbase, aoff, boff, a_kc, m0, M, n0, N, kb + (c + 2) * BKC, kb, ke, rA, rA + RAW_F);
+            else asm volatile("cp.async.commit_group;" ::: "memory");
         }
         // drain: the last commit covers every MMA of the item; both stages are then free for the next item
         if (nch > 0) {
@@ -167,22 +205,16 @@ __global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         if (nch > 0) {
             const int row = m0 + 32 * (warp & 3) + lane, cb = 64 * (warp >> 2);
-            float* out;
-            int ld;
-            if (p == 4) {
-                out = row < M ? P.d_inputs + (int64_t)P.leaves[2 * row + 1] * P.E : nullptr;
-                ld = 0;
-            } else {
-                out = P.grads + P.off[p == 3 ? 0 : p + 1] + (int64_t)row * N;
-                ld = N;
-            }
-            (void)ld;
+            float* out = nullptr;
+            if (row < M)
+                out = p == 4 ? P.d_inputs + (int64_t)P.leaves[2 * row + 1] * P.E
+                             : P.grads + P.off[p == 3 ? 0 : p + 1] + (int64_t)row * N;
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
                 uint32_t r[16];
                 load16(tmem, cb + 16 * q, r);
                 const int nb = n0 + cb + 16 * q;
-                if (row < M && out) {
+                if (out) {
 #pragma unroll
                     for (int j = 0; j < 16; j += 4)
                         if (nb + j < N) {     // N is a multiple of 4
@@ -193,7 +225,7 @@ __global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
                 }
             }
         }
-        // every thread's TMEM reads (and the item's reductions) precede the next item's first MMA
+        // every thread's TMEM reads (and the item's reductions) precede the next item's first MMA and the count
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         __syncthreads();
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
@@ -206,7 +238,7 @@ __global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
         while (true) {
             asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(f) : "l"(P.fin) : "memory");
             if ((int)f >= P.total) break;
-            __nanosleep(100);
+            __nanosleep(64);
         }
     }
     __syncthreads();
@@ -273,7 +305,7 @@ bool launch_dw_tc(const float* pool, const float* inputs, float* d_inputs, float
         chunks_total += P.tm[p] * P.tn[p] * ((Ks[p] + BKC - 1) / BKC);
     }
     // smallest chunks-per-item target whose items fit one wave
-    int target = std::max(1, (chunks_total + n_sm - 1) / n_sm);
+    int target = std::min(std::max(1, (chunks_total + n_sm - 1) / n_sm), KMAXI / BKC);
     while (true) {
         int items = 0;
         for (int p = 0; p < NP; ++p) {
@@ -281,7 +313,7 @@ bool launch_dw_tc(const float* pool, const float* inputs, float* d_inputs, float
             const int sp = P.tm[p] ? std::max(1, (ch + target - 1) / target) : 0;
             items += P.tm[p] * P.tn[p] * sp;
         }
-        if (items <= n_sm || target > 4096) break;
+        if ((items <= n_sm && target * BKC <= KMAXI) || target * BKC >= KMAXI) break;
         ++target;
     }
     P.first[0] = 0;
@@ -301,7 +333,7 @@ bool launch_dw_tc(const float* pool, const float* inputs, float* d_inputs, float
     int dev = 0;
     cudaGetDevice(&dev);
     if (!(attr_done.load() >> (dev & 63) & 1)) {
-        if (cudaFuncSetAttribute(vpps_dw_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dev::tcc::SMEM) != cudaSuccess)
+        if (cudaFuncSetAttribute(vpps_dw_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM_DW) != cudaSuccess)
             return false;
         attr_done.fetch_or(uint64_t(1) << (dev & 63));
     }
@@ -311,7 +343,7 @@ bool launch_dw_tc(const float* pool, const float* inputs, float* d_inputs, float
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.gridDim = dim3(std::max(1, std::min(P.total, n_sm)));
     cfg.blockDim = dim3(dev::tcc::NT);
-    cfg.dynamicSmemBytes = dev::tcc::SMEM;
+    cfg.dynamicSmemBytes = SMEM_DW;
     cfg.stream = s;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
