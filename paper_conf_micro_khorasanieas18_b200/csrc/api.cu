@@ -622,19 +622,19 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
             if (s->s.grp_levels[a] != s->s.grp_levels[b]) return s->s.grp_levels[a] < s->s.grp_levels[b];
             return s->s.grp_nodes[a] < s->s.grp_nodes[b];
         });
-        // weight gradients (L185) + leaf dX after the pass: tensor-core tiles over every node of the batch
-        // (vpps_dwtc.cu), SGD fused in their tail at N = 1; VPPS_DW_ITEMS=1 (measurement) keeps the FFMA2
-        // per-group items that overlap the slowest groups instead
+        // weight gradients (L185) + leaf dX per replica group as the groups finish: tensor-core tiles
+        // (vpps_dwtc.cu), SGD fused in their tail at N = 1; VPPS_DW_ITEMS=1 (measurement) runs the FFMA2
+        // per-group items instead
         static const bool dw_items = getenv("VPPS_DW_ITEMS") && atoi(getenv("VPPS_DW_ITEMS")) != 0;
         if (dw_items || m->gemm_trace) {
             launch_dw_gemm(m->pool, inputs, d_inputs, m->params, m->grads, lists, leaf_list, n_grp, s->s.int_off.data(),
                            s->s.leaf_off.data(), order.data(), m->done, m->cluster, true, m->plan.H, m->plan.E,
                            m->offsets.data(), m->n_floats, mode, lr, wd, st, m->gemm_trace,
                            m->pool + s->s.loss_word, m->d_loss_map + (m->passes & 1));
-        } else if (!launch_dw_tc(m->pool, inputs, d_inputs, m->params, m->grads, lists, leaf_list, (int32_t)s->s.n_int,
-                                 (int32_t)s->s.n_leaf, m->plan.H, m->plan.E, m->offsets.data(), m->n_floats,
-                                 m->done + 32, mode, lr, wd, st, m->pool + s->s.loss_word,
-                                 m->d_loss_map + (m->passes & 1), m->sms)) {
+        } else if (!launch_dw_tc(m->pool, inputs, d_inputs, m->params, m->grads, lists, leaf_list, n_grp,
+                                 s->s.int_off.data(), s->s.leaf_off.data(), order.data(), m->done, m->cluster,
+                                 m->plan.H, m->plan.E, m->offsets.data(), m->n_floats, mode, lr, wd, st,
+                                 m->pool + s->s.loss_word, m->d_loss_map + (m->passes & 1), m->sms)) {
             return fail(VPPS_E_CUDA, "gradient GEMM launch failed");
         }
         CK(cudaGetLastError());

@@ -1,16 +1,18 @@
 // Weight gradients of the binary Tree-LSTM's dataflow path on the tensor cores ("concatenate all
 // the left hand side and all the right hand side tensors that participate in the outer-product for each
-// weight matrix, and use dense matrix-matrix multiplication"), after vpps_df, over every node of the batch:
+// weight matrix, and use dense matrix-matrix multiplication"), per replica group as soon as the group's 16
+// vpps_df CTAs have counted themselves done (the work fills the SMs of finished groups while the slowest
+// group still runs; L185's one GEMM per matrix becomes one GEMM per matrix and group, summed in grads):
 //   p0  dU_iou [3H x 2H] = Σ_int  g_iou [h_l; h_r]ᵀ     A(m, k) = pool[rec_k + 7H + m], B(k, n) = h_l / h_r of k
 //   p1  dU_fl  [H x H]   = Σ_int  g_fl h_lᵀ             A = pool[rec_k + 10H + m],      B = pool[rec_l(k) + n]
 //   p2  dU_fr  [H x H]   = Σ_int  g_fr h_rᵀ             A = pool[rec_k + 11H + m],      B = pool[rec_r(k) + n]
 //   p3  dW_iou [3H x E]  = Σ_leaf g x_tokᵀ              A = pool[rec_k + 5H + m],       B = inputs[tok_k E + n]
 //   p4  dX[tok_m] += g_leaf(m)ᵀ W_iou  [leaves x E]     A(m, k) = pool[rec_m + 5H + k], B(k, n) = W_iou[k E + n]
-// (operands gathered row by row through the node lists by cp.async into a raw ring two chunks deep, then
-// split into tc_common.cuh's 128 x 128 3xTF32 stages).  Work items = (product, 128 x 128 tile, K range); K is
-// split so that the items of all products fill one wave of persistent CTAs; partial tiles are added into grads / dX (cleared by the leaf
-// kernel) with red.global.add.v4.  Then, as in the FFMA2 gradient GEMM it replaces, the CTAs apply the SGD
-// update (L129, L197) once every item is counted, and one CTA copies the summed loss to mapped host memory.
+// Operands are gathered row by row through the group's node lists by 16-byte cp.async into a raw ring two
+// chunks deep, then split into tc_common.cuh's 128 x 128 3xTF32 stages.  Work items = (group, product,
+// 128 x 128 tile, K range); persistent CTAs claim the items of finished groups; partial tiles are added into
+// grads / dX (cleared by the leaf kernel) with red.global.add.v4.  Once every item is counted the CTAs apply
+// the SGD update (L129, L197) and one CTA copies the summed loss to mapped host memory.
 #include <algorithm>
 #include <atomic>
 #include <cstdint>
@@ -27,18 +29,26 @@ using namespace tcc;
 
 constexpr int NP = 5;
 
+constexpr int MAXG = 16;
+
 struct Params {
     const float* pool;
     const float* inputs;
     const float* w_iou;
     float* grads;
     float* d_inputs;                 // dX or nullptr (p4 skipped)
-    const uint32_t* ints;            // n_int x (rec, rec_l, rec_r)
-    const uint32_t* leaves;          // n_leaf x (rec, token)
-    int32_t n_int, n_leaf, H, E;
+    const uint32_t* ints;            // n_int x (rec, rec_l, rec_r), grouped by replica group
+    const uint32_t* leaves;          // n_leaf x (rec, token), grouped by replica group
+    int32_t H, E;
     int64_t off[8];
-    int32_t tm[NP], tn[NP], splits[NP], ksplit[NP], K[NP], M[NP], N[NP];
-    int32_t first[NP + 1];           // item prefix over the products
+    int32_t ksplit[NP];              // K per item (p0-p3: whole group lists up to KMAXI; p4: slices of 3H)
+    int32_t n_grp;
+    int32_t grp[MAXG];               // groups in claiming order (expected to finish first go first)
+    int32_t int_off[MAXG + 1], leaf_off[MAXG + 1];
+    int32_t gfirst[MAXG][NP + 1];    // item prefix over the products of each group
+    const int32_t* done;             // per-group completion counters (vpps_df)
+    int32_t* claim;                  // per-group claim counters (zeroed per pass)
+    int32_t done_target;
     int32_t total;
     // tail
     int32_t* fin;
@@ -50,6 +60,18 @@ struct Params {
     const float* loss_src;
     float* loss_dst;
 };
+
+__host__ __device__ inline void product_shape(int p, int H, int E, int n_int, int n_leaf, bool dx, int& M, int& N,
+                                              int& K) {
+    switch (p) {
+        case 0: M = 3 * H; N = 2 * H; K = n_int; break;
+        case 1:
+        case 2: M = H; N = H; K = n_int; break;
+        case 3: M = 3 * H; N = E; K = n_leaf; break;
+        default: M = n_leaf; N = E; K = dx ? 3 * H : 0;
+    }
+    if (M <= 0 || K <= 0) M = K = 0;
+}
 
 // Staging: the operands are gathered node by node, so each chunk is first copied with 16-byte cp.async into
 // a raw shared-memory ring (two chunks ahead: no registers held across the L2 round trip) and then converted
@@ -126,7 +148,7 @@ __global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
     extern __shared__ __align__(128) float tsm[];
     __shared__ uint32_t tmem_base;
     __shared__ __align__(8) uint64_t mbar[2];
-    __shared__ int pick;
+    __shared__ int pick[3];
     __shared__ uint32_t aoff[KMAXI], boff[KMAXI];
     float* canon = reinterpret_cast<float*>((reinterpret_cast<uintptr_t>(tsm) + 127) & ~uintptr_t(127));
     float* raw = canon + 2 * STAGE_F;                 // 2 stages x (A, B)
@@ -135,36 +157,70 @@ __global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
     setup(&tmem_base, mbar);
     const uint32_t tmem = tmem_base;
     uint32_t phases = 0u;
-    // the records and node lists are complete once vpps_df (the primary grid) has finished
-    asm volatile("griddepcontrol.wait;" ::: "memory");
-    for (int it = blockIdx.x; it < P.total; it += gridDim.x) {
+    while (true) {
+        // claim an item of a group whose CTAs have all counted themselves done (lane q looks at group grp[q])
+        if (tid < 32) {
+            const int g = lane < P.n_grp ? P.grp[lane] : -1;
+            uint32_t c = 0, d = 0;
+            if (g >= 0) {
+                asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(c) : "l"(P.claim + g) : "memory");
+                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(d) : "l"(P.done + g) : "memory");
+            }
+            const int items = g >= 0 ? P.gfirst[g][NP] : 0;
+            const bool left = g >= 0 && (int)c < items;
+            unsigned ready = __ballot_sync(0xffffffffu, left && (int)d >= P.done_target);
+            int got_g = -1, got_i = -1;
+            while (ready && got_g < 0) {
+                const int q = __ffs(ready) - 1;
+                int i = 0;
+                if (lane == q) i = atomicAdd(P.claim + g, 1);
+                i = __shfl_sync(0xffffffffu, i, q);
+                const int gq = __shfl_sync(0xffffffffu, g, q);
+                if (i < P.gfirst[gq][NP]) { got_g = gq; got_i = i; }
+                ready &= ready - 1;
+            }
+            const unsigned any_left = __ballot_sync(0xffffffffu, left);
+            if (lane == 0) { pick[0] = got_g; pick[1] = got_i; pick[2] = any_left != 0; }
+        }
+        __syncthreads();
+        const int g = pick[0], it = pick[1], rem = pick[2];
+        __syncthreads();
+        if (g < 0) {
+            if (!rem) break;
+            __nanosleep(256);
+            continue;
+        }
+        const int n_int = P.int_off[g + 1] - P.int_off[g], n_leaf = P.leaf_off[g + 1] - P.leaf_off[g];
+        const uint32_t* ints = P.ints + 3 * P.int_off[g];
+        const uint32_t* leaves = P.leaves + 2 * P.leaf_off[g];
         int p = 0;
-        while (it >= P.first[p + 1]) ++p;
-        const int local = it - P.first[p];
-        const int per_split = P.tm[p] * P.tn[p];
+        while (it >= P.gfirst[g][p + 1]) ++p;
+        int M, N, K;
+        product_shape(p, H, P.E, n_int, n_leaf, P.d_inputs != nullptr, M, N, K);
+        const int local = it - P.gfirst[g][p];
+        const int tn = (N + BN - 1) / BN, per_split = ((M + BM - 1) / BM) * tn;
         const int sp = local / per_split, t = local - sp * per_split;
-        const int m0 = (t / P.tn[p]) * BM, n0 = (t % P.tn[p]) * BN;
-        const int kb = sp * P.ksplit[p], ke = min(P.K[p], kb + P.ksplit[p]);
-        const int M = P.M[p], N = P.N[p];
+        const int m0 = (t / tn) * BM, n0 = (t % tn) * BN;
+        const int kb = sp * P.ksplit[p], ke = min(K, kb + P.ksplit[p]);
         const int nch = (ke - kb + BKC - 1) / BKC;
         const bool a_kc = p == 4;
         // operand offsets of the item (node lists, PAPER L185's concatenated operands)
         const float* abase = P.pool;
         const float* bbase = p == 3 ? P.inputs : (p == 4 ? P.w_iou : P.pool);
         if (a_kc) {
-            for (int r = tid; r < BM; r += NT) aoff[r] = m0 + r < M ? P.leaves[2 * (m0 + r)] + 5 * H : 0u;
+            for (int r = tid; r < BM; r += NT) aoff[r] = m0 + r < M ? leaves[2 * (m0 + r)] + 5 * H : 0u;
             for (int k = tid; k < ke - kb; k += NT) boff[k] = (uint32_t)(kb + k) * (uint32_t)P.E;
         } else {
             for (int k = tid; k < ke - kb; k += NT) {
                 const int node = kb + k;
                 if (p == 3) {
-                    aoff[k] = P.leaves[2 * node] + 5 * H;
-                    boff[k] = P.leaves[2 * node + 1] * (uint32_t)P.E;
+                    aoff[k] = leaves[2 * node] + 5 * H;
+                    boff[k] = leaves[2 * node + 1] * (uint32_t)P.E;
                 } else {
-                    const uint32_t rec = P.ints[3 * node];
+                    const uint32_t rec = ints[3 * node];
                     aoff[k] = rec + (p == 0 ? 7 : (p == 1 ? 10 : 11)) * H;
-                    boff[k] = p == 1 || (p == 0 && n0 < H) ? P.ints[3 * node + 1]
-                                                           : P.ints[3 * node + 2] - (p == 0 ? H : 0);
+                    boff[k] = p == 1 || (p == 0 && n0 < H) ? ints[3 * node + 1]
+                                                           : ints[3 * node + 2] - (p == 0 ? H : 0);
                 }
             }
         }
@@ -207,7 +263,7 @@ __global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
             const int row = m0 + 32 * (warp & 3) + lane, cb = 64 * (warp >> 2);
             float* out = nullptr;
             if (row < M)
-                out = p == 4 ? P.d_inputs + (int64_t)P.leaves[2 * row + 1] * P.E
+                out = p == 4 ? P.d_inputs + (int64_t)leaves[2 * row + 1] * P.E
                              : P.grads + P.off[p == 3 ? 0 : p + 1] + (int64_t)row * N;
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
@@ -246,9 +302,9 @@ __global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
     constexpr int64_t CH = 4 * CV * NT;
     const int64_t n_chunks = P.mode == 1 ? (P.n_floats + CH - 1) / CH : 0;
     while (true) {
-        if (tid == 0) pick = atomicAdd(P.tail_claim, 1);
+        if (tid == 0) pick[0] = atomicAdd(P.tail_claim, 1);
         __syncthreads();
-        const int64_t c = pick;
+        const int64_t c = pick[0];
         __syncthreads();
         if (c == 0 && P.loss_dst && tid == 0) {
             const float l = *reinterpret_cast<const volatile float*>(P.loss_src);
@@ -279,54 +335,44 @@ __global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
 }  // namespace dwtc
 }  // namespace dev
 
-// Host: products, tiles and K splits so that the items fill about one wave of 148 persistent CTAs.
+// Host: per group and product the 128 x 128 tiles and K slices (p0-p3 take the group's whole node list up to
+// KMAXI nodes per item; the leaf dX's K = 3H runs in slices of 192), groups in the claiming order.
 bool launch_dw_tc(const float* pool, const float* inputs, float* d_inputs, float* params, float* grads,
-                  const uint32_t* ints, const uint32_t* leaves, int32_t n_int, int32_t n_leaf, int32_t H, int32_t E,
-                  const int64_t* off, int64_t n_floats, int32_t* counters, int32_t mode, float lr, float wd,
-                  cudaStream_t s, const float* loss_src, float* loss_dst, int32_t n_sm) {
+                  const uint32_t* ints, const uint32_t* leaves, int32_t n_grp, const int32_t* int_off,
+                  const int32_t* leaf_off, const int32_t* order, int32_t* done, int32_t done_target, int32_t H,
+                  int32_t E, const int64_t* off, int64_t n_floats, int32_t mode, float lr, float wd, cudaStream_t s,
+                  const float* loss_src, float* loss_dst, int32_t n_sm) {
     using namespace dev::dwtc;
     using dev::tcc::BM;
     using dev::tcc::BN;
-    using dev::tcc::BKC;
-    if ((H % 4) || (E % 4) || (n_floats % 4)) return false;
+    if ((H % 4) || (E % 4) || (n_floats % 4) || n_grp > MAXG || !done) return false;
     Params P{};
     P.pool = pool; P.inputs = inputs; P.w_iou = params + off[0]; P.grads = grads; P.d_inputs = d_inputs;
-    P.ints = ints; P.leaves = leaves; P.n_int = n_int; P.n_leaf = n_leaf; P.H = H; P.E = E;
+    P.ints = ints; P.leaves = leaves; P.H = H; P.E = E;
     for (int i = 0; i < 8; ++i) P.off[i] = off[i];
-    const int Ms[NP] = {3 * H, H, H, 3 * H, n_leaf};
-    const int Ns[NP] = {2 * H, H, H, E, E};
-    const int Ks[NP] = {n_int, n_int, n_int, n_leaf, d_inputs ? 3 * H : 0};
-    int chunks_total = 0;
-    for (int p = 0; p < NP; ++p) {
-        P.M[p] = Ms[p]; P.N[p] = Ns[p]; P.K[p] = Ks[p];
-        P.tm[p] = (Ms[p] + BM - 1) / BM;
-        P.tn[p] = (Ns[p] + BN - 1) / BN;
-        if (Ms[p] <= 0 || Ks[p] <= 0) P.tm[p] = 0;
-        chunks_total += P.tm[p] * P.tn[p] * ((Ks[p] + BKC - 1) / BKC);
-    }
-    // smallest chunks-per-item target whose items fit one wave
-    int target = std::min(std::max(1, (chunks_total + n_sm - 1) / n_sm), KMAXI / BKC);
-    while (true) {
-        int items = 0;
+    for (int p = 0; p < NP; ++p) P.ksplit[p] = p == 4 ? 192 : KMAXI;
+    P.n_grp = n_grp;
+    int total = 0;
+    for (int q = 0; q <= n_grp; ++q) { P.int_off[q] = int_off[q]; P.leaf_off[q] = leaf_off[q]; }
+    for (int q = 0; q < n_grp; ++q) {
+        const int g = order ? order[q] : q;
+        P.grp[q] = g;
+        const int ni = int_off[g + 1] - int_off[g], nl = leaf_off[g + 1] - leaf_off[g];
+        P.gfirst[g][0] = 0;
         for (int p = 0; p < NP; ++p) {
-            const int ch = (Ks[p] + BKC - 1) / BKC;
-            const int sp = P.tm[p] ? std::max(1, (ch + target - 1) / target) : 0;
-            items += P.tm[p] * P.tn[p] * sp;
+            int M, N, K;
+            product_shape(p, H, E, ni, nl, d_inputs != nullptr, M, N, K);
+            const int items = M ? ((M + BM - 1) / BM) * ((N + BN - 1) / BN) * ((K + P.ksplit[p] - 1) / P.ksplit[p]) : 0;
+            P.gfirst[g][p + 1] = P.gfirst[g][p] + items;
         }
-        if ((items <= n_sm && target * BKC <= KMAXI) || target * BKC >= KMAXI) break;
-        ++target;
+        total += P.gfirst[g][NP];
     }
-    P.first[0] = 0;
-    for (int p = 0; p < NP; ++p) {
-        const int ch = (Ks[p] + BKC - 1) / BKC;
-        int sp = P.tm[p] ? std::max(1, (ch + target - 1) / target) : 0;
-        P.ksplit[p] = sp ? ((ch + sp - 1) / sp) * BKC : 0;
-        P.splits[p] = sp ? (Ks[p] + P.ksplit[p] - 1) / P.ksplit[p] : 0;
-        P.first[p + 1] = P.first[p] + P.tm[p] * P.tn[p] * P.splits[p];
-    }
-    P.total = P.first[NP];
-    P.fin = counters;
-    P.tail_claim = counters + 1;
+    P.total = total;
+    P.done = done;
+    P.claim = done + 16;
+    P.fin = done + 32;
+    P.tail_claim = done + 33;
+    P.done_target = done_target;
     P.mode = mode; P.params = params; P.n_floats = n_floats; P.lr = lr; P.wd = wd;
     P.loss_src = loss_src; P.loss_dst = loss_dst;
     static std::atomic<uint64_t> attr_done{0};
@@ -337,11 +383,14 @@ bool launch_dw_tc(const float* pool, const float* inputs, float* d_inputs, float
             return false;
         attr_done.fetch_or(uint64_t(1) << (dev & 63));
     }
+    // persistent, one CTA per SM, programmatic dependent of vpps_df: CTAs become resident on the SMs the
+    // finished groups release and claim those groups' items (no griddepcontrol.wait: the per-group counters
+    // order the reads of each group's records)
     cudaLaunchConfig_t cfg = {};
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     attr[0].val.programmaticStreamSerializationAllowed = 1;
-    cfg.gridDim = dim3(std::max(1, std::min(P.total, n_sm)));
+    cfg.gridDim = dim3(std::max(1, std::min(total, n_sm)));
     cfg.blockDim = dim3(dev::tcc::NT);
     cfg.dynamicSmemBytes = SMEM_DW;
     cfg.stream = s;

@@ -82,13 +82,15 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, flo
                     bool early, int32_t H, int32_t E, const int64_t* off, int64_t n_floats, int32_t mode, float lr,
                     float wd, cudaStream_t s, uint64_t* trace = nullptr, const float* loss_src = nullptr,
                     float* loss_dst = nullptr);
-// The dataflow path's weight gradients after vpps_df on the tensor cores (vpps_dwtc.cu): dU_iou, dU_fl,
-// dU_fr, dW_iou over every node and the leaf dX, 128 x 128 3xTF32 tiles with K split to one wave of `n_sm`
-// persistent CTAs, SGD (mode 1) and the loss copy in the tail; counters[0..1] zeroed per pass.
+// The dataflow path's weight gradients on the tensor cores (vpps_dwtc.cu): dU_iou, dU_fl, dU_fr, dW_iou and
+// the leaf dX per replica group, claimed by persistent CTAs once done[group] >= done_target (programmatic
+// dependent of vpps_df), 128 x 128 3xTF32 tiles; SGD (mode 1) and the loss copy in the tail.  Counters as for
+// launch_dw_gemm (done, claim = done + 16, fin / tail = done + 32 / 33; zeroed per pass).
 bool launch_dw_tc(const float* pool, const float* inputs, float* d_inputs, float* params, float* grads,
-                  const uint32_t* ints, const uint32_t* leaves, int32_t n_int, int32_t n_leaf, int32_t H, int32_t E,
-                  const int64_t* off, int64_t n_floats, int32_t* counters, int32_t mode, float lr, float wd,
-                  cudaStream_t s, const float* loss_src, float* loss_dst, int32_t n_sm);
+                  const uint32_t* ints, const uint32_t* leaves, int32_t n_grp, const int32_t* int_off,
+                  const int32_t* leaf_off, const int32_t* order, int32_t* done, int32_t done_target, int32_t H,
+                  int32_t E, const int64_t* off, int64_t n_floats, int32_t mode, float lr, float wd, cudaStream_t s,
+                  const float* loss_src, float* loss_dst, int32_t n_sm);
 // (with completion counters the kernel also applies the SGD update and copies *loss_src to loss_dst, a
 //  device-visible pointer to mapped host memory, after the last item; otherwise separate launches do)
 // Leaf level of the binary cell as one GEMM + fused cell (vpps_leaf.cu): records h, c, i, o, u of every
