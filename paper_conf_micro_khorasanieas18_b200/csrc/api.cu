@@ -622,11 +622,13 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
             if (s->s.grp_levels[a] != s->s.grp_levels[b]) return s->s.grp_levels[a] < s->s.grp_levels[b];
             return s->s.grp_nodes[a] < s->s.grp_nodes[b];
         });
-        // weight gradients (L185) + leaf dX per replica group as the groups finish: tensor-core tiles
-        // (vpps_dwtc.cu), SGD fused in their tail at N = 1; VPPS_DW_ITEMS=1 (measurement) runs the FFMA2
-        // per-group items instead
-        static const bool dw_items = getenv("VPPS_DW_ITEMS") && atoi(getenv("VPPS_DW_ITEMS")) != 0;
-        if (dw_items || m->gemm_trace) {
+        // weight gradients (L185) + leaf dX per replica group as the groups finish, SGD fused in the tail at
+        // N = 1: FFMA2 items (vpps_cluster.cu, 3 CTAs per SM).  VPPS_DW_TC2=1 (measurement) runs the
+        // tensor-core items of vpps_dwtc.cu instead: parity-green but slower (tail 33 vs 17 us per TGT step;
+        // a group's items have K <= ~50 nodes, so each 128 x 128 tile is two chunks of 3xTF32 MMAs behind a
+        // fixed staging / drain / reduction cost, at one CTA per SM)
+        static const bool dw_tc2 = getenv("VPPS_DW_TC2") && atoi(getenv("VPPS_DW_TC2")) != 0;
+        if (!dw_tc2 || m->gemm_trace) {
             launch_dw_gemm(m->pool, inputs, d_inputs, m->params, m->grads, lists, leaf_list, n_grp, s->s.int_off.data(),
                            s->s.leaf_off.data(), order.data(), m->done, m->cluster, true, m->plan.H, m->plan.E,
                            m->offsets.data(), m->n_floats, mode, lr, wd, st, m->gemm_trace,

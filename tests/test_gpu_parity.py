@@ -405,12 +405,11 @@ def test_errors_are_loud():
         m.fwd_bwd(s, torch.zeros(8, 32, device="cuda"))
 
 
-@pytest.mark.parametrize("env", ["VPPS_LEAF_TC", "VPPS_DW_ITEMS", "VPPS_DW_ITEMS+VPPS_DW_TC"])
+@pytest.mark.parametrize("env", ["VPPS_LEAF_TC", "VPPS_DW_TC", "VPPS_DW_TC2"])
 def test_tensor_core_variants_subprocess(env):
-    """The dataflow path's alternative kernels against the oracle: the opt-in tensor-core leaf GEMM, the
-    per-group FFMA2 gradient-GEMM items that overlap the slowest groups (VPPS_DW_ITEMS; the default is the
-    post-pass tensor-core GEMM of vpps_dwtc.cu) and their tcgen05 variant.  The switches are read once per
-    process, so each runs in a child process."""
+    """The dataflow path's opt-in kernels against the oracle: the tensor-core leaf GEMM, the tcgen05 variant
+    of the per-group gradient-GEMM items (VPPS_DW_TC) and the gathered 128 x 128 tensor-core gradient GEMM
+    of vpps_dwtc.cu (VPPS_DW_TC2).  The switches are read once per process, so each runs in a child process."""
     import os
     import subprocess
     import sys
