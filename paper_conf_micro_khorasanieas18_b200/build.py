@@ -19,7 +19,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
          "--expt-relaxed-constexpr", "-I", os.path.join(ROOT, "include")]
 FLAGS += os.environ.get("VPPS_NVCC_EXTRA", "").split()     # measurement-only experiments
-SOURCES = ["host/plan.cpp", "host/script.cpp", "host/tagger.cpp", "kernels/vpps_kernel.cu", "kernels/vpps_cluster.cu", "kernels/vpps_leaf.cu", "kernels/vpps_dataflow.cu", "kernels/vpps_level.cu", "kernels/vpps_gemm.cu", "kernels/vpps_dwtc.cu", "api.cu"]
+SOURCES = ["host/plan.cpp", "host/script.cpp", "host/tagger.cpp", "kernels/vpps_kernel.cu", "kernels/vpps_cluster.cu", "kernels/vpps_leaf.cu", "kernels/vpps_dataflow.cu", "kernels/vpps_level.cu", "kernels/vpps_gemm.cu", "kernels/vpps_dwtc.cu", "kernels/vpps_chain.cu", "api.cu"]
 HEADERS = ["host/host.h", "kernels/vpps_kernel.cuh", "kernels/dev_common.cuh", "kernels/tc_common.cuh"]
 
 

@@ -168,12 +168,23 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
         }
         m->plan.mlp = cell == CELL_BILSTM ? Mw : 0;
         m->plan.level = true;
+        int32_t sms = 148;
         if (!m->plan_only) {
             m->device = o.device;
             CK(cudaSetDevice(o.device));
             cudaDeviceProp prop;
             CK(cudaGetDeviceProperties(&prop, o.device));
             if (prop.major != 10) return fail(VPPS_E_INVALID, "libvpps is built for sm_100a (B200) only");
+            sms = prop.multiProcessorCount;
+        }
+        // LSTM chains: the recurrence runs register-resident in groups of co-resident CTAs (vpps_chain.cu)
+        // when a specialisation exists for H; VPPS_CHAIN=0 (measurement) keeps the per-step products
+        static const bool chain_env = !(getenv("VPPS_CHAIN") && atoi(getenv("VPPS_CHAIN")) == 0);
+        if ((cell == CELL_BILSTM || cell == CELL_LSTM) && chain_env) {
+            const int32_t ncl = chain_group_ctas(H), dirs = cell == CELL_BILSTM ? 2 : 1;
+            m->plan.chain_g = ncl > 0 ? (sms / ncl) / dirs : 0;
+        }
+        if (!m->plan_only) {
             m->level = level_ctx_create(&m->alloc);
             if (!m->level) return fail(VPPS_E_CUDA, "level-path context initialisation failed");
             CK(cudaMallocHost(&m->h_loss, 2 * sizeof(float)));
@@ -389,6 +400,7 @@ vpps_status vpps_build_script(vpps_model m, const vpps_batch* batch, vpps_script
             s->s.tg_fpos = t.tg_fpos + shift;
             s->s.tg_bpos = t.tg_bpos + shift;
             s->s.tg_start = t.tg_start;
+            s->s.tg_chain = t.tg_chain >= 0 ? t.tg_chain + shift : -1;
         }
     } else {
         rc = chains ? build_tagger_script(m->plan, b, INT64_MAX, &s->s, &err)
@@ -661,7 +673,8 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         const int rc = tagger_pass(m->level, m->params, off10, m->grads, m->pool, inputs, d_inputs, dwords,
                                    s->s.tg_tok, s->s.tg_lab, s->s.tg_fpos, s->s.tg_bpos, s->s.tg_start.data(),
                                    (int32_t)s->s.tg_start.size() - 1, s->s.tg_T, m->plan.H, m->plan.E, m->plan.C,
-                                   bi ? m->plan.mlp : 0, bi ? 2 : 1, s->s.loss_word, st);
+                                   bi ? m->plan.mlp : 0, bi ? 2 : 1, s->s.loss_word, st,
+                                   s->s.tg_chain >= 0 ? dwords + s->s.tg_chain : nullptr, m->plan.chain_g);
         if (rc != 0) return fail(VPPS_E_CUDA, "tagger pass failed (code " + std::to_string(rc) + ")");
         if (mode == 1) launch_sgd(m->params, m->grads, m->n_floats, lr, wd, st);
     } else if (m->plan.level) {

@@ -36,6 +36,8 @@ struct Plan {
     int32_t n_cta, n_g, n_act, umax, G;
     bool by_graph = false;   // SPEC S5g: whole graphs assigned to groups (cluster replicas)
     bool level = false;      // level-synchronous GEMM path (binary cell, weights L2-resident)
+    int32_t chain_g = 0;     // chain cells on the level path: groups per direction of the register-resident
+                             // recurrence (vpps_chain.cu); 0 = per-step products
     bool skip_words = false; // dataflow models: the SPEC words (S4-S6, §E) are not built with the device
                              // lowering (its kernels never read them); vpps_script_words builds them on demand
     std::vector<int32_t> table;   // rows of 8 int32
@@ -82,6 +84,7 @@ struct Script {
     // tok[T], lab[T], the forward step lists fpos[T] (positions of step t: sentences longer than t, in
     // batch order, starting at fstart[t]) and the backward step lists bpos[T] (position len-1-t)
     int64_t tg_T = 0, tg_tok = -1, tg_lab = -1, tg_fpos = -1, tg_bpos = -1;
+    int64_t tg_chain = -1;           // blob offset of the chain-recurrence sentence table (SPEC §L), or -1
     std::vector<int32_t> tg_start;   // [maxlen + 1]
 };
 

@@ -60,6 +60,35 @@ int build_tagger_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows
     for (int32_t t = 0; t < maxlen; ++t)
         for (int32_t g : order)
             if (len[g] > t) s.blob.push_back((uint32_t)(off[g] + len[g] - 1 - t));
+    // sentence table of the register-resident recurrence (SPEC §L; vpps_chain.cu): sentences longest first,
+    // each to the group (per direction) with the smallest total length so far (ties: lowest group), at most
+    // 64 per group; [G, pre_0 .. pre_G, (off, len) per sentence], direction 1's groups repeat direction 0's
+    s.tg_chain = -1;
+    if (plan.chain_g > 0 && T > 0) {
+        const int32_t Gd = plan.chain_g, dirs = plan.cell == CELL_BILSTM ? 2 : 1;
+        std::vector<std::vector<int32_t>> mem(Gd);
+        std::vector<int64_t> load(Gd, 0);
+        bool fits = true;
+        for (int32_t g : order) {
+            if (len[g] == 0) continue;
+            int32_t best = -1;
+            for (int32_t q = 0; q < Gd; ++q)
+                if ((int32_t)mem[q].size() < 64 && (best < 0 || load[q] < load[best])) best = q;
+            if (best < 0) { fits = false; break; }
+            mem[best].push_back(g);
+            load[best] += len[g];
+        }
+        if (fits) {
+            s.tg_chain = (int64_t)s.blob.size();
+            const int32_t G = Gd * dirs;
+            s.blob.push_back((uint32_t)G);
+            uint32_t run = 0;
+            s.blob.push_back(0);
+            for (int32_t q = 0; q < G; ++q) { run += (uint32_t)mem[q % Gd].size(); s.blob.push_back(run); }
+            for (int32_t q = 0; q < G; ++q)
+                for (int32_t g : mem[q % Gd]) { s.blob.push_back((uint32_t)off[g]); s.blob.push_back((uint32_t)len[g]); }
+        }
+    }
     // pool: the loss word only (the tagger's activations live in the path's work buffers)
     s.loss_word = 0;
     s.zero_words = 32;

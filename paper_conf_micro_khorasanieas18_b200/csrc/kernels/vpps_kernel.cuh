@@ -108,6 +108,25 @@ void launch_sgd(float* p, const float* g, int64_t n, float lr, float wd, cudaStr
 // Dense FP32 product of the level paths (vpps_gemm.cu): row-major C = op(A) op(B) + beta C (beta 0 or 1).
 cudaError_t gemm_f32(cudaStream_t s, bool ta, bool tb, int M, int N, int K, const float* A, int lda, const float* B,
                      int ldb, float* C, int ldc, float beta);
+// Register-resident recurrence of LSTM chains (vpps_chain.cu): groups of chain_group_ctas(H) co-resident
+// CTAs hold U, whole sentences per group, epoch-tagged slots between the steps.  table (device): [G,
+// pre_0 .. pre_G, (off, len) per sentence]; groups [0, groups_dir0) run direction 0, the rest direction 1.
+struct ChainParams {
+    const uint32_t* table;
+    int32_t groups_dir0;
+    int32_t HW;                      // row stride of HH / dHH (H, or 2H for the tagger)
+    uint32_t epoch;                  // tag of this pass's slots (never 0)
+    const float *U0, *U1, *b0, *b1;  // recurrent matrices and biases of the two directions
+    const float *P0, *P1;            // input projections W x [T][4H] (bias not included)
+    float* HH;                       // h [T][HW] (direction d at column d H)
+    float *C0, *C1, *G0, *G1;        // c [T][H], gates (i, f, o, g) [T][4H] per direction
+    const float* dHH;                // the head's dh [T][HW]
+    float *Gam0, *Gam1;              // γ [T][4H] per direction (left operands of the weight gradients)
+    unsigned long long* hx;          // [T][H] tagged h slots
+    unsigned long long* part;        // [T][NCL][NCL][UM] tagged Uᵀγ parts
+};
+int32_t chain_group_ctas(int32_t H);
+cudaError_t launch_chain(const ChainParams& P, int32_t H, int32_t n_groups, bool backward, cudaStream_t s);
 // Level-synchronous path (vpps_level.cu): context (cuBLAS handle + work buffers) and one training pass.
 void* level_ctx_create(const DevAlloc* alloc);
 void level_ctx_destroy(void* ctx);
@@ -126,7 +145,8 @@ int tdrnn_pass(void* ctx, const float* params, const int64_t* off, float* grads,
 int tagger_pass(void* ctx, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
                 float* d_inputs, const uint32_t* d_blob, int64_t tg_tok, int64_t tg_lab, int64_t tg_fpos,
                 int64_t tg_bpos, const int32_t* start, int32_t maxlen, int64_t T, int32_t H, int32_t E, int32_t C,
-                int32_t Mw, int32_t dirs, int64_t loss_word, cudaStream_t s);
+                int32_t Mw, int32_t dirs, int64_t loss_word, cudaStream_t s, const uint32_t* chain_table = nullptr,
+                int32_t chain_g = 0);
 int gru_pass(void* ctx, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
              float* d_inputs, const uint32_t* d_blob, int64_t tg_tok, int64_t tg_lab, int64_t tg_fpos,
              const int32_t* start, int32_t maxlen, int64_t T, int32_t H, int32_t E, int32_t C, int64_t loss_word,

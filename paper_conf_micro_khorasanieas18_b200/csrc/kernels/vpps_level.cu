@@ -514,6 +514,10 @@ struct LevelCtx {
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     LevelBufs b;
     TaggerBufs tg;
+    // register-resident chain recurrence (vpps_chain.cu): tagged slots, zeroed when (re)allocated; pass tag
+    float *hx = nullptr, *part = nullptr;
+    int64_t cap_hx = 0, cap_part = 0;
+    uint32_t epoch = 0;
     int64_t cap_X_leaf = 0, cap_X_int = 0, cap_Z = 0, cap_G_int = 0, cap_G_leaf = 0, cap_DX = 0;
 };
 
@@ -542,6 +546,8 @@ void level_ctx_destroy(void* p) {
                       t.dHb, t.dCf, t.dCb, t.Gamf, t.Gamb, t.Gs, t.Dh, t.DX, t.Hp2, t.Zs2, t.Gs2, t.Dh2,
                       t.HS0, t.HS1, t.DhB0, t.DhB1, t.EzB};
     for (float* q : tbufs) c->alloc.put(q, nullptr);
+    c->alloc.put(c->hx, nullptr);
+    c->alloc.put(c->part, nullptr);
     delete c;
 }
 
@@ -633,7 +639,8 @@ int level_pass(void* ctx_, const float* params, const int64_t* off, float* grads
 int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
                 float* d_inputs, const uint32_t* d_blob, int64_t tg_tok, int64_t tg_lab, int64_t tg_fpos,
                 int64_t tg_bpos, const int32_t* start, int32_t maxlen, int64_t T, int32_t H, int32_t E, int32_t C,
-                int32_t Mw, int32_t dirs, int64_t loss_word, cudaStream_t s) {
+                int32_t Mw, int32_t dirs, int64_t loss_word, cudaStream_t s, const uint32_t* chain_table,
+                int32_t chain_g) {
     // off: parameter offsets (Wf, Uf, Wb, Ub, W_mlp, W_tag, bf, bb, b_mlp, b_tag); dirs = 1 is the LSTM LM
     // (M1: W, U, -, -, -, W_out, b, -, -, b_out; the head reads h directly), Mw = 0 without the MLP
     using namespace dev::lv;
@@ -674,13 +681,45 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
     tg_gather_x<<<nblk(T * (E / 4)), 256, 0, s>>>(inputs, tok, (int)T, E, tb.X);
     BL(gemm_rm(c->st, false, true, (int)T, 4 * H, E, tb.X, E, Wf, E, tb.Pf, 4 * H, 0.f));
     if (dirs > 1) BL(gemm_rm(c->st, false, true, (int)T, 4 * H, E, tb.X, E, Wb, E, tb.Pb, 4 * H, 0.f));
+    // register-resident recurrence (vpps_chain.cu): U of each direction in the registers of a group of CTAs,
+    // whole sentences per group, tagged slots between the steps — one launch for the forward steps of both
+    // directions, one for the backward steps (instead of a product and a cell launch per step)
+    ChainParams cp{};
+    const int32_t ncl = chain_table ? chain_group_ctas(H) : 0;
+    const bool chain = ncl > 0 && chain_g > 0;
+    if (chain) {
+        // slots: HX [T][H] and PART [T][NCL][H] 64-bit words, never cleared again (epoch tags)
+        const int64_t need_hx = 2 * T * H, need_part = 2 * T * (int64_t)ncl * H;
+        if (need_hx > c->cap_hx) {
+            if (!grow(&c->hx, &c->cap_hx, need_hx)) return (int)cudaErrorMemoryAllocation;
+            cudaMemsetAsync(c->hx, 0, (size_t)c->cap_hx * sizeof(float), s);
+        }
+        if (need_part > c->cap_part) {
+            if (!grow(&c->part, &c->cap_part, need_part)) return (int)cudaErrorMemoryAllocation;
+            cudaMemsetAsync(c->part, 0, (size_t)c->cap_part * sizeof(float), s);
+        }
+        if (++c->epoch == 0) c->epoch = 1;
+        cp.table = chain_table;
+        cp.groups_dir0 = chain_g;
+        cp.HW = HW;
+        cp.epoch = c->epoch;
+        cp.U0 = Uf; cp.U1 = dirs > 1 ? Ub : Uf; cp.b0 = bf; cp.b1 = dirs > 1 ? bb : bf;
+        cp.P0 = tb.Pf; cp.P1 = tb.Pb;
+        cp.HH = tb.HH;
+        cp.C0 = tb.Cf; cp.C1 = tb.Cb; cp.G0 = tb.Gf; cp.G1 = tb.Gb;
+        cp.dHH = tb.dHH;
+        cp.Gam0 = tb.Gamf; cp.Gam1 = tb.Gamb;
+        cp.hx = reinterpret_cast<unsigned long long*>(c->hx);
+        cp.part = reinterpret_cast<unsigned long long*>(c->part);
+        BL(launch_chain(cp, H, chain_g * dirs, false, s));
+    }
     // forward over the time steps; the two directions are independent chains: the backward one runs on
     // the second stream (its own h_prev / recurrent-product buffers), joined before the head
-    if (dirs > 1) {
+    if (!chain && dirs > 1) {
         cudaEventRecord(c->ev_fork, s);
         cudaStreamWaitEvent(c->s2, c->ev_fork, 0);
     }
-    for (int32_t t = 0; t < maxlen; ++t) {
+    for (int32_t t = 0; t < (chain ? 0 : maxlen); ++t) {
         const int32_t r0 = start[t], n = start[t + 1] - r0;
         for (int d = 0; d < dirs; ++d) {
             const uint32_t* pos = (d == 0 ? fpos : bpos) + r0;
@@ -697,7 +736,7 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
                                                             d == 0 ? tb.Gf : tb.Gb, HS + (int64_t)r0 * H);
         }
     }
-    if (dirs > 1) {
+    if (!chain && dirs > 1) {
         cudaEventRecord(c->ev_join, c->s2);
         cudaStreamWaitEvent(s, c->ev_join, 0);
     }
@@ -723,15 +762,18 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
         BL(gemm_rm(c->st, false, false, (int)T, HW, C, tb.dZ, C, Wt, HW, tb.dHH, HW, 0.f));
     }
     // backward through both LSTMs, last step first
-    cudaMemsetAsync(tb.dHf, 0, T * H * sizeof(float), s);
-    cudaMemsetAsync(tb.dHb, 0, T * H * sizeof(float), s);
-    cudaMemsetAsync(tb.dCf, 0, T * H * sizeof(float), s);
-    cudaMemsetAsync(tb.dCb, 0, T * H * sizeof(float), s);
-    if (dirs > 1) {
+    if (chain) BL(launch_chain(cp, H, chain_g * dirs, true, s));
+    if (!chain) {
+        cudaMemsetAsync(tb.dHf, 0, T * H * sizeof(float), s);
+        cudaMemsetAsync(tb.dHb, 0, T * H * sizeof(float), s);
+        cudaMemsetAsync(tb.dCf, 0, T * H * sizeof(float), s);
+        cudaMemsetAsync(tb.dCb, 0, T * H * sizeof(float), s);
+    }
+    if (!chain && dirs > 1) {
         cudaEventRecord(c->ev_fork, s);
         cudaStreamWaitEvent(c->s2, c->ev_fork, 0);
     }
-    for (int32_t t = maxlen - 1; t >= 0; --t) {
+    for (int32_t t = chain ? -1 : maxlen - 1; t >= 0; --t) {
         const int32_t r0 = start[t], n = start[t + 1] - r0;
         for (int d = 0; d < dirs; ++d) {
             const uint32_t* pos = (d == 0 ? fpos : bpos) + r0;
@@ -749,7 +791,7 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
             if (t > 0) BL(gemm_rm(hd, false, false, n, H, 4 * H, Gs, 4 * H, d == 0 ? Uf : Ub, H, DhW, H, 0.f));
         }
     }
-    if (dirs > 1) {
+    if (!chain && dirs > 1) {
         cudaEventRecord(c->ev_join, c->s2);
         cudaStreamWaitEvent(s, c->ev_join, 0);
     }

@@ -523,3 +523,28 @@ def test_full_size_against_oracle_golden(case, cell, H, C, V, mlp, cfg, b, batch
         assert np.abs(flat[idx] - val).max() <= TOL * mx, name
     dflat = dX.cpu().double().numpy().ravel()
     assert np.abs(dflat[g["dX__idx"]] - g["dX__val"]).max() <= TOL * float(g["dX__max"]), "dX"
+
+
+@pytest.mark.parametrize("H,batch", [(64, 5), (128, 40), (256, 70)])
+def test_chain_recurrence_hidden_sizes(H, batch):
+    """The register-resident chain recurrence (vpps_chain.cu) at every hidden size it is built for, against the
+    oracle: LSTM LM at V = C = 100 on ragged sentences (incl. length 1), and a batch larger than one group's
+    16-sentence slice (several groups, several slices per step at H = 256 with 70 sentences)."""
+    rng = np.random.default_rng(300 + H)
+    graphs = [synth.chain(rng, int(rng.integers(1, 30)), 100, lm=True) for _ in range(batch)]
+    check("lstm", H, H, 100, graphs, 100, seed=301 + H)
+
+
+def test_chain_tagger_paths_agree_subprocess():
+    """VPPS_CHAIN=0 (per-step products, the level path before the register-resident recurrence) still matches
+    the oracle on the tagger (both directions)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = ("import sys; sys.path.insert(0, %r); sys.path.insert(0, %r); import test_gpu_parity as t; "
+            "t.test_tagger_small(); t.test_chain_recurrence_hidden_sizes(128, 40); print('ok')"
+            % (root, os.path.join(root, "tests")))
+    r = subprocess.run([sys.executable, "-c", code], env={**os.environ, "VPPS_CHAIN": "0"}, capture_output=True,
+                       text=True, timeout=600)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stdout + r.stderr
