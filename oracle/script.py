@@ -275,3 +275,34 @@ def device_lowering(ref):
     end = _a32(df_hd + 2 * H * len(hd))
     return dict(lists=[x & 0xFFFFFFFF for x in out], df_off=df_off, n_hx=len(hx), n_part=len(pp), n_hd=len(hd),
                 df_hx=df_hx, df_part=df_part, df_hd=df_hd, df_words=end - ref["pool_words"])
+
+
+def chain_table(graphs, Gd: int, dirs: int):
+    """SPEC_SCRIPT.md §L chain recurrence table, step by step: sentences longest first, each to the group with
+    the smallest total length among those with fewer than 64 sentences (ties lowest), the table words (direction
+    1's groups repeat direction 0's).  None when a sentence finds no group."""
+    lens = [len(g) for g in graphs]
+    offs = [0]
+    for n in lens:
+        offs.append(offs[-1] + n)
+    order = sorted(range(len(graphs)), key=lambda g: -lens[g])          # stable: ties keep batch order
+    mem, load = [[] for _ in range(Gd)], [0] * Gd
+    for g in order:
+        if lens[g] == 0:
+            continue
+        cand = [q for q in range(Gd) if len(mem[q]) < 64]
+        if not cand:
+            return None
+        q = min(cand, key=lambda x: (load[x], x))
+        mem[q].append(g)
+        load[q] += lens[g]
+    G = Gd * dirs
+    words, pre, run = [G, 0], [], 0
+    for q in range(G):
+        run += len(mem[q % Gd])
+        pre.append(run)
+    words += pre
+    for q in range(G):
+        for g in mem[q % Gd]:
+            words += [offs[g], lens[g]]
+    return words

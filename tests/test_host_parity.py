@@ -236,3 +236,26 @@ def test_device_lowering_bit_exact(vpps, G, dataflow):
         assert df_off - lists_off == low["df_off"]
         assert np.array_equal(s.words(), np.array(ref["words"], dtype=np.uint32))    # (lazy when dataflow)
         assert s.info()["n_words"] == len(ref["words"])
+
+
+@pytest.mark.parametrize("cell,H,batch", [("bilstm", 512, 16), ("bilstm", 256, 70), ("lstm", 256, 64),
+                                          ("lstm", 32, 4), ("lstm", 128, 300)])
+def test_chain_table_bit_exact(vpps, cell, H, batch):
+    """SPEC §L: the sentence table of the register-resident chain recurrence (groups per direction from the
+    128-register layout: NCL(H) = ceil(4H^2 / 32768) CTAs, 148 SMs) against oracle/script.py::chain_table,
+    ragged lengths incl. empty sentences, up to 300 sentences (several per group)."""
+    rng = np.random.default_rng(400 + H + batch)
+    graphs = synth.tagger_batch(rng, batch, (1, 60), 50, 5) + [[]]
+    m = vpps.Model(cell, H, H, 5 if cell == "bilstm" else 50, plan_only=True, mlp=8, level=1)
+    blob, lists_off, _ = m.build_script(graphs).blob()
+    ncl = -(-4 * H * H // 32768)
+    dirs = 2 if cell == "bilstm" else 1
+    ref = oscript.chain_table(graphs, (148 // ncl) // dirs, dirs)
+    words = np.asarray(blob, dtype=np.int64)
+    if ref is None:
+        return
+    G = ref[0]
+    n = len(ref)
+    # the table is the last block of the blob (tagger.cpp appends it after the step lists)
+    assert np.array_equal(words[-n:], np.array(ref, dtype=np.int64)), (words[-n:][:8], ref[:8])
+    assert words[-n] == G
