@@ -3,8 +3,8 @@
 // rows dealt to the register files, "the loaded weights ... reused by all the nodes that use the same
 // weight matrix"), whole sentences per group (SPEC S5g's whole-graph groups, here per chain direction), and
 // the signal/wait of L165 replaced by epoch-tagged 64-bit slots (as vpps_df):
-//   HX[pos][H]                  h of a position, read by every CTA of the group at the next step
-//   PART[pos][m][k][UM]         CTA k's part of the transposed product Uᵀγ (L94, fn4) for the UM units CTA m
+//   HX[d][pos][H]               h of a position, read by every CTA of the group at the next step
+//   PART[d][pos][m][k][UM]      CTA k's part of the transposed product Uᵀγ (L94, fn4) for the UM units CTA m
 //                               owns, consumed by position pos (the previous step of the same chain)
 // The input projections W x (all positions, one GEMM), the head and the weight gradients are dense
 // products of the level path; this file replaces its per-time-step recurrent products:
@@ -120,7 +120,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_chain_fwd(const ChainParams P) {
     const float* Pin = d == 0 ? P.P0 : P.P1;
     float* Cd = d == 0 ? P.C0 : P.C1;
     float* Gd = d == 0 ? P.G0 : P.G1;
-    u64* HX = P.hx;
+    u64* HX = P.hx + (int64_t)d * P.T * H;             // each direction has its own slots
     __syncthreads();
     const int L = ns > 0 ? (int)s_len[0] : 0;
     int buf = 0;
@@ -250,7 +250,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_chain_bwd(const ChainParams P) {
     const float* Cd = d == 0 ? P.C0 : P.C1;
     const float* Gd = d == 0 ? P.G0 : P.G1;
     float* Gam = d == 0 ? P.Gam0 : P.Gam1;
-    u64* PART = P.part;
+    u64* PART = P.part + (int64_t)d * P.T * NCL * H;   // each direction has its own slots
     __syncthreads();
     const int L = ns > 0 ? (int)s_len[0] : 0;
     int cbuf = 0;

@@ -122,8 +122,9 @@ struct ChainParams {
     float *C0, *C1, *G0, *G1;        // c [T][H], gates (i, f, o, g) [T][4H] per direction
     const float* dHH;                // the head's dh [T][HW]
     float *Gam0, *Gam1;              // γ [T][4H] per direction (left operands of the weight gradients)
-    unsigned long long* hx;          // [T][H] tagged h slots
-    unsigned long long* part;        // [T][NCL][NCL][UM] tagged Uᵀγ parts
+    unsigned long long* hx;          // [dirs][T][H] tagged h slots
+    unsigned long long* part;        // [dirs][T][NCL][NCL][UM] tagged Uᵀγ parts
+    int64_t T;                       // positions
 };
 int32_t chain_group_ctas(int32_t H);
 cudaError_t launch_chain(const ChainParams& P, int32_t H, int32_t n_groups, bool backward, cudaStream_t s);

@@ -689,7 +689,7 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
     const bool chain = ncl > 0 && chain_g > 0;
     if (chain) {
         // slots: HX [T][H] and PART [T][NCL][H] 64-bit words, never cleared again (epoch tags)
-        const int64_t need_hx = 2 * T * H, need_part = 2 * T * (int64_t)ncl * H;
+        const int64_t need_hx = 2 * dirs * T * H, need_part = 2 * dirs * T * (int64_t)ncl * H;
         if (need_hx > c->cap_hx) {
             if (!grow(&c->hx, &c->cap_hx, need_hx)) return (int)cudaErrorMemoryAllocation;
             cudaMemsetAsync(c->hx, 0, (size_t)c->cap_hx * sizeof(float), s);
@@ -711,6 +711,7 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
         cp.Gam0 = tb.Gamf; cp.Gam1 = tb.Gamb;
         cp.hx = reinterpret_cast<unsigned long long*>(c->hx);
         cp.part = reinterpret_cast<unsigned long long*>(c->part);
+        cp.T = T;
         BL(launch_chain(cp, H, chain_g * dirs, false, s));
     }
     // forward over the time steps; the two directions are independent chains: the backward one runs on
