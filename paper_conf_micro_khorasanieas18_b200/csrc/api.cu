@@ -180,7 +180,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
         // LSTM chains: the recurrence runs register-resident in groups of co-resident CTAs (vpps_chain.cu)
         // when a specialisation exists for H; VPPS_CHAIN=0 (measurement) keeps the per-step products
         static const bool chain_env = !(getenv("VPPS_CHAIN") && atoi(getenv("VPPS_CHAIN")) == 0);
-        if ((cell == CELL_BILSTM || cell == CELL_LSTM) && chain_env) {
+        if ((cell == CELL_BILSTM || cell == CELL_LSTM || cell == CELL_GRU) && chain_env) {
             const int32_t ncl = chain_group_ctas(H), dirs = cell == CELL_BILSTM ? 2 : 1;
             m->plan.chain_g = ncl > 0 ? (sms / ncl) / dirs : 0;
         }
@@ -658,7 +658,8 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         const int rc = gru_pass(m->level, m->params, m->offsets.data(), m->grads, m->pool, inputs, d_inputs, dwords,
                                 s->s.tg_tok, s->s.tg_lab, s->s.tg_fpos, s->s.tg_start.data(),
                                 (int32_t)s->s.tg_start.size() - 1, s->s.tg_T, m->plan.H, m->plan.E, m->plan.C,
-                                s->s.loss_word, st);
+                                s->s.loss_word, st, s->s.tg_chain >= 0 ? dwords + s->s.tg_chain : nullptr,
+                                m->plan.chain_g);
         if (rc != 0) return fail(VPPS_E_CUDA, "GRU pass failed (code " + std::to_string(rc) + ")");
         if (mode == 1) launch_sgd(m->params, m->grads, m->n_floats, lr, wd, st);
     } else if (m->plan.level && (m->plan.cell == CELL_BILSTM || m->plan.cell == CELL_LSTM)) {

@@ -74,13 +74,13 @@ __device__ __forceinline__ int pos_of(uint32_t off, uint32_t len, int t, int d) 
     return d == 0 ? (int)off + t : (int)(off + len) - 1 - t;
 }
 
-template <int H>
-__device__ __forceinline__ void load_weights(const ChainParams& P, int d, int lc, float (&w)[4][Cfg<H>::CPT]) {
+template <int H, int NGT>
+__device__ __forceinline__ void load_weights(const ChainParams& P, int d, int lc, float (&w)[NGT][Cfg<H>::CPT]) {
     using C = Cfg<H>;
     const int tid = threadIdx.x, u = tid / C::TU, tau = tid % C::TU, j = lc * C::UM + u;
     const float* U = d == 0 ? P.U0 : P.U1;
 #pragma unroll
-    for (int k = 0; k < 4; ++k)
+    for (int k = 0; k < NGT; ++k)
 #pragma unroll
         for (int t = 0; t < C::NG; ++t) {
             const float* src = U + (int64_t)(k * H + j) * H + C::CG * (tau + C::TU * t);
@@ -94,11 +94,13 @@ __device__ __forceinline__ void load_weights(const ChainParams& P, int d, int lc
         }
 }
 
-// ---- forward: every step of the group's sentences, in order ----
-template <int H>
+// ---- forward: every step of the group's sentences, in order.  CELL 0 = LSTM (gates i, f, o, g), 1 = GRU
+//      (M5, reading R-34: gates r, z, n with the reset on U_n h + b_hn; h' = (1 - z) n + z h) ----
+template <int H, int CELL>
 __global__ void __launch_bounds__(NTH, 1) vpps_chain_fwd(const ChainParams P) {
     using C = Cfg<H>;
     constexpr int TU = C::TU, UM = C::UM, CG = C::CG, NG = C::NG;
+    constexpr int NGT = CELL == 0 ? 4 : 3;               // gate rows per unit
     extern __shared__ __align__(16) float csm[];
     float* xs0 = csm;                                  // two staging buffers [NB][H]
     __shared__ uint32_t s_off[MAXS], s_len[MAXS];
@@ -112,11 +114,13 @@ __global__ void __launch_bounds__(NTH, 1) vpps_chain_fwd(const ChainParams P) {
     const int d = grp < P.groups_dir0 ? 0 : 1;
     const uint32_t ep = P.epoch;
     for (int i = tid; i < ns; i += NTH) { s_off[i] = T[G + 2 + 2 * (s0 + i)]; s_len[i] = T[G + 3 + 2 * (s0 + i)]; }
-    float w[4][C::CPT];
-    load_weights<H>(P, d, lc, w);
-    float bias[4];
+    float w[NGT][C::CPT];
+    load_weights<H, NGT>(P, d, lc, w);
+    float bias[4], bias_h[3];                              // LSTM b; GRU b_i, b_h
 #pragma unroll
-    for (int k = 0; k < 4; ++k) bias[k] = __ldg((d == 0 ? P.b0 : P.b1) + k * H + j);
+    for (int k = 0; k < NGT; ++k) bias[k] = __ldg((CELL == 1 || d == 0 ? P.b0 : P.b1) + k * H + j);
+#pragma unroll
+    for (int k = 0; k < 3; ++k) bias_h[k] = CELL == 1 ? __ldg(P.b1 + k * H + j) : 0.f;
     const float* Pin = d == 0 ? P.P0 : P.P1;
     float* Cd = d == 0 ? P.C0 : P.C1;
     float* Gd = d == 0 ? P.G0 : P.G1;
@@ -151,13 +155,13 @@ __global__ void __launch_bounds__(NTH, 1) vpps_chain_fwd(const ChainParams P) {
             }
             // ---- U h_{t-1}: 4 sentences at a time; the TU lanes of a unit reduce with a butterfly ----
             for (int n0 = 0; n0 < nb; n0 += 4) {
-                float s[4][4];
+                float s[4][NGT];
                 if (t > 0) {
-                    float2 a[4][4];
+                    float2 a[4][NGT];
 #pragma unroll
                     for (int n = 0; n < 4; ++n)
 #pragma unroll
-                        for (int k = 0; k < 4; ++k) a[n][k] = make_float2(0.f, 0.f);
+                        for (int k = 0; k < NGT; ++k) a[n][k] = make_float2(0.f, 0.f);
 #pragma unroll
                     for (int g = 0; g < NG; ++g) {
                         const int col = CG * (tau + TU * g);
@@ -169,18 +173,18 @@ __global__ void __launch_bounds__(NTH, 1) vpps_chain_fwd(const ChainParams P) {
 #pragma unroll
                             for (int q = 0; q + 1 < CG; q += 2)
 #pragma unroll
-                                for (int k = 0; k < 4; ++k)
+                                for (int k = 0; k < NGT; ++k)
                                     a[n][k] = __ffma2_rn(make_float2(w[k][CG * g + q], w[k][CG * g + q + 1]),
                                                          make_float2(xv[q], xv[q + 1]), a[n][k]);
                             if constexpr (CG == 1)
 #pragma unroll
-                                for (int k = 0; k < 4; ++k) a[n][k].x = fmaf(w[k][g], xv[0], a[n][k].x);
+                                for (int k = 0; k < NGT; ++k) a[n][k].x = fmaf(w[k][g], xv[0], a[n][k].x);
                         }
                     }
 #pragma unroll
                     for (int n = 0; n < 4; ++n)
 #pragma unroll
-                        for (int k = 0; k < 4; ++k) {
+                        for (int k = 0; k < NGT; ++k) {
                             float v = a[n][k].x + a[n][k].y;
 #pragma unroll
                             for (int o = TU / 2; o >= 1; o >>= 1) v += __shfl_xor_sync(FULLMASK, v, o);
@@ -190,33 +194,46 @@ __global__ void __launch_bounds__(NTH, 1) vpps_chain_fwd(const ChainParams P) {
 #pragma unroll
                     for (int n = 0; n < 4; ++n)
 #pragma unroll
-                        for (int k = 0; k < 4; ++k) s[n][k] = 0.f;
+                        for (int k = 0; k < NGT; ++k) s[n][k] = 0.f;
                 }
                 // ---- cell: lane τ < 4 of the unit updates sentence n0 + τ ----
                 const int n = n0 + tau;
                 if (tau < 4 && n < nb) {
-                    float a4[4];
+                    float a4[NGT];
 #pragma unroll
-                    for (int k = 0; k < 4; ++k) {
+                    for (int k = 0; k < NGT; ++k) {
                         float v = s[0][k];
 #pragma unroll
                         for (int m = 1; m < 4; ++m) v = tau == m ? s[m][k] : v;
                         a4[k] = v;
                     }
                     const int pos = pos_of(s_off[b0 + n], s_len[b0 + n], t, d);
-                    const float* pr = Pin + (int64_t)pos * 4 * H;
-                    const float ig = fsigm(a4[0] + __ldg(pr + j) + bias[0]);
-                    const float fg = fsigm(a4[1] + __ldg(pr + H + j) + bias[1]);
-                    const float og = fsigm(a4[2] + __ldg(pr + 2 * H + j) + bias[2]);
-                    const float gg = ftanh(a4[3] + __ldg(pr + 3 * H + j) + bias[3]);
-                    const float cp = t > 0 ? Cd[(int64_t)pos_of(s_off[b0 + n], s_len[b0 + n], t - 1, d) * H + j] : 0.f;
-                    const float c = fg * cp + ig * gg;
-                    const float h = og * ftanh(c);
+                    const int ppos = pos_of(s_off[b0 + n], s_len[b0 + n], t - 1, d);
+                    const float* pr = Pin + (int64_t)pos * NGT * H;
+                    float h;
+                    if constexpr (CELL == 0) {
+                        const float ig = fsigm(a4[0] + __ldg(pr + j) + bias[0]);
+                        const float fg = fsigm(a4[1] + __ldg(pr + H + j) + bias[1]);
+                        const float og = fsigm(a4[2] + __ldg(pr + 2 * H + j) + bias[2]);
+                        const float gg = ftanh(a4[3] + __ldg(pr + 3 * H + j) + bias[3]);
+                        const float cp = t > 0 ? Cd[(int64_t)ppos * H + j] : 0.f;
+                        const float c = fg * cp + ig * gg;
+                        h = og * ftanh(c);
+                        Cd[(int64_t)pos * H + j] = c;
+                        float* gr = Gd + (int64_t)pos * 4 * H;
+                        gr[j] = ig; gr[H + j] = fg; gr[2 * H + j] = og; gr[3 * H + j] = gg;
+                    } else {
+                        const float ahr = bias_h[0] + a4[0], ahz = bias_h[1] + a4[1], ahn = bias_h[2] + a4[2];
+                        const float rg = fsigm(__ldg(pr + j) + bias[0] + ahr);
+                        const float zg = fsigm(__ldg(pr + H + j) + bias[1] + ahz);
+                        const float ng = ftanh(__ldg(pr + 2 * H + j) + bias[2] + rg * ahn);
+                        const float hp = t > 0 ? P.HH[(int64_t)ppos * P.HW + j] : 0.f;
+                        h = (1.f - zg) * ng + zg * hp;
+                        float* gr = Gd + (int64_t)pos * 4 * H;
+                        gr[j] = rg; gr[H + j] = zg; gr[2 * H + j] = ng; gr[3 * H + j] = ahn;
+                    }
                     if (t + 1 < (int)s_len[b0 + n]) st_tag(HX + (int64_t)pos * H + j, h, ep);   // next step's input
                     P.HH[(int64_t)pos * P.HW + d * H + j] = h;
-                    Cd[(int64_t)pos * H + j] = c;
-                    float* gr = Gd + (int64_t)pos * 4 * H;
-                    gr[j] = ig; gr[H + j] = fg; gr[2 * H + j] = og; gr[3 * H + j] = gg;
                 }
             }
         }
@@ -224,14 +241,16 @@ __global__ void __launch_bounds__(NTH, 1) vpps_chain_fwd(const ChainParams P) {
 }
 
 // ---- backward: every step of the group's sentences, last first ----
-template <int H>
+template <int H, int CELL>
 __global__ void __launch_bounds__(NTH, 1) vpps_chain_bwd(const ChainParams P) {
     using C = Cfg<H>;
     constexpr int TU = C::TU, UM = C::UM, CG = C::CG, NCL = C::NCL, KEEP = C::KEEP;
+    constexpr int NGT = CELL == 0 ? 4 : 3;
     constexpr int NW = NTH / 32;
     extern __shared__ __align__(16) float csm[];
     float* gam_s = csm;                                // [NB][4][UM] this step's γ of the CTA's units
-    float* dcs = gam_s + NB * 4 * UM;                  // [MAXS][UM] dc carried to the previous step
+    float* dcs = gam_s + NB * 4 * UM;                  // [MAXS][UM] carried to the previous step: the LSTM's
+                                                       // dc_{t-1}, the GRU's direct term dh z of dh_{t-1}
     float* dxb0 = dcs + MAXS * UM;                     // [2][NW][NC][H] warp slices of Uᵀγ
     __shared__ uint32_t s_off[MAXS], s_len[MAXS];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -245,8 +264,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_chain_bwd(const ChainParams P) {
     const uint32_t ep = P.epoch;
     for (int i = tid; i < ns; i += NTH) { s_off[i] = T[G + 2 + 2 * (s0 + i)]; s_len[i] = T[G + 3 + 2 * (s0 + i)]; }
     for (int i = tid; i < MAXS * UM; i += NTH) dcs[i] = 0.f;
-    float w[4][C::CPT];
-    load_weights<H>(P, d, lc, w);
+    float w[NGT][C::CPT];
+    load_weights<H, NGT>(P, d, lc, w);
     const float* Cd = d == 0 ? P.C0 : P.C1;
     const float* Gd = d == 0 ? P.G0 : P.G1;
     float* Gam = d == 0 ? P.Gam0 : P.Gam1;
@@ -280,22 +299,39 @@ __global__ void __launch_bounds__(NTH, 1) vpps_chain_bwd(const ChainParams P) {
 #pragma unroll
                     for (int k = 0; k < NCL; ++k) dh += __uint_as_float((uint32_t)v[k]);
                 }
-                const float dc = t + 1 < (int)len ? dcs[sn * UM + uu] : 0.f;
+                const float carry = t + 1 < (int)len ? dcs[sn * UM + uu] : 0.f;
                 const float* gr = Gd + (int64_t)pos * 4 * H;
-                const float i = gr[jj], f = gr[H + jj], o = gr[2 * H + jj], g = gr[3 * H + jj];
-                const float c = Cd[(int64_t)pos * H + jj];
-                const float cp = t > 0 ? Cd[(int64_t)pos_of(off, len, t - 1, d) * H + jj] : 0.f;
-                const float tc = ftanh(c);
-                const float chat = dc + dh * o * (1.f - tc * tc);
-                const float gam[4] = {chat * g * i * (1.f - i), chat * cp * f * (1.f - f), dh * tc * o * (1.f - o),
-                                      chat * i * (1.f - g * g)};
-                float* go = Gam + (int64_t)pos * 4 * H;
+                if constexpr (CELL == 0) {
+                    const float i = gr[jj], f = gr[H + jj], o = gr[2 * H + jj], g = gr[3 * H + jj];
+                    const float c = Cd[(int64_t)pos * H + jj];
+                    const float cp = t > 0 ? Cd[(int64_t)pos_of(off, len, t - 1, d) * H + jj] : 0.f;
+                    const float tc = ftanh(c);
+                    const float chat = carry + dh * o * (1.f - tc * tc);
+                    const float gam[4] = {chat * g * i * (1.f - i), chat * cp * f * (1.f - f), dh * tc * o * (1.f - o),
+                                          chat * i * (1.f - g * g)};
+                    float* go = Gam + (int64_t)pos * 4 * H;
 #pragma unroll
-                for (int k = 0; k < 4; ++k) {
-                    go[k * H + jj] = gam[k];
-                    gam_s[(n * 4 + k) * UM + uu] = gam[k];
+                    for (int k = 0; k < 4; ++k) {
+                        go[k * H + jj] = gam[k];
+                        gam_s[(n * 4 + k) * UM + uu] = gam[k];
+                    }
+                    dcs[sn * UM + uu] = chat * f;                  // dc of step t-1 (same thread next time)
+                } else {
+                    const float dht = dh + carry;
+                    const float rg = gr[jj], zg = gr[H + jj], ng = gr[2 * H + jj], ahn = gr[3 * H + jj];
+                    const float hp = t > 0 ? P.HH[(int64_t)pos_of(off, len, t - 1, d) * P.HW + jj] : 0.f;
+                    const float dan = dht * (1.f - zg) * (1.f - ng * ng);
+                    const float dar = dan * ahn * rg * (1.f - rg);
+                    const float daz = dht * (hp - ng) * zg * (1.f - zg);
+                    float* gx = P.Gam0 + (int64_t)pos * 3 * H;
+                    float* gh = P.Gam1 + (int64_t)pos * 3 * H;
+                    gx[jj] = dar; gx[H + jj] = daz; gx[2 * H + jj] = dan;
+                    gh[jj] = dar; gh[H + jj] = daz; gh[2 * H + jj] = dan * rg;
+                    gam_s[(n * 4 + 0) * UM + uu] = dar;
+                    gam_s[(n * 4 + 1) * UM + uu] = daz;
+                    gam_s[(n * 4 + 2) * UM + uu] = dan * rg;
+                    dcs[sn * UM + uu] = dht * zg;                  // dh_{t-1} += dh z (same thread next time)
                 }
-                dcs[sn * UM + uu] = chat * f;                  // dc of step t-1 (same thread next time)
             }
             __syncthreads();
             if (t == 0) continue;                              // no predecessor: no Uᵀγ
@@ -308,16 +344,16 @@ __global__ void __launch_bounds__(NTH, 1) vpps_chain_bwd(const ChainParams P) {
                 for (int dn = 0; dn < NC; ++dn) {
                     const int n = n0 + dn;
                     if (n >= nb) break;
-                    float gr[4];
+                    float gr[NGT];
 #pragma unroll
-                    for (int k = 0; k < 4; ++k) gr[k] = gam_s[(n * 4 + k) * UM + u];
+                    for (int k = 0; k < NGT; ++k) gr[k] = gam_s[(n * 4 + k) * UM + u];
                     float v[C::CPT];
 #pragma unroll
                     for (int c = 0; c < C::CPT; c += 2) {
                         float2 a = __ffma2_rn(make_float2(w[0][c], w[0][c + 1]), make_float2(gr[0], gr[0]), make_float2(0.f, 0.f));
-                        a = __ffma2_rn(make_float2(w[1][c], w[1][c + 1]), make_float2(gr[1], gr[1]), a);
-                        a = __ffma2_rn(make_float2(w[2][c], w[2][c + 1]), make_float2(gr[2], gr[2]), a);
-                        a = __ffma2_rn(make_float2(w[3][c], w[3][c + 1]), make_float2(gr[3], gr[3]), a);
+#pragma unroll
+                        for (int k = 1; k < NGT; ++k)
+                            a = __ffma2_rn(make_float2(w[k][c], w[k][c + 1]), make_float2(gr[k], gr[k]), a);
                         v[c] = a.x;
                         v[c + 1] = a.y;
                     }
@@ -398,8 +434,8 @@ constexpr size_t bwd_smem() {
 
 #define VPPS_CHAIN_CASE(HH)                                                                          \
     case HH:                                                                                         \
-        fwd = (const void*)&dev::ch::vpps_chain_fwd<HH>;                                             \
-        bwd = (const void*)&dev::ch::vpps_chain_bwd<HH>;                                             \
+        fwd = gru ? (const void*)&dev::ch::vpps_chain_fwd<HH, 1> : (const void*)&dev::ch::vpps_chain_fwd<HH, 0>; \
+        bwd = gru ? (const void*)&dev::ch::vpps_chain_bwd<HH, 1> : (const void*)&dev::ch::vpps_chain_bwd<HH, 0>; \
         ncl = dev::ch::Cfg<HH>::NCL;                                                                 \
         sm_f = dev::ch::fwd_smem<HH>();                                                              \
         sm_b = dev::ch::bwd_smem<HH>();                                                              \
@@ -417,7 +453,7 @@ int32_t chain_group_ctas(int32_t H) {
     }
 }
 
-cudaError_t launch_chain(const ChainParams& P, int32_t H, int32_t n_groups, bool backward, cudaStream_t s) {
+cudaError_t launch_chain(const ChainParams& P, int32_t H, int32_t n_groups, bool backward, cudaStream_t s, bool gru) {
     const void* fwd = nullptr;
     const void* bwd = nullptr;
     int ncl = 0;

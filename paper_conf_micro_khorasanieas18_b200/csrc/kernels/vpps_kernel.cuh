@@ -116,7 +116,8 @@ struct ChainParams {
     int32_t groups_dir0;
     int32_t HW;                      // row stride of HH / dHH (H, or 2H for the tagger)
     uint32_t epoch;                  // tag of this pass's slots (never 0)
-    const float *U0, *U1, *b0, *b1;  // recurrent matrices and biases of the two directions
+    const float *U0, *U1, *b0, *b1;  // recurrent matrices and biases of the two directions (GRU: U0, b0 = b_i,
+                                     // b1 = b_h; Gam0 = γ_x, Gam1 = γ_h; P0 is W x [T][3H])
     const float *P0, *P1;            // input projections W x [T][4H] (bias not included)
     float* HH;                       // h [T][HW] (direction d at column d H)
     float *C0, *C1, *G0, *G1;        // c [T][H], gates (i, f, o, g) [T][4H] per direction
@@ -127,7 +128,8 @@ struct ChainParams {
     int64_t T;                       // positions
 };
 int32_t chain_group_ctas(int32_t H);
-cudaError_t launch_chain(const ChainParams& P, int32_t H, int32_t n_groups, bool backward, cudaStream_t s);
+cudaError_t launch_chain(const ChainParams& P, int32_t H, int32_t n_groups, bool backward, cudaStream_t s,
+                         bool gru = false);
 // Level-synchronous path (vpps_level.cu): context (cuBLAS handle + work buffers) and one training pass.
 void* level_ctx_create(const DevAlloc* alloc);
 void level_ctx_destroy(void* ctx);
@@ -151,6 +153,6 @@ int tagger_pass(void* ctx, const float* params, const int64_t* off, float* grads
 int gru_pass(void* ctx, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
              float* d_inputs, const uint32_t* d_blob, int64_t tg_tok, int64_t tg_lab, int64_t tg_fpos,
              const int32_t* start, int32_t maxlen, int64_t T, int32_t H, int32_t E, int32_t C, int64_t loss_word,
-             cudaStream_t s);
+             cudaStream_t s, const uint32_t* chain_table = nullptr, int32_t chain_g = 0);
 
 }  // namespace vpps

@@ -826,7 +826,7 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
 int gru_pass(void* ctx_, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
              float* d_inputs, const uint32_t* d_blob, int64_t tg_tok, int64_t tg_lab, int64_t tg_fpos,
              const int32_t* start, int32_t maxlen, int64_t T, int32_t H, int32_t E, int32_t C, int64_t loss_word,
-             cudaStream_t s) {
+             cudaStream_t s, const uint32_t* chain_table, int32_t chain_g) {
     using namespace dev::lv;
     LevelCtx* c = static_cast<LevelCtx*>(ctx_);
     TaggerBufs& tb = c->tg;
@@ -852,7 +852,38 @@ int gru_pass(void* ctx_, const float* params, const int64_t* off, float* grads, 
     if (T == 0) return 0;
     tg_gather_x<<<nblk(T * (E / 4)), 256, 0, s>>>(inputs, tok, (int)T, E, tb.X);
     BL(gemm_rm(c->st, false, true, (int)T, 3 * H, E, tb.X, E, W, E, tb.Pf, 3 * H, 0.f));
-    for (int32_t t = 0; t < maxlen; ++t) {
+    // register-resident recurrence (vpps_chain.cu, GRU cell): one forward and one backward launch
+    ChainParams cp{};
+    const int32_t ncl = chain_table ? chain_group_ctas(H) : 0;
+    const bool chain = ncl > 0 && chain_g > 0;
+    if (chain) {
+        const int64_t need_hx = 2 * T * H, need_part = 2 * T * (int64_t)ncl * H;
+        if (need_hx > c->cap_hx) {
+            if (!grow(&c->hx, &c->cap_hx, need_hx)) return (int)cudaErrorMemoryAllocation;
+            cudaMemsetAsync(c->hx, 0, (size_t)c->cap_hx * sizeof(float), s);
+        }
+        if (need_part > c->cap_part) {
+            if (!grow(&c->part, &c->cap_part, need_part)) return (int)cudaErrorMemoryAllocation;
+            cudaMemsetAsync(c->part, 0, (size_t)c->cap_part * sizeof(float), s);
+        }
+        if (++c->epoch == 0) c->epoch = 1;
+        cp.table = chain_table;
+        cp.groups_dir0 = chain_g;
+        cp.HW = H;
+        cp.epoch = c->epoch;
+        cp.U0 = U; cp.U1 = U; cp.b0 = b_i; cp.b1 = b_h;
+        cp.P0 = tb.Pf; cp.P1 = tb.Pf;
+        cp.HH = tb.HH;
+        cp.C0 = cp.C1 = nullptr;
+        cp.G0 = cp.G1 = tb.Gf;
+        cp.dHH = tb.dHH;
+        cp.Gam0 = tb.Gamf; cp.Gam1 = tb.Gamb;
+        cp.hx = reinterpret_cast<unsigned long long*>(c->hx);
+        cp.part = reinterpret_cast<unsigned long long*>(c->part);
+        cp.T = T;
+        BL(launch_chain(cp, H, chain_g, false, s, true));
+    }
+    for (int32_t t = 0; t < (chain ? 0 : maxlen); ++t) {
         const int32_t r0 = start[t], n = start[t + 1] - r0;
         const uint32_t* pos = fpos + r0;
         if (t > 0)   // h_prev of row r = row r of the previous step's block (longest-first step lists)
@@ -866,8 +897,9 @@ int gru_pass(void* ctx_, const float* params, const int64_t* off, float* grads, 
     BL(gemm_rm(c->st, true, false, C, H, (int)T, tb.dZ, C, tb.HH, H, grads + off[2], H, 0.f));
     colsum<<<nblk(C), 256, 0, s>>>(tb.dZ, (int)T, C, grads + off[5]);
     BL(gemm_rm(c->st, false, false, (int)T, H, C, tb.dZ, C, Wo, H, tb.dHH, H, 0.f));
-    cudaMemsetAsync(tb.dHf, 0, T * H * sizeof(float), s);
-    for (int32_t t = maxlen - 1; t >= 0; --t) {
+    if (chain) BL(launch_chain(cp, H, chain_g, true, s, true));
+    else cudaMemsetAsync(tb.dHf, 0, T * H * sizeof(float), s);
+    for (int32_t t = chain ? -1 : maxlen - 1; t >= 0; --t) {
         const int32_t r0 = start[t], n = start[t + 1] - r0;
         const uint32_t* pos = fpos + r0;
         // Γ_h U and dh ⊙ z of step t go to one buffer pair, read by step t-1 (row-aligned)

@@ -14,9 +14,10 @@ from oracle import models as M  # noqa: E402
 
 for cell, H, batch, lens in [("lstm", 32, 3, (1, 6)), ("lstm", 64, 3, (1, 6)), ("lstm", 128, 3, (1, 6)),
                              ("lstm", 256, 3, (1, 6)), ("lstm", 256, 40, (1, 30)), ("bilstm", 32, 3, (1, 6)),
-                             ("bilstm", 64, 3, (1, 6)), ("bilstm", 256, 5, (1, 12))]:
+                             ("bilstm", 64, 3, (1, 6)), ("bilstm", 256, 5, (1, 12)), ("gru", 32, 3, (1, 6)),
+                             ("gru", 64, 5, (1, 9)), ("gru", 256, 40, (1, 30))]:
     rng = np.random.default_rng(5)
-    if cell == "lstm":
+    if cell in ("lstm", "gru"):
         graphs = [synth.chain(rng, int(rng.integers(lens[0], lens[1] + 1)), 100, lm=True) for _ in range(batch)]
         C, V, kw = 100, 100, {}
     else:
