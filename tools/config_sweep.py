@@ -50,6 +50,17 @@ CASES = [
 ]
 
 
+def kernel_label(cell, H, C, opts):
+    if opts.get("dataflow"):
+        return "vpps_df + GEMMs"
+    chain = cell in ("bilstm", "gru") or (cell == "lstm" and (opts.get("level") or C > 32))
+    if chain and os.environ.get("VPPS_CHAIN", "1") != "0" and H in (32, 64, 128, 256, 512):
+        return "vpps_chain (register-resident recurrence) + GEMMs"
+    if opts.get("level") or H > 256 or cell in ("bilstm", "gru", "rvnn", "tdrnn", "tdlstm") or C > 32:
+        return "level GEMMs"
+    return "vpps_fb (grid)"
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--steps", type=int, default=50)
@@ -108,7 +119,7 @@ def main():
         rec = {"case": label, "ms_per_step": round(ms, 4), "samples_per_s": round(B / ms * 1e3, 1),
                "nodes_per_s": round(nn / ms * 1e3, 1), "gflop_per_step": round(f / 1e9, 4),
                "tflops": round(f / ms / 1e9, 3), "frac_fp32_peak": round(f / (ms * 1e-3) / peak, 4),
-               "kernel": "vpps_df + GEMMs" if opts.get("dataflow") else ("level GEMMs" if (opts.get("level") or H > 256 or cell in ("bilstm", "gru", "rvnn", "tdrnn", "tdlstm") or C > 32) else "vpps_fb (grid)")}
+               "kernel": kernel_label(cell, H, C, opts)}
         lines.append(rec)
         print(json.dumps(rec), flush=True)
         del m
