@@ -122,6 +122,9 @@ typedef struct {
                             FP32 SGEMM), fused cell / head / scatter kernels, dW as one GEMM per
                             matrix.  0 = auto: chosen when no register-resident specialisation
                             exists for (H, E) (config 5: H = E = 1024); -1 = never. */
+    int32_t chain;       /* chain cells on the level path (LSTM LM, BiLSTM tagger, GRU): 0 = the register-
+                            resident recurrence (vpps_chain.cu) when a specialisation exists for H; -1 =
+                            one recurrent product + cell launch per time step */
     vpps_alloc_fn alloc; /* device allocator for library-owned buffers (see above); NULL = default */
     vpps_free_fn free;
     void* alloc_ctx;     /* passed back to alloc / free                                         */

@@ -180,7 +180,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
         // LSTM chains: the recurrence runs register-resident in groups of co-resident CTAs (vpps_chain.cu)
         // when a specialisation exists for H; VPPS_CHAIN=0 (measurement) keeps the per-step products
         static const bool chain_env = !(getenv("VPPS_CHAIN") && atoi(getenv("VPPS_CHAIN")) == 0);
-        if ((cell == CELL_BILSTM || cell == CELL_LSTM || cell == CELL_GRU) && chain_env) {
+        if ((cell == CELL_BILSTM || cell == CELL_LSTM || cell == CELL_GRU) && chain_env && o.chain >= 0) {
             const int32_t ncl = chain_group_ctas(H), dirs = cell == CELL_BILSTM ? 2 : 1;
             m->plan.chain_g = ncl > 0 ? (sms / ncl) / dirs : 0;
         }

@@ -40,7 +40,7 @@ _FREE_FN = ct.CFUNCTYPE(None, ct.c_void_p, ct.c_void_p, ct.c_void_p)
 class _Options(ct.Structure):
     _fields_ = [("n_sm", ct.c_int32), ("ctas_per_sm", ct.c_int32), ("groups", ct.c_int32),
                 ("device", ct.c_int32), ("plan_only", ct.c_int32), ("cluster", ct.c_int32),
-                ("dataflow", ct.c_int32), ("level", ct.c_int32),
+                ("dataflow", ct.c_int32), ("level", ct.c_int32), ("chain", ct.c_int32),
                 ("alloc", _ALLOC_FN), ("free", _FREE_FN), ("alloc_ctx", ct.c_void_p)]
 
 
@@ -248,6 +248,71 @@ def prefetch_scripts(model: "Model", batches, depth: int = 4, workers: int = 3, 
             yield s
 
 
+# ---- profile-guided choice of the device path (kernels are built for several register
+#      layouts and the one to use is picked by timing batches) ----
+def candidate_options(cell: str, H: int, C: int):
+    """The device paths this build offers for an op set (vpps_define_model options), paper order first."""
+    out = []
+    if cell == "binary":
+        if H == 256:
+            out += [dict(cluster=16, dataflow=True), dict(cluster=16)]
+        out += [dict(groups=g, level=-1) for g in (1, 2, 4)] + [dict(level=1)]
+    elif cell == "childsum":
+        out += [dict(groups=g) for g in (1, 2, 4)]
+    elif cell == "lstm":
+        if C <= 32:
+            out += [dict(groups=g, level=-1) for g in (1, 2)]
+        out += [dict(level=1, chain=0), dict(level=1, chain=-1)]
+    elif cell in ("gru", "bilstm"):
+        out += [dict(chain=0), dict(chain=-1)]
+    else:
+        out += [dict()]
+    return out
+
+
+def autotune(cell: str, H: int, E: int, C: int, batches, inputs, candidates=None, mlp: int = 256, device: int = 0,
+             warmup: int = 2, reps: int = 3, timer=None):
+    """Time one training pass per sample batch on every candidate path and return (best options, {options
+    repr: ms per pass}).  Candidates that this build cannot instantiate (VPPS_E_NOFIT / INVALID) are skipped.
+    `timer(model, scripts, inputs)` -> ms overrides the CUDA-event timing (tests)."""
+    import torch
+    results = {}
+    best, best_ms = None, float("inf")
+    for opts in (candidates if candidates is not None else candidate_options(cell, H, C)):
+        try:
+            m = Model(cell, H, E, C, device=device, mlp=mlp, **opts)
+        except VppsError:
+            continue
+        if timer is not None:
+            ms = timer(m, batches, inputs)
+        else:
+            params = torch.zeros(m.n_floats, dtype=torch.float32, device=f"cuda:{device}")
+            torch.nn.init.uniform_(params, -0.05, 0.05)
+            grads = torch.zeros_like(params)
+            m.bind(params, grads)
+            scripts = [m.build_script(b) for b in batches]
+            for s in scripts:
+                s.upload()
+            for _ in range(warmup):
+                for s in scripts:
+                    m.fwd_bwd(s, inputs)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            e0.record()
+            for _ in range(reps):
+                for s in scripts:
+                    m.fwd_bwd(s, inputs)
+            e1.record()
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / (reps * len(scripts))
+        results[repr(opts)] = ms
+        if ms < best_ms:
+            best, best_ms = opts, ms
+    if best is None:
+        raise VppsError(-2, "no candidate device path for this op set")
+    return best, results
+
+
 class Script:
     def __init__(self, model: "Model", handle: ct.c_void_p):
         self._model = model
@@ -291,7 +356,7 @@ class Model:
 
     def __init__(self, cell: str, H: int, E: int, C: int, device: int = 0, n_sm: int = 0, groups: int = 1,
                  plan_only: bool = False, cluster: int = 0, dataflow: bool = False, level: int = 0,
-                 mlp: int = 256, allocator: str = "torch"):
+                 mlp: int = 256, allocator: str = "torch", chain: int = 0):
         """allocator: "torch" (the library's device buffers come from torch's caching allocator) or
         "cuda" (the library's default, stream-ordered cudaMallocAsync)."""
         self.cell, self.H, self.E, self.C = cell, H, E, C
@@ -300,8 +365,9 @@ class Model:
         ops = _Opset(CELLS[cell], E, H, C, mlp)
         self._alloc_cbs = _torch_allocator(device) if (allocator == "torch" and not plan_only) else \
             (_ALLOC_FN(), _FREE_FN())
-        opt = _Options(n_sm, 1, groups, device, int(plan_only), cluster, int(dataflow), int(level),
+        opt = _Options(n_sm, 1, groups, device, int(plan_only), cluster, int(dataflow), int(level), int(chain),
                        self._alloc_cbs[0], self._alloc_cbs[1], None)
+        self.options = dict(groups=groups, cluster=cluster, dataflow=dataflow, level=level, chain=chain)
         h = ct.c_void_p()
         _check(_lib.vpps_define_model(sh, len(self.shapes), ct.byref(ops), ct.byref(opt), ct.byref(h)))
         self._h = h

@@ -548,3 +548,17 @@ def test_chain_tagger_paths_agree_subprocess():
     r = subprocess.run([sys.executable, "-c", code], env={**os.environ, "VPPS_CHAIN": "0"}, capture_output=True,
                        text=True, timeout=600)
     assert r.returncode == 0 and "ok" in r.stdout, r.stdout + r.stderr
+
+
+def test_autotune_on_device_then_parity():
+    """vpps.autotune times every device path this build offers for an LSTM LM at H = 256, C = 32 (grid kernel
+    at G = 1 / 2, chain recurrence, per-step products) on sample batches and keeps the fastest; the chosen
+    path then matches the oracle."""
+    vpps = _vpps()
+    rng = np.random.default_rng(500)
+    sample = [[synth.chain(rng, int(rng.integers(5, 40)), 32, lm=True) for _ in range(16)] for _ in range(2)]
+    X = torch.from_numpy(synth.input_table(rng, 32, 256)).float().cuda()
+    best, res = vpps.autotune("lstm", 256, 256, 32, sample, X)
+    assert len(res) >= 3 and min(res.values()) == res[repr(best)]
+    graphs = synth.config_batch("c3", 7, batch=16, V=32, C=32)
+    check("lstm", 256, 256, 32, graphs, 32, seed=501, groups=best.get("groups", 1), level=best.get("level", 0))

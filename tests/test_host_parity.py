@@ -259,3 +259,18 @@ def test_chain_table_bit_exact(vpps, cell, H, batch):
     # the table is the last block of the blob (tagger.cpp appends it after the step lists)
     assert np.array_equal(words[-n:], np.array(ref, dtype=np.int64)), (words[-n:][:8], ref[:8])
     assert words[-n] == G
+
+
+def test_autotune_picks_the_fastest_candidate(vpps):
+    """Profile-guided path choice: every candidate is timed and the fastest kept; candidates
+    that this build cannot instantiate are skipped (plan-only models stand in for devices here; the timer is
+    injected)."""
+    fake = {1: 3.0, 2: 1.5, 4: 2.0}
+    cands = [dict(groups=g, plan_only=True) for g in (1, 2, 4)] + [dict(groups=3, n_sm=16, plan_only=True)]
+    best, res = vpps.autotune("childsum", 8, 8, 5, [], None, candidates=cands,
+                              timer=lambda m, b, x: fake[m.options["groups"]])
+    assert best == dict(groups=2, plan_only=True)
+    assert min(res.values()) == 1.5
+    opts = vpps.candidate_options("binary", 256, 5)
+    assert opts[0] == dict(cluster=16, dataflow=True) and dict(level=1) in opts
+    assert vpps.candidate_options("gru", 256, 1000) == [dict(chain=0), dict(chain=-1)]
