@@ -50,16 +50,17 @@ __device__ __forceinline__ u64 tagv(float v, uint32_t e) { return ((u64)e << 32)
 __device__ __forceinline__ void st_tag(u64* p, float v, uint32_t e) {
     asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(tagv(v, e)) : "memory");
 }
-// L1-bypassing poll of one slot: an L2-cached (.cg) 8-byte load of an aligned slot that producers write
-// with one 8-byte store, so value and epoch arrive together.  (Strong ld.relaxed.gpu loads issue one at
-// a time: 17 of them took ~3.6K cycles where these pipeline like ordinary loads.)
+// Poll of one slot: a relaxed GPU-scope (morally strong, single-copy atomic) 8-byte load of an aligned slot
+// that producers write with one relaxed 8-byte store, so value and epoch arrive together and the race is
+// one the PTX memory model defines.  It compiles to the same LDG.E.64.STRONG.GPU as the earlier .cg form
+// (profiles/r2_poll_sass.txt) and pipelines like ordinary loads.
 __device__ __forceinline__ u64 ld_slot(const u64* p) {
     u64 v;
-    asm volatile("ld.global.cg.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
 __device__ __forceinline__ void ld_slot2(const u64* p, u64& a, u64& b) {
-    asm volatile("ld.global.cg.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+    asm volatile("ld.relaxed.gpu.global.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
 }
 __device__ __forceinline__ void st_tag4(u64* p, const float* v, uint32_t e) {
     asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(tagv(v[0], e)), "l"(tagv(v[1], e)) : "memory");
