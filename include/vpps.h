@@ -70,9 +70,15 @@ typedef enum {
                                      rows themselves (E = H), every inner node h = tanh(W [h_a; h_b] + b)
                                      with W H×2H, b H, and a node may feed two parents; W_out C×H, b_out C;
                                      level-synchronous path */
-    VPPS_CELL_TDLSTM = 7          /* M8 (DESIGN reading R-37): TREE_BINARY's cell and
+    VPPS_CELL_TDLSTM = 7,         /* M8 (DESIGN reading R-37): TREE_BINARY's cell and
                                      parameters on TD pyramid DAGs (a node may feed two parents, its dh and
                                      dc accumulate from both); level-synchronous path */
+    VPPS_CELL_BILSTM_CHAR = 8     /* M9 BiLSTMwChar (DESIGN reading R-38): the BiLSTM tagger
+                                     whose rare words (a node with a character spelling, vpps_batch.chars)
+                                     take [h→ after the last character; h← after the first] of a character
+                                     BiLSTM (hidden E/2 per direction, table C_emb Vc × Ec) as their input row;
+                                     their table rows get no gradient, C_emb does.  Chain recurrences for the
+                                     characters and the words; needs E/2 and H among the chain sizes */
 } vpps_cell;
 
 typedef struct {
@@ -87,7 +93,9 @@ typedef struct {
  *   LSTM:          W 4H×E, U 4H×H, W_out C×H, b 4H, b_out C
  *   TREE_BINARY:   W_iou 3H×E, U_iou 3H×2H, U_fl H×H, U_fr H×H, W_out C×H, b_iou 3H, b_f H, b_out C
  *   TREE_CHILDSUM: W_iou 3H×E, W_f H×E, U_iou 3H×H, U_f H×H, W_out C×H, b_iou 3H, b_f H, b_out C
- *   BILSTM_TAGGER: Wf 4H×E, Uf 4H×H, Wb 4H×E, Ub 4H×H, W_mlp M×2H, W_tag C×M, bf 4H, bb 4H, b_mlp M, b_tag C */
+ *   BILSTM_TAGGER: Wf 4H×E, Uf 4H×H, Wb 4H×E, Ub 4H×H, W_mlp M×2H, W_tag C×M, bf 4H, bb 4H, b_mlp M, b_tag C
+ *   BILSTM_CHAR:   the tagger's matrices, C_emb Vc×Ec, Wcf 4Hc×Ec, Ucf 4Hc×Hc, Wcb 4Hc×Ec, Ucb 4Hc×Hc, then the
+ *                  tagger's biases, bcf 4Hc, bcb 4Hc (Hc = E/2; Vc, Ec from C_emb's shape) */
 typedef struct {
     int32_t rows, cols;
 } vpps_shape;
@@ -140,6 +148,9 @@ typedef struct {
     const int32_t* children;  /* host [child_ptr[n_nodes]] graph-local indices       */
     const int32_t* token;     /* host [n_nodes] input-table row or -1                */
     const int32_t* label;     /* host [n_nodes] class of a loss head on this node, or -1 */
+    const int32_t* char_ptr;  /* host [n_nodes+1] or NULL: node v's spelling is chars[char_ptr[v] ..
+                                 char_ptr[v+1]) (BILSTM_CHAR only; an empty spelling = a frequent word) */
+    const int32_t* chars;     /* host character ids in [0, Vc)                      */
 } vpps_batch;
 
 typedef struct {

@@ -32,8 +32,14 @@ vpps_status cuda_fail(cudaError_t e, const char* what) {
         if (_e != cudaSuccess) return cuda_fail(_e, #call);    \
     } while (0)
 
-std::vector<Shape> expected_shapes(int32_t cell, int32_t H, int32_t E, int32_t C, int32_t M = 0) {
+std::vector<Shape> expected_shapes(int32_t cell, int32_t H, int32_t E, int32_t C, int32_t M = 0, int32_t Vc = 0,
+                                   int32_t Ec = 0) {
+    const int32_t Hc = E / 2;
     switch (cell) {
+        case CELL_BILSTM_CHAR:
+            return {{4 * H, E}, {4 * H, H}, {4 * H, E}, {4 * H, H}, {M, 2 * H}, {C, M}, {Vc, Ec}, {4 * Hc, Ec},
+                    {4 * Hc, Hc}, {4 * Hc, Ec}, {4 * Hc, Hc}, {4 * H, 1}, {4 * H, 1}, {M, 1}, {C, 1}, {4 * Hc, 1},
+                    {4 * Hc, 1}};
         case CELL_BILSTM:
             return {{4 * H, E}, {4 * H, H}, {4 * H, E}, {4 * H, H}, {M, 2 * H}, {C, M},
                     {4 * H, 1}, {4 * H, 1}, {M, 1}, {C, 1}};
@@ -123,10 +129,16 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     vpps_options o{};
     if (opt) o = *opt;
     const int32_t cell = ops->cell, H = ops->H, E = ops->E, C = ops->C, Mw = ops->mlp;
-    if (cell < 0 || cell > 7 || H <= 0 || E <= 0 || C <= 0) return fail(VPPS_E_INVALID, "bad op set");
+    if (cell < 0 || cell > 8 || H <= 0 || E <= 0 || C <= 0) return fail(VPPS_E_INVALID, "bad op set");
     if (cell == CELL_TDRNN && E != H) return fail(VPPS_E_INVALID, "TD-RNN: the leaves are the input rows (E == H)");
-    if (cell == CELL_BILSTM && Mw <= 0) return fail(VPPS_E_INVALID, "BiLSTM tagger needs mlp > 0");
-    std::vector<Shape> want = expected_shapes(cell, H, E, C, Mw);
+    if ((cell == CELL_BILSTM || cell == CELL_BILSTM_CHAR) && Mw <= 0)
+        return fail(VPPS_E_INVALID, "BiLSTM tagger needs mlp > 0");
+    // BiLSTMwChar: the character table's shape (parameter 6, Vc x Ec) sets Vc and Ec; E must be even
+    const int32_t Vc = cell == CELL_BILSTM_CHAR && n_params > 6 ? params[6].rows : 0;
+    const int32_t Ec = cell == CELL_BILSTM_CHAR && n_params > 6 ? params[6].cols : 0;
+    if (cell == CELL_BILSTM_CHAR && (E % 2 || Vc <= 0 || Ec <= 0 || Ec % 4))
+        return fail(VPPS_E_INVALID, "BiLSTMwChar: E even, C_emb Vc x Ec with Ec a multiple of 4");
+    std::vector<Shape> want = expected_shapes(cell, H, E, C, Mw, Vc, Ec);
     if ((int32_t)want.size() != n_params) return fail(VPPS_E_INVALID, "wrong number of parameters for the op set");
     for (int32_t i = 0; i < n_params; ++i)
         if (params[i].rows != want[i].rows || params[i].cols != want[i].cols)
@@ -150,7 +162,8 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     }
     m->n_floats = cur;
     int32_t n_sm = o.n_sm;
-    if (cell == CELL_BILSTM || cell == CELL_GRU || cell == CELL_RVNN || cell == CELL_TDRNN || cell == CELL_TDLSTM ||
+    if (cell == CELL_BILSTM || cell == CELL_BILSTM_CHAR || cell == CELL_GRU || cell == CELL_RVNN || cell == CELL_TDRNN ||
+        cell == CELL_TDLSTM ||
         (cell == CELL_LSTM && (o.level > 0 || (o.level == 0 && C > 32)))) {
         // M2 and M5 (GRU) run on the level-synchronous path only (vpps_level.cu), and so does an LSTM LM
         // whose vocabulary head exceeds one CTA's shared memory (config 3 at V = 1000): no partition plan
@@ -166,7 +179,9 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
             m->plan.cell = cell; m->plan.H = H; m->plan.E = E; m->plan.C = C;
             m->plan.n_cta = m->plan.n_g = m->plan.n_act = m->plan.umax = m->plan.G = 1;
         }
-        m->plan.mlp = cell == CELL_BILSTM ? Mw : 0;
+        m->plan.mlp = cell == CELL_BILSTM || cell == CELL_BILSTM_CHAR ? Mw : 0;
+        m->plan.vc = Vc;
+        m->plan.ec = Ec;
         m->plan.level = true;
         int32_t sms = 148;
         if (!m->plan_only) {
@@ -180,9 +195,16 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
         // LSTM chains: the recurrence runs register-resident in groups of co-resident CTAs (vpps_chain.cu)
         // when a specialisation exists for H; VPPS_CHAIN=0 (measurement) keeps the per-step products
         static const bool chain_env = !(getenv("VPPS_CHAIN") && atoi(getenv("VPPS_CHAIN")) == 0);
-        if ((cell == CELL_BILSTM || cell == CELL_LSTM || cell == CELL_GRU) && chain_env && o.chain >= 0) {
-            const int32_t ncl = chain_group_ctas(H), dirs = cell == CELL_BILSTM ? 2 : 1;
+        if ((cell == CELL_BILSTM || cell == CELL_BILSTM_CHAR || cell == CELL_LSTM || cell == CELL_GRU) && chain_env &&
+            o.chain >= 0) {
+            const int32_t ncl = chain_group_ctas(H), dirs = cell == CELL_BILSTM || cell == CELL_BILSTM_CHAR ? 2 : 1;
             m->plan.chain_g = ncl > 0 ? (sms / ncl) / dirs : 0;
+        }
+        if (cell == CELL_BILSTM_CHAR) {
+            // the character BiLSTM runs only on the chain recurrence (H_c = E / 2 must be a built size)
+            const int32_t ncl = chain_group_ctas(E / 2);
+            if (ncl <= 0) return fail(VPPS_E_NOFIT, "BiLSTMwChar: no chain specialisation for H_c = E / 2");
+            m->plan.chain_gc = (sms / ncl) / 2;
         }
         if (!m->plan_only) {
             m->level = level_ctx_create(&m->alloc);
@@ -377,10 +399,12 @@ vpps_status vpps_build_script(vpps_model m, const vpps_batch* batch, vpps_script
     std::unique_ptr<vpps_script_s> s(new (std::nothrow) vpps_script_s);
     if (!s) return fail(VPPS_E_NOMEM, "out of host memory");
     s->model = m;
-    BatchIn b{batch->n_graphs, batch->graph_ptr, batch->child_ptr, batch->children, batch->token, batch->label};
+    BatchIn b{batch->n_graphs, batch->graph_ptr, batch->child_ptr, batch->children, batch->token, batch->label,
+              batch->char_ptr, batch->chars};
     std::string err;
     // the input table's row count is not known here; token range is re-checked against it at run time
-    const bool chains = m->plan.level && (m->plan.cell == CELL_BILSTM || m->plan.cell == CELL_LSTM ||
+    const bool chains = m->plan.level && (m->plan.cell == CELL_BILSTM || m->plan.cell == CELL_BILSTM_CHAR ||
+                                          m->plan.cell == CELL_LSTM ||
                                           m->plan.cell == CELL_GRU);
     int rc = 0;
     if (chains && m->plan.cell == CELL_LSTM) {
@@ -661,6 +685,18 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
                                 s->s.loss_word, st, s->s.tg_chain >= 0 ? dwords + s->s.tg_chain : nullptr,
                                 m->plan.chain_g);
         if (rc != 0) return fail(VPPS_E_CUDA, "GRU pass failed (code " + std::to_string(rc) + ")");
+        if (mode == 1) launch_sgd(m->params, m->grads, m->n_floats, lr, wd, st);
+    } else if (m->plan.level && m->plan.cell == CELL_BILSTM_CHAR) {
+        if (s->s.tg_tok < 0) return fail(VPPS_E_INVALID, "script was not built for the level path");
+        CK(cudaMemsetAsync(m->grads, 0, (size_t)m->n_floats * sizeof(float), st));
+        const int rc = bilstmchar_pass(m->level, m->params, m->offsets.data(), m->grads, m->pool, inputs, d_inputs,
+                                       dwords, s->s.tg_tok, s->s.tg_lab, s->s.tg_fpos, s->s.tg_bpos,
+                                       s->s.tg_start.data(), (int32_t)s->s.tg_start.size() - 1, s->s.tg_T, m->plan.H,
+                                       m->plan.E, m->plan.C, m->plan.mlp, s->s.loss_word, st,
+                                       s->s.tg_chain >= 0 ? dwords + s->s.tg_chain : nullptr, m->plan.chain_g,
+                                       s->s.tc_T, s->s.tc_R, s->s.tc_tok, s->s.tc_word, s->s.tc_rare, s->s.tc_list,
+                                       s->s.tc_chain, m->plan.chain_gc, m->plan.ec);
+        if (rc != 0) return fail(VPPS_E_CUDA, "BiLSTMwChar pass failed (code " + std::to_string(rc) + ")");
         if (mode == 1) launch_sgd(m->params, m->grads, m->n_floats, lr, wd, st);
     } else if (m->plan.level && (m->plan.cell == CELL_BILSTM || m->plan.cell == CELL_LSTM)) {
         if (s->s.tg_tok < 0) return fail(VPPS_E_INVALID, "script was not built for the level path");

@@ -9,7 +9,7 @@ namespace vpps {
 
 constexpr uint32_t NONE = 0xFFFFFFFFu;
 
-enum Cell : int32_t { CELL_LSTM = 0, CELL_BINARY = 1, CELL_CHILDSUM = 2, CELL_BILSTM = 3, CELL_GRU = 4, CELL_RVNN = 5, CELL_TDRNN = 6, CELL_TDLSTM = 7 };
+enum Cell : int32_t { CELL_LSTM = 0, CELL_BINARY = 1, CELL_CHILDSUM = 2, CELL_BILSTM = 3, CELL_GRU = 4, CELL_RVNN = 5, CELL_TDRNN = 6, CELL_TDLSTM = 7, CELL_BILSTM_CHAR = 8 };
 
 enum Op : uint32_t {
     OP_S = 0x01, OP_W = 0x02,
@@ -36,6 +36,8 @@ struct Plan {
     int32_t n_cta, n_g, n_act, umax, G;
     bool by_graph = false;   // SPEC S5g: whole graphs assigned to groups (cluster replicas)
     bool level = false;      // level-synchronous GEMM path (binary cell, weights L2-resident)
+    int32_t vc = 0, ec = 0;  // BiLSTMwChar: characters and character-embedding width (C_emb is Vc x Ec)
+    int32_t chain_gc = 0;    // BiLSTMwChar: chain groups per direction of the character recurrence (H_c = E/2)
     int32_t chain_g = 0;     // chain cells on the level path: groups per direction of the register-resident
                              // recurrence (vpps_chain.cu); 0 = per-step products
     bool skip_words = false; // dataflow models: the SPEC words (S4-S6, §E) are not built with the device
@@ -53,6 +55,8 @@ struct BatchIn {
     const int32_t* children;
     const int32_t* token;
     const int32_t* label;
+    const int32_t* char_ptr = nullptr;   // BiLSTMwChar spellings (CSR over the nodes) or nullptr
+    const int32_t* chars = nullptr;
 };
 
 struct Script {
@@ -85,6 +89,11 @@ struct Script {
     // batch order, starting at fstart[t]) and the backward step lists bpos[T] (position len-1-t)
     int64_t tg_T = 0, tg_tok = -1, tg_lab = -1, tg_fpos = -1, tg_bpos = -1;
     int64_t tg_chain = -1;           // blob offset of the chain-recurrence sentence table (SPEC §L), or -1
+    // BiLSTMwChar (SPEC §L): R rare positions, Tc character positions (spellings concatenated in position
+    // order); blob offsets of ctok[Tc] (character ids), cword[Tc] (rare index of each character position),
+    // rare[T] (rare index of a word position or NONE), rlist[R][3] (word position, character offset,
+    // length) and the character chain table
+    int64_t tc_T = 0, tc_R = 0, tc_tok = -1, tc_word = -1, tc_rare = -1, tc_list = -1, tc_chain = -1;
     std::vector<int32_t> tg_start;   // [maxlen + 1]
 };
 

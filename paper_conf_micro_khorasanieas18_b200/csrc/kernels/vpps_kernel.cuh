@@ -145,11 +145,25 @@ int tdrnn_pass(void* ctx, const float* params, const int64_t* off, float* grads,
                float* d_inputs, const uint32_t* d_blob, int64_t lv_int, int64_t lv_leaf, int64_t lv_head,
                const int32_t* lv_start, int32_t L, int64_t n_int, int64_t n_leaf, int64_t n_head, int32_t H,
                int32_t E, int32_t C, int64_t loss_word, cudaStream_t s);
+// BiLSTMwChar: the character recurrence's outputs and the rare-word lists the word tagger reads
+struct CharRows {
+    const uint32_t* rare;    // [T] rare index of a word position or NONE
+    const uint32_t* rlist;   // [R][3] word position, character offset, length
+    const float* HHc;        // [Tc][E] character h of both directions (E = 2 Hc)
+};
 int tagger_pass(void* ctx, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
                 float* d_inputs, const uint32_t* d_blob, int64_t tg_tok, int64_t tg_lab, int64_t tg_fpos,
                 int64_t tg_bpos, const int32_t* start, int32_t maxlen, int64_t T, int32_t H, int32_t E, int32_t C,
                 int32_t Mw, int32_t dirs, int64_t loss_word, cudaStream_t s, const uint32_t* chain_table = nullptr,
-                int32_t chain_g = 0);
+                int32_t chain_g = 0, const CharRows* cr = nullptr);
+// BiLSTMwChar (M9): character BiLSTM (chain recurrence) -> word rows -> tagger_pass -> character backward and
+// the gradients of C_emb and the character LSTMs.  off: the 17 parameter offsets in vpps.h order.
+int bilstmchar_pass(void* ctx, const float* params, const int64_t* off, float* grads, float* pool,
+                    const float* inputs, float* d_inputs, const uint32_t* d_blob, int64_t tg_tok, int64_t tg_lab,
+                    int64_t tg_fpos, int64_t tg_bpos, const int32_t* start, int32_t maxlen, int64_t T, int32_t H,
+                    int32_t E, int32_t C, int32_t Mw, int64_t loss_word, cudaStream_t s, const uint32_t* chain_table,
+                    int32_t chain_g, int64_t tc_T, int64_t tc_R, int64_t tc_tok, int64_t tc_word, int64_t tc_rare,
+                    int64_t tc_list, int64_t tc_chain, int32_t chain_gc, int32_t Ec);
 int gru_pass(void* ctx, const float* params, const int64_t* off, float* grads, float* pool, const float* inputs,
              float* d_inputs, const uint32_t* d_blob, int64_t tg_tok, int64_t tg_lab, int64_t tg_fpos,
              const int32_t* start, int32_t maxlen, int64_t T, int32_t H, int32_t E, int32_t C, int64_t loss_word,

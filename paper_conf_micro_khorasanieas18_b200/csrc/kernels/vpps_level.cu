@@ -334,7 +334,51 @@ __global__ void tg_hprev_all(const float* __restrict__ HH, const uint32_t* __res
 __global__ void tg_scatter_dx(const float* __restrict__ DX, const uint32_t* __restrict__ tok, int T, int E, float* dX) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)T * E) return;
-    atomicAdd(dX + (int64_t)tok[t / E] * E + t % E, DX[t]);
+    const uint32_t k = tok[t / E];
+    if (k != NONE) atomicAdd(dX + (int64_t)k * E + t % E, DX[t]);   // (BiLSTMwChar's rare words: no table row)
+}
+
+// ---- BiLSTMwChar (M9, reading R-38) ----
+// word input rows: the table row of a frequent word, [h→ at the last character; h← at the first character]
+// of the character BiLSTM (HHc [Tc][2 Hc]) for a rare word
+__global__ void wc_gather_x(const float* __restrict__ inputs, const uint32_t* __restrict__ tok,
+                            const uint32_t* __restrict__ rare, const uint32_t* __restrict__ rlist,
+                            const float* __restrict__ HHc, int T, int E, float* __restrict__ X) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= (int64_t)T * E) return;
+    const int p = (int)(i / E), j = (int)(i % E), Hc = E / 2;
+    const uint32_t k = tok[p];
+    float v;
+    if (k != NONE) {
+        v = __ldg(inputs + (int64_t)k * E + j);
+    } else {
+        const uint32_t* e = rlist + 3 * rare[p];
+        const int64_t q = j < Hc ? (int64_t)e[1] + e[2] - 1 : (int64_t)e[1];   // last / first character
+        v = HHc[q * E + j];
+    }
+    X[i] = v;
+}
+// dh seeds of the character chains: a rare word's dX row enters at the forward direction's last character
+// (columns 0 .. Hc) and at the backward direction's first character (Hc .. 2 Hc); dHHc zeroed before
+__global__ void wc_seed(const float* __restrict__ DX, const uint32_t* __restrict__ rlist, int R, int E,
+                        float* __restrict__ dHHc) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= (int64_t)R * E) return;
+    const int r = (int)(i / E), j = (int)(i % E), Hc = E / 2;
+    const uint32_t* e = rlist + 3 * r;
+    const int64_t q = j < Hc ? (int64_t)e[1] + e[2] - 1 : (int64_t)e[1];
+    dHHc[q * E + j] = DX[(int64_t)e[0] * E + j];
+}
+// h_{t-1} of every character position in direction d (0 at a spelling's start in that direction)
+__global__ void wc_hprev(const float* __restrict__ HHc, const uint32_t* __restrict__ cword,
+                         const uint32_t* __restrict__ rlist, int Tc, int Hc, int d, float* __restrict__ Hp) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= (int64_t)Tc * Hc) return;
+    const int q = (int)(i / Hc), j = (int)(i % Hc);
+    const uint32_t* e = rlist + 3 * cword[q];
+    const int k = q - (int)e[1];                       // index inside the spelling
+    const bool has = d == 0 ? k > 0 : k + 1 < (int)e[2];
+    Hp[i] = has ? HHc[(int64_t)(d == 0 ? q - 1 : q + 1) * 2 * Hc + d * Hc + j] : 0.f;
 }
 
 
@@ -505,6 +549,12 @@ struct TaggerBufs {
     int64_t cap3[5] = {0};
 };
 
+struct CharBufs {
+    float *Xc = nullptr, *Pf = nullptr, *Pb = nullptr, *HH = nullptr, *Cf = nullptr, *Cb = nullptr, *Gf = nullptr,
+          *Gb = nullptr, *dHH = nullptr, *Gamf = nullptr, *Gamb = nullptr, *Hp = nullptr, *DX = nullptr;
+    int64_t cap[13] = {0};
+};
+
 struct LevelCtx {
     DevAlloc alloc;
     cudaStream_t st = nullptr;         // stream of the pass in progress (the products run on it)
@@ -514,6 +564,9 @@ struct LevelCtx {
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     LevelBufs b;
     TaggerBufs tg;
+    // BiLSTMwChar's character BiLSTM: X_c, P_f, P_b, HH (both directions), C_f, C_b, G_f, G_b, dHH, Γ_f, Γ_b,
+    // H_prev, DX_c
+    CharBufs ch;
     // register-resident chain recurrence (vpps_chain.cu): tagged slots, zeroed when (re)allocated; pass tag
     float *hx = nullptr, *part = nullptr;
     int64_t cap_hx = 0, cap_part = 0;
@@ -548,6 +601,9 @@ void level_ctx_destroy(void* p) {
     for (float* q : tbufs) c->alloc.put(q, nullptr);
     c->alloc.put(c->hx, nullptr);
     c->alloc.put(c->part, nullptr);
+    CharBufs& cb = c->ch;
+    float* cbufs[] = {cb.Xc, cb.Pf, cb.Pb, cb.HH, cb.Cf, cb.Cb, cb.Gf, cb.Gb, cb.dHH, cb.Gamf, cb.Gamb, cb.Hp, cb.DX};
+    for (float* q : cbufs) c->alloc.put(q, nullptr);
     delete c;
 }
 
@@ -640,7 +696,7 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
                 float* d_inputs, const uint32_t* d_blob, int64_t tg_tok, int64_t tg_lab, int64_t tg_fpos,
                 int64_t tg_bpos, const int32_t* start, int32_t maxlen, int64_t T, int32_t H, int32_t E, int32_t C,
                 int32_t Mw, int32_t dirs, int64_t loss_word, cudaStream_t s, const uint32_t* chain_table,
-                int32_t chain_g) {
+                int32_t chain_g, const CharRows* cr) {
     // off: parameter offsets (Wf, Uf, Wb, Ub, W_mlp, W_tag, bf, bb, b_mlp, b_tag); dirs = 1 is the LSTM LM
     // (M1: W, U, -, -, -, W_out, b, -, -, b_out; the head reads h directly), Mw = 0 without the MLP
     using namespace dev::lv;
@@ -678,7 +734,8 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
     cudaError_t st;
 #define BL(call) do { st = (call); if (st != cudaSuccess) return 1000 + (int)st; } while (0)
     if (T == 0) return 0;
-    tg_gather_x<<<nblk(T * (E / 4)), 256, 0, s>>>(inputs, tok, (int)T, E, tb.X);
+    if (cr) wc_gather_x<<<nblk(T * E), 256, 0, s>>>(inputs, tok, cr->rare, cr->rlist, cr->HHc, (int)T, E, tb.X);
+    else tg_gather_x<<<nblk(T * (E / 4)), 256, 0, s>>>(inputs, tok, (int)T, E, tb.X);
     BL(gemm_rm(c->st, false, true, (int)T, 4 * H, E, tb.X, E, Wf, E, tb.Pf, 4 * H, 0.f));
     if (dirs > 1) BL(gemm_rm(c->st, false, true, (int)T, 4 * H, E, tb.X, E, Wb, E, tb.Pb, 4 * H, 0.f));
     // register-resident recurrence (vpps_chain.cu): U of each direction in the registers of a group of CTAs,
@@ -810,10 +867,10 @@ int tagger_pass(void* ctx_, const float* params, const int64_t* off, float* grad
         BL(gemm_rm(c->st, true, false, 4 * H, H, (int)T, Gam, 4 * H, tb.Hp, H, grads + off[d == 0 ? 1 : 3], H, 0.f));
         colsum<<<nblk(4 * H), 256, 0, s>>>(Gam, (int)T, 4 * H, grads + off[d == 0 ? 6 : 7]);
     }
-    if (d_inputs) {
+    if (d_inputs || cr) {   // (BiLSTMwChar: the rare rows' dX seeds the character chains, cr->DX = tb.DX)
         BL(gemm_rm(c->st, false, false, (int)T, E, 4 * H, tb.Gamf, 4 * H, Wf, E, tb.DX, E, 0.f));
         if (dirs > 1) BL(gemm_rm(c->st, false, false, (int)T, E, 4 * H, tb.Gamb, 4 * H, Wb, E, tb.DX, E, 1.f));
-        tg_scatter_dx<<<nblk(T * E), 256, 0, s>>>(tb.DX, tok, (int)T, E, d_inputs);
+        if (d_inputs) tg_scatter_dx<<<nblk(T * E), 256, 0, s>>>(tb.DX, tok, (int)T, E, d_inputs);
     }
 #undef BL
     return (int)cudaGetLastError();
@@ -1046,6 +1103,104 @@ int tdrnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads
         BL(gemm_rm(c->st, true, false, H, 2 * H, (int)n_int, Gi, H, Xi, 2 * H, grads + off[0], 2 * H, 0.f));
         colsum<<<nblk(H), 256, 0, s>>>(Gi, (int)n_int, H, grads + off[2]);
     }
+#undef BL
+    return (int)cudaGetLastError();
+}
+
+}  // namespace vpps
+
+namespace vpps {
+
+// BiLSTMwChar (M9, PAPER L267 / L281, reading R-38).  The rare words' spellings run through a character
+// BiLSTM on the chain recurrence (hidden Hc = E / 2 per direction; C_emb rows as its inputs, W_c x as one
+// GEMM per direction), its final states become the rare positions' input rows of the word tagger
+// (tagger_pass with CharRows), and the tagger's dX rows of those positions seed dh at the final states of the
+// character chains on the way back; dW / dU / db of the character LSTMs and dC_emb (scatter of Γ W_c by
+// character id) as dense products.  The character passes tag their slots with their own pass counter value.
+int bilstmchar_pass(void* ctx_, const float* params, const int64_t* off, float* grads, float* pool,
+                    const float* inputs, float* d_inputs, const uint32_t* d_blob, int64_t tg_tok, int64_t tg_lab,
+                    int64_t tg_fpos, int64_t tg_bpos, const int32_t* start, int32_t maxlen, int64_t T, int32_t H,
+                    int32_t E, int32_t C, int32_t Mw, int64_t loss_word, cudaStream_t s, const uint32_t* chain_table,
+                    int32_t chain_g, int64_t tc_T, int64_t tc_R, int64_t tc_tok, int64_t tc_word, int64_t tc_rare,
+                    int64_t tc_list, int64_t tc_chain, int32_t chain_gc, int32_t Ec) {
+    using namespace dev::lv;
+    LevelCtx* c = static_cast<LevelCtx*>(ctx_);
+    c->st = s;
+    const int32_t Hc = E / 2;
+    const int64_t Tc = tc_T, R = tc_R;
+    const int64_t off10[10] = {off[0], off[1], off[2], off[3], off[4], off[5], off[11], off[12], off[13], off[14]};
+    const uint32_t* ctok = d_blob + tc_tok;
+    const uint32_t* cword = d_blob + tc_word;
+    CharRows cr{d_blob + tc_rare, d_blob + tc_list, nullptr};
+    cudaError_t st;
+#define BL(call) do { st = (call); if (st != cudaSuccess) return 1000 + (int)st; } while (0)
+    ChainParams cp{};
+    uint32_t e_chars = 0;
+    const int32_t ncl = chain_group_ctas(Hc);
+    CharBufs& cb = c->ch;
+    if (R > 0) {
+        if (tc_chain < 0 || ncl <= 0) return (int)cudaErrorInvalidValue;
+        const int64_t Tn = std::max<int64_t>(Tc, 1);
+        float** bufs[13] = {&cb.Xc, &cb.Pf, &cb.Pb, &cb.HH, &cb.Cf, &cb.Cb, &cb.Gf, &cb.Gb, &cb.dHH, &cb.Gamf, &cb.Gamb,
+                            &cb.Hp, &cb.DX};
+        const int64_t need[13] = {Tn * Ec, Tn * 4 * Hc, Tn * 4 * Hc, Tn * E, Tn * Hc, Tn * Hc, Tn * 4 * Hc, Tn * 4 * Hc,
+                                  Tn * E, Tn * 4 * Hc, Tn * 4 * Hc, Tn * Hc, Tn * Ec};
+        for (int k = 0; k < 13; ++k)
+            if (!grow(bufs[k], &cb.cap[k], need[k])) return (int)cudaErrorMemoryAllocation;
+        const int64_t need_hx = 2 * 2 * Tc * Hc, need_part = 2 * 2 * Tc * (int64_t)ncl * Hc;
+        if (need_hx > c->cap_hx) {
+            if (!grow(&c->hx, &c->cap_hx, need_hx)) return (int)cudaErrorMemoryAllocation;
+            cudaMemsetAsync(c->hx, 0, (size_t)c->cap_hx * sizeof(float), s);
+        }
+        if (need_part > c->cap_part) {
+            if (!grow(&c->part, &c->cap_part, need_part)) return (int)cudaErrorMemoryAllocation;
+            cudaMemsetAsync(c->part, 0, (size_t)c->cap_part * sizeof(float), s);
+        }
+        if (++c->epoch == 0) c->epoch = 1;
+        e_chars = c->epoch;
+        const float *Cemb = params + off[6], *Wcf = params + off[7], *Ucf = params + off[8], *Wcb = params + off[9],
+                    *Ucb = params + off[10], *bcf = params + off[15], *bcb = params + off[16];
+        // character BiLSTM forward: C_emb rows, input projections, the recurrence of both directions
+        tg_gather_x<<<nblk(Tc * (Ec / 4)), 256, 0, s>>>(Cemb, ctok, (int)Tc, Ec, cb.Xc);
+        BL(gemm_rm(s, false, true, (int)Tc, 4 * Hc, Ec, cb.Xc, Ec, Wcf, Ec, cb.Pf, 4 * Hc, 0.f));
+        BL(gemm_rm(s, false, true, (int)Tc, 4 * Hc, Ec, cb.Xc, Ec, Wcb, Ec, cb.Pb, 4 * Hc, 0.f));
+        cp.table = d_blob + tc_chain;
+        cp.groups_dir0 = chain_gc;
+        cp.HW = E;
+        cp.epoch = e_chars;
+        cp.U0 = Ucf; cp.U1 = Ucb; cp.b0 = bcf; cp.b1 = bcb;
+        cp.P0 = cb.Pf; cp.P1 = cb.Pb;
+        cp.HH = cb.HH;
+        cp.C0 = cb.Cf; cp.C1 = cb.Cb; cp.G0 = cb.Gf; cp.G1 = cb.Gb;
+        cp.dHH = cb.dHH;
+        cp.Gam0 = cb.Gamf; cp.Gam1 = cb.Gamb;
+        cp.hx = reinterpret_cast<unsigned long long*>(c->hx);
+        cp.part = reinterpret_cast<unsigned long long*>(c->part);
+        cp.T = Tc;
+        BL(launch_chain(cp, Hc, 2 * chain_gc, false, s));
+        cr.HHc = cb.HH;
+    }
+    // the word tagger over the rows [table row | character states]
+    int rc = tagger_pass(ctx_, params, off10, grads, pool, inputs, d_inputs, d_blob, tg_tok, tg_lab, tg_fpos, tg_bpos,
+                         start, maxlen, T, H, E, C, Mw, 2, loss_word, s, chain_table, chain_g, R > 0 ? &cr : nullptr);
+    if (rc != 0 || R == 0) return rc;
+    // character backward: seeds from the rare rows' dX, the recurrence, then the parameter gradients
+    cudaMemsetAsync(cb.dHH, 0, (size_t)Tc * E * sizeof(float), s);
+    wc_seed<<<nblk(R * E), 256, 0, s>>>(c->tg.DX, d_blob + tc_list, (int)R, E, cb.dHH);
+    cp.hx = reinterpret_cast<unsigned long long*>(c->hx);       // (the word pass may have grown the slots)
+    cp.part = reinterpret_cast<unsigned long long*>(c->part);
+    BL(launch_chain(cp, Hc, 2 * chain_gc, true, s));
+    const float *Wcf = params + off[7], *Wcb = params + off[9];
+    for (int d = 0; d < 2; ++d) {
+        float* Gam = d == 0 ? cb.Gamf : cb.Gamb;
+        wc_hprev<<<nblk(Tc * Hc), 256, 0, s>>>(cb.HH, cword, d_blob + tc_list, (int)Tc, Hc, d, cb.Hp);
+        BL(gemm_rm(s, true, false, 4 * Hc, Ec, (int)Tc, Gam, 4 * Hc, cb.Xc, Ec, grads + off[d == 0 ? 7 : 9], Ec, 0.f));
+        BL(gemm_rm(s, true, false, 4 * Hc, Hc, (int)Tc, Gam, 4 * Hc, cb.Hp, Hc, grads + off[d == 0 ? 8 : 10], Hc, 0.f));
+        colsum<<<nblk(4 * Hc), 256, 0, s>>>(Gam, (int)Tc, 4 * Hc, grads + off[d == 0 ? 15 : 16]);
+    }
+    BL(gemm_rm(s, false, false, (int)Tc, Ec, 4 * Hc, cb.Gamf, 4 * Hc, Wcf, Ec, cb.DX, Ec, 0.f));
+    BL(gemm_rm(s, false, false, (int)Tc, Ec, 4 * Hc, cb.Gamb, 4 * Hc, Wcb, Ec, cb.DX, Ec, 1.f));
+    tg_scatter_dx<<<nblk(Tc * Ec), 256, 0, s>>>(cb.DX, ctok, (int)Tc, Ec, grads + off[6]);
 #undef BL
     return (int)cudaGetLastError();
 }

@@ -15,7 +15,8 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libvpps.so")
 
-CELLS = {"lstm": 0, "binary": 1, "childsum": 2, "bilstm": 3, "gru": 4, "rvnn": 5, "tdrnn": 6, "tdlstm": 7}
+CELLS = {"lstm": 0, "binary": 1, "childsum": 2, "bilstm": 3, "gru": 4, "rvnn": 5, "tdrnn": 6, "tdlstm": 7,
+         "bilstmchar": 8}
 STATUS = {0: "OK", -1: "INVALID", -2: "NOFIT", -3: "CUDA", -4: "GRAPH", -5: "STATE", -6: "NOMEM"}
 
 
@@ -65,7 +66,8 @@ def _torch_allocator(device: int):
 
 class _Batch(ct.Structure):
     _fields_ = [("n_graphs", ct.c_int32), ("graph_ptr", ct.c_void_p), ("child_ptr", ct.c_void_p),
-                ("children", ct.c_void_p), ("token", ct.c_void_p), ("label", ct.c_void_p)]
+                ("children", ct.c_void_p), ("token", ct.c_void_p), ("label", ct.c_void_p),
+                ("char_ptr", ct.c_void_p), ("chars", ct.c_void_p)]
 
 
 class _Info(ct.Structure):
@@ -137,8 +139,16 @@ def _stream_ptr(stream):
     return ct.c_void_p(stream.cuda_stream)
 
 
-def param_shapes(cell: str, H: int, E: int, C: int, mlp: int = 256):
+def param_shapes(cell: str, H: int, E: int, C: int, mlp: int = 256, Ec: int = 64, Vc: int = 64):
     """Parameter order of vpps_define_model (include/vpps.h); bias shapes are (n,)."""
+    if cell == "bilstmchar":
+        Hc = E // 2
+        return [("Wf", (4 * H, E)), ("Uf", (4 * H, H)), ("Wb", (4 * H, E)), ("Ub", (4 * H, H)),
+                ("W_mlp", (mlp, 2 * H)), ("W_tag", (C, mlp)),
+                ("C_emb", (Vc, Ec)), ("Wcf", (4 * Hc, Ec)), ("Ucf", (4 * Hc, Hc)), ("Wcb", (4 * Hc, Ec)),
+                ("Ucb", (4 * Hc, Hc)),
+                ("bf", (4 * H,)), ("bb", (4 * H,)), ("b_mlp", (mlp,)), ("b_tag", (C,)),
+                ("bcf", (4 * Hc,)), ("bcb", (4 * Hc,))]
     if cell == "bilstm":
         return [("Wf", (4 * H, E)), ("Uf", (4 * H, H)), ("Wb", (4 * H, E)), ("Ub", (4 * H, H)),
                 ("W_mlp", (mlp, 2 * H)), ("W_tag", (C, mlp)),
@@ -199,7 +209,8 @@ def paper_choose_cps(mats, n_sm, tb=256, rpw=1, pack_rows=True):
 
 
 def to_csr(graphs):
-    """Graphs as lists of (children, token, label) -> CSR int32 arrays of vpps_batch."""
+    """Graphs as lists of (children, token, label[, chars]) -> CSR int32 arrays of vpps_batch (the last two,
+    the BiLSTMwChar spellings, are None when no node has a fourth element)."""
     nodes = [n for g in graphs for n in g]
     nn = len(nodes)
     gp = np.zeros(len(graphs) + 1, np.int32)
@@ -209,15 +220,22 @@ def to_csr(graphs):
     ch = np.fromiter(itertools.chain.from_iterable(n[0] for n in nodes), np.int32, int(cp[-1]))
     tok = np.fromiter((n[1] for n in nodes), np.int32, nn)
     lab = np.fromiter((n[2] for n in nodes), np.int32, nn)
-    return gp, cp, ch if ch.size else np.zeros(1, np.int32), tok, lab
+    chp = chs = None
+    if any(len(n) > 3 for n in nodes):
+        chp = np.zeros(nn + 1, np.int32)
+        np.cumsum(np.fromiter((len(n[3]) if len(n) > 3 else 0 for n in nodes), np.int32, nn), out=chp[1:])
+        chs = np.fromiter(itertools.chain.from_iterable(n[3] for n in nodes if len(n) > 3), np.int32, int(chp[-1]))
+        chs = chs if chs.size else np.zeros(1, np.int32)
+    return gp, cp, ch if ch.size else np.zeros(1, np.int32), tok, lab, chp, chs
 
 
 class CsrBatch:
     """A batch in the CSR form of vpps_batch (include/vpps.h): graph_ptr, child_ptr, children, token, label."""
 
-    def __init__(self, graph_ptr, child_ptr, children, token, label):
+    def __init__(self, graph_ptr, child_ptr, children, token, label, char_ptr=None, chars=None):
         as32 = lambda a: np.ascontiguousarray(np.asarray(a, dtype=np.int32))
         self.arrays = (as32(graph_ptr), as32(child_ptr), as32(children), as32(token), as32(label))
+        self.chars = (as32(char_ptr), as32(chars)) if char_ptr is not None else (None, None)
 
     @classmethod
     def from_graphs(cls, graphs):
@@ -356,11 +374,11 @@ class Model:
 
     def __init__(self, cell: str, H: int, E: int, C: int, device: int = 0, n_sm: int = 0, groups: int = 1,
                  plan_only: bool = False, cluster: int = 0, dataflow: bool = False, level: int = 0,
-                 mlp: int = 256, allocator: str = "torch", chain: int = 0):
+                 mlp: int = 256, allocator: str = "torch", chain: int = 0, Ec: int = 64, Vc: int = 64):
         """allocator: "torch" (the library's device buffers come from torch's caching allocator) or
         "cuda" (the library's default, stream-ordered cudaMallocAsync)."""
         self.cell, self.H, self.E, self.C = cell, H, E, C
-        self.shapes = param_shapes(cell, H, E, C, mlp)
+        self.shapes = param_shapes(cell, H, E, C, mlp, Ec, Vc)
         sh = (_Shape * len(self.shapes))(*[_Shape(s[0], s[1] if len(s) == 2 else 1) for _, s in self.shapes])
         ops = _Opset(CELLS[cell], E, H, C, mlp)
         self._alloc_cbs = _torch_allocator(device) if (allocator == "torch" and not plan_only) else \
@@ -410,7 +428,9 @@ class Model:
         form a data loader hands over: no per-node Python work)."""
         csr = graphs if isinstance(graphs, CsrBatch) else CsrBatch(*to_csr(graphs))
         gp, cp, ch, tok, lab = csr.arrays
-        b = _Batch(len(gp) - 1, gp.ctypes.data, cp.ctypes.data, ch.ctypes.data, tok.ctypes.data, lab.ctypes.data)
+        chp, chs = csr.chars
+        b = _Batch(len(gp) - 1, gp.ctypes.data, cp.ctypes.data, ch.ctypes.data, tok.ctypes.data, lab.ctypes.data,
+                   chp.ctypes.data if chp is not None else None, chs.ctypes.data if chs is not None else None)
         h = ct.c_void_p()
         _check(_lib.vpps_build_script(self._h, ct.byref(b), ct.byref(h)))
         return Script(self, h)

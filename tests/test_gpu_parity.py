@@ -562,3 +562,52 @@ def test_autotune_on_device_then_parity():
     assert len(res) >= 3 and min(res.values()) == res[repr(best)]
     graphs = synth.config_batch("c3", 7, batch=16, V=32, C=32)
     check("lstm", 256, 256, 32, graphs, 32, seed=501, groups=best.get("groups", 1), level=best.get("level", 0))
+
+
+def _char_check(H, E, graphs, V, seed, mlp, C=9):
+    """BiLSTMwChar through the C ABI against the oracle M9 (loss, every gradient incl. C_emb and the character
+    LSTMs, and dX; rare words' table rows get no gradient)."""
+    vpps = _vpps()
+    rng = np.random.default_rng(seed)
+    shapes = vpps.param_shapes("bilstmchar", H, E, C, mlp)
+    P = synth.init_params(shapes, rng)
+    X = synth.input_table(rng, V, E)
+    m = vpps.Model("bilstmchar", H, E, C, device=0, mlp=mlp)
+    params = torch.zeros(m.n_floats, dtype=torch.float32, device="cuda")
+    grads = torch.full_like(params, float("nan"))
+    for name, _ in shapes:
+        m.views(params)[name].copy_(torch.from_numpy(P[name]).float())
+    m.bind(params, grads)
+    inputs = torch.from_numpy(X).float().cuda()
+    dX = torch.full_like(inputs, float("nan"))
+    m.fwd_bwd(m.build_script(graphs), inputs, dX)
+    loss = m.latest_loss()
+    lo, Go, dXo = M.forward_backward("bilstmchar", P, X, graphs, H)
+    assert abs(loss - lo) <= TOL * abs(lo), (loss, lo)
+    gv = m.views(grads.cpu())
+    for name, _ in shapes:
+        assert rel(gv[name].numpy(), Go[name]) <= TOL, name
+    assert rel(dX.cpu().numpy(), dXo) <= TOL, "dX"
+
+
+def test_bilstmchar_small():
+    """M9 (reading R-38) on the GPU: character BiLSTM (H_c = E/2 = 32) on the chain recurrence feeding the word
+    tagger's rare positions; ragged sentences, spellings of 2-12 characters, repeated rare words."""
+    g = synth.char_tagger_batch(np.random.default_rng(600), 4, (1, 10), 64, 9, 64)
+    assert any(len(nd[3]) for s_ in g for nd in s_)
+    _char_check(32, 64, g, 64, 601, mlp=16)
+
+
+def test_bilstmchar_edge_cases():
+    """No rare word (the tagger alone), a one-character spelling, a sentence of one rare word."""
+    plain = [[(() if t == 0 else (t - 1,), 3 + t, t % 9, ()) for t in range(5)]]
+    _char_check(32, 64, plain, 64, 602, mlp=16)
+    odd = [[((), 60, 1, (7,)), ((0,), 2, 3, ()), ((1,), 61, 0, (1, 2))], [((), 62, 4, (9, 9, 9))]]
+    _char_check(64, 64, odd, 64, 603, mlp=32)
+
+
+def test_bilstmchar_paper_size():
+    """BiLSTMwChar at Fig. 12's sizes (hidden = embedding = 256, MLP 256, character embedding 64), 16
+    WikiNER-length sentences (config 'bilstmchar')."""
+    g = synth.config_batch("bilstmchar", 0)
+    _char_check(256, 256, g, 4096, 604, mlp=256)
