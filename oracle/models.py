@@ -561,12 +561,22 @@ def sgd(P: dict, G: dict, lr: float, weight_decay: float):
     return {k: P[k] - lr * (G[k] + weight_decay * P[k]) for k in P}
 
 
-def flop_count(cell: str, graphs, H: int, E: int, C: int, want_dx: bool = True, M: int = 256):
+def flop_count(cell: str, graphs, H: int, E: int, C: int, want_dx: bool = True, M: int = 256, Ec_: int = 64):
     """Algorithmic FLOPs of one training pass: 2 per MAC, ×3 per matrix use
     (forward, dW, dx), ×2 where the input gradient is not needed."""
     f = 0
     kx = 3 if want_dx else 2
     for nodes in graphs:
+        if cell == "bilstmchar":
+            # M9 (R-38): the word tagger (M2) plus, per rare word of n characters, the character BiLSTM
+            # (Hc = E/2 per direction over Ec-wide character embeddings; dx to C_emb needed: x3)
+            Hc, Ec = E // 2, Ec_
+            f += flop_count("bilstm", [[nd[:3] for nd in nodes]], H, E, C, want_dx, M)
+            for nd in nodes:
+                n = len(nd[3]) if len(nd) > 3 else 0
+                if n:
+                    f += 2 * (2 * 4 * Hc * Ec * 3 * n + 2 * 3 * 4 * Hc * Hc * (n - 1))
+            continue
         if cell == "bilstm":
             # M2 (L265, L281): per position and direction the input product (W x) and, after the first
             # step of that direction, the recurrent product (U h); per labelled position the MLP over

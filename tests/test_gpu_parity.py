@@ -593,7 +593,7 @@ def _char_check(H, E, graphs, V, seed, mlp, C=9):
 def test_bilstmchar_small():
     """M9 (reading R-38) on the GPU: character BiLSTM (H_c = E/2 = 32) on the chain recurrence feeding the word
     tagger's rare positions; ragged sentences, spellings of 2-12 characters, repeated rare words."""
-    g = synth.char_tagger_batch(np.random.default_rng(600), 4, (1, 10), 64, 9, 64)
+    g = synth.char_tagger_batch(np.random.default_rng(600), 4, (1, 10), 64, 9, 64, rare_from=8)
     assert any(len(nd[3]) for s_ in g for nd in s_)
     _char_check(32, 64, g, 64, 601, mlp=16)
 

@@ -274,3 +274,21 @@ def test_autotune_picks_the_fastest_candidate(vpps):
     opts = vpps.candidate_options("binary", 256, 5)
     assert opts[0] == dict(cluster=16, dataflow=True) and dict(level=1) in opts
     assert vpps.candidate_options("gru", 256, 1000) == [dict(chain=0), dict(chain=-1)]
+
+
+def test_bilstmchar_script_host_side(vpps):
+    """BiLSTMwChar scripts (plan-only): the host FLOP count equals the oracle's; spellings are accepted only by
+    this cell; character ids and tokens are range-checked (a rare word's token is never read)."""
+    H, E, C = 32, 64, 9
+    g = synth.char_tagger_batch(np.random.default_rng(7), 5, (1, 12), 64, C, 64, rare_from=8)
+    assert sum(len(nd[3]) for s_ in g for nd in s_) > 0
+    m = vpps.Model("bilstmchar", H, E, C, plan_only=True, mlp=16)
+    info = m.build_script(g).info()
+    assert info["flops"] == M.flop_count("bilstmchar", g, H, E, C, M=16)
+    plain = [[nd[:3] for nd in s] for s in g]
+    assert M.flop_count("bilstmchar", plain, H, E, C, M=16) == M.flop_count("bilstm", plain, H, E, C, M=16)
+    with pytest.raises(vpps.VppsError):
+        vpps.Model("bilstm", H, E, C, plan_only=True, mlp=16).build_script(g)       # spellings need M9
+    with pytest.raises(vpps.VppsError):
+        m.build_script([[((), 3, 1, (64,))]])                                          # character id >= Vc
+    m.build_script([[((), 10 ** 6, 1, (5,))]])                                         # rare: token unused

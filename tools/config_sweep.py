@@ -42,6 +42,8 @@ CASES = [
     ("TD-LSTM H256 B16 (level path)", "tdrnn", "tdlstm", 256, 256, 5, 4096, 16, {}, {}),
     ("c4 BiLSTM tagger H512 B16 (level path)", "c4", "bilstm", 512, 512, 9, 4096, 16, {"mlp": 256}, {}),
     ("c5 binary H1024 B64 (level path)", "c5", "binary", 1024, 1024, 5, 4096, 64, {}, {}),
+    ("BiLSTMwChar H256 E256 MLP256 B16 (chain)", "bilstmchar", "bilstmchar", 256, 256, 9, 4096, 16, {"mlp": 256}, {}),
+    ("c4 BiLSTM tagger H512 B16 (per-step products)", "c4", "bilstm", 512, 512, 9, 4096, 16, {"mlp": 256, "chain": -1}, {}),
     ("tgt binary H256 B16 (level path)", "tgt", "binary", 256, 256, 5, 4096, 16, {"level": 1}, {}),
     ("tgt binary H256 B1 (dataflow)", "tgt", "binary", 256, 256, 5, 4096, 1, {"cluster": 16, "dataflow": True}, {}),
     ("tgt binary H256 B4 (dataflow)", "tgt", "binary", 256, 256, 5, 4096, 4, {"cluster": 16, "dataflow": True}, {}),
@@ -53,8 +55,8 @@ CASES = [
 def kernel_label(cell, H, C, opts):
     if opts.get("dataflow"):
         return "vpps_df + GEMMs"
-    chain = cell in ("bilstm", "gru") or (cell == "lstm" and (opts.get("level") or C > 32))
-    if chain and os.environ.get("VPPS_CHAIN", "1") != "0" and H in (32, 64, 128, 256, 512):
+    chain = cell in ("bilstm", "gru", "bilstmchar") or (cell == "lstm" and (opts.get("level") or C > 32))
+    if chain and os.environ.get("VPPS_CHAIN", "1") != "0" and opts.get("chain", 0) >= 0 and H in (32, 64, 128, 256, 512):
         return "vpps_chain (register-resident recurrence) + GEMMs"
     if opts.get("level") or H > 256 or cell in ("bilstm", "gru", "rvnn", "tdrnn", "tdlstm") or C > 32:
         return "level GEMMs"
