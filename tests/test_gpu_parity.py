@@ -51,6 +51,33 @@ def rel(a, b):
     return float(np.abs(np.asarray(a, np.float64) - b).max() / max(np.abs(b).max(), 1e-30))
 
 
+_STATS = []
+
+
+def elementwise(name, a, b):
+    """R-22's elementwise statistics: |g - o| / max(|o|, 1e-3 ‖o‖∞) per element (max, 99.9th percentile),
+    recorded for the report (VPPS_PARITY_STATS=path writes them as JSON lines at the end of the session)."""
+    a = np.asarray(a, np.float64).ravel()
+    b = np.asarray(b, np.float64).ravel()
+    if b.size == 0:
+        return
+    floor = 1e-3 * max(np.abs(b).max(), 1e-30)
+    r = np.abs(a - b) / np.maximum(np.abs(b), floor)
+    _STATS.append(dict(tensor=name, max=float(r.max()), p999=float(np.quantile(r, 0.999)), n=int(b.size)))
+
+
+@pytest.fixture(scope="session", autouse=True)
+def _write_stats():
+    yield
+    import json
+    import os
+    path = os.environ.get("VPPS_PARITY_STATS")
+    if path and _STATS:
+        with open(path, "w") as f:
+            for row in _STATS:
+                f.write(json.dumps(row) + "\n")
+
+
 def check(cell, H, E, C, graphs, V, seed=0, want_dx=True, groups=1, cluster=0, dataflow=False, level=0, mlp=256):
     m, P, X, loss, params, grads, dX = run_case(cell, H, E, C, graphs, V, seed, want_dx, groups=groups,
                                                 cluster=cluster, dataflow=dataflow, level=level, mlp=mlp)
@@ -59,8 +86,10 @@ def check(cell, H, E, C, graphs, V, seed=0, want_dx=True, groups=1, cluster=0, d
     gv = m.views(grads.cpu())
     for name, _ in m.shapes:
         assert rel(gv[name].numpy(), Go[name]) <= TOL, name
+        elementwise(f"{cell} H{H} {name}", gv[name].numpy(), Go[name])
     if want_dx:
         assert rel(dX.cpu().numpy(), dXo) <= TOL, "dX"
+        elementwise(f"{cell} H{H} dX", dX.cpu().numpy(), dXo)
     return loss, lo
 
 
@@ -231,15 +260,18 @@ def test_childsum_arity_and_missing_tokens():
     check("childsum", 32, 32, 5, [g] + _trees(5, 2, (1, 7), 8, 5), 8)
 
 
-def test_lstm_config1():
+@pytest.mark.parametrize("level", [0, -1])
+def test_lstm_config1(level):
+    """Config 1 on the default path (chain recurrence + dense products) and the one-kernel grid path."""
     graphs = synth.config_batch("c1", 0)
-    check("lstm", 32, 32, 16, graphs, 16, seed=1)
+    check("lstm", 32, 32, 16, graphs, 16, seed=1, level=level)
 
 
 def test_lstm_h256_small_vocab():
     rng = np.random.default_rng(9)
     graphs = [synth.chain(rng, int(rng.integers(5, 30)), 16) for _ in range(4)]
     check("lstm", 256, 256, 16, graphs, 16, seed=9)
+    check("lstm", 256, 256, 16, graphs, 16, seed=9, level=-1)
 
 
 @pytest.mark.parametrize("batch", [1, 4, 16, 64])
@@ -247,6 +279,7 @@ def test_lstm_config3_batch_sweep(batch):
     """Config 3 (LSTM LM, H = E = 256, sentences of 5-60 tokens, batch 1/4/16/64) with the GPU reading of
     the vocabulary (R-31: V = C = 32 symbols, the head held in one CTA's shared memory)."""
     graphs = synth.config_batch("c3", 0, batch=batch, V=32, C=32)
+    check("lstm", 256, 256, 32, graphs, 32, seed=30 + batch, level=-1)
     check("lstm", 256, 256, 32, graphs, 32, seed=30 + batch)
 
 
@@ -256,7 +289,7 @@ def test_grid_replica_groups(cell, H, groups):
     min-load rule, gradients summed across groups in the epilogue."""
     if cell == "lstm":
         graphs = synth.config_batch("c3", 1, batch=16, V=32, C=32)
-        check("lstm", H, H, 32, graphs, 32, seed=40 + groups, groups=groups)
+        check("lstm", H, H, 32, graphs, 32, seed=40 + groups, groups=groups, level=-1)
     else:
         check("childsum", H, H, 5, synth.config_batch("c2", 1), 4096, seed=50 + groups, groups=groups)
 

@@ -21,10 +21,12 @@ sys.path.insert(0, ROOT)
 # (label, config, cell, H, E, C, V, batch, model options, overrides)
 CASES = [
     ("c1 LSTM H32 B4", "c1", "lstm", 32, 32, 16, 16, 4, {}, {}),
+    ("c1 LSTM H32 B4 (grid)", "c1", "lstm", 32, 32, 16, 16, 4, {"level": -1}, {}),
     ("c2 child-sum H128 B16", "c2", "childsum", 128, 128, 5, 4096, 16, {}, {}),
     ("c3 LSTM-LM H256 B1 (V=C=32)", "c3", "lstm", 256, 256, 32, 32, 1, {}, {"V": 32, "C": 32}),
     ("c3 LSTM-LM H256 B4 (V=C=32)", "c3", "lstm", 256, 256, 32, 32, 4, {}, {"V": 32, "C": 32}),
     ("c3 LSTM-LM H256 B16 (V=C=32)", "c3", "lstm", 256, 256, 32, 32, 16, {}, {"V": 32, "C": 32}),
+    ("c3 LSTM-LM H256 B16 (V=C=32, grid)", "c3", "lstm", 256, 256, 32, 32, 16, {"level": -1}, {"V": 32, "C": 32}),
     ("c3 LSTM-LM H256 B64 (V=C=32)", "c3", "lstm", 256, 256, 32, 32, 64, {}, {"V": 32, "C": 32}),
     ("c2 child-sum H128 B16 G4", "c2", "childsum", 128, 128, 5, 4096, 16, {"groups": 4}, {}),
     ("c3 LSTM-LM H256 B16 G2", "c3", "lstm", 256, 256, 32, 32, 16, {"groups": 2}, {"V": 32, "C": 32}),
@@ -55,7 +57,8 @@ CASES = [
 def kernel_label(cell, H, C, opts):
     if opts.get("dataflow"):
         return "vpps_df + GEMMs"
-    chain = cell in ("bilstm", "gru", "bilstmchar") or (cell == "lstm" and (opts.get("level") or C > 32))
+    chain = cell in ("bilstm", "gru", "bilstmchar") or (cell == "lstm" and opts.get("level", 0) >= 0
+                                                          and opts.get("groups", 1) <= 1)
     if chain and os.environ.get("VPPS_CHAIN", "1") != "0" and opts.get("chain", 0) >= 0 and H in (32, 64, 128, 256, 512):
         return "vpps_chain (register-resident recurrence) + GEMMs"
     if opts.get("level") or H > 256 or cell in ("bilstm", "gru", "rvnn", "tdrnn", "tdlstm") or C > 32:
