@@ -165,9 +165,11 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     if (cell == CELL_BILSTM || cell == CELL_BILSTM_CHAR || cell == CELL_GRU || cell == CELL_RVNN || cell == CELL_TDRNN ||
         cell == CELL_TDLSTM ||
         (cell == CELL_LSTM &&
-         (o.level > 0 || (o.level == 0 && (C > 32 || (o.chain >= 0 && o.groups <= 1 && chain_group_ctas(H) > 0)))))) {
-        // (an LSTM takes the chain recurrence + dense products by default when it is built for H — measured
-        //  3.3x faster than the grid kernel at config 3; level = -1 keeps the one-kernel grid path)
+         (o.level > 0 ||
+          (o.level == 0 && (C > 32 || (o.chain >= 0 && o.groups <= 1 && H >= 128 && chain_group_ctas(H) > 0)))))) {
+        // (an LSTM at H >= 128 takes the chain recurrence + dense products by default — 3.6x the grid kernel
+        //  at config 3, H = 256; at config 1's H = 32 the one-kernel grid path is faster, 0.054 vs 0.093 ms;
+        //  level = -1 / 1 force either)
         // M2 and M5 (GRU) run on the level-synchronous path only (vpps_level.cu), and so does an LSTM LM
         // whose vocabulary head exceeds one CTA's shared memory (config 3 at V = 1000): no partition plan
         if (o.cluster > 1 || o.dataflow || o.level < 0) return fail(VPPS_E_INVALID, "this op set runs on the level path only");

@@ -57,8 +57,11 @@ CASES = [
 def kernel_label(cell, H, C, opts):
     if opts.get("dataflow"):
         return "vpps_df + GEMMs"
-    chain = cell in ("bilstm", "gru", "bilstmchar") or (cell == "lstm" and opts.get("level", 0) >= 0
-                                                          and opts.get("groups", 1) <= 1)
+    lvl = opts.get("level", 0)
+    if cell in ("lstm", "childsum", "binary") and lvl == -1:
+        return "vpps_fb (grid)"
+    chain = cell in ("bilstm", "gru", "bilstmchar") or (
+        cell == "lstm" and opts.get("groups", 1) <= 1 and (lvl > 0 or C > 32 or H >= 128))
     if chain and os.environ.get("VPPS_CHAIN", "1") != "0" and opts.get("chain", 0) >= 0 and H in (32, 64, 128, 256, 512):
         return "vpps_chain (register-resident recurrence) + GEMMs"
     if opts.get("level") or H > 256 or cell in ("bilstm", "gru", "rvnn", "tdrnn", "tdlstm") or C > 32:
