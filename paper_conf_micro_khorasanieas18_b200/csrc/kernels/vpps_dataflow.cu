@@ -153,7 +153,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         for (int i = tid; i < C * H; i += NTH) { Wo[i] = __ldg(P.params + off[4] + i); dWo[i] = 0.f; }
         for (int i = tid; i < C; i += NTH) { bo[i] = __ldg(P.params + off[7] + i); dbo[i] = 0.f; }
     }
-    float dbacc[4] = {0.f, 0.f, 0.f, 0.f};   // bias gradients of unit j (thread (u, gl) mapping)
+    float dbacc[4] = {0.f, 0.f, 0.f, 0.f};   // bias gradients of unit lc * UM + tid % UM (INT_B mapping)
     float dbleaf[3] = {0.f, 0.f, 0.f};       // ... of unit lc * UM + tid % UM (LEAF_B mapping)
     uint64_t* prof = PROF && P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
     // section clocks (trace only): 0 program, 1 staging, 2 tag wait, 3 forward, 4 cell-bwd, 5 transposed,
@@ -392,22 +392,22 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             }
             }
         } else {
-            // backward, thread (n = tid / U, u = tid % U): dh = Σ_k PART[parent][lc][k][side][u] (+ HD), its
-            // own 17 slots polled with L1-bypassing relaxed loads; own operands dc (adj + H), c i o u
-            // (fl fr), c_l c_r by cp.async
+            // backward, thread (n = tid / U, uu = tid % U): dh = Σ_k PART[parent][lc][k][side][uu] (+ HD), its
+            // own 17 slots polled with relaxed GPU-scope loads, its own operands (dc at adj + H; c i o u fl fr;
+            // the children's c — all written by this CTA) loaded into registers alongside; then the cell
+            // backward right here: gate gradients to the record (left operands of the gradient GEMM, L185),
+            // the children's dc to theirs, and to shared memory for the transposed product (one barrier)
             const int n = tid / UM, uu = tid % UM, jj = lc * UM + uu;
             const bool act = n < nb;
             const uint32_t* e = ent + (act ? n : 0) * sz;
             const uint32_t dsrc = act ? e[2] : NONE, hd = act ? e[3] : NONE;
+            float rv[9];
             if (act) {
-                float* cv = cin + tid * CINMAX;
-                cp_async4(cv + 1, pool + e[1] + H + jj, 4u);
-                const int nrec = op == INT_B ? 6 : 4;
-                for (int k = 0; k < nrec; ++k) cp_async4(cv + 2 + k, pool + e[0] + (k + 1) * H + jj, 4u);
-                if (op == INT_B) {
-                    cp_async4(cv + 8, pool + e[5] + H + jj, 4u);
-                    cp_async4(cv + 9, pool + e[7] + H + jj, 4u);
-                }
+                rv[0] = pool[e[1] + H + jj];
+#pragma unroll
+                for (int k = 0; k < 6; ++k) rv[1 + k] = pool[e[0] + (k + 1) * H + jj];
+                rv[7] = pool[e[5] + H + jj];
+                rv[8] = pool[e[7] + H + jj];
             }
             const u64* psrc = dsrc != NONE ? PART + ((((int64_t)(dsrc >> 1) * NCL + lc) * NCL) * 2 + (dsrc & 1)) * UM + uu : nullptr;
             const u64* hsrc = hd != NONE ? HD + (int64_t)hd * H + jj : nullptr;
@@ -417,7 +417,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             for (int k = 0; k < NCL; ++k) v[k] = psrc ? ld_slot(psrc + k * 2 * UM) : none;
             v[NCL] = hsrc ? ld_slot(hsrc) : none;
             XST(stB, 23);
-            cp_async_wait_all();
             XST(stB, 24);
             if (bt) bt[1] = clock64();
             mark(2);
@@ -430,15 +429,33 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 if (!stale) break;
                 ++rounds;
             }
+            XST(stB, 25);
+            mark(4);
             if (act) {
                 float dh = 0.f;
 #pragma unroll
                 for (int k = 0; k <= NCL; ++k) dh += __uint_as_float((uint32_t)v[k]);
-                cin[tid * CINMAX] = dh;
+                const float dc = rv[0], c = rv[1], i = rv[2], o = rv[3], uv = rv[4], fl = rv[5], fr = rv[6];
+                const float th = ftanh(c);
+                const float chat = dc + dh * o * (1.f - th * th);
+                float g[5];
+                g[0] = chat * uv * i * (1.f - i);
+                g[1] = dh * th * o * (1.f - o);
+                g[2] = chat * i * (1.f - uv * uv);
+                g[3] = chat * rv[7] * fl * (1.f - fl);
+                g[4] = chat * rv[8] * fr * (1.f - fr);
+                const uint32_t rec = e[0];
+                pool[e[6] + H + jj] = chat * fl;          // dc of the children (unique parent; own units)
+                pool[e[8] + H + jj] = chat * fr;
+#pragma unroll
+                for (int r = 0; r < 5; ++r) {
+                    pool[rec + (7 + r) * H + jj] = g[r];
+                    cin[(n * 5 + r) * UM + uu] = g[r];    // (cin of this batch holds the gate gradients)
+                }
+                dbacc[0] += g[0]; dbacc[1] += g[1]; dbacc[2] += g[2]; dbacc[3] += g[3] + g[4];
             }
-            XST(stB, 25);
-            __syncthreads();
             XST(stB, 26);
+            __syncthreads();
             XST(stBB, 28);
         }
         if (bt) { bt[2] = clock64(); bt[4] |= (uint64_t)rounds << 8; }
@@ -584,40 +601,10 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             if (nb - n0 == 2) fwd_group(std::integral_constant<int, 2>{}, n0);
             else if (nb - n0 == 1) fwd_group(std::integral_constant<int, 1>{}, n0);
         } else {
-            // ---- backward: cell backward by thread (unit u, node gl); gate gradients recorded for the dW
-            //      GEMM (L185) and broadcast to the unit's lanes ----
+            // ---- backward: the gate gradients of the batch are in shared memory (cin), from the staging ----
             const bool kindB = op == INT_B;
-            XST(stB, 5);
-            float g[5] = {0.f, 0.f, 0.f, 0.f, 0.f};
-            if (gl < nb) {
-                const uint32_t* e = ent + gl * sz;
-                const uint32_t rec = e[0];
-                const float* cv = cin + (gl * UM + u) * CINMAX;
-                const float dh = cv[0], dc = cv[1], c = cv[2], i = cv[3], o = cv[4], uv = cv[5];
-                const float th = ftanh(c);
-                const float chat = dc + dh * o * (1.f - th * th);
-                g[0] = chat * uv * i * (1.f - i);
-                g[1] = dh * th * o * (1.f - o);
-                g[2] = chat * i * (1.f - uv * uv);
-                if (kindB) {
-                    const float fl = cv[6], fr = cv[7], cl = cv[8], cr = cv[9];
-                    g[3] = chat * cl * fl * (1.f - fl);
-                    g[4] = chat * cr * fr * (1.f - fr);
-                    pool[e[6] + H + j] = chat * fl;          // dc of the children (unique parent; own units)
-                    pool[e[8] + H + j] = chat * fr;
-                    pool[rec + 7 * H + j] = g[0];
-                    pool[rec + 8 * H + j] = g[1];
-                    pool[rec + 9 * H + j] = g[2];
-                    pool[rec + 10 * H + j] = g[3];
-                    pool[rec + 11 * H + j] = g[4];
-                } else {
-                    pool[rec + 5 * H + j] = g[0];
-                    pool[rec + 6 * H + j] = g[1];
-                    pool[rec + 7 * H + j] = g[2];
-                }
-                dbacc[0] += g[0]; dbacc[1] += g[1]; dbacc[2] += g[2]; dbacc[3] += g[3] + g[4];
-            }
             mark(5);
+            XST(stB, 5);
             XST(stB, 6);
             XST(stBB, 29);
             // transposed products (L94, fn4): per node, this CTA's partial dx = Σ_r W[r] g_r over all 2H
@@ -628,7 +615,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             // reduction of chunk c overlaps the products of chunk c + 1.
             if (kindB) {
                 constexpr int NW = NTH / 32;
-                const int src = lane & 16;
                 const bool hi = lane & 16;
                 for (int n0 = 0; n0 < nb; n0 += NC, cbuf ^= 1) {
                     float* buf = dxb + cbuf * (NW * NC * KP);
@@ -638,7 +624,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                         if (n >= nb) break;
                         float gr[5];
 #pragma unroll
-                        for (int r = 0; r < 5; ++r) gr[r] = __shfl_sync(FULLMASK, g[r], src | (n & 15));
+                        for (int r = 0; r < 5; ++r) gr[r] = cin[(n * 5 + r) * UM + u];
                         float* drow = buf + (warp * NC + dn) * KP;
 #pragma unroll
                         for (int t = 0; t < LB::NT; t += 2) {
@@ -712,14 +698,13 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
 
     // ---- epilogue: bias and head gradients of this group summed into grads (zeroed by the host); the
     //      weight-matrix gradients come from vpps_dw_gemm (L185) ----
+    // (dbacc: unit lc * UM + tid % UM, like dbleaf: lanes l and l ^ 16 share a unit)
 #pragma unroll
-    for (int k = 0; k < 4; ++k)
+    for (int k = 0; k < 4; ++k) dbacc[k] += __shfl_xor_sync(FULLMASK, dbacc[k], 16);
+    if (lane < 16) {
 #pragma unroll
-        for (int s = 8; s >= 1; s >>= 1) dbacc[k] += __shfl_xor_sync(FULLMASK, dbacc[k], s);
-    if (gl == 0) {
-#pragma unroll
-        for (int k = 0; k < 3; ++k) atomicAdd(P.grads + off[5] + k * H + j, dbacc[k]);
-        atomicAdd(P.grads + off[6] + j, dbacc[3]);
+        for (int k = 0; k < 3; ++k) atomicAdd(P.grads + off[5] + k * H + lc * UM + lane, dbacc[k]);
+        atomicAdd(P.grads + off[6] + lc * UM + lane, dbacc[3]);
     }
 #pragma unroll
     for (int k = 0; k < 3; ++k) dbleaf[k] += __shfl_xor_sync(FULLMASK, dbleaf[k], 16);   // lanes l, l^16: same unit
