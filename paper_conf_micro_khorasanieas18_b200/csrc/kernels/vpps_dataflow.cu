@@ -128,12 +128,17 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
 
     if (PROF && P.prof && threadIdx.x == 0) P.prof[(int64_t)blockIdx.x * P.prof_stride + 11] = gtimer();   // entry
     // ---- prologue: this CTA's rows of U_iou, U_fl, U_fr -> registers (L123, L129) ----
+    // register slot t of a lane in the upper half-warp holds granule t ^ 1 (lanes l and l ^ 16 hold the same
+    // columns of the warp's two units): the transposed product's pair exchange then keeps slot t and sends
+    // slot t + 1 in every lane, with no selects (granules t and t ^ 1 sit on the same side of h_l / h_r)
+    const int gsw = (lane & 16) ? 1 : 0;
+    static_assert(T::TH % 2 == 0, "swapped granule pairs stay on one side of [h_l; h_r]");
     float wb[4][LB::NREG];
 #pragma unroll
     for (int r = 0; r < 4; ++r)
 #pragma unroll
         for (int t = 0; t < LB::NT; ++t) {
-            const int col = LB::CG * (tu + TU * t);
+            const int col = LB::CG * (tu + TU * (t ^ gsw));
             const float* src = r < 3 ? P.params + off[1] + (int64_t)(r * H + j) * (2 * H) + col
                                      : (col < H ? P.params + off[2] + (int64_t)j * H + col
                                                 : P.params + off[3] + (int64_t)j * H + col - H);
@@ -534,7 +539,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                     for (int o = 0; o < 5; ++o) a[n][o] = make_float2(0.f, 0.f);
 #pragma unroll
                 for (int t = 0; t < LB::NT; ++t) {
-                    const int col0 = LB::CG * (tu + TU * t);
+                    const int col0 = LB::CG * (tu + TU * (t ^ gsw));
                     constexpr int of0 = 3;                  // granules t < T::TH read h_l (U_fl), the rest h_r (U_fr)
 #pragma unroll
                     for (int n = 0; n < NN; ++n) {
@@ -649,8 +654,8 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                             float kv[LB::CG];
 #pragma unroll
                             for (int q = 0; q < LB::CG; ++q) {
-                                const float send = hi ? dx[0][q] : dx[1][q];
-                                kv[q] = (hi ? dx[1][q] : dx[0][q]) + __shfl_xor_sync(FULLMASK, send, 16);
+                                // slot t is granule t (t + 1 in the upper half-warp): keep it, send slot t + 1
+                                kv[q] = dx[0][q] + __shfl_xor_sync(FULLMASK, dx[1][q], 16);
                             }
                             const int col0 = LB::CG * (tu + TU * (t + (hi ? 1 : 0)));
                             sts_granule<LB::CG>(drow + col0, kv, true);
