@@ -182,7 +182,7 @@ def build(cell: str, graphs, H: int, E: int, C: int, G: int = 1, n_act: int = 14
                 graph_group=graph_group, G=G, H=H)
 
 
-DF_OP = dict(LEAF_F=0x20, LEAF_B=0x21, INT_F=0x22, INT_B=0x23, HEAD_FB=0x42)
+DF_OP = dict(LEAF_B=0x21, INT_F=0x22, INT_B=0x23, HEAD_FB=0x42)
 
 
 def device_lowering(ref):
@@ -217,7 +217,7 @@ def device_lowering(ref):
             head_of[n["children"][0]] = i
     hx, pp, hd = {}, {}, {}
     for i, n in enumerate(nodes):
-        if n["kind"] in ("INT", "LEAF") and (i in parent or i in head_of):
+        if n["kind"] == "INT" and (i in parent or i in head_of):
             hx[i] = len(hx)
         if n["kind"] == "INT":
             pp[i] = len(pp)
@@ -238,12 +238,10 @@ def device_lowering(ref):
         if op == "INT_B":
             l, r = n["children"]
             return [rec[i], adj[i], dsrc(i), hd.get(i, NONE_), pp[i], rec[l], adj[l], rec[r], adj[r]]
-        if op == "LEAF_F":
-            return [rec[i], n["token"], hx.get(i, NONE_)]
         return [rec[i], adj[i], dsrc(i), hd.get(i, NONE_)]          # LEAF_B
 
     def batches(op, ids):
-        cap = {"LEAF_B": 64, "LEAF_F": 32}.get(op, 16)
+        cap = 64 if op == "LEAF_B" else 16
         w = []
         for b0 in range(0, len(ids), cap):
             chunk = ids[b0:b0 + cap]
@@ -256,7 +254,6 @@ def device_lowering(ref):
     for g in range(G):
         w = []
         mine = [i for i in range(len(nodes)) if group[i] == g]
-        w += batches("LEAF_F", [i for i in mine if nodes[i]["kind"] == "LEAF"])     # level 0 by the group
         for lv in range(1, L + 1):                 # forward levels: cells, then the heads of that level
             w += batches("INT_F", [i for i in mine if level[i] == lv and nodes[i]["kind"] == "INT"])
             w += batches("HEAD_FB", [i for i in mine if level[i] == lv and nodes[i]["kind"] == "HEAD"])

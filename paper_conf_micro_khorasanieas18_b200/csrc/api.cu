@@ -612,7 +612,6 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         // gradient GEMM (programmatic dependent, per-group completion counters) -> SGD
         DfParams dp{};
         dp.params = m->params;
-        dp.inputs = inputs;
         dp.grads = m->grads;
         dp.pool = m->pool;
         dp.script = dwords;
@@ -646,10 +645,12 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         const uint32_t* lists = dwords + s->s.lists_off;
         const uint32_t* leaf_list = lists + 3 * s->s.n_int;
         const float* W_iou = m->params + m->offsets[0];
-        // the per-pass clearing and the pass counter (the leaf kernel with no leaves: the leaves are LEAF_F
-        // batches of vpps_df); its CTAs also pull every parameter into L2 for vpps_df's prologue
-        launch_leaf_fwd(W_iou, m->params + m->offsets[5], inputs, m->pool, leaf_list, 0, m->plan.H, m->plan.E,
-                        zero_ptr, zero_n, m->d_epoch, st, m->params, m->n_floats * (int64_t)sizeof(float));
+        // U_iou, U_fl, U_fr, W_out and the biases (contiguous after W_iou in the flat layout) are pulled into
+        // L2 by the leaf kernel's clearing warps for vpps_df's prologue
+        const int64_t pf_floats = m->n_floats - m->offsets[1];
+        launch_leaf_fwd(W_iou, m->params + m->offsets[5], inputs, m->pool, leaf_list, (int32_t)s->s.n_leaf,
+                        m->plan.H, m->plan.E, zero_ptr, zero_n, m->d_epoch, st, m->params + m->offsets[1],
+                        pf_floats * (int64_t)sizeof(float));
         if (m->k_before) CK(cudaEventRecord(m->k_before, st));
         const void* dfn = m->prof ? df_prof_fn(m->var->fn) : m->var->fn;
         if (m->prof) CK(cudaFuncSetAttribute(dfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)m->smem));

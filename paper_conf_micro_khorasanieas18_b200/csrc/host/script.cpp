@@ -424,10 +424,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
         }
         std::vector<uint32_t> hx(N, NONE), pp(N, NONE), hd(N, NONE);
         for (int64_t i = 0; i < N; ++i) {
-            // h of every cell another CTA reads: internal cells and (computed in the kernel since the leaf
-            // fusion) leaves with a parent or a head
-            if ((nodes[i].kind == K_INT || nodes[i].kind == K_LEAF) && (parent[i] >= 0 || head_of[i] >= 0))
-                hx[i] = (uint32_t)s.n_hx++;
+            if (nodes[i].kind == K_INT && (parent[i] >= 0 || head_of[i] >= 0)) hx[i] = (uint32_t)s.n_hx++;
             if (nodes[i].kind == K_INT) pp[i] = (uint32_t)s.n_part++;
             if (head_of[i] >= 0) hd[i] = (uint32_t)s.n_hd++;
         }
@@ -436,9 +433,7 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
         };
         std::vector<std::vector<uint32_t>> prog(G);
         auto emit_batches = [&](int32_t g, uint32_t op, const std::vector<int64_t>& list) {
-            // leaf backward needs no shared staging; a leaf forward stages E floats per leaf (32 fill the
-            // shared row buffer of 16 internal nodes' [h_l; h_r])
-            const size_t cap = op == OP_LEAF_B ? 64 : (op == OP_LEAF_F ? 32 : 16);
+            const size_t cap = op == OP_LEAF_B ? 64 : 16;   // leaf backward needs no shared staging
             for (size_t b0 = 0; b0 < list.size(); b0 += cap) {
                 const size_t nb = std::min<size_t>(cap, list.size() - b0);
                 std::vector<uint32_t>& w = prog[g];
@@ -449,9 +444,6 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
                     switch (op) {
                         case OP_INT_F:
                             w.insert(w.end(), {rec[i], hx[i], rec[ch[0]], hx[ch[0]], rec[ch[1]], hx[ch[1]]});
-                            break;
-                        case OP_LEAF_F:
-                            w.insert(w.end(), {rec[i], (uint32_t)nodes[i].token, hx[i]});
                             break;
                         case OP_HEAD_FB:
                             w.insert(w.end(), {rec[i], rec[ch[0]], (uint32_t)nodes[i].label, hx[ch[0]], hd[ch[0]]});
@@ -468,11 +460,6 @@ int build_script(const Plan& plan, const BatchIn& b, int64_t n_input_rows, Scrip
         };
         std::vector<std::vector<int64_t>> lists(5);
         for (int32_t g = 0; g < G; ++g) {
-            // level 0: the group's leaves (W_iou x + b, the leaf cell) computed by the group itself
-            for (auto& l : lists) l.clear();
-            for (int64_t i : at_level[0])
-                if (graph_group[nodes[i].graph] == g && nodes[i].kind == K_LEAF) lists[2].push_back(i);
-            emit_batches(g, OP_LEAF_F, lists[2]);
             for (int32_t lv = 1; lv <= L; ++lv) {
                 for (auto& l : lists) l.clear();
                 for (int64_t i : at_level[lv]) {

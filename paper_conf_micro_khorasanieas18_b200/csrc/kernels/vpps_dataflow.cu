@@ -34,15 +34,13 @@ constexpr int CINMAX = 10;
 constexpr uint32_t NONE = 0xFFFFFFFFu;
 // HEAD_FB: the loss head's forward and backward in one batch (L42: softmax-NLL; dz = p - onehot needs
 // nothing but the head's own forward), emitted at the labelled cell's forward level
-enum : uint32_t { LEAF_F = 0x20, LEAF_B = 0x21, INT_F = 0x22, INT_B = 0x23, HEAD_FB = 0x42 };
-constexpr int NBF = 32;        // leaves per LEAF_F batch (E = H floats each: the shared row buffer of NB nodes)
+enum : uint32_t { LEAF_B = 0x21, INT_F = 0x22, INT_B = 0x23, HEAD_FB = 0x42 };
 
 __device__ __forceinline__ int entry_words(uint32_t op) {
     switch (op) {
         case INT_F: return 6;    // rec, hx, rec_l, hx_l, rec_r, hx_r
         case INT_B: return 9;    // rec, adj, dsrc, hd, pp, rec_l, adj_l, rec_r, adj_r
         case HEAD_FB: return 5;  // rec, rec_c, label, hx_c, hd_c
-        case LEAF_F: return 3;   // rec, token, hx
         default: return 4;       // LEAF_B: rec, adj, dsrc, hd
     }
 }
@@ -90,7 +88,6 @@ struct DCfg {
     static constexpr int O_CIN2 = O_X2 + NB * KP;
     static constexpr int O_HEAD = O_CIN2 + NB * UM * CINMAX;
     static_assert(DXB >= 2 * NB * KP && DXB >= 2 * NB * NCL * 2 * UM, "u64 staging fits in dxb");
-    static_assert(NBF * E <= NB * KP, "a LEAF_F batch's input rows fit the shared row buffer");
     static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 2 * C + 8); }
 };
 
@@ -153,17 +150,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 for (int q = 0; q < LB::CG; ++q) wb[r][t * LB::CG + q] = __ldg(src + q);
             }
         }
-    // the leaves (level 0) are computed by the group too: this CTA's rows of W_iou (3 gates x UM units x E)
-    // in the transposed-product buffers, which the first internal batch after the leaves takes over
-    static_assert(3 * UM * E <= T::DXB, "W_iou slice fits the transposed-product buffers");
-    {
-        float* Wl = sm + T::O_DXB;
-        for (int q = tid; q < 3 * UM * (E / 4); q += NTH) {
-            const int row = q / (E / 4), c4 = q - row * (E / 4), k = row / UM, uu = row - k * UM;
-            *reinterpret_cast<float4*>(Wl + row * E + 4 * c4) =
-                __ldg(reinterpret_cast<const float4*>(P.params + off[0] + (int64_t)(k * H + lc * UM + uu) * E + 4 * c4));
-        }
-    }
     if (tid < UM * 4) {
         const int uu = tid / 4, k = tid % 4, jj = lc * UM + uu;
         bias[tid] = k < 3 ? __ldg(P.params + off[5] + k * H + jj) : __ldg(P.params + off[6] + jj);
@@ -253,85 +239,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         XST(stB, 22);
         XST(stBB, 27);
         mark(1);
-        if (op == LEAF_F) {
-            // ---- leaf cells (level 0): a = W_iou x + b_iou from the shared W_iou slice, 4 leaves at a time, the
-            //      unit's 16 lanes reduce with a transposed butterfly; the leaf record [h c i o u] of this
-            //      CTA's units, h published as a tagged HX slot for the parent ----
-            constexpr int EQ = E / 4;                      // 16-byte pieces of an input row
-            for (int q = tid; q < nb * EQ; q += NTH) {
-                const int n = q / EQ, c4 = q - n * EQ;
-                const uint32_t tok = ent[n * sz + 1];
-                cp_async16(xs + n * E + 4 * c4, P.inputs + (int64_t)tok * E + 4 * c4, 16u);
-            }
-            cp_async_wait_all();
-            __syncthreads();
-            if (bt) bt[1] = bt[2] = clock64();
-            mark(3);
-            const float* Wl = sm + T::O_DXB;
-            auto leaf_group = [&](auto nnc, int n0) {
-                constexpr int NN = decltype(nnc)::value;
-                float2 a[NN][3];
-#pragma unroll
-                for (int n = 0; n < NN; ++n)
-#pragma unroll
-                    for (int k = 0; k < 3; ++k) a[n][k] = make_float2(0.f, 0.f);
-#pragma unroll
-                for (int t = 0; t < E / (4 * TU); ++t) {
-                    const int col0 = 4 * (tu + TU * t);
-                    float w[3][4];
-#pragma unroll
-                    for (int k = 0; k < 3; ++k) lds<4>(Wl + (k * UM + u) * E + col0, w[k]);
-#pragma unroll
-                    for (int n = 0; n < NN; ++n) {
-                        float xv[4];
-                        lds<4>(xs + (n0 + n) * E + col0, xv);
-#pragma unroll
-                        for (int q = 0; q < 4; q += 2)
-#pragma unroll
-                            for (int k = 0; k < 3; ++k)
-                                a[n][k] = __ffma2_rn(make_float2(w[k][q], w[k][q + 1]), make_float2(xv[q], xv[q + 1]), a[n][k]);
-                    }
-                }
-                float g3[3];
-#pragma unroll
-                for (int o = 0; o < 3; ++o) {
-                    if constexpr (NN == 4) {
-                        g3[o] = treduce4_16(a[0][o].x + a[0][o].y, a[1][o].x + a[1][o].y, a[2][o].x + a[2][o].y,
-                                            a[3][o].x + a[3][o].y, gl);
-                    } else {
-                        float k = a[0][o].x + a[0][o].y;
-#pragma unroll
-                        for (int d = 8; d >= 1; d >>= 1) k += __shfl_xor_sync(FULLMASK, k, d);
-                        g3[o] = k;
-                    }
-                }
-                constexpr int SPAN = 16 / NN;
-                const int n = n0 + gl / SPAN;
-                if (gl % SPAN == 0 && n < nb) {
-                    const uint32_t* e = ent + n * sz;
-                    const uint32_t rec = e[0];
-                    const float* b = bias + u * 4;
-                    const float i = fsigm(g3[0] + b[0]), o = fsigm(g3[1] + b[1]), uv = ftanh(g3[2] + b[2]);
-                    const float c = i * uv;
-                    const float h = o * ftanh(c);
-                    if (e[2] != NONE) st_tag(HX + (int64_t)e[2] * H + j, h, ep);
-                    pool[rec + j] = h;
-                    pool[rec + H + j] = c;
-                    pool[rec + 2 * H + j] = i;
-                    pool[rec + 3 * H + j] = o;
-                    pool[rec + 4 * H + j] = uv;
-                }
-            };
-            int n0 = 0;
-            for (; n0 + 2 < nb; n0 += 4) leaf_group(std::integral_constant<int, 4>{}, n0);
-            for (; n0 < nb; ++n0) leaf_group(std::integral_constant<int, 1>{}, n0);
-            // (the W_iou slice shares its buffer with the internal batches' scratch: every warp is done with it
-            //  before the next batch may stage there)
-            __syncthreads();
-            if (bt) bt[3] = clock64();
-            pos = next;
-            continue;
-        }
         if (op == LEAF_B) {
             // leaf backward, thread (leaf tid / U + 16 p, unit tid % U): consecutive threads read consecutive
             // units of the same slot row (coalesced), own operands and the 17 dh slots straight into

@@ -25,7 +25,6 @@ struct KParams {
 // Dataflow kernel (vpps_dataflow.cu): groups of 16 co-resident CTAs, epoch-tagged cross-CTA slots.
 struct DfParams {
     float* params;
-    const float* inputs;        // input table [rows x E]: the leaves' word vectors (level 0 runs in the kernel)
     float* grads;
     float* pool;
     const uint32_t* script;     // device blob; the group programs start at df_off

@@ -187,30 +187,25 @@ def test_device_lowering_invariants():
             pos, end = G + 2 + pre[g], G + 2 + pre[g + 1]
             while pos < end:
                 op, nb = w[pos] & 0xFF, w[pos] >> 8
-                sz = {0x20: 3, 0x22: 6, 0x42: 5, 0x23: 9, 0x21: 4}[op]
-                assert 1 <= nb <= {0x21: 64, 0x20: 32}.get(op, 16)
+                sz = {0x22: 6, 0x42: 5, 0x23: 9, 0x21: 4}[op]
+                assert 1 <= nb <= (64 if op == 0x21 else 16)
                 for k in range(nb):
                     e = w[pos + 1 + k * sz: pos + 1 + (k + 1) * sz]
                     i = rec_id[e[0]]
                     node = ref["nodes"][i]
                     assert ref["graph_group"][node["graph"]] == g
                     t += 1
-                    if op == 0x20:                      # leaf forward, before any level-1 cell of the group
-                        assert i not in seen_f and node["kind"] == "LEAF"
-                        seen_f[i] = t
-                        if e[2] != script.NONE:
-                            assert e[2] not in hx_seen
-                            hx_seen.add(e[2])
-                    elif op == 0x22:
+                    if op == 0x22:
                         assert i not in seen_f
                         for c in node["children"]:
-                            assert c in seen_f                 # leaves and internal children computed earlier
+                            assert ref["nodes"][c]["kind"] == "LEAF" or c in seen_f
                         seen_f[i] = t
                         if e[1] != script.NONE:
                             assert e[1] not in hx_seen
                             hx_seen.add(e[1])
                     elif op == 0x42:
-                        assert rec_id[e[1]] == node["children"][0] and rec_id[e[1]] in seen_f
+                        assert rec_id[e[1]] == node["children"][0] and (ref["nodes"][rec_id[e[1]]]["kind"] == "LEAF"
+                                                                         or rec_id[e[1]] in seen_f)
                         heads.add(i)
                     else:
                         assert i not in seen_b
@@ -225,5 +220,5 @@ def test_device_lowering_invariants():
         n_int = sum(n["kind"] == "INT" for n in ref["nodes"])
         n_leaf = sum(n["kind"] == "LEAF" for n in ref["nodes"])
         n_head = sum(n["kind"] == "HEAD" for n in ref["nodes"])
-        assert len(seen_f) == n_int + n_leaf and len(seen_b) == n_int + n_leaf and len(heads) == n_head
+        assert len(seen_f) == n_int and len(seen_b) == n_int + n_leaf and len(heads) == n_head
         assert len(pp_seen) == n_int == low["n_part"] and len(hx_seen) == low["n_hx"]
