@@ -100,7 +100,7 @@ def main():
     if args.batches:
         last = int(np.argmax(raw[:, 1]))
         g0 = (last // 16) * 16
-        ops = {0x21: "LEAF_B", 0x22: "INT_F", 0x23: "INT_B", 0x42: "HEAD_FB"}
+        ops = {0x20: "LEAF_F", 0x21: "LEAF_B", 0x22: "INT_F", 0x23: "INT_B", 0x42: "HEAD_FB"}
         print(f"per-batch cycles of group {last // 16} (CTA {g0} | CTA {last}): issue->staged, staged->fresh "
               f"(retry rounds), compute, batch end relative to CTA {g0}")
         nbt = int(raw[last, 2])
