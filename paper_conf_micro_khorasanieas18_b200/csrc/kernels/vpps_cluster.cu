@@ -625,14 +625,7 @@ struct GemmParams {
     int32_t tc;                  // 1: weight-gradient tiles on the tensor cores (tcgen05, 3xTF32, TMEM)
 };
 
-constexpr int TM = 128;          // tile rows (gate-gradient rows) of the tensor-core items
-// rows of an FFMA2 item: 64 (twice the items of 128-row tiles, each half as long: the slowest group's
-// items, which end the pass, spread over more SMs)
-#ifndef VPPS_DW_TMS
-#define VPPS_DW_TMS 64
-#endif
-constexpr int TMS = VPPS_DW_TMS;
-constexpr int RPT = TMS / 16;    // rows per thread
+constexpr int TM = 128;          // tile rows (gate-gradient rows)
 constexpr int TN = 64;           // tile cols (input columns)
 
 constexpr int KCH = 96;          // nodes per work item (split-K)
@@ -710,13 +703,12 @@ constexpr int KTC = 48;          // nodes per tensor-core work item (6 MMA k-ste
 
 __host__ __device__ inline int job_items(int m, int n_int, int n_leaf, int H, int E, bool dx, bool tc = false) {
     const int kch = tc ? KTC : KCH;
-    const int tm = tc ? TM : TMS;
     const int ki = (n_int + kch - 1) / kch, kl = (n_leaf + kch - 1) / kch;
     switch (m) {
-        case 0: return (3 * H / tm) * (2 * H / TN) * ki;
+        case 0: return (3 * H / TM) * (2 * H / TN) * ki;
         case 1:
-        case 2: return (H / tm) * (H / TN) * ki;
-        case 3: return (3 * H / tm) * (E / TN) * kl;
+        case 2: return (H / TM) * (H / TN) * ki;
+        case 3: return (3 * H / TM) * (E / TN) * kl;
         default: return (dx && n_leaf > 0) ? ((n_leaf + DXM - 1) / DXM) * (E / DXN) * ((3 * H + DXK - 1) / DXK) : 0;
     }
 }
@@ -932,13 +924,13 @@ __device__ __forceinline__ void dw_item(const GemmParams& P, int g, int i, float
     const int rows = (m == 0 || m == 3) ? 3 * H : H;
     const int cols = m == 0 ? 2 * H : (m == 3 ? E : H);
     const int K = m == 3 ? n_leaf : n_int;
-    const int tiles_r = rows / TMS, tiles_c = cols / TN;
+    const int tiles_r = rows / TM, tiles_c = cols / TN;
     const int kc = b / (tiles_r * tiles_c), t = b - kc * (tiles_r * tiles_c);
-    const int r0 = (t / tiles_c) * TMS, c0 = (t % tiles_c) * TN;
+    const int r0 = (t / tiles_c) * TM, c0 = (t % tiles_c) * TN;
     const int k0 = kc * KCH, nk = min(K, k0 + KCH) - k0;
     const int goff = m == 0 ? 7 * H : (m == 1 ? 10 * H : (m == 2 ? 11 * H : 5 * H));
-    float* Gs = sm;                      // [KCH][TMS]
-    float* Xs = sm + KCH * TMS;          // [KCH][TN]
+    float* Gs = sm;                      // [KCH][TM]
+    float* Xs = sm + KCH * TM;           // [KCH][TN]
     // node operands: idx[3k] = g row base, idx[3k+1] / idx[3k+2] = x row bases (left / right or token)
     if (tid < nk) {
         const int node = k0 + tid;
@@ -952,9 +944,9 @@ __device__ __forceinline__ void dw_item(const GemmParams& P, int g, int i, float
         }
     }
     __syncthreads();
-    for (int e = tid; e < nk * (TMS / 4); e += 256) {
-        const int k = e / (TMS / 4), p = (e % (TMS / 4)) * 4;
-        cp_async16(Gs + k * TMS + p, P.pool + idx[3 * k] + goff + r0 + p, 16u);
+    for (int e = tid; e < nk * (TM / 4); e += 256) {
+        const int k = e / (TM / 4), p = (e % (TM / 4)) * 4;
+        cp_async16(Gs + k * TM + p, P.pool + idx[3 * k] + goff + r0 + p, 16u);
     }
     for (int e = tid; e < nk * (TN / 4); e += 256) {
         const int k = e / (TN / 4), p = (e % (TN / 4)) * 4, c = c0 + p;
@@ -966,22 +958,19 @@ __device__ __forceinline__ void dw_item(const GemmParams& P, int g, int i, float
     }
     cp_async_wait_all();
     __syncthreads();
-    const int ty = tid / 16, tx = tid % 16;        // rows ty*RPT .. +RPT-1, cols tx*4 .. +3
-    float2 acc[RPT][2];
+    const int ty = tid / 16, tx = tid % 16;        // rows ty*8 .. +7, cols tx*4 .. +3
+    float2 acc[8][2];
 #pragma unroll
-    for (int a = 0; a < RPT; ++a) acc[a][0] = acc[a][1] = make_float2(0.f, 0.f);
+    for (int a = 0; a < 8; ++a) acc[a][0] = acc[a][1] = make_float2(0.f, 0.f);
 #pragma unroll 4
     for (int k = 0; k < nk; ++k) {
-        float ga[RPT];
-#pragma unroll
-        for (int a = 0; a < RPT; a += 4) {
-            const float4 g4 = *reinterpret_cast<const float4*>(Gs + k * TMS + ty * RPT + a);
-            ga[a] = g4.x; ga[a + 1] = g4.y; ga[a + 2] = g4.z; ga[a + 3] = g4.w;
-        }
+        const float4 g0 = *reinterpret_cast<const float4*>(Gs + k * TM + ty * 8);
+        const float4 g1 = *reinterpret_cast<const float4*>(Gs + k * TM + ty * 8 + 4);
         const float4 xv = *reinterpret_cast<const float4*>(Xs + k * TN + tx * 4);
+        const float ga[8] = {g0.x, g0.y, g0.z, g0.w, g1.x, g1.y, g1.z, g1.w};
         const float2 x01 = make_float2(xv.x, xv.y), x23 = make_float2(xv.z, xv.w);
 #pragma unroll
-        for (int a = 0; a < RPT; ++a) {
+        for (int a = 0; a < 8; ++a) {
             const float2 gg = make_float2(ga[a], ga[a]);
             acc[a][0] = __ffma2_rn(gg, x01, acc[a][0]);
             acc[a][1] = __ffma2_rn(gg, x23, acc[a][1]);
@@ -989,9 +978,13 @@ __device__ __forceinline__ void dw_item(const GemmParams& P, int g, int i, float
     }
     float* base = P.grads + P.off[m == 3 ? 0 : m + 1];
 #pragma unroll
-    for (int a = 0; a < RPT; ++a) {
+    for (int a = 0; a < 8; ++a) {
         const float v[4] = {acc[a][0].x, acc[a][0].y, acc[a][1].x, acc[a][1].y};
-        red_add<4>(base + (int64_t)(r0 + ty * RPT + a) * cols + c0 + tx * 4, v);
+#ifdef VPPS_EXP_STORE
+        *reinterpret_cast<float4*>(base + (int64_t)(r0 + ty * 8 + a) * cols + c0 + tx * 4) = make_float4(v[0], v[1], v[2], v[3]);
+#else
+        red_add<4>(base + (int64_t)(r0 + ty * 8 + a) * cols + c0 + tx * 4, v);
+#endif
     }
 }
 
