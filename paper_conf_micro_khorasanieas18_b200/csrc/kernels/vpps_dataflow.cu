@@ -23,7 +23,7 @@ namespace dev {
 namespace df {
 
 constexpr int NTH = 256;
-constexpr int NCL = 16;        // CTAs per group
+constexpr int UMC = 16;        // hidden units per CTA (CTAs per group: NCL = H / 16)
 constexpr int CHUNK = 4096;    // program words staged in shared memory
 constexpr int NB = 16;         // nodes per batch (LEAF_B: up to NBL)
 constexpr int NBL = 64;        // leaves per LEAF_B batch (no shared staging: one (unit, leaf) pair per thread pass)
@@ -69,9 +69,10 @@ __device__ __forceinline__ void st_tag4(u64* p, const float* v, uint32_t e) {
 
 template <int H, int E>
 struct DCfg {
-    static constexpr int UM = H / NCL;             // hidden units per CTA
+    static constexpr int UM = UMC;                 // hidden units per CTA
+    static constexpr int NCL = H / UM;             // CTAs per group (16 at H = 256, 8 at H = 128)
     static constexpr int TU = NTH / UM;            // threads per unit
-    static_assert(H % NCL == 0 && TU == 16, "dataflow kernel: 16 units per CTA, 16 threads per unit");
+    static_assert(H % UM == 0 && TU == 16, "dataflow kernel: 16 units per CTA, 16 threads per unit");
     using LB = Lay<2 * H, TU>;                     // internal bundle rows (i, o, u of U_iou; f) over [h_l; h_r]
     static constexpr int KP = LB::KP;              // 2H
     // column granule t of a thread covers h_l iff t < TH, for every thread of the unit (compile-time split)
@@ -97,7 +98,7 @@ template <int H, int E, bool PROF>
 __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     using T = DCfg<H, E>;
     using LB = typename T::LB;
-    constexpr int TU = T::TU, UM = T::UM, KP = T::KP;
+    constexpr int TU = T::TU, UM = T::UM, KP = T::KP, NCL = T::NCL;
     extern __shared__ __align__(16) uint32_t smw[];
     float* sm = reinterpret_cast<float*>(smw);
     uint32_t* chunk = smw;
@@ -735,15 +736,22 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
 }  // namespace dev
 
 #define VPPS_DF_VARIANT(H, E) \
-    {1, H, E, 16, (const void*)&dev::df::vpps_df<H, E, false>, &dev::df::DCfg<H, E>::smem_bytes}
+    {1, H, E, dev::df::DCfg<H, E>::NCL, (const void*)&dev::df::vpps_df<H, E, false>, &dev::df::DCfg<H, E>::smem_bytes}
 
 static const Variant kDfVariants[] = {
     VPPS_DF_VARIANT(256, 256),    // target: binary Tree-LSTM H = E = 256, groups of 16 CTAs
+    VPPS_DF_VARIANT(128, 128),    // H = 128: groups of 8 CTAs (16 groups on 128 SMs)
+    VPPS_DF_VARIANT(128, 256),
 };
 
 // the profiling instantiation of a dataflow variant (same shared memory, in-kernel trace enabled)
 const void* df_prof_fn(const void* fn) {
-    if (fn == (const void*)&dev::df::vpps_df<256, 256, false>) return (const void*)&dev::df::vpps_df<256, 256, true>;
+#define VPPS_DF_PROF(H, E) \
+    if (fn == (const void*)&dev::df::vpps_df<H, E, false>) return (const void*)&dev::df::vpps_df<H, E, true>;
+    VPPS_DF_PROF(256, 256)
+    VPPS_DF_PROF(128, 128)
+    VPPS_DF_PROF(128, 256)
+#undef VPPS_DF_PROF
     return nullptr;
 }
 

@@ -18,7 +18,7 @@
 // per thread runs the cell.  (A 4 x 3 thread tile was shared-memory-issue bound: mio_throttle and short
 // scoreboard stalls, FMA pipe 30 %, 13 us per TGT pass, profiles/r03 ncu.)
 // The input-table gradient dX = W_iouᵀ g_leaf is a job of the gradient GEMM (vpps_dw_gemm, vpps_cluster.cu).
-// Requires E == KMAX and H % 16 == 0 (the cluster / dataflow variants are H = E = 256).
+// Requires E in {128, 256} (the tensor-core variant: E == 256) and H % 16 == 0.
 #include <algorithm>
 #include <cstdlib>
 #include "vpps_kernel.cuh"
@@ -32,12 +32,11 @@ constexpr int LM = 64;          // leaves per tile
 constexpr int LU = 16;          // hidden units per tile (x 3 gates = 48 W_iou rows)
 constexpr int NT = 256;         // 4 K slices (alternating 4-column steps) x 64 threads
 constexpr int NTC = 128;        // + 4 warps that only clear (warp-specialised: the GEMM never waits for them)
-constexpr int KMAX = 256;       // E == KMAX
-constexpr int KST = 64;         // K columns per cp.async group
-constexpr int NSTG = KMAX / KST;
-static_assert(NSTG == 4, "the wait_group sequence below assumes 4 K groups");
-constexpr int KS = KMAX + 4;    // row stride in floats (= 4 mod 32: conflict-free 16-byte column reads)
-constexpr size_t SMEM = (size_t)(LM + 3 * LU) * KS * sizeof(float);
+constexpr int KMAX = 256;       // largest E (the tensor-core variant: E == KMAX)
+constexpr int KST = 64;         // K columns per cp.async group (E / KST groups)
+// row stride in floats E + 4 (= 4 mod 32: conflict-free 16-byte column reads)
+template <int E>
+constexpr size_t smem_of() { return (size_t)(LM + 3 * LU) * (E + 4) * sizeof(float); }
 
 // Per-pass clearing folded into the leaf kernel (it runs first in the pass): up to 4 float ranges
 // (multiples of 4 floats) are zeroed by a grid-stride loop, and the device pass counter is advanced.
@@ -61,7 +60,8 @@ __global__ void __launch_bounds__(NT + NTC, 1) vpps_leaf_fwd(const float* __rest
                                                        const float* __restrict__ inputs, float* pool,
                                                        const uint32_t* __restrict__ leaves, int n_leaf, int H,
                                                        const PassClear pc) {
-    static_assert(E == KMAX, "leaf GEMM: E == 256");
+    static_assert(E == 128 || E == 256, "leaf GEMM: E in {128, 256}");
+    constexpr int NSTG = E / KST, KS = E + 4;
     extern __shared__ __align__(16) float lsm[];
     __shared__ uint32_t lrec[LM];
     float* As = lsm;                 // [64 leaves][KS]: x rows
@@ -148,20 +148,25 @@ __global__ void __launch_bounds__(NT + NTC, 1) vpps_leaf_fwd(const float* __rest
             }
         }
     };
-    asm volatile("cp.async.wait_group 3;" ::: "memory");
-    gemm_sync();
-    if (pf) pst[2] = gtimer();
-    stage(0);
-    asm volatile("cp.async.wait_group 2;" ::: "memory");
-    gemm_sync();
-    stage(1);
+    if constexpr (NSTG == 4) {
+        asm volatile("cp.async.wait_group 3;" ::: "memory");
+        gemm_sync();
+        if (pf) pst[2] = gtimer();
+        stage(0);
+        asm volatile("cp.async.wait_group 2;" ::: "memory");
+        gemm_sync();
+        stage(1);
+    } else {
+        static_assert(NSTG == 2, "E / KST cp.async groups: 2 or 4");
+    }
     asm volatile("cp.async.wait_group 1;" ::: "memory");
     gemm_sync();
-    stage(2);
+    if (NSTG == 2 && pf) pst[2] = gtimer();
+    stage(NSTG - 2);
     asm volatile("cp.async.wait_group 0;" ::: "memory");
     gemm_sync();
     if (pf) pst[3] = gtimer();
-    stage(3);
+    stage(NSTG - 1);
     if (pf) pst[4] = gtimer();
     // sum the K slices through shared memory (the staging is dead): red[slice][t64][49]
     constexpr int RS = 49;
@@ -422,13 +427,14 @@ void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float*
                      int32_t n_leaf, int32_t H, int32_t E, float* const* zero_ptr, const int64_t* zero_n,
                      uint32_t* epoch, cudaStream_t s, const void* prefetch, int64_t prefetch_bytes) {
     using namespace dev::leaf;
-    if (E != KMAX || H % LU) return;   // the cluster / dataflow variants are H = E = 256 (api.cu checks)
+    if ((E != 128 && E != KMAX) || H % LU) return;   // (api.cu admits only built (H, E) variants)
     PassClear pc{};
     static const int exp_ = getenv("VPPS_LEAF_EXP") ? atoi(getenv("VPPS_LEAF_EXP")) : 0;   // measurement only
     // VPPS_LEAF_TC=1: the tensor-core variant (parity-green; measured slower than the FFMA tiles, 17.5 vs
     // 12.3 us per TGT pass: the register-transit staging of the hi / lo split and the first TMEM allocation
     // sit on its critical path)
-    static const bool simt = !(getenv("VPPS_LEAF_TC") && atoi(getenv("VPPS_LEAF_TC")) != 0);
+    static const bool simt_env = !(getenv("VPPS_LEAF_TC") && atoi(getenv("VPPS_LEAF_TC")) != 0);
+    const bool simt = simt_env || E != KMAX;
     for (int r = 0; r < 4; ++r) { pc.ptr[r] = zero_ptr ? zero_ptr[r] : nullptr; pc.n[r] = zero_ptr ? zero_n[r] : 0; }
     if (exp_ & 1) for (int r = 0; r < 4; ++r) if (r != 2) pc.n[r] = 0;     // no clearing (but the counters)
     if (exp_ & 2) n_leaf = 0;                                                // clearing only
@@ -437,8 +443,13 @@ void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float*
     pc.pf_bytes = prefetch ? prefetch_bytes : 0;
     if (simt) {
         const int tiles = std::max(((n_leaf + LM - 1) / LM) * (H / LU), 148);
-        if (h_leaf_prof_on) vpps_leaf_fwd<256, true><<<tiles, NT + NTC, SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
-        else vpps_leaf_fwd<256, false><<<tiles, NT + NTC, SMEM, s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
+        if (E == 128) {
+            if (h_leaf_prof_on) vpps_leaf_fwd<128, true><<<tiles, NT + NTC, smem_of<128>(), s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
+            else vpps_leaf_fwd<128, false><<<tiles, NT + NTC, smem_of<128>(), s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
+        } else {
+            if (h_leaf_prof_on) vpps_leaf_fwd<256, true><<<tiles, NT + NTC, smem_of<256>(), s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
+            else vpps_leaf_fwd<256, false><<<tiles, NT + NTC, smem_of<256>(), s>>>(W, b, inputs, pool, leaves, n_leaf, H, pc);
+        }
     } else {
         // GEMM tiles first, then clearing CTAs: the SMs left over (at least 32 CTAs)
         const int tiles = ((n_leaf + TL - 1) / TL) * (H / LU);
@@ -450,8 +461,10 @@ void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float*
 // per-device launch attributes of the leaf kernels (vpps_define_model calls this after cudaSetDevice)
 cudaError_t setup_leaf_attrs() {
     using namespace dev::leaf;
-    cudaError_t e = cudaFuncSetAttribute(vpps_leaf_fwd<256, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
-    if (e == cudaSuccess) e = cudaFuncSetAttribute(vpps_leaf_fwd<256, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+    cudaError_t e = cudaFuncSetAttribute(vpps_leaf_fwd<256, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_of<256>());
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(vpps_leaf_fwd<256, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_of<256>());
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(vpps_leaf_fwd<128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_of<128>());
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(vpps_leaf_fwd<128, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_of<128>());
     if (e == cudaSuccess) e = cudaFuncSetAttribute(vpps_leaf_fwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TC_SMEM);
     return e;
 }

@@ -274,6 +274,8 @@ def candidate_options(cell: str, H: int, C: int):
     if cell == "binary":
         if H == 256:
             out += [dict(cluster=16, dataflow=True), dict(cluster=16)]
+        elif H == 128:
+            out += [dict(cluster=8, dataflow=True)]          # groups of H / 16 CTAs
         out += [dict(groups=g, level=-1) for g in (1, 2, 4)] + [dict(level=1)]
     elif cell == "childsum":
         out += [dict(groups=g) for g in (1, 2, 4)]

@@ -126,6 +126,14 @@ def test_binary_target_dataflow_groups(b):
     check("binary", 256, 256, 5, synth.config_batch("tgt", b), 4096, seed=21 + b, cluster=16, dataflow=True)
 
 
+@pytest.mark.parametrize("E,b", [(128, 0), (256, 5), (128, 11)])
+def test_dataflow_groups_hidden_128(E, b):
+    """Dataflow path at H = 128: groups of 8 CTAs (H / 16 units of 16), 16 groups; the leaf GEMM at E = 128
+    (two K groups) or 256 (PAPER L241 / Fig.9: the hidden size sets the register partition)."""
+    check("binary", 128, E, 5, synth.config_batch("tgt", b), 4096, seed=41 + b, cluster=8, dataflow=True)
+    check("binary", 128, E, 5, [[((), 3, 2)]], 8, cluster=8, dataflow=True)               # one leaf
+
+
 def test_dataflow_degenerate_and_repeated_passes():
     check("binary", 256, 256, 5, [[((), 3, 2)]], 8, cluster=16, dataflow=True)           # one leaf
     check("binary", 256, 256, 5, _trees(12, 3, (1, 9), 30, 5), 30, cluster=16, dataflow=True, want_dx=False)

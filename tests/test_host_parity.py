@@ -220,8 +220,18 @@ def test_device_lowering_bit_exact(vpps, G, dataflow):
     SST-shaped batches of 1 / 4 / 16 / 64 trees, degenerate ones (a lone labelled leaf, labels on inner
     nodes) and the bench's TGT batches.  A dataflow model leaves the SPEC words out of the blob and still
     returns them, bit-exact, on request."""
-    H, E, C = 256, 256, 5
-    m = vpps.Model("binary", H, E, C, n_sm=16 * G, groups=G, cluster=16, dataflow=dataflow, plan_only=True)
+    _lowering_case(vpps, 256, 256, 16, G, dataflow)
+
+
+def test_device_lowering_bit_exact_h128(vpps):
+    """The same at H = 128 (groups of 8 CTAs, 16 groups, E = 128): the lowering does not depend on the
+    group size; the kernel derives its slot strides from H."""
+    _lowering_case(vpps, 128, 128, 8, 16, True)
+
+
+def _lowering_case(vpps, H, E, ncl, G, dataflow):
+    C = 5
+    m = vpps.Model("binary", H, E, C, n_sm=ncl * G, groups=G, cluster=ncl, dataflow=dataflow, plan_only=True)
     rng = np.random.default_rng(200 + G)
     inner = [((), 0, 1), ((), 1, -1), ((0, 1), -1, 3), ((), 2, -1), ((2, 3), -1, 0)]
     batches = [synth.tree_batch(rng, b, (1, 50), 64, C) for b in (1, 4, 16, 64)]

@@ -47,6 +47,9 @@ CASES = [
     ("BiLSTMwChar H256 E256 MLP256 B16 (chain)", "bilstmchar", "bilstmchar", 256, 256, 9, 4096, 16, {"mlp": 256}, {}),
     ("c4 BiLSTM tagger H512 B16 (per-step products)", "c4", "bilstm", 512, 512, 9, 4096, 16, {"mlp": 256, "chain": -1}, {}),
     ("tgt binary H256 B16 (level path)", "tgt", "binary", 256, 256, 5, 4096, 16, {"level": 1}, {}),
+    ("tgt binary H128 E128 B16 (dataflow, 8-CTA groups)", "tgt", "binary", 128, 128, 5, 4096, 16, {"cluster": 8, "dataflow": True}, {}),
+    ("tgt binary H128 E128 B16 (level path)", "tgt", "binary", 128, 128, 5, 4096, 16, {"level": 1}, {}),
+    ("tgt binary H128 E128 B16 (grid)", "tgt", "binary", 128, 128, 5, 4096, 16, {"level": -1}, {}),
     ("tgt binary H256 B1 (dataflow)", "tgt", "binary", 256, 256, 5, 4096, 1, {"cluster": 16, "dataflow": True}, {}),
     ("tgt binary H256 B4 (dataflow)", "tgt", "binary", 256, 256, 5, 4096, 4, {"cluster": 16, "dataflow": True}, {}),
     ("tgt binary H256 B16 (dataflow)", "tgt", "binary", 256, 256, 5, 4096, 16, {"cluster": 16, "dataflow": True}, {}),
