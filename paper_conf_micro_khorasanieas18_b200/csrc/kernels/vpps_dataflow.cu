@@ -155,10 +155,10 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         const int uu = tid / 4, k = tid % 4, jj = lc * UM + uu;
         bias[tid] = k < 3 ? __ldg(P.params + off[5] + k * H + jj) : __ldg(P.params + off[6] + jj);
     }
-    if (holds_head) {
-        for (int i = tid; i < C * H; i += NTH) { Wo[i] = __ldg(P.params + off[4] + i); dWo[i] = 0.f; }
-        for (int i = tid; i < C; i += NTH) { bo[i] = __ldg(P.params + off[7] + i); dbo[i] = 0.f; }
-    }
+    // the loss head runs in every CTA of the group (each needs dz for its own units' dh): W_out, b_out in
+    // every CTA; dW_out accumulates this CTA's columns only
+    for (int i = tid; i < C * H; i += NTH) { Wo[i] = __ldg(P.params + off[4] + i); dWo[i] = 0.f; }
+    for (int i = tid; i < C; i += NTH) { bo[i] = __ldg(P.params + off[7] + i); dbo[i] = 0.f; }
     float dbacc[4] = {0.f, 0.f, 0.f, 0.f};   // bias gradients of unit lc * UM + tid % UM (INT_B mapping)
     float dbleaf[3] = {0.f, 0.f, 0.f};       // ... of unit lc * UM + tid % UM (LEAF_B mapping)
     uint64_t* prof = PROF && P.prof ? P.prof + (int64_t)blockIdx.x * P.prof_stride : nullptr;
@@ -219,7 +219,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         const uint32_t* ent = chunk + (pos - cbase) + 1;
         const uint32_t next = pos + 1 + nb * sz;
         const bool is_head = op == HEAD_FB;
-        if (is_head && !holds_head) { pos = next; continue; }
         ++nbatch;
         // staging buffers of this batch: the other pair than the previous batch's (a thread still computing
         // that batch reads only those); batch b+2 reuses them after batch b+1's staging barrier
@@ -467,64 +466,58 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         if (bt) { bt[2] = clock64(); bt[4] |= (uint64_t)rounds << 8; }
 
         mark(is_head ? 6 : (op == INT_F ? 3 : 4));
-        if (is_head) {            // loss heads (L42) on the CTA holding W_out
-            constexpr int KPH = KP;
-            // forward: logits z = W_out h + b_out, softmax-NLL (L42); backward: dz = p - onehot(y),
-            // dW_out += dz h^T, db_out += dz, dh = W_out^T dz -> HD slots of the labelled cell
-            for (int pi = warp; pi < nb * C; pi += NTH / 32) {
-                const int n = pi / C, c = pi - n * C;
-                float s = 0.f;
-                for (int k = 4 * lane; k < H; k += 128) {
-                    const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
-                    const float4 h4 = *reinterpret_cast<const float4*>(xs + n * KPH + k);
-                    s += w4.x * h4.x + w4.y * h4.y + w4.z * h4.z + w4.w * h4.w;
-                }
-                s = warp_sum(s);
-                if (lane == 0) zs[n * ZC + c] = s + bo[c];
-            }
-            __syncthreads();
+        if (is_head) {
+            // loss heads (L42) in every CTA of the group, one warp per labelled node: logits z = W_out h + b_out
+            // (lane c keeps z_c), softmax-NLL, dz = p - onehot(y); the dh = W_out^T dz of this CTA's own units
+            // goes to its HD slots, which only this CTA's backward of the labelled cell reads (no cross-CTA
+            // exchange: every CTA forms dz itself from the staged h).  CTA 0 writes p and the loss.
             for (int n = warp; n < nb; n += NTH / 32) {
                 const uint32_t* e = ent + n * sz;
-                const float zl = lane < C ? zs[n * ZC + lane] : -INFINITY;
-                const float m = warp_max(zl);
-                const float lse = m + logf(warp_sum(lane < C ? expf(zl - m) : 0.f));
-                const float p = expf(zl - lse);
-                if (lane < C) {
-                    pool[e[0] + lane] = p;
-                    zs[n * ZC + lane] = p - (lane == (int)e[2] ? 1.f : 0.f);
+                float z = -INFINITY;
+                for (int c = 0; c < C; ++c) {
+                    float s = 0.f;
+#pragma unroll
+                    for (int k = 4 * lane; k < H; k += 128) {
+                        const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
+                        const float4 h4 = *reinterpret_cast<const float4*>(xs + n * KP + k);
+                        s += w4.x * h4.x + w4.y * h4.y + w4.z * h4.z + w4.w * h4.w;
+                    }
+                    s = warp_sum(s);
+                    if (lane == c) z = s + bo[c];
                 }
-                const float zy = __shfl_sync(FULLMASK, zl, (int)e[2]);
-                if (lane == 0) {
-                    pool[e[0] + C] = lse - zy;
-                    atomicAdd(pool + P.loss_word, lse - zy);   // aggregated loss node (L205)
+                const float m = warp_max(z);
+                const float lse = m + logf(warp_sum(lane < C ? expf(z - m) : 0.f));
+                const float p = expf(z - lse);
+                const int y = (int)e[2];
+                const float dz = lane < C ? p - (lane == y ? 1.f : 0.f) : 0.f;
+                zs[n * ZC + lane] = dz;
+                if (holds_head) {
+                    if (lane < C) pool[e[0] + lane] = p;
+                    const float zy = __shfl_sync(FULLMASK, z, y);
+                    if (lane == 0) {
+                        pool[e[0] + C] = lse - zy;
+                        atomicAdd(pool + P.loss_word, lse - zy);   // aggregated loss node (L205)
+                    }
                 }
+                const int jh = lc * UM + (lane % UM);
+                float dh = 0.f;
+                for (int c = 0; c < C; ++c) dh = fmaf(Wo[c * H + jh], __shfl_sync(FULLMASK, dz, c), dh);
+                const uint32_t hd = e[4];
+                if (hd != NONE && lane < UM) st_tag(HD + (int64_t)hd * H + jh, dh, ep);
             }
             __syncthreads();
-            // the labelled cell's dh first: the group's CTAs wait on these HD slots; the head's own
-            // parameter gradients follow off the critical path
-            for (int i = tid; i < nb * (H / 4); i += NTH) {   // dh of the labelled node -> HD slots
-                const int n = i / (H / 4), k = (i - n * (H / 4)) * 4;
-                float v4[4] = {0.f, 0.f, 0.f, 0.f};
-                for (int c = 0; c < C; ++c) {
-                    const float dzc = zs[n * ZC + c];
-                    const float4 w4 = *reinterpret_cast<const float4*>(Wo + c * H + k);
-                    v4[0] = fmaf(w4.x, dzc, v4[0]); v4[1] = fmaf(w4.y, dzc, v4[1]);
-                    v4[2] = fmaf(w4.z, dzc, v4[2]); v4[3] = fmaf(w4.w, dzc, v4[3]);
+            for (int i = tid; i < C * UM; i += NTH) {             // dW_out of this CTA's columns
+                const int c = i / UM, k = lc * UM + (i - c * UM);
+                float s = 0.f;
+                for (int n = 0; n < nb; ++n) s = fmaf(zs[n * ZC + c], xs[n * KP + k], s);
+                dWo[c * H + k] += s;
+            }
+            if (holds_head)
+                for (int c = tid; c < C; c += NTH) {
+                    float s = 0.f;
+                    for (int n = 0; n < nb; ++n) s += zs[n * ZC + c];
+                    dbo[c] += s;
                 }
-                const uint32_t hd = ent[n * sz + 4];
-                if (hd != NONE) st_tag4(HD + (int64_t)hd * H + k, v4, ep);
-            }
-            for (int c = tid; c < C; c += NTH) {
-                float s = 0.f;
-                for (int n = 0; n < nb; ++n) s += zs[n * ZC + c];
-                dbo[c] += s;
-            }
-            for (int i = tid; i < C * H; i += NTH) {
-                const int c = i / H, k = i - c * H;
-                float s = 0.f;
-                for (int n = 0; n < nb; ++n) s = fmaf(zs[n * ZC + c], xs[n * KPH + k], s);
-                dWo[i] += s;
-            }
         } else if (op == INT_F) {
             // ---- forward of internal cells: matvec from registers (L123), 4 nodes at a time; the unit's
             //      16 lanes reduce with a transposed butterfly; the lane holding node n's gates updates it ----
@@ -718,11 +711,13 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
 #pragma unroll
         for (int k = 0; k < 3; ++k) atomicAdd(P.grads + off[5] + k * H + lc * UM + lane, dbleaf[k]);
     }
-    if (holds_head) {
-        __syncthreads();
-        for (int i = tid; i < C * H; i += NTH) atomicAdd(P.grads + off[4] + i, dWo[i]);
-        for (int i = tid; i < C; i += NTH) atomicAdd(P.grads + off[7] + i, dbo[i]);
+    __syncthreads();
+    for (int i = tid; i < C * UM; i += NTH) {
+        const int c = i / UM, k = lc * UM + (i - c * UM);
+        atomicAdd(P.grads + off[4] + c * H + k, dWo[c * H + k]);
     }
+    if (holds_head)
+        for (int i = tid; i < C; i += NTH) atomicAdd(P.grads + off[7] + i, dbo[i]);
     // this CTA's records and gradient contributions are complete: count it for the GEMM tiles of its group
     if (P.done) {
         __threadfence();
