@@ -92,6 +92,20 @@ def main():
                 print(f"  group {g}: done {gend[g]:.1f} us; its {int(sel.sum())} items run {st[sel].min():.1f}-{en[sel].max():.1f} us")
         kern_end = (raw[:, 1].max() - t0) / 1e3
         print(f"  items finished before the last group ended: {(en <= kern_end).mean()*100:.0f} %")
+        # the last group's items: how they spread over SMs (items sharing an SM run slower)
+        gl = int(np.argmax(gend))
+        sel = gtr[:, 0] == gl
+        sms = gtr[sel, 4].astype(int)
+        cnt = np.bincount(sms, minlength=160)
+        dur = en[sel] - st[sel]
+        occ = []
+        for k in np.nonzero(sel)[0]:
+            same = (gtr[:, 4] == gtr[k, 4]) & (st < en[k]) & (en > st[k])
+            occ.append(int(same.sum()))
+        occ = np.array(occ)
+        print(f"  last group {gl}: {int(sel.sum())} items on {int((cnt > 0).sum())} SMs (max {int(cnt.max())} per SM); "
+              f"item time {dur.min():.1f}-{dur.max():.1f} us; items overlapping on their SM: "
+              + ", ".join(f"{v}: {int((occ == v).sum())}" for v in sorted(set(occ.tolist()))))
     mean = secs.mean(0)
     slow = secs[np.argmax(raw[:, 1])]
     tot = mean.sum()
