@@ -650,7 +650,7 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         const int64_t pf_floats = m->n_floats - m->offsets[1];
         launch_leaf_fwd(W_iou, m->params + m->offsets[5], inputs, m->pool, leaf_list, (int32_t)s->s.n_leaf,
                         m->plan.H, m->plan.E, zero_ptr, zero_n, m->d_epoch, st, m->params + m->offsets[1],
-                        pf_floats * (int64_t)sizeof(float));
+                        pf_floats * (int64_t)sizeof(float), n_rows);
         if (m->k_before) CK(cudaEventRecord(m->k_before, st));
         const void* dfn = m->prof ? df_prof_fn(m->var->fn) : m->var->fn;
         if (m->prof) CK(cudaFuncSetAttribute(dfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)m->smem));

@@ -99,7 +99,8 @@ bool launch_dw_tc(const float* pool, const float* inputs, float* d_inputs, float
 // and advances the device pass counter `epoch` (if not null): the per-pass clearing without memset calls.
 void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float* pool, const uint32_t* leaves,
                      int32_t n_leaf, int32_t H, int32_t E, float* const* zero_ptr, const int64_t* zero_n,
-                     uint32_t* epoch, cudaStream_t s, const void* prefetch = nullptr, int64_t prefetch_bytes = 0);
+                     uint32_t* epoch, cudaStream_t s, const void* prefetch = nullptr, int64_t prefetch_bytes = 0,
+                     int64_t n_rows = 0);   // n_rows > 0: rows of `inputs` (enables the TMA-fed variant)
 // Per-device function attributes (dynamic shared memory) of the gradient GEMM and the leaf kernels.
 cudaError_t setup_dw_gemm_attrs();
 cudaError_t setup_leaf_attrs();

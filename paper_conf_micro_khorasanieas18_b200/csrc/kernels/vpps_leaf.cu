@@ -21,6 +21,10 @@
 // Requires E in {128, 256} (the tensor-core variant: E == 256) and H % 16 == 0.
 #include <algorithm>
 #include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include "vpps_kernel.cuh"
 #include "dev_common.cuh"
 
@@ -253,6 +257,18 @@ __device__ __forceinline__ void split_store(float* hi, float* lo, uint32_t off, 
     *reinterpret_cast<float4*>(hi + off) = h;
     *reinterpret_cast<float4*>(lo + off) = make_float4(v.x - h.x, v.y - h.y, v.z - h.z, v.w - h.w);
 }
+__device__ __forceinline__ void mbar_wait_parity(uint32_t mbar, uint32_t parity) {
+    uint32_t ok = 0;
+    while (!ok)
+        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}\n"
+                     : "=r"(ok) : "r"(mbar), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void tcl_ld16(uint32_t ta, uint32_t (&r)[16]) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+                   "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+                 : "r"(ta));
+}
 #define LF_LD8(r, addr)                                                                                        \
     asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"                     \
                  : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]) \
@@ -414,6 +430,218 @@ __global__ void __launch_bounds__(NT, 1) vpps_leaf_fwd_tc(const float* __restric
     if (pf) pst[5] = gtimer();
 }
 
+
+// ---- TMA-fed tensor-core variant (opt-in, VPPS_LEAF_TMA=1): vpps_leaf_fwd_tma ----
+// D[128 leaves][48 rows] = Σ_k x[tok_l][k] W_iou[row][k] as tcgen05.mma kind::tf32 with both operands fed by
+// the Tensor Memory Accelerator: the leaf rows gathered by token (cp.async.bulk.tensor.2d ... tile::gather4,
+// 4 rows per copy) and the 3 x 16 W_iou rows of the tile's units as 2D tiles, K-major in the SWIZZLE_128B
+// layout (8-row x 128-byte atoms; the UMMA descriptor advances 32 B per k-step of 8).  The tensor core
+// reads an FP32 operand as TF32 by truncation (tools/tma_probe.cu pins it: raw TF32 2.4e-4, 3xTF32 with
+// lo = v - trunc(v) 7.6e-7 relative), so the raw tiles are the hi halves and six converter warps only write
+// the lo halves (elementwise, same swizzled offsets): D = A·B + A·B_lo + A_lo·B, FP32 accuracy.
+// Warp roles: warp 0 issues the TMA copies of every 32-column K chunk at once (8 raw chunks of 22 KB),
+// warps 2-7 write the lo halves into a 2-stage ring, warp 1 issues the MMAs (12 per chunk) and frees a lo
+// stage by tcgen05.commit; warps 4-7 then read the accumulator (TMEM lane = leaf) and run the leaf cell.
+// CTAs behind the tiles do the per-pass clearing and pull vpps_df's recurrent weights into L2.
+// Parity-green but measured slower than the FFMA tiles (TGT step 133 -> 145 us; leaf phase ~20 vs ~9 us):
+// the 32 gather4 copies per K chunk (4 rows x 128 B each, the widest box SWIZZLE_128B allows) arrive one
+// chunk per ~1.5 us, while the MMAs of a chunk take ~0.3 us (tools/tma_probe.cu: M = 128, N = 48 kind::tf32
+// 50 cycles per MMA, N = 128 65 cycles = the TF32 peak).
+namespace tma {
+constexpr int ML = 128, NR = 48, KCT = 32;
+constexpr int NRAW = 8, NLO = 2;                                     // raw chunks (all of K <= 256) / lo stages
+constexpr int A_BYTES = ML * KCT * 4, B_BYTES = NR * KCT * 4;          // one raw chunk (16 KB, 6 KB)
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;                       // A | B of one chunk (raw or lo)
+constexpr size_t SMEM = (size_t)(NRAW + NLO) * STAGE_BYTES + 1024;
+constexpr int NCONV = 192;                                           // converter threads (warps 2-7)
+constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(NR >> 3) << 17) | ((uint32_t)(ML >> 4) << 24);
+
+__device__ __forceinline__ uint64_t desc_sw128(uint32_t saddr) {
+    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
+           ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
+}
+__device__ __forceinline__ void mma(uint32_t d, uint64_t a, uint64_t b, int acc) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                 "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}\n"
+                 ::"r"(d), "l"(a), "l"(b), "r"(IDESC), "r"(acc));
+}
+__device__ __forceinline__ void arrive(uint32_t mbar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(mbar) : "memory");
+}
+}  // namespace tma
+
+__global__ void __launch_bounds__(256, 1) vpps_leaf_fwd_tma(const __grid_constant__ CUtensorMap tmX,
+                                                          const __grid_constant__ CUtensorMap tmW,
+                                                          const float* __restrict__ b, float* pool,
+                                                          const uint32_t* __restrict__ leaves, int n_leaf, int H, int E,
+                                                          int tiles, const PassClear pc) {
+    using namespace tma;
+    extern __shared__ __align__(1024) uint8_t msm[];
+    uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(msm) + 1023) & ~uintptr_t(1023));
+    __shared__ uint32_t tmem_base;
+    __shared__ __align__(8) uint64_t full[NRAW], lo_full[NLO], lo_empty[NLO], done;
+    __shared__ float bias_s[3 * LU];
+    __shared__ int tok_s[ML];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    const bool pfon = g_leaf_prof_on && blockIdx.x < 1024;           // measurement only (tools/leaf_prof.py)
+    const bool pf = pfon && tid == 0;
+    uint64_t* pst = g_leaf_prof + blockIdx.x * 8;
+    if (pf) pst[0] = gtimer();
+    if ((int)blockIdx.x >= tiles) {
+        // clearing CTAs: per-pass clearing, the pass counter, and vpps_df's recurrent weights into L2
+        const int cb = blockIdx.x - tiles, ncb = gridDim.x - tiles;
+        if (pc.epoch && cb == 0 && tid == 0) {
+            uint32_t e = *pc.epoch + 1;
+            *pc.epoch = e ? e : 1u;                               // 0 marks never-written slots
+        }
+        const int64_t stride = (int64_t)ncb * 256;
+        for (int r = 0; r < 4; ++r) {
+            float4* p = reinterpret_cast<float4*>(pc.ptr[r]);
+            const int64_t n4 = pc.ptr[r] ? pc.n[r] / 4 : 0;
+            for (int64_t i = (int64_t)cb * 256 + tid; i < n4; i += stride) p[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+        for (int64_t i = (int64_t)cb * 256 + tid; i < pc.pf_bytes / 128; i += stride)
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(pc.pf + i * 128));
+        if (pf) pst[6] = gtimer();
+        return;
+    }
+    const int tiles_u = H / LU;
+    const int l0 = (blockIdx.x / tiles_u) * ML, j0 = (blockIdx.x % tiles_u) * LU;
+    const int nch = E / KCT;
+    if (warp == 0) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base)), "r"(64));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+        // the tile's tokens (rows past n_leaf gather row 0; their results are dropped)
+#pragma unroll
+        for (int q = 0; q < ML / 32; ++q) {
+            const int l = l0 + 32 * q + lane;
+            tok_s[32 * q + lane] = l < n_leaf ? (int)__ldg(leaves + 2 * l + 1) : 0;
+        }
+    }
+    if (tid == 32) {
+        for (int st = 0; st < NRAW; ++st) asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&full[st])));
+        for (int st = 0; st < NLO; ++st) {
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(&lo_full[st])), "r"(NCONV));
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&lo_empty[st])));
+        }
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&done)));
+        asm volatile("fence.mbarrier_init.release.cluster;");
+        asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmW)) : "memory");
+    }
+    if (tid >= 64 && tid < 64 + 3 * LU) {                          // b_iou of the tile's units
+        const int k = tid - 64;
+        bias_s[k] = __ldg(b + (k / LU) * H + j0 + k % LU);
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem = tmem_base;
+    if (pf) pst[1] = gtimer();
+    // raw chunk c at sm + c * STAGE_BYTES (every K chunk in flight at once), lo stage q after them
+    auto raw_at = [&](int c) { return sm + c * STAGE_BYTES; };
+    auto lo_at = [&](int q) { return sm + (NRAW + q) * STAGE_BYTES; };
+    if (warp == 0) {
+        if (lane == 0) {
+            const uint64_t mx = reinterpret_cast<uint64_t>(&tmX), mw = reinterpret_cast<uint64_t>(&tmW);
+            for (int c = 0; c < nch; ++c) {
+                uint8_t* Ar = raw_at(c);
+                uint8_t* Br = Ar + A_BYTES;
+                const uint32_t fb = smem_u32(&full[c]);
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(fb), "r"(A_BYTES + B_BYTES) : "memory");
+                for (int q = 0; q < ML / 4; ++q)
+                    asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes"
+                                 " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];"
+                                 ::"r"(smem_u32(Ar + q * 512)), "l"(mx), "r"(c * KCT), "r"(tok_s[4 * q]), "r"(tok_s[4 * q + 1]),
+                                   "r"(tok_s[4 * q + 2]), "r"(tok_s[4 * q + 3]), "r"(fb) : "memory");
+                for (int g = 0; g < 3; ++g)
+                    asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+                                 " [%0], [%1, {%2, %3}], [%4];"
+                                 ::"r"(smem_u32(Br + g * LU * 128)), "l"(mw), "r"(c * KCT), "r"(g * H + j0), "r"(fb) : "memory");
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            for (int c = 0; c < nch; ++c) {
+                const int q = c % NLO;
+                mbar_wait_parity(smem_u32(&lo_full[q]), (c / NLO) & 1);
+                asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                const uint32_t a = smem_u32(raw_at(c)), bb = a + A_BYTES, al = smem_u32(lo_at(q)), bl = al + A_BYTES;
+#pragma unroll
+                for (int k = 0; k < KCT / 8; ++k) {
+                    const uint32_t o = 32 * k;
+                    mma(tmem, desc_sw128(a + o), desc_sw128(bb + o), c > 0 || k > 0);
+                    mma(tmem, desc_sw128(a + o), desc_sw128(bl + o), 1);
+                    mma(tmem, desc_sw128(al + o), desc_sw128(bb + o), 1);
+                }
+                asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                             ::"r"(smem_u32(&lo_empty[q])) : "memory");
+            }
+            asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                         ::"r"(smem_u32(&done)) : "memory");
+        }
+    } else {
+        // converters: lo = v - trunc_tf32(v) of the landed chunk, at the same (swizzled) offsets
+        const int ct = tid - 64;
+        for (int c = 0; c < nch; ++c) {
+            const int q = c % NLO;
+            mbar_wait_parity(smem_u32(&full[c]), 0);
+            if (c >= NLO) mbar_wait_parity(smem_u32(&lo_empty[q]), ((c / NLO) - 1) & 1);   // chunk c - 2's MMAs
+            if (pfon && ct == 0 && (c == 0 || c == nch - 1)) pst[c == 0 ? 2 : 3] = gtimer();
+            const uint8_t* raw = raw_at(c);
+            uint8_t* lo = lo_at(q);
+            for (int i = ct; i < STAGE_BYTES / 16; i += NCONV) {
+                const float4 v = *reinterpret_cast<const float4*>(raw + i * 16);
+                const float4 h = make_float4(__uint_as_float(__float_as_uint(v.x) & 0xFFFFE000u), __uint_as_float(__float_as_uint(v.y) & 0xFFFFE000u),
+                                             __uint_as_float(__float_as_uint(v.z) & 0xFFFFE000u), __uint_as_float(__float_as_uint(v.w) & 0xFFFFE000u));
+                *reinterpret_cast<float4*>(lo + i * 16) = make_float4(v.x - h.x, v.y - h.y, v.z - h.z, v.w - h.w);
+            }
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic smem writes -> tensor core
+            tma::arrive(smem_u32(&lo_full[q]));
+        }
+        if (warp >= 4) {
+            // epilogue: warp w reads TMEM lanes 32 (w - 4) .. +31 = leaves, all 48 columns (i, o, u of 16 units)
+            const int eli = 32 * (warp - 4) + lane;
+            const uint32_t erec = l0 + eli < n_leaf ? __ldg(leaves + 2 * (l0 + eli)) : 0u;
+            mbar_wait_parity(smem_u32(&done), 0);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            if (pfon && warp == 4 && lane == 0) pst[4] = gtimer();
+            const uint32_t ta = tmem + ((uint32_t)(32 * (warp - 4)) << 16);
+            uint32_t gi[16], go[16], gu[16];
+            tcl_ld16(ta, gi);
+            tcl_ld16(ta + LU, go);
+            tcl_ld16(ta + 2 * LU, gu);
+            asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+            if (l0 + eli < n_leaf) {
+                float* r = pool + erec;
+#pragma unroll
+                for (int t = 0; t < LU; t += 4) {
+                    float hv[4], cv[4], iv[4], ov[4], uv[4];
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        const int u = t + q;
+                        const float ig = fsigm(__uint_as_float(gi[u]) + bias_s[u]);
+                        const float og = fsigm(__uint_as_float(go[u]) + bias_s[LU + u]);
+                        const float ug = ftanh(__uint_as_float(gu[u]) + bias_s[2 * LU + u]);
+                        const float cc = ig * ug;
+                        hv[q] = og * ftanh(cc); cv[q] = cc; iv[q] = ig; ov[q] = og; uv[q] = ug;
+                    }
+                    *reinterpret_cast<float4*>(r + j0 + t) = make_float4(hv[0], hv[1], hv[2], hv[3]);
+                    *reinterpret_cast<float4*>(r + H + j0 + t) = make_float4(cv[0], cv[1], cv[2], cv[3]);
+                    *reinterpret_cast<float4*>(r + 2 * H + j0 + t) = make_float4(iv[0], iv[1], iv[2], iv[3]);
+                    *reinterpret_cast<float4*>(r + 3 * H + j0 + t) = make_float4(ov[0], ov[1], ov[2], ov[3]);
+                    *reinterpret_cast<float4*>(r + 4 * H + j0 + t) = make_float4(uv[0], uv[1], uv[2], uv[3]);
+                }
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(64));
+    if (pf) pst[5] = gtimer();
+}
+
 }  // namespace leaf
 }  // namespace dev
 
@@ -423,9 +651,29 @@ extern "C" int vpps_leaf_prof(int on, uint64_t* out) {   // measurement tool hoo
     return (int)cudaMemcpyToSymbol(dev::leaf::g_leaf_prof_on, &on, sizeof(int));
 }
 
+// 2D FP32 tensor map [rows][cols] (row stride cols * 4 bytes), box KCT columns x box_rows rows, SWIZZLE_128B;
+// cuTensorMapEncodeTiled comes from the driver through the runtime's entry-point query (no libcuda link)
+static bool encode_map(CUtensorMap* map, const float* base, int64_t rows, int64_t cols, int box_rows) {
+    static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            enc = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+    });
+    if (!enc) return false;
+    const cuuint64_t gd[2] = {(cuuint64_t)cols, (cuuint64_t)rows}, gs[1] = {(cuuint64_t)cols * 4};
+    const cuuint32_t bx[2] = {(cuuint32_t)dev::leaf::tma::KCT, (cuuint32_t)box_rows}, es[2] = {1, 1};
+    return enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), gd, gs, bx, es,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float* pool, const uint32_t* leaves,
                      int32_t n_leaf, int32_t H, int32_t E, float* const* zero_ptr, const int64_t* zero_n,
-                     uint32_t* epoch, cudaStream_t s, const void* prefetch, int64_t prefetch_bytes) {
+                     uint32_t* epoch, cudaStream_t s, const void* prefetch, int64_t prefetch_bytes, int64_t n_rows) {
     using namespace dev::leaf;
     if ((E != 128 && E != KMAX) || H % LU) return;   // (api.cu admits only built (H, E) variants)
     PassClear pc{};
@@ -441,6 +689,18 @@ void launch_leaf_fwd(const float* W, const float* b, const float* inputs, float*
     pc.epoch = epoch;
     pc.pf = static_cast<const char*>(prefetch);
     pc.pf_bytes = prefetch ? prefetch_bytes : 0;
+    // VPPS_LEAF_TMA=1: the TMA-fed tensor-core tiles (parity-green, slower: see vpps_leaf_fwd_tma)
+    static const bool tma_env = getenv("VPPS_LEAF_TMA") && atoi(getenv("VPPS_LEAF_TMA")) != 0;
+    if (tma_env && n_rows > 0 && (E == 128 || E == 256) && H % LU == 0) {
+        CUtensorMap mx, mw;
+        if (encode_map(&mx, inputs, n_rows, E, 1) && encode_map(&mw, W, 3 * (int64_t)H, E, LU)) {
+            // GEMM tiles first, then clearing CTAs: the SMs left over (at least 32 CTAs)
+            const int tiles = ((n_leaf + tma::ML - 1) / tma::ML) * (H / LU);
+            const int grid = tiles + std::max(148 - tiles, 32);
+            vpps_leaf_fwd_tma<<<grid, 256, tma::SMEM, s>>>(mx, mw, b, pool, leaves, n_leaf, H, E, tiles, pc);
+            return;
+        }
+    }
     if (simt) {
         const int tiles = std::max(((n_leaf + LM - 1) / LM) * (H / LU), 148);
         if (E == 128) {
@@ -466,6 +726,7 @@ cudaError_t setup_leaf_attrs() {
     if (e == cudaSuccess) e = cudaFuncSetAttribute(vpps_leaf_fwd<128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_of<128>());
     if (e == cudaSuccess) e = cudaFuncSetAttribute(vpps_leaf_fwd<128, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_of<128>());
     if (e == cudaSuccess) e = cudaFuncSetAttribute(vpps_leaf_fwd_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TC_SMEM);
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(vpps_leaf_fwd_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tma::SMEM);
     return e;
 }
 

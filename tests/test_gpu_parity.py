@@ -447,7 +447,7 @@ def test_errors_are_loud():
         m.fwd_bwd(s, torch.zeros(8, 32, device="cuda"))
 
 
-@pytest.mark.parametrize("env", ["VPPS_LEAF_TC", "VPPS_DW_TC", "VPPS_DW_TC2"])
+@pytest.mark.parametrize("env", ["VPPS_LEAF_TC", "VPPS_LEAF_TMA", "VPPS_DW_TC", "VPPS_DW_TC2"])
 def test_tensor_core_variants_subprocess(env):
     """The dataflow path's opt-in kernels against the oracle: the tensor-core leaf GEMM, the tcgen05 variant
     of the per-group gradient-GEMM items (VPPS_DW_TC) and the gathered 128 x 128 tensor-core gradient GEMM

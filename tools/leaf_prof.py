@@ -21,7 +21,7 @@ def main():
     rng = np.random.default_rng(0)
     shapes = vpps.param_shapes("binary", H, E, C)
     P = synth.init_params(shapes, rng)
-    m = vpps.Model("binary", H, E, C, groups=4, cluster=16, dataflow=True)
+    m = vpps.Model("binary", H, E, C, cluster=16, dataflow=True)
     params = torch.zeros(m.n_floats, device="cuda")
     grads = torch.zeros_like(params)
     for n, _ in shapes:
@@ -48,7 +48,7 @@ def main():
         work = b[:, 2] > 0
         rel = (b - t0) / 1e3
         print(f"step {step}: CTAs {len(b)}, working {work.sum()}")
-        names = ["entry", "issued", "K0 landed", "K3 landed", "FMA done", "exit", "clear done"]
+        names = ["entry", "issued / setup", "K0 landed", "K last landed", "FMA done", "exit", "clear done"]
         for k, nm in enumerate(names):
             sel = rel[work, k] if 2 <= k <= 5 else rel[:, k]
             print(f"  {nm:15s} min {sel.min():6.2f} mean {sel.mean():6.2f} max {sel.max():6.2f} us")
