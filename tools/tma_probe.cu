@@ -193,6 +193,115 @@ static void rate(int reps) {
     cudaFree(o);
 }
 
+// MN-major operand check: D[128 x 128] = Aᵀᵀ B with A stored transposed (At [K][M], M contiguous) loaded as
+// SWIZZLE_128B MN-major atoms (32 M x 8 K, 1 KB) by 2D TMA boxes {32 M, 32 K}, and B [N][K] K-major
+// (boxes {32 K, 128 N}).  UMMA: A MN-major (idesc bit 15), LBO = 4 KB between M atoms, SBO = 1 KB between
+// K atoms, +1 KB per k-step of 8; B K-major as above.  Plain TF32 (relative error ~1e-4 expected).
+__global__ void __launch_bounds__(128, 1) mn_probe(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                                                   int K, uint32_t lbo, uint32_t sbo, float* D) {
+    extern __shared__ __align__(1024) uint8_t dsm[];
+    uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(dsm) + 1023) & ~uintptr_t(1023));
+    uint8_t* As = sm;              // 4 boxes x 4 KB
+    uint8_t* Bs = sm + 16384;      // 16 KB
+    __shared__ __align__(8) uint64_t full, mdone;
+    __shared__ uint32_t tmem_base;
+    const int tid = threadIdx.x, warp = tid >> 5;
+    if (warp == 0) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base)), "r"(128));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    if (tid == 32) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&full)));
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&mdone)));
+        asm volatile("fence.mbarrier_init.release.cluster;");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem = tmem_base;
+    constexpr uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | (1u << 15) | ((uint32_t)(128 >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+    for (int c = 0; c < K / 32; ++c) {
+        if (tid == 0) {
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&full)), "r"(32768) : "memory");
+            for (int i = 0; i < 4; ++i)
+                asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+                             ::"r"(smem_u32(As + 4096 * i)), "l"(reinterpret_cast<uint64_t>(&tmA)), "r"(32 * i), "r"(32 * c),
+                               "r"(smem_u32(&full)) : "memory");
+            asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+                         ::"r"(smem_u32(Bs)), "l"(reinterpret_cast<uint64_t>(&tmB)), "r"(32 * c), "r"(0), "r"(smem_u32(&full)) : "memory");
+        }
+        mbar_wait(smem_u32(&full), c & 1);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        if (tid == 0) {
+            for (int s = 0; s < 4; ++s) {
+                const uint32_t a = smem_u32(As) + sbo * s;
+                const uint64_t ad = (uint64_t)((a >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
+                                    ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
+                asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                             "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}\n"
+                             ::"r"(tmem), "l"(ad), "l"(desc_sw128(smem_u32(Bs) + 32 * s)), "r"(idesc), "r"((c > 0 || s > 0) ? 1 : 0));
+            }
+            asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(&mdone)) : "memory");
+        }
+        mbar_wait(smem_u32(&mdone), c & 1);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        __syncthreads();
+    }
+    const int lane = tid & 31, row = 32 * warp + lane;
+    for (int q = 0; q < 8; ++q) {
+        uint32_t r[16];
+        const uint32_t ta = tmem + ((uint32_t)(32 * warp) << 16) + 16 * q;
+        asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+                     : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+                       "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+                     : "r"(ta));
+        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+        for (int k = 0; k < 16; ++k) D[row * 128 + 16 * q + k] = __uint_as_float(r[k]);
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(128));
+}
+
+static void mn_check(PFN_cuTensorMapEncodeTiled_v12000 enc) {
+    const int M = 128, N = 128, K = 96;
+    std::mt19937 rng(11);
+    std::uniform_real_distribution<float> U(-1.f, 1.f);
+    std::vector<float> At(K * M), B(N * K), D(M * N);
+    for (auto& v : At) v = U(rng);
+    for (auto& v : B) v = U(rng);
+    float *dA, *dB, *dD;
+    cudaMalloc(&dA, At.size() * 4); cudaMalloc(&dB, B.size() * 4); cudaMalloc(&dD, D.size() * 4);
+    cudaMemcpy(dA, At.data(), At.size() * 4, cudaMemcpyHostToDevice);
+    cudaMemcpy(dB, B.data(), B.size() * 4, cudaMemcpyHostToDevice);
+    CUtensorMap ta, tb;
+    cuuint64_t gda[2] = {(cuuint64_t)M, (cuuint64_t)K}, gsa[1] = {(cuuint64_t)M * 4};
+    cuuint32_t ba[2] = {32, 32}, es[2] = {1, 1};
+    enc(&ta, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, dA, gda, gsa, ba, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    cuuint64_t gdb[2] = {(cuuint64_t)K, (cuuint64_t)N}, gsb[1] = {(cuuint64_t)K * 4};
+    cuuint32_t bb[2] = {32, 128};
+    enc(&tb, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, dB, gdb, gsb, bb, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    const size_t smem = 32768 + 1024;
+    cudaFuncSetAttribute(mn_probe, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const uint32_t cand[][2] = {{4096, 1024}, {1024, 4096}, {16, 1024}, {4096, 16}};
+    for (auto& cd : cand) {
+        cudaMemset(dD, 0, D.size() * 4);
+        mn_probe<<<1, 128, smem>>>(ta, tb, K, cd[0], cd[1], dD);
+        cudaError_t e = cudaDeviceSynchronize();
+        cudaMemcpy(D.data(), dD, D.size() * 4, cudaMemcpyDeviceToHost);
+        double mx = 0;
+        for (int m = 0; m < M; ++m)
+            for (int n = 0; n < N; ++n) {
+                double sref = 0, sa = 0;
+                for (int k = 0; k < K; ++k) { sref += (double)At[k * M + m] * B[n * K + k]; sa += fabs((double)At[k * M + m] * B[n * K + k]); }
+                mx = std::max(mx, fabs(D[m * N + n] - sref) / sa);
+            }
+        printf("MN-major A (LBO %u, SBO %u): %s, max |err| / sum|terms| = %.3g\n", cd[0], cd[1], cudaGetErrorString(e), mx);
+    }
+}
+
 static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
     void* fn = nullptr;
     cudaDriverEntryPointQueryResult q;
@@ -256,5 +365,6 @@ int main() {
         cudaFree(tokd);
     }
     for (int reps : {12, 96, 384}) { rate<48>(reps); rate<128>(reps); rate<256>(reps); }
+    mn_check(enc);
     return 0;
 }
