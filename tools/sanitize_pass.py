@@ -1,5 +1,5 @@
 """One small training pass per device path, for compute-sanitizer (memcheck / racecheck / synccheck):
-    compute-sanitizer --tool memcheck python tools/sanitize_pass.py [dataflow|level|grid]
+    compute-sanitizer --tool memcheck python tools/sanitize_pass.py [dataflow|dataflow128|levelgemm|chain|level|grid]
 Exits non-zero if a pass disagrees with the oracle (so a sanitizer-induced change in behaviour shows)."""
 import os
 import sys
@@ -19,6 +19,15 @@ def main(which):
     if which == "dataflow":
         cell, H, C, V, kw = "binary", 256, 5, 64, dict(cluster=16, dataflow=True)
         graphs = synth.tree_batch(np.random.default_rng(1), 3, (2, 12), V, C)
+    elif which == "dataflow128":                 # H = 128: groups of 8 CTAs
+        cell, H, C, V, kw = "binary", 128, 5, 64, dict(cluster=8, dataflow=True)
+        graphs = synth.tree_batch(np.random.default_rng(1), 3, (2, 12), V, C)
+    elif which == "levelgemm":                   # level path with the library's own GEMM tiles
+        cell, H, C, V, kw = "binary", 64, 5, 64, dict(level=1)
+        graphs = synth.tree_batch(np.random.default_rng(1), 3, (2, 12), V, C)
+    elif which == "chain":                       # LSTM LM on the chain recurrence
+        cell, H, C, V, kw = "lstm", 128, 40, 40, dict(level=1)
+        graphs = synth.config_batch("c3", 0, batch=3, V=40, C=40)
     elif which == "grid":
         cell, H, C, V, kw = "binary", 32, 5, 64, {}
         graphs = synth.tree_batch(np.random.default_rng(1), 3, (2, 12), V, C)
