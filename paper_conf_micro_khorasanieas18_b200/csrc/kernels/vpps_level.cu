@@ -88,6 +88,10 @@ __global__ void int_cell(const float* __restrict__ Z, const float* __restrict__ 
 
 // loss heads (L42), one CTA per head: z = W_out h + b_out, softmax-NLL into the record and the summed loss
 // (L205); dz = p - onehot(y): dW_out += dz hᵀ, db_out += dz (atomics), the cell's dh += W_outᵀ dz
+// shared logits of one head: C floats, padded to whole float4 plus one more (the unrolled dh loop reads the
+// logits in vector pieces; compute-sanitizer memcheck flagged the 12-byte read past an unpadded C = 5 block)
+inline size_t heads_smem(int C) { return (size_t)(((C + 3) & ~3) + 4) * sizeof(float); }
+
 __global__ void heads(const float* __restrict__ Wo, const float* __restrict__ bo, const uint32_t* __restrict__ hl,
                       int H, int C, float* pool, int64_t loss_word, float* dWo, float* dbo) {
     extern __shared__ float zsh[];      // [C]
@@ -659,7 +663,7 @@ int level_pass(void* ctx_, const float* params, const int64_t* off, float* grads
     }
     // ---- loss heads: forward and backward (they feed nothing forward) ----
     if (n_head > 0)
-        heads<<<(unsigned)n_head, 256, C * sizeof(float), s>>>(W_out, b_out, hl, H, C, pool, loss_word, grads + off[4],
+        heads<<<(unsigned)n_head, 256, heads_smem(C), s>>>(W_out, b_out, hl, H, C, pool, loss_word, grads + off[4],
                                                              grads + off[7]);
     // ---- backward: internal levels L .. 1, then the leaves ----
     for (int32_t l = L; l >= 1; --l) {
@@ -1027,7 +1031,7 @@ int rvnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads,
         rv_cell<<<nblk(n * H), 256, 0, s>>>(Z, b_int, ints + 6 * r0, 6, (int)n, H, pool);
     }
     if (n_head > 0)
-        heads<<<(unsigned)n_head, 256, C * sizeof(float), s>>>(W_out, b_out, hl, H, C, pool, loss_word, grads + off[2],
+        heads<<<(unsigned)n_head, 256, heads_smem(C), s>>>(W_out, b_out, hl, H, C, pool, loss_word, grads + off[2],
                                                              grads + off[5]);
     for (int32_t l = L; l >= 1; --l) {
         const int64_t r0 = lv_start[l], n = lv_start[l + 1] - r0;
@@ -1088,7 +1092,7 @@ int tdrnn_pass(void* ctx_, const float* params, const int64_t* off, float* grads
         rv_cell<<<nblk(n * H), 256, 0, s>>>(Z, b, ints + 6 * r0, 6, (int)n, H, pool);
     }
     if (n_head > 0)
-        heads<<<(unsigned)n_head, 256, C * sizeof(float), s>>>(W_out, b_out, hl, H, C, pool, loss_word, grads + off[1],
+        heads<<<(unsigned)n_head, 256, heads_smem(C), s>>>(W_out, b_out, hl, H, C, pool, loss_word, grads + off[1],
                                                              grads + off[3]);
     for (int32_t l = L; l >= 1; --l) {
         const int64_t r0 = lv_start[l], n = lv_start[l + 1] - r0;
