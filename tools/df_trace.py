@@ -23,6 +23,7 @@ def main():
     ap.add_argument("--config", default="tgt")
     ap.add_argument("--batches", action="store_true", help="per-batch timeline of the last CTA's group")
     ap.add_argument("--sgd", action="store_true", help="fused SGD step (the bench mode)")
+    ap.add_argument("--flush", action="store_true", help="256 MiB L2 flush before the traced pass (the bench mode)")
     args = ap.parse_args()
     import torch
     import synth
@@ -51,6 +52,9 @@ def main():
         if r == args.reps - 1:
             torch.cuda.synchronize()
             buf.zero_()
+            if args.flush:
+                torch.empty(64 * 1024 * 1024, dtype=torch.float32, device="cuda").zero_()
+                torch.cuda.synchronize()
         if args.sgd:
             m.fwd_bwd_sgd(s, X, dX, lr=1e-3)
         else:
