@@ -62,9 +62,11 @@ __device__ __forceinline__ u64 ld_slot(const u64* p) {
 __device__ __forceinline__ void ld_slot2(const u64* p, u64& a, u64& b) {
     asm volatile("ld.relaxed.gpu.global.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
 }
+// four tagged slots in one 32-byte store (STG.E.ENL2.256.STRONG.GPU; each 8-byte element stays single-copy
+// atomic, so every slot's value and tag still arrive together); p is 32-byte aligned
 __device__ __forceinline__ void st_tag4(u64* p, const float* v, uint32_t e) {
-    asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(tagv(v[0], e)), "l"(tagv(v[1], e)) : "memory");
-    asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p + 2), "l"(tagv(v[2], e)), "l"(tagv(v[3], e)) : "memory");
+    asm volatile("st.relaxed.gpu.global.v4.b64 [%0], {%1, %2, %3, %4};"
+                 ::"l"(p), "l"(tagv(v[0], e)), "l"(tagv(v[1], e)), "l"(tagv(v[2], e)), "l"(tagv(v[3], e)) : "memory");
 }
 
 template <int H, int E>

@@ -196,6 +196,19 @@ def test_fused_sgd_target_groups(groups, cluster, dataflow):
     check_update(m, P, M.sgd(P, Go, lr, wd), params)
 
 
+@pytest.mark.parametrize("E", [128, 256])
+def test_fused_sgd_dataflow_hidden_128(E):
+    """vpps_fwd_bwd_sgd on 8-CTA dataflow groups (H = 128): the updated parameters against the FP64 oracle's
+    SGD step at 1e-4 of the step (+ two FP32 roundings)."""
+    graphs = synth.config_batch("tgt", 6)
+    lr, wd = 0.05, 1e-3
+    m, P, X, loss, params, grads, dX = run_case("binary", 128, E, 5, graphs, 4096, seed=8, sgd=(lr, wd),
+                                                cluster=8, dataflow=True)
+    lo, Go, _ = M.forward_backward("binary", P, X, graphs, 128)
+    assert abs(loss - lo) <= TOL * abs(lo)
+    check_update(m, P, M.sgd(P, Go, lr, wd), params)
+
+
 @pytest.mark.parametrize("cell,H,level", [("binary", 256, 0), ("binary", 256, 1), ("bilstm", 64, 0),
                                           ("gru", 64, 0), ("rvnn", 64, 0)])
 def test_fwd_bwd_then_sgd_step(cell, H, level):
