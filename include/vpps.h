@@ -113,7 +113,9 @@ typedef void (*vpps_free_fn)(void* ptr, void* stream, void* ctx);
 typedef struct {
     int32_t n_sm;        /* SMs to spread the weights over; 0 = all SMs of `device`            */
     int32_t ctas_per_sm; /* 1 (0 = auto = 1)                                                   */
-    int32_t groups;      /* replica groups G (SPEC P1); 0 = 1.  G > 1 is plan-only in v1       */
+    int32_t groups;      /* replica groups G (SPEC P1); 0 = 1; < 0 = automatic: the grid kernel of
+                            the tree cells takes the most replicas (4, 2, 1) with a built
+                            specialisation, every other path G = 1 (vpps_define_model)            */
     int32_t device;      /* CUDA device ordinal; ignored when plan_only                         */
     int32_t plan_only;   /* 1: no CUDA calls (partition + script generation only, CPU tests)   */
     int32_t cluster;     /* > 1: each replica group is one thread-block cluster of this many CTAs

@@ -128,6 +128,24 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
     *out = nullptr;
     vpps_options o{};
     if (opt) o = *opt;
+    if (o.groups < 0) {
+        // automatic replica groups (SPEC P1 from the register budget): on the grid kernel of the tree cells
+        // (child-sum, binary without clusters / forced level path) the most replicas that fit a built
+        // specialisation — G = 4, 2, 1 — since more replicas of the weights process more graphs at once
+        // (config 2: 1.15 / 0.67 / 0.43 ms for G = 1 / 2 / 4; TGT on the grid kernel 0.51 / 0.36 / 0.31 ms,
+        // profiles/r2_grid_groups_sweep.jsonl); every other path keeps G = 1
+        vpps_options o2 = o;
+        const bool grid_tree = (ops->cell == CELL_CHILDSUM || ops->cell == CELL_BINARY) && o.cluster <= 1 &&
+                               !o.dataflow && o.level <= 0;
+        if (grid_tree) {
+            for (int32_t g : {4, 2}) {
+                o2.groups = g;
+                if (vpps_define_model(params, n_params, ops, &o2, out) == VPPS_OK) return VPPS_OK;
+            }
+        }
+        o2.groups = 1;
+        return vpps_define_model(params, n_params, ops, &o2, out);
+    }
     const int32_t cell = ops->cell, H = ops->H, E = ops->E, C = ops->C, Mw = ops->mlp;
     if (cell < 0 || cell > 8 || H <= 0 || E <= 0 || C <= 0) return fail(VPPS_E_INVALID, "bad op set");
     if (cell == CELL_TDRNN && E != H) return fail(VPPS_E_INVALID, "TD-RNN: the leaves are the input rows (E == H)");

@@ -276,9 +276,9 @@ def candidate_options(cell: str, H: int, C: int):
             out += [dict(cluster=16, dataflow=True), dict(cluster=16)]
         elif H == 128:
             out += [dict(cluster=8, dataflow=True)]          # groups of H / 16 CTAs
-        out += [dict(groups=g, level=-1) for g in (1, 2, 4)] + [dict(level=1)]
+        out += [dict(groups=g, level=-1) for g in (4, 2, 1)] + [dict(level=1)]
     elif cell == "childsum":
-        out += [dict(groups=g) for g in (1, 2, 4)]
+        out += [dict(groups=g) for g in (4, 2, 1)]
     elif cell == "lstm":
         if C <= 32:
             out += [dict(groups=g, level=-1) for g in (1, 2)]

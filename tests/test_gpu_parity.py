@@ -134,6 +134,13 @@ def test_dataflow_groups_hidden_128(E, b):
     check("binary", 128, E, 5, [[((), 3, 2)]], 8, cluster=8, dataflow=True)               # one leaf
 
 
+@pytest.mark.parametrize("cell,H", [("childsum", 128), ("binary", 64)])
+def test_auto_replica_groups_grid(cell, H):
+    """groups = -1 (automatic): the grid kernel with 4 replica groups, parity against the FP64 oracle."""
+    graphs = synth.config_batch("c2", 2) if cell == "childsum" else _trees(9, 12, (2, 20), 4096, 5)
+    check(cell, H, H, 5, graphs, 4096, seed=12, groups=-1)
+
+
 def test_dataflow_degenerate_and_repeated_passes():
     check("binary", 256, 256, 5, [[((), 3, 2)]], 8, cluster=16, dataflow=True)           # one leaf
     check("binary", 256, 256, 5, _trees(12, 3, (1, 9), 30, 5), 30, cluster=16, dataflow=True, want_dx=False)

@@ -286,6 +286,16 @@ def test_autotune_picks_the_fastest_candidate(vpps):
     assert vpps.candidate_options("gru", 256, 1000) == [dict(chain=0), dict(chain=-1)]
 
 
+def test_auto_replica_groups(vpps):
+    """groups < 0: the grid kernel of the tree cells takes 4 replica groups (SPEC P1: 148 CTAs -> 37 per
+    group), every other path one group (the LSTM LM at V = 1000 runs on the chain recurrence)."""
+    assert vpps.Model("childsum", 128, 128, 5, groups=-1, plan_only=True).plan_info()["n_g"] == 37
+    assert vpps.Model("binary", 256, 256, 5, groups=-1, plan_only=True).plan_info()["n_g"] == 37
+    assert vpps.Model("lstm", 256, 256, 1000, groups=-1, plan_only=True).plan_info()["n_g"] == 148
+    assert vpps.Model("binary", 256, 256, 5, groups=-1, cluster=16, dataflow=True,
+                      plan_only=True).plan_info()["n_g"] == 16
+
+
 def test_bilstmchar_script_host_side(vpps):
     """BiLSTMwChar scripts (plan-only): the host FLOP count equals the oracle's; spellings are accepted only by
     this cell; character ids and tokens are range-checked (a rare word's token is never read)."""

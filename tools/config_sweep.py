@@ -50,6 +50,16 @@ CASES = [
     ("tgt binary H128 E128 B16 (dataflow, 8-CTA groups)", "tgt", "binary", 128, 128, 5, 4096, 16, {"cluster": 8, "dataflow": True}, {}),
     ("tgt binary H128 E128 B16 (level path)", "tgt", "binary", 128, 128, 5, 4096, 16, {"level": 1}, {}),
     ("tgt binary H128 E128 B16 (grid)", "tgt", "binary", 128, 128, 5, 4096, 16, {"level": -1}, {}),
+    ("c2 child-sum H128 B16 (auto groups)", "c2", "childsum", 128, 128, 5, 4096, 16, {"groups": -1}, {}),
+    ("tgt binary H256 B16 (grid, auto groups)", "tgt", "binary", 256, 256, 5, 4096, 16, {"groups": -1, "level": -1}, {}),
+    ("grid-G c1 LSTM H32 B4 G2", "c1", "lstm", 32, 32, 16, 16, 4, {"groups": 2, "level": -1}, {}),
+    ("grid-G c1 LSTM H32 B4 G4", "c1", "lstm", 32, 32, 16, 16, 4, {"groups": 4, "level": -1}, {}),
+    ("grid-G c2 child-sum H128 B16 G2", "c2", "childsum", 128, 128, 5, 4096, 16, {"groups": 2}, {}),
+    ("grid-G tgt binary H256 B16 G1", "tgt", "binary", 256, 256, 5, 4096, 16, {"groups": 1, "level": -1}, {}),
+    ("grid-G tgt binary H256 B16 G2", "tgt", "binary", 256, 256, 5, 4096, 16, {"groups": 2, "level": -1}, {}),
+    ("grid-G tgt binary H256 B16 G4", "tgt", "binary", 256, 256, 5, 4096, 16, {"groups": 4, "level": -1}, {}),
+    ("grid-G tgt binary H128 B16 G4", "tgt", "binary", 128, 128, 5, 4096, 16, {"groups": 4, "level": -1}, {}),
+    ("grid-G c3 LSTM-LM H256 B16 (V=C=32) G4", "c3", "lstm", 256, 256, 32, 32, 16, {"groups": 4, "level": -1}, {"V": 32, "C": 32}),
     ("tgt binary H256 B1 (dataflow)", "tgt", "binary", 256, 256, 5, 4096, 1, {"cluster": 16, "dataflow": True}, {}),
     ("tgt binary H256 B4 (dataflow)", "tgt", "binary", 256, 256, 5, 4096, 4, {"cluster": 16, "dataflow": True}, {}),
     ("tgt binary H256 B16 (dataflow)", "tgt", "binary", 256, 256, 5, 4096, 16, {"cluster": 16, "dataflow": True}, {}),
