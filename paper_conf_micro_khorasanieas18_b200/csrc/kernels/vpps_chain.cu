@@ -53,9 +53,10 @@ __device__ __forceinline__ u64 tagv(float v, uint32_t e) { return ((u64)e << 32)
 __device__ __forceinline__ void st_tag(u64* p, float v, uint32_t e) {
     asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(tagv(v, e)) : "memory");
 }
+// four tagged slots in one 32-byte store (each 8-byte element single-copy atomic); p is 32-byte aligned
 __device__ __forceinline__ void st_tag4(u64* p, const float* v, uint32_t e) {
-    asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(tagv(v[0], e)), "l"(tagv(v[1], e)) : "memory");
-    asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p + 2), "l"(tagv(v[2], e)), "l"(tagv(v[3], e)) : "memory");
+    asm volatile("st.relaxed.gpu.global.v4.b64 [%0], {%1, %2, %3, %4};"
+                 ::"l"(p), "l"(tagv(v[0], e)), "l"(tagv(v[1], e)), "l"(tagv(v[2], e)), "l"(tagv(v[3], e)) : "memory");
 }
 // polls of slots other CTAs write in this kernel: relaxed GPU-scope loads (single-copy atomic 8 / 16 bytes)
 __device__ __forceinline__ u64 ld_slot(const u64* p) {
