@@ -31,6 +31,9 @@ constexpr int MAXB = 1 + (NB * 9 > NBL * 4 ? NB * 9 : NBL * 4);   // words of th
 constexpr int NC = 2;          // nodes per transposed-product chunk (two chunk buffers; 4 measured slower)
 constexpr int ZC = 32;         // classes per head (C <= 32)
 constexpr int CINMAX = 10;
+#ifndef VPPS_DF_NP
+#define VPPS_DF_NP 2         // nodes per transposed-product step
+#endif
 constexpr uint32_t NONE = 0xFFFFFFFFu;
 // HEAD_FB: the loss head's forward and backward in one batch (L42: softmax-NLL; dz = p - onehot needs
 // nothing but the head's own forward), emitted at the labelled cell's forward level
@@ -62,6 +65,10 @@ __device__ __forceinline__ u64 ld_slot(const u64* p) {
 __device__ __forceinline__ void ld_slot2(const u64* p, u64& a, u64& b) {
     asm volatile("ld.relaxed.gpu.global.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
 }
+// two adjacent tagged slots in one 16-byte store (p 16-byte aligned)
+__device__ __forceinline__ void st_tag2(u64* p, float a, float b, uint32_t e) {
+    asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(tagv(a, e)), "l"(tagv(b, e)) : "memory");
+}
 // four tagged slots in one 32-byte store (STG.E.ENL2.256.STRONG.GPU; each 8-byte element stays single-copy
 // atomic, so every slot's value and tag still arrive together); p is 32-byte aligned
 __device__ __forceinline__ void st_tag4(u64* p, const float* v, uint32_t e) {
@@ -89,8 +96,17 @@ struct DCfg {
     // second staging buffers: consecutive batches alternate, so a batch needs no closing barrier
     static constexpr int O_X2 = O_ZS + NB * ZC;
     static constexpr int O_CIN2 = O_X2 + NB * KP;
-    static constexpr int O_HEAD = O_CIN2 + NB * UM * CINMAX;
+    // forward partial gate sums of the 8 warps (column slices), two buffers: [2][8 warps][4 nodes][UM][4 rows]
+    static constexpr int O_FP = O_CIN2 + NB * UM * CINMAX;
+    static constexpr int O_HEAD = O_FP + 2 * 8 * 4 * UM * 4;
     static_assert(DXB >= 2 * NB * KP && DXB >= 2 * NB * NCL * 2 * UM, "u64 staging fits in dxb");
+    // register layout (unit pairs x column slices): warp w owns columns [w CW, (w + 1) CW) of [h_l; h_r] for
+    // all UM units of the CTA; lane = 4 ug + cg holds units 2 ug, 2 ug + 1 (one float2 per (row, column):
+    // FFMA2 over the unit pair) and the CPL columns w CW + 16 t + 4 cg + q (granule t, q < 4)
+    static constexpr int CW = KP / 8;              // columns per warp
+    static constexpr int CPL = KP / 32;            // columns per lane
+    static constexpr int NG = CPL / 4;             // 4-column granules per lane
+    static_assert(CPL % 4 == 0 && UM == 16 && NTH == 256, "dataflow kernel: 8 warps x (8 unit pairs x 4 column groups)");
     static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 2 * C + 8); }
 };
 
@@ -100,7 +116,7 @@ template <int H, int E, bool PROF>
 __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     using T = DCfg<H, E>;
     using LB = typename T::LB;
-    constexpr int TU = T::TU, UM = T::UM, KP = T::KP, NCL = T::NCL;
+    constexpr int UM = T::UM, KP = T::KP, NCL = T::NCL;
     extern __shared__ __align__(16) uint32_t smw[];
     float* sm = reinterpret_cast<float*>(smw);
     uint32_t* chunk = smw;
@@ -108,7 +124,6 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     float* dxb = sm + T::O_DXB;
     u64* tbuf = reinterpret_cast<u64*>(sm + T::O_DXB);     // tagged staging (aliases dxb)
     float* cin = sm + T::O_CIN;
-    int cbuf = 0;                                          // transposed-product buffer, alternating across batches
     float* bias = sm + T::O_BIAS;
     float* zs = sm + T::O_ZS;
     const int C = P.C;
@@ -125,34 +140,37 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     u64* HX = reinterpret_cast<u64*>(pool + P.df_hx);
     u64* PART = reinterpret_cast<u64*>(pool + P.df_part);
     u64* HD = reinterpret_cast<u64*>(pool + P.df_hd);
-    const int u = tid / TU, tu = tid % TU, gl = lane & 15;      // unit slot, thread in unit, lane in group
-    const int j = lc * UM + u;                                  // hidden unit of this thread (blocked)
     const bool holds_head = (lc == 0);
 
     if (PROF && P.prof && threadIdx.x == 0) P.prof[(int64_t)blockIdx.x * P.prof_stride + 11] = gtimer();   // entry
     // ---- prologue: this CTA's rows of U_iou, U_fl, U_fr -> registers (L123, L129) ----
-    // register slot t of a lane in the upper half-warp holds granule t ^ 1 (lanes l and l ^ 16 hold the same
-    // columns of the warp's two units): the transposed product's pair exchange then keeps slot t and sends
-    // slot t + 1 in every lane, with no selects (granules t and t ^ 1 sit on the same side of h_l / h_r)
-    const int gsw = (lane & 16) ? 1 : 0;
-    static_assert(T::TH % 2 == 0, "swapped granule pairs stay on one side of [h_l; h_r]");
-    float wb[4][LB::NREG];
+    // lane (ug, cg) of warp w: units 2 ug, 2 ug + 1 of this CTA as float2 pairs, rows i, o, u of U_iou and the
+    // forget row of the warp's side (U_fl over h_l for w < 4, U_fr over h_r otherwise), columns
+    // w CW + 16 t + 4 cg + q
+    constexpr int CW = T::CW, CPL = T::CPL, NG = T::NG;
+    const int cg = lane & 3, ug = lane >> 2;
+    const int side = warp >= 4 ? 1 : 0;                         // the warp's columns read h_l (0) or h_r (1)
+    float2 wp[4][CPL];
 #pragma unroll
     for (int r = 0; r < 4; ++r)
 #pragma unroll
-        for (int t = 0; t < LB::NT; ++t) {
-            const int col = LB::CG * (tu + TU * (t ^ gsw));
-            const float* src = r < 3 ? P.params + off[1] + (int64_t)(r * H + j) * (2 * H) + col
-                                     : (col < H ? P.params + off[2] + (int64_t)j * H + col
-                                                : P.params + off[3] + (int64_t)j * H + col - H);
-            if constexpr (LB::CG == 4) {
-                const float4 v = __ldg(reinterpret_cast<const float4*>(src));
-                wb[r][t * 4] = v.x; wb[r][t * 4 + 1] = v.y; wb[r][t * 4 + 2] = v.z; wb[r][t * 4 + 3] = v.w;
-            } else {
+        for (int t = 0; t < NG; ++t) {
+            const int col = warp * CW + 16 * t + 4 * cg;
+            float4 v[2];
 #pragma unroll
-                for (int q = 0; q < LB::CG; ++q) wb[r][t * LB::CG + q] = __ldg(src + q);
+            for (int m = 0; m < 2; ++m) {
+                const int jm = lc * UM + 2 * ug + m;
+                const float* src = r < 3 ? P.params + off[1] + (int64_t)(r * H + jm) * (2 * H) + col
+                                         : P.params + off[2 + side] + (int64_t)jm * H + col - side * H;
+                v[m] = __ldg(reinterpret_cast<const float4*>(src));
             }
+            wp[r][4 * t] = make_float2(v[0].x, v[1].x);
+            wp[r][4 * t + 1] = make_float2(v[0].y, v[1].y);
+            wp[r][4 * t + 2] = make_float2(v[0].z, v[1].z);
+            wp[r][4 * t + 3] = make_float2(v[0].w, v[1].w);
         }
+    float* fpb = sm + T::O_FP;     // forward partials, two alternating buffers
+    int fbuf = 0;
     if (tid < UM * 4) {
         const int uu = tid / 4, k = tid % 4, jj = lc * UM + uu;
         bias[tid] = k < 3 ? __ldg(P.params + off[5] + k * H + jj) : __ldg(P.params + off[6] + jj);
@@ -521,80 +539,99 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                     dbo[c] += s;
                 }
         } else if (op == INT_F) {
-            // ---- forward of internal cells: matvec from registers (L123), 4 nodes at a time; the unit's
-            //      16 lanes reduce with a transposed butterfly; the lane holding node n's gates updates it ----
-            // groups of NN in {4, 2, 1} nodes: the unit's 16 lanes reduce NN partial sums with a transposed
-            // butterfly, after which lane 16/NN * m holds node m's gates
+            // ---- forward of internal cells: matvec from registers (L123), NN in {4, 2, 1} nodes at a time.
+            //      Each lane forms 8 NN partial gate sums (NN nodes x 4 rows x its unit pair) over its CPL
+            //      columns; the 4 column-group lanes reduce them with a transposed halving (each lane keeps a
+            //      quarter), the 8 warps' column slices meet in shared memory, and thread (node, unit) sums
+            //      them and updates the cell ----
             auto fwd_group = [&](auto nnc, int n0) {
                 constexpr int NN = decltype(nnc)::value;
+                constexpr int V = NN * 8;
                 XST(stF, 0);
-                float2 a[NN][5];
+                float2 a[NN][4];
 #pragma unroll
                 for (int n = 0; n < NN; ++n)
 #pragma unroll
-                    for (int o = 0; o < 5; ++o) a[n][o] = make_float2(0.f, 0.f);
+                    for (int r = 0; r < 4; ++r) a[n][r] = make_float2(0.f, 0.f);
 #pragma unroll
-                for (int t = 0; t < LB::NT; ++t) {
-                    const int col0 = LB::CG * (tu + TU * (t ^ gsw));
-                    constexpr int of0 = 3;                  // granules t < T::TH read h_l (U_fl), the rest h_r (U_fr)
+                for (int t = 0; t < NG; ++t)
 #pragma unroll
                     for (int n = 0; n < NN; ++n) {
-                        float xv[LB::CG];
-                        lds<LB::CG>(xs + (n0 + n) * KP + col0, xv);
+                        const float4 x4 = *reinterpret_cast<const float4*>(xs + (n0 + n) * KP + warp * CW + 16 * t + 4 * cg);
+                        const float xv[4] = {x4.x, x4.y, x4.z, x4.w};
 #pragma unroll
-                        for (int q = 0; q < LB::CG; q += 2) {
-                            const float2 x2 = make_float2(xv[q], xv[q + 1]);
-                            const int k = t * LB::CG + q;
+                        for (int q = 0; q < 4; ++q)
 #pragma unroll
-                            for (int r = 0; r < 3; ++r)
-                                a[n][r] = __ffma2_rn(make_float2(wb[r][k], wb[r][k + 1]), x2, a[n][r]);
-                            a[n][of0 + (t >= T::TH)] = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), x2, a[n][of0 + (t >= T::TH)]);
-                        }
+                            for (int r = 0; r < 4; ++r)
+                                a[n][r] = __ffma2_rn(wp[r][4 * t + q], make_float2(xv[q], xv[q]), a[n][r]);
                     }
-                }
                 XST(stF, 1);
-                float g5[5];
+                // value v = (n * 4 + r) * 2 + unit; halving over lane bit 0, then bit 1
+                float val[V];
 #pragma unroll
-                for (int o = 0; o < 5; ++o) {
-                    if constexpr (NN == 4) {
-                        g5[o] = treduce4_16(a[0][o].x + a[0][o].y, a[1][o].x + a[1][o].y, a[2][o].x + a[2][o].y,
-                                            a[3][o].x + a[3][o].y, gl);
-                    } else if constexpr (NN == 2) {
-                        const bool b3 = gl & 8;
-                        const float v0 = a[0][o].x + a[0][o].y, v1 = a[1][o].x + a[1][o].y;
-                        float k = b3 ? v1 : v0;
-                        k += __shfl_xor_sync(FULLMASK, b3 ? v0 : v1, 8);
-                        k += __shfl_xor_sync(FULLMASK, k, 4);
-                        k += __shfl_xor_sync(FULLMASK, k, 2);
-                        g5[o] = k + __shfl_xor_sync(FULLMASK, k, 1);
-                    } else {
-                        float k = a[0][o].x + a[0][o].y;
+                for (int n = 0; n < NN; ++n)
 #pragma unroll
-                        for (int d = 8; d >= 1; d >>= 1) k += __shfl_xor_sync(FULLMASK, k, d);
-                        g5[o] = k;
+                    for (int r = 0; r < 4; ++r) { val[(n * 4 + r) * 2] = a[n][r].x; val[(n * 4 + r) * 2 + 1] = a[n][r].y; }
+                const bool c0 = lane & 1, c1 = lane & 2;
+#pragma unroll
+                for (int i = 0; i < V / 2; ++i) {
+                    const float snd = c0 ? val[i] : val[i + V / 2];
+                    const float kp = c0 ? val[i + V / 2] : val[i];
+                    val[i] = kp + __shfl_xor_sync(FULLMASK, snd, 1);
+                }
+#pragma unroll
+                for (int i = 0; i < V / 4; ++i) {
+                    const float snd = c1 ? val[i] : val[i + V / 4];
+                    const float kp = c1 ? val[i + V / 4] : val[i];
+                    val[i] = kp + __shfl_xor_sync(FULLMASK, snd, 2);
+                }
+                // kept value i is v = i + (2 c0 + c1) V / 4: node v / 8, row (v / 2) % 4, unit v % 2
+                float* fb = fpb + fbuf * (8 * 4 * UM * 4) + warp * (4 * UM * 4);
+                const int vb = ((c0 ? 2 : 0) + (c1 ? 1 : 0)) * (V / 4);
+                if constexpr (NN == 4) {
+                    float* d = fb + (vb / 8) * (UM * 4) + 2 * ug * 4;
+                    *reinterpret_cast<float4*>(d) = make_float4(val[0], val[2], val[4], val[6]);
+                    *reinterpret_cast<float4*>(d + 4) = make_float4(val[1], val[3], val[5], val[7]);
+                } else {
+#pragma unroll
+                    for (int i = 0; i < V / 4; ++i) {
+                        const int v = vb + i;
+                        fb[(v / 8) * (UM * 4) + (2 * ug + (v & 1)) * 4 + ((v >> 1) & 3)] = val[i];
                     }
                 }
+                __syncthreads();
                 XST(stF, 2);
-                constexpr int SPAN = 16 / NN;
-                const int n = n0 + gl / SPAN;
-                if (gl % SPAN == 0 && n < nb) {
-                    const uint32_t* e = ent + n * sz;
-                    const uint32_t rec = e[0];
-                    const float* b = bias + u * 4;
-                    const float* cv = cin + (n * UM + u) * CINMAX;
-                    const float i = fsigm(g5[0] + b[0]), o = fsigm(g5[1] + b[1]), uv = ftanh(g5[2] + b[2]);
-                    const float fl = fsigm(g5[3] + b[3]), fr = fsigm(g5[4] + b[3]);
-                    const float c = i * uv + fl * cv[0] + fr * cv[1];
-                    const float h = o * ftanh(c);
-                    if (e[1] != NONE) st_tag(HX + (int64_t)e[1] * H + j, h, ep);   // read by the whole group
-                    pool[rec + j] = h;                                              // the rest: this CTA, GEMMs
-                    pool[rec + H + j] = c;
-                    pool[rec + 2 * H + j] = i;
-                    pool[rec + 3 * H + j] = o;
-                    pool[rec + 4 * H + j] = uv;
-                    pool[rec + 5 * H + j] = fl;
-                    pool[rec + 6 * H + j] = fr;
+                if (tid < NN * UM) {
+                    const int n = n0 + tid / UM, uu = tid % UM;
+                    if (n < nb) {
+                        const float* fs = fpb + fbuf * (8 * 4 * UM * 4) + ((tid / UM) * UM + uu) * 4;
+                        float gi = 0.f, go = 0.f, gu = 0.f, gfl = 0.f, gfr = 0.f;
+#pragma unroll
+                        for (int w = 0; w < 8; ++w) {
+                            const float4 p4 = *reinterpret_cast<const float4*>(fs + w * (4 * UM * 4));
+                            gi += p4.x; go += p4.y; gu += p4.z;
+                            if (w < 4) gfl += p4.w; else gfr += p4.w;
+                        }
+                        const uint32_t* e = ent + n * sz;
+                        const uint32_t rec = e[0];
+                        const int j = lc * UM + uu;
+                        const float* b = bias + uu * 4;
+                        const float* cv = cin + (n * UM + uu) * CINMAX;
+                        const float i = fsigm(gi + b[0]), o = fsigm(go + b[1]), uv = ftanh(gu + b[2]);
+                        const float fl = fsigm(gfl + b[3]), fr = fsigm(gfr + b[3]);
+                        const float c = i * uv + fl * cv[0] + fr * cv[1];
+                        const float h = o * ftanh(c);
+                        if (e[1] != NONE) st_tag(HX + (int64_t)e[1] * H + j, h, ep);   // read by the whole group
+                        pool[rec + j] = h;                                              // the rest: this CTA, GEMMs
+                        pool[rec + H + j] = c;
+                        pool[rec + 2 * H + j] = i;
+                        pool[rec + 3 * H + j] = o;
+                        pool[rec + 4 * H + j] = uv;
+                        pool[rec + 5 * H + j] = fl;
+                        pool[rec + 6 * H + j] = fr;
+                    }
                 }
+                fbuf ^= 1;
                 XST(stF, 3);
             };
             int n0 = 0;
@@ -609,75 +646,78 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             XST(stB, 6);
             XST(stBB, 29);
             // transposed products (L94, fn4): per node, this CTA's partial dx = Σ_r W[r] g_r over all 2H
-            // columns.  The two units of a warp are pre-summed with one shuffle exchange (lane l keeps the
-            // even or odd granules of the pair, l ^ 16 the others), the 8 warp slices are summed in shared
-            // memory and published as tagged PART slots.  Chunks of NC nodes alternate between two
-            // buffers, so one barrier per chunk separates a chunk's stores from its reduction and the
-            // reduction of chunk c overlaps the products of chunk c + 1.
+            // columns.  Lane (ug, cg) of warp w forms the sums of its unit pair over its CPL columns (FFMA2 over
+            // the pair, then the two halves added); the 8 unit-pair lanes of a column group reduce them with a
+            // transposed halving (lane bits 2, 3, 4), so each lane ends with CPL / 8 adjacent columns summed
+            // over all UM units of the CTA and publishes them as tagged PART slots: no shared memory and no
+            // barrier between the products and the publish.
             if (kindB) {
-                constexpr int NW = NTH / 32;
-                const bool hi = lane & 16;
-                for (int n0 = 0; n0 < nb; n0 += NC, cbuf ^= 1) {
-                    float* buf = dxb + cbuf * (NW * NC * KP);
+                const bool b2 = lane & 4, b3 = lane & 8, b4 = lane & 16;
+                // NP nodes at a time (independent product and shuffle chains interleave)
+                auto tmv = [&](auto npc, int n0) {
+                    constexpr int NP = decltype(npc)::value;
+                    float dv[NP][CPL];
 #pragma unroll
-                    for (int dn = 0; dn < NC; ++dn) {
-                        const int n = n0 + dn;
-                        if (n >= nb) break;
-                        float gr[5];
+                    for (int p = 0; p < NP; ++p) {
+                        const int n = n0 + p;
+                        float2 gp[4];
 #pragma unroll
-                        for (int r = 0; r < 5; ++r) gr[r] = cin[(n * 5 + r) * UM + u];
-                        float* drow = buf + (warp * NC + dn) * KP;
+                        for (int r = 0; r < 3; ++r) gp[r] = *reinterpret_cast<const float2*>(cin + (n * 5 + r) * UM + 2 * ug);
+                        gp[3] = *reinterpret_cast<const float2*>(cin + (n * 5 + 3 + side) * UM + 2 * ug);
 #pragma unroll
-                        for (int t = 0; t < LB::NT; t += 2) {
-                            // granules t, t + 1; lanes < 16 keep granule t, lanes >= 16 granule t + 1 (the
-                            // partner lane l ^ 16 holds the same columns of the warp's other unit)
-                            float dx[2][LB::CG];
-#pragma unroll
-                            for (int h = 0; h < 2; ++h) {
-                                const float gf = t + h < T::TH ? gr[3] : gr[4];
-#pragma unroll
-                                for (int q = 0; q < LB::CG; q += 2) {
-                                    const int k = (t + h) * LB::CG + q;
-                                    float2 d = __ffma2_rn(make_float2(wb[0][k], wb[0][k + 1]), make_float2(gr[0], gr[0]),
-                                                          make_float2(0.f, 0.f));
-                                    d = __ffma2_rn(make_float2(wb[1][k], wb[1][k + 1]), make_float2(gr[1], gr[1]), d);
-                                    d = __ffma2_rn(make_float2(wb[2][k], wb[2][k + 1]), make_float2(gr[2], gr[2]), d);
-                                    d = __ffma2_rn(make_float2(wb[3][k], wb[3][k + 1]), make_float2(gf, gf), d);
-                                    dx[h][q] = d.x;
-                                    dx[h][q + 1] = d.y;
-                                }
-                            }
-                            float kv[LB::CG];
-#pragma unroll
-                            for (int q = 0; q < LB::CG; ++q) {
-                                // slot t is granule t (t + 1 in the upper half-warp): keep it, send slot t + 1
-                                kv[q] = dx[0][q] + __shfl_xor_sync(FULLMASK, dx[1][q], 16);
-                            }
-                            const int col0 = LB::CG * (tu + TU * (t + (hi ? 1 : 0)));
-                            sts_granule<LB::CG>(drow + col0, kv, true);
+                        for (int k = 0; k < CPL; ++k) {
+                            float2 d = __ffma2_rn(wp[0][k], gp[0], make_float2(0.f, 0.f));
+                            d = __ffma2_rn(wp[1][k], gp[1], d);
+                            d = __ffma2_rn(wp[2][k], gp[2], d);
+                            d = __ffma2_rn(wp[3][k], gp[3], d);
+                            dv[p][k] = d.x + d.y;
                         }
                     }
-                    XST(stB, 7);
-                    __syncthreads();
-                    XST(stB, 8);
-                    constexpr int q4 = KP / 4;
-                    for (int i = tid; i < NC * q4; i += NTH) {
-                        const int dn = i / q4, c = (i - dn * q4) * 4, n = n0 + dn;
-                        if (n >= nb) continue;
-                        float s4[4] = {0.f, 0.f, 0.f, 0.f};
+                    // halving over lane bits 2, 3, 4: kept value i is column index
+                    // k = i + b2 CPL / 2 + b3 CPL / 4 + b4 CPL / 8 of the lane's CPL (k = 4 t + q)
 #pragma unroll
-                        for (int w = 0; w < NW; ++w) {
-                            const float4 x = *reinterpret_cast<const float4*>(buf + (w * NC + dn) * KP + c);
-                            s4[0] += x.x; s4[1] += x.y; s4[2] += x.z; s4[3] += x.w;
+                    for (int i = 0; i < CPL / 2; ++i)
+#pragma unroll
+                        for (int p = 0; p < NP; ++p) {
+                            const float snd = b2 ? dv[p][i] : dv[p][i + CPL / 2];
+                            const float kp = b2 ? dv[p][i + CPL / 2] : dv[p][i];
+                            dv[p][i] = kp + __shfl_xor_sync(FULLMASK, snd, 4);
                         }
-                        // column c: child side = c / H, unit jj = c % H, owner CTA m = jj / U, slot jj % U
-                        const int side = c >= H, jj = c - side * H, m = jj / UM;
-                        const uint32_t pp = ent[n * sz + 4];
-                        st_tag4(PART + ((((int64_t)pp * NCL + m) * NCL + lc) * 2 + side) * UM + (jj - m * UM), s4, ep);
+#pragma unroll
+                    for (int i = 0; i < CPL / 4; ++i)
+#pragma unroll
+                        for (int p = 0; p < NP; ++p) {
+                            const float snd = b3 ? dv[p][i] : dv[p][i + CPL / 4];
+                            const float kp = b3 ? dv[p][i + CPL / 4] : dv[p][i];
+                            dv[p][i] = kp + __shfl_xor_sync(FULLMASK, snd, 8);
+                        }
+#pragma unroll
+                    for (int i = 0; i < CPL / 8; ++i)
+#pragma unroll
+                        for (int p = 0; p < NP; ++p) {
+                            const float snd = b4 ? dv[p][i] : dv[p][i + CPL / 8];
+                            const float kp = b4 ? dv[p][i + CPL / 8] : dv[p][i];
+                            dv[p][i] = kp + __shfl_xor_sync(FULLMASK, snd, 16);
+                        }
+                    const int k0 = (b2 ? CPL / 2 : 0) + (b3 ? CPL / 4 : 0) + (b4 ? CPL / 8 : 0);
+                    // column c: child side = c / H, unit jj = c % H, owner CTA m = jj / U, slot jj % U
+                    const int c = warp * CW + 16 * (k0 / 4) + 4 * cg + (k0 % 4);
+                    const int jj = c - side * H, m = jj / UM;
+#pragma unroll
+                    for (int p = 0; p < NP; ++p) {
+                        const uint32_t pp = ent[(n0 + p) * sz + 4];
+                        u64* dst = PART + ((((int64_t)pp * NCL + m) * NCL + lc) * 2 + side) * UM + (jj - m * UM);
+                        if constexpr (CPL / 8 == 2) st_tag2(dst, dv[p][0], dv[p][1], ep);
+                        else st_tag(dst, dv[p][0], ep);
                     }
-                    XST(stB, 9);
-                    XST(stB, 10);
-                }
+                };
+                int n0 = 0;
+                for (; n0 + VPPS_DF_NP <= nb; n0 += VPPS_DF_NP) tmv(std::integral_constant<int, VPPS_DF_NP>{}, n0);
+                for (; n0 < nb; ++n0) tmv(std::integral_constant<int, 1>{}, n0);
+                XST(stB, 7);
+                XST(stB, 8);
+                XST(stB, 9);
+                XST(stB, 10);
                 XST(stBB, 30);
             }
         }
