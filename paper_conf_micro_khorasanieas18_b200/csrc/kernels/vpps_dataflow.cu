@@ -31,6 +31,9 @@ constexpr int MAXB = 1 + (NB * 9 > NBL * 4 ? NB * 9 : NBL * 4);   // words of th
 constexpr int NC = 2;          // nodes per transposed-product chunk (two chunk buffers; 4 measured slower)
 constexpr int ZC = 32;         // classes per head (C <= 32)
 constexpr int CINMAX = 10;
+#ifndef VPPS_DF_WARP_STAGE
+#define VPPS_DF_WARP_STAGE 1 // INT_F batches staged per warp (only the warp's own columns)
+#endif
 #ifndef VPPS_DF_NP
 #define VPPS_DF_NP 2         // nodes per transposed-product step
 #endif
@@ -308,7 +311,66 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
             pos = next;
             continue;
         }
-        if (op == INT_F || is_head) {
+        if (op == INT_F && VPPS_DF_WARP_STAGE) {
+            // per-warp staging: warp w computes only with the CW columns [w CW, (w + 1) CW) of [h_l; h_r], so
+            // it loads, checks and converts exactly those (child side = w / 4) for every node of the batch into
+            // its own slice of xs, with a warp-level retry loop — no CTA barrier before the products (the
+            // forward group's barrier orders the children's c below for the cell threads)
+            constexpr int CPW = CW / 32;                   // columns per lane (2 at H = 256, 1 at H = 128)
+            u64* tw = tbuf + warp * (NB * CW);             // this warp's tagged staging
+            const int cb = (warp & 3) * CW + CPW * lane;   // column in the child's h
+            uint32_t pend = 0;                             // bit n: node n's slots are tagged and not yet converted
+            for (int n = 0; n < nb; ++n) {
+                const uint32_t* e = ent + n * sz;
+                const uint32_t hx = e[3 + 2 * side];
+                float* xd = xs + n * KP + warp * CW + CPW * lane;
+                if (hx == NONE) {
+                    if constexpr (CPW == 2) cp_async8(xd, pool + e[2 + 2 * side] + cb);
+                    else cp_async4(xd, pool + e[2 + 2 * side] + cb, 4u);
+                } else {
+                    if constexpr (CPW == 2) cp_async16(tw + n * CW + CPW * lane, HX + (int64_t)hx * H + cb, 16u);
+                    else cp_async8(tw + n * CW + CPW * lane, HX + (int64_t)hx * H + cb);
+                    pend |= 1u << n;
+                }
+            }
+            XST(stF, 17);
+            if (tid < nb * UM) {                           // c_l, c_r of this CTA's units (own records)
+                const int n = tid / UM, uu = tid % UM;
+                const uint32_t* e = ent + n * sz;
+                cp_async4(cin + tid * CINMAX, pool + e[2] + H + lc * UM + uu, 4u);
+                cp_async4(cin + tid * CINMAX + 1, pool + e[4] + H + lc * UM + uu, 4u);
+            }
+            cp_async_wait_all();
+            XST(stF, 18);
+            if (bt) bt[1] = clock64();
+            mark(2);
+            while (true) {
+                uint32_t stale = 0;
+                for (uint32_t m = pend; m; m &= m - 1) {
+                    const int n = __ffs(m) - 1;
+                    const u64* src = tw + n * CW + CPW * lane;
+                    bool fresh = (uint32_t)(src[0] >> 32) == ep;
+                    if constexpr (CPW == 2) fresh = fresh && (uint32_t)(src[1] >> 32) == ep;
+                    if (fresh) {
+                        float* xd = xs + n * KP + warp * CW + CPW * lane;
+                        xd[0] = __uint_as_float((uint32_t)src[0]);
+                        if constexpr (CPW == 2) xd[1] = __uint_as_float((uint32_t)src[1]);
+                        pend &= ~(1u << n);
+                    } else {
+                        const uint32_t hx = ent[n * sz + 3 + 2 * side];
+                        if constexpr (CPW == 2) cp_async16(tw + n * CW + CPW * lane, HX + (int64_t)hx * H + cb, 16u);
+                        else cp_async8(tw + n * CW + CPW * lane, HX + (int64_t)hx * H + cb);
+                        stale = 1;
+                    }
+                }
+                XST(stF && rounds == 0, 19);
+                XST(stF && rounds == 0, 20);
+                if (!__any_sync(FULLMASK, stale)) break;
+                ++rounds;
+                cp_async_wait_all();
+            }
+            __syncwarp();
+        } else if (op == INT_F || is_head) {
             // rows [h_l; h_r] (INT_F) or h of the labelled node (heads), one half row (H values) per
             // (node, side).  Internal children: H tagged slots = H/2 16-byte pieces -> u64 scratch; leaf
             // children (leaf GEMM output): H floats = H/4 pieces straight into xs.  Half rows are spread
