@@ -265,7 +265,7 @@ vpps_status vpps_define_model(const vpps_shape* params, int32_t n_params, const 
         m->smem = m->var->smem_bytes(C);
         CK(cudaFuncSetAttribute(m->var->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)m->smem));
         int per_sm = 0;
-        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, m->var->fn, 256, m->smem));
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, m->var->fn, df_block(m->var->fn), m->smem));
         if (per_sm < 1) return fail(VPPS_E_NOFIT, "dataflow kernel does not fit on an SM");
         o.groups = std::min(n_sm / m->cluster, vpps_model_s::kMaxGroups);
         if (o.groups < 1) return fail(VPPS_E_NOFIT, "fewer SMs than one group");
@@ -650,7 +650,7 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         attr[0].id = cudaLaunchAttributeCooperative;
         attr[0].val.cooperative = 1;
         cfg.gridDim = dim3(m->plan.n_cta);
-        cfg.blockDim = dim3(256);
+        cfg.blockDim = dim3(df_block(m->var->fn));
         cfg.dynamicSmemBytes = m->smem;
         cfg.stream = st;
         // programmatic dependent of the leaf kernel: its launch overlaps the leaf grid's tail; the kernel

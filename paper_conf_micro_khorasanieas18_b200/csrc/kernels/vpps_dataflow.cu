@@ -22,7 +22,6 @@ namespace vpps {
 namespace dev {
 namespace df {
 
-constexpr int NTH = 256;
 constexpr int UMC = 16;        // hidden units per CTA (CTAs per group: NCL = H / 16)
 constexpr int CHUNK = 4096;    // program words staged in shared memory
 constexpr int NB = 16;         // nodes per batch (LEAF_B: up to NBL)
@@ -81,50 +80,55 @@ __device__ __forceinline__ void st_tag4(u64* p, const float* v, uint32_t e) {
 
 template <int H, int E>
 struct DCfg {
+    // threads per CTA (512 threads at 128 registers were measured slower: spills, 112 K vs 129 K samples/s)
+    static constexpr int NTH = 256;
+    static constexpr int NW = NTH / 32;            // warps per CTA
     static constexpr int UM = UMC;                 // hidden units per CTA
     static constexpr int NCL = H / UM;             // CTAs per group (16 at H = 256, 8 at H = 128)
     static constexpr int TU = NTH / UM;            // threads per unit
-    static_assert(H % UM == 0 && TU == 16, "dataflow kernel: 16 units per CTA, 16 threads per unit");
+    static_assert(H % UM == 0, "dataflow kernel: 16 units per CTA");
     using LB = Lay<2 * H, TU>;                     // internal bundle rows (i, o, u of U_iou; f) over [h_l; h_r]
     static constexpr int KP = LB::KP;              // 2H
     // column granule t of a thread covers h_l iff t < TH, for every thread of the unit (compile-time split)
     static constexpr int TH = H / (LB::CG * TU);
     static_assert(H % (LB::CG * TU) == 0, "h_l / h_r boundary on a granule-round boundary");
     static constexpr int O_X = CHUNK;                               // xs [NB][KP] floats
-    static constexpr int O_DXB = O_X + NB * KP;                     // dxb [2][NTH/32][NC][KP] floats / u64 scratch
-    static constexpr int DXB = 2 * (NTH / 32) * NC * KP;           // two buffers of 8 warp slices
+    static constexpr int O_DXB = O_X + NB * KP;                     // u64 staging of tagged rows (NB x KP slots)
+    static constexpr int DXB = 2 * NB * KP;
     static constexpr int O_CIN = O_DXB + DXB;
     static constexpr int O_BIAS = O_CIN + NB * UM * CINMAX;
     static constexpr int O_ZS = O_BIAS + UM * 4;
     // second staging buffers: consecutive batches alternate, so a batch needs no closing barrier
     static constexpr int O_X2 = O_ZS + NB * ZC;
     static constexpr int O_CIN2 = O_X2 + NB * KP;
-    // forward partial gate sums of the 8 warps (column slices), two buffers: [2][8 warps][4 nodes][UM][4 rows]
+    // forward partial gate sums of the NW warps (column slices), two buffers: [2][NW][4 nodes][UM][4 rows]
     static constexpr int O_FP = O_CIN2 + NB * UM * CINMAX;
-    static constexpr int O_HEAD = O_FP + 2 * 8 * 4 * UM * 4;
+    static constexpr int FPB = NW * 4 * UM * 4;
+    static constexpr int O_HEAD = O_FP + 2 * FPB;
     static_assert(DXB >= 2 * NB * KP && DXB >= 2 * NB * NCL * 2 * UM, "u64 staging fits in dxb");
     // register layout (unit pairs x column slices): warp w owns columns [w CW, (w + 1) CW) of [h_l; h_r] for
     // all UM units of the CTA; lane = 4 ug + cg holds units 2 ug, 2 ug + 1 (one float2 per (row, column):
     // FFMA2 over the unit pair) and the CPL columns w CW + 16 t + 4 cg + q (granule t, q < 4)
-    static constexpr int CW = KP / 8;              // columns per warp
-    static constexpr int CPL = KP / 32;            // columns per lane
+    static constexpr int CW = KP / NW;             // columns per warp
+    static constexpr int CPL = CW / 4;             // columns per lane
     static constexpr int NG = CPL / 4;             // 4-column granules per lane
-    static_assert(CPL % 4 == 0 && UM == 16 && NTH == 256, "dataflow kernel: 8 warps x (8 unit pairs x 4 column groups)");
+    static_assert(CPL % 8 == 0 && UM == 16 && (NTH == 256 || NTH == 512),
+                  "dataflow kernel: NW warps x (8 unit pairs x 4 column groups), >= 8 columns per lane");
     static size_t smem_bytes(int32_t C) { return 4 * (size_t)(O_HEAD + 2 * C * H + 2 * C + 8); }
 };
 
 // PROF = false (the production instantiation): every trace stamp, section clock and per-batch record folds
 // away at compile time (prof is a constant nullptr); PROF = true when vpps_set_profile_buffer is active
 template <int H, int E, bool PROF>
-__global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
+__global__ void __launch_bounds__(DCfg<H, E>::NTH, 1) vpps_df(const DfParams P) {
     using T = DCfg<H, E>;
+    constexpr int NTH = T::NTH, NW = T::NW;
     using LB = typename T::LB;
     constexpr int UM = T::UM, KP = T::KP, NCL = T::NCL;
     extern __shared__ __align__(16) uint32_t smw[];
     float* sm = reinterpret_cast<float*>(smw);
     uint32_t* chunk = smw;
     float* xs = sm + T::O_X;
-    float* dxb = sm + T::O_DXB;
     u64* tbuf = reinterpret_cast<u64*>(sm + T::O_DXB);     // tagged staging (aliases dxb)
     float* cin = sm + T::O_CIN;
     float* bias = sm + T::O_BIAS;
@@ -152,7 +156,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
     // w CW + 16 t + 4 cg + q
     constexpr int CW = T::CW, CPL = T::CPL, NG = T::NG;
     const int cg = lane & 3, ug = lane >> 2;
-    const int side = warp >= 4 ? 1 : 0;                         // the warp's columns read h_l (0) or h_r (1)
+    const int side = warp >= NW / 2 ? 1 : 0;                    // the warp's columns read h_l (0) or h_r (1)
     float2 wp[4][CPL];
 #pragma unroll
     for (int r = 0; r < 4; ++r)
@@ -313,26 +317,26 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
         }
         if (op == INT_F && VPPS_DF_WARP_STAGE) {
             // per-warp staging: warp w computes only with the CW columns [w CW, (w + 1) CW) of [h_l; h_r], so
-            // it loads, checks and converts exactly those (child side = w / 4) for every node of the batch into
+            // it loads, checks and converts exactly those (child side = w / (NW / 2)) for every node of the batch into
             // its own slice of xs, with a warp-level retry loop — no CTA barrier before the products (the
             // forward group's barrier orders the children's c below for the cell threads)
-            constexpr int CPW = CW / 32;                   // columns per lane (2 at H = 256, 1 at H = 128)
+            // 16-byte L2-only copies (cp.async.cg; an L1-cached poll could keep returning a stale line): lane l
+            // carries tagged piece l (slots 2l, 2l + 1 of the slice) and leaf piece l (floats 4l .. 4l + 3)
+            const bool tl = 2 * lane < CW, ll = 4 * lane < CW;
             u64* tw = tbuf + warp * (NB * CW);             // this warp's tagged staging
-            const int cb = (warp & 3) * CW + CPW * lane;   // column in the child's h
+            const int cs = (warp % (NW / 2)) * CW;         // the slice's first column in the child's h
             uint32_t pend = 0;                             // bit n: node n's slots are tagged and not yet converted
             for (int n = 0; n < nb; ++n) {
                 const uint32_t* e = ent + n * sz;
                 const uint32_t hx = e[3 + 2 * side];
-                float* xd = xs + n * KP + warp * CW + CPW * lane;
                 if (hx == NONE) {
-                    if constexpr (CPW == 2) cp_async8(xd, pool + e[2 + 2 * side] + cb);
-                    else cp_async4(xd, pool + e[2 + 2 * side] + cb, 4u);
+                    if (ll) cp_async16(xs + n * KP + warp * CW + 4 * lane, pool + e[2 + 2 * side] + cs + 4 * lane, 16u);
                 } else {
-                    if constexpr (CPW == 2) cp_async16(tw + n * CW + CPW * lane, HX + (int64_t)hx * H + cb, 16u);
-                    else cp_async8(tw + n * CW + CPW * lane, HX + (int64_t)hx * H + cb);
+                    if (tl) cp_async16(tw + n * CW + 2 * lane, HX + (int64_t)hx * H + cs + 2 * lane, 16u);
                     pend |= 1u << n;
                 }
             }
+            if (!tl) pend = 0;
             XST(stF, 17);
             if (tid < nb * UM) {                           // c_l, c_r of this CTA's units (own records)
                 const int n = tid / UM, uu = tid % UM;
@@ -348,18 +352,14 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 uint32_t stale = 0;
                 for (uint32_t m = pend; m; m &= m - 1) {
                     const int n = __ffs(m) - 1;
-                    const u64* src = tw + n * CW + CPW * lane;
-                    bool fresh = (uint32_t)(src[0] >> 32) == ep;
-                    if constexpr (CPW == 2) fresh = fresh && (uint32_t)(src[1] >> 32) == ep;
-                    if (fresh) {
-                        float* xd = xs + n * KP + warp * CW + CPW * lane;
-                        xd[0] = __uint_as_float((uint32_t)src[0]);
-                        if constexpr (CPW == 2) xd[1] = __uint_as_float((uint32_t)src[1]);
+                    const u64* src = tw + n * CW + 2 * lane;
+                    if ((uint32_t)(src[0] >> 32) == ep && (uint32_t)(src[1] >> 32) == ep) {
+                        *reinterpret_cast<float2*>(xs + n * KP + warp * CW + 2 * lane) =
+                            make_float2(__uint_as_float((uint32_t)src[0]), __uint_as_float((uint32_t)src[1]));
                         pend &= ~(1u << n);
                     } else {
                         const uint32_t hx = ent[n * sz + 3 + 2 * side];
-                        if constexpr (CPW == 2) cp_async16(tw + n * CW + CPW * lane, HX + (int64_t)hx * H + cb, 16u);
-                        else cp_async8(tw + n * CW + CPW * lane, HX + (int64_t)hx * H + cb);
+                        cp_async16(tw + n * CW + 2 * lane, HX + (int64_t)hx * H + cs + 2 * lane, 16u);
                         stale = 1;
                     }
                 }
@@ -648,7 +648,7 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                     val[i] = kp + __shfl_xor_sync(FULLMASK, snd, 2);
                 }
                 // kept value i is v = i + (2 c0 + c1) V / 4: node v / 8, row (v / 2) % 4, unit v % 2
-                float* fb = fpb + fbuf * (8 * 4 * UM * 4) + warp * (4 * UM * 4);
+                float* fb = fpb + fbuf * T::FPB + warp * (4 * UM * 4);
                 const int vb = ((c0 ? 2 : 0) + (c1 ? 1 : 0)) * (V / 4);
                 if constexpr (NN == 4) {
                     float* d = fb + (vb / 8) * (UM * 4) + 2 * ug * 4;
@@ -666,13 +666,13 @@ __global__ void __launch_bounds__(NTH, 1) vpps_df(const DfParams P) {
                 if (tid < NN * UM) {
                     const int n = n0 + tid / UM, uu = tid % UM;
                     if (n < nb) {
-                        const float* fs = fpb + fbuf * (8 * 4 * UM * 4) + ((tid / UM) * UM + uu) * 4;
+                        const float* fs = fpb + fbuf * T::FPB + ((tid / UM) * UM + uu) * 4;
                         float gi = 0.f, go = 0.f, gu = 0.f, gfl = 0.f, gfr = 0.f;
 #pragma unroll
-                        for (int w = 0; w < 8; ++w) {
+                        for (int w = 0; w < NW; ++w) {
                             const float4 p4 = *reinterpret_cast<const float4*>(fs + w * (4 * UM * 4));
                             gi += p4.x; go += p4.y; gu += p4.z;
-                            if (w < 4) gfl += p4.w; else gfr += p4.w;
+                            if (w < NW / 2) gfl += p4.w; else gfr += p4.w;
                         }
                         const uint32_t* e = ent + n * sz;
                         const uint32_t rec = e[0];
@@ -853,6 +853,8 @@ const void* df_prof_fn(const void* fn) {
 #undef VPPS_DF_PROF
     return nullptr;
 }
+
+int df_block(const void*) { return dev::df::DCfg<256, 256>::NTH; }
 
 const Variant* df_variants(int32_t* n) {
     *n = (int32_t)(sizeof(kDfVariants) / sizeof(kDfVariants[0]));

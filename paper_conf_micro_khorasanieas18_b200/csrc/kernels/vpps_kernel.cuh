@@ -70,6 +70,7 @@ const Variant* cluster_variants(int32_t* n);
 // Dataflow specialisations (vpps_dataflow.cu); Variant.umax holds the group size.
 const Variant* df_variants(int32_t* n);
 const void* df_prof_fn(const void* fn);   // the trace-enabled instantiation of a dataflow variant
+int df_block(const void* fn);             // threads per CTA of a dataflow specialisation
 const void* fb_prof_fn(const void* fn);   // ... of a grid-kernel variant
 // dW = Σ g xᵀ per weight matrix from the recorded operands, fused SGD when mode == 1.
 // Also forms the leaf input gradient dX[tok] += W_iouᵀ g_leaf when d_inputs is not null.  Node lists are

@@ -10,7 +10,7 @@ for i in $(seq 1 $N); do
   for v in "${VARS[@]}"; do
     IFS=: read -r name so envs <<< "$v"
     cp ab/$so $LIB
-    ( [ -n "$envs" ] && export $(echo $envs | tr ',' ' '); timeout 300 python bench.py --no-cpu-baseline --steps 200 2>/dev/null ) | tail -1 | python -c "
+    ( [ -n "$envs" ] && export $(echo $envs | tr ',' ' '); timeout 150 python bench.py --no-cpu-baseline --steps 200 2>/dev/null ) | tail -1 | python -c "
 import json,sys; d=json.loads(sys.stdin.read()); print('$name', round(d['value']), round(d['ms_per_step']*1e3,1), round(d['roofline']['kernel_ms']*1e3,1), round(d['e2e']['value']))" >> gpurun_out/ab_$TAG.txt
   done
 done
