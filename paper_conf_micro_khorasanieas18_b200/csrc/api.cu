@@ -647,8 +647,14 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         void* dargs[] = {&dp};
         cudaLaunchConfig_t cfg = {};
         cudaLaunchAttribute attr[2];
+        // Co-residency of a group's CTAs (they poll each other's slots) needs no cooperative launch: the grid
+        // fits the GPU at one CTA per SM (checked above) and nothing it waits for runs behind it, so CTAs
+        // that start early only spin until their group is complete.  Without the all-or-nothing cooperative
+        // start, the CTAs take SMs as the leaf grid's CTAs exit (programmatic launch) and load their weights
+        // while the leaf GEMM's slowest tiles finish.  VPPS_DF_COOP=1 restores the cooperative launch.
+        static const bool coop_df = getenv("VPPS_DF_COOP") && atoi(getenv("VPPS_DF_COOP")) != 0;
         attr[0].id = cudaLaunchAttributeCooperative;
-        attr[0].val.cooperative = 1;
+        attr[0].val.cooperative = coop_df ? 1 : 0;
         cfg.gridDim = dim3(m->plan.n_cta);
         cfg.blockDim = dim3(df_block(m->var->fn));
         cfg.dynamicSmemBytes = m->smem;
