@@ -626,8 +626,8 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
     if (m->t_before) CK(cudaEventRecord(m->t_before, st));
     if (m->dataflow) {
         // leaf GEMM (also clears the pass's accumulators, advances the pass counter) -> vpps_df
-        // (cooperative: the groups' CTAs must be co-resident because consumers spin on producers) ->
-        // gradient GEMM (programmatic dependent, per-group completion counters) -> SGD
+        // (one CTA per SM; a group's CTAs are co-resident because the whole grid fits, consumers spin on
+        // producers) -> gradient GEMM (programmatic dependent, per-group completion counters) -> SGD
         DfParams dp{};
         dp.params = m->params;
         dp.grads = m->grads;
