@@ -126,7 +126,11 @@ typedef struct {
                             per SM (floor(n_sm / cluster) groups; the whole grid fits, so no
                             cooperative launch is needed), and the signal/wait of L165 is replaced by
                             epoch-tagged 64-bit slots that consumers poll (vpps_df); 0 = barrier
-                            synchronisation. */
+                            synchronisation.  Because the launch is not cooperative, two dataflow
+                            passes must not run concurrently on one device (e.g. two models on two
+                            streams): each could hold part of the SMs while its other CTAs wait for
+                            them.  Serialise such passes, or set VPPS_DF_COOP=1 (cooperative launch,
+                            the driver then guarantees co-residency). */
     int32_t level;       /* binary cell only.  1: level-synchronous GEMM path — per level one dense
                             product of the gathered children rows with the weights (PAPER L185's
                             concatenation applied to every matrix use; weights L2-resident, plain
