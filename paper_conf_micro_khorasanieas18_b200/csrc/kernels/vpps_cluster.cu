@@ -628,7 +628,13 @@ struct GemmParams {
 constexpr int TM = 128;          // tile rows (gate-gradient rows)
 constexpr int TN = 64;           // tile cols (input columns)
 
-constexpr int KCH = 96;          // nodes per work item (split-K)
+#ifndef VPPS_DW_KCH
+#define VPPS_DW_KCH 96           // nodes per work item
+#endif
+#ifndef VPPS_DW_CPS
+#define VPPS_DW_CPS 3            // gradient-GEMM CTAs per SM
+#endif
+constexpr int KCH = VPPS_DW_KCH;          // nodes per work item (split-K)
 
 // work items of one group: job m = 0 dU_iou, 1 dU_fl, 2 dU_fr, 3 dW_iou (split-K over the group's nodes),
 // 4 leaf dX (split-K over the 3H gate rows)
@@ -637,7 +643,10 @@ constexpr int KCH = 96;          // nodes per work item (split-K)
 // leaves).  Tile 64 leaves x 64 columns, split-K over the 3H gate rows in chunks of DXK, 4 x 4 per thread.
 // The item stages all of its operands with one batch of cp.async (one L2 round trip): the leaf gate
 // gradients row-major ([leaf][k], stride DXS ≡ 4 mod 32: conflict-free column reads) and DXK rows of W_iou.
-constexpr int DXM = 64, DXN = 64, DXK = 128, DXS = DXK + 4;
+#ifndef VPPS_DW_DXK
+#define VPPS_DW_DXK 128          // gate rows per leaf-dX work item
+#endif
+constexpr int DXM = 64, DXN = 64, DXK = VPPS_DW_DXK, DXS = DXK + 4;
 constexpr size_t DW_SMEM = 4 * (size_t)((KCH * TM + KCH * TN) > (DXM * DXS + DXK * DXN) ? (KCH * TM + KCH * TN)
                                                                                           : (DXM * DXS + DXK * DXN));
 __device__ __forceinline__ void leaf_dx_tile(const GemmParams& P, const uint32_t* leaf_nodes, int n_leaf, int b,
@@ -992,7 +1001,7 @@ __device__ __forceinline__ void dw_item(const GemmParams& P, int g, int i, float
 // ever sits on an SM waiting for a group that is still running); groups are scanned in the host's order.
 // Without counters (P.done == nullptr) item = blockIdx.x over the groups in order.
 template <bool TC>
-__global__ void __launch_bounds__(256, 3) vpps_dw_gemm(const GemmParams P) {
+__global__ void __launch_bounds__(256, VPPS_DW_CPS) vpps_dw_gemm(const GemmParams P) {
     extern __shared__ __align__(16) float dsm[];
     __shared__ uint32_t idx[3 * KCH];
     __shared__ int pick[3];
@@ -1197,7 +1206,7 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, flo
         attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
         attr[0].val.programmaticStreamSerializationAllowed = 1;
         g.static_items = stat;
-        cfg.gridDim = dim3(done && !stat ? std::min(items, 148 * 3) : items);   // persistent when claiming
+        cfg.gridDim = dim3(done && !stat ? std::min(items, 148 * VPPS_DW_CPS) : items);   // persistent when claiming
         cfg.blockDim = dim3(256);
         cfg.dynamicSmemBytes = DW_SMEM;
         cfg.stream = s;
