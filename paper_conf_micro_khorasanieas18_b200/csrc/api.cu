@@ -641,6 +641,10 @@ static vpps_status run(vpps_model m, vpps_script s, const float* inputs, int64_t
         dp.df_hx = s->s.df_hx;
         dp.df_part = s->s.df_part;
         dp.df_hd = s->s.df_hd;
+        dp.pool_words = s->s.pool_words;
+        dp.n_hx = s->s.n_hx;
+        dp.n_part = s->s.n_part;
+        dp.n_hd = s->s.n_hd;
         dp.prof = m->prof;
         dp.prof_stride = m->prof_stride;
         dp.done = m->done;

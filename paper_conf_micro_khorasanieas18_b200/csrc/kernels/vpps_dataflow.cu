@@ -14,6 +14,7 @@
 //   HD[node][H]          the loss head's contribution to a labelled node's dh
 // The epoch is the pass counter, so slots never need clearing.  Without hardware clusters the groups
 // are ordinary co-resident CTAs of a cooperative launch: 9 groups on 144 SMs instead of 7 clusters.
+#include <cstdio>
 #include <type_traits>
 #include "vpps_kernel.cuh"
 #include "dev_common.cuh"
@@ -32,6 +33,9 @@ constexpr int ZC = 32;         // classes per head (C <= 32)
 constexpr int CINMAX = 10;
 #ifndef VPPS_DF_WARP_STAGE
 #define VPPS_DF_WARP_STAGE 1 // INT_F batches staged per warp (only the warp's own columns)
+#endif
+#ifndef VPPS_DF_CHECK
+#define VPPS_DF_CHECK 0      // 1: bounds-checked build (every batch entry against its region; traps)
 #endif
 #ifndef VPPS_DF_NP
 #define VPPS_DF_NP 2         // nodes per transposed-product step
@@ -246,6 +250,40 @@ __global__ void __launch_bounds__(DCfg<H, E>::NTH, 1) vpps_df(const DfParams P) 
         const uint32_t* ent = chunk + (pos - cbase) + 1;
         const uint32_t next = pos + 1 + nb * sz;
         const bool is_head = op == HEAD_FB;
+#if VPPS_DF_CHECK
+        // checked build (tests only; compute-sanitizer is not available on the pool): every field of the
+        // batch within its region before anything is staged — a violation traps (the pass fails loudly)
+        {
+            const bool okh = (op == INT_F || op == INT_B || op == HEAD_FB) ? (nb >= 1 && nb <= NB)
+                           : (op == LEAF_B && nb >= 1 && nb <= NBL);
+            if (!okh || next > s1 || 1 + nb * sz > MAXB) {
+                if (tid == 0) printf("vpps_df check: CTA %d batch %d op %x nb %d\n", blockIdx.x, nbatch, op, nb);
+                __trap();
+            }
+            // record extents: internal record 12 H (h c i o u fl fr + 5 gate gradients), leaf record 8 H,
+            // dc slot at adj + H, head record C + 1 (p, loss)
+            auto in = [&](uint32_t r, int64_t ext) { return (int64_t)r + ext <= P.pool_words; };
+            auto opt_ok = [&](uint32_t v, int64_t n) { return v == NONE || (int64_t)v < n; };
+            for (int i = tid; i < nb; i += NTH) {
+                const uint32_t* e = ent + i * sz;
+                bool ok = true;
+                if (op == INT_F) ok = in(e[0], 12 * H) && in(e[2], 2 * H) && in(e[4], 2 * H) && opt_ok(e[1], P.n_hx) &&
+                                      opt_ok(e[3], P.n_hx) && opt_ok(e[5], P.n_hx);
+                else if (op == INT_B) ok = in(e[0], 12 * H) && in(e[1], 2 * H) && in(e[5], 2 * H) && in(e[6], 2 * H) &&
+                                           in(e[7], 2 * H) && in(e[8], 2 * H) &&
+                                           (e[2] == NONE || (int64_t)(e[2] >> 1) < P.n_part) &&
+                                           opt_ok(e[3], P.n_hd) && (int64_t)e[4] < P.n_part;
+                else if (op == HEAD_FB) ok = in(e[0], C + 1) && in(e[1], H) && (int)e[2] < C && opt_ok(e[3], P.n_hx) &&
+                                             opt_ok(e[4], P.n_hd);
+                else ok = in(e[0], 8 * H) && in(e[1], 2 * H) && (e[2] == NONE || (int64_t)(e[2] >> 1) < P.n_part) &&
+                          opt_ok(e[3], P.n_hd);
+                if (!ok) {
+                    printf("vpps_df check: CTA %d batch %d op %x entry %d out of range\n", blockIdx.x, nbatch, op, i);
+                    __trap();
+                }
+            }
+        }
+#endif
         ++nbatch;
         // staging buffers of this batch: the other pair than the previous batch's (a thread still computing
         // that batch reads only those); batch b+2 reuses them after batch b+1's staging barrier

@@ -37,6 +37,7 @@ struct DfParams {
     uint64_t* prof;
     int64_t prof_stride;
     int32_t* done;              // per-group completion counters, or nullptr
+    int64_t pool_words, n_hx, n_part, n_hd;   // record region and slot counts (bounds of the checked build)
 };
 
 // Device allocations of library-owned buffers (include/vpps.h vpps_alloc_fn / vpps_free_fn): the caller's
