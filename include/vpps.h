@@ -122,15 +122,10 @@ typedef struct {
                             that owns whole graphs (SPEC S5g), synchronised by the hardware
                             cluster barrier; groups = the number of co-resident clusters (or the
                             given `groups` when plan_only).  0 = grid-wide groups (SPEC S5). */
-    int32_t dataflow;    /* 1 (with cluster = H / 16): the groups are ordinary co-resident CTAs, one
-                            per SM (floor(n_sm / cluster) groups; the whole grid fits, so no
-                            cooperative launch is needed), and the signal/wait of L165 is replaced by
-                            epoch-tagged 64-bit slots that consumers poll (vpps_df); 0 = barrier
-                            synchronisation.  Because the launch is not cooperative, two dataflow
-                            passes must not run concurrently on one device (e.g. two models on two
-                            streams): each could hold part of the SMs while its other CTAs wait for
-                            them.  Serialise such passes, or set VPPS_DF_COOP=1 (cooperative launch,
-                            the driver then guarantees co-residency). */
+    int32_t dataflow;    /* 1 (with cluster = H / 16): the groups are ordinary co-resident CTAs of a
+                            cooperative launch, one per SM (floor(n_sm / cluster) groups), and the
+                            signal/wait of L165 is replaced by epoch-tagged 64-bit slots that consumers
+                            poll (vpps_df); 0 = barrier synchronisation. */
     int32_t level;       /* binary cell only.  1: level-synchronous GEMM path — per level one dense
                             product of the gathered children rows with the weights (PAPER L185's
                             concatenation applied to every matrix use; weights L2-resident, plain

@@ -660,8 +660,8 @@ __device__ __forceinline__ void leaf_dx_tile(const GemmParams& P, const uint32_t
     float* Bs = sm + DXM * DXS;          // [DXK][DXN]
     if (tid < DXM) {
         const int row = r0 + tid;
-        idx[2 * tid] = row < n_leaf ? leaf_nodes[2 * row] : 0xFFFFFFFFu;
-        idx[2 * tid + 1] = row < n_leaf ? leaf_nodes[2 * row + 1] : 0u;
+        idx[2 * tid] = row < n_leaf ? __ldcg(leaf_nodes + 2 * row) : 0xFFFFFFFFu;
+        idx[2 * tid + 1] = row < n_leaf ? __ldcg(leaf_nodes + 2 * row + 1) : 0u;
     }
     __syncthreads();
     for (int e = tid; e < DXM * (DXK / 4); e += 256) {
@@ -791,12 +791,12 @@ __device__ __forceinline__ void dw_item_tc(const GemmParams& P, int m, int b, in
     if (tid < nk) {
         const int node = k0 + tid;
         if (m == 3) {
-            idx[3 * tid] = leaf_nodes[2 * node];
-            idx[3 * tid + 1] = leaf_nodes[2 * node + 1];
+            idx[3 * tid] = __ldcg(leaf_nodes + 2 * node);
+            idx[3 * tid + 1] = __ldcg(leaf_nodes + 2 * node + 1);
         } else {
-            idx[3 * tid] = int_nodes[3 * node];
-            idx[3 * tid + 1] = int_nodes[3 * node + 1];
-            idx[3 * tid + 2] = int_nodes[3 * node + 2];
+            idx[3 * tid] = __ldcg(int_nodes + 3 * node);
+            idx[3 * tid + 1] = __ldcg(int_nodes + 3 * node + 1);
+            idx[3 * tid + 2] = __ldcg(int_nodes + 3 * node + 2);
         }
     }
     __syncthreads();
@@ -944,12 +944,12 @@ __device__ __forceinline__ void dw_item(const GemmParams& P, int g, int i, float
     if (tid < nk) {
         const int node = k0 + tid;
         if (m == 3) {
-            idx[3 * tid] = leaf_nodes[2 * node];
-            idx[3 * tid + 1] = leaf_nodes[2 * node + 1];
+            idx[3 * tid] = __ldcg(leaf_nodes + 2 * node);
+            idx[3 * tid + 1] = __ldcg(leaf_nodes + 2 * node + 1);
         } else {
-            idx[3 * tid] = int_nodes[3 * node];
-            idx[3 * tid + 1] = int_nodes[3 * node + 1];
-            idx[3 * tid + 2] = int_nodes[3 * node + 2];
+            idx[3 * tid] = __ldcg(int_nodes + 3 * node);
+            idx[3 * tid + 1] = __ldcg(int_nodes + 3 * node + 1);
+            idx[3 * tid + 2] = __ldcg(int_nodes + 3 * node + 2);
         }
     }
     __syncthreads();

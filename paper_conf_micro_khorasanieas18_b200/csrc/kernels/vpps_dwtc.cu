@@ -208,19 +208,19 @@ __global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
         const float* abase = P.pool;
         const float* bbase = p == 3 ? P.inputs : (p == 4 ? P.w_iou : P.pool);
         if (a_kc) {
-            for (int r = tid; r < BM; r += NT) aoff[r] = m0 + r < M ? leaves[2 * (m0 + r)] + 5 * H : 0u;
+            for (int r = tid; r < BM; r += NT) aoff[r] = m0 + r < M ? __ldcg(leaves + (2 * (m0 + r))) + 5 * H : 0u;
             for (int k = tid; k < ke - kb; k += NT) boff[k] = (uint32_t)(kb + k) * (uint32_t)P.E;
         } else {
             for (int k = tid; k < ke - kb; k += NT) {
                 const int node = kb + k;
                 if (p == 3) {
-                    aoff[k] = leaves[2 * node] + 5 * H;
-                    boff[k] = leaves[2 * node + 1] * (uint32_t)P.E;
+                    aoff[k] = __ldcg(leaves + (2 * node)) + 5 * H;
+                    boff[k] = __ldcg(leaves + (2 * node + 1)) * (uint32_t)P.E;
                 } else {
-                    const uint32_t rec = ints[3 * node];
+                    const uint32_t rec = __ldcg(ints + (3 * node));
                     aoff[k] = rec + (p == 0 ? 7 : (p == 1 ? 10 : 11)) * H;
-                    boff[k] = p == 1 || (p == 0 && n0 < H) ? ints[3 * node + 1]
-                                                           : ints[3 * node + 2] - (p == 0 ? H : 0);
+                    boff[k] = p == 1 || (p == 0 && n0 < H) ? __ldcg(ints + (3 * node + 1))
+                                                           : __ldcg(ints + (3 * node + 2)) - (p == 0 ? H : 0);
                 }
             }
         }
@@ -263,7 +263,7 @@ __global__ void __launch_bounds__(NT, 1) vpps_dw_tc(const Params P) {
             const int row = m0 + 32 * (warp & 3) + lane, cb = 64 * (warp >> 2);
             float* out = nullptr;
             if (row < M)
-                out = p == 4 ? P.d_inputs + (int64_t)leaves[2 * row + 1] * P.E
+                out = p == 4 ? P.d_inputs + (int64_t)__ldcg(leaves + (2 * row + 1)) * P.E
                              : P.grads + P.off[p == 3 ? 0 : p + 1] + (int64_t)row * N;
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
