@@ -1211,8 +1211,12 @@ void launch_dw_gemm(const float* pool, const float* inputs, float* d_inputs, flo
         cfg.dynamicSmemBytes = DW_SMEM;
         cfg.stream = s;
         cfg.attrs = attr;
-        static const bool no_pdl = getenv("VPPS_DW_NOPDL") != nullptr;   // measurement only: no overlap
-        cfg.numAttrs = early && !no_pdl ? 1 : 0;
+        // Launched after vpps_df has completed.  As a programmatic dependent (its items overlapping the
+        // slowest groups, 8 % more samples/s) the dataflow test selection failed intermittently — a wrong
+        // loss or weight gradient in about one stress run in 20 (4 of 72), none of 72 without it;
+        // until the cause is isolated that launch is opt-in: VPPS_DW_PDL=1 (measurement only).
+        static const bool pdl = getenv("VPPS_DW_PDL") && atoi(getenv("VPPS_DW_PDL")) != 0;
+        cfg.numAttrs = early && pdl ? 1 : 0;
         if (g.tc) cudaLaunchKernelEx(&cfg, vpps_dw_gemm<true>, g);
         else cudaLaunchKernelEx(&cfg, vpps_dw_gemm<false>, g);
     }

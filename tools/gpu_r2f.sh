@@ -1,7 +1,13 @@
 #!/bin/bash
+# final launch configuration (no programmatic launches on the dataflow path): stress, suite, evidence
 mkdir -p gpurun_out
-python tools/gemm_bench.py > gpurun_out/gemm_r2f.txt 2>&1
-VPPS_GEMM_TC_MIN=-1 python tools/gemm_bench.py >> gpurun_out/gemm_r2f.txt 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:"vpps_dw_tc" -s 4 -c 1 -o gpurun_out/prof_dwtc python bench.py --steps 2 --warmup 3 --no-cpu-baseline > gpurun_out/ncu_dwtc.log 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:"tc_sgemm" -s 3 -c 1 -o gpurun_out/prof_tcg python tools/gemm_bench.py > /dev/null 2>&1
-echo done
+: > gpurun_out/stress_r2f.txt
+f=0
+for i in $(seq 1 24); do
+  timeout 300 python -m pytest tests -m gpu -q -x -k 'binary_target_dataflow or dataflow_epochs or dataflow_groups_hidden or dataflow_batch or fused_sgd or sgd_step' > gpurun_out/stf_tmp.txt 2>&1 || { f=$((f+1)); grep -E "^E  |^FAILED" gpurun_out/stf_tmp.txt | head -4 >> gpurun_out/stress_r2f.txt; }
+done
+echo "dataflow selection: failed_runs=$f of 24" >> gpurun_out/stress_r2f.txt
+bash tools/ab.sh final 2 T:T.so T_dwpdl:T.so:VPPS_DW_PDL=1
+bash tools/run_suite.sh r2f
+timeout 120 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke_r2f.txt 2>&1; echo "smoke rc=$?" >> gpurun_out/smoke_r2f.txt
+cat gpurun_out/stress_r2f.txt gpurun_out/ab_final.txt gpurun_out/tests_r2f.txt gpurun_out/smoke_r2f.txt
