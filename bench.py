@@ -108,7 +108,7 @@ class ClockSampler:
                 "samples": len(self.sm), "source": "nvml" if self.nvml else "nvidia-smi"}
 
 
-PROFILE_TAG = "r2e"     # profiles/<tag>_ncu_summary.json: ncu capture of the kernels this bench times
+PROFILE_TAG = "r2f"     # profiles/<tag>_ncu_summary.json: ncu capture of the kernels this bench times
 
 
 def make_batches(rank: int, batch: int):
