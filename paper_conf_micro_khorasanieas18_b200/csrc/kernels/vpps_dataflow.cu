@@ -861,10 +861,15 @@ __global__ void __launch_bounds__(DCfg<H, E>::NTH, 1) vpps_df(const DfParams P) 
     if (holds_head)
         for (int i = tid; i < C; i += NTH) atomicAdd(P.grads + off[7] + i, dbo[i]);
     // this CTA's records and gradient contributions are complete: count it for the GEMM tiles of its group
+    // (every thread's writes, then the CTA barrier, then one GPU-scope fence and a release add by thread 0:
+    //  the barrier orders the other threads' writes before thread 0's fence, whose cumulativity carries
+    //  them to a grid that acquires the counter)
     if (P.done) {
-        __threadfence();
         __syncthreads();
-        if (tid == 0) atomicAdd(P.done + grp, 1);
+        if (tid == 0) {
+            __threadfence();
+            asm volatile("red.release.gpu.global.add.s32 [%0], 1;" ::"l"(P.done + grp) : "memory");
+        }
     }
     if (prof && tid == 0) prof[12] = gtimer();   // exit
 }
