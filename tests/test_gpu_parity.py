@@ -165,10 +165,11 @@ def test_dataflow_epochs_across_passes():
     batches = [_trees(40 + i, 6, (2, 30), V, C) for i in range(3)]
     scripts = [m.build_script(b) for b in batches]
     for rep in range(2):
-        for b, s in zip(batches, scripts):
+        for k, (b, s) in enumerate(zip(batches, scripts)):
             m.fwd_bwd(s, X)
             lo, Go, _ = M.forward_backward("binary", P, X.cpu().double().numpy(), b, H)
-            assert abs(m.latest_loss() - lo) <= TOL * abs(lo)
+            loss = m.latest_loss()
+            assert abs(loss - lo) <= TOL * abs(lo), (rep, k, loss, lo)
             gv = m.views(grads.cpu())
             for name, _ in m.shapes:
                 assert rel(gv[name].numpy(), Go[name]) <= TOL, (rep, name)
