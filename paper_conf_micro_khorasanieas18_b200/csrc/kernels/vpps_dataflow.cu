@@ -82,6 +82,27 @@ __device__ __forceinline__ void st_tag4(u64* p, const float* v, uint32_t e) {
                  ::"l"(p), "l"(tagv(v[0], e)), "l"(tagv(v[1], e)), "l"(tagv(v[2], e)), "l"(tagv(v[3], e)) : "memory");
 }
 
+// Loads of record words (children's c, the INT_B operands): L1-cached by default; VPPS_DF_L2REC=1 routes
+// them through L2 (measurement build for the intermittent failure of DESIGN §6)
+#ifndef VPPS_DF_L2REC
+#define VPPS_DF_L2REC 0
+#endif
+__device__ __forceinline__ void cin_ld2(float* dst, const float* l, const float* r) {
+#if VPPS_DF_L2REC
+    const float a = __ldcg(l), b = __ldcg(r);
+    dst[0] = a;
+    dst[1] = b;
+#else
+    cp_async4(dst, l, 4u);
+    cp_async4(dst + 1, r, 4u);
+#endif
+}
+#if VPPS_DF_L2REC
+#define RV_LD(p) __ldcg(p)
+#else
+#define RV_LD(p) (*(p))
+#endif
+
 template <int H, int E>
 struct DCfg {
     // threads per CTA (512 threads at 128 registers were measured slower: spills, 112 K vs 129 K samples/s)
@@ -379,8 +400,7 @@ __global__ void __launch_bounds__(DCfg<H, E>::NTH, 1) vpps_df(const DfParams P) 
             if (tid < nb * UM) {                           // c_l, c_r of this CTA's units (own records)
                 const int n = tid / UM, uu = tid % UM;
                 const uint32_t* e = ent + n * sz;
-                cp_async4(cin + tid * CINMAX, pool + e[2] + H + lc * UM + uu, 4u);
-                cp_async4(cin + tid * CINMAX + 1, pool + e[4] + H + lc * UM + uu, 4u);
+                cin_ld2(cin + tid * CINMAX, pool + e[2] + H + lc * UM + uu, pool + e[4] + H + lc * UM + uu);
             }
             cp_async_wait_all();
             XST(stF, 18);
@@ -441,8 +461,7 @@ __global__ void __launch_bounds__(DCfg<H, E>::NTH, 1) vpps_df(const DfParams P) 
                 if (op == INT_F && tid < nb * UM) {        // c_l, c_r of this CTA's units (own records)
                     const int n = tid / UM, uu = tid % UM;
                     const uint32_t* e = ent + n * sz;
-                    cp_async4(cin + tid * CINMAX, pool + e[2] + H + lc * UM + uu, 4u);
-                    cp_async4(cin + tid * CINMAX + 1, pool + e[4] + H + lc * UM + uu, 4u);
+                    cin_ld2(cin + tid * CINMAX, pool + e[2] + H + lc * UM + uu, pool + e[4] + H + lc * UM + uu);
                 }
                 cp_async_wait_all();
                 XST(stF, 18);
@@ -486,8 +505,7 @@ __global__ void __launch_bounds__(DCfg<H, E>::NTH, 1) vpps_df(const DfParams P) 
             if (op == INT_F && tid < nb * UM) {            // c_l, c_r of this CTA's units (own records)
                 const int n = tid / UM, uu = tid % UM;
                 const uint32_t* e = ent + n * sz;
-                cp_async4(cin + tid * CINMAX, pool + e[2] + H + lc * UM + uu, 4u);
-                cp_async4(cin + tid * CINMAX + 1, pool + e[4] + H + lc * UM + uu, 4u);
+                cin_ld2(cin + tid * CINMAX, pool + e[2] + H + lc * UM + uu, pool + e[4] + H + lc * UM + uu);
             }
             cp_async_wait_all();
             __syncthreads();
@@ -528,11 +546,11 @@ __global__ void __launch_bounds__(DCfg<H, E>::NTH, 1) vpps_df(const DfParams P) 
             const uint32_t dsrc = act ? e[2] : NONE, hd = act ? e[3] : NONE;
             float rv[9];
             if (act) {
-                rv[0] = pool[e[1] + H + jj];
+                rv[0] = RV_LD(pool + e[1] + H + jj);
 #pragma unroll
-                for (int k = 0; k < 6; ++k) rv[1 + k] = pool[e[0] + (k + 1) * H + jj];
-                rv[7] = pool[e[5] + H + jj];
-                rv[8] = pool[e[7] + H + jj];
+                for (int k = 0; k < 6; ++k) rv[1 + k] = RV_LD(pool + e[0] + (k + 1) * H + jj);
+                rv[7] = RV_LD(pool + e[5] + H + jj);
+                rv[8] = RV_LD(pool + e[7] + H + jj);
             }
             const u64* psrc = dsrc != NONE ? PART + ((((int64_t)(dsrc >> 1) * NCL + lc) * NCL) * 2 + (dsrc & 1)) * UM + uu : nullptr;
             const u64* hsrc = hd != NONE ? HD + (int64_t)hd * H + jj : nullptr;
